@@ -1,0 +1,299 @@
+/*
+ * mg_oracle.c -- CPU ORACLE for the brick-GMG V-cycle.  TEST INFRASTRUCTURE ONLY.
+ *
+ * Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline / --impl
+ * reference legs may load this file's library.  The product path
+ * (paper_conf_sc_antepara0jh24_b200/) never links, imports or calls it and
+ * shares no code, header, table or helper with it.
+ *
+ * What it is: a plain, slow, obviously-correct multigrid on a GLOBAL
+ * lexicographic periodic cell-centred grid (never decomposed, never
+ * bricked), index p = i + nx*(j + ny*k), i fastest.  Every function follows
+ * one passage of PAPER.md (Antepara et al., SC'24), cited as P:Lnn:
+ *
+ *   applyOp               P:L117, L133, L148 (7-point stencil, alpha=-6/h^2,
+ *                         beta=1/h^2, h = spacing of the level), Fig 1 DSL P:L44-55
+ *   smooth                P:L118, L148   x := x + gamma*(Ax - b), gamma = h^2/12
+ *   smooth+residual       P:L119, L133, L148  r = b - Ax computed from the same Ax
+ *   restriction           P:L69, L120    average of the 8 fine cells of a coarse cell
+ *   initZero              P:L146 (Alg 2 step 8)
+ *   interpolation+incr.   P:L69, L123, L135  x^h = x^h + I(x^2h), piecewise constant
+ *   V-cycle               P:L144-146 (Alg 2), readings A1-A3 of DESIGN.md
+ *   maxNormRes            P:L139-141 (Alg 1), P:L148 (max residual, 1e-10)
+ *
+ * Readings of garbled / silent passages:
+ *   - expression order (A8): neighbour sum pairwise by axis
+ *       ((xW+xE)+(xS+xN))+(xB+xT); restriction pairwise i -> j -> k;
+ *     every + - * separately rounded binary64, NO FMA (-ffp-contract=off).
+ *   - residual restricted is the one smooth+residual writes, i.e. b - A x
+ *     with x the iterate BEFORE that sweep (A5, lagged; Table IV
+ *     0.15 FLOP/B = 6 flop / 40 B).
+ *   - exactly `pre`, `post`, `bottom` sweeps (A1, A3); levels 0..L-1,
+ *     bottom at L-1 (A2).
+ *   - the exchange() of Alg 2 is the periodic wrap of the global grid.
+ *
+ * Threads: OpenMP over k-planes; every output point is computed by one fixed
+ * expression, and max is exact, so results do not depend on the thread count.
+ */
+#include <math.h>
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+#ifdef _OPENMP
+#include <omp.h>
+#endif
+
+#define IDX(i, j, k, nx, ny) ((size_t)(i) + (size_t)(nx) * ((size_t)(j) + (size_t)(ny) * (size_t)(k)))
+
+void oracle_set_threads(int n) {
+#ifdef _OPENMP
+  if (n > 0) omp_set_num_threads(n);
+#else
+  (void)n;
+#endif
+}
+
+int oracle_get_threads(void) {
+#ifdef _OPENMP
+  return omp_get_max_threads();
+#else
+  return 1;
+#endif
+}
+
+/* applyOp (Fig 1): Ax = alpha*x + beta*(6 neighbours),
+ * alpha = -6/h^2, beta = 1/h^2, periodic wrap stands for exchange(). */
+void oracle_apply_op(int nx, int ny, int nz, double h, const double *x, double *Ax) {
+  const double inv = 1.0 / (h * h);
+  const double alpha = -6.0 * inv;
+  const double beta = inv;
+#pragma omp parallel for schedule(static)
+  for (int k = 0; k < nz; ++k) {
+    const int kb = (k + nz - 1) % nz, kt = (k + 1) % nz;
+    for (int j = 0; j < ny; ++j) {
+      const int js = (j + ny - 1) % ny, jn = (j + 1) % ny;
+      for (int i = 0; i < nx; ++i) {
+        const int iw = (i + nx - 1) % nx, ie = (i + 1) % nx;
+        const double xw = x[IDX(iw, j, k, nx, ny)], xe = x[IDX(ie, j, k, nx, ny)];
+        const double xs = x[IDX(i, js, k, nx, ny)], xn = x[IDX(i, jn, k, nx, ny)];
+        const double xb = x[IDX(i, j, kb, nx, ny)], xt = x[IDX(i, j, kt, nx, ny)];
+        const double sum = ((xw + xe) + (xs + xn)) + (xb + xt);
+        Ax[IDX(i, j, k, nx, ny)] = alpha * x[IDX(i, j, k, nx, ny)] + beta * sum;
+      }
+    }
+  }
+}
+
+/* smooth: point Jacobi x := x + gamma*(Ax - b), gamma = h^2/12. */
+void oracle_smooth(size_t n, double h, double *x, const double *Ax, const double *b) {
+  const double gamma = (h * h) / 12.0;
+#pragma omp parallel for schedule(static)
+  for (size_t p = 0; p < n; ++p) x[p] = x[p] + gamma * (Ax[p] - b[p]);
+}
+
+/* smooth+residual: the smooth above and r = b - Ax from the
+ * SAME Ax ("simultaneously calculates the residual"). */
+void oracle_smooth_residual(size_t n, double h, double *x, const double *Ax, const double *b, double *r) {
+  const double gamma = (h * h) / 12.0;
+#pragma omp parallel for schedule(static)
+  for (size_t p = 0; p < n; ++p) {
+    r[p] = b[p] - Ax[p];
+    x[p] = x[p] + gamma * (Ax[p] - b[p]);
+  }
+}
+
+/* restriction: b^{2h} = average of the 8 fine cells of each coarse
+ * cell (finite-volume volume average).  nx,ny,nz are FINE dims (even). */
+void oracle_restriction(int nx, int ny, int nz, const double *r, double *bc) {
+  const int cx = nx / 2, cy = ny / 2, cz = nz / 2;
+#pragma omp parallel for schedule(static)
+  for (int K = 0; K < cz; ++K)
+    for (int J = 0; J < cy; ++J)
+      for (int I = 0; I < cx; ++I) {
+        const int i = 2 * I, j = 2 * J, k = 2 * K;
+        const double r000 = r[IDX(i, j, k, nx, ny)], r100 = r[IDX(i + 1, j, k, nx, ny)];
+        const double r010 = r[IDX(i, j + 1, k, nx, ny)], r110 = r[IDX(i + 1, j + 1, k, nx, ny)];
+        const double r001 = r[IDX(i, j, k + 1, nx, ny)], r101 = r[IDX(i + 1, j, k + 1, nx, ny)];
+        const double r011 = r[IDX(i, j + 1, k + 1, nx, ny)], r111 = r[IDX(i + 1, j + 1, k + 1, nx, ny)];
+        bc[IDX(I, J, K, cx, cy)] = 0.125 * (((r000 + r100) + (r010 + r110)) + ((r001 + r101) + (r011 + r111)));
+      }
+}
+
+/* initZero (Alg 2 step 8): coarse initial guess x^{2h} = 0. */
+void oracle_init_zero(size_t n, double *x) {
+#pragma omp parallel for schedule(static)
+  for (size_t p = 0; p < n; ++p) x[p] = 0.0;
+}
+
+/* interpolation+increment: x^h = x^h + I(x^{2h}), each coarse
+ * value increments its 8 fine cells.  nx,ny,nz are FINE dims. */
+void oracle_interpolation_increment(int nx, int ny, int nz, const double *xc, double *x) {
+  const int cx = nx / 2, cy = ny / 2;
+#pragma omp parallel for schedule(static)
+  for (int k = 0; k < nz; ++k)
+    for (int j = 0; j < ny; ++j)
+      for (int i = 0; i < nx; ++i)
+        x[IDX(i, j, k, nx, ny)] = x[IDX(i, j, k, nx, ny)] + xc[IDX(i / 2, j / 2, k / 2, cx, cy)];
+}
+
+/* maxNormRes (Alg 1): max over the domain of |b - Ax|, with a
+ * fresh applyOp on the current x (reading A6). */
+double oracle_max_norm_residual(int nx, int ny, int nz, double h, const double *x, const double *b) {
+  const size_t n = (size_t)nx * ny * nz;
+  double *Ax = (double *)malloc(n * sizeof(double));
+  if (!Ax) return NAN;
+  oracle_apply_op(nx, ny, nz, h, x, Ax);
+  double m = 0.0;
+#pragma omp parallel for schedule(static) reduction(max : m)
+  for (size_t p = 0; p < n; ++p) {
+    const double a = fabs(b[p] - Ax[p]);
+    if (a > m) m = a;
+  }
+  free(Ax);
+  return m;
+}
+
+/* ---------------------------------------------------------------------------
+ * V-cycle hierarchy (Alg 2)
+ * ------------------------------------------------------------------------- */
+#define ORACLE_MAX_LEVELS 16
+typedef struct {
+  int L, pre, post, bottom;
+  int n[ORACLE_MAX_LEVELS][3];
+  double h[ORACLE_MAX_LEVELS];
+  double *x[ORACLE_MAX_LEVELS], *b[ORACLE_MAX_LEVELS], *Ax[ORACLE_MAX_LEVELS], *r[ORACLE_MAX_LEVELS];
+} oracle_mg;
+
+static size_t lvl_n(const oracle_mg *m, int l) { return (size_t)m->n[l][0] * m->n[l][1] * m->n[l][2]; }
+
+void oracle_mg_destroy(oracle_mg *m) {
+  if (!m) return;
+  for (int l = 0; l < m->L; ++l) {
+    free(m->x[l]);
+    free(m->b[l]);
+    free(m->Ax[l]);
+    free(m->r[l]);
+  }
+  free(m);
+}
+
+/* Level l has spacing h_l = h0 * 2^l ("on each coarser level the grid
+ * size is multiplied by two"; h is the spacing of the given level). */
+oracle_mg *oracle_mg_create(int nx, int ny, int nz, int L, double h0, int pre, int post, int bottom) {
+  if (L < 1 || L > ORACLE_MAX_LEVELS) return NULL;
+  oracle_mg *m = (oracle_mg *)calloc(1, sizeof(oracle_mg));
+  if (!m) return NULL;
+  m->L = L;
+  m->pre = pre;
+  m->post = post;
+  m->bottom = bottom;
+  for (int l = 0; l < L; ++l) {
+    const int s = 1 << l;
+    if (nx % s || ny % s || nz % s) {
+      oracle_mg_destroy(m);
+      return NULL;
+    }
+    m->n[l][0] = nx / s;
+    m->n[l][1] = ny / s;
+    m->n[l][2] = nz / s;
+    m->h[l] = h0 * (double)s;
+    const size_t n = lvl_n(m, l);
+    m->x[l] = (double *)calloc(n, sizeof(double));
+    m->b[l] = (double *)calloc(n, sizeof(double));
+    m->Ax[l] = (double *)calloc(n, sizeof(double));
+    m->r[l] = (double *)calloc(n, sizeof(double));
+    if (!m->x[l] || !m->b[l] || !m->Ax[l] || !m->r[l]) {
+      oracle_mg_destroy(m);
+      return NULL;
+    }
+  }
+  return m;
+}
+
+void oracle_mg_set_b(oracle_mg *m, const double *b) { memcpy(m->b[0], b, lvl_n(m, 0) * sizeof(double)); }
+void oracle_mg_set_x(oracle_mg *m, const double *x) {
+  if (x)
+    memcpy(m->x[0], x, lvl_n(m, 0) * sizeof(double));
+  else
+    memset(m->x[0], 0, lvl_n(m, 0) * sizeof(double));
+}
+void oracle_mg_get_x(const oracle_mg *m, double *x) { memcpy(x, m->x[0], lvl_n(m, 0) * sizeof(double)); }
+/* debug/test access to any level's fields: which = 0 x, 1 b, 2 r, 3 Ax */
+int oracle_mg_get_level(const oracle_mg *m, int l, int which, double *out) {
+  if (l < 0 || l >= m->L) return -1;
+  const double *src = which == 0 ? m->x[l] : which == 1 ? m->b[l] : which == 2 ? m->r[l] : m->Ax[l];
+  memcpy(out, src, lvl_n(m, l) * sizeof(double));
+  return 0;
+}
+
+/* Alg 2, levels 0..L-1 with the bottom solver at L-1 (readings A1-A3). */
+void oracle_mg_vcycle(oracle_mg *m) {
+  const int L = m->L;
+  for (int l = 0; l + 1 < L; ++l) {
+    const int *n = m->n[l];
+    for (int it = 0; it < m->pre; ++it) {                       /* steps 2-6 */
+      oracle_apply_op(n[0], n[1], n[2], m->h[l], m->x[l], m->Ax[l]); /* exchange()+applyOp */
+      oracle_smooth_residual(lvl_n(m, l), m->h[l], m->x[l], m->Ax[l], m->b[l], m->r[l]);
+    }
+    oracle_restriction(n[0], n[1], n[2], m->r[l], m->b[l + 1]); /* step 7 */
+    oracle_init_zero(lvl_n(m, l + 1), m->x[l + 1]);             /* step 8 */
+  }
+  {                                                             /* steps 10-15: bottom */
+    const int l = L - 1;
+    const int *n = m->n[l];
+    for (int it = 0; it < m->bottom; ++it) {
+      oracle_apply_op(n[0], n[1], n[2], m->h[l], m->x[l], m->Ax[l]);
+      oracle_smooth(lvl_n(m, l), m->h[l], m->x[l], m->Ax[l], m->b[l]);
+    }
+  }
+  for (int l = L - 2; l >= 0; --l) {                            /* steps 16-23 */
+    const int *n = m->n[l];
+    oracle_interpolation_increment(n[0], n[1], n[2], m->x[l + 1], m->x[l]);
+    for (int it = 0; it < m->post; ++it) {
+      oracle_apply_op(n[0], n[1], n[2], m->h[l], m->x[l], m->Ax[l]);
+      oracle_smooth_residual(lvl_n(m, l), m->h[l], m->x[l], m->Ax[l], m->b[l], m->r[l]);
+    }
+  }
+}
+
+double oracle_mg_norm(const oracle_mg *m) {
+  return oracle_max_norm_residual(m->n[0][0], m->n[0][1], m->n[0][2], m->h[0], m->x[0], m->b[0]);
+}
+
+/* Alg 1: while maxNormRes > tol: V-cycle; maxNormRes.  The cycle
+ * cap (20, "-n 20") is a parameter.  norms[0..cycles] are recorded if
+ * norms != NULL (norms[0] = initial). Returns cycles done. */
+int oracle_mg_solve(oracle_mg *m, double tol, int max_cycles, double *norms) {
+  double nr = oracle_mg_norm(m);
+  if (norms) norms[0] = nr;
+  int c = 0;
+  while (nr > tol && c < max_cycles) {
+    oracle_mg_vcycle(m);
+    nr = oracle_mg_norm(m);
+    ++c;
+    if (norms) norms[c] = nr;
+  }
+  return c;
+}
+
+/* Point evaluation of one smooth+residual sweep for sampled parity checks at
+ * full size: for each listed point p (lexicographic index), the value x' and
+ * r that smooth+residual produces from x, b at level spacing h. */
+void oracle_sweep_points(int nx, int ny, int nz, double h, const double *x, const double *b, const int64_t *pts,
+                         int64_t npts, double *xn_out, double *r_out) {
+  const double inv = 1.0 / (h * h);
+  const double alpha = -6.0 * inv, beta = inv, gamma = (h * h) / 12.0;
+#pragma omp parallel for schedule(static)
+  for (int64_t q = 0; q < npts; ++q) {
+    const int64_t p = pts[q];
+    const int i = (int)(p % nx), j = (int)((p / nx) % ny), k = (int)(p / ((int64_t)nx * ny));
+    const int iw = (i + nx - 1) % nx, ie = (i + 1) % nx, js = (j + ny - 1) % ny, jn = (j + 1) % ny;
+    const int kb = (k + nz - 1) % nz, kt = (k + 1) % nz;
+    const double sum = ((x[IDX(iw, j, k, nx, ny)] + x[IDX(ie, j, k, nx, ny)]) +
+                        (x[IDX(i, js, k, nx, ny)] + x[IDX(i, jn, k, nx, ny)])) +
+                       (x[IDX(i, j, kb, nx, ny)] + x[IDX(i, j, kt, nx, ny)]);
+    const double a = alpha * x[p] + beta * sum;
+    r_out[q] = b[p] - a;
+    xn_out[q] = x[p] + gamma * (a - b[p]);
+  }
+}

@@ -1,0 +1,332 @@
+"""Pins for the CPU oracle against things OTHER than itself (-m "not gpu").
+
+Each test names the paper passage the pinned function follows and what fixes
+the expected value: a closed form, an invariant, exact arithmetic, or an
+independent SciPy sparse-matrix formulation of the same algorithm.  Chosen so
+that a plausible slip (dropped neighbour, wrong sign of gamma, transposed
+axis, wrong parent index, missing initZero, wrong h per level) fails one.
+"""
+import json
+import os
+
+import numpy as np
+import pytest
+import scipy.sparse as sp
+
+import mg_inputs
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden", "paper_constants.json")
+
+
+def centres(shape, h):
+    nz, ny, nx = shape
+    z = (np.arange(nz) + 0.5) * h
+    y = (np.arange(ny) + 0.5) * h
+    x = (np.arange(nx) + 0.5) * h
+    return np.meshgrid(z, y, x, indexing="ij")  # Z, Y, X each (nz, ny, nx)
+
+
+def mode(shape, h, k=(1, 2, 3)):
+    """Periodic Fourier mode s = sin(w_x x) cos(w_y y) sin(w_z z), w_d = 2 pi k_d / L_d."""
+    nz, ny, nx = shape
+    Z, Y, X = centres(shape, h)
+    kx, ky, kz = k
+    wx, wy, wz = (2 * np.pi * kx / (nx * h), 2 * np.pi * ky / (ny * h), 2 * np.pi * kz / (nz * h))
+    lam = -(4.0 / h**2) * (np.sin(wx * h / 2) ** 2 + np.sin(wy * h / 2) ** 2 + np.sin(wz * h / 2) ** 2)
+    return np.sin(wx * X) * np.cos(wy * Y) * np.sin(wz * Z), lam, (wx, wy, wz)
+
+
+# ---------------------------------------------------------------- golden
+def test_golden_constants_match_table_iv_bytes():
+    """Table IV AI = flops / algorithmic bytes; the byte counts the
+    bench's roofline uses must reproduce the paper's AI."""
+    g = json.load(open(GOLDEN))
+    ai = g["table_iv_theoretical_ai_flop_per_byte"]
+    # (flops, bytes) per point, DESIGN.md "Algorithmic bytes"
+    per_pt = {"applyOp": (8, 16), "smooth": (4, 32), "smooth+residual": (6, 40),
+              "restriction": (8, 72), "interpolation+increment": (8, 136)}
+    for op, (fl, by) in per_pt.items():
+        assert abs(fl / by - ai[op]) <= 0.006, op
+    assert g["operator"]["alpha_times_h2"] == -6.0 and g["smoother"]["gamma_over_h2"] == 1.0 / 12.0
+
+
+# --------------------------------------------------------------- applyOp
+@pytest.mark.parametrize("q_kind", ["harmonic", "six"])
+def test_apply_op_exact_on_quadratics(oracle_mod, q_kind):
+    """applyOp is exact on quadratics: away from the periodic seam
+    A q == Laplacian(q) exactly (dyadic h, exact arithmetic)."""
+    shape = (16, 16, 16)
+    h = 1.0 / 16
+    Z, Y, X = centres(shape, h)
+    if q_kind == "harmonic":
+        q, lap = X**2 + 2 * Y**2 - 3 * Z**2 + X * Y, 0.0
+    else:
+        q, lap = X**2 + Y**2 + Z**2, 6.0
+    Aq = oracle_mod.apply_op(q, h)
+    inner = Aq[1:-1, 1:-1, 1:-1]
+    assert np.all(inner == lap), np.abs(inner - lap).max()
+
+
+def test_apply_op_fourier_eigenvalue(oracle_mod):
+    """Periodic modes are eigenvectors: A s = lambda s, lambda = -(4/h^2) sum sin^2(w_d h/2).
+    Non-cubic grid + distinct wave numbers catch transposed axes / wrong wrap."""
+    shape = (16, 8, 32)  # nz, ny, nx
+    h = 1.0 / 32
+    s, lam, _ = mode(shape, h, k=(3, 1, 2))
+    As = oracle_mod.apply_op(s, h)
+    assert np.abs(As - lam * s).max() <= 1e-12 * abs(lam)
+
+
+def test_apply_op_matches_kronecker_matrix_and_norm(oracle_mod):
+    """Brute force: A as a Kronecker sum of 1D periodic Laplacians (SciPy);
+    maxNormRes = max |b - A x| computed from that matrix."""
+    shape = (6, 4, 10)
+    h = 0.1
+    x = mg_inputs.random_field(shape, 3)
+    b = mg_inputs.random_field(shape, 4)
+    A = kron_laplacian(shape, h)
+    Ax_ref = (A @ x.ravel()).reshape(shape)
+    Ax = oracle_mod.apply_op(x, h)
+    assert np.abs(Ax - Ax_ref).max() <= 1e-13 * np.abs(Ax_ref).max()
+    n_ref = np.abs(b.ravel() - A @ x.ravel()).max()
+    assert abs(oracle_mod.max_norm_residual(x, b, h) - n_ref) <= 1e-13 * n_ref
+
+
+# ------------------------------------------------------ smooth / residual
+def test_smooth_closed_form_on_mode(oracle_mod):
+    """Jacobi x := x + gamma(Ax-b), gamma=h^2/12.  With b = s (an
+    eigenmode) and x0 = 0: c_{k+1} = c_k(1+gamma*lam) - gamma, so
+    c_k = (1 - (1+gamma*lam)^k)/lam.  A wrong sign of gamma diverges."""
+    shape = (8, 8, 8)
+    h = 1.0 / 8
+    s, lam, _ = mode(shape, h, k=(1, 1, 1))
+    x = np.zeros(shape)
+    g = h * h / 12.0
+    for _ in range(100):  # the paper's 100 bottom sweeps
+        x = oracle_mod.smooth(x, oracle_mod.apply_op(x, h), s, h)
+    c = (1.0 - (1.0 + g * lam) ** 100) / lam
+    assert np.abs(x - c * s).max() <= 1e-13 * abs(c)
+
+
+def test_smooth_residual_zero_at_discrete_solution(oracle_mod):
+    """r = b - Ax vanishes (to rounding) at x = b/lambda, and the x
+    that smooth+residual writes equals the x smooth writes (same Ax)."""
+    shape = (16, 8, 32)
+    h = 1.0 / 32
+    s, lam, _ = mode(shape, h, k=(2, 1, 1))
+    x = s / lam
+    Ax = oracle_mod.apply_op(x, h)
+    xs, r = oracle_mod.smooth_residual(x, Ax, s, h)
+    assert np.abs(r).max() <= 1e-13
+    assert np.array_equal(xs, oracle_mod.smooth(x, Ax, s, h))
+    # residual sign: b - Ax, not Ax - b
+    x2 = np.zeros(shape)
+    _, r2 = oracle_mod.smooth_residual(x2, oracle_mod.apply_op(x2, h), s, h)
+    assert np.array_equal(r2, s)
+
+
+# ---------------------------------------------------- restriction / interp
+def test_restriction_constants_and_mode(oracle_mod):
+    """Restriction = volume average of 8 fine cells: R 1 = 1 exactly;
+    on a cell-centred mode R s_h = prod_d cos(w_d h/2) s_2h."""
+    shape = (16, 8, 32)
+    ones = np.ones(shape)
+    assert np.array_equal(oracle_mod.restriction(ones), np.ones((8, 4, 16)))
+    h = 1.0 / 32
+    s, _, (wx, wy, wz) = mode(shape, h, k=(3, 1, 2))
+    sc, _, _ = mode((8, 4, 16), 2 * h, k=(3, 1, 2))
+    fac = np.cos(wx * h / 2) * np.cos(wy * h / 2) * np.cos(wz * h / 2)
+    assert np.abs(oracle_mod.restriction(s) - fac * sc).max() <= 1e-14
+
+
+def test_interpolation_constants(oracle_mod):
+    """Piecewise-constant interpolation + increment: P 1 = 1, and
+    the increment adds onto x."""
+    xc = np.ones((4, 2, 8))
+    assert np.array_equal(oracle_mod.interpolation_increment(xc, np.zeros((8, 4, 16))), np.ones((8, 4, 16)))
+    x = mg_inputs.random_field((8, 4, 16), 1)
+    xc = mg_inputs.random_field((4, 2, 8), 2)
+    out = oracle_mod.interpolation_increment(xc, x)
+    # parent of (k,j,i) is (k//2, j//2, i//2): check by explicit repeat
+    up = np.repeat(np.repeat(np.repeat(xc, 2, axis=0), 2, axis=1), 2, axis=2)
+    assert np.array_equal(out, x + up)
+
+
+def test_restriction_interpolation_adjoint(oracle_mod):
+    """Volume-weighted adjointness 8 <R r, e>_2h = <r, P e>_h (R = P^T/8), random
+    non-cubic data: catches a wrong parent index or a transposed axis."""
+    shape = (8, 12, 16)
+    r = mg_inputs.random_field(shape, 10)
+    e = mg_inputs.random_field((4, 6, 8), 11)
+    Pe = oracle_mod.interpolation_increment(e, np.zeros(shape))
+    lhs = 8.0 * np.sum(oracle_mod.restriction(r) * e)
+    rhs = np.sum(r * Pe)
+    assert abs(lhs - rhs) <= 1e-13 * np.sum(np.abs(r * Pe))
+
+
+def test_restriction_of_interpolation_is_identity_bitwise(oracle_mod):
+    """R(P(e)) == e bitwise with the pairwise summation order (reading A8)."""
+    e = mg_inputs.random_field((4, 6, 8), 12)
+    Pe = oracle_mod.interpolation_increment(e, np.zeros((8, 12, 16)))
+    assert np.array_equal(oracle_mod.restriction(Pe), e)
+
+
+# ------------------------------------------------------------ V-cycle
+def periodic_T(n):
+    T = sp.lil_matrix((n, n))
+    for i in range(n):
+        T[i, i] = -2.0
+        T[i, (i + 1) % n] += 1.0
+        T[i, (i - 1) % n] += 1.0
+    return T.tocsr()
+
+
+def kron_laplacian(shape, h):
+    nz, ny, nx = shape
+    Ix, Iy, Iz = sp.identity(nx), sp.identity(ny), sp.identity(nz)
+    A = (sp.kron(Iz, sp.kron(Iy, periodic_T(nx))) + sp.kron(Iz, sp.kron(periodic_T(ny), Ix))
+         + sp.kron(periodic_T(nz), sp.kron(Iy, Ix)))
+    return (A / (h * h)).tocsr()
+
+
+def prolong_1d(nf):
+    P = sp.lil_matrix((nf, nf // 2))
+    for i in range(nf):
+        P[i, i // 2] = 1.0
+    return P.tocsr()
+
+
+def matrix_vcycle(b0, x0, L, h0, pre, post, bottom):
+    """Alg 2 written with SciPy sparse matrices: A_l Kronecker sum at h_l = 2^l h0,
+    P_l = piecewise-constant prolongation, R_l = P_l^T / 8.  An independent
+    formulation (different summation order) of the same algorithm."""
+    shapes = [tuple(s >> l for s in b0.shape) for l in range(L)]
+    A = [kron_laplacian(shapes[l], h0 * 2**l) for l in range(L)]
+    P = [sp.kron(prolong_1d(shapes[l][0]), sp.kron(prolong_1d(shapes[l][1]), prolong_1d(shapes[l][2]))).tocsr()
+         for l in range(L - 1)]
+    g = [(h0 * 2**l) ** 2 / 12.0 for l in range(L)]
+    x = [None] * L
+    b = [None] * L
+    x[0], b[0] = x0.ravel().copy(), b0.ravel().copy()
+    for l in range(L - 1):
+        for _ in range(pre):
+            Ax = A[l] @ x[l]
+            r = b[l] - Ax
+            x[l] = x[l] + g[l] * (Ax - b[l])
+        b[l + 1] = (P[l].T @ r) / 8.0
+        x[l + 1] = np.zeros_like(b[l + 1])
+    for _ in range(bottom):
+        Ax = A[L - 1] @ x[L - 1]
+        x[L - 1] = x[L - 1] + g[L - 1] * (Ax - b[L - 1])
+    for l in range(L - 2, -1, -1):
+        x[l] = x[l] + P[l] @ x[l + 1]
+        for _ in range(post):
+            Ax = A[l] @ x[l]
+            x[l] = x[l] + g[l] * (Ax - b[l])
+    return x[0].reshape(b0.shape)
+
+
+@pytest.mark.parametrize("shape,L,sweeps", [((16, 16, 16), 2, (3, 3, 10)), ((16, 32, 24), 3, (4, 2, 20)),
+                                             ((32, 32, 32), 3, (12, 12, 100))])
+def test_vcycle_matches_sparse_matrix_vcycle(oracle_mod, shape, L, sweeps):
+    """The stencil V-cycle (Alg 2) equals the sparse-matrix V-cycle to
+    rounding after 1 and 2 cycles (non-cubic grids, 2-3 levels)."""
+    pre, post, bottom = sweeps
+    h0 = mg_inputs.default_h0(shape)
+    b = mg_inputs.random_rhs(shape, 0)
+    mg = oracle_mod.OracleMG(shape, L, pre, post, bottom, h0)
+    mg.set_b(b)
+    mg.set_x(None)
+    xm = np.zeros(shape)
+    for _ in range(2):
+        mg.vcycle()
+        xm = matrix_vcycle(b, xm, L, h0, pre, post, bottom)
+        xo = mg.get_x()
+        assert np.abs(xo - xm).max() <= 1e-12 * np.abs(xm).max()
+
+
+def _rho(oracle_mod, N, L, b):
+    mg = oracle_mod.OracleMG((N, N, N), L)
+    mg.set_b(b)
+    mg.set_x(None)
+    norms = [mg.norm()]
+    for _ in range(6):
+        mg.vcycle()
+        norms.append(mg.norm())
+    ratios = [norms[c] / norms[c - 1] for c in range(2, 7)]
+    return float(np.exp(np.mean(np.log(ratios))))
+
+
+def test_vcycle_convergence_level_independent(oracle_mod):
+    """V-cycle convergence factor is level independent (north_star check 4):
+    fixed 8^3 coarsest grid, 12/12/100, random zero-mean b, rho(L) for
+    L = 2..5 (N = 16..128) all in [0.01, 0.04] with max/min <= 1.5."""
+    rhos = []
+    for L in range(2, 6):
+        N = 8 * 2 ** (L - 1)
+        rhos.append(_rho(oracle_mod, N, L, mg_inputs.random_rhs((N, N, N), 0)))
+    assert all(0.01 <= r <= 0.04 for r in rhos), rhos
+    assert max(rhos) / min(rhos) <= 1.5, rhos
+
+
+def test_second_order_convergence_to_continuum(oracle_mod):
+    """Manufactured solution (north_star check 3): for b = sin sin sin
+    the exact solution is u = -b/(12 pi^2); the converged discrete x (mean
+    removed, reading A12) converges at second order: error ratios -> 4.
+    Also: converged x equals the discrete solution b/lambda_h."""
+    errs = []
+    for N, L in ((16, 2), (32, 3), (64, 4)):
+        b = mg_inputs.sin_rhs((N, N, N))
+        mg = oracle_mod.OracleMG((N, N, N), L)
+        mg.set_b(b)
+        mg.set_x(None)
+        cycles, norms = mg.solve(1e-10, 20)
+        assert norms[-1] < 1e-10 and cycles <= 12
+        x = mg.get_x()
+        x = x - x.mean()
+        h = 1.0 / N
+        lam = -(4.0 / h**2) * 3 * np.sin(np.pi * h) ** 2
+        assert np.abs(x - b / lam).max() <= 1e-9 * np.abs(b / lam).max()
+        errs.append(np.abs(x + b / (12 * np.pi**2)).max())
+    r1, r2 = errs[0] / errs[1], errs[1] / errs[2]
+    assert 3.6 <= r1 <= 4.4 and 3.8 <= r2 <= 4.2, (errs, r1, r2)
+
+
+def test_solve_reaches_paper_tolerance(oracle_mod):
+    """Alg 1: loop until max-norm residual < 1e-10."""
+    b = mg_inputs.random_rhs((32, 32, 32), 1)
+    mg = oracle_mod.OracleMG((32, 32, 32), 3)
+    mg.set_b(b)
+    mg.set_x(None)
+    cycles, norms = mg.solve(1e-10, 20)
+    assert norms[-1] < 1e-10 and 1 <= cycles <= 12
+    assert np.all(np.diff(norms) < 0)
+
+
+def test_oracle_thread_count_invariant(oracle_mod):
+    """Per-point expressions + exact max: identical bits for 1 and N threads."""
+    b = mg_inputs.random_rhs((32, 32, 32), 2)
+    outs = []
+    nthreads = oracle_mod.get_threads()
+    for t in (1, max(2, nthreads)):
+        oracle_mod.set_threads(t)
+        mg = oracle_mod.OracleMG((32, 32, 32), 3)
+        mg.set_b(b)
+        mg.set_x(None)
+        mg.vcycle()
+        outs.append((mg.get_x(), mg.norm()))
+    oracle_mod.set_threads(nthreads)
+    assert np.array_equal(outs[0][0], outs[1][0]) and outs[0][1] == outs[1][1]
+
+
+def test_sweep_points_matches_full_sweep(oracle_mod):
+    """The point-sampled smooth+residual used for full-size sampled parity agrees
+    bitwise with applyOp + smooth+residual on the whole grid."""
+    shape = (8, 12, 16)
+    h = 1.0 / 16
+    x = mg_inputs.random_field(shape, 5)
+    b = mg_inputs.random_field(shape, 6)
+    xs, r = oracle_mod.smooth_residual(x, oracle_mod.apply_op(x, h), b, h)
+    pts = np.arange(x.size)
+    xn_p, r_p = oracle_mod.sweep_points(x, b, h, pts)
+    assert np.array_equal(xn_p, xs.ravel()) and np.array_equal(r_p, r.ravel())
