@@ -1,0 +1,369 @@
+#!/usr/bin/env python
+"""bench.py -- V-cycle DOF/s and finest-level smoother HBM GB/s on B200.
+
+Workload (BASELINE.json configs[3] at N GPUs, configs[2]'s size at N=1):
+512^3 FP64 Poisson per GPU, 8^3 bricks, L = 6 levels (512 -> 16), 12 pre /
+12 post smooths, 100 bottom sweeps, weak scaling with a 3D
+decomposition (1x1x1, 2x1x1, 2x2x1, 2x2x2).  b = sin(2 pi x) sin(2 pi y)
+sin(2 pi z), x0 = 0.  One "step" = one V-cycle (Alg 2).
+
+Usage:  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+        torchrun --nproc-per-node N bench.py --gpus N ...   (one rank per GPU, NCCL)
+Prints ONE JSON line on rank 0 (contract in DESIGN.md "Measurement").
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "V-cycle DOF/s and finest-level smoother HBM GB/s (fraction of 8 TB/s) at 1/2/4/8 B200"
+PROC_GRIDS = {1: (1, 1, 1), 2: (2, 1, 1), 4: (2, 2, 1), 8: (2, 2, 2)}
+# algorithmic bytes per fine point (Table IV)
+B_SWEEP = 24.0          # fused sweep: read x, b; write x'
+B_SWEEP_R = 32.0        # + write r
+B_COARSE_PER_FINE = 1.0  # fused restriction output / interpolation input (8 B per coarse point)
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=30)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--n", type=int, default=512, help="cells per GPU per axis")
+    ap.add_argument("--levels", type=int, default=6)
+    ap.add_argument("--pre", type=int, default=12)
+    ap.add_argument("--post", type=int, default=12)
+    ap.add_argument("--bottom", type=int, default=100)
+    ap.add_argument("--ca-period", type=int, default=0)
+    ap.add_argument("--fusion", type=int, default=0)
+    ap.add_argument("--ghost-all", action="store_true", help="self-exchange ghost shell on every axis")
+    ap.add_argument("--no-graph", action="store_true")
+    ap.add_argument("--no-overlap", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--ref-n", type=int, default=0, help="reference arm: grid side of the bounded sample")
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--quiet", action="store_true")
+    return ap.parse_args()
+
+
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+def workload_name(a, pg):
+    return (f"{a.n}^3 FP64 Poisson per GPU, 8^3 bricks, L={a.levels} ({a.n}->{a.n >> (a.levels - 1)}), "
+            f"{a.pre}/{a.post}/{a.bottom} smooths, 3D decomposition {pg[0]}x{pg[1]}x{pg[2]}")
+
+
+# ------------------------------------------------------------------ clocks
+class ClockSampler:
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index):
+        self.gpu = gpu_index
+        self.proc = None
+        self.path = None
+
+    def start(self):
+        try:
+            fd, self.path = tempfile.mkstemp(suffix=".csv")
+            os.close(fd)
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.FIELDS}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if not self.proc:
+            return None
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        rows = []
+        for line in open(self.path):
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                rows.append((float(parts[1]), float(parts[2]), float(parts[3]), parts[5:9]))
+            except ValueError:
+                continue
+        os.unlink(self.path)
+        if not rows:
+            return None
+        load = [r for r in rows if r[2] > 200.0] or rows
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in load for i, v in enumerate(r[3]) if v.lower() == "active"})
+        return {"sm_mhz": statistics.median(r[0] for r in load), "sm_max_mhz": max(r[1] for r in rows),
+                "reasons": reasons, "samples": len(rows), "samples_under_load": len(load),
+                "power_w_max": max(r[2] for r in rows)}
+
+
+def measured_peaks():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(path):
+        d = json.load(open(path))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, STREAM-style copy)"
+    return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
+
+
+def ncu_traffic(n):
+    """Per-launch DRAM bytes of the level-0 sweep from the committed ncu --set full summary."""
+    path = os.path.join(ROOT, "profiles", "ncu_sweep_summary.json")
+    if not os.path.exists(path):
+        return None
+    try:
+        d = json.load(open(path))
+        if int(d.get("n", -1)) == n:
+            return float(d["dram_bytes_per_launch"])
+    except Exception:
+        pass
+    return None
+
+
+# ------------------------------------------------------------------ oracle timing
+def oracle_dofs(n, levels, pre, post, bottom, seconds, min_cycles=1, max_cycles=1000):
+    """Time the CPU oracle (as it stands) running V-cycles on an n^3 grid."""
+    import mg_inputs
+    import oracle
+
+    oracle.build()
+    b = mg_inputs.sin_rhs((n, n, n))
+    m = oracle.OracleMG((n, n, n), levels, pre, post, bottom)
+    m.set_b(b)
+    m.set_x(None)
+    t0 = time.perf_counter()
+    c = 0
+    while c < min_cycles or (time.perf_counter() - t0 < seconds and c < max_cycles):
+        m.vcycle()
+        c += 1
+    dt = time.perf_counter() - t0
+    m.close()
+    return n**3 * c / dt, c, dt, oracle.get_threads()
+
+
+def cpu_baseline(a):
+    # estimate with one 256^3 cycle, use the real workload size when it fits the budget
+    small = min(a.n, 256)
+    lv_small = max(1, min(a.levels, (small // 8).bit_length()))
+    v, c, dt, cores = oracle_dofs(small, lv_small, a.pre, a.post, a.bottom, 0.0)
+    est_full = dt * (a.n / small) ** 3
+    if a.n != small and est_full <= a.cpu_seconds:
+        v, c, dt, cores = oracle_dofs(a.n, a.levels, a.pre, a.post, a.bottom, a.cpu_seconds)
+        sample = f"{c} oracle V-cycle(s) of the {a.n}^3 workload itself (L={a.levels}), {dt:.1f} s"
+    else:
+        lv = lv_small
+        v, c2, dt2, cores = oracle_dofs(small, lv, a.pre, a.post, a.bottom, a.cpu_seconds)
+        sample = (f"{c2} oracle V-cycle(s) on a {small}^3 grid (L={lv}, same sweeps), {dt2:.1f} s; "
+                  f"DOF/s of that sample")
+    return {"value": v, "unit": "DOF/s", "cores": cores, "kind": "oracle", "sample": sample}
+
+
+def run_reference(a, rank, world):
+    """--impl reference: the CPU oracle as it stands on the host cores (rank 0 only)."""
+    if rank != 0:
+        return
+    import oracle
+
+    oracle.build()
+    n = a.ref_n or min(a.n, 256)
+    lv = max(1, min(a.levels, (n // 8).bit_length()))
+    import mg_inputs
+
+    b = mg_inputs.sin_rhs((n, n, n))
+    m = oracle.OracleMG((n, n, n), lv, a.pre, a.post, a.bottom)
+    m.set_b(b)
+    m.set_x(None)
+    for _ in range(a.warmup):
+        m.vcycle()
+    t0 = time.perf_counter()
+    for _ in range(a.steps):
+        m.vcycle()
+    dt = time.perf_counter() - t0
+    value = n**3 * a.steps / dt
+    pg = PROC_GRIDS.get(a.gpus, (1, 1, 1))
+    sample = f"each step = one oracle V-cycle on a {n}^3 grid (L={lv}, {a.pre}/{a.post}/{a.bottom}), bounded sample"
+    line = {"metric": METRIC, "value": value, "unit": "DOF/s", "n_gpus": a.gpus, "steps": a.steps,
+            "warmup": a.warmup, "ms_per_step": dt / a.steps * 1e3, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
+            "config": {"workload": workload_name(a, pg), "sample_grid": n, "levels": lv},
+            "cpu_baseline": {"value": value, "unit": "DOF/s", "cores": oracle.get_threads(), "kind": "oracle",
+                             "sample": sample},
+            "e2e": {"value": value, "unit": "DOF/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------ GPU arm
+def main():
+    a = parse()
+    rank, world, local = dist_env()
+    if a.impl == "reference":
+        run_reference(a, rank, world)
+        return
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import mg_inputs
+    from paper_conf_sc_antepara0jh24_b200 import mg
+    from paper_conf_sc_antepara0jh24_b200.solver import Multigrid
+
+    if world != a.gpus:
+        a.gpus = world if world > 1 else a.gpus
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    pg = PROC_GRIDS[world]
+    n = a.n
+    m = Multigrid((n, n, n), pg, a.levels, a.pre, a.post, a.bottom, ca_period=a.ca_period, fusion=a.fusion,
+                  ghost_mode=1 if a.ghost_all else 0, use_graph=not a.no_graph, overlap=not a.no_overlap,
+                  rank=rank, world_size=world, device=local)
+    gshape = (n * pg[2], n * pg[1], n * pg[0])
+    b_host = torch.from_numpy(mg_inputs.local_sin_rhs(gshape, rank, pg)).pin_memory()
+    b_dev = b_host.to(dev)
+    m.set_rhs(b_dev)
+    m.set_solution(None)
+    s = m.stream
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    def max_over_ranks(v):
+        if world > 1:
+            t = torch.tensor([v], dtype=torch.float64, device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            return float(t.item())
+        return v
+
+    # ---- warm-up (also captures the CUDA graph)
+    for _ in range(a.warmup):
+        m.vcycle()
+    barrier()
+    clocks = ClockSampler(local)
+    clocks.start()
+    time.sleep(0.3)
+    # ---- timed region: K V-cycles, device-timed with events on the library's stream
+    barrier()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(s)
+    for _ in range(a.steps):
+        m.vcycle()
+    e1.record(s)
+    barrier()
+    t_ms = max_over_ranks(e0.elapsed_time(e1))
+    clk = clocks.stop()
+    dofs = world * n**3 * a.steps / (t_ms / 1e3)
+    norm = m.residual_norm()
+
+    # ---- instrumented pass: per (level, op) device times with CUDA events (no graph)
+    m.set_timing(True)
+    ninst = max(1, min(a.steps, 5))
+    for _ in range(ninst):
+        m.vcycle()
+    torch.cuda.synchronize()
+    tm = m.timings()
+    m.set_timing(False)
+    nsweep0 = a.pre + a.post
+    sweep0_ms = tm[0][mg.OP_NAMES.index("sweep")] / ninst
+    launch_ms = sweep0_ms / nsweep0
+    # algorithmic bytes of the level-0 sweeps of one V-cycle (fully fused: restriction / interpolation fused)
+    pts = n**3
+    bytes0 = pts * (B_SWEEP * nsweep0 + 2 * B_COARSE_PER_FINE)
+    fusion0 = a.fusion or mg.MG_FUSION_FULL
+    if fusion0 != mg.MG_FUSION_FULL:
+        bytes0 = pts * (B_SWEEP * (nsweep0 - 1) + B_SWEEP_R)
+    achieved = bytes0 / (sweep0_ms / 1e3) / 1e9
+    peak, peak_src = measured_peaks()
+    traffic = ncu_traffic(n)
+    levels = []
+    total_inst = sum(sum(r) for r in tm) / ninst
+    for l, row in enumerate(tm):
+        nl = n >> l
+        d = {"level": l, "n": nl, "ms": {k: round(v / ninst, 4) for k, v in zip(mg.OP_NAMES, row) if v > 0}}
+        if row[0] > 0 and l < a.levels - 1:
+            lb = nl**3 * (B_SWEEP * (a.pre + a.post) + (2 if fusion0 == mg.MG_FUSION_FULL else 8) * B_COARSE_PER_FINE)
+            d["sweep_gbs_algorithmic"] = round(lb / (row[0] / ninst / 1e3) / 1e9, 1)
+        levels.append(d)
+
+    # ---- e2e: public API with host buffers (H2D of b, V-cycle, D2H of the norm) per step
+    e2e = None
+    if not a.no_e2e:
+        ke = max(3, min(a.steps, 10))
+        m.set_rhs_host(b_host)
+        m.residual_norm()
+        barrier()
+        t0 = time.perf_counter()
+        f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        f0.record(s)
+        for _ in range(ke):
+            m.set_rhs_host(b_host)          # H2D of this step's input + brick conversion (+ b ghost exchange)
+            m.vcycle()
+            m.residual_norm()               # D2H of the step's result (8 bytes), host sync
+        f1.record(s)
+        barrier()
+        te = max_over_ranks(f0.elapsed_time(f1))
+        e2e = {"value": world * n**3 * ke / (te / 1e3), "unit": "DOF/s", "h2d_bytes_per_step": int(b_host.numel() * 8),
+               "d2h_bytes_per_step": 8, "steps": ke, "ms_per_step": te / ke}
+
+    launches = m.launches_per_vcycle()
+    xbytes, xmsgs = m.exchange_stats()
+    cpu = None
+    if rank == 0 and world == 1 and not a.no_cpu_baseline:
+        cpu = cpu_baseline(a)
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": dofs, "unit": "DOF/s", "n_gpus": world, "steps": a.steps,
+            "warmup": a.warmup, "ms_per_step": t_ms / a.steps, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": workload_name(a, pg), "n_local": [n, n, n], "proc_grid": list(pg),
+                       "levels": a.levels, "smooths": [a.pre, a.post, a.bottom], "brick": 8,
+                       "fusion": "auto(full)" if not a.fusion else a.fusion,
+                       "ca_period": a.ca_period or "auto(8)", "ghost_mode": "all" if a.ghost_all else "auto",
+                       "cuda_graph": not a.no_graph, "overlap": not a.no_overlap,
+                       "l2": "no flush: every level-0 field is 1 GiB > 126 MB L2 (inputs larger than L2)",
+                       "parallelism": f"3D domain decomposition {pg[0]}x{pg[1]}x{pg[2]}"},
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": traffic,
+                         "kernel": "level-0 fused sweep (sweep_kernel), avg over the 24 level-0 sweeps of a V-cycle",
+                         "launch_ms": launch_ms, "bytes_per_point": bytes0 / pts / nsweep0,
+                         "peak_source": peak_src, "frac_of_8TBs": achieved / 8000.0},
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": launches * a.steps,
+            "launches_per_step": launches,
+            "clocks": clk,
+            "final_residual_norm": norm,
+            "exchange": {"bytes_per_cycle_per_rank": xbytes, "messages_per_cycle_per_rank": xmsgs},
+            "levels": levels,
+            "instrumented_ms_per_step": total_inst,
+        }
+        print(json.dumps(line), flush=True)
+    m.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,228 @@
+/*
+ * mg.h -- C ABI of the B200-native brick geometric-multigrid V-cycle.
+ *
+ * The library (paper_conf_sc_antepara0jh24_b200/libmg_b200.so) implements the
+ * FP64 V-cycle of Antepara, Williams, Johansen, Hall, "High-Performance,
+ * Scalable Geometric Multigrid via Fine-Grain Data Blocking for GPUs"
+ * (SC'24).  Citations "P:Lnn" are lines of that paper's text.
+ *
+ *   problem     3D periodic Poisson, 7-point operator A x = alpha x + beta *
+ *               (sum of 6 neighbours), alpha = -6/h^2, beta = 1/h^2, h the
+ *               spacing of the level (Fig 1)
+ *   smoother    point Jacobi x := x + gamma (Ax - b), gamma = h^2/12
+ *   residual    r = b - Ax from the same Ax as the smooth
+ *   restriction average of the 8 fine cells of a coarse cell
+ *   interp.     piecewise-constant x^h += I(x^2h)
+ *   V-cycle     Alg 2; GMG loop Alg 1
+ *   layout      8^3 bricks stored contiguously with an adjacency table
+ *               (P:L17, L59, L61, L154); surface bricks ordered so that the
+ *               ghost exchange sends contiguous brick runs with no packing,
+ *               one brick-deep ghost zone shared by several smooths
+ *               (communication avoiding).
+ *
+ * Conventions
+ *   - Every function returns mg_status: 0 success, >0 warning, <0 error.  No
+ *     exception or exit() crosses the ABI.  On error a thread-local message
+ *     is available from mg_last_error().  A CUDA or NCCL error poisons the
+ *     context: later calls on it return MG_ERR_STATE.
+ *   - Field arrays passed in/out are FP64, C-contiguous, local lexicographic
+ *     with x fastest: index i + n_local[0]*(j + n_local[1]*k).  "_dev"
+ *     pointers are CUDA device pointers on the context's device; "_host"
+ *     pointers are host memory (pinned or pageable).  The caller owns all
+ *     arrays and the workspace; the workspace must outlive the context.
+ *   - The library owns its host tables, streams, events, CUDA graphs and the
+ *     NCCL communicator and frees them in mg_destroy / mg_group_destroy.
+ *   - Collective calls (mg_setup, mg_set_rhs, mg_set_solution, mg_vcycle,
+ *     mg_residual_norm, mg_solve) must be made by all ranks in the same order.
+ *   - mg_vcycle is stream-ordered and never synchronises the host; only
+ *     mg_residual_norm, mg_solve and the *_host copies synchronise.
+ *   - One context per process and GPU; not thread-safe.
+ *   - There is no CPU fallback: without a usable CUDA device mg_setup fails
+ *     with MG_ERR_CUDA.
+ */
+#ifndef MG_B200_H
+#define MG_B200_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  MG_OK = 0,
+  MG_NOT_CONVERGED = 1,   /* mg_solve hit max_cycles before tol (warning) */
+  MG_ERR_INVALID_ARG = -1,
+  MG_ERR_CUDA = -2,
+  MG_ERR_NCCL = -3,
+  MG_ERR_OOM = -4,        /* workspace too small */
+  MG_ERR_STATE = -5       /* context poisoned by an earlier error, or wrong call order */
+} mg_status;
+
+#define MG_MAX_LEVELS 16
+#define MG_BRICK 8          /* brick edge: 8^3 bricks */
+#define MG_MAX_PERIOD 8     /* ghost depth in cells = brick edge */
+
+/* fusion[l] variants.  Every variant produces bit-identical results. */
+enum {
+  MG_FUSION_AUTO = 0,
+  MG_FUSION_PAPER = 1,    /* the paper's kernel set: applyOp, smooth+residual, restriction,
+                             initZero, interpolation+increment as separate kernels (Alg 2) */
+  MG_FUSION_SWEEP = 2,    /* applyOp+smooth(+residual) fused into one ping-pong sweep kernel */
+  MG_FUSION_FULL = 3      /* + restriction fused into the last pre-sweep, interpolation into the
+                             first post-sweep, initZero folded into the first coarse sweep */
+};
+
+/* ghost_mode */
+enum {
+  MG_GHOST_AUTO = 0,      /* ghost shell only on axes with proc_grid > 1; periodic wrap
+                             through the adjacency table on the others */
+  MG_GHOST_ALL = 1        /* ghost shell on every axis, even when the neighbour is this rank
+                             (self-exchange: measures communication avoiding on 1 GPU) */
+};
+
+/* transport */
+enum { MG_TRANSPORT_AUTO = 0, MG_TRANSPORT_NCCL = 1, MG_TRANSPORT_LOCAL = 2 };
+
+/* bottom_mode */
+enum { MG_BOTTOM_AUTO = 0, MG_BOTTOM_SWEEPS = 1, MG_BOTTOM_RESIDENT = 2 };
+
+typedef struct {
+  int32_t n_local[3];            /* cells per rank per axis (x,y,z); each divisible by 8*2^(num_levels-1) */
+  int32_t proc_grid[3];          /* ranks per axis; product == world_size; rank = cx + px*(cy + py*cz) */
+  int32_t num_levels;            /* >= 1; levels 0..L-1, bottom solve on L-1 (reading A2) */
+  int32_t pre_smooths;           /* paper: 12 */
+  int32_t post_smooths;          /* paper: 12 */
+  int32_t bottom_smooths;        /* paper: 100 */
+  int32_t ca_period[MG_MAX_LEVELS]; /* sweeps per x-exchange per level, 1..8; 0 = auto (8) */
+  int32_t fusion[MG_MAX_LEVELS];    /* MG_FUSION_*; 0 = auto */
+  int32_t ghost_mode;            /* MG_GHOST_* */
+  int32_t transport;             /* MG_TRANSPORT_*: auto = NCCL when world_size > 1 or a
+                                    self-exchange is needed and an NCCL id is given, else local */
+  int32_t use_graph;             /* 1 = replay the V-cycle as one CUDA graph (default 1) */
+  int32_t bottom_mode;           /* MG_BOTTOM_* (resident = one CTA runs all bottom sweeps in smem) */
+  int32_t overlap;               /* 1 = sweep interior bricks while the exchange is in flight */
+  int32_t reserved[7];
+  double h0;                     /* finest spacing; <= 0 => 1 / max_d(global N_d) (reading A7) */
+} mg_params;
+
+typedef struct mg_ctx mg_ctx;      /* one rank (process, GPU) */
+typedef struct mg_group mg_group;  /* several ranks driven by one process on one GPU (loopback) */
+typedef struct mg_layout mg_layout;/* host-only layout tables (no GPU needed) */
+
+/* Fill *p with the paper's defaults (12/12/100, L=6, 1 rank, auto everything). */
+void mg_params_default(mg_params* p);
+
+/* Bytes of device workspace one rank needs (fields of every level + tables). */
+mg_status mg_workspace_bytes(const mg_params* p, int32_t rank, int32_t world_size, size_t* out_bytes);
+
+/* rank 0 creates the NCCL unique id (128 bytes) and broadcasts it itself
+ * (torch.distributed in the Python harness). */
+mg_status mg_nccl_unique_id(uint8_t out_id[128]);
+
+/* Collective.  nccl_id may be NULL when world_size == 1 and no NCCL is wanted.
+ * cuda_stream: the cudaStream_t every call enqueues on (NULL = legacy default).
+ * workspace: device memory of >= mg_workspace_bytes, 256-byte aligned. */
+mg_status mg_setup(const mg_params* p, int32_t rank, int32_t world_size, const uint8_t* nccl_id,
+                   int32_t device, void* cuda_stream, void* workspace, size_t ws_bytes, mg_ctx** out);
+
+/* Right-hand side b of level 0, local lexicographic, device / host. */
+mg_status mg_set_rhs(mg_ctx* c, const double* b_dev);
+mg_status mg_set_rhs_host(mg_ctx* c, const double* b_host);
+/* Initial guess; NULL => x = 0 (reading A9). */
+mg_status mg_set_solution(mg_ctx* c, const double* x_dev);
+mg_status mg_get_solution(mg_ctx* c, double* x_dev);
+mg_status mg_get_solution_host(mg_ctx* c, double* x_host);
+
+/* One V-cycle (Alg 2).  Collective, stream-ordered, asynchronous. */
+mg_status mg_vcycle(mg_ctx* c);
+
+/* Global max_p |b_p - (A x)_p| at level 0 with a fresh applyOp (Alg 1
+ * "maxNormRes").  Collective; synchronises the stream. */
+mg_status mg_residual_norm(mg_ctx* c, double* out_max_abs);
+
+/* Alg 1: while norm > tol and cycles < max_cycles: V-cycle.
+ * Returns MG_NOT_CONVERGED (1) if the cap was hit. */
+mg_status mg_solve(mg_ctx* c, double tol, int32_t max_cycles, int32_t* cycles_done, double* final_norm);
+
+/* Per (level, op) device times in ms of the last mg_vcycle run with
+ * timing enabled (mg_set_timing(c, 1) disables graph replay and brackets each
+ * op with CUDA events).  out[l*MG_NUM_OPS + op], op: MG_OP_*.  cap = capacity
+ * in doubles.  Also returns counts of kernel launches in out_launches if not NULL. */
+enum { MG_OP_SWEEP = 0, MG_OP_APPLYOP = 1, MG_OP_SMOOTH = 2, MG_OP_RESTRICT = 3, MG_OP_INTERP = 4,
+       MG_OP_ZERO = 5, MG_OP_EXCHANGE = 6, MG_OP_BOTTOM = 7, MG_NUM_OPS = 8 };
+mg_status mg_set_timing(mg_ctx* c, int32_t enabled);
+mg_status mg_get_timings(mg_ctx* c, double* out, int32_t cap);
+
+/* Number of kernel launches (own kernels) one mg_vcycle issues. */
+mg_status mg_vcycle_launches(mg_ctx* c, int64_t* out);
+
+/* Exchange statistics: bytes this rank sends per V-cycle and message count. */
+mg_status mg_exchange_stats(mg_ctx* c, int64_t* bytes_per_cycle, int64_t* messages_per_cycle);
+
+mg_status mg_destroy(mg_ctx* c);
+
+/* Thread-local description of the last error (never NULL). */
+const char* mg_last_error(void);
+
+/* ----------------------------------------------------------------------------
+ * Per-operator entry points (tests / per-op measurement).  They act on the
+ * context's level-l fields in place; "field" is MG_FIELD_*.  Level fields are
+ * read/written in local lexicographic order (device pointers).
+ * -------------------------------------------------------------------------- */
+enum { MG_FIELD_X = 0, MG_FIELD_B = 1, MG_FIELD_R = 2 };
+mg_status mg_level_set(mg_ctx* c, int32_t level, int32_t field, const double* src_dev);
+mg_status mg_level_get(mg_ctx* c, int32_t level, int32_t field, double* dst_dev);
+/* n sweeps of smooth+residual at level l with variant `fusion`
+ * (MG_FUSION_PAPER: applyOp then smooth+residual kernels; otherwise the fused
+ * sweep); write_r = 1 writes r of the last sweep.  Exchanges as the ghost
+ * rule requires. */
+mg_status mg_op_smooth(mg_ctx* c, int32_t level, int32_t n, int32_t write_r, int32_t fusion);
+/* restriction: b_{l+1} = R r_l, fine level l. */
+mg_status mg_op_restrict(mg_ctx* c, int32_t level);
+/* interpolation+increment: x_l += I x_{l+1}, fine level l. */
+mg_status mg_op_interp(mg_ctx* c, int32_t level);
+/* bottom solve at level l: n Jacobi sweeps with the configured bottom mode. */
+mg_status mg_op_bottom(mg_ctx* c, int32_t level, int32_t n);
+mg_status mg_sync(mg_ctx* c);
+
+/* ----------------------------------------------------------------------------
+ * Loopback group: world_size ranks in ONE process on ONE device, exchanging
+ * ghost bricks through device copies with the same exchange plan the NCCL
+ * path uses.  Lets one GPU run (and test) any 3D decomposition.
+ * The workspace is world_size * per-rank bytes (mg_workspace_bytes of rank 0).
+ * -------------------------------------------------------------------------- */
+mg_status mg_group_setup(const mg_params* p, int32_t world_size, int32_t device, void* cuda_stream,
+                         void* workspace, size_t ws_bytes, mg_group** out);
+mg_status mg_group_ctx(mg_group* g, int32_t rank, mg_ctx** out); /* per-rank view for set/get */
+mg_status mg_group_vcycle(mg_group* g);
+mg_status mg_group_residual_norm(mg_group* g, double* out_max_abs);
+mg_status mg_group_set_rhs(mg_group* g, int32_t rank, const double* b_dev); /* then mg_group_commit_rhs */
+mg_status mg_group_commit_rhs(mg_group* g); /* exchanges level-0 b ghosts of every rank */
+mg_status mg_group_set_solution(mg_group* g, int32_t rank, const double* x_dev);
+mg_status mg_group_destroy(mg_group* g);
+
+/* ----------------------------------------------------------------------------
+ * Host-only layout queries (no GPU needed; used by the CPU tests).
+ * info[0..2] n_local, [3..5] bricks per axis, [6..8] ghost flags,
+ * [9] owned, [10] interior, [11] ghost, [12] allocated bricks (incl. zero
+ * brick), [13] send runs, [14] recv runs, [15] zero-brick index.
+ * adjacency: int32 [stored][8] = W,E,S,N,B,T,self,0 (stored = owned+ghost).
+ * coords: int32 [stored][3] extended brick coords (ghost: -1 or nb).
+ * parent: int32 [stored] = coarse brick index*8 + octant (-1 if none).
+ * plan: int64 [runs][6] = peer, direction(0..26), run index, local brick offset,
+ * remote brick offset, brick count.
+ * -------------------------------------------------------------------------- */
+mg_status mg_layout_create(const mg_params* p, int32_t rank, int32_t world_size, mg_layout** out);
+mg_status mg_layout_level_info(const mg_layout* lay, int32_t level, int64_t info[16]);
+mg_status mg_layout_adjacency(const mg_layout* lay, int32_t level, int32_t* out);
+mg_status mg_layout_coords(const mg_layout* lay, int32_t level, int32_t* out);
+mg_status mg_layout_parent(const mg_layout* lay, int32_t level, int32_t* out);
+mg_status mg_layout_plan(const mg_layout* lay, int32_t level, int32_t which /*0 send,1 recv*/, int64_t* out);
+mg_status mg_layout_destroy(mg_layout* lay);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MG_B200_H */

@@ -1,0 +1,987 @@
+// api.cu -- C ABI (include/mg.h), device workspace, executor, exchange transport.
+//
+// Runtime structure:
+//   mg_setup     validate -> host layout (layout.cpp) -> carve the caller's
+//                workspace into per-level brick fields + tables -> upload tables
+//                -> NCCL communicator (ncclCommInitRank from a torch-broadcast id)
+//   mg_vcycle    Builder (schedule.cpp) compiles Alg 2 into ops once per starting
+//                state; the op list is captured into ONE CUDA graph and replayed
+//                (kernels + NCCL send/recv + event fork/join for overlap)
+//   exchange     ghost bricks arrive as contiguous brick runs straight from the
+//                peer's field (no packing): ncclSend/ncclRecv per run inside one
+//                ncclGroup, or device copies for the in-process loopback group
+//   norm         fused applyOp + |b - Ax| + block max + atomicMax on the uint64
+//                bits (exact, order-free), ncclAllReduce(MAX) of 1 value
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "kernels.h"
+#include "mg_internal.h"
+#include "schedule.h"
+
+using namespace mgb;
+
+namespace {
+thread_local std::string g_err = "no error";
+
+mg_status set_err(mg_status s, const std::string& m) {
+  g_err = m;
+  return s;
+}
+
+struct DevLevel {
+  double* x[2] = {nullptr, nullptr};
+  double* b = nullptr;
+  double* r = nullptr;
+  double* Ax = nullptr;
+  int32_t* adj = nullptr;
+  int32_t* parent = nullptr;
+  int32_t* coord = nullptr;
+  Coeffs c{};
+  double h = 0;
+};
+
+struct Plan {
+  std::vector<Op> ops;
+  LevelState final_st[MG_MAX_LEVELS];
+  int64_t launches = 0;
+};
+
+struct TimerRec {
+  int slot;
+  cudaEvent_t a, b;
+};
+
+size_t align256(size_t v) { return (v + 255) & ~(size_t)255; }
+}  // namespace
+
+struct mg_group;
+
+struct mg_ctx {
+  Layout lay;
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  cudaStream_t comm = nullptr;
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+  std::vector<DevLevel> dl;
+  double* stage = nullptr;
+  unsigned long long* acc = nullptr;
+  double* h_pinned = nullptr;
+  ncclComm_t nccl = nullptr;
+  bool use_nccl = false;
+  mg_group* group = nullptr;
+  int grank = 0;
+  LevelState st[MG_MAX_LEVELS];
+  bool poisoned = false;
+  bool timing = false;
+  std::vector<double> tm;
+  std::vector<TimerRec> trec;
+  std::vector<cudaEvent_t> evpool;
+  size_t evnext = 0;
+  cudaGraphExec_t gexec[2] = {nullptr, nullptr};
+  Plan gplan[2];
+  bool gvalid[2] = {false, false};
+  int64_t last_launches = 0;
+};
+
+struct mg_group {
+  std::vector<mg_ctx*> r;
+  cudaStream_t stream = nullptr;
+  cudaGraphExec_t gexec[2] = {nullptr, nullptr};
+  Plan gplan[2];
+  bool gvalid[2] = {false, false};
+};
+
+#define CKC(ctx, call)                                                                        \
+  do {                                                                                        \
+    cudaError_t e_ = (call);                                                                  \
+    if (e_ != cudaSuccess) {                                                                  \
+      if (ctx) (ctx)->poisoned = true;                                                        \
+      return set_err(MG_ERR_CUDA, std::string(#call) + ": " + cudaGetErrorString(e_));        \
+    }                                                                                         \
+  } while (0)
+
+#define CKN(ctx, call)                                                                        \
+  do {                                                                                        \
+    ncclResult_t e_ = (call);                                                                 \
+    if (e_ != ncclSuccess) {                                                                  \
+      if (ctx) (ctx)->poisoned = true;                                                        \
+      return set_err(MG_ERR_NCCL, std::string(#call) + ": " + ncclGetErrorString(e_));        \
+    }                                                                                         \
+  } while (0)
+
+#define CKS(expr)                  \
+  do {                             \
+    mg_status s_ = (expr);         \
+    if (s_ != MG_OK) return s_;    \
+  } while (0)
+
+namespace {
+
+// ------------------------------------------------------------- workspace
+size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double** stage, unsigned long long** acc) {
+  size_t off = 0;
+  auto take = [&](size_t bytes) -> char* {
+    const size_t o = align256(off);
+    off = o + bytes;
+    return base ? base + o : nullptr;
+  };
+  if (out) out->assign(lay.L, DevLevel());
+  for (int l = 0; l < lay.L; ++l) {
+    const LevelLayout& L = lay.lv[l];
+    const size_t fb = (size_t)L.n_alloc * kBV * sizeof(double);
+    DevLevel d;
+    d.x[0] = (double*)take(fb);
+    d.x[1] = (double*)take(fb);
+    d.b = (double*)take(fb);
+    d.r = (double*)take(fb);
+    d.Ax = (double*)take(fb);
+    d.adj = (int32_t*)take((size_t)L.n_stored * 8 * sizeof(int32_t));
+    d.parent = (int32_t*)take((size_t)L.n_alloc * sizeof(int32_t));
+    d.coord = (int32_t*)take((size_t)L.n_stored * 3 * sizeof(int32_t));
+    d.h = lay.p.h0 * (double)(1 << l);
+    d.c = level_coeffs(d.h);
+    if (out) (*out)[l] = d;
+  }
+  double* st = (double*)take((size_t)lay.lv[0].n_owned * kBV * sizeof(double));
+  unsigned long long* ac = (unsigned long long*)take(256);
+  if (stage) *stage = st;
+  if (acc) *acc = ac;
+  return align256(off);
+}
+
+mg_params normalized(const mg_params* p) {
+  mg_params q = *p;
+  if (q.h0 <= 0) {
+    int64_t m = 0;
+    for (int a = 0; a < 3; ++a) {
+      const int64_t n = (int64_t)q.n_local[a] * q.proc_grid[a];
+      if (n > m) m = n;
+    }
+    q.h0 = m > 0 ? 1.0 / (double)m : 1.0;
+  }
+  return q;
+}
+
+mg_status check_params(const mg_params& p) {
+  if (p.num_levels > 1 && p.pre_smooths < 1)
+    return set_err(MG_ERR_INVALID_ARG, "pre_smooths must be >= 1 when num_levels > 1 (restriction reads its r)");
+  if (p.transport < 0 || p.transport > MG_TRANSPORT_LOCAL) return set_err(MG_ERR_INVALID_ARG, "bad transport");
+  if (p.bottom_mode < 0 || p.bottom_mode > MG_BOTTOM_RESIDENT) return set_err(MG_ERR_INVALID_ARG, "bad bottom_mode");
+  return MG_OK;
+}
+
+cudaEvent_t pool_event(mg_ctx* c) {
+  if (c->evnext == c->evpool.size()) {
+    cudaEvent_t e;
+    cudaEventCreate(&e);
+    c->evpool.push_back(e);
+  }
+  return c->evpool[c->evnext++];
+}
+
+// ------------------------------------------------------------- exchange
+double* field_ptr(mg_ctx* c, int l, int field, int xbuf) { return field ? c->dl[l].b : c->dl[l].x[xbuf]; }
+
+mg_status do_exchange(mg_ctx* c, int l, int field, int xbuf, cudaStream_t s) {
+  const LevelLayout& L = c->lay.lv[l];
+  double* f = field_ptr(c, l, field, xbuf);
+  const size_t bb = (size_t)kBV;
+  if (c->use_nccl) {
+    CKN(c, ncclGroupStart());
+    for (const Run& r : L.recvs)
+      CKN(c, ncclRecv(f + r.local * bb, (size_t)r.count * bb, ncclFloat64, r.peer, c->nccl, s));
+    for (const Run& r : L.sends)
+      CKN(c, ncclSend(f + r.local * bb, (size_t)r.count * bb, ncclFloat64, r.peer, c->nccl, s));
+    CKN(c, ncclGroupEnd());
+  } else {
+    for (const Run& r : L.recvs) {
+      mg_ctx* src = c->group ? c->group->r[r.peer] : c;
+      const double* sp = field_ptr(src, l, field, xbuf);
+      CKC(c, cudaMemcpyAsync(f + r.local * bb, sp + r.remote * bb, (size_t)r.count * bb * sizeof(double),
+                             cudaMemcpyDeviceToDevice, s));
+    }
+  }
+  return MG_OK;
+}
+
+// ------------------------------------------------------------- executor
+mg_status sweep_range(mg_ctx* c, const Op& o, int64_t b0, int64_t b1, cudaStream_t s) {
+  if (b1 <= b0) return MG_OK;
+  DevLevel& d = c->dl[o.level];
+  const int l = o.level;
+  if (o.paper) {
+    CKC(c, launch_apply_op(d.x[o.src], d.Ax, d.adj, b0, b1 - b0, d.c, s));
+    CKC(c, launch_smooth(d.x[o.src], d.Ax, d.b, d.r, b0, b1 - b0, d.c, (o.flags & SW_WRITE_R) != 0, s));
+    return MG_OK;
+  }
+  SweepArgs a{};
+  a.x = d.x[o.src];
+  a.xo = d.x[o.dst];
+  a.b = d.b;
+  a.r = d.r;
+  a.adj = d.adj;
+  a.parent = d.parent;
+  if (l + 1 < c->lay.L) {
+    a.bc = c->dl[l + 1].b;
+    a.xc = c->dl[l + 1].x[o.cbuf];
+  }
+  a.brick0 = b0;
+  a.nbricks = b1 - b0;
+  a.c = d.c;
+  CKC(c, launch_sweep(a, o.flags, s));
+  return MG_OK;
+}
+
+mg_status timer_begin(mg_ctx* c, cudaStream_t s, cudaEvent_t* ev) {
+  if (!c->timing) return MG_OK;
+  *ev = pool_event(c);
+  CKC(c, cudaEventRecord(*ev, s));
+  return MG_OK;
+}
+mg_status timer_end(mg_ctx* c, cudaStream_t s, cudaEvent_t a, int level, int op) {
+  if (!c->timing) return MG_OK;
+  cudaEvent_t b = pool_event(c);
+  CKC(c, cudaEventRecord(b, s));
+  c->trec.push_back({level * MG_NUM_OPS + op, a, b});
+  return MG_OK;
+}
+
+mg_status exec_op(mg_ctx* c, const Op& o, cudaStream_t s) {
+  const LevelLayout& L = c->lay.lv[o.level];
+  DevLevel& d = c->dl[o.level];
+  cudaEvent_t t0 = nullptr;
+  switch (o.kind) {
+    case OP_SWEEP: {
+      const int64_t end = o.ghosts ? L.n_stored : L.n_owned;
+      if (o.exch_before) {
+        const bool split = c->lay.p.overlap && L.n_interior > 0;
+        if (split) {
+          CKS(timer_begin(c, s, &t0));
+          CKC(c, cudaEventRecord(c->ev_fork, s));
+          CKC(c, cudaStreamWaitEvent(c->comm, c->ev_fork, 0));
+          CKS(do_exchange(c, o.level, 0, o.src, c->comm));
+          CKC(c, cudaEventRecord(c->ev_join, c->comm));
+          CKS(sweep_range(c, o, 0, L.n_interior, s));
+          CKC(c, cudaStreamWaitEvent(s, c->ev_join, 0));
+          CKS(sweep_range(c, o, L.n_interior, end, s));
+          CKS(timer_end(c, s, t0, o.level, o.timer));
+          return MG_OK;
+        }
+        CKS(timer_begin(c, s, &t0));
+        CKS(do_exchange(c, o.level, 0, o.src, s));
+        CKS(timer_end(c, s, t0, o.level, MG_OP_EXCHANGE));
+      }
+      CKS(timer_begin(c, s, &t0));
+      CKS(sweep_range(c, o, 0, end, s));
+      CKS(timer_end(c, s, t0, o.level, o.timer));
+      return MG_OK;
+    }
+    case OP_RESTRICT:
+      CKS(timer_begin(c, s, &t0));
+      CKC(c, launch_restrict(d.r, c->dl[o.level + 1].b, d.parent, L.n_owned, s));
+      CKS(timer_end(c, s, t0, o.level, o.timer));
+      return MG_OK;
+    case OP_INTERP:
+      CKS(timer_begin(c, s, &t0));
+      CKC(c, launch_interp(d.x[o.src], c->dl[o.level + 1].x[o.cbuf], d.parent, L.n_owned, s));
+      CKS(timer_end(c, s, t0, o.level, o.timer));
+      return MG_OK;
+    case OP_ZERO:
+      CKS(timer_begin(c, s, &t0));
+      CKC(c, launch_zero(d.x[o.src], 0, L.n_stored, s));
+      CKS(timer_end(c, s, t0, o.level, o.timer));
+      return MG_OK;
+    case OP_EXCH:
+      CKS(timer_begin(c, s, &t0));
+      CKS(do_exchange(c, o.level, o.field, o.src, s));
+      CKS(timer_end(c, s, t0, o.level, o.timer));
+      return MG_OK;
+    case OP_BOTTOM_RES:
+      CKS(timer_begin(c, s, &t0));
+      CKC(c, launch_bottom_resident(d.x[o.src], d.x[o.dst], d.b, d.adj, (int)L.n_stored, o.n, o.zero, d.c, s));
+      CKS(timer_end(c, s, t0, o.level, o.timer));
+      return MG_OK;
+  }
+  return set_err(MG_ERR_STATE, "unknown op");
+}
+
+Plan make_plan(const Builder& b, const Layout& lay) {
+  Plan p;
+  p.ops = b.ops;
+  for (int l = 0; l < MG_MAX_LEVELS; ++l) p.final_st[l] = b.st[l];
+  for (const Op& o : p.ops) p.launches += op_launches(o, lay, lay.p.overlap != 0);
+  return p;
+}
+
+// execute a plan on one context or, in lockstep, on every rank of a group
+mg_status run_plan(mg_ctx* c, mg_group* g, const Plan& p, cudaStream_t s) {
+  for (const Op& o : p.ops) {
+    if (g) {
+      for (mg_ctx* r : g->r) CKS(exec_op(r, o, s));
+    } else {
+      CKS(exec_op(c, o, s));
+    }
+  }
+  return MG_OK;
+}
+
+mg_status collect_timings(mg_ctx* c) {
+  if (!c->timing) return MG_OK;
+  CKC(c, cudaStreamSynchronize(c->stream));
+  for (const TimerRec& t : c->trec) {
+    float ms = 0;
+    CKC(c, cudaEventElapsedTime(&ms, t.a, t.b));
+    if (t.slot >= 0 && t.slot < (int)c->tm.size()) c->tm[t.slot] += ms;
+  }
+  c->trec.clear();
+  c->evnext = 0;
+  return MG_OK;
+}
+
+mg_status check_ctx(mg_ctx* c) {
+  if (!c) return set_err(MG_ERR_INVALID_ARG, "null context");
+  if (c->poisoned) return set_err(MG_ERR_STATE, "context poisoned by an earlier CUDA/NCCL error");
+  if (cudaSetDevice(c->device) != cudaSuccess) return set_err(MG_ERR_CUDA, "cudaSetDevice failed");
+  return MG_OK;
+}
+
+mg_status build_and_run(mg_ctx* c, mg_group* g, bool vcycle_graph, Builder& b) {
+  const Plan p = make_plan(b, c->lay);
+  CKS(run_plan(c, g, p, g ? g->stream : c->stream));
+  if (g) {
+    for (mg_ctx* r : g->r)
+      for (int l = 0; l < MG_MAX_LEVELS; ++l) r->st[l] = p.final_st[l];
+  } else {
+    for (int l = 0; l < MG_MAX_LEVELS; ++l) c->st[l] = p.final_st[l];
+  }
+  c->last_launches = p.launches * (g ? (int64_t)g->r.size() : 1);
+  (void)vcycle_graph;
+  return MG_OK;
+}
+
+// V-cycle for a single context or a lockstep group, via a cached CUDA graph
+mg_status vcycle_impl(mg_ctx* c, mg_group* g) {
+  mg_ctx* c0 = g ? g->r[0] : c;
+  cudaStream_t s = g ? g->stream : c->stream;
+  const int key = c0->st[0].cur & 1;
+  const bool graph = c0->lay.p.use_graph && !c0->timing;
+  cudaGraphExec_t* gexec = g ? g->gexec : c->gexec;
+  Plan* gplan = g ? g->gplan : c->gplan;
+  bool* gvalid = g ? g->gvalid : c->gvalid;
+  if (!graph || !gvalid[key]) {
+    Builder b(c0->lay);
+    for (int l = 0; l < MG_MAX_LEVELS; ++l) b.st[l] = c0->st[l];
+    b.vcycle();
+    Plan p = make_plan(b, c0->lay);
+    if (graph) {
+      CKC(c0, cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
+      mg_status rs = run_plan(c0, g, p, s);
+      cudaGraph_t gr = nullptr;
+      cudaError_t ce = cudaStreamEndCapture(s, &gr);
+      if (rs != MG_OK) return rs;
+      CKC(c0, ce);
+      CKC(c0, cudaGraphInstantiate(&gexec[key], gr, 0));
+      cudaGraphDestroy(gr);
+      gplan[key] = p;
+      gvalid[key] = true;
+    } else {
+      CKS(run_plan(c0, g, p, s));
+      if (g) {
+        for (mg_ctx* r : g->r) {
+          for (int l = 0; l < MG_MAX_LEVELS; ++l) r->st[l] = p.final_st[l];
+          CKS(collect_timings(r));
+        }
+      } else {
+        for (int l = 0; l < MG_MAX_LEVELS; ++l) c->st[l] = p.final_st[l];
+        CKS(collect_timings(c));
+      }
+      c0->last_launches = p.launches * (g ? (int64_t)g->r.size() : 1);
+      return MG_OK;
+    }
+  }
+  CKC(c0, cudaGraphLaunch(gexec[key], s));
+  const Plan& p = gplan[key];
+  if (g) {
+    for (mg_ctx* r : g->r)
+      for (int l = 0; l < MG_MAX_LEVELS; ++l) r->st[l] = p.final_st[l];
+  } else {
+    for (int l = 0; l < MG_MAX_LEVELS; ++l) c->st[l] = p.final_st[l];
+  }
+  c0->last_launches = p.launches * (g ? (int64_t)g->r.size() : 1);
+  return MG_OK;
+}
+
+mg_status init_ctx(mg_ctx* c, const mg_params& p, int rank, int world, int device, cudaStream_t stream,
+                   void* workspace, size_t ws_bytes, bool tables_only_upload) {
+  std::string msg;
+  mg_status s = build_layout(p, rank, world, c->lay, msg);
+  if (s != MG_OK) return set_err(s, msg);
+  c->device = device;
+  c->stream = stream;
+  const size_t need = carve(c->lay, nullptr, nullptr, nullptr, nullptr);
+  if (!workspace || ws_bytes < need)
+    return set_err(MG_ERR_OOM, "workspace too small: need " + std::to_string(need) + " bytes");
+  if (((uintptr_t)workspace & 255) != 0) return set_err(MG_ERR_INVALID_ARG, "workspace must be 256-byte aligned");
+  carve(c->lay, (char*)workspace, &c->dl, &c->stage, &c->acc);
+  (void)tables_only_upload;
+  CKC(c, cudaMemsetAsync(workspace, 0, need, stream));
+  for (int l = 0; l < c->lay.L; ++l) {
+    const LevelLayout& L = c->lay.lv[l];
+    DevLevel& d = c->dl[l];
+    CKC(c, cudaMemcpyAsync(d.adj, L.adj.data(), L.adj.size() * sizeof(int32_t), cudaMemcpyHostToDevice, stream));
+    std::vector<int32_t> par = L.parent;
+    par.resize((size_t)L.n_alloc, -1);
+    CKC(c, cudaMemcpyAsync(d.parent, par.data(), par.size() * sizeof(int32_t), cudaMemcpyHostToDevice, stream));
+    CKC(c, cudaMemcpyAsync(d.coord, L.coord.data(), L.coord.size() * sizeof(int32_t), cudaMemcpyHostToDevice,
+                           stream));
+  }
+  CKC(c, cudaStreamSynchronize(stream));  // host vectors above are temporaries
+  CKC(c, cudaStreamCreateWithFlags(&c->comm, cudaStreamNonBlocking));
+  CKC(c, cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
+  CKC(c, cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming));
+  CKC(c, cudaMallocHost((void**)&c->h_pinned, 64));
+  c->tm.assign((size_t)c->lay.L * MG_NUM_OPS, 0.0);
+  for (int l = 0; l < MG_MAX_LEVELS; ++l) c->st[l] = LevelState();
+  c->st[0].db = 0;
+  return MG_OK;
+}
+
+void free_ctx(mg_ctx* c) {
+  if (!c) return;
+  for (int k = 0; k < 2; ++k)
+    if (c->gexec[k]) cudaGraphExecDestroy(c->gexec[k]);
+  if (c->nccl) ncclCommDestroy(c->nccl);
+  if (c->comm) cudaStreamDestroy(c->comm);
+  if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+  if (c->ev_join) cudaEventDestroy(c->ev_join);
+  for (cudaEvent_t e : c->evpool) cudaEventDestroy(e);
+  if (c->h_pinned) cudaFreeHost(c->h_pinned);
+  delete c;
+}
+
+mg_status set_level_field(mg_ctx* c, int l, int field, const double* src, bool exchange_b) {
+  if (l < 0 || l >= c->lay.L) return set_err(MG_ERR_INVALID_ARG, "level out of range");
+  if (((uintptr_t)src & 15) != 0) return set_err(MG_ERR_INVALID_ARG, "field pointer must be 16-byte aligned");
+  DevLevel& d = c->dl[l];
+  const LevelLayout& L = c->lay.lv[l];
+  double* dst = field == MG_FIELD_X ? d.x[c->st[l].cur] : field == MG_FIELD_B ? d.b : d.r;
+  CKC(c, launch_lex_to_brick(src, dst, d.coord, L.n_owned, L.n[0], L.n[1], c->stream));
+  if (field == MG_FIELD_X) {
+    c->st[l].dx = 0;
+    c->st[l].since = 1 << 20;
+  }
+  if (field == MG_FIELD_B) {
+    c->st[l].db = 0;
+    if (exchange_b && L.n_ghost > 0) {
+      CKS(do_exchange(c, l, 1, 0, c->stream));
+      c->st[l].db = MG_MAX_PERIOD;
+    }
+  }
+  return MG_OK;
+}
+
+}  // namespace
+
+// =====================================================================================
+extern "C" {
+
+void mg_params_default(mg_params* p) {
+  if (!p) return;
+  std::memset(p, 0, sizeof(*p));
+  for (int a = 0; a < 3; ++a) {
+    p->n_local[a] = 256;
+    p->proc_grid[a] = 1;
+  }
+  p->num_levels = 6;  // -l 6
+  p->pre_smooths = 12;
+  p->post_smooths = 12;
+  p->bottom_smooths = 100;
+  p->use_graph = 1;
+  p->overlap = 1;
+  p->h0 = 0.0;
+}
+
+mg_status mg_workspace_bytes(const mg_params* p, int32_t rank, int32_t world_size, size_t* out_bytes) {
+  if (!p || !out_bytes) return set_err(MG_ERR_INVALID_ARG, "null argument");
+  Layout lay;
+  std::string msg;
+  const mg_params q = normalized(p);
+  mg_status s = build_layout(q, rank, world_size, lay, msg);
+  if (s != MG_OK) return set_err(s, msg);
+  *out_bytes = carve(lay, nullptr, nullptr, nullptr, nullptr);
+  return MG_OK;
+}
+
+mg_status mg_nccl_unique_id(uint8_t out_id[128]) {
+  if (!out_id) return set_err(MG_ERR_INVALID_ARG, "null argument");
+  ncclUniqueId id;
+  ncclResult_t r = ncclGetUniqueId(&id);
+  if (r != ncclSuccess) return set_err(MG_ERR_NCCL, std::string("ncclGetUniqueId: ") + ncclGetErrorString(r));
+  static_assert(sizeof(id) == 128, "ncclUniqueId size");
+  std::memcpy(out_id, &id, 128);
+  return MG_OK;
+}
+
+mg_status mg_setup(const mg_params* p, int32_t rank, int32_t world_size, const uint8_t* nccl_id, int32_t device,
+                   void* cuda_stream, void* workspace, size_t ws_bytes, mg_ctx** out) {
+  if (!p || !out) return set_err(MG_ERR_INVALID_ARG, "null argument");
+  *out = nullptr;
+  const mg_params q = normalized(p);
+  CKS(check_params(q));
+  int ndev = 0;
+  cudaError_t ce = cudaGetDeviceCount(&ndev);
+  if (ce != cudaSuccess || ndev == 0)
+    return set_err(MG_ERR_CUDA, std::string("no CUDA device (no CPU fallback): ") + cudaGetErrorString(ce));
+  if (device < 0 || device >= ndev) return set_err(MG_ERR_INVALID_ARG, "device out of range");
+  ce = cudaSetDevice(device);
+  if (ce != cudaSuccess) return set_err(MG_ERR_CUDA, std::string("cudaSetDevice: ") + cudaGetErrorString(ce));
+  ce = kernels_init();
+  if (ce != cudaSuccess) return set_err(MG_ERR_CUDA, std::string("kernels_init: ") + cudaGetErrorString(ce));
+  mg_ctx* c = new mg_ctx();
+  mg_status s = init_ctx(c, q, rank, world_size, device, (cudaStream_t)cuda_stream, workspace, ws_bytes, false);
+  if (s != MG_OK) {
+    free_ctx(c);
+    return s;
+  }
+  bool any_ghost = false;
+  for (const auto& L : c->lay.lv) any_ghost |= L.n_ghost > 0;
+  const bool want_nccl = world_size > 1 || q.transport == MG_TRANSPORT_NCCL;
+  if (world_size > 1 && q.transport == MG_TRANSPORT_LOCAL) {
+    free_ctx(c);
+    return set_err(MG_ERR_INVALID_ARG, "multi-process runs need the NCCL transport (use mg_group_* for loopback)");
+  }
+  if (want_nccl) {
+    ncclUniqueId id;
+    if (nccl_id) {
+      std::memcpy(&id, nccl_id, 128);
+    } else if (world_size == 1) {
+      ncclResult_t r = ncclGetUniqueId(&id);
+      if (r != ncclSuccess) {
+        free_ctx(c);
+        return set_err(MG_ERR_NCCL, std::string("ncclGetUniqueId: ") + ncclGetErrorString(r));
+      }
+    } else {
+      free_ctx(c);
+      return set_err(MG_ERR_INVALID_ARG, "world_size > 1 needs an NCCL unique id");
+    }
+    ncclResult_t r = ncclCommInitRank(&c->nccl, world_size, id, rank);
+    if (r != ncclSuccess) {
+      c->nccl = nullptr;
+      free_ctx(c);
+      return set_err(MG_ERR_NCCL, std::string("ncclCommInitRank: ") + ncclGetErrorString(r));
+    }
+    c->use_nccl = true;
+  }
+  (void)any_ghost;
+  *out = c;
+  return MG_OK;
+}
+
+mg_status mg_set_rhs(mg_ctx* c, const double* b_dev) {
+  CKS(check_ctx(c));
+  if (!b_dev) return set_err(MG_ERR_INVALID_ARG, "null b");
+  return set_level_field(c, 0, MG_FIELD_B, b_dev, c->group == nullptr);
+}
+
+mg_status mg_set_rhs_host(mg_ctx* c, const double* b_host) {
+  CKS(check_ctx(c));
+  if (!b_host) return set_err(MG_ERR_INVALID_ARG, "null b");
+  const size_t bytes = (size_t)c->lay.lv[0].n_owned * kBV * sizeof(double);
+  CKC(c, cudaMemcpyAsync(c->stage, b_host, bytes, cudaMemcpyHostToDevice, c->stream));
+  return set_level_field(c, 0, MG_FIELD_B, c->stage, c->group == nullptr);
+}
+
+mg_status mg_set_solution(mg_ctx* c, const double* x_dev) {
+  CKS(check_ctx(c));
+  if (!x_dev) {
+    const LevelLayout& L = c->lay.lv[0];
+    CKC(c, cudaMemsetAsync(c->dl[0].x[c->st[0].cur], 0, (size_t)L.n_stored * kBV * sizeof(double), c->stream));
+    c->st[0].dx = 0;
+    return MG_OK;
+  }
+  return set_level_field(c, 0, MG_FIELD_X, x_dev, false);
+}
+
+mg_status mg_get_solution(mg_ctx* c, double* x_dev) {
+  CKS(check_ctx(c));
+  if (!x_dev || ((uintptr_t)x_dev & 15)) return set_err(MG_ERR_INVALID_ARG, "x must be a 16-byte aligned pointer");
+  const LevelLayout& L = c->lay.lv[0];
+  CKC(c, launch_brick_to_lex(c->dl[0].x[c->st[0].cur], x_dev, c->dl[0].coord, L.n_owned, L.n[0], L.n[1], c->stream));
+  return MG_OK;
+}
+
+mg_status mg_get_solution_host(mg_ctx* c, double* x_host) {
+  CKS(check_ctx(c));
+  if (!x_host) return set_err(MG_ERR_INVALID_ARG, "null x");
+  CKS(mg_get_solution(c, c->stage));
+  const size_t bytes = (size_t)c->lay.lv[0].n_owned * kBV * sizeof(double);
+  CKC(c, cudaMemcpyAsync(x_host, c->stage, bytes, cudaMemcpyDeviceToHost, c->stream));
+  CKC(c, cudaStreamSynchronize(c->stream));
+  return MG_OK;
+}
+
+mg_status mg_vcycle(mg_ctx* c) {
+  CKS(check_ctx(c));
+  if (c->group) return set_err(MG_ERR_STATE, "group member: use mg_group_vcycle");
+  return vcycle_impl(c, nullptr);
+}
+
+mg_status mg_residual_norm(mg_ctx* c, double* out) {
+  CKS(check_ctx(c));
+  if (!out) return set_err(MG_ERR_INVALID_ARG, "null out");
+  if (c->group) return set_err(MG_ERR_STATE, "group member: use mg_group_residual_norm");
+  const LevelLayout& L = c->lay.lv[0];
+  DevLevel& d = c->dl[0];
+  if (L.n_ghost > 0) {
+    CKS(do_exchange(c, 0, 0, c->st[0].cur, c->stream));
+    c->st[0].dx = MG_MAX_PERIOD;
+    c->st[0].since = 0;
+  }
+  CKC(c, cudaMemsetAsync(c->acc, 0, sizeof(unsigned long long), c->stream));
+  CKC(c, launch_norm(d.x[c->st[0].cur], d.b, d.adj, L.n_owned, d.c, c->acc, c->stream));
+  if (c->use_nccl && c->lay.world > 1)
+    CKN(c, ncclAllReduce(c->acc, c->acc, 1, ncclUint64, ncclMax, c->nccl, c->stream));
+  CKC(c, cudaMemcpyAsync(c->h_pinned, c->acc, sizeof(unsigned long long), cudaMemcpyDeviceToHost, c->stream));
+  CKC(c, cudaStreamSynchronize(c->stream));
+  std::memcpy(out, c->h_pinned, sizeof(double));
+  return MG_OK;
+}
+
+mg_status mg_solve(mg_ctx* c, double tol, int32_t max_cycles, int32_t* cycles_done, double* final_norm) {
+  CKS(check_ctx(c));
+  double nr = 0;
+  CKS(mg_residual_norm(c, &nr));
+  int k = 0;
+  while (nr > tol && k < max_cycles) {
+    CKS(mg_vcycle(c));
+    CKS(mg_residual_norm(c, &nr));
+    ++k;
+  }
+  if (cycles_done) *cycles_done = k;
+  if (final_norm) *final_norm = nr;
+  return nr > tol ? MG_NOT_CONVERGED : MG_OK;
+}
+
+mg_status mg_set_timing(mg_ctx* c, int32_t enabled) {
+  CKS(check_ctx(c));
+  c->timing = enabled != 0;
+  std::fill(c->tm.begin(), c->tm.end(), 0.0);
+  return MG_OK;
+}
+
+mg_status mg_get_timings(mg_ctx* c, double* out, int32_t cap) {
+  CKS(check_ctx(c));
+  if (!out) return set_err(MG_ERR_INVALID_ARG, "null out");
+  CKS(collect_timings(c));
+  const int n = std::min<int>(cap, (int)c->tm.size());
+  for (int i = 0; i < n; ++i) out[i] = c->tm[i];
+  return MG_OK;
+}
+
+mg_status mg_vcycle_launches(mg_ctx* c, int64_t* out) {
+  CKS(check_ctx(c));
+  if (!out) return set_err(MG_ERR_INVALID_ARG, "null out");
+  Builder b(c->lay);
+  for (int l = 0; l < MG_MAX_LEVELS; ++l) b.st[l] = c->st[l];
+  b.vcycle();
+  *out = make_plan(b, c->lay).launches;
+  return MG_OK;
+}
+
+mg_status mg_exchange_stats(mg_ctx* c, int64_t* bytes_per_cycle, int64_t* messages_per_cycle) {
+  CKS(check_ctx(c));
+  Builder b(c->lay);
+  for (int l = 0; l < MG_MAX_LEVELS; ++l) b.st[l] = c->st[l];
+  b.vcycle();
+  int64_t bytes = 0, msgs = 0;
+  for (const Op& o : b.ops) {
+    const bool ex = o.kind == OP_EXCH || (o.kind == OP_SWEEP && o.exch_before);
+    if (!ex) continue;
+    for (const Run& r : c->lay.lv[o.level].sends) {
+      bytes += r.count * kBV * (int64_t)sizeof(double);
+      ++msgs;
+    }
+  }
+  if (bytes_per_cycle) *bytes_per_cycle = bytes;
+  if (messages_per_cycle) *messages_per_cycle = msgs;
+  return MG_OK;
+}
+
+mg_status mg_destroy(mg_ctx* c) {
+  if (!c) return MG_OK;
+  if (c->group) return set_err(MG_ERR_STATE, "group member: use mg_group_destroy");
+  cudaSetDevice(c->device);
+  free_ctx(c);
+  return MG_OK;
+}
+
+const char* mg_last_error(void) { return g_err.c_str(); }
+
+// ---------------------------------------------------------------- per-op
+mg_status mg_level_set(mg_ctx* c, int32_t level, int32_t field, const double* src_dev) {
+  CKS(check_ctx(c));
+  if (!src_dev || field < 0 || field > MG_FIELD_R) return set_err(MG_ERR_INVALID_ARG, "bad field/pointer");
+  return set_level_field(c, level, field, src_dev, c->group == nullptr);
+}
+
+mg_status mg_level_get(mg_ctx* c, int32_t level, int32_t field, double* dst_dev) {
+  CKS(check_ctx(c));
+  if (!dst_dev || field < 0 || field > MG_FIELD_R || ((uintptr_t)dst_dev & 15))
+    return set_err(MG_ERR_INVALID_ARG, "bad field/pointer");
+  if (level < 0 || level >= c->lay.L) return set_err(MG_ERR_INVALID_ARG, "level out of range");
+  DevLevel& d = c->dl[level];
+  const LevelLayout& L = c->lay.lv[level];
+  const double* src = field == MG_FIELD_X ? d.x[c->st[level].cur] : field == MG_FIELD_B ? d.b : d.r;
+  CKC(c, launch_brick_to_lex(src, dst_dev, d.coord, L.n_owned, L.n[0], L.n[1], c->stream));
+  return MG_OK;
+}
+
+static mg_status single_only(mg_ctx* c) {
+  if (c->group) return set_err(MG_ERR_STATE, "per-op entry points are for single contexts");
+  return MG_OK;
+}
+
+mg_status mg_op_smooth(mg_ctx* c, int32_t level, int32_t n, int32_t write_r, int32_t fusion) {
+  CKS(check_ctx(c));
+  CKS(single_only(c));
+  if (level < 0 || level >= c->lay.L || n < 0 || fusion < 0 || fusion > MG_FUSION_FULL)
+    return set_err(MG_ERR_INVALID_ARG, "bad level/n/fusion");
+  Builder b(c->lay);
+  for (int l = 0; l < MG_MAX_LEVELS; ++l) b.st[l] = c->st[l];
+  b.fusion_override[level] = fusion == MG_FUSION_PAPER ? MG_FUSION_PAPER : MG_FUSION_SWEEP;
+  b.phase(level, n, false, write_r ? 1 : 0, false, MG_OP_SWEEP);
+  return build_and_run(c, nullptr, false, b);
+}
+
+mg_status mg_op_restrict(mg_ctx* c, int32_t level) {
+  CKS(check_ctx(c));
+  CKS(single_only(c));
+  if (level < 0 || level + 1 >= c->lay.L) return set_err(MG_ERR_INVALID_ARG, "restriction needs level+1 < L");
+  Builder b(c->lay);
+  for (int l = 0; l < MG_MAX_LEVELS; ++l) b.st[l] = c->st[l];
+  b.restrict_op(level);
+  return build_and_run(c, nullptr, false, b);
+}
+
+mg_status mg_op_interp(mg_ctx* c, int32_t level) {
+  CKS(check_ctx(c));
+  CKS(single_only(c));
+  if (level < 0 || level + 1 >= c->lay.L) return set_err(MG_ERR_INVALID_ARG, "interpolation needs level+1 < L");
+  Builder b(c->lay);
+  for (int l = 0; l < MG_MAX_LEVELS; ++l) b.st[l] = c->st[l];
+  b.interp_op(level);
+  return build_and_run(c, nullptr, false, b);
+}
+
+mg_status mg_op_bottom(mg_ctx* c, int32_t level, int32_t n) {
+  CKS(check_ctx(c));
+  CKS(single_only(c));
+  if (level < 0 || level >= c->lay.L || n < 0) return set_err(MG_ERR_INVALID_ARG, "bad level/n");
+  Builder b(c->lay);
+  for (int l = 0; l < MG_MAX_LEVELS; ++l) b.st[l] = c->st[l];
+  b.bottom(level, n, false);
+  return build_and_run(c, nullptr, false, b);
+}
+
+mg_status mg_sync(mg_ctx* c) {
+  CKS(check_ctx(c));
+  CKC(c, cudaStreamSynchronize(c->stream));
+  return MG_OK;
+}
+
+// ---------------------------------------------------------------- loopback group
+mg_status mg_group_setup(const mg_params* p, int32_t world_size, int32_t device, void* cuda_stream, void* workspace,
+                         size_t ws_bytes, mg_group** out) {
+  if (!p || !out || world_size < 1) return set_err(MG_ERR_INVALID_ARG, "bad argument");
+  *out = nullptr;
+  const mg_params q = normalized(p);
+  CKS(check_params(q));
+  int ndev = 0;
+  cudaError_t ce = cudaGetDeviceCount(&ndev);
+  if (ce != cudaSuccess || ndev == 0)
+    return set_err(MG_ERR_CUDA, std::string("no CUDA device (no CPU fallback): ") + cudaGetErrorString(ce));
+  ce = cudaSetDevice(device);
+  if (ce != cudaSuccess) return set_err(MG_ERR_CUDA, std::string("cudaSetDevice: ") + cudaGetErrorString(ce));
+  ce = kernels_init();
+  if (ce != cudaSuccess) return set_err(MG_ERR_CUDA, std::string("kernels_init: ") + cudaGetErrorString(ce));
+  size_t per = 0;
+  CKS(mg_workspace_bytes(&q, 0, world_size, &per));
+  per = align256(per);
+  if (!workspace || ws_bytes < per * (size_t)world_size)
+    return set_err(MG_ERR_OOM, "group workspace too small: need " + std::to_string(per * (size_t)world_size));
+  mg_group* g = new mg_group();
+  g->stream = (cudaStream_t)cuda_stream;
+  for (int r = 0; r < world_size; ++r) {
+    mg_ctx* c = new mg_ctx();
+    mg_status s = init_ctx(c, q, r, world_size, device, g->stream, (char*)workspace + per * (size_t)r, per, false);
+    c->group = g;
+    c->grank = r;
+    g->r.push_back(c);
+    if (s != MG_OK) {
+      mg_group_destroy(g);
+      return s;
+    }
+  }
+  *out = g;
+  return MG_OK;
+}
+
+mg_status mg_group_ctx(mg_group* g, int32_t rank, mg_ctx** out) {
+  if (!g || !out || rank < 0 || rank >= (int)g->r.size()) return set_err(MG_ERR_INVALID_ARG, "bad rank");
+  *out = g->r[rank];
+  return MG_OK;
+}
+
+mg_status mg_group_set_rhs(mg_group* g, int32_t rank, const double* b_dev) {
+  mg_ctx* c = nullptr;
+  CKS(mg_group_ctx(g, rank, &c));
+  return mg_set_rhs(c, b_dev);
+}
+
+mg_status mg_group_set_solution(mg_group* g, int32_t rank, const double* x_dev) {
+  mg_ctx* c = nullptr;
+  CKS(mg_group_ctx(g, rank, &c));
+  return mg_set_solution(c, x_dev);
+}
+
+mg_status mg_group_commit_rhs(mg_group* g) {
+  if (!g) return set_err(MG_ERR_INVALID_ARG, "null group");
+  for (mg_ctx* c : g->r) {
+    CKS(check_ctx(c));
+    if (c->lay.lv[0].n_ghost > 0) CKS(do_exchange(c, 0, 1, 0, g->stream));
+    c->st[0].db = MG_MAX_PERIOD;
+  }
+  return MG_OK;
+}
+
+mg_status mg_group_vcycle(mg_group* g) {
+  if (!g) return set_err(MG_ERR_INVALID_ARG, "null group");
+  CKS(check_ctx(g->r[0]));
+  return vcycle_impl(g->r[0], g);
+}
+
+mg_status mg_group_residual_norm(mg_group* g, double* out) {
+  if (!g || !out) return set_err(MG_ERR_INVALID_ARG, "null argument");
+  mg_ctx* c0 = g->r[0];
+  CKS(check_ctx(c0));
+  for (mg_ctx* c : g->r) {
+    if (c->lay.lv[0].n_ghost > 0) {
+      CKS(do_exchange(c, 0, 0, c->st[0].cur, g->stream));
+    }
+  }
+  for (mg_ctx* c : g->r) {
+    c->st[0].dx = MG_MAX_PERIOD;
+    c->st[0].since = 0;
+  }
+  CKC(c0, cudaMemsetAsync(c0->acc, 0, sizeof(unsigned long long), g->stream));
+  for (mg_ctx* c : g->r) {
+    const LevelLayout& L = c->lay.lv[0];
+    DevLevel& d = c->dl[0];
+    CKC(c0, launch_norm(d.x[c->st[0].cur], d.b, d.adj, L.n_owned, d.c, c0->acc, g->stream));
+  }
+  CKC(c0, cudaMemcpyAsync(c0->h_pinned, c0->acc, 8, cudaMemcpyDeviceToHost, g->stream));
+  CKC(c0, cudaStreamSynchronize(g->stream));
+  std::memcpy(out, c0->h_pinned, sizeof(double));
+  return MG_OK;
+}
+
+mg_status mg_group_destroy(mg_group* g) {
+  if (!g) return MG_OK;
+  for (int k = 0; k < 2; ++k)
+    if (g->gexec[k]) cudaGraphExecDestroy(g->gexec[k]);
+  for (mg_ctx* c : g->r) free_ctx(c);
+  delete g;
+  return MG_OK;
+}
+
+// ---------------------------------------------------------------- layout queries
+struct mg_layout {
+  Layout lay;
+};
+
+mg_status mg_layout_create(const mg_params* p, int32_t rank, int32_t world_size, mg_layout** out) {
+  if (!p || !out) return set_err(MG_ERR_INVALID_ARG, "null argument");
+  mg_layout* m = new mg_layout();
+  std::string msg;
+  const mg_params q = normalized(p);
+  mg_status s = build_layout(q, rank, world_size, m->lay, msg);
+  if (s != MG_OK) {
+    delete m;
+    return set_err(s, msg);
+  }
+  *out = m;
+  return MG_OK;
+}
+
+static mg_status lay_level(const mg_layout* m, int32_t level, const LevelLayout** L) {
+  if (!m || level < 0 || level >= m->lay.L) return set_err(MG_ERR_INVALID_ARG, "bad layout/level");
+  *L = &m->lay.lv[level];
+  return MG_OK;
+}
+
+mg_status mg_layout_level_info(const mg_layout* m, int32_t level, int64_t info[16]) {
+  const LevelLayout* L = nullptr;
+  CKS(lay_level(m, level, &L));
+  for (int a = 0; a < 3; ++a) {
+    info[a] = L->n[a];
+    info[3 + a] = L->nb[a];
+    info[6 + a] = L->g[a];
+  }
+  info[9] = L->n_owned;
+  info[10] = L->n_interior;
+  info[11] = L->n_ghost;
+  info[12] = L->n_alloc;
+  info[13] = (int64_t)L->sends.size();
+  info[14] = (int64_t)L->recvs.size();
+  info[15] = L->zero_brick;
+  return MG_OK;
+}
+
+mg_status mg_layout_adjacency(const mg_layout* m, int32_t level, int32_t* out) {
+  const LevelLayout* L = nullptr;
+  CKS(lay_level(m, level, &L));
+  std::memcpy(out, L->adj.data(), L->adj.size() * sizeof(int32_t));
+  return MG_OK;
+}
+
+mg_status mg_layout_coords(const mg_layout* m, int32_t level, int32_t* out) {
+  const LevelLayout* L = nullptr;
+  CKS(lay_level(m, level, &L));
+  std::memcpy(out, L->coord.data(), L->coord.size() * sizeof(int32_t));
+  return MG_OK;
+}
+
+mg_status mg_layout_parent(const mg_layout* m, int32_t level, int32_t* out) {
+  const LevelLayout* L = nullptr;
+  CKS(lay_level(m, level, &L));
+  for (int64_t b = 0; b < L->n_stored; ++b) out[b] = L->parent.empty() ? -1 : L->parent[(size_t)b];
+  return MG_OK;
+}
+
+mg_status mg_layout_plan(const mg_layout* m, int32_t level, int32_t which, int64_t* out) {
+  const LevelLayout* L = nullptr;
+  CKS(lay_level(m, level, &L));
+  const std::vector<Run>& v = which ? L->recvs : L->sends;
+  for (size_t i = 0; i < v.size(); ++i) {
+    out[i * 6 + 0] = v[i].peer;
+    out[i * 6 + 1] = v[i].dir;
+    out[i * 6 + 2] = v[i].run;
+    out[i * 6 + 3] = v[i].local;
+    out[i * 6 + 4] = v[i].remote;
+    out[i * 6 + 5] = v[i].count;
+  }
+  return MG_OK;
+}
+
+mg_status mg_layout_destroy(mg_layout* m) {
+  delete m;
+  return MG_OK;
+}
+
+}  // extern "C"

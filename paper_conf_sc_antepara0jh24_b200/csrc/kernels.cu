@@ -1,0 +1,465 @@
+// kernels.cu -- sm_100a FP64 brick kernels of the GMG V-cycle.
+//
+// Arithmetic: every operation is a separately rounded
+// binary64 op written with __dmul_rn / __dadd_rn / __dsub_rn (no FMA
+// contraction; the library is also compiled with --fmad=false), in the
+// canonical order of reading A8:
+//   sum = ((xW + xE) + (xS + xN)) + (xB + xT)
+//   a   = alpha*x + beta*sum                        applyOp
+//   r   = b - a                                     residual
+//   x'  = x + gamma*(a - b)                         smooth
+//   bc  = 0.125*(((r000+r100)+(r010+r110)) + ((r001+r101)+(r011+r111)))  restriction
+//   x  += xc(parent)                                interpolation+increment
+// so the result is bit-identical to the lexicographic CPU oracle whatever the
+// brick order, fusion variant, decomposition or ghost-exchange period.
+//
+// Brick cell (i,j,k) lives at i + 8j + 64k of its 512-double brick (A16).
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "kernels.h"
+
+namespace mgb {
+
+Coeffs level_coeffs(double h) {
+  const double inv = 1.0 / (h * h);
+  Coeffs c;
+  c.alpha = -6.0 * inv;
+  c.beta = inv;
+  c.gamma = (h * h) / 12.0;
+  return c;
+}
+
+#define DMUL __dmul_rn
+#define DADD __dadd_rn
+#define DSUB __dsub_rn
+
+__device__ __forceinline__ double stencil_a(double c, double w, double e, double s, double n, double bt, double tp,
+                                            double alpha, double beta) {
+  const double sum = DADD(DADD(DADD(w, e), DADD(s, n)), DADD(bt, tp));
+  return DADD(DMUL(alpha, c), DMUL(beta, sum));
+}
+
+// max that propagates NaN (a diverged iterate must not hide in the norm)
+__device__ __forceinline__ double nan_max(double a, double b) { return (b > a || b != b) ? b : a; }
+
+__device__ __forceinline__ double2 ldg2(const double* p) { return __ldg(reinterpret_cast<const double2*>(p)); }
+__device__ __forceinline__ double2 ld_stream2(const double* p) {
+  double2 v;
+  asm volatile("ld.global.nc.L1::no_allocate.v2.f64 {%0, %1}, [%2];"
+               : "=d"(v.x), "=d"(v.y)
+               : "l"(p));
+  return v;
+}
+__device__ __forceinline__ void st_stream2(double* p, double2 v) {
+  asm volatile("st.global.L1::no_allocate.v2.f64 [%0], {%1, %2};" ::"l"(p), "d"(v.x), "d"(v.y) : "memory");
+}
+
+// coarse-cell offset of fine cell (i,j,k) of a fine brick with octant o
+__device__ __forceinline__ int coarse_off(int oct, int i, int j, int k) {
+  const int ox = oct & 1, oy = (oct >> 1) & 1, oz = oct >> 2;
+  return (4 * ox + (i >> 1)) + 8 * (4 * oy + (j >> 1)) + 64 * (4 * oz + (k >> 1));
+}
+
+// ---------------------------------------------------------------------------
+// Fused sweep: one CTA (256 threads) per brick, 2 cells per thread.  The brick
+// is staged in shared memory (coalesced 128-bit loads), the six face halos are
+// gathered from the neighbour bricks named by the adjacency table, then
+//   x' = x + gamma (Ax - b)  and optionally  r = b - Ax  /  b_c = R r.
+// Modes: MODE_SWEEP (x', r?), MODE_APPLY (Ax only -> xo), MODE_NORM (max|b-Ax|).
+// ---------------------------------------------------------------------------
+enum { MODE_SWEEP = 0, MODE_APPLY = 1, MODE_NORM = 2 };
+
+template <int MODE, unsigned FLAGS>
+__global__ void __launch_bounds__(256) sweep_kernel(SweepArgs p, unsigned long long* acc) {
+  constexpr bool WRITE_R = (FLAGS & SW_WRITE_R) != 0;
+  constexpr bool RESTRICT = (FLAGS & SW_RESTRICT) != 0;
+  constexpr bool INTERP = (FLAGS & SW_INTERP) != 0;
+  constexpr bool ZERO_X = (FLAGS & SW_ZERO_X) != 0;
+  __shared__ __align__(16) double xs[512];
+  __shared__ double hw[64], he[64], hs[64], hn[64], hb[64], ht[64];
+  __shared__ __align__(16) double rs[RESTRICT ? 512 : 1];
+
+  const int t = threadIdx.x;
+  const int64_t brick = p.brick0 + blockIdx.x;
+  const int i0 = 2 * (t & 3), j = (t >> 2) & 7, k = t >> 5;
+  const int32_t* adj = p.adj + brick * 8;
+
+  double2 bv = make_double2(0.0, 0.0);
+  if (MODE != MODE_APPLY) bv = ld_stream2(p.b + brick * 512 + 2 * t);
+
+  if (!ZERO_X) {
+    double2 xv = ldg2(p.x + brick * 512 + 2 * t);
+    if (INTERP) {
+      const int pr = __ldg(p.parent + brick);
+      if (pr >= 0) {
+        const double* xc = p.xc + (int64_t)(pr >> 3) * 512;
+        const int co = coarse_off(pr & 7, i0, j, k);  // i0, i0+1 share a coarse cell
+        const double cv = __ldg(xc + co);
+        xv.x = DADD(xv.x, cv);
+        xv.y = DADD(xv.y, cv);
+      }
+    }
+    xs[2 * t] = xv.x;
+    xs[2 * t + 1] = xv.y;
+    // halos: faces W,E,S,N (t = 0..255), B,T (t = 0..127)
+    {
+      const int f = t >> 6, m = t & 63;
+      const int nb = __ldg(adj + f);
+      int ci, cj, ck;
+      if (f < 2) {
+        ci = f == 0 ? 7 : 0;
+        cj = m & 7;
+        ck = m >> 3;
+      } else {
+        ci = m & 7;
+        cj = f == 2 ? 7 : 0;
+        ck = m >> 3;
+      }
+      double v = __ldg(p.x + (int64_t)nb * 512 + ci + 8 * cj + 64 * ck);
+      if (INTERP) {
+        const int pr = __ldg(p.parent + nb);
+        if (pr >= 0) v = DADD(v, __ldg(p.xc + (int64_t)(pr >> 3) * 512 + coarse_off(pr & 7, ci, cj, ck)));
+      }
+      double* h = f == 0 ? hw : f == 1 ? he : f == 2 ? hs : hn;
+      h[m] = v;
+    }
+    if (t < 128) {
+      const int f = 4 + (t >> 6), m = t & 63;
+      const int nb = __ldg(adj + f);
+      const int ck = f == 4 ? 7 : 0;
+      double v = __ldg(p.x + (int64_t)nb * 512 + m + 64 * ck);
+      if (INTERP) {
+        const int pr = __ldg(p.parent + nb);
+        if (pr >= 0) v = DADD(v, __ldg(p.xc + (int64_t)(pr >> 3) * 512 + coarse_off(pr & 7, m & 7, m >> 3, ck)));
+      }
+      (f == 4 ? hb : ht)[m] = v;
+    }
+    __syncthreads();
+  }
+
+  double out[2], res[2];
+  double mx = 0.0;
+#pragma unroll
+  for (int ii = 0; ii < 2; ++ii) {
+    const int i = i0 + ii;
+    const int o = i + 8 * j + 64 * k;
+    double c, w, e, s, n, bt, tp;
+    if (ZERO_X) {
+      c = w = e = s = n = bt = tp = 0.0;
+    } else {
+      c = xs[o];
+      w = i > 0 ? xs[o - 1] : hw[j + 8 * k];
+      e = i < 7 ? xs[o + 1] : he[j + 8 * k];
+      s = j > 0 ? xs[o - 8] : hs[i + 8 * k];
+      n = j < 7 ? xs[o + 8] : hn[i + 8 * k];
+      bt = k > 0 ? xs[o - 64] : hb[i + 8 * j];
+      tp = k < 7 ? xs[o + 64] : ht[i + 8 * j];
+    }
+    const double a = stencil_a(c, w, e, s, n, bt, tp, p.c.alpha, p.c.beta);
+    const double bb = ii ? bv.y : bv.x;
+    if (MODE == MODE_APPLY) {
+      out[ii] = a;
+    } else if (MODE == MODE_NORM) {
+      mx = nan_max(mx, fabs(DSUB(bb, a)));
+    } else {
+      res[ii] = DSUB(bb, a);
+      out[ii] = DADD(c, DMUL(p.c.gamma, DSUB(a, bb)));
+    }
+  }
+
+  if (MODE == MODE_NORM) {
+    // exact max: compare as doubles, publish the bit pattern (monotone for >= 0)
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) mx = nan_max(mx, __shfl_xor_sync(0xffffffffu, mx, off));
+    __shared__ double wm[8];
+    if ((t & 31) == 0) wm[t >> 5] = mx;
+    __syncthreads();
+    if (t == 0) {
+      double m = wm[0];
+      for (int w = 1; w < 8; ++w) m = nan_max(m, wm[w]);
+      atomicMax(acc, (unsigned long long)__double_as_longlong(m));
+    }
+    return;
+  }
+  if (MODE == MODE_APPLY) {
+    st_stream2(p.xo + brick * 512 + 2 * t, make_double2(out[0], out[1]));
+    return;
+  }
+  st_stream2(p.xo + brick * 512 + 2 * t, make_double2(out[0], out[1]));
+  if (WRITE_R) st_stream2(p.r + brick * 512 + 2 * t, make_double2(res[0], res[1]));
+  if (RESTRICT) {
+    rs[2 * t] = res[0];
+    rs[2 * t + 1] = res[1];
+    __syncthreads();
+    if (t < 64) {
+      const int I = t & 3, J = (t >> 2) & 3, K = t >> 4;
+      const int f = 2 * I + 8 * (2 * J) + 64 * (2 * K);
+      const double r000 = rs[f], r100 = rs[f + 1], r010 = rs[f + 8], r110 = rs[f + 9];
+      const double r001 = rs[f + 64], r101 = rs[f + 65], r011 = rs[f + 72], r111 = rs[f + 73];
+      const double v =
+          DMUL(0.125, DADD(DADD(DADD(r000, r100), DADD(r010, r110)), DADD(DADD(r001, r101), DADD(r011, r111))));
+      const int pr = __ldg(p.parent + brick);
+      const int oct = pr & 7;
+      const int ox = oct & 1, oy = (oct >> 1) & 1, oz = oct >> 2;
+      p.bc[(int64_t)(pr >> 3) * 512 + (4 * ox + I) + 8 * (4 * oy + J) + 64 * (4 * oz + K)] = v;
+    }
+  }
+}
+
+template <unsigned FLAGS>
+static cudaError_t launch_sweep_t(const SweepArgs& a, cudaStream_t s) {
+  if (a.nbricks <= 0) return cudaSuccess;
+  sweep_kernel<MODE_SWEEP, FLAGS><<<(unsigned)a.nbricks, 256, 0, s>>>(a, nullptr);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_sweep(const SweepArgs& a, unsigned flags, cudaStream_t s) {
+  switch (flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP | SW_ZERO_X)) {
+    case 0: return launch_sweep_t<0>(a, s);
+    case SW_WRITE_R: return launch_sweep_t<SW_WRITE_R>(a, s);
+    case SW_RESTRICT: return launch_sweep_t<SW_RESTRICT>(a, s);
+    case SW_INTERP: return launch_sweep_t<SW_INTERP>(a, s);
+    case SW_INTERP | SW_WRITE_R: return launch_sweep_t<SW_INTERP | SW_WRITE_R>(a, s);
+    case SW_INTERP | SW_RESTRICT: return launch_sweep_t<SW_INTERP | SW_RESTRICT>(a, s);
+    case SW_ZERO_X: return launch_sweep_t<SW_ZERO_X>(a, s);
+    case SW_ZERO_X | SW_WRITE_R: return launch_sweep_t<SW_ZERO_X | SW_WRITE_R>(a, s);
+    case SW_ZERO_X | SW_RESTRICT: return launch_sweep_t<SW_ZERO_X | SW_RESTRICT>(a, s);
+    default: return cudaErrorInvalidValue;
+  }
+}
+
+cudaError_t launch_apply_op(const double* x, double* Ax, const int32_t* adj, int64_t brick0, int64_t nbricks,
+                            Coeffs c, cudaStream_t s) {
+  if (nbricks <= 0) return cudaSuccess;
+  SweepArgs a{};
+  a.x = x;
+  a.xo = Ax;
+  a.adj = adj;
+  a.brick0 = brick0;
+  a.nbricks = nbricks;
+  a.c = c;
+  sweep_kernel<MODE_APPLY, 0><<<(unsigned)nbricks, 256, 0, s>>>(a, nullptr);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_norm(const double* x, const double* b, const int32_t* adj, int64_t nbricks, Coeffs c,
+                        unsigned long long* acc, cudaStream_t s) {
+  if (nbricks <= 0) return cudaSuccess;
+  SweepArgs a{};
+  a.x = x;
+  a.b = b;
+  a.adj = adj;
+  a.brick0 = 0;
+  a.nbricks = nbricks;
+  a.c = c;
+  sweep_kernel<MODE_NORM, 0><<<(unsigned)nbricks, 256, 0, s>>>(a, acc);
+  return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------------------
+// smooth(+residual) of the paper's kernel set: pointwise, reads x, Ax, b.
+// ---------------------------------------------------------------------------
+template <bool WRITE_R>
+__global__ void __launch_bounds__(256) smooth_kernel(double* __restrict__ x, const double* __restrict__ Ax,
+                                                     const double* __restrict__ b, double* __restrict__ r,
+                                                     int64_t base, int64_t n2, double gamma) {
+  for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < n2; q += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t o = base + 2 * q;
+    const double2 xv = ldg2(x + o);
+    const double2 av = ld_stream2(Ax + o);
+    const double2 bv = ld_stream2(b + o);
+    double2 xn, rv;
+    rv.x = DSUB(bv.x, av.x);
+    rv.y = DSUB(bv.y, av.y);
+    xn.x = DADD(xv.x, DMUL(gamma, DSUB(av.x, bv.x)));
+    xn.y = DADD(xv.y, DMUL(gamma, DSUB(av.y, bv.y)));
+    st_stream2(x + o, xn);
+    if (WRITE_R) st_stream2(r + o, rv);
+  }
+}
+
+static int g_num_sms = 148;
+
+static unsigned grid_for(int64_t n2) {
+  const int64_t want = (n2 + 255) / 256;
+  const int64_t cap = (int64_t)g_num_sms * 8;
+  return (unsigned)(want < cap ? (want > 0 ? want : 1) : cap);
+}
+
+cudaError_t launch_smooth(double* x, const double* Ax, const double* b, double* r, int64_t brick0, int64_t nbricks,
+                          Coeffs c, bool write_r, cudaStream_t s) {
+  if (nbricks <= 0) return cudaSuccess;
+  const int64_t n2 = nbricks * 256;
+  if (write_r)
+    smooth_kernel<true><<<grid_for(n2), 256, 0, s>>>(x, Ax, b, r, brick0 * 512, n2, c.gamma);
+  else
+    smooth_kernel<false><<<grid_for(n2), 256, 0, s>>>(x, Ax, b, r, brick0 * 512, n2, c.gamma);
+  return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------------------
+// restriction: one CTA (128 threads) per fine brick -> 64 coarse cells of the
+// parent's octant.
+// ---------------------------------------------------------------------------
+__global__ void __launch_bounds__(128) restrict_kernel(const double* __restrict__ r, double* __restrict__ bc,
+                                                       const int32_t* __restrict__ parent) {
+  __shared__ __align__(16) double rs[512];
+  const int64_t f = blockIdx.x;
+  const int t = threadIdx.x;
+  const double2* src = reinterpret_cast<const double2*>(r + f * 512);
+  reinterpret_cast<double2*>(rs)[t] = __ldg(src + t);
+  reinterpret_cast<double2*>(rs)[t + 128] = __ldg(src + t + 128);
+  __syncthreads();
+  if (t < 64) {
+    const int I = t & 3, J = (t >> 2) & 3, K = t >> 4;
+    const int o = 2 * I + 16 * J + 128 * K;
+    const double v = DMUL(0.125, DADD(DADD(DADD(rs[o], rs[o + 1]), DADD(rs[o + 8], rs[o + 9])),
+                                      DADD(DADD(rs[o + 64], rs[o + 65]), DADD(rs[o + 72], rs[o + 73]))));
+    const int pr = __ldg(parent + f);
+    const int oct = pr & 7;
+    const int ox = oct & 1, oy = (oct >> 1) & 1, oz = oct >> 2;
+    bc[(int64_t)(pr >> 3) * 512 + (4 * ox + I) + 8 * (4 * oy + J) + 64 * (4 * oz + K)] = v;
+  }
+}
+
+cudaError_t launch_restrict(const double* r, double* bc, const int32_t* parent, int64_t nfine, cudaStream_t s) {
+  if (nfine <= 0) return cudaSuccess;
+  restrict_kernel<<<(unsigned)nfine, 128, 0, s>>>(r, bc, parent);
+  return cudaGetLastError();
+}
+
+// interpolation+increment: one CTA (256 threads) per fine brick, 2 cells each.
+__global__ void __launch_bounds__(256) interp_kernel(double* __restrict__ x, const double* __restrict__ xc,
+                                                     const int32_t* __restrict__ parent) {
+  const int64_t f = blockIdx.x;
+  const int t = threadIdx.x;
+  const int i0 = 2 * (t & 3), j = (t >> 2) & 7, k = t >> 5;
+  const int pr = __ldg(parent + f);
+  const double cv = __ldg(xc + (int64_t)(pr >> 3) * 512 + coarse_off(pr & 7, i0, j, k));
+  double2* px = reinterpret_cast<double2*>(x + f * 512) + t;
+  double2 v = *px;
+  v.x = DADD(v.x, cv);
+  v.y = DADD(v.y, cv);
+  *px = v;
+}
+
+cudaError_t launch_interp(double* x, const double* xc, const int32_t* parent, int64_t nfine, cudaStream_t s) {
+  if (nfine <= 0) return cudaSuccess;
+  interp_kernel<<<(unsigned)nfine, 256, 0, s>>>(x, xc, parent);
+  return cudaGetLastError();
+}
+
+__global__ void __launch_bounds__(256) zero_kernel(double* __restrict__ x, int64_t base, int64_t n2) {
+  for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < n2; q += (int64_t)gridDim.x * blockDim.x)
+    reinterpret_cast<double2*>(x + base)[q] = make_double2(0.0, 0.0);
+}
+
+cudaError_t launch_zero(double* x, int64_t brick0, int64_t nbricks, cudaStream_t s) {
+  if (nbricks <= 0) return cudaSuccess;
+  const int64_t n2 = nbricks * 256;
+  zero_kernel<<<grid_for(n2), 256, 0, s>>>(x, brick0 * 512, n2);
+  return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------------------
+// Resident bottom solver: all bricks of the coarsest level (no
+// ghosts, <= 8 bricks) in one CTA's shared memory; `sweeps` Jacobi sweeps with
+// a CTA barrier between sweeps instead of `sweeps` kernel launches.
+// ---------------------------------------------------------------------------
+__global__ void __launch_bounds__(1024) bottom_resident_kernel(const double* __restrict__ x, double* __restrict__ xo,
+                                                               const double* __restrict__ b,
+                                                               const int32_t* __restrict__ adj, int nbricks,
+                                                               int sweeps, int zero_x, Coeffs c) {
+  extern __shared__ __align__(16) double sm[];
+  const int n = nbricks * 512;
+  double* xa = sm;
+  double* xb = sm + n;
+  double* bs = sm + 2 * n;
+  __shared__ int sadj[kResidentMaxBricks * 8];
+  for (int q = threadIdx.x; q < n; q += blockDim.x) {
+    xa[q] = zero_x ? 0.0 : x[q];
+    bs[q] = b[q];
+  }
+  for (int q = threadIdx.x; q < nbricks * 8; q += blockDim.x) sadj[q] = adj[q];
+  __syncthreads();
+  for (int s = 0; s < sweeps; ++s) {
+    for (int q = threadIdx.x; q < n; q += blockDim.x) {
+      const int br = q >> 9, o = q & 511;
+      const int i = o & 7, j = (o >> 3) & 7, k = o >> 6;
+      const int* a = sadj + br * 8;
+      const double cc = xa[q];
+      const double w = i > 0 ? xa[q - 1] : xa[a[0] * 512 + o + 7];
+      const double e = i < 7 ? xa[q + 1] : xa[a[1] * 512 + o - 7];
+      const double ss = j > 0 ? xa[q - 8] : xa[a[2] * 512 + o + 56];
+      const double nn = j < 7 ? xa[q + 8] : xa[a[3] * 512 + o - 56];
+      const double bt = k > 0 ? xa[q - 64] : xa[a[4] * 512 + o + 448];
+      const double tp = k < 7 ? xa[q + 64] : xa[a[5] * 512 + o - 448];
+      const double av = stencil_a(cc, w, e, ss, nn, bt, tp, c.alpha, c.beta);
+      xb[q] = DADD(cc, DMUL(c.gamma, DSUB(av, bs[q])));
+    }
+    __syncthreads();
+    double* tmp = xa;
+    xa = xb;
+    xb = tmp;
+  }
+  for (int q = threadIdx.x; q < n; q += blockDim.x) xo[q] = xa[q];
+}
+
+cudaError_t launch_bottom_resident(const double* x, double* xo, const double* b, const int32_t* adj, int nbricks,
+                                   int sweeps, bool zero_x, Coeffs c, cudaStream_t s) {
+  if (nbricks <= 0 || nbricks > kResidentMaxBricks) return cudaErrorInvalidValue;
+  const size_t smem = (size_t)nbricks * 512 * 3 * sizeof(double);
+  bottom_resident_kernel<<<1, 1024, smem, s>>>(x, xo, b, adj, nbricks, sweeps, zero_x ? 1 : 0, c);
+  return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------------------
+// Layout conversion (mg_set_rhs / mg_get_solution; not timed in the V-cycle).
+// ---------------------------------------------------------------------------
+__global__ void __launch_bounds__(256) lex_to_brick_kernel(const double* __restrict__ lex, double* __restrict__ br,
+                                                           const int32_t* __restrict__ coord, int nx, int ny) {
+  const int64_t bI = blockIdx.x;
+  const int t = threadIdx.x;
+  const int i0 = 2 * (t & 3), j = (t >> 2) & 7, k = t >> 5;
+  const int cx = coord[bI * 3], cy = coord[bI * 3 + 1], cz = coord[bI * 3 + 2];
+  const int64_t li = (int64_t)(8 * cx + i0) + (int64_t)nx * ((int64_t)(8 * cy + j) + (int64_t)ny * (8 * cz + k));
+  reinterpret_cast<double2*>(br + bI * 512)[t] = *reinterpret_cast<const double2*>(lex + li);
+}
+
+__global__ void __launch_bounds__(256) brick_to_lex_kernel(const double* __restrict__ br, double* __restrict__ lex,
+                                                           const int32_t* __restrict__ coord, int nx, int ny) {
+  const int64_t bI = blockIdx.x;
+  const int t = threadIdx.x;
+  const int i0 = 2 * (t & 3), j = (t >> 2) & 7, k = t >> 5;
+  const int cx = coord[bI * 3], cy = coord[bI * 3 + 1], cz = coord[bI * 3 + 2];
+  const int64_t li = (int64_t)(8 * cx + i0) + (int64_t)nx * ((int64_t)(8 * cy + j) + (int64_t)ny * (8 * cz + k));
+  *reinterpret_cast<double2*>(lex + li) = reinterpret_cast<const double2*>(br + bI * 512)[t];
+}
+
+cudaError_t launch_lex_to_brick(const double* lex, double* bricks, const int32_t* coord, int64_t nowned, int nx,
+                                int ny, cudaStream_t s) {
+  if (nowned <= 0) return cudaSuccess;
+  lex_to_brick_kernel<<<(unsigned)nowned, 256, 0, s>>>(lex, bricks, coord, nx, ny);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_brick_to_lex(const double* bricks, double* lex, const int32_t* coord, int64_t nowned, int nx,
+                                int ny, cudaStream_t s) {
+  if (nowned <= 0) return cudaSuccess;
+  brick_to_lex_kernel<<<(unsigned)nowned, 256, 0, s>>>(bricks, lex, coord, nx, ny);
+  return cudaGetLastError();
+}
+
+cudaError_t kernels_init() {
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  e = cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev);
+  if (e != cudaSuccess) return e;
+  return cudaFuncSetAttribute(bottom_resident_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                              kResidentMaxBricks * 512 * 3 * (int)sizeof(double));
+}
+
+}  // namespace mgb

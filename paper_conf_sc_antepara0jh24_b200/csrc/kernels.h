@@ -1,0 +1,65 @@
+// kernels.h -- launchers for the sm_100a brick kernels (kernels.cu).
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+namespace mgb {
+
+// Level constants: alpha = -6/h^2, beta = 1/h^2, gamma = h^2/12.
+struct Coeffs {
+  double alpha, beta, gamma;
+};
+Coeffs level_coeffs(double h);
+
+// Fused sweep flags (template specialisations in kernels.cu)
+enum SweepFlags : unsigned {
+  SW_WRITE_R = 1u,     // write r = b - Ax (smooth+residual)
+  SW_RESTRICT = 2u,    // write b_coarse = R r into the parent octant instead of r
+  SW_INTERP = 4u,      // read x as x_fine + x_coarse(parent) (interpolation+increment fused)
+  SW_ZERO_X = 8u,      // x == 0 (initZero folded into the first coarse sweep)
+  SW_NO_SMOOTH = 16u,  // do not write x' (restriction-only last sweep is never used; kept for tests)
+};
+
+struct SweepArgs {
+  const double* x;       // input x (brick layout)
+  double* xo;            // output x'
+  const double* b;
+  double* r;
+  const int32_t* adj;    // [brick][8]
+  const int32_t* parent; // fine brick -> coarse brick*8 + octant
+  double* bc;            // coarse b (SW_RESTRICT)
+  const double* xc;      // coarse x (SW_INTERP)
+  int64_t brick0, nbricks;
+  Coeffs c;
+};
+
+cudaError_t launch_sweep(const SweepArgs& a, unsigned flags, cudaStream_t s);
+// applyOp (paper kernel set): Ax = alpha x + beta sum6
+cudaError_t launch_apply_op(const double* x, double* Ax, const int32_t* adj, int64_t brick0, int64_t nbricks,
+                            Coeffs c, cudaStream_t s);
+// smooth(+residual) pointwise (paper kernel set): x += gamma (Ax - b); r = b - Ax
+cudaError_t launch_smooth(double* x, const double* Ax, const double* b, double* r, int64_t brick0, int64_t nbricks,
+                          Coeffs c, bool write_r, cudaStream_t s);
+// restriction over fine bricks [0, nfine): bc[parent octant] = avg8(r)
+cudaError_t launch_restrict(const double* r, double* bc, const int32_t* parent, int64_t nfine, cudaStream_t s);
+// interpolation+increment over fine bricks [0, nfine): x += xc(parent)
+cudaError_t launch_interp(double* x, const double* xc, const int32_t* parent, int64_t nfine, cudaStream_t s);
+// initZero over bricks [brick0, brick0+n)
+cudaError_t launch_zero(double* x, int64_t brick0, int64_t nbricks, cudaStream_t s);
+// max |b - Ax| over bricks [0, n) -> atomicMax on *acc (uint64 bits of a non-negative double)
+cudaError_t launch_norm(const double* x, const double* b, const int32_t* adj, int64_t nbricks, Coeffs c,
+                        unsigned long long* acc, cudaStream_t s);
+// resident bottom solve: all `nbricks` (<= kResidentMaxBricks, no ghosts) in one CTA's shared memory
+constexpr int kResidentMaxBricks = 8;
+cudaError_t launch_bottom_resident(const double* x, double* xo, const double* b, const int32_t* adj, int nbricks,
+                                   int sweeps, bool zero_x, Coeffs c, cudaStream_t s);
+// layout conversion (not part of the V-cycle): lexicographic local <-> bricks [0, nowned)
+cudaError_t launch_lex_to_brick(const double* lex, double* bricks, const int32_t* coord, int64_t nowned, int nx,
+                                int ny, cudaStream_t s);
+cudaError_t launch_brick_to_lex(const double* bricks, double* lex, const int32_t* coord, int64_t nowned, int nx,
+                                int ny, cudaStream_t s);
+cudaError_t kernels_init();  // one-time attribute setup
+
+}  // namespace mgb

@@ -1,0 +1,268 @@
+// layout.cpp -- brick grids, adjacency, region ordering and exchange plans.
+//
+// Implements the data layout the paper's method rests on:
+//  * bricks: 8^3 blocks stored contiguously; an adjacency table replaces ijk
+//    indexing ("the brick data layout provides indirection from ijk stencil
+//    grids"; bricks P:L17, L59, L154);
+//  * communication avoiding: the ghost zone is one brick deep (8 cells), so
+//    several smooths run per exchange, with 26 neighbours;
+//  * packing/unpacking-free exchange: owned bricks are physically ordered by
+//    surface region, so each neighbour's data is a few contiguous brick runs
+//    sent straight from the field, and ghost bricks are stored in arrival
+//    order ("optimal brick layout", "packing- and unpacking-free
+//    communication buffers").  The order of the 26 surface regions below was
+//    found by tools/region_order_search.py: 42 runs for 26 neighbours.
+#include <algorithm>
+#include <array>
+#include <cstdio>
+#include <tuple>
+
+#include "mg_internal.h"
+
+namespace mgb {
+
+// Surface regions s in {-1,0,1}^3 \ 0 in physical storage order (after the
+// interior region).  Found offline (tools/region_order_search.py).
+static const int kRegionOrder[26][3] = {
+    {0, 1, 0},   {0, 1, -1},  {1, 1, -1},  {1, 1, 0},   {1, 1, 1},   {0, 1, 1},  {-1, 1, 1},
+    {-1, 1, 0},  {-1, 1, -1}, {-1, 0, -1}, {-1, -1, -1}, {0, -1, -1}, {0, 0, -1}, {1, 0, -1},
+    {1, -1, -1}, {1, -1, 0},  {1, 0, 0},   {-1, 0, 0},  {-1, 0, 1},  {0, 0, 1},  {1, 0, 1},
+    {1, -1, 1},  {0, -1, 1},  {-1, -1, 1}, {-1, -1, 0}, {0, -1, 0}};
+
+int neighbour_rank(const Layout& lay, int dx, int dy, int dz) {
+  const int* P = lay.p.proc_grid;
+  const int cx = (lay.coords[0] + dx + P[0]) % P[0];
+  const int cy = (lay.coords[1] + dy + P[1]) % P[1];
+  const int cz = (lay.coords[2] + dz + P[2]) % P[2];
+  return cx + P[0] * (cy + P[1] * cz);
+}
+
+int64_t LevelLayout::ext_index(int x, int y, int z) const {
+  const int ex = nb[0] + 2 * g[0], ey = nb[1] + 2 * g[1];
+  const int ez = nb[2] + 2 * g[2];
+  const int X = x + g[0], Y = y + g[1], Z = z + g[2];
+  if (X < 0 || Y < 0 || Z < 0 || X >= ex || Y >= ey || Z >= ez) return -1;
+  return ext2idx[(size_t)X + (size_t)ex * ((size_t)Y + (size_t)ey * Z)];
+}
+
+// Region code per axis: 0 mid, 1 low, 2 high, 3 both (one brick on that axis).
+static int axis_code(int c, int nb, int g) {
+  if (!g) return 0;
+  const bool lo = c == 0, hi = c == nb - 1;
+  return (lo && hi) ? 3 : lo ? 1 : hi ? 2 : 0;
+}
+
+static int region_rank(int cx, int cy, int cz) {
+  if (cx == 0 && cy == 0 && cz == 0) return 0;
+  if (cx == 3 || cy == 3 || cz == 3) return 100 + cx + 4 * cy + 16 * cz;
+  auto s = [](int c) { return c == 0 ? 0 : (c == 1 ? -1 : 1); };
+  const int sx = s(cx), sy = s(cy), sz = s(cz);
+  for (int r = 0; r < 26; ++r)
+    if (kRegionOrder[r][0] == sx && kRegionOrder[r][1] == sy && kRegionOrder[r][2] == sz) return 1 + r;
+  return 99;  // unreachable
+}
+
+static void build_level(const Layout& lay, int l, LevelLayout& L) {
+  const mg_params& p = lay.p;
+  for (int a = 0; a < 3; ++a) {
+    L.n[a] = p.n_local[a] >> l;
+    L.nb[a] = L.n[a] / kB;
+    L.g[a] = (p.ghost_mode == MG_GHOST_ALL || p.proc_grid[a] > 1) ? 1 : 0;
+  }
+  const int nbx = L.nb[0], nby = L.nb[1], nbz = L.nb[2];
+  const int ex = nbx + 2 * L.g[0], ey = nby + 2 * L.g[1], ez = nbz + 2 * L.g[2];
+  L.ext2idx.assign((size_t)ex * ey * ez, -1);
+
+  // ---- owned bricks, region-ordered ----
+  struct Key {
+    int rr, z, y, x;
+  };
+  std::vector<Key> owned;
+  owned.reserve((size_t)nbx * nby * nbz);
+  for (int z = 0; z < nbz; ++z)
+    for (int y = 0; y < nby; ++y)
+      for (int x = 0; x < nbx; ++x) {
+        const int rr = region_rank(axis_code(x, nbx, L.g[0]), axis_code(y, nby, L.g[1]), axis_code(z, nbz, L.g[2]));
+        owned.push_back({rr, z, y, x});
+      }
+  std::stable_sort(owned.begin(), owned.end(), [](const Key& a, const Key& b) {
+    return std::tie(a.rr, a.z, a.y, a.x) < std::tie(b.rr, b.z, b.y, b.x);
+  });
+  L.n_owned = (int64_t)owned.size();
+  L.n_interior = 0;
+  L.coord.clear();
+  for (size_t i = 0; i < owned.size(); ++i) {
+    const Key& k = owned[i];
+    if (k.rr == 0) ++L.n_interior;
+    L.coord.push_back(k.x);
+    L.coord.push_back(k.y);
+    L.coord.push_back(k.z);
+    L.ext2idx[(size_t)(k.x + L.g[0]) + (size_t)ex * ((size_t)(k.y + L.g[1]) + (size_t)ey * (k.z + L.g[2]))] =
+        (int32_t)i;
+  }
+  auto own_idx = [&](int x, int y, int z) -> int64_t { return L.ext_index(x, y, z); };
+
+  // ---- ghost bricks, by receiver direction, in the sender's storage order ----
+  L.sends.clear();
+  L.recvs.clear();
+  int64_t next = L.n_owned;
+  for (int d = 0; d < 27; ++d) {
+    int dx, dy, dz;
+    dir_from_index(d, dx, dy, dz);
+    if (dx == 0 && dy == 0 && dz == 0) continue;
+    const int dd[3] = {dx, dy, dz};
+    bool ok = true;
+    for (int a = 0; a < 3; ++a)
+      if (dd[a] != 0 && !L.g[a]) ok = false;
+    if (!ok) continue;
+    // sender-side brick set: c_a = nb-1 if d_a=-1, 0 if d_a=+1, all if 0
+    int lo[3], hi[3];
+    for (int a = 0; a < 3; ++a) {
+      if (dd[a] == -1) {
+        lo[a] = L.nb[a] - 1;
+        hi[a] = L.nb[a];
+      } else if (dd[a] == 1) {
+        lo[a] = 0;
+        hi[a] = 1;
+      } else {
+        lo[a] = 0;
+        hi[a] = L.nb[a];
+      }
+    }
+    std::vector<std::pair<int64_t, std::array<int, 3>>> set;  // (sender own idx, sender coords)
+    for (int z = lo[2]; z < hi[2]; ++z)
+      for (int y = lo[1]; y < hi[1]; ++y)
+        for (int x = lo[0]; x < hi[0]; ++x) set.push_back({own_idx(x, y, z), {x, y, z}});
+    std::sort(set.begin(), set.end());
+    const int recv_peer = neighbour_rank(lay, dx, dy, dz);     // my ghost d comes from me+d
+    const int send_peer = neighbour_rank(lay, -dx, -dy, -dz);  // my bricks go to me-d (its ghost d)
+    const int64_t gstart = next;
+    int run = 0;
+    for (size_t m = 0; m < set.size();) {
+      size_t e = m + 1;
+      while (e < set.size() && set[e].first == set[e - 1].first + 1) ++e;
+      const int64_t cnt = (int64_t)(e - m);
+      const int64_t goff = gstart + (int64_t)m;
+      L.recvs.push_back({recv_peer, d, run, goff, set[m].first, cnt});
+      L.sends.push_back({send_peer, d, run, set[m].first, goff, cnt});
+      ++run;
+      m = e;
+    }
+    // ghost bricks: extended coords of receiver ghost region d
+    for (size_t m = 0; m < set.size(); ++m) {
+      const auto& c = set[m].second;
+      int e3[3];
+      for (int a = 0; a < 3; ++a) e3[a] = dd[a] == -1 ? -1 : dd[a] == 1 ? L.nb[a] : c[a];
+      L.coord.push_back(e3[0]);
+      L.coord.push_back(e3[1]);
+      L.coord.push_back(e3[2]);
+      L.ext2idx[(size_t)(e3[0] + L.g[0]) + (size_t)ex * ((size_t)(e3[1] + L.g[1]) + (size_t)ey * (e3[2] + L.g[2]))] =
+          (int32_t)(gstart + (int64_t)m);
+    }
+    next += (int64_t)set.size();
+  }
+  L.n_stored = next;
+  L.n_ghost = next - L.n_owned;
+  L.zero_brick = next;
+  L.n_alloc = next + 1;
+  // NCCL matches sends/recvs between a pair in posting order: sort both by (peer, dir, run)
+  auto cmp = [](const Run& a, const Run& b) { return std::tie(a.peer, a.dir, a.run) < std::tie(b.peer, b.dir, b.run); };
+  std::sort(L.sends.begin(), L.sends.end(), cmp);
+  std::sort(L.recvs.begin(), L.recvs.end(), cmp);
+
+  // ---- adjacency: W,E,S,N,B,T,self,0 ----
+  L.adj.assign((size_t)L.n_stored * 8, 0);
+  static const int F[6][3] = {{-1, 0, 0}, {1, 0, 0}, {0, -1, 0}, {0, 1, 0}, {0, 0, -1}, {0, 0, 1}};
+  for (int64_t b = 0; b < L.n_stored; ++b) {
+    const int* e = &L.coord[(size_t)b * 3];
+    for (int f = 0; f < 6; ++f) {
+      int q[3];
+      bool zero = false;
+      for (int a = 0; a < 3; ++a) {
+        q[a] = e[a] + F[f][a];
+        if (!L.g[a]) {
+          q[a] = (q[a] % L.nb[a] + L.nb[a]) % L.nb[a];
+        } else if (q[a] < -1 || q[a] > L.nb[a]) {
+          zero = true;
+        }
+      }
+      int64_t idx = zero ? -1 : L.ext_index(q[0], q[1], q[2]);
+      L.adj[(size_t)b * 8 + f] = (int32_t)(idx < 0 ? L.zero_brick : idx);
+    }
+    L.adj[(size_t)b * 8 + 6] = (int32_t)b;
+    L.adj[(size_t)b * 8 + 7] = 0;
+  }
+}
+
+static void build_parents(LevelLayout& F, const LevelLayout& C) {
+  F.parent.assign((size_t)F.n_alloc, -1);  // zero brick has no parent
+  for (int64_t b = 0; b < F.n_stored; ++b) {
+    const int* e = &F.coord[(size_t)b * 3];
+    int E[3], o[3];
+    for (int a = 0; a < 3; ++a) {
+      E[a] = (e[a] >= 0) ? e[a] / 2 : -1;  // floor(e/2) for e >= -1
+      o[a] = e[a] - 2 * E[a];
+    }
+    const int64_t ci = C.ext_index(E[0], E[1], E[2]);
+    if (ci >= 0) F.parent[(size_t)b] = (int32_t)(ci * 8 + o[0] + 2 * o[1] + 4 * o[2]);
+  }
+}
+
+mg_status build_layout(const mg_params& p, int rank, int world, Layout& out, std::string& msg) {
+  char buf[256];
+  if (world < 1 || rank < 0 || rank >= world) {
+    msg = "rank/world_size out of range";
+    return MG_ERR_INVALID_ARG;
+  }
+  if (p.proc_grid[0] < 1 || p.proc_grid[1] < 1 || p.proc_grid[2] < 1 ||
+      (int64_t)p.proc_grid[0] * p.proc_grid[1] * p.proc_grid[2] != world) {
+    snprintf(buf, sizeof buf, "proc_grid %dx%dx%d does not match world_size %d", p.proc_grid[0], p.proc_grid[1],
+             p.proc_grid[2], world);
+    msg = buf;
+    return MG_ERR_INVALID_ARG;
+  }
+  if (p.num_levels < 1 || p.num_levels > MG_MAX_LEVELS) {
+    msg = "num_levels must be in [1, 16]";
+    return MG_ERR_INVALID_ARG;
+  }
+  const int64_t unit = (int64_t)kB << (p.num_levels - 1);
+  for (int a = 0; a < 3; ++a) {
+    if (p.n_local[a] <= 0 || p.n_local[a] % unit != 0) {
+      snprintf(buf, sizeof buf, "n_local[%d]=%d must be a positive multiple of 8*2^(num_levels-1)=%lld", a,
+               p.n_local[a], (long long)unit);
+      msg = buf;
+      return MG_ERR_INVALID_ARG;
+    }
+  }
+  if (p.pre_smooths < 0 || p.post_smooths < 0 || p.bottom_smooths < 0) {
+    msg = "sweep counts must be >= 0";
+    return MG_ERR_INVALID_ARG;
+  }
+  for (int l = 0; l < MG_MAX_LEVELS; ++l) {
+    if (p.ca_period[l] < 0 || p.ca_period[l] > MG_MAX_PERIOD) {
+      msg = "ca_period must be in [0, 8] (ghost depth = brick edge, P:L156)";
+      return MG_ERR_INVALID_ARG;
+    }
+    if (p.fusion[l] < 0 || p.fusion[l] > MG_FUSION_FULL) {
+      msg = "fusion must be in [0, 3]";
+      return MG_ERR_INVALID_ARG;
+    }
+  }
+  if (p.ghost_mode != MG_GHOST_AUTO && p.ghost_mode != MG_GHOST_ALL) {
+    msg = "ghost_mode must be 0 or 1";
+    return MG_ERR_INVALID_ARG;
+  }
+  out.p = p;
+  out.rank = rank;
+  out.world = world;
+  out.coords[0] = rank % p.proc_grid[0];
+  out.coords[1] = (rank / p.proc_grid[0]) % p.proc_grid[1];
+  out.coords[2] = rank / (p.proc_grid[0] * p.proc_grid[1]);
+  out.L = p.num_levels;
+  out.lv.assign(out.L, LevelLayout());
+  for (int l = 0; l < out.L; ++l) build_level(out, l, out.lv[l]);
+  for (int l = 0; l + 1 < out.L; ++l) build_parents(out.lv[l], out.lv[l + 1]);
+  return MG_OK;
+}
+
+}  // namespace mgb

@@ -1,0 +1,72 @@
+// mg_internal.h -- host-side structures of the B200 brick-GMG library.
+//
+// Brick layout: every level's local subdomain is cut
+// into 8^3 bricks, each stored contiguously (512 doubles, cell (i,j,k) of the
+// brick at i + 8j + 64k, reading A16).  A brick table gives, per stored brick,
+// its 6 face neighbours (adjacency), so kernels never compute ijk -> address.
+//
+// Storage order per level:  [interior owned | surface owned (26 regions in
+// kRegionOrder) | ghost bricks (by direction, in the sender's order) | zero brick]
+// Periodic axes that are not decomposed are closed by wrapping the adjacency;
+// decomposed axes (or all axes in MG_GHOST_ALL) get a one-brick ghost shell
+// (P:L156).
+#pragma once
+
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "../../include/mg.h"
+
+namespace mgb {
+
+constexpr int kB = MG_BRICK;          // brick edge
+constexpr int kBV = kB * kB * kB;     // values per brick (512)
+
+// One message of an exchange: contiguous bricks [local, local+count) on this
+// rank are sent to / received from `peer`.  `remote` is the brick offset of
+// the same run on the peer (known because every rank has the same layout).
+struct Run {
+  int32_t peer;
+  int32_t dir;      // direction index 0..26 of the RECEIVER's ghost region (d+1 base 3)
+  int32_t run;      // index of the run within (peer, dir)
+  int64_t local;    // brick offset on this rank
+  int64_t remote;   // brick offset on the peer
+  int64_t count;    // bricks
+};
+
+struct LevelLayout {
+  int n[3] = {0, 0, 0};    // cells per axis
+  int nb[3] = {0, 0, 0};   // owned bricks per axis
+  int g[3] = {0, 0, 0};    // ghost layer on axis (0 = periodic wrap inside the rank)
+  int64_t n_owned = 0, n_interior = 0, n_ghost = 0, n_stored = 0, n_alloc = 0;
+  int64_t zero_brick = 0;  // index of the all-zero brick (neighbour of the outermost ghosts)
+  std::vector<int32_t> adj;     // [n_stored][8]
+  std::vector<int32_t> coord;   // [n_stored][3] extended brick coords
+  std::vector<int32_t> parent;  // [n_stored] coarse brick * 8 + octant, -1 if none
+  std::vector<Run> sends, recvs;
+  int64_t ext_index(int x, int y, int z) const;  // -1 if not stored
+  std::vector<int32_t> ext2idx;  // dense map over the extended box
+};
+
+struct Layout {
+  mg_params p{};
+  int rank = 0, world = 1;
+  int coords[3] = {0, 0, 0};
+  int L = 0;
+  std::vector<LevelLayout> lv;
+};
+
+// Validates params and builds every level.  Returns MG_OK or an error with msg.
+mg_status build_layout(const mg_params& p, int rank, int world, Layout& out, std::string& msg);
+
+// ---- neighbour helpers ----
+inline int dir_index(int dx, int dy, int dz) { return (dx + 1) + 3 * (dy + 1) + 9 * (dz + 1); }
+inline void dir_from_index(int d, int& dx, int& dy, int& dz) {
+  dx = d % 3 - 1;
+  dy = (d / 3) % 3 - 1;
+  dz = d / 9 - 1;
+}
+int neighbour_rank(const Layout& lay, int dx, int dy, int dz);
+
+}  // namespace mgb

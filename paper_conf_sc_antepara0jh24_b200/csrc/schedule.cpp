@@ -1,0 +1,187 @@
+// schedule.cpp -- compiles Alg 2 into device ops; see schedule.h.
+#include "schedule.h"
+
+#include <algorithm>
+
+#include "kernels.h"
+
+namespace mgb {
+
+Builder::Builder(const Layout& l) : lay(l) {
+  for (int i = 0; i < MG_MAX_LEVELS; ++i) fusion_override[i] = 0;
+}
+
+int Builder::fusion(int l) const {
+  if (fusion_override[l]) return fusion_override[l];
+  const int f = lay.p.fusion[l];
+  return f ? f : MG_FUSION_FULL;
+}
+
+int Builder::period(int l) const {
+  const int k = lay.p.ca_period[l];
+  return k ? k : MG_MAX_PERIOD;
+}
+
+void Builder::phase(int l, int n, bool zero_first, int last, bool interp_first, int timer) {
+  const bool g = ghosts(l);
+  const int k = period(l);
+  const bool paper = fusion(l) == MG_FUSION_PAPER;
+  LevelState& S = st[l];
+  for (int s = 0; s < n; ++s) {
+    Op o;
+    o.kind = OP_SWEEP;
+    o.level = l;
+    o.paper = paper;
+    o.timer = timer;
+    const bool zero = zero_first && s == 0;
+    const bool ex = g && !zero && (S.dx < 1 || S.since >= k);
+    if (ex) {
+      S.dx = MG_MAX_PERIOD;
+      S.since = 0;
+    }
+    o.exch_before = ex;
+    const int d_inc = zero ? S.db : std::min(S.dx - 1, S.db);
+    const bool last_s = s == n - 1;
+    o.ghosts = g && !last_s && d_inc >= 1 && (S.since + 1) < k;
+    if (zero) o.flags |= SW_ZERO_X;
+    if (interp_first && s == 0) {
+      o.flags |= SW_INTERP;
+      o.cbuf = st[l + 1].cur;
+    }
+    if (last_s && last == 1) o.flags |= SW_WRITE_R;
+    if (last_s && last == 2) o.flags |= SW_RESTRICT;
+    o.src = S.cur;
+    o.dst = paper ? S.cur : 1 - S.cur;
+    S.cur = o.dst;
+    S.dx = o.ghosts ? d_inc : 0;
+    S.since += 1;
+    ops.push_back(o);
+  }
+}
+
+void Builder::exchange_b(int l) {
+  if (!ghosts(l)) return;
+  Op o;
+  o.kind = OP_EXCH;
+  o.level = l;
+  o.field = 1;
+  o.timer = MG_OP_EXCHANGE;
+  ops.push_back(o);
+  st[l].db = MG_MAX_PERIOD;
+}
+
+void Builder::restrict_op(int l) {
+  Op o;
+  o.kind = OP_RESTRICT;
+  o.level = l;
+  o.timer = MG_OP_RESTRICT;
+  ops.push_back(o);
+  exchange_b(l + 1);
+}
+
+void Builder::zero_op(int l) {
+  Op o;
+  o.kind = OP_ZERO;
+  o.level = l;
+  o.src = o.dst = st[l].cur;
+  o.timer = MG_OP_ZERO;
+  ops.push_back(o);
+  st[l].dx = MG_MAX_PERIOD;  // zero is the true value of every ghost too
+  st[l].since = 0;
+}
+
+void Builder::interp_op(int l) {
+  Op o;
+  o.kind = OP_INTERP;
+  o.level = l;
+  o.src = o.dst = st[l].cur;
+  o.cbuf = st[l + 1].cur;
+  o.timer = MG_OP_INTERP;
+  ops.push_back(o);
+  st[l].dx = 0;  // owned bricks only: ghosts stale until the next exchange
+}
+
+void Builder::bottom(int l, int n, bool zero) {
+  if (n <= 0) return;
+  const LevelLayout& L = lay.lv[l];
+  const int bm = lay.p.bottom_mode;
+  const bool can_res = !ghosts(l) && L.n_stored <= kResidentMaxBricks;
+  const bool res = can_res && (bm == MG_BOTTOM_RESIDENT || (bm == MG_BOTTOM_AUTO && fusion(l) != MG_FUSION_PAPER));
+  const bool fold_zero = zero && fusion(l) == MG_FUSION_FULL;
+  if (res) {
+    Op o;
+    o.kind = OP_BOTTOM_RES;
+    o.level = l;
+    o.src = st[l].cur;
+    o.dst = 1 - st[l].cur;
+    o.n = n;
+    o.zero = fold_zero;
+    o.timer = MG_OP_BOTTOM;
+    st[l].cur = o.dst;
+    st[l].dx = 0;
+    ops.push_back(o);
+    return;
+  }
+  phase(l, n, fold_zero, 0, false, MG_OP_BOTTOM);
+}
+
+void Builder::vcycle() {
+  const int L = lay.L;
+  const mg_params& p = lay.p;
+  // Coarse x is dead at the start of a cycle (zeroed below): normalise its buffer.
+  for (int l = 1; l < L; ++l) {
+    st[l].cur = 0;
+    st[l].dx = 0;
+    st[l].db = 0;
+    st[l].since = 1 << 20;
+  }
+  // level-0 ghosts of x are conservatively stale at the start of a cycle
+  st[0].dx = 0;
+  st[0].since = 1 << 20;
+  if (L == 1) {
+    bottom(0, p.bottom_smooths, false);
+    return;
+  }
+  for (int l = 0; l + 1 < L; ++l) {  // Alg 2 steps 1-8
+    const bool full = fusion(l) == MG_FUSION_FULL;
+    const bool zero_first = l > 0 && full;
+    phase(l, p.pre_smooths, zero_first, full ? 2 : 1, false, MG_OP_SWEEP);
+    if (full)
+      exchange_b(l + 1);  // restriction fused into the last pre-sweep
+    else
+      restrict_op(l);
+    // the fold needs a first coarse sweep to absorb it (pre_smooths >= 1 is validated)
+    const bool fold = fusion(l + 1) == MG_FUSION_FULL && (l + 2 < L || p.bottom_smooths > 0);
+    if (!fold)  // initZero as its own kernel (Alg 2 step 8)
+      zero_op(l + 1);
+    else {
+      st[l + 1].dx = MG_MAX_PERIOD;  // folded into the first coarse sweep
+      st[l + 1].since = 0;
+    }
+  }
+  bottom(L - 1, p.bottom_smooths, true);  // steps 10-15
+  for (int l = L - 2; l >= 0; --l) {       // steps 16-23
+    const bool fuse_i = fusion(l) == MG_FUSION_FULL && !ghosts(l) && p.post_smooths > 0;
+    if (!fuse_i) interp_op(l);
+    phase(l, p.post_smooths, false, 0, fuse_i, MG_OP_SWEEP);
+  }
+}
+
+int64_t op_launches(const Op& o, const Layout& lay, bool overlap) {
+  switch (o.kind) {
+    case OP_SWEEP: {
+      const int per = o.paper ? 2 : 1;
+      const bool split = o.exch_before && overlap && lay.lv[o.level].n_interior > 0;
+      return per * (split ? 2 : 1);
+    }
+    case OP_RESTRICT:
+    case OP_INTERP:
+    case OP_ZERO:
+    case OP_BOTTOM_RES:
+      return 1;
+    default:
+      return 0;
+  }
+}
+
+}  // namespace mgb

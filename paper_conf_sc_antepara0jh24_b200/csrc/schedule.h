@@ -1,0 +1,65 @@
+// schedule.h -- the V-cycle as a host-compiled list of device operations.
+//
+// Alg 2 is compiled once per starting state into a flat list of ops
+// (sweeps, transfers, exchanges).  The builder applies the per-level fusion
+// policy and the communication-avoiding ghost rule (DESIGN.md
+// "Ghost-validity rule"): it tracks, per level, how many cells deep the ghost
+// bricks of x and b are valid, inserts an x-exchange only when a sweep would
+// read a stale ghost (or the CA period is reached), and sweeps ghost bricks
+// redundantly only when the next sweep will read them without an exchange.
+// Every schedule computes bit-identical values; only traffic changes.
+#pragma once
+
+#include <vector>
+
+#include "mg_internal.h"
+
+namespace mgb {
+
+enum OpKind { OP_SWEEP = 0, OP_RESTRICT, OP_INTERP, OP_ZERO, OP_EXCH, OP_BOTTOM_RES };
+
+struct Op {
+  int kind = OP_SWEEP;
+  int level = 0;
+  int src = 0, dst = 0;     // x buffers (ping-pong) at `level`
+  int cbuf = 0;             // coarse x buffer (interp)
+  unsigned flags = 0;       // SW_* (kernels.h)
+  bool paper = false;       // applyOp + smooth(+residual) kernels instead of the fused sweep
+  bool ghosts = false;      // also sweep the ghost bricks (redundant CA computation)
+  bool exch_before = false; // exchange x[src] ghosts before the sweep
+  int field = 0;            // OP_EXCH: 0 = x[src], 1 = b
+  int n = 0;                // OP_BOTTOM_RES: sweeps
+  bool zero = false;        // OP_BOTTOM_RES: x == 0 on entry
+  int timer = 0;            // MG_OP_*
+};
+
+struct LevelState {
+  int cur = 0;       // which x buffer holds x
+  int dx = 0;        // valid ghost depth of x (cells)
+  int db = 0;        // valid ghost depth of b (cells)
+  int since = 1 << 20;  // sweeps since the last x exchange
+};
+
+struct Builder {
+  const Layout& lay;
+  std::vector<Op> ops;
+  LevelState st[MG_MAX_LEVELS];
+  int fusion_override[MG_MAX_LEVELS];
+
+  explicit Builder(const Layout& l);
+  bool ghosts(int l) const { return lay.lv[l].n_ghost > 0; }
+  int fusion(int l) const;
+  int period(int l) const;
+  // `n` smooth(+residual) sweeps at level l.  last: 0 none, 1 write r, 2 fused restriction.
+  void phase(int l, int n, bool zero_first, int last, bool interp_first, int timer);
+  void restrict_op(int l);  // b_{l+1} = R r_l (+ b ghost exchange)
+  void zero_op(int l);
+  void interp_op(int l);
+  void bottom(int l, int n, bool zero);
+  void exchange_b(int l);
+  void vcycle();
+};
+
+int64_t op_launches(const Op& o, const Layout& lay, bool overlap);
+
+}  // namespace mgb

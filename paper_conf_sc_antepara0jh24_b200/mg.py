@@ -1,0 +1,354 @@
+"""Thin ctypes binding of include/mg.h (argument marshalling only).
+
+Every function here has the C name and forwards to libmg_b200.so; every step
+of the V-cycle runs in the library's sm_100a kernels.  There is no CPU
+fallback: if the library is missing or fails to load, ``lib()`` raises.
+PyTorch is used only for device memory (the workspace and field tensors),
+streams and (in the harness) process groups.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(PKG, "libmg_b200.so")
+
+MG_OK, MG_NOT_CONVERGED = 0, 1
+MG_MAX_LEVELS = 16
+MG_FUSION_AUTO, MG_FUSION_PAPER, MG_FUSION_SWEEP, MG_FUSION_FULL = 0, 1, 2, 3
+MG_GHOST_AUTO, MG_GHOST_ALL = 0, 1
+MG_TRANSPORT_AUTO, MG_TRANSPORT_NCCL, MG_TRANSPORT_LOCAL = 0, 1, 2
+MG_BOTTOM_AUTO, MG_BOTTOM_SWEEPS, MG_BOTTOM_RESIDENT = 0, 1, 2
+MG_FIELD_X, MG_FIELD_B, MG_FIELD_R = 0, 1, 2
+OP_NAMES = ["sweep", "applyOp", "smooth", "restriction", "interpolation", "initZero", "exchange", "bottom"]
+MG_NUM_OPS = len(OP_NAMES)
+
+
+class MGError(RuntimeError):
+    def __init__(self, status: int, where: str, msg: str):
+        super().__init__(f"{where} -> status {status}: {msg}")
+        self.status = status
+
+
+class mg_params(ctypes.Structure):
+    _fields_ = [
+        ("n_local", ctypes.c_int32 * 3),
+        ("proc_grid", ctypes.c_int32 * 3),
+        ("num_levels", ctypes.c_int32),
+        ("pre_smooths", ctypes.c_int32),
+        ("post_smooths", ctypes.c_int32),
+        ("bottom_smooths", ctypes.c_int32),
+        ("ca_period", ctypes.c_int32 * MG_MAX_LEVELS),
+        ("fusion", ctypes.c_int32 * MG_MAX_LEVELS),
+        ("ghost_mode", ctypes.c_int32),
+        ("transport", ctypes.c_int32),
+        ("use_graph", ctypes.c_int32),
+        ("bottom_mode", ctypes.c_int32),
+        ("overlap", ctypes.c_int32),
+        ("reserved", ctypes.c_int32 * 7),
+        ("h0", ctypes.c_double),
+    ]
+
+
+_lib = None
+
+_SIGS = {
+    "mg_params_default": (None, [ctypes.POINTER(mg_params)]),
+    "mg_workspace_bytes": (ctypes.c_int, [ctypes.POINTER(mg_params), ctypes.c_int32, ctypes.c_int32,
+                                          ctypes.POINTER(ctypes.c_size_t)]),
+    "mg_nccl_unique_id": (ctypes.c_int, [ctypes.c_char_p]),
+    "mg_setup": (ctypes.c_int, [ctypes.POINTER(mg_params), ctypes.c_int32, ctypes.c_int32, ctypes.c_char_p,
+                                ctypes.c_int32, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_size_t,
+                                ctypes.POINTER(ctypes.c_void_p)]),
+    "mg_set_rhs": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
+    "mg_set_rhs_host": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
+    "mg_set_solution": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
+    "mg_get_solution": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
+    "mg_get_solution_host": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
+    "mg_vcycle": (ctypes.c_int, [ctypes.c_void_p]),
+    "mg_residual_norm": (ctypes.c_int, [ctypes.c_void_p, ctypes.POINTER(ctypes.c_double)]),
+    "mg_solve": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_double, ctypes.c_int32, ctypes.POINTER(ctypes.c_int32),
+                                ctypes.POINTER(ctypes.c_double)]),
+    "mg_set_timing": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32]),
+    "mg_get_timings": (ctypes.c_int, [ctypes.c_void_p, ctypes.POINTER(ctypes.c_double), ctypes.c_int32]),
+    "mg_vcycle_launches": (ctypes.c_int, [ctypes.c_void_p, ctypes.POINTER(ctypes.c_int64)]),
+    "mg_exchange_stats": (ctypes.c_int, [ctypes.c_void_p, ctypes.POINTER(ctypes.c_int64),
+                                         ctypes.POINTER(ctypes.c_int64)]),
+    "mg_destroy": (ctypes.c_int, [ctypes.c_void_p]),
+    "mg_last_error": (ctypes.c_char_p, []),
+    "mg_level_set": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32, ctypes.c_void_p]),
+    "mg_level_get": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32, ctypes.c_void_p]),
+    "mg_op_smooth": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32, ctypes.c_int32,
+                                    ctypes.c_int32]),
+    "mg_op_restrict": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32]),
+    "mg_op_interp": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32]),
+    "mg_op_bottom": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32]),
+    "mg_sync": (ctypes.c_int, [ctypes.c_void_p]),
+    "mg_group_setup": (ctypes.c_int, [ctypes.POINTER(mg_params), ctypes.c_int32, ctypes.c_int32, ctypes.c_void_p,
+                                      ctypes.c_void_p, ctypes.c_size_t, ctypes.POINTER(ctypes.c_void_p)]),
+    "mg_group_ctx": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.POINTER(ctypes.c_void_p)]),
+    "mg_group_vcycle": (ctypes.c_int, [ctypes.c_void_p]),
+    "mg_group_residual_norm": (ctypes.c_int, [ctypes.c_void_p, ctypes.POINTER(ctypes.c_double)]),
+    "mg_group_set_rhs": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_void_p]),
+    "mg_group_commit_rhs": (ctypes.c_int, [ctypes.c_void_p]),
+    "mg_group_set_solution": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_void_p]),
+    "mg_group_destroy": (ctypes.c_int, [ctypes.c_void_p]),
+    "mg_layout_create": (ctypes.c_int, [ctypes.POINTER(mg_params), ctypes.c_int32, ctypes.c_int32,
+                                        ctypes.POINTER(ctypes.c_void_p)]),
+    "mg_layout_level_info": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.POINTER(ctypes.c_int64)]),
+    "mg_layout_adjacency": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_void_p]),
+    "mg_layout_coords": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_void_p]),
+    "mg_layout_parent": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_void_p]),
+    "mg_layout_plan": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32, ctypes.c_void_p]),
+    "mg_layout_destroy": (ctypes.c_int, [ctypes.c_void_p]),
+}
+
+
+def lib():
+    """Load libmg_b200.so (raises if it is missing: there is no fallback)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} not built: run __graft_entry__.build() (no CPU fallback exists)")
+        # torch first, so the NCCL torch bundles is the libnccl.so.2 in the process
+        try:
+            import torch  # noqa: F401
+        except Exception:
+            pass
+        L = ctypes.CDLL(LIB_PATH)
+        for name, (res, args) in _SIGS.items():
+            f = getattr(L, name)
+            f.restype = res
+            f.argtypes = args
+        _lib = L
+    return _lib
+
+
+def header_symbols():
+    return list(_SIGS)
+
+
+def check(status: int, where: str) -> int:
+    if status < 0:
+        raise MGError(status, where, lib().mg_last_error().decode())
+    return status
+
+
+def params(n_local, proc_grid=(1, 1, 1), num_levels=6, pre=12, post=12, bottom=100, ca_period=None, fusion=None,
+           ghost_mode=MG_GHOST_AUTO, transport=MG_TRANSPORT_AUTO, use_graph=1, bottom_mode=MG_BOTTOM_AUTO,
+           overlap=1, h0=0.0) -> mg_params:
+    p = mg_params()
+    lib().mg_params_default(ctypes.byref(p))
+    p.n_local[:] = [int(v) for v in n_local]
+    p.proc_grid[:] = [int(v) for v in proc_grid]
+    p.num_levels = int(num_levels)
+    p.pre_smooths, p.post_smooths, p.bottom_smooths = int(pre), int(post), int(bottom)
+    for l in range(MG_MAX_LEVELS):
+        p.ca_period[l] = 0 if ca_period is None else int(ca_period[l] if isinstance(ca_period, (list, tuple))
+                                                          else ca_period)
+        p.fusion[l] = 0 if fusion is None else int(fusion[l] if isinstance(fusion, (list, tuple)) else fusion)
+    p.ghost_mode, p.transport, p.use_graph = int(ghost_mode), int(transport), int(use_graph)
+    p.bottom_mode, p.overlap, p.h0 = int(bottom_mode), int(overlap), float(h0)
+    return p
+
+
+# ----------------------------------------------------------------- C names
+def mg_workspace_bytes(p: mg_params, rank: int = 0, world_size: int = 1) -> int:
+    out = ctypes.c_size_t()
+    check(lib().mg_workspace_bytes(ctypes.byref(p), rank, world_size, ctypes.byref(out)), "mg_workspace_bytes")
+    return out.value
+
+
+def mg_nccl_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    check(lib().mg_nccl_unique_id(buf), "mg_nccl_unique_id")
+    return buf.raw
+
+
+def mg_setup(p, rank, world_size, nccl_id, device, stream, workspace_ptr, ws_bytes):
+    ctx = ctypes.c_void_p()
+    check(lib().mg_setup(ctypes.byref(p), rank, world_size, nccl_id, device, stream, workspace_ptr, ws_bytes,
+                         ctypes.byref(ctx)), "mg_setup")
+    return ctx
+
+
+def mg_set_rhs(ctx, b_ptr):
+    return check(lib().mg_set_rhs(ctx, b_ptr), "mg_set_rhs")
+
+
+def mg_set_rhs_host(ctx, b_host_ptr):
+    return check(lib().mg_set_rhs_host(ctx, b_host_ptr), "mg_set_rhs_host")
+
+
+def mg_set_solution(ctx, x_ptr):
+    return check(lib().mg_set_solution(ctx, x_ptr), "mg_set_solution")
+
+
+def mg_get_solution(ctx, x_ptr):
+    return check(lib().mg_get_solution(ctx, x_ptr), "mg_get_solution")
+
+
+def mg_get_solution_host(ctx, x_host_ptr):
+    return check(lib().mg_get_solution_host(ctx, x_host_ptr), "mg_get_solution_host")
+
+
+def mg_vcycle(ctx):
+    return check(lib().mg_vcycle(ctx), "mg_vcycle")
+
+
+def mg_residual_norm(ctx) -> float:
+    out = ctypes.c_double()
+    check(lib().mg_residual_norm(ctx, ctypes.byref(out)), "mg_residual_norm")
+    return out.value
+
+
+def mg_solve(ctx, tol=1e-10, max_cycles=20):
+    cyc, fin = ctypes.c_int32(), ctypes.c_double()
+    st = check(lib().mg_solve(ctx, tol, max_cycles, ctypes.byref(cyc), ctypes.byref(fin)), "mg_solve")
+    return st, cyc.value, fin.value
+
+
+def mg_set_timing(ctx, enabled: bool):
+    return check(lib().mg_set_timing(ctx, 1 if enabled else 0), "mg_set_timing")
+
+
+def mg_get_timings(ctx, num_levels: int):
+    n = num_levels * MG_NUM_OPS
+    buf = (ctypes.c_double * n)()
+    check(lib().mg_get_timings(ctx, buf, n), "mg_get_timings")
+    return [[buf[l * MG_NUM_OPS + o] for o in range(MG_NUM_OPS)] for l in range(num_levels)]
+
+
+def mg_vcycle_launches(ctx) -> int:
+    out = ctypes.c_int64()
+    check(lib().mg_vcycle_launches(ctx, ctypes.byref(out)), "mg_vcycle_launches")
+    return out.value
+
+
+def mg_exchange_stats(ctx):
+    b, m = ctypes.c_int64(), ctypes.c_int64()
+    check(lib().mg_exchange_stats(ctx, ctypes.byref(b), ctypes.byref(m)), "mg_exchange_stats")
+    return b.value, m.value
+
+
+def mg_destroy(ctx):
+    return check(lib().mg_destroy(ctx), "mg_destroy")
+
+
+def mg_level_set(ctx, level, field, ptr):
+    return check(lib().mg_level_set(ctx, level, field, ptr), "mg_level_set")
+
+
+def mg_level_get(ctx, level, field, ptr):
+    return check(lib().mg_level_get(ctx, level, field, ptr), "mg_level_get")
+
+
+def mg_op_smooth(ctx, level, n, write_r, fusion=MG_FUSION_SWEEP):
+    return check(lib().mg_op_smooth(ctx, level, n, 1 if write_r else 0, fusion), "mg_op_smooth")
+
+
+def mg_op_restrict(ctx, level):
+    return check(lib().mg_op_restrict(ctx, level), "mg_op_restrict")
+
+
+def mg_op_interp(ctx, level):
+    return check(lib().mg_op_interp(ctx, level), "mg_op_interp")
+
+
+def mg_op_bottom(ctx, level, n):
+    return check(lib().mg_op_bottom(ctx, level, n), "mg_op_bottom")
+
+
+def mg_sync(ctx):
+    return check(lib().mg_sync(ctx), "mg_sync")
+
+
+def mg_group_setup(p, world_size, device, stream, workspace_ptr, ws_bytes):
+    g = ctypes.c_void_p()
+    check(lib().mg_group_setup(ctypes.byref(p), world_size, device, stream, workspace_ptr, ws_bytes,
+                               ctypes.byref(g)), "mg_group_setup")
+    return g
+
+
+def mg_group_ctx(g, rank):
+    c = ctypes.c_void_p()
+    check(lib().mg_group_ctx(g, rank, ctypes.byref(c)), "mg_group_ctx")
+    return c
+
+
+def mg_group_vcycle(g):
+    return check(lib().mg_group_vcycle(g), "mg_group_vcycle")
+
+
+def mg_group_residual_norm(g) -> float:
+    out = ctypes.c_double()
+    check(lib().mg_group_residual_norm(g, ctypes.byref(out)), "mg_group_residual_norm")
+    return out.value
+
+
+def mg_group_set_rhs(g, rank, ptr):
+    return check(lib().mg_group_set_rhs(g, rank, ptr), "mg_group_set_rhs")
+
+
+def mg_group_commit_rhs(g):
+    return check(lib().mg_group_commit_rhs(g), "mg_group_commit_rhs")
+
+
+def mg_group_set_solution(g, rank, ptr):
+    return check(lib().mg_group_set_solution(g, rank, ptr), "mg_group_set_solution")
+
+
+def mg_group_destroy(g):
+    return check(lib().mg_group_destroy(g), "mg_group_destroy")
+
+
+# ------------------------------------------------------- layout (host only)
+class Layout:
+    """Host-side brick layout tables of one rank (no GPU needed)."""
+
+    def __init__(self, p: mg_params, rank: int = 0, world_size: int = 1):
+        import numpy as np
+
+        self._np = np
+        self.p = p
+        self.h = ctypes.c_void_p()
+        check(lib().mg_layout_create(ctypes.byref(p), rank, world_size, ctypes.byref(self.h)), "mg_layout_create")
+
+    def __del__(self):
+        if getattr(self, "h", None):
+            lib().mg_layout_destroy(self.h)
+            self.h = None
+
+    def info(self, level):
+        buf = (ctypes.c_int64 * 16)()
+        check(lib().mg_layout_level_info(self.h, level, buf), "mg_layout_level_info")
+        v = list(buf)
+        return {"n": v[0:3], "nb": v[3:6], "ghost": v[6:9], "owned": v[9], "interior": v[10], "nghost": v[11],
+                "alloc": v[12], "send_runs": v[13], "recv_runs": v[14], "zero_brick": v[15]}
+
+    def adjacency(self, level):
+        inf = self.info(level)
+        a = self._np.zeros((inf["owned"] + inf["nghost"], 8), dtype=self._np.int32)
+        check(lib().mg_layout_adjacency(self.h, level, a.ctypes.data), "mg_layout_adjacency")
+        return a
+
+    def coords(self, level):
+        inf = self.info(level)
+        a = self._np.zeros((inf["owned"] + inf["nghost"], 3), dtype=self._np.int32)
+        check(lib().mg_layout_coords(self.h, level, a.ctypes.data), "mg_layout_coords")
+        return a
+
+    def parent(self, level):
+        inf = self.info(level)
+        a = self._np.zeros(inf["owned"] + inf["nghost"], dtype=self._np.int32)
+        check(lib().mg_layout_parent(self.h, level, a.ctypes.data), "mg_layout_parent")
+        return a
+
+    def plan(self, level, which):
+        inf = self.info(level)
+        n = inf["recv_runs"] if which else inf["send_runs"]
+        a = self._np.zeros((n, 6), dtype=self._np.int64)
+        if n:
+            check(lib().mg_layout_plan(self.h, level, which, a.ctypes.data), "mg_layout_plan")
+        return a

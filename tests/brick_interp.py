@@ -1,0 +1,147 @@
+"""Host brick interpreter (TEST INFRASTRUCTURE; neither the oracle nor the product).
+
+Runs the V-cycle in numpy directly on the library's brick layout tables
+(adjacency, coords, parent map, exchange plans obtained through the C ABI's
+host-only ``mg_layout_*`` queries), so the layout and the packing-free
+exchange plans can be checked against the lexicographic oracle on a machine
+without a GPU.  numpy float64 ufuncs are separately rounded IEEE ops, written
+in the canonical order of DESIGN.md reading A8, so the comparison is bitwise.
+
+Schedule: exchange x before EVERY sweep (no communication avoiding), b after
+every restriction -- the simplest legal schedule; the CA schedules are
+exercised on the GPU.
+"""
+from __future__ import annotations
+
+import numpy as np
+
+
+class RankLevel:
+    def __init__(self, lay, level):
+        self.info = lay.info(level)
+        self.adj = lay.adjacency(level)
+        self.coords = lay.coords(level)
+        self.parent = lay.parent(level)
+        self.sends = lay.plan(level, 0)
+        self.recvs = lay.plan(level, 1)
+        self.n_owned = self.info["owned"]
+        self.n_alloc = self.info["alloc"]
+        self.n = self.info["n"]  # x, y, z
+
+    def zeros(self):
+        return np.zeros((self.n_alloc, 8, 8, 8))  # [brick][k][j][i]
+
+    def to_bricks(self, lex):  # lex (nz, ny, nx)
+        out = self.zeros()
+        c = self.coords[: self.n_owned]
+        for q in range(self.n_owned):
+            cx, cy, cz = c[q]
+            out[q] = lex[8 * cz:8 * cz + 8, 8 * cy:8 * cy + 8, 8 * cx:8 * cx + 8]
+        return out
+
+    def from_bricks(self, br):
+        nx, ny, nz = self.n
+        lex = np.empty((nz, ny, nx))
+        c = self.coords[: self.n_owned]
+        for q in range(self.n_owned):
+            cx, cy, cz = c[q]
+            lex[8 * cz:8 * cz + 8, 8 * cy:8 * cy + 8, 8 * cx:8 * cx + 8] = br[q]
+        return lex
+
+
+def padded(x, adj, nb):
+    """(nb, 10, 10, 10) = each brick plus its 6 face halos via the adjacency table."""
+    X = np.zeros((nb, 10, 10, 10))
+    X[:, 1:9, 1:9, 1:9] = x[:nb]
+    X[:, 1:9, 1:9, 0] = x[adj[:nb, 0]][:, :, :, 7]  # W: neighbour's i = 7
+    X[:, 1:9, 1:9, 9] = x[adj[:nb, 1]][:, :, :, 0]  # E
+    X[:, 1:9, 0, 1:9] = x[adj[:nb, 2]][:, :, 7, :]  # S
+    X[:, 1:9, 9, 1:9] = x[adj[:nb, 3]][:, :, 0, :]  # N
+    X[:, 0, 1:9, 1:9] = x[adj[:nb, 4]][:, 7, :, :]  # B
+    X[:, 9, 1:9, 1:9] = x[adj[:nb, 5]][:, 0, :, :]  # T
+    return X
+
+
+def coeffs(h):
+    inv = 1.0 / (h * h)
+    return -6.0 * inv, inv, (h * h) / 12.0
+
+
+def sweep(x, b, adj, nb, h):
+    """Returns (x', r) on bricks [0, nb): a = alpha x + beta sum6; r = b - a; x' = x + gamma (a - b)."""
+    al, be, ga = coeffs(h)
+    X = padded(x, adj, nb)
+    c = X[:, 1:9, 1:9, 1:9]
+    s = ((X[:, 1:9, 1:9, 0:8] + X[:, 1:9, 1:9, 2:10]) + (X[:, 1:9, 0:8, 1:9] + X[:, 1:9, 2:10, 1:9])) + \
+        (X[:, 0:8, 1:9, 1:9] + X[:, 2:10, 1:9, 1:9])
+    a = al * c + be * s
+    xn = x.copy()
+    r = np.zeros_like(x)
+    r[:nb] = b[:nb] - a
+    xn[:nb] = c + ga * (a - b[:nb])
+    return xn, r
+
+
+def restrict(rf, fine: RankLevel, bc):
+    for q in range(fine.n_owned):
+        pr = int(fine.parent[q])
+        cb, o = pr >> 3, pr & 7
+        ox, oy, oz = o & 1, (o >> 1) & 1, o >> 2
+        f = rf[q]
+        v = 0.125 * (((f[0::2, 0::2, 0::2] + f[0::2, 0::2, 1::2]) + (f[0::2, 1::2, 0::2] + f[0::2, 1::2, 1::2]))
+                     + ((f[1::2, 0::2, 0::2] + f[1::2, 0::2, 1::2]) + (f[1::2, 1::2, 0::2] + f[1::2, 1::2, 1::2])))
+        bc[cb, 4 * oz:4 * oz + 4, 4 * oy:4 * oy + 4, 4 * ox:4 * ox + 4] = v
+
+
+def interp(xf, fine: RankLevel, xc):
+    for q in range(fine.n_owned):
+        pr = int(fine.parent[q])
+        cb, o = pr >> 3, pr & 7
+        ox, oy, oz = o & 1, (o >> 1) & 1, o >> 2
+        blk = xc[cb, 4 * oz:4 * oz + 4, 4 * oy:4 * oy + 4, 4 * ox:4 * ox + 4]
+        xf[q] = xf[q] + np.repeat(np.repeat(np.repeat(blk, 2, 0), 2, 1), 2, 2)
+
+
+def exchange_local(fields, levels):
+    """In-process exchange of ghost bricks for all ranks (fields[r] is that rank's array)."""
+    out = [f.copy() for f in fields]
+    for r, L in enumerate(levels):
+        for peer, d, run, local, remote, count in L.recvs:
+            out[r][local:local + count] = fields[peer][remote:remote + count]
+    return out
+
+
+def vcycle_ranks(xs, bs, ranks, L, h0, pre, post, bottom, exchange=exchange_local):
+    """One V-cycle (Alg 2) over every rank's brick fields.  ranks[r][l] = RankLevel.
+    xs, bs: per-rank lists of per-level arrays (level-0 b must already hold valid ghosts).
+    `exchange(fields, levels)` fills ghost bricks (in-process or over torch.distributed)."""
+    R = len(ranks)
+    own = lambda r, l: ranks[r][l].n_owned  # noqa: E731
+    rs = [[None] * L for _ in range(R)]
+    for l in range(L - 1):
+        h = h0 * 2**l
+        for s in range(pre):
+            xs_l = exchange([xs[r][l] for r in range(R)], [ranks[r][l] for r in range(R)])
+            for r in range(R):
+                xs[r][l], rs[r][l] = sweep(xs_l[r], bs[r][l], ranks[r][l].adj, own(r, l), h)
+        for r in range(R):
+            bs[r][l + 1] = ranks[r][l + 1].zeros()
+            restrict(rs[r][l], ranks[r][l], bs[r][l + 1])
+            xs[r][l + 1] = ranks[r][l + 1].zeros()
+        bl = exchange([bs[r][l + 1] for r in range(R)], [ranks[r][l + 1] for r in range(R)])
+        for r in range(R):
+            bs[r][l + 1] = bl[r]
+    h = h0 * 2 ** (L - 1)
+    for s in range(bottom):
+        xl = exchange([xs[r][L - 1] for r in range(R)], [ranks[r][L - 1] for r in range(R)])
+        for r in range(R):
+            xs[r][L - 1], _ = sweep(xl[r], bs[r][L - 1], ranks[r][L - 1].adj, own(r, L - 1), h)
+    for l in range(L - 2, -1, -1):
+        h = h0 * 2**l
+        for r in range(R):
+            interp(xs[r][l], ranks[r][l], xs[r][l + 1])
+        for s in range(post):
+            xl = exchange([xs[r][l] for r in range(R)], [ranks[r][l] for r in range(R)])
+            for r in range(R):
+                xs[r][l], _ = sweep(xl[r], bs[r][l], ranks[r][l].adj, own(r, l), h)
+    return xs

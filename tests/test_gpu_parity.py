@@ -1,0 +1,297 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Tolerances (north_star): 1e-12 relative per operator application, 1e-10
+relative on the residual norm after each V-cycle.  The design target is
+BITWISE equality (same expression DAG, no FMA), so most
+assertions are exact; the stated tolerances are asserted too.
+"""
+import numpy as np
+import pytest
+
+import mg_inputs
+
+torch = pytest.importorskip("torch")
+pytestmark = [pytest.mark.gpu,
+              pytest.mark.skipif(not torch.cuda.is_available(), reason="needs a CUDA device")]
+
+
+def _mg():
+    from paper_conf_sc_antepara0jh24_b200 import mg, solver
+
+    return mg, solver
+
+
+def dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+def host(t):
+    torch.cuda.synchronize()
+    return t.cpu().numpy()
+
+
+def assert_bitwise(got, want, rel=1e-12, what=""):
+    scale = max(np.abs(want).max(), 1e-300)
+    err = np.abs(got - want).max()
+    assert err <= rel * scale, f"{what}: max err {err:.3e} (rel {err / scale:.3e})"
+    assert np.array_equal(got, want), f"{what}: not bitwise (max err {err:.3e})"
+
+
+def new(shape_zyx, L, **kw):
+    mg, solver = _mg()
+    nz, ny, nx = shape_zyx
+    return solver.Multigrid((nx, ny, nz), num_levels=L, **kw)
+
+
+# ------------------------------------------------------------------ per-op
+@pytest.mark.parametrize("fusion", [2, 1])
+@pytest.mark.parametrize("shape", [(32, 16, 48), (64, 64, 64)])
+def test_smooth_residual_per_op(oracle_mod, fusion, shape):
+    """applyOp + smooth+residual, fused sweep and paper kernel set."""
+    mg, _ = _mg()
+    m = new(shape, 1, pre=1, post=1, bottom=1)
+    h = mg_inputs.default_h0(shape)
+    x = mg_inputs.random_field(shape, 1)
+    b = mg_inputs.random_field(shape, 2)
+    m.level_set(0, mg.MG_FIELD_X, dev(x))
+    m.level_set(0, mg.MG_FIELD_B, dev(b))
+    mg.mg_op_smooth(m.ctx, 0, 3, 1, fusion)
+    xo, ro = x, None
+    for _ in range(3):
+        xo, ro = oracle_mod.smooth_residual(xo, oracle_mod.apply_op(xo, h), b, h)
+    assert_bitwise(host(m.level_get(0, mg.MG_FIELD_X)), xo, what="x")
+    assert_bitwise(host(m.level_get(0, mg.MG_FIELD_R)), ro, what="r")
+    m.close()
+
+
+def test_apply_op_via_residual(oracle_mod):
+    """applyOp alone: with b = 0 the residual is r = -Ax exactly."""
+    mg, _ = _mg()
+    shape = (16, 24, 40)
+    m = new(shape, 1)
+    h = mg_inputs.default_h0(shape)
+    x = mg_inputs.random_field(shape, 3)
+    m.level_set(0, mg.MG_FIELD_X, dev(x))
+    m.level_set(0, mg.MG_FIELD_B, dev(np.zeros(shape)))
+    mg.mg_op_smooth(m.ctx, 0, 1, 1, 2)
+    assert_bitwise(-host(m.level_get(0, mg.MG_FIELD_R)), oracle_mod.apply_op(x, h), what="Ax")
+    m.close()
+
+
+def test_restriction_and_interpolation_per_op(oracle_mod):
+    mg, _ = _mg()
+    shape = (32, 48, 64)
+    m = new(shape, 3, pre=1)
+    r = mg_inputs.random_field(shape, 4)
+    m.level_set(0, mg.MG_FIELD_R, dev(r))
+    mg.mg_op_restrict(m.ctx, 0)
+    assert_bitwise(host(m.level_get(1, mg.MG_FIELD_B)), oracle_mod.restriction(r), what="restriction")
+    xf = mg_inputs.random_field(shape, 5)
+    xc = mg_inputs.random_field(tuple(s // 2 for s in shape), 6)
+    m.level_set(0, mg.MG_FIELD_X, dev(xf))
+    m.level_set(1, mg.MG_FIELD_X, dev(xc))
+    mg.mg_op_interp(m.ctx, 0)
+    assert_bitwise(host(m.level_get(0, mg.MG_FIELD_X)), oracle_mod.interpolation_increment(xc, xf), what="interp")
+    m.close()
+
+
+@pytest.mark.parametrize("bottom_mode", [1, 2])
+@pytest.mark.parametrize("shape", [(8, 8, 8), (16, 16, 16), (8, 16, 32)])
+def test_bottom_solver(oracle_mod, bottom_mode, shape):
+    """100 point-Jacobi sweeps: resident one-CTA kernel and per-sweep launches."""
+    mg, _ = _mg()
+    m = new(shape, 1, bottom_mode=bottom_mode)
+    h = mg_inputs.default_h0(shape)
+    x = mg_inputs.random_field(shape, 7)
+    b = mg_inputs.random_field(shape, 8)
+    m.level_set(0, mg.MG_FIELD_X, dev(x))
+    m.level_set(0, mg.MG_FIELD_B, dev(b))
+    mg.mg_op_bottom(m.ctx, 0, 100)
+    xo = x
+    for _ in range(100):
+        xo = oracle_mod.smooth(xo, oracle_mod.apply_op(xo, h), b, h)
+    assert_bitwise(host(m.level_get(0, mg.MG_FIELD_X)), xo, what="bottom")
+    m.close()
+
+
+def test_residual_norm(oracle_mod):
+    mg, _ = _mg()
+    shape = (32, 64, 16)
+    m = new(shape, 2)
+    h = mg_inputs.default_h0(shape)
+    x = mg_inputs.random_field(shape, 9)
+    b = mg_inputs.random_field(shape, 10)
+    m.set_rhs(dev(b))
+    m.set_solution(dev(x))
+    assert m.residual_norm() == oracle_mod.max_norm_residual(x, b, h)
+    m.close()
+
+
+# ------------------------------------------------------------------ V-cycle
+def oracle_cycles(oracle_mod, b, L, ncyc, pre=12, post=12, bottom=100):
+    orc = oracle_mod.OracleMG(b.shape, L, pre, post, bottom)
+    orc.set_b(b)
+    orc.set_x(None)
+    xs, ns = [], []
+    for _ in range(ncyc):
+        orc.vcycle()
+        xs.append(orc.get_x())
+        ns.append(orc.norm())
+    return xs, ns
+
+
+def check_cycles(m, xs, ns, get=None):
+    for c in range(len(xs)):
+        m.vcycle()
+        nr = m.residual_norm()
+        assert abs(nr - ns[c]) <= 1e-10 * ns[c], (c, nr, ns[c])
+        got = host(m.get_solution()) if get is None else get()
+        assert_bitwise(got, xs[c], what=f"x after cycle {c + 1}")
+        assert nr == ns[c]
+
+
+@pytest.mark.parametrize("rhs", ["random", "sin"])
+def test_vcycle_config1_bitwise(oracle_mod, rhs):
+    """Config 1: 64^3, L = 4 (64 -> 8), 12/12/100; x and the residual norm after each of 3 cycles."""
+    shape = (64, 64, 64)
+    b = mg_inputs.random_rhs(shape, 0) if rhs == "random" else mg_inputs.sin_rhs(shape)
+    xs, ns = oracle_cycles(oracle_mod, b, 4, 3)
+    m = new(shape, 4)
+    m.set_rhs(dev(b))
+    m.set_solution(None)
+    check_cycles(m, xs, ns)
+    m.close()
+
+
+@pytest.mark.parametrize("fusion", [1, 2, 3])
+@pytest.mark.parametrize("use_graph", [True, False])
+def test_vcycle_fusion_variants_bitwise(oracle_mod, fusion, use_graph):
+    """Every fusion variant (paper kernel set / fused sweep / full fusion) and graph
+    replay give the oracle's bits.  Non-cubic, ragged brick counts."""
+    shape = (32, 48, 80)
+    b = mg_inputs.random_rhs(shape, 3)
+    xs, ns = oracle_cycles(oracle_mod, b, 2, 2, 4, 3, 30)
+    m = new(shape, 2, pre=4, post=3, bottom=30, fusion=fusion, use_graph=use_graph)
+    m.set_rhs(dev(b))
+    m.set_solution(None)
+    check_cycles(m, xs, ns)
+    m.close()
+
+
+@pytest.mark.parametrize("transport", [2, 1])
+@pytest.mark.parametrize("period", [1, 2, 4, 8])
+def test_self_exchange_ca_periods_bitwise(oracle_mod, transport, period):
+    """Ghost shell on every axis with self-exchange (communication avoiding on one
+    GPU): local copies and NCCL send/recv; any CA period gives the same bits."""
+    shape = (64, 64, 64)
+    b = mg_inputs.random_rhs(shape, 4)
+    xs, ns = oracle_cycles(oracle_mod, b, 3, 2, 12, 12, 100)
+    m = new(shape, 3, ghost_mode=1, transport=transport, ca_period=period)
+    m.set_rhs(dev(b))
+    m.set_solution(None)
+    check_cycles(m, xs, ns)
+    m.close()
+
+
+@pytest.mark.parametrize("pg,n_local,L", [((2, 1, 1), (32, 32, 32), 3), ((2, 2, 2), (32, 32, 32), 3),
+                                          ((1, 2, 3), (16, 32, 16), 2), ((2, 2, 1), (16, 16, 16), 2)])
+@pytest.mark.parametrize("overlap", [True, False])
+def test_loopback_decomposition_bitwise(oracle_mod, pg, n_local, L, overlap):
+    """A 3D decomposition run on one GPU (ranks exchange ghost bricks through the
+    same plans the NCCL path uses) reproduces the undecomposed oracle bit for bit."""
+    _, solver = _mg()
+    gshape = (n_local[2] * pg[2], n_local[1] * pg[1], n_local[0] * pg[0])
+    b = mg_inputs.random_rhs(gshape, 5)
+    xs, ns = oracle_cycles(oracle_mod, b, L, 2)
+    g = solver.LoopbackGroup(n_local, pg, num_levels=L, overlap=overlap)
+    g.set_rhs([dev(mg_inputs.local_block(b, r, pg)) for r in range(g.world_size)])
+    g.set_solution(None)
+    for c in range(2):
+        g.vcycle()
+        nr = g.residual_norm()
+        assert nr == ns[c]
+        for r in range(g.world_size):
+            assert_bitwise(host(g.get_solution(r)), mg_inputs.local_block(xs[c], r, pg), what=f"rank {r}")
+    g.close()
+
+
+def test_solve_matches_oracle(oracle_mod):
+    """Alg 1 to max-norm 1e-10: same cycle count and final norm."""
+    shape = (64, 64, 64)
+    b = mg_inputs.sin_rhs(shape)
+    orc = oracle_mod.OracleMG(shape, 4)
+    orc.set_b(b)
+    orc.set_x(None)
+    c_o, norms = orc.solve(1e-10, 20)
+    m = new(shape, 4)
+    m.set_rhs(dev(b))
+    m.set_solution(None)
+    st, c_g, fin = m.solve(1e-10, 20)
+    assert st == 0 and c_g == c_o and fin == norms[-1] and fin < 1e-10
+    m.close()
+
+
+def test_edge_cases_single_level_and_minimal_sweeps(oracle_mod):
+    """L = 1 (bottom only), pre = 1, post = 0, bottom = 0."""
+    for shape, L, pre, post, bottom in [((16, 8, 24), 1, 1, 1, 7), ((32, 32, 32), 3, 1, 0, 0),
+                                        ((32, 32, 32), 2, 1, 1, 1)]:
+        b = mg_inputs.random_rhs(shape, 6)
+        xs, ns = oracle_cycles(oracle_mod, b, L, 2, pre, post, bottom)
+        m = new(shape, L, pre=pre, post=post, bottom=bottom)
+        m.set_rhs(dev(b))
+        m.set_solution(None)
+        check_cycles(m, xs, ns)
+        m.close()
+
+
+def test_host_api_e2e(oracle_mod):
+    """mg_set_rhs_host / mg_get_solution_host (the e2e path bench.py times)."""
+    shape = (32, 32, 32)
+    b = mg_inputs.random_rhs(shape, 8)
+    xs, ns = oracle_cycles(oracle_mod, b, 3, 1)
+    m = new(shape, 3)
+    bh = torch.from_numpy(b).pin_memory()
+    m.set_rhs_host(bh)
+    m.set_solution(None)
+    m.vcycle()
+    out = torch.empty(shape, dtype=torch.float64).pin_memory()
+    m.get_solution_host(out)
+    assert np.array_equal(out.numpy(), xs[0])
+    assert m.residual_norm() == ns[0]
+    m.close()
+
+
+# ------------------------------------------------------------- full sizes
+def test_full_size_512_sweep_sampled(oracle_mod):
+    """512^3 (the bench workload), level-0 fused sweep: 20k sampled points vs the
+    oracle's point evaluation, plus r."""
+    mg, _ = _mg()
+    shape = (512, 512, 512)
+    m = new(shape, 6)
+    h = mg_inputs.default_h0(shape)
+    x = mg_inputs.random_field(shape, 12)
+    b = mg_inputs.sin_rhs(shape)
+    m.level_set(0, mg.MG_FIELD_X, dev(x))
+    m.level_set(0, mg.MG_FIELD_B, dev(b))
+    mg.mg_op_smooth(m.ctx, 0, 1, 1, 2)
+    rng = np.random.default_rng(0)
+    pts = rng.integers(0, x.size, 20000)
+    pts = np.concatenate([pts, [0, x.size - 1, 511, 512 * 512 - 1]])  # corners (periodic wrap)
+    xn, r = oracle_mod.sweep_points(x, b, h, pts)
+    gx = host(m.level_get(0, mg.MG_FIELD_X)).ravel()[pts]
+    gr = host(m.level_get(0, mg.MG_FIELD_R)).ravel()[pts]
+    assert np.array_equal(gx, xn) and np.array_equal(gr, r)
+    m.close()
+
+
+@pytest.mark.slow
+def test_full_size_512_vcycle_bitwise(oracle_mod):
+    """512^3, L = 6, 12/12/100 (bench configuration): one full V-cycle bitwise + norm."""
+    shape = (512, 512, 512)
+    b = mg_inputs.sin_rhs(shape)
+    xs, ns = oracle_cycles(oracle_mod, b, 6, 1)
+    m = new(shape, 6)
+    m.set_rhs(dev(b))
+    m.set_solution(None)
+    check_cycles(m, xs, ns)
+    m.close()

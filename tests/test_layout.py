@@ -1,0 +1,180 @@
+"""CPU tests of the brick layout, adjacency, region ordering and exchange plans
+(host-only C-ABI queries; no GPU), plus a bitwise V-cycle of the host brick
+interpreter on those tables against the lexicographic oracle."""
+import itertools
+
+import numpy as np
+import pytest
+
+import mg_inputs
+from paper_conf_sc_antepara0jh24_b200 import mg
+from tests import brick_interp as bi
+
+FACE = [(-1, 0, 0), (1, 0, 0), (0, -1, 0), (0, 1, 0), (0, 0, -1), (0, 0, 1)]
+
+
+def layouts(n_local, proc_grid, L, ghost_mode=0):
+    p = mg.params(n_local, proc_grid, num_levels=L, ghost_mode=ghost_mode)
+    world = proc_grid[0] * proc_grid[1] * proc_grid[2]
+    return p, [mg.Layout(p, r, world) for r in range(world)]
+
+
+CASES = [((32, 32, 32), (1, 1, 1), 3, 0), ((32, 32, 32), (1, 1, 1), 3, 1), ((32, 16, 16), (2, 1, 1), 2, 0),
+         ((16, 16, 16), (2, 2, 2), 2, 0), ((16, 16, 32), (1, 2, 3), 2, 0), ((48, 32, 16), (3, 1, 2), 2, 0)]
+
+
+@pytest.mark.parametrize("n_local,pg,L,gm", CASES)
+def test_adjacency_consistent_with_coords(n_local, pg, L, gm):
+    """adj[b][face] is the brick at coords(b) + face (periodic wrap on non-ghost axes;
+    the zero brick past the ghost shell), and adjacency is symmetric."""
+    _, lays = layouts(n_local, pg, L, gm)
+    for lay in lays:
+        for l in range(L):
+            inf = lay.info(l)
+            adj, co = lay.adjacency(l), lay.coords(l)
+            stored = inf["owned"] + inf["nghost"]
+            index = {tuple(c): q for q, c in enumerate(co)}
+            assert len(index) == stored  # no duplicates
+            assert np.all(adj[:, 6] == np.arange(stored))
+            for q in range(stored):
+                for f, d in enumerate(FACE):
+                    e = [int(co[q][a]) + d[a] for a in range(3)]
+                    for a in range(3):
+                        if not inf["ghost"][a]:
+                            e[a] %= inf["nb"][a]
+                    want = index.get(tuple(e), inf["zero_brick"])
+                    assert adj[q, f] == want
+                    if q < inf["owned"]:  # owned bricks: every neighbour exists, symmetric
+                        assert want != inf["zero_brick"]
+                        back = adj[want, f ^ 1]
+                        assert back == q
+
+
+@pytest.mark.parametrize("n_local,pg,L,gm", CASES)
+def test_region_order_interior_first_and_ghost_coverage(n_local, pg, L, gm):
+    """Owned bricks: interior region first; ghosts: every ghost brick received
+    exactly once from one contiguous run (packing-free)."""
+    _, lays = layouts(n_local, pg, L, gm)
+    for lay in lays:
+        for l in range(L):
+            inf = lay.info(l)
+            co = lay.coords(l)
+            nb, g = inf["nb"], inf["ghost"]
+            own = co[: inf["owned"]]
+            on_surface = np.zeros(inf["owned"], dtype=bool)
+            for a in range(3):
+                if g[a]:
+                    on_surface |= (own[:, a] == 0) | (own[:, a] == nb[a] - 1)
+            assert inf["interior"] == int((~on_surface).sum())
+            assert not on_surface[: inf["interior"]].any() and on_surface[inf["interior"]:].all()
+            recv = lay.plan(l, 1)
+            hit = np.zeros(inf["nghost"], dtype=int)
+            for peer, d, run, local, remote, count in recv:
+                hit[local - inf["owned"]: local - inf["owned"] + count] += 1
+                assert 0 <= remote and remote + count <= inf["owned"]
+            assert np.all(hit == 1)
+
+
+def test_42_messages_for_26_neighbours():
+    """With the searched region order, a 3D decomposition needs 42 contiguous
+    runs for the 26 neighbours (BrickLib-style message consolidation)."""
+    _, lays = layouts((64, 64, 64), (2, 2, 2), 1)
+    inf = lays[0].info(0)
+    assert inf["send_runs"] == 42 and inf["recv_runs"] == 42
+    assert inf["nghost"] == 10**3 - 8**3
+
+
+def test_ghost_counts_match_survey():
+    """512^3 per GPU ghost-shell bricks 8192 / 16640 / 25352 at 2 / 4 / 8 GPUs."""
+    for pg, want in (((2, 1, 1), 8192), ((2, 2, 1), 16640), ((2, 2, 2), 25352)):
+        p = mg.params((512, 512, 512), pg, num_levels=1)
+        assert mg.Layout(p, 0, pg[0] * pg[1] * pg[2]).info(0)["nghost"] == want
+
+
+@pytest.mark.parametrize("n_local,pg,L,gm", CASES)
+def test_plans_match_pairwise_in_order(n_local, pg, L, gm):
+    """NCCL matches sends and recvs of a rank pair in posting order: rank S's
+    sends to R must equal R's recvs from S, run for run, in the same order."""
+    _, lays = layouts(n_local, pg, L, gm)
+    world = len(lays)
+    for l in range(L):
+        sends = [lay.plan(l, 0) for lay in lays]
+        recvs = [lay.plan(l, 1) for lay in lays]
+        for S in range(world):
+            for R in range(world):
+                s = sends[S][sends[S][:, 0] == R] if len(sends[S]) else np.zeros((0, 6))
+                r = recvs[R][recvs[R][:, 0] == S] if len(recvs[R]) else np.zeros((0, 6))
+                assert len(s) == len(r)
+                for a, b in zip(s, r):
+                    assert a[1] == b[1] and a[2] == b[2] and a[5] == b[5]  # dir, run, count
+                    assert a[3] == b[4] and a[4] == b[3]  # sender local == receiver remote, and back
+
+
+@pytest.mark.parametrize("n_local,pg,L,gm", CASES)
+def test_parent_map(n_local, pg, L, gm):
+    """Fine brick e -> coarse brick floor(e/2), octant e mod 2 (brick-by-brick
+    inter-level operators)."""
+    _, lays = layouts(n_local, pg, L, gm)
+    lay = lays[-1]
+    for l in range(L - 1):
+        co, cco = lay.coords(l), lay.coords(l + 1)
+        par = lay.parent(l)
+        inf = lay.info(l)
+        for q in range(inf["owned"]):
+            pr = int(par[q])
+            assert pr >= 0
+            cb, o = pr >> 3, pr & 7
+            e = co[q]
+            assert tuple(cco[cb]) == tuple(int(v) // 2 for v in e)
+            assert o == (e[0] % 2) + 2 * (e[1] % 2) + 4 * (e[2] % 2)
+
+
+def global_to_ranks(glob, pg, L, lays):
+    R = len(lays)
+    ranks = [[bi.RankLevel(lays[r], l) for l in range(L)] for r in range(R)]
+    return ranks
+
+
+@pytest.mark.parametrize("n_local,pg,L,gm", CASES)
+def test_brick_interpreter_vcycle_bitwise_vs_oracle(oracle_mod, n_local, pg, L, gm):
+    """The layout tables + exchange plans reproduce the oracle's V-cycle bit for
+    bit (12/12/100 scaled down to 3/3/20 for CPU time)."""
+    p, lays = layouts(n_local, pg, L, gm)
+    gshape = (n_local[2] * pg[2], n_local[1] * pg[1], n_local[0] * pg[0])
+    b = mg_inputs.random_rhs(gshape, 7)
+    pre, post, bottom = 3, 3, 20
+    h0 = mg_inputs.default_h0(gshape)
+    orc = oracle_mod.OracleMG(gshape, L, pre, post, bottom, h0)
+    orc.set_b(b)
+    orc.set_x(None)
+    orc.vcycle()
+    want = orc.get_x()
+    R = len(lays)
+    ranks = [[bi.RankLevel(lays[r], l) for l in range(L)] for r in range(R)]
+    xs = [[ranks[r][l].zeros() for l in range(L)] for r in range(R)]
+    bs = [[None] * L for _ in range(R)]
+    for r in range(R):
+        bs[r][0] = ranks[r][0].to_bricks(mg_inputs.local_block(b, r, pg))
+    b0 = bi.exchange_local([bs[r][0] for r in range(R)], [ranks[r][0] for r in range(R)])
+    for r in range(R):
+        bs[r][0] = b0[r]
+    xs = bi.vcycle_ranks(xs, bs, ranks, L, h0, pre, post, bottom)
+    got = np.zeros(gshape)
+    px, py, pz = pg
+    for r in range(R):
+        cx, cy, cz = mg_inputs.rank_coords(r, pg)
+        nx, ny, nz = n_local
+        got[cz * nz:(cz + 1) * nz, cy * ny:(cy + 1) * ny, cx * nx:(cx + 1) * nx] = ranks[r][0].from_bricks(xs[r][0])
+    assert np.array_equal(got, want)
+
+
+def test_invalid_params_rejected():
+    bad = [mg.params((30, 32, 32), num_levels=1),  # not a multiple of 8
+           mg.params((32, 32, 32), num_levels=4),  # 32 not a multiple of 8*2^3
+           mg.params((32, 32, 32), (2, 1, 1), num_levels=1)]  # proc grid != world 1
+    for p in bad:
+        with pytest.raises(mg.MGError):
+            mg.Layout(p, 0, 1)
+    p = mg.params((32, 32, 32), num_levels=2, ca_period=9)
+    with pytest.raises(mg.MGError):
+        mg.Layout(p, 0, 1)
