@@ -67,6 +67,7 @@ struct mg_ctx {
   int device = 0;
   cudaStream_t stream = nullptr;
   cudaStream_t comm = nullptr;
+  cudaStream_t cap = nullptr;  // private stream the V-cycle graph is captured on (the caller's may be legacy)
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
   std::vector<DevLevel> dl;
   double* stage = nullptr;
@@ -92,6 +93,7 @@ struct mg_ctx {
 struct mg_group {
   std::vector<mg_ctx*> r;
   cudaStream_t stream = nullptr;
+  cudaStream_t cap = nullptr;
   cudaGraphExec_t gexec[2] = {nullptr, nullptr};
   Plan gplan[2];
   bool gvalid[2] = {false, false};
@@ -380,10 +382,12 @@ mg_status vcycle_impl(mg_ctx* c, mg_group* g) {
     b.vcycle();
     Plan p = make_plan(b, c0->lay);
     if (graph) {
-      CKC(c0, cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
-      mg_status rs = run_plan(c0, g, p, s);
+      // capture on a private non-blocking stream; the graph is then launched on the caller's stream
+      cudaStream_t cs = g ? g->cap : c->cap;
+      CKC(c0, cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal));
+      mg_status rs = run_plan(c0, g, p, cs);
       cudaGraph_t gr = nullptr;
-      cudaError_t ce = cudaStreamEndCapture(s, &gr);
+      cudaError_t ce = cudaStreamEndCapture(cs, &gr);
       if (rs != MG_OK) return rs;
       CKC(c0, ce);
       CKC(c0, cudaGraphInstantiate(&gexec[key], gr, 0));
@@ -443,6 +447,7 @@ mg_status init_ctx(mg_ctx* c, const mg_params& p, int rank, int world, int devic
   }
   CKC(c, cudaStreamSynchronize(stream));  // host vectors above are temporaries
   CKC(c, cudaStreamCreateWithFlags(&c->comm, cudaStreamNonBlocking));
+  CKC(c, cudaStreamCreateWithFlags(&c->cap, cudaStreamNonBlocking));
   CKC(c, cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
   CKC(c, cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming));
   CKC(c, cudaMallocHost((void**)&c->h_pinned, 64));
@@ -458,6 +463,7 @@ void free_ctx(mg_ctx* c) {
     if (c->gexec[k]) cudaGraphExecDestroy(c->gexec[k]);
   if (c->nccl) ncclCommDestroy(c->nccl);
   if (c->comm) cudaStreamDestroy(c->comm);
+  if (c->cap) cudaStreamDestroy(c->cap);
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
   if (c->ev_join) cudaEventDestroy(c->ev_join);
   for (cudaEvent_t e : c->evpool) cudaEventDestroy(e);
@@ -817,6 +823,10 @@ mg_status mg_group_setup(const mg_params* p, int32_t world_size, int32_t device,
     return set_err(MG_ERR_OOM, "group workspace too small: need " + std::to_string(per * (size_t)world_size));
   mg_group* g = new mg_group();
   g->stream = (cudaStream_t)cuda_stream;
+  if (cudaStreamCreateWithFlags(&g->cap, cudaStreamNonBlocking) != cudaSuccess) {
+    delete g;
+    return set_err(MG_ERR_CUDA, "cudaStreamCreate failed");
+  }
   for (int r = 0; r < world_size; ++r) {
     mg_ctx* c = new mg_ctx();
     mg_status s = init_ctx(c, q, r, world_size, device, g->stream, (char*)workspace + per * (size_t)r, per, false);
@@ -896,6 +906,7 @@ mg_status mg_group_destroy(mg_group* g) {
   for (int k = 0; k < 2; ++k)
     if (g->gexec[k]) cudaGraphExecDestroy(g->gexec[k]);
   for (mg_ctx* c : g->r) free_ctx(c);
+  if (g->cap) cudaStreamDestroy(g->cap);
   delete g;
   return MG_OK;
 }

@@ -81,7 +81,7 @@ def test_apply_op_via_residual(oracle_mod):
 def test_restriction_and_interpolation_per_op(oracle_mod):
     mg, _ = _mg()
     shape = (32, 48, 64)
-    m = new(shape, 3, pre=1)
+    m = new(shape, 2, pre=1)
     r = mg_inputs.random_field(shape, 4)
     m.level_set(0, mg.MG_FIELD_R, dev(r))
     mg.mg_op_restrict(m.ctx, 0)

@@ -1,0 +1,47 @@
+"""Mutation check for the oracle pins (run by hand: python tools/oracle_mutations.py).
+
+Applies one plausible slip at a time to oracle/mg_oracle.c, rebuilds, runs
+tests/test_oracle_pins.py and reports whether some pin catches it.  The
+source is restored afterwards.  Last run: every mutation below CAUGHT.
+"""
+import os
+import subprocess
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+SRC = os.path.join(ROOT, "oracle", "mg_oracle.c")
+
+MUTATIONS = {
+    "gamma_sign_smooth_residual": ("    x[p] = x[p] + gamma * (Ax[p] - b[p]);\n  }", "    x[p] = x[p] - gamma * (Ax[p] - b[p]);\n  }"),
+    "restriction_index": ("r010 = r[IDX(i, j + 1, k, nx, ny)]", "r010 = r[IDX(i + 1, j, k, nx, ny)]"),
+    "interp_parent_axes": ("xc[IDX(i / 2, j / 2, k / 2, cx, cy)]", "xc[IDX(i / 2, k / 2 % cy, j / 2 % (nz/2), cx, cy)]"),
+    "missing_initZero": ("    oracle_init_zero(lvl_n(m, l + 1), m->x[l + 1]);", ""),
+    "h_not_doubled_per_level": ("m->h[l] = h0 * (double)s;", "m->h[l] = h0;"),
+    "dropped_neighbour": ("(xb + xt)", "(xb + xb)"),
+    "residual_sign": ("r[p] = b[p] - Ax[p];", "r[p] = Ax[p] - b[p];"),
+    "bottom_without_smooth": ("      oracle_smooth(lvl_n(m, l), m->h[l], m->x[l], m->Ax[l], m->b[l]);", ""),
+}
+
+
+def main():
+    orig = open(SRC).read()
+    ok = True
+    try:
+        for name, (a, b) in MUTATIONS.items():
+            assert a in orig, name
+            open(SRC, "w").write(orig.replace(a, b, 1))
+            r = subprocess.run([sys.executable, "-m", "pytest", "tests/test_oracle_pins.py", "-q", "-x",
+                                "-p", "no:cacheprovider"], capture_output=True, text=True, cwd=ROOT)
+            caught = r.returncode != 0
+            ok &= caught
+            print(f"{name:32s} {'CAUGHT' if caught else 'MISSED'}")
+    finally:
+        open(SRC, "w").write(orig)
+        sys.path.insert(0, ROOT)
+        import oracle
+        oracle.build(force=True)
+    return 0 if ok else 1
+
+
+if __name__ == "__main__":
+    sys.exit(main())
