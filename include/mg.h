@@ -103,7 +103,9 @@ typedef struct {
   int32_t use_graph;             /* 1 = replay the V-cycle as one CUDA graph (default 1) */
   int32_t bottom_mode;           /* MG_BOTTOM_* (resident = one CTA runs all bottom sweeps in smem) */
   int32_t overlap;               /* 1 = sweep interior bricks while the exchange is in flight */
-  int32_t reserved[7];
+  int32_t sweep_kernel;          /* 0 = auto (streaming column kernel on levels >= 16384 bricks),
+                                    1 = one-brick-per-CTA kernel only, 2 = streaming kernel on every level */
+  int32_t reserved[6];
   double h0;                     /* finest spacing; <= 0 => 1 / max_d(global N_d) (reading A7) */
 } mg_params;
 

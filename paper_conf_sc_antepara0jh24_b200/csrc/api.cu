@@ -44,6 +44,11 @@ struct DevLevel {
   int32_t* coord = nullptr;
   Coeffs c{};
   double h = 0;
+  struct Col {
+    int64_t b0, b1;
+    ColArgs args;
+  };
+  std::vector<Col> cols;  // streaming-sweep plans (column segments) per brick range
 };
 
 struct Plan {
@@ -80,6 +85,7 @@ struct mg_ctx {
   LevelState st[MG_MAX_LEVELS];
   bool poisoned = false;
   bool timing = false;
+  bool use_col = true;  // streaming column kernel where a plan exists (sweep_kernel == 1 disables)
   std::vector<double> tm;
   std::vector<TimerRec> trec;
   std::vector<cudaEvent_t> evpool;
@@ -146,6 +152,16 @@ size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double**
     d.adj = (int32_t*)take((size_t)L.n_stored * 8 * sizeof(int32_t));
     d.parent = (int32_t*)take((size_t)L.n_alloc * sizeof(int32_t));
     d.coord = (int32_t*)take((size_t)L.n_stored * 3 * sizeof(int32_t));
+    for (const auto& ct : L.cols) {
+      DevLevel::Col col;
+      col.b0 = ct.b0;
+      col.b1 = ct.b1;
+      col.args.bricks = (const int32_t*)take(ct.bricks.size() * sizeof(int32_t));
+      col.args.side = (const int4*)take(ct.side.size() * sizeof(int32_t));
+      col.args.segs = (const int2*)take(ct.segs.size() * sizeof(int32_t));
+      col.args.nseg = (int64_t)ct.segs.size() / 2;
+      d.cols.push_back(col);
+    }
     d.h = lay.p.h0 * (double)(1 << l);
     d.c = level_coeffs(d.h);
     if (out) (*out)[l] = d;
@@ -236,6 +252,14 @@ mg_status sweep_range(mg_ctx* c, const Op& o, int64_t b0, int64_t b1, cudaStream
   a.brick0 = b0;
   a.nbricks = b1 - b0;
   a.c = d.c;
+  if (c->use_col && col_supports(o.flags)) {
+    for (const auto& col : d.cols) {
+      if (col.b0 == b0 && col.b1 == b1) {
+        CKC(c, launch_sweep_col(a, col.args, o.flags, s));
+        return MG_OK;
+      }
+    }
+  }
   CKC(c, launch_sweep(a, o.flags, s));
   return MG_OK;
 }
@@ -428,6 +452,7 @@ mg_status init_ctx(mg_ctx* c, const mg_params& p, int rank, int world, int devic
   if (s != MG_OK) return set_err(s, msg);
   c->device = device;
   c->stream = stream;
+  c->use_col = p.sweep_kernel != 1;
   const size_t need = carve(c->lay, nullptr, nullptr, nullptr, nullptr);
   if (!workspace || ws_bytes < need)
     return set_err(MG_ERR_OOM, "workspace too small: need " + std::to_string(need) + " bytes");
@@ -444,6 +469,13 @@ mg_status init_ctx(mg_ctx* c, const mg_params& p, int rank, int world, int devic
     CKC(c, cudaMemcpyAsync(d.parent, par.data(), par.size() * sizeof(int32_t), cudaMemcpyHostToDevice, stream));
     CKC(c, cudaMemcpyAsync(d.coord, L.coord.data(), L.coord.size() * sizeof(int32_t), cudaMemcpyHostToDevice,
                            stream));
+    for (size_t k = 0; k < L.cols.size(); ++k) {
+      const auto& ct = L.cols[k];
+      const ColArgs& ca = d.cols[k].args;
+      CKC(c, cudaMemcpyAsync((void*)ca.bricks, ct.bricks.data(), ct.bricks.size() * 4, cudaMemcpyHostToDevice, stream));
+      CKC(c, cudaMemcpyAsync((void*)ca.side, ct.side.data(), ct.side.size() * 4, cudaMemcpyHostToDevice, stream));
+      CKC(c, cudaMemcpyAsync((void*)ca.segs, ct.segs.data(), ct.segs.size() * 4, cudaMemcpyHostToDevice, stream));
+    }
   }
   CKC(c, cudaStreamSynchronize(stream));  // host vectors above are temporaries
   CKC(c, cudaStreamCreateWithFlags(&c->comm, cudaStreamNonBlocking));

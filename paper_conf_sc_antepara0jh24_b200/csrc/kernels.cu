@@ -230,6 +230,223 @@ cudaError_t launch_sweep(const SweepArgs& a, unsigned flags, cudaStream_t s) {
   }
 }
 
+// ---------------------------------------------------------------------------
+// Streaming column sweep (the level-0 hot kernel).
+//
+// One CTA of 4 warps streams a segment of <= 16 consecutive bricks of one
+// z-column (7 CTAs per SM).  Warp w owns planes 2w, 2w+1 of every brick; lane l
+// owns the cell pair (2(l&3), l>>2) of a plane and walks its planes in k,
+// keeping planes k-1, k, k+1 of x in registers.
+// In-plane neighbours: i+-1 by warp shuffles, j+-1 by 128-bit shared loads of
+// the neighbouring rows.  The x and b bricks arrive by TMA bulk copies
+// (cp.async.bulk, 4 KiB each, lane 0) into a 3-stage shared-memory ring
+// completed on mbarriers, two bricks ahead; the 256 W/E/S/N face-halo values of
+// a brick (neighbour columns, through L2) arrive by 8-byte cp.async into the
+// same stage, tracked by the same mbarrier (cp.async.mbarrier.arrive.noinc).
+// The k-halo is the previous brick's plane 7 (a 512-byte carry buffer) and the
+// next brick's plane 0 (ring); one 512-byte plane below / above the segment.  Stores of x'
+// (and r) are coalesced 128-bit streaming stores.  DRAM traffic per point:
+// read x, b; write x' (+ r): the algorithmic 24 (32) bytes.
+// ---------------------------------------------------------------------------
+constexpr int COL_NST = 3;  // ring stages: current, next (plane 0 = k-halo), one in flight
+constexpr int COL_MAXSEG = 16;
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_fence_init() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n .reg .pred p;\n"
+      "MBW_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n @!p bra MBW_%=;\n}" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   smem_u32(dst)),
+               "l"(src), "r"(bytes), "r"(smem_u32(bar))
+               : "memory");
+}
+__device__ __forceinline__ void cp_async8(void* dst, const void* src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_arrive_noinc(uint64_t* bar) {
+  asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+
+struct ColStage {
+  double x[512];
+  double b[512];
+  double face[4][64];  // W (i=7 of the W brick, [k][j]), E (i=0, [k][j]), S (j=7, [k][i]), N (j=0, [k][i])
+};
+
+template <bool RESTRICT>
+struct ColSmem {
+  ColStage st[COL_NST];
+  double edge[2][64];   // plane 7 of the brick below the segment, plane 0 of the brick above
+  double carry[2][64];  // plane 7 of the previous brick (k-halo of plane 0), double-buffered
+  double rs[RESTRICT ? 2 : 1][RESTRICT ? 512 : 2];  // residual of the current brick (fused restriction)
+  uint64_t bar[COL_NST + 1];
+  int sid[COL_MAXSEG];
+  int spar[COL_MAXSEG];
+  int4 sside[COL_MAXSEG];
+};
+
+constexpr int COL_WARPS = 4;  // warp w streams planes 2w, 2w+1 of every brick
+
+template <unsigned FLAGS>
+__global__ void __launch_bounds__(COL_WARPS * 32, 7) sweep_col_kernel(SweepArgs p, ColArgs ca) {
+  constexpr bool WRITE_R = (FLAGS & SW_WRITE_R) != 0;
+  constexpr bool RESTRICT = (FLAGS & SW_RESTRICT) != 0;
+  constexpr int NT = COL_WARPS * 32;
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  ColSmem<RESTRICT>& S = *reinterpret_cast<ColSmem<RESTRICT>*>(smem_raw);
+  const int t = threadIdx.x, w = t >> 5, l = t & 31;
+  const int i0 = 2 * (l & 3), j = l >> 2;
+  const int q = 8 * j + i0;  // this lane's pair inside a plane
+  const int2 sg = ca.segs[blockIdx.x];
+  const int cnt = sg.y;
+  if (t < cnt) {
+    const int id = ca.bricks[sg.x + t];
+    S.sid[t] = id;
+    S.sside[t] = ca.side[sg.x + t];
+    if (RESTRICT) S.spar[t] = p.parent[id];
+  }
+  if (t == 0) {
+    // a ring stage completes after thread 0's expect_tx arrive + NT cp.async arrivals (+ the TMA bytes)
+    for (int s = 0; s < COL_NST; ++s) mbar_init(&S.bar[s], NT + 1);
+    mbar_init(&S.bar[COL_NST], 1);
+    mbar_fence_init();
+  }
+  __syncthreads();
+  // stage brick n: x and b by TMA (thread 0); 256 face values by 8-byte cp.async
+  auto issue = [&](int n) {
+    const int s = n % COL_NST;
+    if (t == 0) {
+      const int64_t id = S.sid[n];
+      mbar_expect_tx(&S.bar[s], 8192);
+      tma_load_1d(S.st[s].x, p.x + id * 512, 4096, &S.bar[s]);
+      tma_load_1d(S.st[s].b, p.b + id * 512, 4096, &S.bar[s]);
+    }
+    const int4 sd = S.sside[n];
+#pragma unroll
+    for (int u = 0; u < 256 / NT; ++u) {
+      const int e = t + NT * u;  // 0..255
+      const int f = e >> 6, m = e & 63;
+      const int nb = f == 0 ? sd.x : f == 1 ? sd.y : f == 2 ? sd.z : sd.w;
+      const int off = f == 0 ? 7 + 8 * (m & 7) + 64 * (m >> 3)
+                    : f == 1 ? 8 * (m & 7) + 64 * (m >> 3)
+                    : f == 2 ? (m & 7) + 56 + 64 * (m >> 3)
+                             : (m & 7) + 64 * (m >> 3);
+      cp_async8(&S.st[s].face[f][m], p.x + (int64_t)nb * 512 + off);
+    }
+    cp_async_arrive_noinc(&S.bar[s]);
+  };
+  if (t == 0) {
+    const int64_t below = __ldg(p.adj + (int64_t)S.sid[0] * 8 + 4);
+    const int64_t above = __ldg(p.adj + (int64_t)S.sid[cnt - 1] * 8 + 5);
+    mbar_expect_tx(&S.bar[COL_NST], 1024);
+    tma_load_1d(S.edge[0], p.x + below * 512 + 448, 512, &S.bar[COL_NST]);
+    tma_load_1d(S.edge[1], p.x + above * 512, 512, &S.bar[COL_NST]);
+  }
+  issue(0);
+  if (cnt > 1) issue(1);
+  if (w == 0 || w == COL_WARPS - 1) mbar_wait(&S.bar[COL_NST], 0);
+
+  for (int n = 0; n < cnt; ++n) {
+    if (n + 2 < cnt) {
+      fence_proxy_async();  // the generic-proxy reads of the stage being refilled are complete
+      issue(n + 2);         // (its last readers finished before the barrier that ended step n-1)
+    }
+    const int s = n % COL_NST;
+    mbar_wait(&S.bar[s], (uint32_t)((n / COL_NST) & 1));
+    const ColStage& G = S.st[s];
+    const double* X = G.x;
+    const int k0 = 2 * w;
+    double2 xm, xc, xp;
+    if (w > 0)
+      xm = *reinterpret_cast<const double2*>(X + 64 * (k0 - 1) + q);
+    else
+      xm = *reinterpret_cast<const double2*>((n > 0 ? S.carry[(n - 1) & 1] : S.edge[0]) + q);
+    xc = *reinterpret_cast<const double2*>(X + 64 * k0 + q);
+    const int64_t gbase = (int64_t)S.sid[n] * 512 + q;
+#pragma unroll
+    for (int kk = 0; kk < 2; ++kk) {
+      const int k = k0 + kk;
+      if (k < 7) {
+        xp = *reinterpret_cast<const double2*>(X + 64 * (k + 1) + q);
+      } else if (n + 1 < cnt) {
+        const int s1 = (n + 1) % COL_NST;
+        mbar_wait(&S.bar[s1], (uint32_t)(((n + 1) / COL_NST) & 1));
+        xp = *reinterpret_cast<const double2*>(S.st[s1].x + q);
+      } else {
+        xp = *reinterpret_cast<const double2*>(S.edge[1] + q);
+      }
+      const double2 bb = *reinterpret_cast<const double2*>(G.b + 64 * k + q);
+      const double2 rs_ = *reinterpret_cast<const double2*>(X + 64 * k + (j > 0 ? q - 8 : q));
+      const double2 rn_ = *reinterpret_cast<const double2*>(X + 64 * k + (j < 7 ? q + 8 : q));
+      const double fw = G.face[0][j + 8 * k];
+      const double fe = G.face[1][j + 8 * k];
+      const double2 fs = *reinterpret_cast<const double2*>(&G.face[2][i0 + 8 * k]);
+      const double2 fn = *reinterpret_cast<const double2*>(&G.face[3][i0 + 8 * k]);
+      const double wl = __shfl_up_sync(0xffffffffu, xc.y, 1);
+      const double er = __shfl_down_sync(0xffffffffu, xc.x, 1);
+      const double wv = i0 > 0 ? wl : fw;
+      const double ev = i0 < 6 ? er : fe;
+      const double2 sv = j > 0 ? rs_ : fs;
+      const double2 nv = j < 7 ? rn_ : fn;
+      const double a0 = stencil_a(xc.x, wv, xc.y, sv.x, nv.x, xm.x, xp.x, p.c.alpha, p.c.beta);
+      const double a1 = stencil_a(xc.y, xc.x, ev, sv.y, nv.y, xm.y, xp.y, p.c.alpha, p.c.beta);
+      double2 xn, rv;
+      xn.x = DADD(xc.x, DMUL(p.c.gamma, DSUB(a0, bb.x)));
+      xn.y = DADD(xc.y, DMUL(p.c.gamma, DSUB(a1, bb.y)));
+      rv.x = DSUB(bb.x, a0);
+      rv.y = DSUB(bb.y, a1);
+      st_stream2(p.xo + gbase + 64 * k, xn);
+      if (WRITE_R) st_stream2(p.r + gbase + 64 * k, rv);
+      if (RESTRICT) *reinterpret_cast<double2*>(S.rs[n & 1] + 64 * k + q) = rv;
+      if (k == 7) *reinterpret_cast<double2*>(S.carry[n & 1] + q) = xc;  // k-halo of the next brick
+      xm = xc;
+      xc = xp;
+    }
+    __syncthreads();  // stage n-1 free for refill; carry / rs of brick n complete
+    if (RESTRICT && t < 64) {
+      const double* R = S.rs[n & 1];
+      const int I = t & 3, J = (t >> 2) & 3, K = t >> 4;
+      const int f = 2 * I + 16 * J + 128 * K;
+      const double v = DMUL(0.125, DADD(DADD(DADD(R[f], R[f + 1]), DADD(R[f + 8], R[f + 9])),
+                                        DADD(DADD(R[f + 64], R[f + 65]), DADD(R[f + 72], R[f + 73]))));
+      const int pr = S.spar[n];
+      const int oct = pr & 7;
+      const int ox = oct & 1, oy = (oct >> 1) & 1, oz = oct >> 2;
+      p.bc[(int64_t)(pr >> 3) * 512 + (4 * ox + I) + 8 * (4 * oy + J) + 64 * (4 * oz + K)] = v;
+    }
+  }
+}
+
+bool col_supports(unsigned flags) {
+  const unsigned f = flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP | SW_ZERO_X);
+  return f == 0 || f == SW_WRITE_R || f == SW_RESTRICT;
+}
+
+cudaError_t launch_sweep_col(const SweepArgs& a, const ColArgs& c, unsigned flags, cudaStream_t s) {
+  if (c.nseg <= 0) return cudaSuccess;
+  const size_t sm = sizeof(ColSmem<false>), smr = sizeof(ColSmem<true>);
+  switch (flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP | SW_ZERO_X)) {
+    case 0: sweep_col_kernel<0><<<(unsigned)c.nseg, COL_WARPS * 32, sm, s>>>(a, c); break;
+    case SW_WRITE_R: sweep_col_kernel<SW_WRITE_R><<<(unsigned)c.nseg, COL_WARPS * 32, sm, s>>>(a, c); break;
+    case SW_RESTRICT: sweep_col_kernel<SW_RESTRICT><<<(unsigned)c.nseg, COL_WARPS * 32, smr, s>>>(a, c); break;
+    default: return cudaErrorInvalidValue;
+  }
+  return cudaGetLastError();
+}
+
 cudaError_t launch_apply_op(const double* x, double* Ax, const int32_t* adj, int64_t brick0, int64_t nbricks,
                             Coeffs c, cudaStream_t s) {
   if (nbricks <= 0) return cudaSuccess;
@@ -458,6 +675,16 @@ cudaError_t kernels_init() {
   if (e != cudaSuccess) return e;
   e = cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev);
   if (e != cudaSuccess) return e;
+  const int colsm = (int)sizeof(ColSmem<false>), colsmr = (int)sizeof(ColSmem<true>);
+  const void* colk[3] = {(const void*)sweep_col_kernel<0>, (const void*)sweep_col_kernel<SW_WRITE_R>,
+                         (const void*)sweep_col_kernel<SW_RESTRICT>};
+  for (int k = 0; k < 3; ++k) {
+    e = cudaFuncSetAttribute(colk[k], cudaFuncAttributeMaxDynamicSharedMemorySize, k == 2 ? colsmr : colsm);
+    if (e != cudaSuccess) return e;
+    // the streaming kernel is shared-memory-resident: ask for the full 228 KB carveout
+    e = cudaFuncSetAttribute(colk[k], cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+    if (e != cudaSuccess) return e;
+  }
   return cudaFuncSetAttribute(bottom_resident_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                               kResidentMaxBricks * 512 * 3 * (int)sizeof(double));
 }

@@ -36,6 +36,18 @@ struct SweepArgs {
 };
 
 cudaError_t launch_sweep(const SweepArgs& a, unsigned flags, cudaStream_t s);
+
+// Streaming (column) sweep: one CTA per segment of a z-column of bricks;
+// bricks of x and b arrive by TMA bulk copies into a shared-memory ring.
+struct ColArgs {
+  const int32_t* bricks;  // brick ids, segment after segment
+  const int4* side;       // W,E,S,N neighbour ids per entry of `bricks`
+  const int2* segs;       // (offset, count) per segment, count <= 16
+  int64_t nseg;
+};
+// true if the streaming kernel implements `flags` (plain, +r, +restriction)
+bool col_supports(unsigned flags);
+cudaError_t launch_sweep_col(const SweepArgs& a, const ColArgs& c, unsigned flags, cudaStream_t s);
 // applyOp (paper kernel set): Ax = alpha x + beta sum6
 cudaError_t launch_apply_op(const double* x, double* Ax, const int32_t* adj, int64_t brick0, int64_t nbricks,
                             Coeffs c, cudaStream_t s);

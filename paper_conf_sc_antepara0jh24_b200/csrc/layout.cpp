@@ -261,8 +261,71 @@ mg_status build_layout(const mg_params& p, int rank, int world, Layout& out, std
   out.L = p.num_levels;
   out.lv.assign(out.L, LevelLayout());
   for (int l = 0; l < out.L; ++l) build_level(out, l, out.lv[l]);
+  const int64_t min_b = p.sweep_kernel == 1 ? INT64_MAX : p.sweep_kernel == 2 ? 0 : kColMinBricks;
+  for (int l = 0; l < out.L; ++l) build_col_tables(out.lv[l], min_b);
   for (int l = 0; l + 1 < out.L; ++l) build_parents(out.lv[l], out.lv[l + 1]);
   return MG_OK;
+}
+
+}  // namespace mgb
+
+namespace mgb {
+
+// Column plans for the streaming sweep (kernels.cu sweep_col_kernel): every
+// brick of [b0,b1) exactly once, as z-chains following the adjacency T link
+// (periodic columns are cycles; ghost-shell columns end at the zero brick),
+// each chain cut into near-equal segments of <= kColSeg bricks.
+static LevelLayout::ColTable col_table(const LevelLayout& L, int64_t b0, int64_t b1) {
+  LevelLayout::ColTable t;
+  t.b0 = b0;
+  t.b1 = b1;
+  std::vector<char> vis((size_t)(b1 - b0), 0);
+  auto in = [&](int64_t q) { return q >= b0 && q < b1; };
+  for (int64_t q = b0; q < b1; ++q) {
+    if (vis[(size_t)(q - b0)]) continue;
+    int64_t s = q;
+    for (;;) {
+      const int64_t pb = L.adj[(size_t)s * 8 + 4];
+      if (!in(pb) || vis[(size_t)(pb - b0)] || pb == q) break;
+      s = pb;
+    }
+    std::vector<int32_t> chain;
+    for (int64_t c = s; in(c) && !vis[(size_t)(c - b0)]; c = L.adj[(size_t)c * 8 + 5]) {
+      vis[(size_t)(c - b0)] = 1;
+      chain.push_back((int32_t)c);
+    }
+    const int64_t len = (int64_t)chain.size();
+    const int64_t nseg = (len + kColSeg - 1) / kColSeg;
+    int64_t off = 0;
+    for (int64_t g = 0; g < nseg; ++g) {
+      const int64_t cnt = len / nseg + (g < len % nseg ? 1 : 0);
+      t.segs.push_back((int32_t)t.bricks.size());
+      t.segs.push_back((int32_t)cnt);
+      for (int64_t m = 0; m < cnt; ++m) {
+        const int32_t id = chain[(size_t)(off + m)];
+        t.bricks.push_back(id);
+        for (int f = 0; f < 4; ++f) t.side.push_back(L.adj[(size_t)id * 8 + f]);
+      }
+      off += cnt;
+    }
+  }
+  return t;
+}
+
+void build_col_tables(LevelLayout& L, int64_t min_bricks) {
+  L.cols.clear();
+  if (L.n_stored < min_bricks) return;
+  const int64_t ranges[5][2] = {{0, L.n_owned},
+                                {0, L.n_stored},
+                                {0, L.n_interior},
+                                {L.n_interior, L.n_owned},
+                                {L.n_interior, L.n_stored}};
+  for (auto& r : ranges) {
+    if (r[1] <= r[0]) continue;
+    bool dup = false;
+    for (auto& c : L.cols) dup |= (c.b0 == r[0] && c.b1 == r[1]);
+    if (!dup) L.cols.push_back(col_table(L, r[0], r[1]));
+  }
 }
 
 }  // namespace mgb

@@ -47,7 +47,21 @@ struct LevelLayout {
   std::vector<Run> sends, recvs;
   int64_t ext_index(int x, int y, int z) const;  // -1 if not stored
   std::vector<int32_t> ext2idx;  // dense map over the extended box
+  // Column plans for the streaming sweep kernel: the bricks of a range [b0,b1)
+  // arranged as z-columns (chains along the adjacency T link) cut into
+  // segments of <= kColSeg bricks; one CTA streams one segment.
+  struct ColTable {
+    int64_t b0 = 0, b1 = 0;
+    std::vector<int32_t> bricks;  // brick ids, segment after segment
+    std::vector<int32_t> side;    // [bricks][4] W,E,S,N neighbour ids
+    std::vector<int32_t> segs;    // [nseg][2] offset into bricks, count
+  };
+  std::vector<ColTable> cols;     // one per distinct range the schedule sweeps
 };
+
+constexpr int kColSeg = 16;             // bricks per streamed segment
+constexpr int64_t kColMinBricks = 16384;  // levels smaller than this use the one-brick-per-CTA kernel
+void build_col_tables(LevelLayout& L, int64_t min_bricks);
 
 struct Layout {
   mg_params p{};

@@ -46,7 +46,8 @@ class mg_params(ctypes.Structure):
         ("use_graph", ctypes.c_int32),
         ("bottom_mode", ctypes.c_int32),
         ("overlap", ctypes.c_int32),
-        ("reserved", ctypes.c_int32 * 7),
+        ("sweep_kernel", ctypes.c_int32),
+        ("reserved", ctypes.c_int32 * 6),
         ("h0", ctypes.c_double),
     ]
 
@@ -137,7 +138,7 @@ def check(status: int, where: str) -> int:
 
 def params(n_local, proc_grid=(1, 1, 1), num_levels=6, pre=12, post=12, bottom=100, ca_period=None, fusion=None,
            ghost_mode=MG_GHOST_AUTO, transport=MG_TRANSPORT_AUTO, use_graph=1, bottom_mode=MG_BOTTOM_AUTO,
-           overlap=1, h0=0.0) -> mg_params:
+           overlap=1, h0=0.0, sweep_kernel=0) -> mg_params:
     p = mg_params()
     lib().mg_params_default(ctypes.byref(p))
     p.n_local[:] = [int(v) for v in n_local]
@@ -150,6 +151,7 @@ def params(n_local, proc_grid=(1, 1, 1), num_levels=6, pre=12, post=12, bottom=1
         p.fusion[l] = 0 if fusion is None else int(fusion[l] if isinstance(fusion, (list, tuple)) else fusion)
     p.ghost_mode, p.transport, p.use_graph = int(ghost_mode), int(transport), int(use_graph)
     p.bottom_mode, p.overlap, p.h0 = int(bottom_mode), int(overlap), float(h0)
+    p.sweep_kernel = int(sweep_kernel)
     return p
 
 

@@ -295,3 +295,50 @@ def test_full_size_512_vcycle_bitwise(oracle_mod):
     m.set_solution(None)
     check_cycles(m, xs, ns)
     m.close()
+
+
+# ------------------------------------------------- streaming (column) kernel
+@pytest.mark.parametrize("fusion", [2, 3])
+@pytest.mark.parametrize("ghost_mode,period", [(0, 0), (1, 1), (1, 3), (1, 8)])
+def test_streaming_kernel_forced_bitwise(oracle_mod, fusion, ghost_mode, period):
+    """sweep_kernel = 2 forces the TMA-streamed column kernel on every level (plain,
+    +r and +restriction variants; owned, owned+ghost, interior and surface ranges)."""
+    shape = (64, 32, 96)
+    b = mg_inputs.random_rhs(shape, 13)
+    xs, ns = oracle_cycles(oracle_mod, b, 3, 2, 5, 4, 20)
+    m = new(shape, 3, pre=5, post=4, bottom=20, fusion=fusion, ghost_mode=ghost_mode, ca_period=period,
+            sweep_kernel=2)
+    m.set_rhs(dev(b))
+    m.set_solution(None)
+    check_cycles(m, xs, ns)
+    m.close()
+
+
+@pytest.mark.parametrize("pg", [(2, 2, 2), (2, 1, 1)])
+def test_streaming_kernel_loopback_bitwise(oracle_mod, pg):
+    _, solver = _mg()
+    n_local = (32, 32, 32)
+    gshape = (32 * pg[2], 32 * pg[1], 32 * pg[0])
+    b = mg_inputs.random_rhs(gshape, 14)
+    xs, ns = oracle_cycles(oracle_mod, b, 3, 1)
+    g = solver.LoopbackGroup(n_local, pg, num_levels=3, sweep_kernel=2)
+    g.set_rhs([dev(mg_inputs.local_block(b, r, pg)) for r in range(g.world_size)])
+    g.set_solution(None)
+    g.vcycle()
+    assert g.residual_norm() == ns[0]
+    for r in range(g.world_size):
+        assert_bitwise(host(g.get_solution(r)), mg_inputs.local_block(xs[0], r, pg), what=f"rank {r}")
+    g.close()
+
+
+def test_vcycle_config2_256_bitwise(oracle_mod):
+    """Config 2: 256^3 on one GPU, L = 6 (256 -> 8), 12/12/100: the auto kernel choice
+    (streaming on levels 0-1) gives the oracle's bits for 2 cycles."""
+    shape = (256, 256, 256)
+    b = mg_inputs.sin_rhs(shape)
+    xs, ns = oracle_cycles(oracle_mod, b, 6, 2)
+    m = new(shape, 6)
+    m.set_rhs(dev(b))
+    m.set_solution(None)
+    check_cycles(m, xs, ns)
+    m.close()
