@@ -49,6 +49,7 @@ struct DevLevel {
     ColArgs args;
   };
   std::vector<Col> cols;  // streaming-sweep plans (column segments) per brick range
+  FaceMaps fmaps[2];      // TMA face-halo tensor maps over x[0], x[1] (levels with column plans)
 };
 
 struct Plan {
@@ -255,7 +256,7 @@ mg_status sweep_range(mg_ctx* c, const Op& o, int64_t b0, int64_t b1, cudaStream
   if (c->use_col && col_supports(o.flags)) {
     for (const auto& col : d.cols) {
       if (col.b0 == b0 && col.b1 == b1) {
-        CKC(c, launch_sweep_col(a, col.args, o.flags, s));
+        CKC(c, launch_sweep_col(a, col.args, d.fmaps[o.src], o.flags, s));
         return MG_OK;
       }
     }
@@ -476,6 +477,8 @@ mg_status init_ctx(mg_ctx* c, const mg_params& p, int rank, int world, int devic
       CKC(c, cudaMemcpyAsync((void*)ca.side, ct.side.data(), ct.side.size() * 4, cudaMemcpyHostToDevice, stream));
       CKC(c, cudaMemcpyAsync((void*)ca.segs, ct.segs.data(), ct.segs.size() * 4, cudaMemcpyHostToDevice, stream));
     }
+    if (!L.cols.empty())
+      for (int xb = 0; xb < 2; ++xb) CKC(c, encode_face_maps(d.x[xb], L.n_alloc, &d.fmaps[xb]));
   }
   CKC(c, cudaStreamSynchronize(stream));  // host vectors above are temporaries
   CKC(c, cudaStreamCreateWithFlags(&c->comm, cudaStreamNonBlocking));

@@ -18,6 +18,8 @@
 
 #include <cstdint>
 
+#include <cudaTypedefs.h>
+
 #include "kernels.h"
 
 namespace mgb {
@@ -272,25 +274,29 @@ __device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t
                "l"(src), "r"(bytes), "r"(smem_u32(bar))
                : "memory");
 }
-__device__ __forceinline__ void cp_async8(void* dst, const void* src) {
-  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
-}
-__device__ __forceinline__ void cp_async_arrive_noinc(uint64_t* bar) {
-  asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(bar)) : "memory");
+__device__ __forceinline__ void tma_load_3d(void* dst, const CUtensorMap* map, int c0, int c1, int c2,
+                                            uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], "
+      "[%5];" ::"r"(smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(c2), "r"(smem_u32(bar))
+      : "memory");
 }
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 
 struct ColStage {
   double x[512];
   double b[512];
-  double face[4][64];  // W (i=7 of the W brick, [k][j]), E (i=0, [k][j]), S (j=7, [k][i]), N (j=0, [k][i])
+  double fwe[2][64][2];  // W box (i=6,7 of the W brick) and E box (i=0,1 of the E brick), [k][j][2]
+  double fsn[2][64];     // S row (j=7 of the S brick) and N row (j=0 of the N brick), [k][i]
 };
+constexpr uint32_t kStageBytes = 8192 + 2 * 1024 + 2 * 512;  // TMA bytes landing in one full stage
 
 template <bool RESTRICT>
 struct ColSmem {
-  ColStage st[COL_NST];
-  double edge[2][64];   // plane 7 of the brick below the segment, plane 0 of the brick above
-  double carry[2][64];  // plane 7 of the previous brick (k-halo of plane 0), double-buffered
+  ColStage st[COL_NST];  // stage of "brick" cnt holds only plane 0 of the brick above the segment
+  double carry[2][64];   // plane 7 of the previous brick (k-halo of plane 0), double-buffered;
+                         // carry[1] first holds plane 7 of the brick below the segment
   double rs[RESTRICT ? 2 : 1][RESTRICT ? 512 : 2];  // residual of the current brick (fused restriction)
   uint64_t bar[COL_NST + 1];
   int sid[COL_MAXSEG];
@@ -301,10 +307,10 @@ struct ColSmem {
 constexpr int COL_WARPS = 4;  // warp w streams planes 2w, 2w+1 of every brick
 
 template <unsigned FLAGS>
-__global__ void __launch_bounds__(COL_WARPS * 32, 7) sweep_col_kernel(SweepArgs p, ColArgs ca) {
+__global__ void __launch_bounds__(COL_WARPS * 32, 6)
+    sweep_col_kernel(SweepArgs p, ColArgs ca, const __grid_constant__ FaceMaps fm) {
   constexpr bool WRITE_R = (FLAGS & SW_WRITE_R) != 0;
   constexpr bool RESTRICT = (FLAGS & SW_RESTRICT) != 0;
-  constexpr int NT = COL_WARPS * 32;
   extern __shared__ __align__(128) unsigned char smem_raw[];
   ColSmem<RESTRICT>& S = *reinterpret_cast<ColSmem<RESTRICT>*>(smem_raw);
   const int t = threadIdx.x, w = t >> 5, l = t & 31;
@@ -319,48 +325,42 @@ __global__ void __launch_bounds__(COL_WARPS * 32, 7) sweep_col_kernel(SweepArgs 
     if (RESTRICT) S.spar[t] = p.parent[id];
   }
   if (t == 0) {
-    // a ring stage completes after thread 0's expect_tx arrive + NT cp.async arrivals (+ the TMA bytes)
-    for (int s = 0; s < COL_NST; ++s) mbar_init(&S.bar[s], NT + 1);
-    mbar_init(&S.bar[COL_NST], 1);
+    for (int s = 0; s <= COL_NST; ++s) mbar_init(&S.bar[s], 1);  // thread 0's expect_tx arrive + TMA bytes
     mbar_fence_init();
   }
   __syncthreads();
-  // stage brick n: x and b by TMA (thread 0); 256 face values by 8-byte cp.async
+  // stage brick n (thread 0): x and b bricks by 1D bulk copies, the four face halos
+  // by 3D tensor copies.  n == cnt stages only plane 0 of the brick above the segment.
   auto issue = [&](int n) {
+    if (t != 0) return;
     const int s = n % COL_NST;
-    if (t == 0) {
-      const int64_t id = S.sid[n];
-      mbar_expect_tx(&S.bar[s], 8192);
-      tma_load_1d(S.st[s].x, p.x + id * 512, 4096, &S.bar[s]);
-      tma_load_1d(S.st[s].b, p.b + id * 512, 4096, &S.bar[s]);
+    if (n == cnt) {
+      const int64_t above = __ldg(p.adj + (int64_t)S.sid[cnt - 1] * 8 + 5);
+      mbar_expect_tx(&S.bar[s], 512);
+      tma_load_1d(S.st[s].x, p.x + above * 512, 512, &S.bar[s]);
+      return;
     }
+    const int64_t id = S.sid[n];
     const int4 sd = S.sside[n];
-#pragma unroll
-    for (int u = 0; u < 256 / NT; ++u) {
-      const int e = t + NT * u;  // 0..255
-      const int f = e >> 6, m = e & 63;
-      const int nb = f == 0 ? sd.x : f == 1 ? sd.y : f == 2 ? sd.z : sd.w;
-      const int off = f == 0 ? 7 + 8 * (m & 7) + 64 * (m >> 3)
-                    : f == 1 ? 8 * (m & 7) + 64 * (m >> 3)
-                    : f == 2 ? (m & 7) + 56 + 64 * (m >> 3)
-                             : (m & 7) + 64 * (m >> 3);
-      cp_async8(&S.st[s].face[f][m], p.x + (int64_t)nb * 512 + off);
-    }
-    cp_async_arrive_noinc(&S.bar[s]);
+    mbar_expect_tx(&S.bar[s], kStageBytes);
+    tma_load_1d(S.st[s].x, p.x + id * 512, 4096, &S.bar[s]);
+    tma_load_1d(S.st[s].b, p.b + id * 512, 4096, &S.bar[s]);
+    tma_load_3d(S.st[s].fwe[0], &fm.we, 6, 0, sd.x * 8, &S.bar[s]);  // W brick, i = 6..7
+    tma_load_3d(S.st[s].fwe[1], &fm.we, 0, 0, sd.y * 8, &S.bar[s]);  // E brick, i = 0..1
+    tma_load_3d(S.st[s].fsn[0], &fm.sn, 0, 7, sd.z * 8, &S.bar[s]);  // S brick, j = 7
+    tma_load_3d(S.st[s].fsn[1], &fm.sn, 0, 0, sd.w * 8, &S.bar[s]);  // N brick, j = 0
   };
   if (t == 0) {
     const int64_t below = __ldg(p.adj + (int64_t)S.sid[0] * 8 + 4);
-    const int64_t above = __ldg(p.adj + (int64_t)S.sid[cnt - 1] * 8 + 5);
-    mbar_expect_tx(&S.bar[COL_NST], 1024);
-    tma_load_1d(S.edge[0], p.x + below * 512 + 448, 512, &S.bar[COL_NST]);
-    tma_load_1d(S.edge[1], p.x + above * 512, 512, &S.bar[COL_NST]);
+    mbar_expect_tx(&S.bar[COL_NST], 512);
+    tma_load_1d(S.carry[1], p.x + below * 512 + 448, 512, &S.bar[COL_NST]);
   }
   issue(0);
-  if (cnt > 1) issue(1);
-  if (w == 0 || w == COL_WARPS - 1) mbar_wait(&S.bar[COL_NST], 0);
+  issue(1);  // brick 1, or the plane above when cnt == 1
+  if (w == 0) mbar_wait(&S.bar[COL_NST], 0);
 
   for (int n = 0; n < cnt; ++n) {
-    if (n + 2 < cnt) {
+    if (n + 2 <= cnt) {
       fence_proxy_async();  // the generic-proxy reads of the stage being refilled are complete
       issue(n + 2);         // (its last readers finished before the barrier that ended step n-1)
     }
@@ -373,7 +373,7 @@ __global__ void __launch_bounds__(COL_WARPS * 32, 7) sweep_col_kernel(SweepArgs 
     if (w > 0)
       xm = *reinterpret_cast<const double2*>(X + 64 * (k0 - 1) + q);
     else
-      xm = *reinterpret_cast<const double2*>((n > 0 ? S.carry[(n - 1) & 1] : S.edge[0]) + q);
+      xm = *reinterpret_cast<const double2*>(S.carry[(n + 1) & 1] + q);  // = carry[(n-1)&1]
     xc = *reinterpret_cast<const double2*>(X + 64 * k0 + q);
     const int64_t gbase = (int64_t)S.sid[n] * 512 + q;
 #pragma unroll
@@ -381,20 +381,18 @@ __global__ void __launch_bounds__(COL_WARPS * 32, 7) sweep_col_kernel(SweepArgs 
       const int k = k0 + kk;
       if (k < 7) {
         xp = *reinterpret_cast<const double2*>(X + 64 * (k + 1) + q);
-      } else if (n + 1 < cnt) {
+      } else {  // plane 0 of the next brick (or of the brick above the segment)
         const int s1 = (n + 1) % COL_NST;
         mbar_wait(&S.bar[s1], (uint32_t)(((n + 1) / COL_NST) & 1));
         xp = *reinterpret_cast<const double2*>(S.st[s1].x + q);
-      } else {
-        xp = *reinterpret_cast<const double2*>(S.edge[1] + q);
       }
       const double2 bb = *reinterpret_cast<const double2*>(G.b + 64 * k + q);
       const double2 rs_ = *reinterpret_cast<const double2*>(X + 64 * k + (j > 0 ? q - 8 : q));
       const double2 rn_ = *reinterpret_cast<const double2*>(X + 64 * k + (j < 7 ? q + 8 : q));
-      const double fw = G.face[0][j + 8 * k];
-      const double fe = G.face[1][j + 8 * k];
-      const double2 fs = *reinterpret_cast<const double2*>(&G.face[2][i0 + 8 * k]);
-      const double2 fn = *reinterpret_cast<const double2*>(&G.face[3][i0 + 8 * k]);
+      const double fw = G.fwe[0][j + 8 * k][1];  // i = 7 of the W brick
+      const double fe = G.fwe[1][j + 8 * k][0];  // i = 0 of the E brick
+      const double2 fs = *reinterpret_cast<const double2*>(&G.fsn[0][i0 + 8 * k]);
+      const double2 fn = *reinterpret_cast<const double2*>(&G.fsn[1][i0 + 8 * k]);
       const double wl = __shfl_up_sync(0xffffffffu, xc.y, 1);
       const double er = __shfl_down_sync(0xffffffffu, xc.x, 1);
       const double wv = i0 > 0 ? wl : fw;
@@ -435,16 +433,43 @@ bool col_supports(unsigned flags) {
   return f == 0 || f == SW_WRITE_R || f == SW_RESTRICT;
 }
 
-cudaError_t launch_sweep_col(const SweepArgs& a, const ColArgs& c, unsigned flags, cudaStream_t s) {
+cudaError_t launch_sweep_col(const SweepArgs& a, const ColArgs& c, const FaceMaps& fm, unsigned flags,
+                             cudaStream_t s) {
   if (c.nseg <= 0) return cudaSuccess;
   const size_t sm = sizeof(ColSmem<false>), smr = sizeof(ColSmem<true>);
+  const unsigned g = (unsigned)c.nseg, b = COL_WARPS * 32;
   switch (flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP | SW_ZERO_X)) {
-    case 0: sweep_col_kernel<0><<<(unsigned)c.nseg, COL_WARPS * 32, sm, s>>>(a, c); break;
-    case SW_WRITE_R: sweep_col_kernel<SW_WRITE_R><<<(unsigned)c.nseg, COL_WARPS * 32, sm, s>>>(a, c); break;
-    case SW_RESTRICT: sweep_col_kernel<SW_RESTRICT><<<(unsigned)c.nseg, COL_WARPS * 32, smr, s>>>(a, c); break;
+    case 0: sweep_col_kernel<0><<<g, b, sm, s>>>(a, c, fm); break;
+    case SW_WRITE_R: sweep_col_kernel<SW_WRITE_R><<<g, b, sm, s>>>(a, c, fm); break;
+    case SW_RESTRICT: sweep_col_kernel<SW_RESTRICT><<<g, b, smr, s>>>(a, c, fm); break;
     default: return cudaErrorInvalidValue;
   }
   return cudaGetLastError();
+}
+
+cudaError_t encode_face_maps(const double* x, int64_t n_alloc, FaceMaps* out) {
+  static PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
+  if (!encode) {
+    void* fn = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    cudaError_t e = cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q);
+    if (e != cudaSuccess) return e;
+    if (q != cudaDriverEntryPointSuccess || !fn) return cudaErrorNotSupported;
+    encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
+  }
+  const cuuint64_t dims[3] = {8, 8, (cuuint64_t)n_alloc * 8};  // i, j, planes
+  const cuuint64_t strides[2] = {64, 512};                      // bytes of one j row, one plane
+  const cuuint32_t estr[3] = {1, 1, 1};
+  const cuuint32_t box_we[3] = {2, 8, 8};
+  const cuuint32_t box_sn[3] = {8, 1, 8};
+  CUresult r = encode(&out->we, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, const_cast<double*>(x), dims, strides, box_we,
+                      estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_NONE,
+                      CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return cudaErrorInvalidValue;
+  r = encode(&out->sn, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, const_cast<double*>(x), dims, strides, box_sn, estr,
+             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_NONE,
+             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
 }
 
 cudaError_t launch_apply_op(const double* x, double* Ax, const int32_t* adj, int64_t brick0, int64_t nbricks,

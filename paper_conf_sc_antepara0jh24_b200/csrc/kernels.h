@@ -1,6 +1,7 @@
 // kernels.h -- launchers for the sm_100a brick kernels (kernels.cu).
 #pragma once
 
+#include <cuda.h>  // CUtensorMap (types only; the driver entry point is fetched at run time)
 #include <cuda_runtime.h>
 
 #include <cstdint>
@@ -45,9 +46,20 @@ struct ColArgs {
   const int2* segs;       // (offset, count) per segment, count <= 16
   int64_t nseg;
 };
+// TMA tensor maps over one x field seen as [n_alloc*8 planes][8 j][8 i] doubles:
+// `we` boxes {2 i, 8 j, 8 k} (the W / E face columns), `sn` boxes {8 i, 1 j, 8 k}
+// (the S / N face rows).  One tensor copy per face per brick, no LSU gathers.
+struct FaceMaps {
+  CUtensorMap we;
+  CUtensorMap sn;
+};
+// Encodes the two maps for the field at `x` with `n_alloc` bricks (driver entry
+// point obtained through the runtime; no libcuda link).
+cudaError_t encode_face_maps(const double* x, int64_t n_alloc, FaceMaps* out);
 // true if the streaming kernel implements `flags` (plain, +r, +restriction)
 bool col_supports(unsigned flags);
-cudaError_t launch_sweep_col(const SweepArgs& a, const ColArgs& c, unsigned flags, cudaStream_t s);
+cudaError_t launch_sweep_col(const SweepArgs& a, const ColArgs& c, const FaceMaps& fm, unsigned flags,
+                             cudaStream_t s);
 // applyOp (paper kernel set): Ax = alpha x + beta sum6
 cudaError_t launch_apply_op(const double* x, double* Ax, const int32_t* adj, int64_t brick0, int64_t nbricks,
                             Coeffs c, cudaStream_t s);
