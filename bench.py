@@ -346,7 +346,8 @@ def main():
                        "parallelism": f"3D domain decomposition {pg[0]}x{pg[1]}x{pg[2]}"},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic,
-                         "kernel": "level-0 fused sweep (sweep_kernel), avg over the 24 level-0 sweeps of a V-cycle",
+                         "kernel": "level-0 fused sweeps (sweep_col_kernel streaming + the interp-fused "
+                                   "sweep_kernel), avg over the 24 level-0 sweeps of a V-cycle",
                          "launch_ms": launch_ms, "bytes_per_point": bytes0 / pts / nsweep0,
                          "peak_source": peak_src, "frac_of_8TBs": achieved / 8000.0},
             "cpu_baseline": cpu,
