@@ -105,7 +105,9 @@ typedef struct {
   int32_t overlap;               /* 1 = sweep interior bricks while the exchange is in flight */
   int32_t sweep_kernel;          /* 0 = auto (streaming column kernel on levels >= 16384 bricks),
                                     1 = one-brick-per-CTA kernel only, 2 = streaming kernel on every level */
-  int32_t reserved[6];
+  int32_t temporal_blocking;     /* 1 = two Jacobi sweeps per HBM pass on streaming levels (sweep2.cu,
+                                    bit-identical), 0 = one sweep per pass (default: faster today) */
+  int32_t reserved[5];
   double h0;                     /* finest spacing; <= 0 => 1 / max_d(global N_d) (reading A7) */
 } mg_params;
 

@@ -50,6 +50,12 @@ struct DevLevel {
   };
   std::vector<Col> cols;  // streaming-sweep plans (column segments) per brick range
   FaceMaps fmaps[2];      // TMA face-halo tensor maps over x[0], x[1] (levels with column plans)
+  struct Pair {
+    int64_t b0, b1;
+    PairArgs args;
+  };
+  std::vector<Pair> pairs;  // two-sweep item streams per brick range
+  PairMaps pmaps[2];        // tensor maps for the two-sweep kernel reading x[0] / x[1]
 };
 
 struct Plan {
@@ -163,6 +169,15 @@ size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double**
       col.args.nseg = (int64_t)ct.segs.size() / 2;
       d.cols.push_back(col);
     }
+    for (const auto& pt : L.pairs) {
+      DevLevel::Pair pr;
+      pr.b0 = pt.b0;
+      pr.b1 = pt.b1;
+      pr.args.meta = (const int32_t*)take(pt.meta.size() * sizeof(int32_t));
+      pr.args.ctas = (const int2*)take(pt.ctas.size() * sizeof(int32_t));
+      pr.args.nctas = (int64_t)pt.ctas.size() / 2;
+      d.pairs.push_back(pr);
+    }
     d.h = lay.p.h0 * (double)(1 << l);
     d.c = level_coeffs(d.h);
     if (out) (*out)[l] = d;
@@ -253,6 +268,15 @@ mg_status sweep_range(mg_ctx* c, const Op& o, int64_t b0, int64_t b1, cudaStream
   a.brick0 = b0;
   a.nbricks = b1 - b0;
   a.c = d.c;
+  if (o.kind == OP_SWEEP2) {  // two sweeps in one pass: the builder only emits it where a plan exists
+    for (const auto& pr : d.pairs) {
+      if (pr.b0 == b0 && pr.b1 == b1) {
+        CKC(c, launch_sweep2(a, pr.args, d.pmaps[o.src], o.flags, s));
+        return MG_OK;
+      }
+    }
+    return set_err(MG_ERR_STATE, "no two-sweep plan for this brick range");
+  }
   if (c->use_col && col_supports(o.flags)) {
     for (const auto& col : d.cols) {
       if (col.b0 == b0 && col.b1 == b1) {
@@ -284,7 +308,8 @@ mg_status exec_op(mg_ctx* c, const Op& o, cudaStream_t s) {
   DevLevel& d = c->dl[o.level];
   cudaEvent_t t0 = nullptr;
   switch (o.kind) {
-    case OP_SWEEP: {
+    case OP_SWEEP:
+    case OP_SWEEP2: {
       const int64_t end = o.ghosts ? L.n_stored : L.n_owned;
       if (o.exch_before) {
         const bool split = c->lay.p.overlap && L.n_interior > 0;
@@ -479,6 +504,14 @@ mg_status init_ctx(mg_ctx* c, const mg_params& p, int rank, int world, int devic
     }
     if (!L.cols.empty())
       for (int xb = 0; xb < 2; ++xb) CKC(c, encode_face_maps(d.x[xb], L.n_alloc, &d.fmaps[xb]));
+    for (size_t k = 0; k < L.pairs.size(); ++k) {
+      const auto& pt = L.pairs[k];
+      const PairArgs& pa = d.pairs[k].args;
+      CKC(c, cudaMemcpyAsync((void*)pa.meta, pt.meta.data(), pt.meta.size() * 4, cudaMemcpyHostToDevice, stream));
+      CKC(c, cudaMemcpyAsync((void*)pa.ctas, pt.ctas.data(), pt.ctas.size() * 4, cudaMemcpyHostToDevice, stream));
+    }
+    if (!L.pairs.empty())
+      for (int xb = 0; xb < 2; ++xb) CKC(c, encode_pair_maps(d.x[xb], d.b, L.n_alloc, &d.pmaps[xb]));
   }
   CKC(c, cudaStreamSynchronize(stream));  // host vectors above are temporaries
   CKC(c, cudaStreamCreateWithFlags(&c->comm, cudaStreamNonBlocking));
@@ -545,6 +578,7 @@ void mg_params_default(mg_params* p) {
   p->bottom_smooths = 100;
   p->use_graph = 1;
   p->overlap = 1;
+  p->temporal_blocking = 0;  // see include/mg.h: the two-sweep kernel is correct but not yet faster
   p->h0 = 0.0;
 }
 
@@ -742,7 +776,7 @@ mg_status mg_exchange_stats(mg_ctx* c, int64_t* bytes_per_cycle, int64_t* messag
   b.vcycle();
   int64_t bytes = 0, msgs = 0;
   for (const Op& o : b.ops) {
-    const bool ex = o.kind == OP_EXCH || (o.kind == OP_SWEEP && o.exch_before);
+    const bool ex = o.kind == OP_EXCH || ((o.kind == OP_SWEEP || o.kind == OP_SWEEP2) && o.exch_before);
     if (!ex) continue;
     for (const Run& r : c->lay.lv[o.level].sends) {
       bytes += r.count * kBV * (int64_t)sizeof(double);

@@ -21,6 +21,7 @@
 #include <cudaTypedefs.h>
 
 #include "kernels.h"
+#include "ptx.cuh"
 
 namespace mgb {
 
@@ -33,30 +34,8 @@ Coeffs level_coeffs(double h) {
   return c;
 }
 
-#define DMUL __dmul_rn
-#define DADD __dadd_rn
-#define DSUB __dsub_rn
-
-__device__ __forceinline__ double stencil_a(double c, double w, double e, double s, double n, double bt, double tp,
-                                            double alpha, double beta) {
-  const double sum = DADD(DADD(DADD(w, e), DADD(s, n)), DADD(bt, tp));
-  return DADD(DMUL(alpha, c), DMUL(beta, sum));
-}
-
 // max that propagates NaN (a diverged iterate must not hide in the norm)
 __device__ __forceinline__ double nan_max(double a, double b) { return (b > a || b != b) ? b : a; }
-
-__device__ __forceinline__ double2 ldg2(const double* p) { return __ldg(reinterpret_cast<const double2*>(p)); }
-__device__ __forceinline__ double2 ld_stream2(const double* p) {
-  double2 v;
-  asm volatile("ld.global.nc.L1::no_allocate.v2.f64 {%0, %1}, [%2];"
-               : "=d"(v.x), "=d"(v.y)
-               : "l"(p));
-  return v;
-}
-__device__ __forceinline__ void st_stream2(double* p, double2 v) {
-  asm volatile("st.global.L1::no_allocate.v2.f64 [%0], {%1, %2};" ::"l"(p), "d"(v.x), "d"(v.y) : "memory");
-}
 
 // coarse-cell offset of fine cell (i,j,k) of a fine brick with octant o
 __device__ __forceinline__ int coarse_off(int oct, int i, int j, int k) {
@@ -253,37 +232,6 @@ cudaError_t launch_sweep(const SweepArgs& a, unsigned flags, cudaStream_t s) {
 constexpr int COL_NST = 3;  // ring stages: current, next (plane 0 = k-halo), one in flight
 constexpr int COL_MAXSEG = 16;
 
-__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
-__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_fence_init() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
-__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-  asm volatile(
-      "{\n .reg .pred p;\n"
-      "MBW_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n @!p bra MBW_%=;\n}" ::"r"(smem_u32(bar)),
-      "r"(parity)
-      : "memory");
-}
-__device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-                   smem_u32(dst)),
-               "l"(src), "r"(bytes), "r"(smem_u32(bar))
-               : "memory");
-}
-__device__ __forceinline__ void tma_load_3d(void* dst, const CUtensorMap* map, int c0, int c1, int c2,
-                                            uint64_t* bar) {
-  asm volatile(
-      "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], "
-      "[%5];" ::"r"(smem_u32(dst)),
-      "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(c2), "r"(smem_u32(bar))
-      : "memory");
-}
-__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
-
 struct ColStage {
   double x[512];
   double b[512];
@@ -447,7 +395,7 @@ cudaError_t launch_sweep_col(const SweepArgs& a, const ColArgs& c, const FaceMap
   return cudaGetLastError();
 }
 
-cudaError_t encode_face_maps(const double* x, int64_t n_alloc, FaceMaps* out) {
+cudaError_t encode_box_map(const double* base, int64_t n_alloc, const unsigned box[3], CUtensorMap* out) {
   static PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
   if (!encode) {
     void* fn = nullptr;
@@ -460,16 +408,28 @@ cudaError_t encode_face_maps(const double* x, int64_t n_alloc, FaceMaps* out) {
   const cuuint64_t dims[3] = {8, 8, (cuuint64_t)n_alloc * 8};  // i, j, planes
   const cuuint64_t strides[2] = {64, 512};                      // bytes of one j row, one plane
   const cuuint32_t estr[3] = {1, 1, 1};
-  const cuuint32_t box_we[3] = {2, 8, 8};
-  const cuuint32_t box_sn[3] = {8, 1, 8};
-  CUresult r = encode(&out->we, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, const_cast<double*>(x), dims, strides, box_we,
-                      estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_NONE,
-                      CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-  if (r != CUDA_SUCCESS) return cudaErrorInvalidValue;
-  r = encode(&out->sn, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, const_cast<double*>(x), dims, strides, box_sn, estr,
-             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_NONE,
-             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  const cuuint32_t bx[3] = {box[0], box[1], box[2]};
+  const CUresult r = encode(out, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, const_cast<double*>(base), dims, strides, bx,
+                            estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                            CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
+}
+
+cudaError_t encode_face_maps(const double* x, int64_t n_alloc, FaceMaps* out) {
+  const unsigned box_we[3] = {2, 8, 8}, box_sn[3] = {8, 1, 8};
+  cudaError_t e = encode_box_map(x, n_alloc, box_we, &out->we);
+  if (e != cudaSuccess) return e;
+  return encode_box_map(x, n_alloc, box_sn, &out->sn);
+}
+
+cudaError_t encode_pair_maps(const double* x, const double* b, int64_t n_alloc, PairMaps* out) {
+  const unsigned we[3] = {2, 8, 8}, sn2[3] = {8, 2, 8}, cor[3] = {2, 1, 8}, sn1[3] = {8, 1, 8};
+  cudaError_t e;
+  if ((e = encode_box_map(x, n_alloc, we, &out->xwe)) != cudaSuccess) return e;
+  if ((e = encode_box_map(x, n_alloc, sn2, &out->xsn)) != cudaSuccess) return e;
+  if ((e = encode_box_map(x, n_alloc, cor, &out->xcor)) != cudaSuccess) return e;
+  if ((e = encode_box_map(b, n_alloc, we, &out->bwe)) != cudaSuccess) return e;
+  return encode_box_map(b, n_alloc, sn1, &out->bsn);
 }
 
 cudaError_t launch_apply_op(const double* x, double* Ax, const int32_t* adj, int64_t brick0, int64_t nbricks,
@@ -710,8 +670,10 @@ cudaError_t kernels_init() {
     e = cudaFuncSetAttribute(colk[k], cudaFuncAttributePreferredSharedMemoryCarveout, 100);
     if (e != cudaSuccess) return e;
   }
-  return cudaFuncSetAttribute(bottom_resident_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                              kResidentMaxBricks * 512 * 3 * (int)sizeof(double));
+  e = cudaFuncSetAttribute(bottom_resident_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           kResidentMaxBricks * 512 * 3 * (int)sizeof(double));
+  if (e != cudaSuccess) return e;
+  return pair_kernels_init();
 }
 
 }  // namespace mgb

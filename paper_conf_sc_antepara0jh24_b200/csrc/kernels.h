@@ -56,6 +56,30 @@ struct FaceMaps {
 // Encodes the two maps for the field at `x` with `n_alloc` bricks (driver entry
 // point obtained through the runtime; no libcuda link).
 cudaError_t encode_face_maps(const double* x, int64_t n_alloc, FaceMaps* out);
+// One TMA tensor map over a brick field seen as [n_alloc*8 planes][8 j][8 i]
+// doubles with the given box {i, j, planes}.
+cudaError_t encode_box_map(const double* base, int64_t n_alloc, const unsigned box[3], CUtensorMap* out);
+
+// Two-sweep (temporally blocked) streaming kernel, sweep2.cu.
+struct PairArgs {
+  const int32_t* meta;  // [items][11] id, flags, W,E,S,N, SW,NW,SE,NE, parent
+  const int2* ctas;     // (first item, item count) per CTA
+  int64_t nctas;
+};
+struct PairMaps {
+  CUtensorMap xwe;   // x boxes {2,8,8}: W (i=6,7) / E (i=0,1) face slabs
+  CUtensorMap xsn;   // x boxes {8,2,8}: S (j=6,7) / N (j=0,1) face slabs
+  CUtensorMap xcor;  // x boxes {2,1,8}: the four diagonal-corner columns
+  CUtensorMap bwe;   // b boxes {2,8,8}
+  CUtensorMap bsn;   // b boxes {8,1,8}
+};
+cudaError_t encode_pair_maps(const double* x, const double* b, int64_t n_alloc, PairMaps* out);
+// flags apply to the SECOND sweep of the pair: plain, +r, +restriction
+bool pair_supports(unsigned flags);
+cudaError_t launch_sweep2(const SweepArgs& a, const PairArgs& pa, const PairMaps& pm, unsigned flags,
+                          cudaStream_t s);
+cudaError_t pair_kernels_init();
+
 // true if the streaming kernel implements `flags` (plain, +r, +restriction)
 bool col_supports(unsigned flags);
 cudaError_t launch_sweep_col(const SweepArgs& a, const ColArgs& c, const FaceMaps& fm, unsigned flags,

@@ -264,6 +264,8 @@ mg_status build_layout(const mg_params& p, int rank, int world, Layout& out, std
   const int64_t min_b = p.sweep_kernel == 1 ? INT64_MAX : p.sweep_kernel == 2 ? 0 : kColMinBricks;
   for (int l = 0; l < out.L; ++l) build_col_tables(out.lv[l], min_b);
   for (int l = 0; l + 1 < out.L; ++l) build_parents(out.lv[l], out.lv[l + 1]);
+  if (p.temporal_blocking != 0)
+    for (int l = 0; l < out.L; ++l) build_pair_tables(out.lv[l], min_b);
   return MG_OK;
 }
 
@@ -275,10 +277,10 @@ namespace mgb {
 // brick of [b0,b1) exactly once, as z-chains following the adjacency T link
 // (periodic columns are cycles; ghost-shell columns end at the zero brick),
 // each chain cut into near-equal segments of <= kColSeg bricks.
-static LevelLayout::ColTable col_table(const LevelLayout& L, int64_t b0, int64_t b1) {
-  LevelLayout::ColTable t;
-  t.b0 = b0;
-  t.b1 = b1;
+// The bricks of [b0,b1) as z-chains along the T link, each brick exactly once,
+// chains in order of their first brick's storage index.
+static std::vector<std::vector<int32_t>> z_chains(const LevelLayout& L, int64_t b0, int64_t b1) {
+  std::vector<std::vector<int32_t>> out;
   std::vector<char> vis((size_t)(b1 - b0), 0);
   auto in = [&](int64_t q) { return q >= b0 && q < b1; };
   for (int64_t q = b0; q < b1; ++q) {
@@ -294,6 +296,16 @@ static LevelLayout::ColTable col_table(const LevelLayout& L, int64_t b0, int64_t
       vis[(size_t)(c - b0)] = 1;
       chain.push_back((int32_t)c);
     }
+    out.push_back(std::move(chain));
+  }
+  return out;
+}
+
+static LevelLayout::ColTable col_table(const LevelLayout& L, int64_t b0, int64_t b1) {
+  LevelLayout::ColTable t;
+  t.b0 = b0;
+  t.b1 = b1;
+  for (const auto& chain : z_chains(L, b0, b1)) {
     const int64_t len = (int64_t)chain.size();
     const int64_t nseg = (len + kColSeg - 1) / kColSeg;
     int64_t off = 0;
@@ -325,6 +337,81 @@ void build_col_tables(LevelLayout& L, int64_t min_bricks) {
     bool dup = false;
     for (auto& c : L.cols) dup |= (c.b0 == r[0] && c.b1 == r[1]);
     if (!dup) L.cols.push_back(col_table(L, r[0], r[1]));
+  }
+}
+
+// Item streams for the two-sweep kernel (sweep2.cu), one per resident CTA
+// (G = kPairCtas).  Whole z-chains are dealt round-robin -- CTA g takes chains
+// g, g+G, g+2G, ... -- so the CTAs running at any moment work on neighbouring
+// columns at about the same height and their side-face reads hit L2.  The
+// chains of the last, incomplete round are concatenated and cut into G equal
+// pieces, so every CTA gets the same number of bricks.  Each run of bricks of
+// one chain becomes [warm-up, run..., cool-down], warm-up / cool-down being the
+// B / T neighbours of the run's ends: the kernel computes the first sweep on
+// them too (their x1 planes 7 / 0 are k-halos of the run's second sweep).
+static LevelLayout::PairTable pair_table(const LevelLayout& L, int64_t b0, int64_t b1) {
+  LevelLayout::PairTable t;
+  t.b0 = b0;
+  t.b1 = b1;
+  const auto chains = z_chains(L, b0, b1);
+  const int64_t nch = (int64_t)chains.size();
+  int64_t nb = 0;
+  for (const auto& c : chains) nb += (int64_t)c.size();
+  const int64_t G = std::max<int64_t>(1, std::min<int64_t>(kPairCtas, nb / 8));
+  auto adj = [&](int64_t id, int f) -> int32_t {
+    return id >= L.n_stored ? (int32_t)L.zero_brick : L.adj[(size_t)id * 8 + f];
+  };
+  std::vector<std::vector<int32_t>> stream((size_t)G);  // per CTA: its item metadata
+  auto push_item = [&](std::vector<int32_t>& v, int32_t id, int32_t flags) {
+    const int32_t W = adj(id, 0), E = adj(id, 1), S = adj(id, 2), N = adj(id, 3);
+    const int32_t par = (id < L.n_stored && !L.parent.empty()) ? L.parent[(size_t)id] : -1;
+    const int32_t m[kPairMeta] = {id, flags, W, E, S, N, adj(W, 2), adj(W, 3), adj(E, 2), adj(E, 3), par};
+    v.insert(v.end(), m, m + kPairMeta);
+  };
+  auto push_run = [&](std::vector<int32_t>& v, const int32_t* run, int64_t len) {
+    push_item(v, adj(run[0], 4), 0);  // warm-up
+    for (int64_t q = 0; q < len; ++q) push_item(v, run[q], q > 0 ? 1 : 0);
+    push_item(v, adj(run[len - 1], 5), 1);  // cool-down
+  };
+  const int64_t full = (nch / G) * G;  // chains dealt round-robin
+  for (int64_t c = 0; c < full; ++c) push_run(stream[(size_t)(c % G)], chains[(size_t)c].data(), chains[(size_t)c].size());
+  std::vector<int32_t> rest, rest_chain;
+  for (int64_t c = full; c < nch; ++c)
+    for (int32_t id : chains[(size_t)c]) {
+      rest.push_back(id);
+      rest_chain.push_back((int32_t)c);
+    }
+  const int64_t nr = (int64_t)rest.size();
+  int64_t off = 0;
+  for (int64_t g = 0; g < G && nr > 0; ++g) {
+    const int64_t cnt = nr / G + (g < nr % G ? 1 : 0);
+    for (int64_t m = off; m < off + cnt;) {
+      int64_t e = m + 1;
+      while (e < off + cnt && rest_chain[(size_t)e] == rest_chain[(size_t)m]) ++e;
+      push_run(stream[(size_t)g], &rest[(size_t)m], e - m);
+      m = e;
+    }
+    off += cnt;
+  }
+  for (int64_t g = 0; g < G; ++g) {
+    const auto& v = stream[(size_t)g];
+    if (v.empty()) continue;
+    t.ctas.push_back((int32_t)((int64_t)t.meta.size() / kPairMeta));
+    t.ctas.push_back((int32_t)((int64_t)v.size() / kPairMeta));
+    t.meta.insert(t.meta.end(), v.begin(), v.end());
+  }
+  return t;
+}
+
+void build_pair_tables(LevelLayout& L, int64_t min_bricks) {
+  L.pairs.clear();
+  if (L.n_stored < min_bricks) return;
+  const int64_t ranges[3][2] = {{0, L.n_owned}, {0, L.n_interior}, {L.n_interior, L.n_owned}};
+  for (auto& r : ranges) {
+    if (r[1] <= r[0]) continue;
+    bool dup = false;
+    for (auto& c : L.pairs) dup |= (c.b0 == r[0] && c.b1 == r[1]);
+    if (!dup) L.pairs.push_back(pair_table(L, r[0], r[1]));
   }
 }
 

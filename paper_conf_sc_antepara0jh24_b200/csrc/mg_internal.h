@@ -57,7 +57,22 @@ struct LevelLayout {
     std::vector<int32_t> segs;    // [nseg][2] offset into bricks, count
   };
   std::vector<ColTable> cols;     // one per distinct range the schedule sweeps
+  // Item streams for the two-sweep (temporally blocked) kernel: the bricks of a
+  // range as z-chains, cut into near-equal CTA pieces; each piece is preceded by
+  // its warm-up brick (the B neighbour of its first brick) and followed by its
+  // cool-down brick (T neighbour of its last): item = (id, flags, W,E,S,N,
+  // SW,NW,SE,NE, parent), flags bit0 = "previous item is a range brick".
+  struct PairTable {
+    int64_t b0 = 0, b1 = 0;
+    std::vector<int32_t> meta;  // [items][kPairMeta]
+    std::vector<int32_t> ctas;  // [nctas][2] offset (items), count
+  };
+  std::vector<PairTable> pairs;
 };
+
+constexpr int kPairMeta = 11;
+constexpr int64_t kPairCtas = 148 * 3;  // one item stream per resident two-sweep CTA (148 SMs x 3)
+void build_pair_tables(LevelLayout& L, int64_t min_bricks);
 
 constexpr int kColSeg = 16;             // bricks per streamed segment
 constexpr int64_t kColMinBricks = 16384;  // levels smaller than this use the one-brick-per-CTA kernel

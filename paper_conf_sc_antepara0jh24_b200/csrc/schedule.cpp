@@ -22,12 +22,54 @@ int Builder::period(int l) const {
   return k ? k : MG_MAX_PERIOD;
 }
 
+bool Builder::pair_ok(int l) const {
+  if (!lay.p.temporal_blocking || fusion(l) == MG_FUSION_PAPER) return false;
+  const LevelLayout& L = lay.lv[l];
+  auto has = [&](int64_t b0, int64_t b1) {
+    for (const auto& pt : L.pairs)
+      if (pt.b0 == b0 && pt.b1 == b1) return true;
+    return false;
+  };
+  if (!has(0, L.n_owned)) return false;
+  if (ghosts(l)) {
+    if (period(l) < 2) return false;  // a pair is two sweeps per exchange
+    if (lay.p.overlap && L.n_interior > 0 && !(has(0, L.n_interior) && has(L.n_interior, L.n_owned))) return false;
+  }
+  return true;
+}
+
 void Builder::phase(int l, int n, bool zero_first, int last, bool interp_first, int timer) {
   const bool g = ghosts(l);
   const int k = period(l);
   const bool paper = fusion(l) == MG_FUSION_PAPER;
+  const bool pairs = pair_ok(l);
   LevelState& S = st[l];
   for (int s = 0; s < n; ++s) {
+    const bool single_only = (zero_first && s == 0) || (interp_first && s == 0);
+    if (pairs && !single_only && s + 1 < n) {
+      // sweeps s and s+1 in one pass (temporal blocking); x1 never leaves the chip
+      Op o;
+      o.kind = OP_SWEEP2;
+      o.level = l;
+      o.timer = timer;
+      const bool ex = g && (S.dx < 2 || S.since + 2 > k);
+      if (ex) {
+        S.dx = MG_MAX_PERIOD;
+        S.since = 0;
+      }
+      o.exch_before = ex;
+      o.ghosts = false;
+      if (s + 1 == n - 1 && last == 1) o.flags |= SW_WRITE_R;
+      if (s + 1 == n - 1 && last == 2) o.flags |= SW_RESTRICT;
+      o.src = S.cur;
+      o.dst = 1 - S.cur;
+      S.cur = o.dst;
+      S.dx = 0;
+      S.since += 2;
+      ops.push_back(o);
+      ++s;
+      continue;
+    }
     Op o;
     o.kind = OP_SWEEP;
     o.level = l;
@@ -169,7 +211,8 @@ void Builder::vcycle() {
 
 int64_t op_launches(const Op& o, const Layout& lay, bool overlap) {
   switch (o.kind) {
-    case OP_SWEEP: {
+    case OP_SWEEP:
+    case OP_SWEEP2: {
       const int per = o.paper ? 2 : 1;
       const bool split = o.exch_before && overlap && lay.lv[o.level].n_interior > 0;
       return per * (split ? 2 : 1);

@@ -16,7 +16,9 @@
 
 namespace mgb {
 
-enum OpKind { OP_SWEEP = 0, OP_RESTRICT, OP_INTERP, OP_ZERO, OP_EXCH, OP_BOTTOM_RES };
+enum OpKind { OP_SWEEP = 0, OP_RESTRICT, OP_INTERP, OP_ZERO, OP_EXCH, OP_BOTTOM_RES, OP_SWEEP2 };
+// OP_SWEEP2: two consecutive plain sweeps in one pass (sweep2.cu); `flags` are the
+// second sweep's (r / restriction); owned bricks only; needs ghost depth >= 2.
 
 struct Op {
   int kind = OP_SWEEP;
@@ -50,6 +52,7 @@ struct Builder {
   bool ghosts(int l) const { return lay.lv[l].n_ghost > 0; }
   int fusion(int l) const;
   int period(int l) const;
+  bool pair_ok(int l) const;  // two-sweep passes possible at level l
   // `n` smooth(+residual) sweeps at level l.  last: 0 none, 1 write r, 2 fused restriction.
   void phase(int l, int n, bool zero_first, int last, bool interp_first, int timer);
   void restrict_op(int l);  // b_{l+1} = R r_l (+ b ghost exchange)

@@ -298,30 +298,33 @@ def test_full_size_512_vcycle_bitwise(oracle_mod):
 
 
 # ------------------------------------------------- streaming (column) kernel
+@pytest.mark.parametrize("tb", [0, 1])
 @pytest.mark.parametrize("fusion", [2, 3])
 @pytest.mark.parametrize("ghost_mode,period", [(0, 0), (1, 1), (1, 3), (1, 8)])
-def test_streaming_kernel_forced_bitwise(oracle_mod, fusion, ghost_mode, period):
-    """sweep_kernel = 2 forces the TMA-streamed column kernel on every level (plain,
-    +r and +restriction variants; owned, owned+ghost, interior and surface ranges)."""
+def test_streaming_kernel_forced_bitwise(oracle_mod, fusion, ghost_mode, period, tb):
+    """sweep_kernel = 2 forces the TMA-streamed column kernel (tb = 0) or the two-sweep
+    kernel (tb = 1) on every level (plain, +r and +restriction variants; owned,
+    owned+ghost, interior and surface ranges)."""
     shape = (64, 32, 96)
     b = mg_inputs.random_rhs(shape, 13)
     xs, ns = oracle_cycles(oracle_mod, b, 3, 2, 5, 4, 20)
     m = new(shape, 3, pre=5, post=4, bottom=20, fusion=fusion, ghost_mode=ghost_mode, ca_period=period,
-            sweep_kernel=2)
+            sweep_kernel=2, temporal_blocking=tb)
     m.set_rhs(dev(b))
     m.set_solution(None)
     check_cycles(m, xs, ns)
     m.close()
 
 
+@pytest.mark.parametrize("tb", [0, 1])
 @pytest.mark.parametrize("pg", [(2, 2, 2), (2, 1, 1)])
-def test_streaming_kernel_loopback_bitwise(oracle_mod, pg):
+def test_streaming_kernel_loopback_bitwise(oracle_mod, pg, tb):
     _, solver = _mg()
     n_local = (32, 32, 32)
     gshape = (32 * pg[2], 32 * pg[1], 32 * pg[0])
     b = mg_inputs.random_rhs(gshape, 14)
     xs, ns = oracle_cycles(oracle_mod, b, 3, 1)
-    g = solver.LoopbackGroup(n_local, pg, num_levels=3, sweep_kernel=2)
+    g = solver.LoopbackGroup(n_local, pg, num_levels=3, sweep_kernel=2, temporal_blocking=tb)
     g.set_rhs([dev(mg_inputs.local_block(b, r, pg)) for r in range(g.world_size)])
     g.set_solution(None)
     g.vcycle()
@@ -338,6 +341,42 @@ def test_vcycle_config2_256_bitwise(oracle_mod):
     b = mg_inputs.sin_rhs(shape)
     xs, ns = oracle_cycles(oracle_mod, b, 6, 2)
     m = new(shape, 6)
+    m.set_rhs(dev(b))
+    m.set_solution(None)
+    check_cycles(m, xs, ns)
+    m.close()
+
+
+# ------------------------------------------------- two sweeps per pass (temporal blocking)
+@pytest.mark.parametrize("n", [2, 3, 5])
+@pytest.mark.parametrize("shape,ghost_mode", [((64, 32, 96), 0), ((32, 48, 64), 1)])
+def test_two_sweep_pass_per_op(oracle_mod, n, shape, ghost_mode):
+    """OP_SWEEP2 (x0 -> x1 -> x2 in one pass, redundant x1 on the side faces) equals
+    n separate sweeps of the oracle bit for bit, including r of the last sweep."""
+    mg, _ = _mg()
+    m = new(shape, 1, pre=1, post=1, bottom=1, sweep_kernel=2, ghost_mode=ghost_mode, temporal_blocking=1)
+    h = mg_inputs.default_h0(shape)
+    x = mg_inputs.random_field(shape, 21)
+    b = mg_inputs.random_field(shape, 22)
+    m.level_set(0, mg.MG_FIELD_X, dev(x))
+    m.level_set(0, mg.MG_FIELD_B, dev(b))
+    mg.mg_op_smooth(m.ctx, 0, n, 1, 2)
+    xo, ro = x, None
+    for _ in range(n):
+        xo, ro = oracle_mod.smooth_residual(xo, oracle_mod.apply_op(xo, h), b, h)
+    assert_bitwise(host(m.level_get(0, mg.MG_FIELD_X)), xo, what="x")
+    assert_bitwise(host(m.level_get(0, mg.MG_FIELD_R)), ro, what="r")
+    m.close()
+
+
+@pytest.mark.parametrize("tb", [0, 1])
+def test_temporal_blocking_on_off_bitwise(oracle_mod, tb):
+    """The V-cycle with and without temporal blocking gives the oracle's bits (256^3, L = 6,
+    where levels 0 and 1 stream; 12/12/100)."""
+    shape = (256, 256, 256)
+    b = mg_inputs.random_rhs(shape, 23)
+    xs, ns = oracle_cycles(oracle_mod, b, 6, 1)
+    m = new(shape, 6, temporal_blocking=tb)
     m.set_rhs(dev(b))
     m.set_solution(None)
     check_cycles(m, xs, ns)
