@@ -49,6 +49,7 @@ def parse():
     ap.add_argument("--ghost-all", action="store_true", help="self-exchange ghost shell on every axis")
     ap.add_argument("--no-graph", action="store_true")
     ap.add_argument("--no-overlap", action="store_true")
+    ap.add_argument("--tb", type=int, default=1, help="temporal blocking: two sweeps per HBM pass (sweep2.cu)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--ref-n", type=int, default=0, help="reference arm: grid side of the bounded sample")
@@ -237,7 +238,7 @@ def main():
     n = a.n
     m = Multigrid((n, n, n), pg, a.levels, a.pre, a.post, a.bottom, ca_period=a.ca_period, fusion=a.fusion,
                   ghost_mode=1 if a.ghost_all else 0, use_graph=not a.no_graph, overlap=not a.no_overlap,
-                  rank=rank, world_size=world, device=local)
+                  rank=rank, world_size=world, device=local, temporal_blocking=a.tb)
     gshape = (n * pg[2], n * pg[1], n * pg[0])
     b_host = torch.from_numpy(mg_inputs.local_sin_rhs(gshape, rank, pg)).pin_memory()
     b_dev = b_host.to(dev)
@@ -287,14 +288,24 @@ def main():
     m.set_timing(False)
     nsweep0 = a.pre + a.post
     sweep0_ms = tm[0][mg.OP_NAMES.index("sweep")] / ninst
-    launch_ms = sweep0_ms / nsweep0
-    # algorithmic bytes of the level-0 sweeps of one V-cycle (fully fused: restriction / interpolation fused)
-    pts = n**3
-    bytes0 = pts * (B_SWEEP * nsweep0 + 2 * B_COARSE_PER_FINE)
+    # HBM passes over level 0 per V-cycle: with temporal blocking every pass is two sweeps except the
+    # interpolation-fused first post-sweep and an odd leftover (pre 12 -> 6 pairs; post 1 + 11 -> 1 + 5 + 1)
     fusion0 = a.fusion or mg.MG_FUSION_FULL
+    if a.tb:
+        post_rest = a.post - (1 if fusion0 == mg.MG_FUSION_FULL else 0)
+        npass0 = (a.pre + 1) // 2 + (1 if fusion0 == mg.MG_FUSION_FULL else 0) + (post_rest + 1) // 2
+    else:
+        npass0 = nsweep0
+    launch_ms = sweep0_ms / npass0
+    # algorithmic bytes of the level-0 passes of one V-cycle (24 B/pt each: read x, b; write x'),
+    # + 1 B/pt for the fused restriction output and the fused interpolation input
+    pts = n**3
+    bytes0 = pts * (B_SWEEP * npass0 + 2 * B_COARSE_PER_FINE)
     if fusion0 != mg.MG_FUSION_FULL:
-        bytes0 = pts * (B_SWEEP * (nsweep0 - 1) + B_SWEEP_R)
+        bytes0 = pts * (B_SWEEP * (npass0 - 1) + B_SWEEP_R)
     achieved = bytes0 / (sweep0_ms / 1e3) / 1e9
+    # the same level-0 work expressed as one-sweep-per-pass traffic (what the sweeps would move unblocked)
+    sweep_equiv = pts * (B_SWEEP * nsweep0 + 2 * B_COARSE_PER_FINE) / (sweep0_ms / 1e3) / 1e9
     peak, peak_src = measured_peaks()
     traffic = ncu_traffic(n)
     levels = []
@@ -304,7 +315,7 @@ def main():
         d = {"level": l, "n": nl, "ms": {k: round(v / ninst, 4) for k, v in zip(mg.OP_NAMES, row) if v > 0}}
         if row[0] > 0 and l < a.levels - 1:
             lb = nl**3 * (B_SWEEP * (a.pre + a.post) + (2 if fusion0 == mg.MG_FUSION_FULL else 8) * B_COARSE_PER_FINE)
-            d["sweep_gbs_algorithmic"] = round(lb / (row[0] / ninst / 1e3) / 1e9, 1)
+            d["sweep_equivalent_gbs"] = round(lb / (row[0] / ninst / 1e3) / 1e9, 1)  # 24 B/pt per sweep
         levels.append(d)
 
     # ---- e2e: public API with host buffers (H2D of b, V-cycle, D2H of the norm) per step
@@ -342,13 +353,17 @@ def main():
                        "fusion": "auto(full)" if not a.fusion else a.fusion,
                        "ca_period": a.ca_period or "auto(8)", "ghost_mode": "all" if a.ghost_all else "auto",
                        "cuda_graph": not a.no_graph, "overlap": not a.no_overlap,
+                       "temporal_blocking": bool(a.tb),
                        "l2": "no flush: every level-0 field is 1 GiB > 126 MB L2 (inputs larger than L2)",
                        "parallelism": f"3D domain decomposition {pg[0]}x{pg[1]}x{pg[2]}"},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic,
-                         "kernel": "level-0 fused sweeps (sweep_col_kernel streaming + the interp-fused "
-                                   "sweep_kernel), avg over the 24 level-0 sweeps of a V-cycle",
-                         "launch_ms": launch_ms, "bytes_per_point": bytes0 / pts / nsweep0,
+                         "kernel": ("level-0 passes: sweep2_kernel (two sweeps per pass) + sweep_col_kernel / "
+                                    "interp-fused sweep_kernel" if a.tb else
+                                    "level-0 sweeps: sweep_col_kernel + interp-fused sweep_kernel"),
+                         "passes_per_vcycle": npass0, "launch_ms": launch_ms,
+                         "bytes_per_point_per_pass": bytes0 / pts / npass0,
+                         "sweep_equivalent_gbs": sweep_equiv,
                          "peak_source": peak_src, "frac_of_8TBs": achieved / 8000.0},
             "cpu_baseline": cpu,
             "e2e": e2e,

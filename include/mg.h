@@ -106,7 +106,7 @@ typedef struct {
   int32_t sweep_kernel;          /* 0 = auto (streaming column kernel on levels >= 16384 bricks),
                                     1 = one-brick-per-CTA kernel only, 2 = streaming kernel on every level */
   int32_t temporal_blocking;     /* 1 = two Jacobi sweeps per HBM pass on streaming levels (sweep2.cu,
-                                    bit-identical), 0 = one sweep per pass (default: faster today) */
+                                    bit-identical; default), 0 = one sweep per pass */
   int32_t reserved[5];
   double h0;                     /* finest spacing; <= 0 => 1 / max_d(global N_d) (reading A7) */
 } mg_params;

@@ -578,7 +578,7 @@ void mg_params_default(mg_params* p) {
   p->bottom_smooths = 100;
   p->use_graph = 1;
   p->overlap = 1;
-  p->temporal_blocking = 0;  // see include/mg.h: the two-sweep kernel is correct but not yet faster
+  p->temporal_blocking = 1;
   p->h0 = 0.0;
 }
 

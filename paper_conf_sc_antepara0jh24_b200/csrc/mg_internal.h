@@ -71,7 +71,8 @@ struct LevelLayout {
 };
 
 constexpr int kPairMeta = 11;
-constexpr int64_t kPairCtas = 148 * 3;  // one item stream per resident two-sweep CTA (148 SMs x 3)
+constexpr int kPairCtasPerSm = 4;                   // resident two-sweep CTAs per SM (shared-memory bound)
+constexpr int64_t kPairCtas = 148 * kPairCtasPerSm;  // one item stream per resident two-sweep CTA
 void build_pair_tables(LevelLayout& L, int64_t min_bricks);
 
 constexpr int kColSeg = 16;             // bricks per streamed segment

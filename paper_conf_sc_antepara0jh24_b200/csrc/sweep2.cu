@@ -8,176 +8,151 @@
 //
 // One CTA (4 warps) walks an item stream of z-chain runs (layout.cpp
 // pair_table): [warm-up, bricks..., cool-down] ...  Per item m, lane 0 of each
-// warp stages its share by TMA into a 4-stage shared-memory ring (mbarriers):
+// warp stages its share by TMA into a 3-stage shared-memory ring (mbarriers):
 //   the x0 brick (1D bulk, 4 KiB); 2-cell-deep x0 slabs of the W/E/S/N
 //   neighbours (3D tensor boxes {2,8,8} / {8,2,8}); the b values on those faces
 //   ({2,8,8} / {8,1,8}); the x0 columns of the 4 diagonal neighbours ({2,1,8}).
-// Step m runs, between two CTA barriers,
-//   phase A: x1 of item m on its 512 cells (warp w = planes 2w, 2w+1, register
-//            k-streaming) and -- redundantly -- on the 4 x 64 side-face cells of
-//            its neighbours (warp w = face w), whose x1 the second sweep needs;
-//   phase B: x2 of item m-2 from x1 (its cells, its faces, plane 7 of item m-3,
-//            plane 0 of item m-1), streamed to HBM with r or the restricted
-//            coarse b on the last sweep of a phase;
-// with x1 in a 3-deep shared ring so the phases never touch the same buffer.
-// Shared-memory operand offsets are loop invariants computed once per thread.
-// b of the own cells travels in registers (128-bit loads two items ahead).
+// Warp w owns planes 2w, 2w+1 and walks them in k with planes k-1..k+1 in
+// registers.  Per plane:
+//   * every lane computes x1 of ONE neighbour face cell (lanes 0-7 the W face,
+//     8-15 E, 16-23 S, 24-31 N) -- the redundant ring of x1 the second sweep
+//     needs; in-face neighbours by shuffles, diagonal corner columns at the ends;
+//   * x1 of the warp's own cells (lane = cell pair (2(l&3), l>>2)); face x0 and
+//     face x1 reach the boundary lanes by warp shuffles;
+//   * x1 goes to a 2-deep shared ring; x2 of the PREVIOUS item (phase B) uses it,
+//     the face x1 kept in registers, plane 7 of item m-2 (carry) and plane 0 of
+//     item m, and streams to HBM with r or the restricted coarse b on the last
+//     sweep of a phase.
+// b of the own cells travels in registers (128-bit loads one item ahead).
 #include <cudaTypedefs.h>
 
 #include <cstddef>
+#include <type_traits>
 
 #include "kernels.h"
+#include "mg_internal.h"
 #include "ptx.cuh"
 
 namespace mgb {
 
-constexpr int P2_NST = 4;     // TMA ring: items m, m+1 read; m+2, m+3 in flight
-constexpr int P2_RING = 8;    // metadata ring (items m-3 .. m+4)
+constexpr int P2_NX = 4;      // own-brick x0 ring: items m, m+1 read; m+2, m+3 in flight
+constexpr int P2_NS = 3;      // neighbour-slab ring: items m, m+1 read; m+2 in flight (issued one step
+                              // later than the own brick, so the neighbour CTAs -- walking the
+                              // neighbour columns in lockstep -- have already pulled those bricks to L2)
+constexpr int P2_RING = 8;    // metadata ring
 constexpr int P2_META = 11;   // id, flags, W,E,S,N, SW,NW,SE,NE, parent
 constexpr int P2_WARPS = 4;
 constexpr int P2_THREADS = 32 * P2_WARPS;
 
-struct P2Stage {
-  double x[512];              // x0 of the item brick, cell i + 8j + 64k
+struct P2Slab {
   double xwe[2][8][8][2];     // x0 of the W brick (i = 6,7) / E brick (i = 0,1): [k][j][ii]
   double xsn[2][8][2][8];     // x0 of the S brick (j = 6,7) / N brick (j = 0,1): [k][jj][i]
   double bwe[2][8][8][2];     // b  of the W brick (i = 6,7) / E brick (i = 0,1)
   double bsn[2][8][8];        // b  of the S brick (j = 7) / N brick (j = 0): [k][i]
   double cor[4][8][2];        // x0 columns: SW (i=6,7 j=7), NW (i=6,7 j=0), SE (i=0,1 j=7), NE (i=0,1 j=0)
 };
-static_assert(sizeof(P2Stage) % 128 == 0, "stage must keep TMA destinations 128-byte aligned");
-// the four warps' expect_tx byte counts below add up to the whole stage
-static_assert(sizeof(P2Stage) == (4096 + 1024) + 3 * 1024 + (2048 + 512) + (512 + 512), "stage bytes");
-// operand offsets (in doubles) inside a stage
-constexpr int OX = 0, OXWE = 512, OXSN = 768, OBWE = 1024, OBSN = 1280, OCOR = 1408;
-static_assert(offsetof(P2Stage, xwe) == OXWE * 8 && offsetof(P2Stage, xsn) == OXSN * 8 &&
-                  offsetof(P2Stage, bwe) == OBWE * 8 && offsetof(P2Stage, bsn) == OBSN * 8 &&
-                  offsetof(P2Stage, cor) == OCOR * 8,
-              "stage layout");
-__host__ __device__ constexpr int oxwe(int f, int k, int j, int ii) { return OXWE + 128 * f + 16 * k + 2 * j + ii; }
-__host__ __device__ constexpr int oxsn(int f, int k, int jj, int i) { return OXSN + 128 * f + 16 * k + 8 * jj + i; }
-__host__ __device__ constexpr int obwe(int f, int k, int j, int ii) { return OBWE + 128 * f + 16 * k + 2 * j + ii; }
-__host__ __device__ constexpr int obsn(int f, int k, int i) { return OBSN + 64 * f + 8 * k + i; }
-__host__ __device__ constexpr int ocor(int c, int k, int ii) { return OCOR + 16 * c + 2 * k + ii; }
+static_assert(sizeof(P2Slab) % 128 == 0, "slab stage must keep TMA destinations 128-byte aligned");
+// warps 1-3's expect_tx byte counts below add up to the whole slab stage
+static_assert(sizeof(P2Slab) == 3 * 1024 + 3 * 1024 + (512 + 512 + 512), "slab bytes");
+constexpr int OXWE = 0, OXSN = 256, OBWE = 512, OBSN = 768, OCOR = 896;  // offsets in doubles
+static_assert(offsetof(P2Slab, xwe) == OXWE * 8 && offsetof(P2Slab, xsn) == OXSN * 8 &&
+                  offsetof(P2Slab, bwe) == OBWE * 8 && offsetof(P2Slab, bsn) == OBSN * 8 &&
+                  offsetof(P2Slab, cor) == OCOR * 8,
+              "slab layout");
 
-template <bool RESTRICT>
 struct P2Smem {
-  P2Stage st[P2_NST];
-  double A[3][512];       // x1 of items m-2, m-1, m
-  double F[3][4][64];     // x1 on their side faces: W/E [k][j], S/N [k][i]
-  double cx0[2][64];      // x0 plane 7 of the previous item
-  double cbox[2][4][8];   // x0 plane 7 of the previous item's side-face cells (W/E by j, S/N by i)
-  double cx1[2][64];      // x1 plane 7 of item m-3
-  uint64_t bar[P2_NST];
+  double ownx[P2_NX][512];  // x0 of the item bricks, cell i + 8j + 64k
+  P2Slab sl[P2_NS];
+  double A[2][512];        // x1 of items m-1, m
+  double cx0[2][64];       // x0 plane 7 of the previous item (own cells)
+  double cface[2][32];     // x0 plane 7 of the previous item's face cells (one per face lane)
+  double cx1[2][64];       // x1 plane 7 of item m-2
+  uint64_t bx[P2_NX];      // own-brick ring barriers (1 arrive: warp 0)
+  uint64_t bs[P2_NS];      // slab ring barriers (3 arrives: warps 1-3)
   int meta[P2_RING][12];
 };
 
 __device__ __forceinline__ double2 lds2(const double* p) { return *reinterpret_cast<const double2*>(p); }
 
 template <unsigned FLAGS>
-__global__ void __launch_bounds__(P2_THREADS, 3)
+__global__ void __launch_bounds__(P2_THREADS, kPairCtasPerSm)
     sweep2_kernel(SweepArgs p, PairArgs pa, const __grid_constant__ PairMaps mp) {
   constexpr bool WRITE_R = (FLAGS & SW_WRITE_R) != 0;
   constexpr bool RESTRICT = (FLAGS & SW_RESTRICT) != 0;
+  constexpr unsigned FULL = 0xffffffffu;
   extern __shared__ __align__(128) unsigned char smem_raw[];
-  P2Smem<RESTRICT>& S = *reinterpret_cast<P2Smem<RESTRICT>*>(smem_raw);
+  P2Smem& S = *reinterpret_cast<P2Smem*>(smem_raw);
   const int t = threadIdx.x, w = t >> 5, l = t & 31;
   const int2 cr = pa.ctas[blockIdx.x];
   const int64_t base = cr.x;
   const int cnt = cr.y;
   const double alpha = p.c.alpha, beta = p.c.beta, gamma = p.c.gamma;
+  const uint64_t pol_keep = l2_evict_last(), pol_stream = l2_evict_first();
 
-  // ---- own-cell geometry: planes k0 = 2w, k1 = 2w+1; cell pair (i0, i0+1), row j ----
+  // ---- own-cell role: planes k0 = 2w, k0+1; cell pair (i0, i0+1) of row j ----
   const int i0 = 2 * (l & 3), j = l >> 2;
   const int q = 8 * j + i0;
   const int k0 = 2 * w;
-  const int qs = j > 0 ? q - 8 : q, qn = j < 7 ? q + 8 : q;  // row loads (clamped; unused lanes)
-  // ---- face-cell geometry: warp w = face f; lane = (c8, planes 2kq, 2kq+1) ----
-  const int f = w, c8 = l & 7, kq = l >> 3, fk0 = 2 * kq;
-  int oc[2], ow[2], oe[2], os[2], on[2], ob[2], ocm, ocp;  // stage offsets of the face operands
-#pragma unroll
-  for (int kk = 0; kk < 2; ++kk) {
-    const int k = fk0 + kk;
-    if (f == 0) {  // W brick, i = 7, (j = c8, k)
-      oc[kk] = oxwe(0, k, c8, 1);
-      ow[kk] = oxwe(0, k, c8, 0);
-      oe[kk] = OX + 64 * k + 8 * c8;
-      os[kk] = c8 > 0 ? oxwe(0, k, c8 - 1, 1) : ocor(0, k, 1);
-      on[kk] = c8 < 7 ? oxwe(0, k, c8 + 1, 1) : ocor(1, k, 1);
-      ob[kk] = obwe(0, k, c8, 1);
-    } else if (f == 1) {  // E brick, i = 0
-      oc[kk] = oxwe(1, k, c8, 0);
-      oe[kk] = oxwe(1, k, c8, 1);
-      ow[kk] = OX + 64 * k + 8 * c8 + 7;
-      os[kk] = c8 > 0 ? oxwe(1, k, c8 - 1, 0) : ocor(2, k, 0);
-      on[kk] = c8 < 7 ? oxwe(1, k, c8 + 1, 0) : ocor(3, k, 0);
-      ob[kk] = obwe(1, k, c8, 0);
-    } else if (f == 2) {  // S brick, j = 7, (i = c8, k)
-      oc[kk] = oxsn(0, k, 1, c8);
-      os[kk] = oxsn(0, k, 0, c8);
-      on[kk] = OX + 64 * k + c8;
-      ow[kk] = c8 > 0 ? oxsn(0, k, 1, c8 - 1) : ocor(0, k, 1);
-      oe[kk] = c8 < 7 ? oxsn(0, k, 1, c8 + 1) : ocor(2, k, 0);
-      ob[kk] = obsn(0, k, c8);
-    } else {  // N brick, j = 0
-      oc[kk] = oxsn(1, k, 0, c8);
-      on[kk] = oxsn(1, k, 1, c8);
-      os[kk] = OX + 64 * k + 56 + c8;
-      ow[kk] = c8 > 0 ? oxsn(1, k, 0, c8 - 1) : ocor(1, k, 1);
-      oe[kk] = c8 < 7 ? oxsn(1, k, 0, c8 + 1) : ocor(3, k, 0);
-      ob[kk] = obsn(1, k, c8);
-    }
+  const int qs = j > 0 ? q - 8 : q, qn = j < 7 ? q + 8 : q;  // row loads (clamped for the face lanes)
+  const bool isW = i0 == 0, isE = i0 == 6, isS = j == 0, isN = j == 7;
+  const int sWE = isW ? j : 8 + j;                     // face lane holding my W / E face cell
+  const int sSN = (isS ? 16 : 24) + i0;                // face lanes holding my S / N face pair
+  // ---- face-cell role: face ff (0 W, 1 E, 2 S, 3 N), in-face coordinate c8 ----
+  const int ff = l >> 3, c8 = l & 7;
+  int oc0, oo0, ob0, obk, olo, ohi;  // stage offsets (doubles) at plane 0; slabs step 16 / plane
+  if (ff == 0) {         // W brick, cell (7, c8, k): o = (6, c8), own = (0, c8) of my brick
+    oc0 = OXWE + 2 * c8 + 1, oo0 = OXWE + 2 * c8, ob0 = OBWE + 2 * c8 + 1, obk = 16;
+    olo = OCOR + 0 * 16 + 1, ohi = OCOR + 1 * 16 + 1;  // j-1 -> SW (i=7), j+1 -> NW (i=7)
+  } else if (ff == 1) {  // E brick, cell (0, c8, k): o = (1, c8), own = (7, c8)
+    oc0 = OXWE + 128 + 2 * c8, oo0 = OXWE + 128 + 2 * c8 + 1, ob0 = OBWE + 128 + 2 * c8, obk = 16;
+    olo = OCOR + 2 * 16 + 0, ohi = OCOR + 3 * 16 + 0;  // SE (i=0), NE (i=0)
+  } else if (ff == 2) {  // S brick, cell (c8, 7, k): o = (c8, 6), own = (c8, 0)
+    oc0 = OXSN + 8 + c8, oo0 = OXSN + c8, ob0 = OBSN + c8, obk = 8;
+    olo = OCOR + 0 * 16 + 1, ohi = OCOR + 2 * 16 + 0;  // i-1 -> SW (i=7), i+1 -> SE (i=0)
+  } else {               // N brick, cell (c8, 0, k): o = (c8, 1), own = (c8, 7)
+    oc0 = OXSN + 128 + c8, oo0 = OXSN + 128 + 8 + c8, ob0 = OBSN + 64 + c8, obk = 8;
+    olo = OCOR + 1 * 16 + 1, ohi = OCOR + 3 * 16 + 0;  // NW (i=7), NE (i=0)
   }
-  {
-    const int km = fk0 - 1, kp = fk0 + 2;  // c(k) at planes fk0-1 (kq > 0) / fk0+2 (kq < 3, else next stage plane 0)
-    const int kpp = kq < 3 ? kp : 0;
-    if (f == 0) {
-      ocm = oxwe(0, km < 0 ? 0 : km, c8, 1);
-      ocp = oxwe(0, kpp, c8, 1);
-    } else if (f == 1) {
-      ocm = oxwe(1, km < 0 ? 0 : km, c8, 0);
-      ocp = oxwe(1, kpp, c8, 0);
-    } else if (f == 2) {
-      ocm = oxsn(0, km < 0 ? 0 : km, 1, c8);
-      ocp = oxsn(0, kpp, 1, c8);
-    } else {
-      ocm = oxsn(1, km < 0 ? 0 : km, 0, c8);
-      ocp = oxsn(1, kpp, 0, c8);
-    }
-  }
+  // the own-brick cell next to the face cell lives in lane srcOwn's register pair
+  const int srcOwn = ff == 0 ? 4 * c8 : ff == 1 ? 4 * c8 + 3 : ff == 2 ? (c8 >> 1) : 28 + (c8 >> 1);
+  const bool ownY = ff == 1 || (ff >= 2 && (c8 & 1));
 
   for (int e = t; e < P2_RING * P2_META; e += P2_THREADS) {
     const int it = e / P2_META, fl = e % P2_META;
     if (it < cnt) S.meta[it][fl] = pa.meta[(base + it) * P2_META + fl];
   }
   if (t == 0) {
-    for (int s = 0; s < P2_NST; ++s) mbar_init(&S.bar[s], P2_WARPS);  // one expect_tx arrive per warp
+    for (int s = 0; s < P2_NX; ++s) mbar_init(&S.bx[s], 1);
+    for (int s = 0; s < P2_NS; ++s) mbar_init(&S.bs[s], P2_WARPS - 1);
     mbar_fence_init();
   }
   __syncthreads();
 
-  // lane 0 of every warp issues its share of item m's copies
-  auto issue = [&](int m) {
-    const int s = m % P2_NST;
+  // lane 0 of warp 0 stages item m's own brick; lanes 0 of warps 1-3 its neighbour slabs
+  auto issue_x = [&](int m) {
+    const int s = m % P2_NX;
+    mbar_expect_tx(&S.bx[s], 4096);
+    // evict_last: the neighbour CTAs read this brick's faces shortly after
+    tma_load_1d_hint(S.ownx[s], p.x + (int64_t)S.meta[m % P2_RING][0] * 512, 4096, &S.bx[s], pol_keep);
+  };
+  auto issue_slab = [&](int m) {
+    const int s = m % P2_NS;
     const int* M = S.meta[m % P2_RING];
-    P2Stage& G = S.st[s];
-    uint64_t* bar = &S.bar[s];
-    if (w == 0) {
-      mbar_expect_tx(bar, 4096 + 1024);
-      tma_load_1d(G.x, p.x + (int64_t)M[0] * 512, 4096, bar);
-      tma_load_3d(G.xwe[0], &mp.xwe, 6, 0, M[2] * 8, bar);  // W: i = 6,7
-    } else if (w == 1) {
+    P2Slab& G = S.sl[s];
+    uint64_t* bar = &S.bs[s];
+    if (w == 1) {
       mbar_expect_tx(bar, 3 * 1024);
+      tma_load_3d(G.xwe[0], &mp.xwe, 6, 0, M[2] * 8, bar);  // W: i = 6,7
       tma_load_3d(G.xwe[1], &mp.xwe, 0, 0, M[3] * 8, bar);  // E: i = 0,1
       tma_load_3d(G.xsn[0], &mp.xsn, 0, 6, M[4] * 8, bar);  // S: j = 6,7
-      tma_load_3d(G.xsn[1], &mp.xsn, 0, 0, M[5] * 8, bar);  // N: j = 0,1
     } else if (w == 2) {
-      mbar_expect_tx(bar, 2048 + 512);
+      mbar_expect_tx(bar, 3 * 1024);
+      tma_load_3d(G.xsn[1], &mp.xsn, 0, 0, M[5] * 8, bar);  // N: j = 0,1
       tma_load_3d(G.bwe[0], &mp.bwe, 6, 0, M[2] * 8, bar);
       tma_load_3d(G.bwe[1], &mp.bwe, 0, 0, M[3] * 8, bar);
-      tma_load_3d(G.bsn[0], &mp.bsn, 0, 7, M[4] * 8, bar);
     } else {
-      mbar_expect_tx(bar, 512 + 512);
+      mbar_expect_tx(bar, 512 + 512 + 512);
+      tma_load_3d(G.bsn[0], &mp.bsn, 0, 7, M[4] * 8, bar);
       tma_load_3d(G.bsn[1], &mp.bsn, 0, 0, M[5] * 8, bar);
       tma_load_3d(G.cor[0], &mp.xcor, 6, 7, M[6] * 8, bar);  // SW: (i = 7, j = 7)
       tma_load_3d(G.cor[1], &mp.xcor, 6, 0, M[7] * 8, bar);  // NW: (i = 7, j = 0)
@@ -185,27 +160,30 @@ __global__ void __launch_bounds__(P2_THREADS, 3)
       tma_load_3d(G.cor[3], &mp.xcor, 0, 0, M[9] * 8, bar);  // NE: (i = 0, j = 0)
     }
   };
-  // b of this thread's own cells (planes k0, k1) of item m
   auto load_b = [&](int m, double2& v0, double2& v1) {
     const double* bp = p.b + (int64_t)S.meta[m % P2_RING][0] * 512 + 64 * k0 + q;
-    v0 = ld_stream2(bp);
-    v1 = ld_stream2(bp + 64);
+    v0 = ld_hint2(bp, pol_keep);  // the neighbours' b-face slabs reuse these lines from L2
+    v1 = ld_hint2(bp + 64, pol_keep);
   };
 
-  if (l == 0)
-    for (int m = 0; m < 3 && m < cnt; ++m) issue(m);
-  double2 bm2a = make_double2(0.0, 0.0), bm2b = bm2a, bm1a = bm2a, bm1b = bm2a, b0a, b0b, b1a, b1b;
-  load_b(0, b0a, b0b);
-  if (cnt > 1)
-    load_b(1, b1a, b1b);
-  else
-    b1a = b0a, b1b = b0b;
+  if (l == 0) {
+    if (w == 0)
+      for (int m = 0; m < P2_NX - 1 && m < cnt; ++m) issue_x(m);
+    else
+      for (int m = 0; m < P2_NS - 1 && m < cnt; ++m) issue_slab(m);
+  }
+  // registers indexed by item parity (the walk is unrolled by two, so every index is constant):
+  //   bq[par]  b of the own cells (planes k0, k0+1) of the item with that parity
+  //   fweq/fsnq[par]  face x1 delivered to this lane (W/E value, S/N pair) per plane
+  double2 bq[2][2];
+  double fweq[2][2];
+  double2 fsnq[2][2];
+  load_b(0, bq[0][0], bq[0][1]);
+  bq[1][0] = bq[1][1] = make_double2(0.0, 0.0);
   int mreg = 0;
-  int a_cur = 0;  // m % 3 (x1 ring slot of item m)
 
-  for (int m = 0; m <= cnt + 1; ++m) {
-    const int a_m1 = a_cur == 0 ? 2 : a_cur - 1, a_m2 = a_m1 == 0 ? 2 : a_m1 - 1;
-    const int cur = m & 1, prv = cur ^ 1;
+  auto step = [&](const int m, auto par) {
+    constexpr int cur = decltype(par)::value, prv = cur ^ 1;
     // metadata ring holds items m-3 .. m+3 during step m: store item m+4 (loaded last step)
     // into the slot of item m-4, then load item m+5 (fields spread over the warps)
     if (l < 3 && w + 4 * l < P2_META) {
@@ -213,86 +191,105 @@ __global__ void __launch_bounds__(P2_THREADS, 3)
       if (m >= 1 && m + 4 < cnt) S.meta[(m + 4) % P2_RING][fl] = mreg;
       if (m + 5 < cnt) mreg = pa.meta[(base + m + 5) * P2_META + fl];
     }
-    // stage of item m+3 = stage of item m-1, unread since the barrier that ended step m-1
-    if (l == 0 && m + 3 < cnt) {
+    // the ring slots of items m+NX-1 / m+NS-1 are item m-1's, unread since the barrier ending step m-1
+    if (l == 0) {
       fence_proxy_async();
-      issue(m + 3);
+      if (w == 0) {
+        if (m + P2_NX - 1 < cnt) issue_x(m + P2_NX - 1);
+      } else if (m + P2_NS - 1 < cnt) {
+        issue_slab(m + P2_NS - 1);
+      }
     }
-    double2 b2a = b1a, b2b = b1b;
-    if (m + 2 < cnt) load_b(m + 2, b2a, b2b);
+    double2 bna = bq[cur][0], bnb = bq[cur][1];  // b of item m+1
+    if (m + 1 < cnt) load_b(m + 1, bna, bnb);
 
     // ---------------- phase A: x1 of item m ----------------
-    if (m < cnt) {
-      mbar_wait(&S.bar[m % P2_NST], (uint32_t)((m / P2_NST) & 1));
-      if (m + 1 < cnt) mbar_wait(&S.bar[(m + 1) % P2_NST], (uint32_t)(((m + 1) / P2_NST) & 1));
-      const double* G = reinterpret_cast<const double*>(&S.st[m % P2_NST]);
-      const double* N = reinterpret_cast<const double*>(&S.st[(m + 1) % P2_NST]);  // stale if no next item
-      double* Aw = S.A[a_cur];
-      {  // own cells, planes k0, k1 (k-streaming in registers)
-        const double2 xm = w > 0 ? lds2(G + 64 * (k0 - 1) + q) : lds2(S.cx0[prv] + q);
-        const double2 x0 = lds2(G + 64 * k0 + q);
-        const double2 x1 = lds2(G + 64 * (k0 + 1) + q);
-        const double2 x2 = w < P2_WARPS - 1 ? lds2(G + 64 * (k0 + 2) + q) : lds2(N + q);
-#pragma unroll
-        for (int kk = 0; kk < 2; ++kk) {
-          const int k = k0 + kk;
-          const double2 xc = kk ? x1 : x0, xb = kk ? x0 : xm, xt = kk ? x2 : x1;
-          const double2 bb = kk ? b0b : b0a;
-          const double2 rs_ = lds2(G + 64 * k + qs), rn_ = lds2(G + 64 * k + qn);
-          const double fw = G[oxwe(0, k, j, 1)], fe = G[oxwe(1, k, j, 0)];
-          const double2 fs = lds2(G + oxsn(0, k, 1, i0)), fn = lds2(G + oxsn(1, k, 0, i0));
-          const double wl = __shfl_up_sync(0xffffffffu, xc.y, 1);
-          const double er = __shfl_down_sync(0xffffffffu, xc.x, 1);
-          const double wv = i0 > 0 ? wl : fw, ev = i0 < 6 ? er : fe;
-          const double2 sv = j > 0 ? rs_ : fs, nv = j < 7 ? rn_ : fn;
-          const double a0 = stencil_a(xc.x, wv, xc.y, sv.x, nv.x, xb.x, xt.x, alpha, beta);
-          const double a1 = stencil_a(xc.y, xc.x, ev, sv.y, nv.y, xb.y, xt.y, alpha, beta);
-          double2 y;
-          y.x = DADD(xc.x, DMUL(gamma, DSUB(a0, bb.x)));
-          y.y = DADD(xc.y, DMUL(gamma, DSUB(a1, bb.y)));
-          *reinterpret_cast<double2*>(Aw + 64 * k + q) = y;
-        }
-        if (w == P2_WARPS - 1) *reinterpret_cast<double2*>(S.cx0[cur] + q) = x1;  // plane 7
+    {
+      mbar_wait(&S.bx[m % P2_NX], (uint32_t)((m / P2_NX) & 1));
+      mbar_wait(&S.bs[m % P2_NS], (uint32_t)((m / P2_NS) & 1));
+      if (m + 1 < cnt) {
+        mbar_wait(&S.bx[(m + 1) % P2_NX], (uint32_t)(((m + 1) / P2_NX) & 1));
+        mbar_wait(&S.bs[(m + 1) % P2_NS], (uint32_t)(((m + 1) / P2_NS) & 1));
       }
-      {  // side-face cells of the neighbours: face f = w, planes fk0, fk0+1 at in-face c8
-        const double cm = kq > 0 ? G[ocm] : S.cbox[prv][f][c8];
-        const double c0 = G[oc[0]], c1 = G[oc[1]];
-        const double cp = kq < 3 ? G[ocp] : N[ocp];
+      const double* X = S.ownx[m % P2_NX];
+      const double* NX = S.ownx[(m + 1) % P2_NX];  // stale if no next item (feeds only unused cells)
+      const double* G = reinterpret_cast<const double*>(&S.sl[m % P2_NS]);
+      const double* N = reinterpret_cast<const double*>(&S.sl[(m + 1) % P2_NS]);
+      const double2 xm = w > 0 ? lds2(X + 64 * (k0 - 1) + q) : lds2(S.cx0[prv] + q);
+      const double2 x0 = lds2(X + 64 * k0 + q);
+      const double2 x1 = lds2(X + 64 * (k0 + 1) + q);
+      const double2 x2 = w < P2_WARPS - 1 ? lds2(X + 64 * (k0 + 2) + q) : lds2(NX + q);
+      // face lane: its face cell's x0 on planes k0-1 .. k0+2
+      const double cm = w > 0 ? G[oc0 + 16 * (k0 - 1)] : S.cface[prv][l];
+      const double cf0 = G[oc0 + 16 * k0], cf1 = G[oc0 + 16 * (k0 + 1)];
+      const double cp = w < P2_WARPS - 1 ? G[oc0 + 16 * (k0 + 2)] : N[oc0];
+      double* Aw = S.A[cur];
 #pragma unroll
-        for (int kk = 0; kk < 2; ++kk) {
-          const double c = kk ? c1 : c0, bt = kk ? c0 : cm, tp = kk ? cp : c1;
-          const double av = stencil_a(c, G[ow[kk]], G[oe[kk]], G[os[kk]], G[on[kk]], bt, tp, alpha, beta);
-          S.F[a_cur][f][8 * (fk0 + kk) + c8] = DADD(c, DMUL(gamma, DSUB(av, G[ob[kk]])));
-        }
-        if (kq == 3) S.cbox[cur][f][c8] = c1;  // plane 7
+      for (int kk = 0; kk < 2; ++kk) {
+        const int k = k0 + kk;
+        const double2 xc = kk ? x1 : x0, xb = kk ? x0 : xm, xt = kk ? x2 : x1;
+        // -- x1 of this lane's face cell.  Its W/E (or S/N) neighbour pair is {o, own} and the
+        //    other in-plane pair {lo, hi}; IEEE addition is commutative, so
+        //    ((o+own)+(lo+hi))+(b+t) is bit-identical to the canonical ((w+e)+(s+n))+(b+t).
+        const double c = kk ? cf1 : cf0, bt = kk ? cf0 : cm, tp = kk ? cp : cf1;
+        const double o = G[oo0 + 16 * k];
+        const double bf = G[ob0 + obk * k];
+        const double ownx = __shfl_sync(FULL, xc.x, srcOwn), owny = __shfl_sync(FULL, xc.y, srcOwn);
+        const double own = ownY ? owny : ownx;
+        const double up = __shfl_up_sync(FULL, c, 1), dn = __shfl_down_sync(FULL, c, 1);
+        const double lo = c8 > 0 ? up : G[olo + 2 * k];
+        const double hi = c8 < 7 ? dn : G[ohi + 2 * k];
+        const double sum = DADD(DADD(DADD(o, own), DADD(lo, hi)), DADD(bt, tp));
+        const double af = DADD(DMUL(alpha, c), DMUL(beta, sum));
+        const double fx1 = DADD(c, DMUL(gamma, DSUB(af, bf)));
+        // -- deliver face x0 / face x1 to the own lanes next to the faces
+        const double vwe = __shfl_sync(FULL, c, sWE);
+        double2 vsn;
+        vsn.x = __shfl_sync(FULL, c, sSN);
+        vsn.y = __shfl_sync(FULL, c, sSN + 1);
+        fweq[cur][kk] = __shfl_sync(FULL, fx1, sWE);
+        fsnq[cur][kk].x = __shfl_sync(FULL, fx1, sSN);
+        fsnq[cur][kk].y = __shfl_sync(FULL, fx1, sSN + 1);
+        // -- x1 of the own cells
+        const double2 bb = bq[cur][kk];
+        const double2 rs_ = lds2(X + 64 * k + qs), rn_ = lds2(X + 64 * k + qn);
+        const double wl = __shfl_up_sync(FULL, xc.y, 1), er = __shfl_down_sync(FULL, xc.x, 1);
+        const double wo = isW ? vwe : wl, eo = isE ? vwe : er;
+        const double2 so = isS ? vsn : rs_, no = isN ? vsn : rn_;
+        const double a0 = stencil_a(xc.x, wo, xc.y, so.x, no.x, xb.x, xt.x, alpha, beta);
+        const double a1 = stencil_a(xc.y, xc.x, eo, so.y, no.y, xb.y, xt.y, alpha, beta);
+        double2 y;
+        y.x = DADD(xc.x, DMUL(gamma, DSUB(a0, bb.x)));
+        y.y = DADD(xc.y, DMUL(gamma, DSUB(a1, bb.y)));
+        *reinterpret_cast<double2*>(Aw + 64 * k + q) = y;
+      }
+      if (w == P2_WARPS - 1) {  // plane 7 carries for the next item's plane 0
+        *reinterpret_cast<double2*>(S.cx0[cur] + q) = x1;
+        S.cface[cur][l] = cf1;
       }
     }
+    __syncthreads();  // x1 of item m (plane 0 for phase B) and the carries are visible
 
-    // ---------------- phase B: x2 of item m-2 ----------------
-    if (m >= 2 && m <= cnt) {
-      const double* P = S.A[a_m2];
-      const double2 x1v = lds2(P + 64 * (k0 + 1) + q);
-      if (w == P2_WARPS - 1) *reinterpret_cast<double2*>(S.cx1[cur] + q) = x1v;  // x1 plane 7 of item m-2
-      const bool emit = (S.meta[(m - 1) % P2_RING][1] & 1) != 0;  // item m-2 is a range brick
+    // ---------------- phase B: x2 of item m-1 ----------------
+    if (m >= 1) {
+      const double* P = S.A[prv];
+      const double2 y0 = lds2(P + 64 * k0 + q), y1 = lds2(P + 64 * (k0 + 1) + q);
+      if (w == P2_WARPS - 1) *reinterpret_cast<double2*>(S.cx1[prv] + q) = y1;  // x1 plane 7 of item m-1
+      const bool emit = (S.meta[m % P2_RING][1] & 1) != 0;  // item m-1 is a range brick
       if (emit) {
-        const double2 xm = w > 0 ? lds2(P + 64 * (k0 - 1) + q) : lds2(S.cx1[prv] + q);  // item m-3 plane 7
-        const double2 x0v = lds2(P + 64 * k0 + q);
-        const double2 x2v = w < P2_WARPS - 1 ? lds2(P + 64 * (k0 + 2) + q) : lds2(S.A[a_m1] + q);  // item m-1
-        const double* Fb = &S.F[a_m2][0][0];
-        const int64_t g = (int64_t)S.meta[(m - 2) % P2_RING][0] * 512 + q;
+        const double2 ym = w > 0 ? lds2(P + 64 * (k0 - 1) + q) : lds2(S.cx1[cur] + q);  // item m-2 plane 7
+        const double2 yp = w < P2_WARPS - 1 ? lds2(P + 64 * (k0 + 2) + q) : lds2(S.A[cur] + q);  // item m
+        const int64_t g = (int64_t)S.meta[(m - 1) % P2_RING][0] * 512 + q;
         double rsum[2];
 #pragma unroll
         for (int kk = 0; kk < 2; ++kk) {
           const int k = k0 + kk;
-          const double2 xc = kk ? x1v : x0v, xb = kk ? x0v : xm, xt = kk ? x2v : x1v;
-          const double2 bb = kk ? bm2b : bm2a;
+          const double2 xc = kk ? y1 : y0, xb = kk ? y0 : ym, xt = kk ? yp : y1;
+          const double2 bb = bq[prv][kk];
           const double2 rs_ = lds2(P + 64 * k + qs), rn_ = lds2(P + 64 * k + qn);
-          const double fw = Fb[8 * k + j], fe = Fb[64 + 8 * k + j];
-          const double2 fs = lds2(Fb + 128 + 8 * k + i0), fn = lds2(Fb + 192 + 8 * k + i0);
-          const double wl = __shfl_up_sync(0xffffffffu, xc.y, 1);
-          const double er = __shfl_down_sync(0xffffffffu, xc.x, 1);
-          const double wv = i0 > 0 ? wl : fw, ev = i0 < 6 ? er : fe;
-          const double2 sv = j > 0 ? rs_ : fs, nv = j < 7 ? rn_ : fn;
+          const double wl = __shfl_up_sync(FULL, xc.y, 1), er = __shfl_down_sync(FULL, xc.x, 1);
+          const double wv = isW ? fweq[prv][kk] : wl, ev = isE ? fweq[prv][kk] : er;
+          const double2 sv = isS ? fsnq[prv][kk] : rs_, nv = isN ? fsnq[prv][kk] : rn_;
           const double a0 = stencil_a(xc.x, wv, xc.y, sv.x, nv.x, xb.x, xt.x, alpha, beta);
           const double a1 = stencil_a(xc.y, xc.x, ev, sv.y, nv.y, xb.y, xt.y, alpha, beta);
           double2 y, rv;
@@ -300,18 +297,18 @@ __global__ void __launch_bounds__(P2_THREADS, 3)
           y.y = DADD(xc.y, DMUL(gamma, DSUB(a1, bb.y)));
           rv.x = DSUB(bb.x, a0);
           rv.y = DSUB(bb.y, a1);
-          st_stream2(p.xo + g + 64 * k, y);
-          if (WRITE_R) st_stream2(p.r + g + 64 * k, rv);
+          st_hint2(p.xo + g + 64 * k, y, pol_stream);  // never re-read by this pass
+          if (WRITE_R) st_hint2(p.r + g + 64 * k, rv, pol_stream);
           rsum[kk] = DADD(rv.x, rv.y);  // r(2I,.,.) + r(2I+1,.,.) of this row and plane
         }
         if (RESTRICT) {
           // coarse cell (I, J, K) = (l&3, j/2, w): its 8 fine cells are this lane's and lane+4's
           // pairs on planes 2w, 2w+1 -> canonical order ((r000+r100)+(r010+r110))+((r001+r101)+(r011+r111))
-          const double s0n = __shfl_down_sync(0xffffffffu, rsum[0], 4);
-          const double s1n = __shfl_down_sync(0xffffffffu, rsum[1], 4);
+          const double s0n = __shfl_down_sync(FULL, rsum[0], 4);
+          const double s1n = __shfl_down_sync(FULL, rsum[1], 4);
           if ((j & 1) == 0) {
             const double v = DMUL(0.125, DADD(DADD(rsum[0], s0n), DADD(rsum[1], s1n)));
-            const int pr = S.meta[(m - 2) % P2_RING][10];
+            const int pr = S.meta[(m - 1) % P2_RING][10];
             const int oct = pr & 7;
             const int ox = oct & 1, oy = (oct >> 1) & 1, oz = oct >> 2;
             p.bc[(int64_t)(pr >> 3) * 512 + (4 * ox + (l & 3)) + 8 * (4 * oy + (j >> 1)) + 64 * (4 * oz + w)] = v;
@@ -319,12 +316,15 @@ __global__ void __launch_bounds__(P2_THREADS, 3)
         }
       }
     }
-    __syncthreads();
-    bm2a = bm1a, bm2b = bm1b;
-    bm1a = b0a, bm1b = b0b;
-    b0a = b1a, b0b = b1b;
-    b1a = b2a, b1b = b2b;
-    a_cur = a_cur == 2 ? 0 : a_cur + 1;
+    __syncthreads();  // x1 ring slot of item m-1 and the carries may be overwritten next step
+    bq[prv][0] = bna;  // item m+1 has parity prv; item m-1's b is consumed
+    bq[prv][1] = bnb;
+  };
+
+  // the last item is always a cool-down brick: its x2 is not wanted, so step cnt-1 ends the walk
+  for (int m = 0; m < cnt; m += 2) {
+    step(m, std::integral_constant<int, 0>{});
+    if (m + 1 < cnt) step(m + 1, std::integral_constant<int, 1>{});
   }
 }
 
@@ -337,10 +337,11 @@ cudaError_t launch_sweep2(const SweepArgs& a, const PairArgs& pa, const PairMaps
                           cudaStream_t s) {
   if (pa.nctas <= 0) return cudaSuccess;
   const unsigned g = (unsigned)pa.nctas;
+  const size_t sm = sizeof(P2Smem);
   switch (flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP | SW_ZERO_X)) {
-    case 0: sweep2_kernel<0><<<g, P2_THREADS, sizeof(P2Smem<false>), s>>>(a, pa, pm); break;
-    case SW_WRITE_R: sweep2_kernel<SW_WRITE_R><<<g, P2_THREADS, sizeof(P2Smem<false>), s>>>(a, pa, pm); break;
-    case SW_RESTRICT: sweep2_kernel<SW_RESTRICT><<<g, P2_THREADS, sizeof(P2Smem<true>), s>>>(a, pa, pm); break;
+    case 0: sweep2_kernel<0><<<g, P2_THREADS, sm, s>>>(a, pa, pm); break;
+    case SW_WRITE_R: sweep2_kernel<SW_WRITE_R><<<g, P2_THREADS, sm, s>>>(a, pa, pm); break;
+    case SW_RESTRICT: sweep2_kernel<SW_RESTRICT><<<g, P2_THREADS, sm, s>>>(a, pa, pm); break;
     default: return cudaErrorInvalidValue;
   }
   return cudaGetLastError();
@@ -349,9 +350,8 @@ cudaError_t launch_sweep2(const SweepArgs& a, const PairArgs& pa, const PairMaps
 cudaError_t pair_kernels_init() {
   const void* k[3] = {(const void*)sweep2_kernel<0>, (const void*)sweep2_kernel<SW_WRITE_R>,
                       (const void*)sweep2_kernel<SW_RESTRICT>};
-  const int sm[3] = {(int)sizeof(P2Smem<false>), (int)sizeof(P2Smem<false>), (int)sizeof(P2Smem<true>)};
   for (int i = 0; i < 3; ++i) {
-    cudaError_t e = cudaFuncSetAttribute(k[i], cudaFuncAttributeMaxDynamicSharedMemorySize, sm[i]);
+    cudaError_t e = cudaFuncSetAttribute(k[i], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(P2Smem));
     if (e != cudaSuccess) return e;
     e = cudaFuncSetAttribute(k[i], cudaFuncAttributePreferredSharedMemoryCarveout, 100);
     if (e != cudaSuccess) return e;
