@@ -93,7 +93,6 @@ __global__ void __launch_bounds__(P2_THREADS, kPairCtasPerSm)
   const int i0 = 2 * (l & 3), j = l >> 2;
   const int q = 8 * j + i0;
   const int k0 = 2 * w;
-  const int qs = j > 0 ? q - 8 : q, qn = j < 7 ? q + 8 : q;  // row loads (clamped for the face lanes)
   const bool isW = i0 == 0, isE = i0 == 6, isS = j == 0, isN = j == 7;
   const int sWE = isW ? j : 8 + j;                     // face lane holding my W / E face cell
   const int sSN = (isS ? 16 : 24) + i0;                // face lanes holding my S / N face pair
@@ -252,7 +251,9 @@ __global__ void __launch_bounds__(P2_THREADS, kPairCtasPerSm)
         fsnq[cur][kk].y = __shfl_sync(FULL, fx1, sSN + 1);
         // -- x1 of the own cells
         const double2 bb = bq[cur][kk];
-        const double2 rs_ = lds2(X + 64 * k + qs), rn_ = lds2(X + 64 * k + qn);
+        double2 rs_, rn_;  // rows j-1, j+1 of the plane live in lanes l-4, l+4
+        rs_.x = __shfl_up_sync(FULL, xc.x, 4), rs_.y = __shfl_up_sync(FULL, xc.y, 4);
+        rn_.x = __shfl_down_sync(FULL, xc.x, 4), rn_.y = __shfl_down_sync(FULL, xc.y, 4);
         const double wl = __shfl_up_sync(FULL, xc.y, 1), er = __shfl_down_sync(FULL, xc.x, 1);
         const double wo = isW ? vwe : wl, eo = isE ? vwe : er;
         const double2 so = isS ? vsn : rs_, no = isN ? vsn : rn_;
@@ -286,7 +287,9 @@ __global__ void __launch_bounds__(P2_THREADS, kPairCtasPerSm)
           const int k = k0 + kk;
           const double2 xc = kk ? y1 : y0, xb = kk ? y0 : ym, xt = kk ? yp : y1;
           const double2 bb = bq[prv][kk];
-          const double2 rs_ = lds2(P + 64 * k + qs), rn_ = lds2(P + 64 * k + qn);
+          double2 rs_, rn_;
+          rs_.x = __shfl_up_sync(FULL, xc.x, 4), rs_.y = __shfl_up_sync(FULL, xc.y, 4);
+          rn_.x = __shfl_down_sync(FULL, xc.x, 4), rn_.y = __shfl_down_sync(FULL, xc.y, 4);
           const double wl = __shfl_up_sync(FULL, xc.y, 1), er = __shfl_down_sync(FULL, xc.x, 1);
           const double wv = isW ? fweq[prv][kk] : wl, ev = isE ? fweq[prv][kk] : er;
           const double2 sv = isS ? fsnq[prv][kk] : rs_, nv = isN ? fsnq[prv][kk] : rn_;
