@@ -34,8 +34,9 @@
  *     NCCL communicator and frees them in mg_destroy / mg_group_destroy.
  *   - Collective calls (mg_setup, mg_set_rhs, mg_set_solution, mg_vcycle,
  *     mg_residual_norm, mg_solve) must be made by all ranks in the same order.
- *   - mg_vcycle is stream-ordered and never synchronises the host; only
- *     mg_residual_norm, mg_solve and the *_host copies synchronise.
+ *   - mg_vcycle, mg_set_rhs_host and mg_residual_norm_async are stream-ordered
+ *     and never synchronise the host; mg_residual_norm, mg_residual_norm_wait,
+ *     mg_solve and mg_get_solution_host synchronise.
  *   - One context per process and GPU; not thread-safe.
  *   - There is no CPU fallback: without a usable CUDA device mg_setup fails
  *     with MG_ERR_CUDA.
@@ -131,7 +132,13 @@ mg_status mg_nccl_unique_id(uint8_t out_id[128]);
 mg_status mg_setup(const mg_params* p, int32_t rank, int32_t world_size, const uint8_t* nccl_id,
                    int32_t device, void* cuda_stream, void* workspace, size_t ws_bytes, mg_ctx** out);
 
-/* Right-hand side b of level 0, local lexicographic, device / host. */
+/* Right-hand side b of level 0, local lexicographic, device / host.
+ * mg_set_rhs_host does not block the host: the upload runs on an internal copy
+ * stream into one of two staging fields and overlaps work already enqueued on
+ * the context's stream (e.g. the V-cycle of the previous right-hand side); the
+ * conversion into bricks is ordered on the context's stream.  b_host must not
+ * be modified until the next synchronising call returns; pinned memory gives a
+ * truly asynchronous copy. */
 mg_status mg_set_rhs(mg_ctx* c, const double* b_dev);
 mg_status mg_set_rhs_host(mg_ctx* c, const double* b_host);
 /* Initial guess; NULL => x = 0 (reading A9). */
@@ -145,6 +152,12 @@ mg_status mg_vcycle(mg_ctx* c);
 /* Global max_p |b_p - (A x)_p| at level 0 with a fresh applyOp (Alg 1
  * "maxNormRes").  Collective; synchronises the stream. */
 mg_status mg_residual_norm(mg_ctx* c, double* out_max_abs);
+/* The same split in two: _async enqueues the norm (and its 8-byte read-back)
+ * on the stream and returns; _wait blocks until it is done and returns the
+ * value.  At most one norm may be pending (MG_ERR_STATE otherwise).
+ * mg_residual_norm == _async + _wait. */
+mg_status mg_residual_norm_async(mg_ctx* c);
+mg_status mg_residual_norm_wait(mg_ctx* c, double* out_max_abs);
 
 /* Alg 1: while norm > tol and cycles < max_cycles: V-cycle.
  * Returns MG_NOT_CONVERGED (1) if the cap was hit. */

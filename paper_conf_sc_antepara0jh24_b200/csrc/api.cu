@@ -82,7 +82,12 @@ struct mg_ctx {
   cudaStream_t cap = nullptr;  // private stream the V-cycle graph is captured on (the caller's may be legacy)
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
   std::vector<DevLevel> dl;
-  double* stage = nullptr;
+  double* stage[2] = {nullptr, nullptr};  // host-upload staging fields
+  int stage_k = 0;
+  cudaStream_t h2d = nullptr;              // copy stream of host uploads
+  cudaEvent_t ev_h2d[2] = {nullptr, nullptr}, ev_free[2] = {nullptr, nullptr};
+  cudaEvent_t ev_norm = nullptr;           // completion of the last enqueued residual norm
+  bool norm_pending = false;
   unsigned long long* acc = nullptr;
   double* h_pinned = nullptr;
   ncclComm_t nccl = nullptr;
@@ -182,9 +187,13 @@ size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double**
     d.c = level_coeffs(d.h);
     if (out) (*out)[l] = d;
   }
-  double* st = (double*)take((size_t)lay.lv[0].n_owned * kBV * sizeof(double));
+  // two staging fields for host uploads (double-buffered: the upload of the next right-hand
+  // side overlaps the current V-cycle)
+  for (int k = 0; k < 2; ++k) {
+    double* st = (double*)take((size_t)lay.lv[0].n_owned * kBV * sizeof(double));
+    if (stage) stage[k] = st;
+  }
   unsigned long long* ac = (unsigned long long*)take(256);
-  if (stage) *stage = st;
   if (acc) *acc = ac;
   return align256(off);
 }
@@ -483,7 +492,7 @@ mg_status init_ctx(mg_ctx* c, const mg_params& p, int rank, int world, int devic
   if (!workspace || ws_bytes < need)
     return set_err(MG_ERR_OOM, "workspace too small: need " + std::to_string(need) + " bytes");
   if (((uintptr_t)workspace & 255) != 0) return set_err(MG_ERR_INVALID_ARG, "workspace must be 256-byte aligned");
-  carve(c->lay, (char*)workspace, &c->dl, &c->stage, &c->acc);
+  carve(c->lay, (char*)workspace, &c->dl, c->stage, &c->acc);
   (void)tables_only_upload;
   CKC(c, cudaMemsetAsync(workspace, 0, need, stream));
   for (int l = 0; l < c->lay.L; ++l) {
@@ -518,6 +527,12 @@ mg_status init_ctx(mg_ctx* c, const mg_params& p, int rank, int world, int devic
   CKC(c, cudaStreamCreateWithFlags(&c->cap, cudaStreamNonBlocking));
   CKC(c, cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
   CKC(c, cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming));
+  CKC(c, cudaStreamCreateWithFlags(&c->h2d, cudaStreamNonBlocking));
+  for (int k = 0; k < 2; ++k) {
+    CKC(c, cudaEventCreateWithFlags(&c->ev_h2d[k], cudaEventDisableTiming));
+    CKC(c, cudaEventCreateWithFlags(&c->ev_free[k], cudaEventDisableTiming));
+  }
+  CKC(c, cudaEventCreateWithFlags(&c->ev_norm, cudaEventDisableTiming));
   CKC(c, cudaMallocHost((void**)&c->h_pinned, 64));
   c->tm.assign((size_t)c->lay.L * MG_NUM_OPS, 0.0);
   for (int l = 0; l < MG_MAX_LEVELS; ++l) c->st[l] = LevelState();
@@ -532,6 +547,15 @@ void free_ctx(mg_ctx* c) {
   if (c->nccl) ncclCommDestroy(c->nccl);
   if (c->comm) cudaStreamDestroy(c->comm);
   if (c->cap) cudaStreamDestroy(c->cap);
+  if (c->h2d) {
+    cudaStreamSynchronize(c->h2d);
+    cudaStreamDestroy(c->h2d);
+  }
+  for (int k = 0; k < 2; ++k) {
+    if (c->ev_h2d[k]) cudaEventDestroy(c->ev_h2d[k]);
+    if (c->ev_free[k]) cudaEventDestroy(c->ev_free[k]);
+  }
+  if (c->ev_norm) cudaEventDestroy(c->ev_norm);
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
   if (c->ev_join) cudaEventDestroy(c->ev_join);
   for (cudaEvent_t e : c->evpool) cudaEventDestroy(e);
@@ -668,8 +692,18 @@ mg_status mg_set_rhs_host(mg_ctx* c, const double* b_host) {
   CKS(check_ctx(c));
   if (!b_host) return set_err(MG_ERR_INVALID_ARG, "null b");
   const size_t bytes = (size_t)c->lay.lv[0].n_owned * kBV * sizeof(double);
-  CKC(c, cudaMemcpyAsync(c->stage, b_host, bytes, cudaMemcpyHostToDevice, c->stream));
-  return set_level_field(c, 0, MG_FIELD_B, c->stage, c->group == nullptr);
+  // Upload on the copy stream into staging field k (free once its previous conversion ran), so
+  // the transfer overlaps whatever the caller's stream is still executing (the V-cycle of the
+  // previous right-hand side); the conversion into bricks is ordered on the caller's stream.
+  const int k = c->stage_k;
+  c->stage_k ^= 1;
+  CKC(c, cudaStreamWaitEvent(c->h2d, c->ev_free[k], 0));
+  CKC(c, cudaMemcpyAsync(c->stage[k], b_host, bytes, cudaMemcpyHostToDevice, c->h2d));
+  CKC(c, cudaEventRecord(c->ev_h2d[k], c->h2d));
+  CKC(c, cudaStreamWaitEvent(c->stream, c->ev_h2d[k], 0));
+  CKS(set_level_field(c, 0, MG_FIELD_B, c->stage[k], c->group == nullptr));
+  CKC(c, cudaEventRecord(c->ev_free[k], c->stream));
+  return MG_OK;
 }
 
 mg_status mg_set_solution(mg_ctx* c, const double* x_dev) {
@@ -694,9 +728,11 @@ mg_status mg_get_solution(mg_ctx* c, double* x_dev) {
 mg_status mg_get_solution_host(mg_ctx* c, double* x_host) {
   CKS(check_ctx(c));
   if (!x_host) return set_err(MG_ERR_INVALID_ARG, "null x");
-  CKS(mg_get_solution(c, c->stage));
+  const int k = c->stage_k;  // every upload into it is already ordered before its conversion
+  CKS(mg_get_solution(c, c->stage[k]));
   const size_t bytes = (size_t)c->lay.lv[0].n_owned * kBV * sizeof(double);
-  CKC(c, cudaMemcpyAsync(x_host, c->stage, bytes, cudaMemcpyDeviceToHost, c->stream));
+  CKC(c, cudaMemcpyAsync(x_host, c->stage[k], bytes, cudaMemcpyDeviceToHost, c->stream));
+  CKC(c, cudaEventRecord(c->ev_free[k], c->stream));
   CKC(c, cudaStreamSynchronize(c->stream));
   return MG_OK;
 }
@@ -707,10 +743,10 @@ mg_status mg_vcycle(mg_ctx* c) {
   return vcycle_impl(c, nullptr);
 }
 
-mg_status mg_residual_norm(mg_ctx* c, double* out) {
+mg_status mg_residual_norm_async(mg_ctx* c) {
   CKS(check_ctx(c));
-  if (!out) return set_err(MG_ERR_INVALID_ARG, "null out");
   if (c->group) return set_err(MG_ERR_STATE, "group member: use mg_group_residual_norm");
+  if (c->norm_pending) return set_err(MG_ERR_STATE, "a residual norm is already pending: call mg_residual_norm_wait");
   const LevelLayout& L = c->lay.lv[0];
   DevLevel& d = c->dl[0];
   if (L.n_ghost > 0) {
@@ -723,9 +759,26 @@ mg_status mg_residual_norm(mg_ctx* c, double* out) {
   if (c->use_nccl && c->lay.world > 1)
     CKN(c, ncclAllReduce(c->acc, c->acc, 1, ncclUint64, ncclMax, c->nccl, c->stream));
   CKC(c, cudaMemcpyAsync(c->h_pinned, c->acc, sizeof(unsigned long long), cudaMemcpyDeviceToHost, c->stream));
-  CKC(c, cudaStreamSynchronize(c->stream));
+  CKC(c, cudaEventRecord(c->ev_norm, c->stream));
+  c->norm_pending = true;
+  return MG_OK;
+}
+
+mg_status mg_residual_norm_wait(mg_ctx* c, double* out) {
+  CKS(check_ctx(c));
+  if (!out) return set_err(MG_ERR_INVALID_ARG, "null out");
+  if (!c->norm_pending) return set_err(MG_ERR_STATE, "no residual norm pending: call mg_residual_norm_async");
+  c->norm_pending = false;
+  CKC(c, cudaEventSynchronize(c->ev_norm));
   std::memcpy(out, c->h_pinned, sizeof(double));
   return MG_OK;
+}
+
+mg_status mg_residual_norm(mg_ctx* c, double* out) {
+  CKS(check_ctx(c));
+  if (!out) return set_err(MG_ERR_INVALID_ARG, "null out");
+  CKS(mg_residual_norm_async(c));
+  return mg_residual_norm_wait(c, out);
 }
 
 mg_status mg_solve(mg_ctx* c, double tol, int32_t max_cycles, int32_t* cycles_done, double* final_norm) {

@@ -70,6 +70,8 @@ _SIGS = {
     "mg_get_solution_host": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
     "mg_vcycle": (ctypes.c_int, [ctypes.c_void_p]),
     "mg_residual_norm": (ctypes.c_int, [ctypes.c_void_p, ctypes.POINTER(ctypes.c_double)]),
+    "mg_residual_norm_async": (ctypes.c_int, [ctypes.c_void_p]),
+    "mg_residual_norm_wait": (ctypes.c_int, [ctypes.c_void_p, ctypes.POINTER(ctypes.c_double)]),
     "mg_solve": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_double, ctypes.c_int32, ctypes.POINTER(ctypes.c_int32),
                                 ctypes.POINTER(ctypes.c_double)]),
     "mg_set_timing": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32]),
@@ -204,6 +206,16 @@ def mg_vcycle(ctx):
 def mg_residual_norm(ctx) -> float:
     out = ctypes.c_double()
     check(lib().mg_residual_norm(ctx, ctypes.byref(out)), "mg_residual_norm")
+    return out.value
+
+
+def mg_residual_norm_async(ctx) -> None:
+    check(lib().mg_residual_norm_async(ctx), "mg_residual_norm_async")
+
+
+def mg_residual_norm_wait(ctx) -> float:
+    out = ctypes.c_double()
+    check(lib().mg_residual_norm_wait(ctx, ctypes.byref(out)), "mg_residual_norm_wait")
     return out.value
 
 

@@ -99,6 +99,12 @@ class Multigrid:
     def residual_norm(self) -> float:
         return mg.mg_residual_norm(self.ctx)
 
+    def residual_norm_async(self) -> None:
+        mg.mg_residual_norm_async(self.ctx)
+
+    def residual_norm_wait(self) -> float:
+        return mg.mg_residual_norm_wait(self.ctx)
+
     def solve(self, tol=1e-10, max_cycles=20):
         return mg.mg_solve(self.ctx, tol, max_cycles)
 

@@ -261,6 +261,46 @@ def test_host_api_e2e(oracle_mod):
     m.close()
 
 
+@pytest.mark.parametrize("ghost_mode", [0, 1])
+def test_host_api_pipelined(oracle_mod, ghost_mode):
+    """The pipelined e2e pattern bench.py times: a different b per step, uploaded on the copy
+    stream (double-buffered staging) while the previous V-cycle runs, async norm + wait.  Each
+    step's norm and the final x must equal the oracle driven step by step."""
+    mg, _ = _mg()
+    shape = (32, 32, 64)
+    bs = [mg_inputs.random_rhs(shape, 20 + s) for s in range(4)]
+    orc = oracle_mod.OracleMG(shape, 3, 12, 12, 100)
+    orc.set_x(None)
+    want = []
+    for b in bs:
+        orc.set_b(b)
+        orc.vcycle()
+        want.append(orc.norm())
+    m = new(shape, 3, ghost_mode=ghost_mode)
+    m.set_solution(None)
+    bh = [torch.from_numpy(b).pin_memory() for b in bs]
+    got = []
+    m.set_rhs_host(bh[0])
+    for s in range(len(bs)):
+        m.vcycle()
+        m.residual_norm_async()
+        if s + 1 < len(bs):
+            m.set_rhs_host(bh[s + 1])
+        got.append(m.residual_norm_wait())
+    assert got == want
+    out = torch.empty(shape, dtype=torch.float64).pin_memory()
+    m.get_solution_host(out)
+    assert np.array_equal(out.numpy(), orc.get_x())
+    with pytest.raises(RuntimeError):
+        m.residual_norm_wait()  # nothing pending
+    m.residual_norm_async()
+    with pytest.raises(RuntimeError):
+        m.residual_norm_async()  # one pending at most
+    assert m.residual_norm_wait() == orc.norm()
+    m.close()
+    orc.close()
+
+
 # ------------------------------------------------------------- full sizes
 def test_full_size_512_sweep_sampled(oracle_mod):
     """512^3 (the bench workload), level-0 fused sweep: 20k sampled points vs the
