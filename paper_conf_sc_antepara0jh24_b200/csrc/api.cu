@@ -178,9 +178,12 @@ size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double**
       DevLevel::Pair pr;
       pr.b0 = pt.b0;
       pr.b1 = pt.b1;
+      pr.args.kind = pt.kind;
       pr.args.meta = (const int32_t*)take(pt.meta.size() * sizeof(int32_t));
       pr.args.ctas = (const int2*)take(pt.ctas.size() * sizeof(int32_t));
       pr.args.nctas = (int64_t)pt.ctas.size() / 2;
+      pr.args.warps = (const int4*)take(pt.warps.size() * sizeof(int32_t));
+      pr.args.nwarps = (int64_t)pt.warps.size() / 4;
       d.pairs.push_back(pr);
     }
     d.h = lay.p.h0 * (double)(1 << l);
@@ -280,7 +283,10 @@ mg_status sweep_range(mg_ctx* c, const Op& o, int64_t b0, int64_t b1, cudaStream
   if (o.kind == OP_SWEEP2) {  // two sweeps in one pass: the builder only emits it where a plan exists
     for (const auto& pr : d.pairs) {
       if (pr.b0 == b0 && pr.b1 == b1) {
-        CKC(c, launch_sweep2(a, pr.args, d.pmaps[o.src], o.flags, s));
+        if (pr.args.kind == 2)
+          CKC(c, launch_sweep2w(a, pr.args, d.pmaps[o.src], o.flags, s));
+        else
+          CKC(c, launch_sweep2(a, pr.args, d.pmaps[o.src], o.flags, s));
         return MG_OK;
       }
     }
@@ -518,6 +524,7 @@ mg_status init_ctx(mg_ctx* c, const mg_params& p, int rank, int world, int devic
       const PairArgs& pa = d.pairs[k].args;
       CKC(c, cudaMemcpyAsync((void*)pa.meta, pt.meta.data(), pt.meta.size() * 4, cudaMemcpyHostToDevice, stream));
       CKC(c, cudaMemcpyAsync((void*)pa.ctas, pt.ctas.data(), pt.ctas.size() * 4, cudaMemcpyHostToDevice, stream));
+      CKC(c, cudaMemcpyAsync((void*)pa.warps, pt.warps.data(), pt.warps.size() * 4, cudaMemcpyHostToDevice, stream));
     }
     if (!L.pairs.empty())
       for (int xb = 0; xb < 2; ++xb) CKC(c, encode_pair_maps(d.x[xb], d.b, L.n_alloc, &d.pmaps[xb]));

@@ -673,7 +673,9 @@ cudaError_t kernels_init() {
   e = cudaFuncSetAttribute(bottom_resident_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                            kResidentMaxBricks * 512 * 3 * (int)sizeof(double));
   if (e != cudaSuccess) return e;
-  return pair_kernels_init();
+  e = pair_kernels_init();
+  if (e != cudaSuccess) return e;
+  return pairw_kernels_init();
 }
 
 }  // namespace mgb

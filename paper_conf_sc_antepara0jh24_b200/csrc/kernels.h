@@ -62,9 +62,12 @@ cudaError_t encode_box_map(const double* base, int64_t n_alloc, const unsigned b
 
 // Two-sweep (temporally blocked) streaming kernel, sweep2.cu.
 struct PairArgs {
-  const int32_t* meta;  // [items][11] id, flags, W,E,S,N, SW,NW,SE,NE, parent
-  const int2* ctas;     // (first item, item count) per CTA
+  int kind;             // 1: CTA item streams (sweep2.cu), 2: half-warp plane streams (sweep2w.cu)
+  const int32_t* meta;  // kind 1: [items][11] id, flags, W,E,S,N, SW,NW,SE,NE, parent; kind 2: [items][12]
+  const int2* ctas;     // kind 1: (first item, item count) per CTA
   int64_t nctas;
+  const int4* warps;    // kind 2: (first item half 0, first item half 1, steps, items0 | items1<<16) per warp
+  int64_t nwarps;
 };
 struct PairMaps {
   CUtensorMap xwe;   // x boxes {2,8,8}: W (i=6,7) / E (i=0,1) face slabs
@@ -79,6 +82,9 @@ bool pair_supports(unsigned flags);
 cudaError_t launch_sweep2(const SweepArgs& a, const PairArgs& pa, const PairMaps& pm, unsigned flags,
                           cudaStream_t s);
 cudaError_t pair_kernels_init();
+cudaError_t launch_sweep2w(const SweepArgs& a, const PairArgs& pa, const PairMaps& pm, unsigned flags,
+                           cudaStream_t s);
+cudaError_t pairw_kernels_init();
 
 // true if the streaming kernel implements `flags` (plain, +r, +restriction)
 bool col_supports(unsigned flags);

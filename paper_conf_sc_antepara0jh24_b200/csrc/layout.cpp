@@ -265,7 +265,7 @@ mg_status build_layout(const mg_params& p, int rank, int world, Layout& out, std
   for (int l = 0; l < out.L; ++l) build_col_tables(out.lv[l], min_b);
   for (int l = 0; l + 1 < out.L; ++l) build_parents(out.lv[l], out.lv[l + 1]);
   if (p.temporal_blocking != 0)
-    for (int l = 0; l < out.L; ++l) build_pair_tables(out.lv[l], min_b);
+    for (int l = 0; l < out.L; ++l) build_pair_tables(out.lv[l], min_b, p.temporal_blocking == 1 ? 1 : 2);
   return MG_OK;
 }
 
@@ -403,7 +403,97 @@ static LevelLayout::PairTable pair_table(const LevelLayout& L, int64_t b0, int64
   return t;
 }
 
-void build_pair_tables(LevelLayout& L, int64_t min_bricks) {
+// Plane streams for the warp two-sweep kernel (sweep2w.cu), one per half-warp
+// (G = kW2Streams, even).  Chains are dealt round-robin and the remainder cut
+// into equal pieces exactly as in pair_table; each run becomes
+// [warm-up (planes 5..7), bricks (0..7, emitted), cool-down (plane 0)].  The two
+// streams of a warp are padded with dummy items (zero brick, nothing emitted) to
+// the same number of steps, so the warp's two halves step in lockstep.
+// Returns an empty table (kind 0: the schedule then uses single-sweep passes) if a
+// stream would overflow the kernel's 16-bit item counts.
+static LevelLayout::PairTable warp_table(const LevelLayout& L, int64_t b0, int64_t b1) {
+  LevelLayout::PairTable t;
+  t.kind = 2;
+  t.b0 = b0;
+  t.b1 = b1;
+  const auto chains = z_chains(L, b0, b1);
+  const int64_t nch = (int64_t)chains.size();
+  int64_t nb = 0;
+  for (const auto& c : chains) nb += (int64_t)c.size();
+  int64_t G = std::max<int64_t>(2, std::min<int64_t>(kW2Streams, nb / 4));
+  G += G & 1;
+  auto adj = [&](int64_t id, int f) -> int32_t {
+    return id >= L.n_stored ? (int32_t)L.zero_brick : L.adj[(size_t)id * 8 + f];
+  };
+  struct Stream {
+    std::vector<int32_t> meta;
+    int64_t items = 0, steps = 0;
+  };
+  std::vector<Stream> st((size_t)G);
+  auto push_item = [&](Stream& s, int32_t id, int emit, int kb, int ke) {
+    const int32_t W = adj(id, 0), E = adj(id, 1), S = adj(id, 2), N = adj(id, 3);
+    const int32_t par = (id < L.n_stored && !L.parent.empty()) ? L.parent[(size_t)id] : -1;
+    const int32_t m[kW2Meta] = {id, emit | kb << 8 | ke << 16, W, E, S, N, adj(W, 2), adj(W, 3), adj(E, 2), adj(E, 3),
+                                par, 0};
+    s.meta.insert(s.meta.end(), m, m + kW2Meta);
+    s.items += 1;
+    s.steps += ke - kb;
+  };
+  auto push_run = [&](Stream& s, const int32_t* run, int64_t len) {
+    push_item(s, adj(run[0], 4), 0, 5, 8);  // warm-up: planes 5, 6 prime, plane 7 is the run's k-halo
+    for (int64_t q = 0; q < len; ++q) push_item(s, run[q], 1, 0, 8);
+    push_item(s, adj(run[len - 1], 5), 0, 0, 1);  // cool-down: plane 0 is the run's k-halo
+  };
+  const int64_t full = (nch / G) * G;
+  for (int64_t c = 0; c < full; ++c) push_run(st[(size_t)(c % G)], chains[(size_t)c].data(), chains[(size_t)c].size());
+  std::vector<int32_t> rest, rest_chain;
+  for (int64_t c = full; c < nch; ++c)
+    for (int32_t id : chains[(size_t)c]) {
+      rest.push_back(id);
+      rest_chain.push_back((int32_t)c);
+    }
+  const int64_t nr = (int64_t)rest.size();
+  int64_t off = 0;
+  for (int64_t g = 0; g < G && nr > 0; ++g) {
+    const int64_t cnt = nr / G + (g < nr % G ? 1 : 0);
+    for (int64_t m = off; m < off + cnt;) {
+      int64_t e = m + 1;
+      while (e < off + cnt && rest_chain[(size_t)e] == rest_chain[(size_t)m]) ++e;
+      push_run(st[(size_t)g], &rest[(size_t)m], e - m);
+      m = e;
+    }
+    off += cnt;
+  }
+  const int32_t z = (int32_t)L.zero_brick;
+  for (int64_t w = 0; w < G / 2; ++w) {
+    Stream& A = st[(size_t)(2 * w)];
+    Stream& B = st[(size_t)(2 * w + 1)];
+    if (A.steps == 0 && B.steps == 0) continue;
+    for (Stream* s : {&A, &B}) {
+      const int64_t other = s == &A ? B.steps : A.steps;
+      while (s->steps < other) {
+        const int c = (int)std::min<int64_t>(8, other - s->steps);
+        push_item(*s, z, 0, 8 - c, 8);
+      }
+    }
+    const int64_t steps = A.steps, na = A.items, nbi = B.items;
+    if (na > 0xffff || nbi > 0xffff || steps > INT32_MAX) return LevelLayout::PairTable{0};
+    for (Stream* s : {&A, &B})
+      for (int i = 0; i < kW2Tail; ++i) push_item(*s, z, 0, 0, 8);
+    const int64_t oa = (int64_t)t.meta.size() / kW2Meta;
+    t.meta.insert(t.meta.end(), A.meta.begin(), A.meta.end());
+    const int64_t ob = (int64_t)t.meta.size() / kW2Meta;
+    t.meta.insert(t.meta.end(), B.meta.begin(), B.meta.end());
+    if (ob + B.items > INT32_MAX) return LevelLayout::PairTable{0};
+    t.warps.push_back((int32_t)oa);
+    t.warps.push_back((int32_t)ob);
+    t.warps.push_back((int32_t)steps);
+    t.warps.push_back((int32_t)(na | (nbi << 16)));
+  }
+  return t;
+}
+
+void build_pair_tables(LevelLayout& L, int64_t min_bricks, int kind) {
   L.pairs.clear();
   if (L.n_stored < min_bricks) return;
   const int64_t ranges[3][2] = {{0, L.n_owned}, {0, L.n_interior}, {L.n_interior, L.n_owned}};
@@ -411,7 +501,9 @@ void build_pair_tables(LevelLayout& L, int64_t min_bricks) {
     if (r[1] <= r[0]) continue;
     bool dup = false;
     for (auto& c : L.pairs) dup |= (c.b0 == r[0] && c.b1 == r[1]);
-    if (!dup) L.pairs.push_back(pair_table(L, r[0], r[1]));
+    if (dup) continue;
+    LevelLayout::PairTable t = kind == 2 ? warp_table(L, r[0], r[1]) : pair_table(L, r[0], r[1]);
+    if (t.kind != 0) L.pairs.push_back(std::move(t));
   }
 }
 

@@ -62,10 +62,18 @@ struct LevelLayout {
   // its warm-up brick (the B neighbour of its first brick) and followed by its
   // cool-down brick (T neighbour of its last): item = (id, flags, W,E,S,N,
   // SW,NW,SE,NE, parent), flags bit0 = "previous item is a range brick".
+  //
+  // kind 2 (sweep2w.cu): one stream per HALF-WARP, two streams per warp with
+  // equal step counts.  A step is one z-plane; item = (id, emit | kb<<8 | ke<<16,
+  // W,E,S,N, SW,NW,SE,NE, parent, 0) with [kb, ke) the planes the stream steps
+  // through: warm-up [5,8) (planes 5,6 prime the register windows), range bricks
+  // [0,8) (emit = 1), cool-down [0,1).  Streams end with kW2Tail dummy items.
   struct PairTable {
+    int kind = 1;
     int64_t b0 = 0, b1 = 0;
-    std::vector<int32_t> meta;  // [items][kPairMeta]
-    std::vector<int32_t> ctas;  // [nctas][2] offset (items), count
+    std::vector<int32_t> meta;   // [items][kPairMeta] (kind 1) / [items][kW2Meta] (kind 2)
+    std::vector<int32_t> ctas;   // kind 1: [nctas][2] offset (items), count
+    std::vector<int32_t> warps;  // kind 2: [nwarps][4] first item of half 0, of half 1, steps, items0 | items1<<16
   };
   std::vector<PairTable> pairs;
 };
@@ -73,7 +81,12 @@ struct LevelLayout {
 constexpr int kPairMeta = 11;
 constexpr int kPairCtasPerSm = 4;                   // resident two-sweep CTAs per SM (shared-memory bound)
 constexpr int64_t kPairCtas = 148 * kPairCtasPerSm;  // one item stream per resident two-sweep CTA
-void build_pair_tables(LevelLayout& L, int64_t min_bricks);
+constexpr int kW2Meta = 12;
+constexpr int kW2WarpsPerSm = 7;                    // resident one-warp CTAs per SM (shared-memory bound)
+constexpr int64_t kW2Streams = 148 * kW2WarpsPerSm * 2;
+constexpr int kW2Tail = 9;                          // trailing dummy items per stream (lookahead + meta prefetch)
+// kind 1: CTA item streams (sweep2.cu), kind 2: half-warp plane streams (sweep2w.cu)
+void build_pair_tables(LevelLayout& L, int64_t min_bricks, int kind);
 
 constexpr int kColSeg = 16;             // bricks per streamed segment
 constexpr int64_t kColMinBricks = 16384;  // levels smaller than this use the one-brick-per-CTA kernel

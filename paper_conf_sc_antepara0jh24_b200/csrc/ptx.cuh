@@ -83,6 +83,14 @@ __device__ __forceinline__ void tma_load_1d_hint(void* dst, const void* src, uin
       "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(pol)
       : "memory");
 }
+// bulk prefetch of [src, src+bytes) into L2 (no shared memory, no completion)
+__device__ __forceinline__ void prefetch_l2(const void* src, uint32_t bytes) {
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(src), "r"(bytes) : "memory");
+}
+// per-thread prefetch of the line holding p into L2
+__device__ __forceinline__ void prefetch_l2_line(const void* p) {
+  asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
+}
 __device__ __forceinline__ double2 ld_hint2(const double* p, uint64_t pol) {
   double2 v;
   asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.f64 {%0, %1}, [%2], %3;"

@@ -338,12 +338,12 @@ def test_full_size_512_vcycle_bitwise(oracle_mod):
 
 
 # ------------------------------------------------- streaming (column) kernel
-@pytest.mark.parametrize("tb", [0, 1])
+@pytest.mark.parametrize("tb", [0, 1, 2])
 @pytest.mark.parametrize("fusion", [2, 3])
 @pytest.mark.parametrize("ghost_mode,period", [(0, 0), (1, 1), (1, 3), (1, 8)])
 def test_streaming_kernel_forced_bitwise(oracle_mod, fusion, ghost_mode, period, tb):
-    """sweep_kernel = 2 forces the TMA-streamed column kernel (tb = 0) or the two-sweep
-    kernel (tb = 1) on every level (plain, +r and +restriction variants; owned,
+    """sweep_kernel = 2 forces the TMA-streamed column kernel (tb = 0) or a two-sweep
+    kernel (tb = 1: CTA streams, tb = 2: warp plane streams) on every level (plain, +r and +restriction variants; owned,
     owned+ghost, interior and surface ranges)."""
     shape = (64, 32, 96)
     b = mg_inputs.random_rhs(shape, 13)
@@ -356,7 +356,7 @@ def test_streaming_kernel_forced_bitwise(oracle_mod, fusion, ghost_mode, period,
     m.close()
 
 
-@pytest.mark.parametrize("tb", [0, 1])
+@pytest.mark.parametrize("tb", [0, 1, 2])
 @pytest.mark.parametrize("pg", [(2, 2, 2), (2, 1, 1)])
 def test_streaming_kernel_loopback_bitwise(oracle_mod, pg, tb):
     _, solver = _mg()
@@ -388,13 +388,14 @@ def test_vcycle_config2_256_bitwise(oracle_mod):
 
 
 # ------------------------------------------------- two sweeps per pass (temporal blocking)
+@pytest.mark.parametrize("tb", [1, 2])
 @pytest.mark.parametrize("n", [2, 3, 5])
-@pytest.mark.parametrize("shape,ghost_mode", [((64, 32, 96), 0), ((32, 48, 64), 1)])
-def test_two_sweep_pass_per_op(oracle_mod, n, shape, ghost_mode):
+@pytest.mark.parametrize("shape,ghost_mode", [((64, 32, 96), 0), ((32, 48, 64), 1), ((40, 24, 56), 0)])
+def test_two_sweep_pass_per_op(oracle_mod, n, shape, ghost_mode, tb):
     """OP_SWEEP2 (x0 -> x1 -> x2 in one pass, redundant x1 on the side faces) equals
     n separate sweeps of the oracle bit for bit, including r of the last sweep."""
     mg, _ = _mg()
-    m = new(shape, 1, pre=1, post=1, bottom=1, sweep_kernel=2, ghost_mode=ghost_mode, temporal_blocking=1)
+    m = new(shape, 1, pre=1, post=1, bottom=1, sweep_kernel=2, ghost_mode=ghost_mode, temporal_blocking=tb)
     h = mg_inputs.default_h0(shape)
     x = mg_inputs.random_field(shape, 21)
     b = mg_inputs.random_field(shape, 22)
@@ -409,7 +410,7 @@ def test_two_sweep_pass_per_op(oracle_mod, n, shape, ghost_mode):
     m.close()
 
 
-@pytest.mark.parametrize("tb", [0, 1])
+@pytest.mark.parametrize("tb", [0, 1, 2])
 def test_temporal_blocking_on_off_bitwise(oracle_mod, tb):
     """The V-cycle with and without temporal blocking gives the oracle's bits (256^3, L = 6,
     where levels 0 and 1 stream; 12/12/100)."""
