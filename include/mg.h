@@ -171,6 +171,11 @@ enum { MG_OP_SWEEP = 0, MG_OP_APPLYOP = 1, MG_OP_SMOOTH = 2, MG_OP_RESTRICT = 3,
        MG_OP_ZERO = 5, MG_OP_EXCHANGE = 6, MG_OP_BOTTOM = 7, MG_NUM_OPS = 8 };
 mg_status mg_set_timing(mg_ctx* c, int32_t enabled);
 mg_status mg_get_timings(mg_ctx* c, double* out, int32_t cap);
+/* The individual timed ops since mg_set_timing, in issue order: slots[i] =
+ * level*MG_NUM_OPS + op, ms[i] = its device time.  Writes min(cap, *count)
+ * records; *count = number available (call with cap = 0 to size the buffers).
+ * Input for the latency/throughput fits t = alpha + x/beta (tools/model_fit.py). */
+mg_status mg_get_timing_records(mg_ctx* c, int32_t* slots, double* ms, int32_t cap, int32_t* count);
 
 /* Number of kernel launches (own kernels) one mg_vcycle issues. */
 mg_status mg_vcycle_launches(mg_ctx* c, int64_t* out);

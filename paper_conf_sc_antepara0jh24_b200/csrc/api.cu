@@ -56,6 +56,10 @@ struct DevLevel {
   };
   std::vector<Pair> pairs;  // two-sweep item streams per brick range
   PairMaps pmaps[2];        // tensor maps for the two-sweep kernel reading x[0] / x[1]
+  // local-transport exchange: [x[0] | x[1] | b][recv run] copy descriptors (device), one launch
+  CopyRun* cruns = nullptr;
+  int ncruns = 0;
+  int64_t cmax = 0;
 };
 
 struct Plan {
@@ -100,6 +104,7 @@ struct mg_ctx {
   bool use_col = true;  // streaming column kernel where a plan exists (sweep_kernel == 1 disables)
   std::vector<double> tm;
   std::vector<TimerRec> trec;
+  std::vector<std::pair<int, double>> recs;  // (level*MG_NUM_OPS + op, ms) per timed op, since mg_set_timing
   std::vector<cudaEvent_t> evpool;
   size_t evnext = 0;
   cudaGraphExec_t gexec[2] = {nullptr, nullptr};
@@ -186,6 +191,8 @@ size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double**
       pr.args.nwarps = (int64_t)pt.warps.size() / 4;
       d.pairs.push_back(pr);
     }
+    d.ncruns = (int)L.recvs.size();
+    d.cruns = (CopyRun*)take((size_t)d.ncruns * 3 * sizeof(CopyRun));
     d.h = lay.p.h0 * (double)(1 << l);
     d.c = level_coeffs(d.h);
     if (out) (*out)[l] = d;
@@ -246,12 +253,36 @@ mg_status do_exchange(mg_ctx* c, int l, int field, int xbuf, cudaStream_t s) {
       CKN(c, ncclSend(f + r.local * bb, (size_t)r.count * bb, ncclFloat64, r.peer, c->nccl, s));
     CKN(c, ncclGroupEnd());
   } else {
-    for (const Run& r : L.recvs) {
-      mg_ctx* src = c->group ? c->group->r[r.peer] : c;
-      const double* sp = field_ptr(src, l, field, xbuf);
-      CKC(c, cudaMemcpyAsync(f + r.local * bb, sp + r.remote * bb, (size_t)r.count * bb * sizeof(double),
-                             cudaMemcpyDeviceToDevice, s));
+    // every run of the exchange in one copy kernel (tables built by fill_copy_tables)
+    const DevLevel& d = c->dl[l];
+    const int fv = field ? 2 : xbuf;
+    CKC(c, launch_copy_runs(d.cruns + (size_t)fv * d.ncruns, d.ncruns, d.cmax, s));
+  }
+  return MG_OK;
+}
+
+// Copy descriptors of the local transport: receiver ghost run <- sender surface run, for the
+// three exchanged fields (x[0], x[1], b).  Needs every rank's workspace carved (loopback groups).
+mg_status fill_copy_tables(mg_ctx* c) {
+  const size_t bb = (size_t)kBV;
+  for (int l = 0; l < c->lay.L; ++l) {
+    const LevelLayout& L = c->lay.lv[l];
+    DevLevel& d = c->dl[l];
+    if (d.ncruns == 0) continue;
+    std::vector<CopyRun> h((size_t)d.ncruns * 3);
+    d.cmax = 0;
+    for (int fv = 0; fv < 3; ++fv) {
+      const int field = fv == 2 ? 1 : 0, xbuf = fv == 2 ? 0 : fv;
+      double* f = field_ptr(c, l, field, xbuf);
+      for (int i = 0; i < d.ncruns; ++i) {
+        const Run& r = L.recvs[(size_t)i];
+        mg_ctx* src = c->group ? c->group->r[r.peer] : c;
+        h[(size_t)fv * d.ncruns + i] = {field_ptr(src, l, field, xbuf) + r.remote * bb, f + r.local * bb,
+                                        (int64_t)r.count * (int64_t)bb};
+        d.cmax = std::max<int64_t>(d.cmax, (int64_t)r.count * (int64_t)bb);
+      }
     }
+    CKC(c, cudaMemcpy(d.cruns, h.data(), h.size() * sizeof(CopyRun), cudaMemcpyHostToDevice));
   }
   return MG_OK;
 }
@@ -405,6 +436,7 @@ mg_status collect_timings(mg_ctx* c) {
     float ms = 0;
     CKC(c, cudaEventElapsedTime(&ms, t.a, t.b));
     if (t.slot >= 0 && t.slot < (int)c->tm.size()) c->tm[t.slot] += ms;
+    c->recs.push_back({t.slot, (double)ms});
   }
   c->trec.clear();
   c->evnext = 0;
@@ -685,6 +717,13 @@ mg_status mg_setup(const mg_params* p, int32_t rank, int32_t world_size, const u
     c->use_nccl = true;
   }
   (void)any_ghost;
+  if (!c->use_nccl) {
+    s = fill_copy_tables(c);
+    if (s != MG_OK) {
+      free_ctx(c);
+      return s;
+    }
+  }
   *out = c;
   return MG_OK;
 }
@@ -807,6 +846,20 @@ mg_status mg_set_timing(mg_ctx* c, int32_t enabled) {
   CKS(check_ctx(c));
   c->timing = enabled != 0;
   std::fill(c->tm.begin(), c->tm.end(), 0.0);
+  c->recs.clear();
+  return MG_OK;
+}
+
+mg_status mg_get_timing_records(mg_ctx* c, int32_t* slots, double* ms, int32_t cap, int32_t* count) {
+  CKS(check_ctx(c));
+  if (!count || (cap > 0 && (!slots || !ms))) return set_err(MG_ERR_INVALID_ARG, "null out");
+  CKS(collect_timings(c));
+  const int n = std::min<int>(cap, (int)c->recs.size());
+  for (int i = 0; i < n; ++i) {
+    slots[i] = c->recs[(size_t)i].first;
+    ms[i] = c->recs[(size_t)i].second;
+  }
+  *count = (int32_t)c->recs.size();
   return MG_OK;
 }
 
@@ -962,6 +1015,13 @@ mg_status mg_group_setup(const mg_params* p, int32_t world_size, int32_t device,
     c->group = g;
     c->grank = r;
     g->r.push_back(c);
+    if (s != MG_OK) {
+      mg_group_destroy(g);
+      return s;
+    }
+  }
+  for (mg_ctx* c : g->r) {  // every rank's fields exist now: the cross-rank copy tables
+    mg_status s = fill_copy_tables(c);
     if (s != MG_OK) {
       mg_group_destroy(g);
       return s;

@@ -16,6 +16,7 @@
 // Brick cell (i,j,k) lives at i + 8j + 64k of its 512-double brick (A16).
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cstdint>
 
 #include <cudaTypedefs.h>
@@ -651,6 +652,26 @@ cudaError_t launch_brick_to_lex(const double* bricks, double* lex, const int32_t
                                 int ny, cudaStream_t s) {
   if (nowned <= 0) return cudaSuccess;
   brick_to_lex_kernel<<<(unsigned)nowned, 256, 0, s>>>(bricks, lex, coord, nx, ny);
+  return cudaGetLastError();
+}
+
+// blockIdx.y = run; the x-blocks stride over its 16-byte words
+__global__ void __launch_bounds__(256) copy_runs_kernel(const CopyRun* __restrict__ runs) {
+  const CopyRun r = runs[blockIdx.y];
+  const double2* src = reinterpret_cast<const double2*>(r.src);
+  double2* dst = reinterpret_cast<double2*>(r.dst);
+  const int64_t n2 = r.n / 2;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n2; i += (int64_t)gridDim.x * blockDim.x)
+    dst[i] = ldg2(reinterpret_cast<const double*>(src + i));
+}
+
+cudaError_t launch_copy_runs(const CopyRun* runs, int nruns, int64_t max_n, cudaStream_t s) {
+  if (nruns <= 0 || max_n <= 0) return cudaSuccess;
+  // about 4 waves of 256-thread blocks over the whole exchange, at least one block per run
+  const int64_t words = max_n / 2;
+  const int64_t want = (int64_t)148 * 8 * 4 / nruns;
+  const unsigned gx = (unsigned)std::max<int64_t>(1, std::min<int64_t>((words + 255) / 256, std::max<int64_t>(1, want)));
+  copy_runs_kernel<<<dim3(gx, (unsigned)nruns), 256, 0, s>>>(runs);
   return cudaGetLastError();
 }
 

@@ -114,6 +114,14 @@ cudaError_t launch_lex_to_brick(const double* lex, double* bricks, const int32_t
                                 int ny, cudaStream_t s);
 cudaError_t launch_brick_to_lex(const double* bricks, double* lex, const int32_t* coord, int64_t nowned, int nx,
                                 int ny, cudaStream_t s);
+// Local (self / loopback) ghost exchange: every run of one exchange in ONE launch instead of one
+// cudaMemcpyAsync per run (n doubles from src to dst, both 16-byte aligned, n even).
+struct CopyRun {
+  const double* src;
+  double* dst;
+  int64_t n;
+};
+cudaError_t launch_copy_runs(const CopyRun* runs, int nruns, int64_t max_n, cudaStream_t s);
 cudaError_t kernels_init();  // one-time attribute setup
 
 }  // namespace mgb

@@ -496,7 +496,13 @@ static LevelLayout::PairTable warp_table(const LevelLayout& L, int64_t b0, int64
 void build_pair_tables(LevelLayout& L, int64_t min_bricks, int kind) {
   L.pairs.clear();
   if (L.n_stored < min_bricks) return;
-  const int64_t ranges[3][2] = {{0, L.n_owned}, {0, L.n_interior}, {L.n_interior, L.n_owned}};
+  // owned, interior / surface (overlap), and the same with the ghost shell (two-sweep passes
+  // that also sweep the ghosts redundantly, so an exchange serves several passes)
+  const int64_t ranges[5][2] = {{0, L.n_owned},
+                                {0, L.n_interior},
+                                {L.n_interior, L.n_owned},
+                                {0, L.n_stored},
+                                {L.n_interior, L.n_stored}};
   for (auto& r : ranges) {
     if (r[1] <= r[0]) continue;
     bool dup = false;

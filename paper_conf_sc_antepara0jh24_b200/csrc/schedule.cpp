@@ -22,20 +22,29 @@ int Builder::period(int l) const {
   return k ? k : MG_MAX_PERIOD;
 }
 
+bool Builder::has_pair_table(int l, int64_t b0, int64_t b1) const {
+  for (const auto& pt : lay.lv[l].pairs)
+    if (pt.b0 == b0 && pt.b1 == b1) return true;
+  return false;
+}
+
 bool Builder::pair_ok(int l) const {
   if (!lay.p.temporal_blocking || fusion(l) == MG_FUSION_PAPER) return false;
   const LevelLayout& L = lay.lv[l];
-  auto has = [&](int64_t b0, int64_t b1) {
-    for (const auto& pt : L.pairs)
-      if (pt.b0 == b0 && pt.b1 == b1) return true;
-    return false;
-  };
-  if (!has(0, L.n_owned)) return false;
+  if (!has_pair_table(l, 0, L.n_owned)) return false;
   if (ghosts(l)) {
     if (period(l) < 2) return false;  // a pair is two sweeps per exchange
-    if (lay.p.overlap && L.n_interior > 0 && !(has(0, L.n_interior) && has(L.n_interior, L.n_owned))) return false;
+    if (lay.p.overlap && L.n_interior > 0 &&
+        !(has_pair_table(l, 0, L.n_interior) && has_pair_table(l, L.n_interior, L.n_owned)))
+      return false;
   }
   return true;
+}
+
+bool Builder::pair_ghosts_ok(int l) const {
+  const LevelLayout& L = lay.lv[l];
+  if (!has_pair_table(l, 0, L.n_stored)) return false;
+  return !(lay.p.overlap && L.n_interior > 0) || has_pair_table(l, L.n_interior, L.n_stored);
 }
 
 void Builder::phase(int l, int n, bool zero_first, int last, bool interp_first, int timer) {
@@ -58,13 +67,17 @@ void Builder::phase(int l, int n, bool zero_first, int last, bool interp_first, 
         S.since = 0;
       }
       o.exch_before = ex;
-      o.ghosts = false;
-      if (s + 1 == n - 1 && last == 1) o.flags |= SW_WRITE_R;
-      if (s + 1 == n - 1 && last == 2) o.flags |= SW_RESTRICT;
+      // ghost validity after two sweeps over the ghost shell too (x1 needs x0 one cell further
+      // out and b at its own depth; x2 likewise from x1): min(d_x - 2, d_b - 1)
+      const int d_inc = std::min(S.dx - 2, S.db - 1);
+      const bool last_p = s + 1 == n - 1;
+      o.ghosts = g && !last_p && d_inc >= 1 && (S.since + 2) < k && pair_ghosts_ok(l);
+      if (last_p && last == 1) o.flags |= SW_WRITE_R;
+      if (last_p && last == 2) o.flags |= SW_RESTRICT;
       o.src = S.cur;
       o.dst = 1 - S.cur;
       S.cur = o.dst;
-      S.dx = 0;
+      S.dx = o.ghosts ? d_inc : 0;
       S.since += 2;
       ops.push_back(o);
       ++s;

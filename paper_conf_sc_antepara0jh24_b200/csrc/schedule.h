@@ -53,6 +53,8 @@ struct Builder {
   int fusion(int l) const;
   int period(int l) const;
   bool pair_ok(int l) const;  // two-sweep passes possible at level l
+  bool pair_ghosts_ok(int l) const;  // two-sweep passes may include the ghost shell at level l
+  bool has_pair_table(int l, int64_t b0, int64_t b1) const;
   // `n` smooth(+residual) sweeps at level l.  last: 0 none, 1 write r, 2 fused restriction.
   void phase(int l, int n, bool zero_first, int last, bool interp_first, int timer);
   void restrict_op(int l);  // b_{l+1} = R r_l (+ b ghost exchange)

@@ -71,6 +71,9 @@ _SIGS = {
     "mg_vcycle": (ctypes.c_int, [ctypes.c_void_p]),
     "mg_residual_norm": (ctypes.c_int, [ctypes.c_void_p, ctypes.POINTER(ctypes.c_double)]),
     "mg_residual_norm_async": (ctypes.c_int, [ctypes.c_void_p]),
+    "mg_get_timing_records": (ctypes.c_int, [ctypes.c_void_p, ctypes.POINTER(ctypes.c_int32),
+                                             ctypes.POINTER(ctypes.c_double), ctypes.c_int32,
+                                             ctypes.POINTER(ctypes.c_int32)]),
     "mg_residual_norm_wait": (ctypes.c_int, [ctypes.c_void_p, ctypes.POINTER(ctypes.c_double)]),
     "mg_solve": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_double, ctypes.c_int32, ctypes.POINTER(ctypes.c_int32),
                                 ctypes.POINTER(ctypes.c_double)]),
@@ -234,6 +237,17 @@ def mg_get_timings(ctx, num_levels: int):
     buf = (ctypes.c_double * n)()
     check(lib().mg_get_timings(ctx, buf, n), "mg_get_timings")
     return [[buf[l * MG_NUM_OPS + o] for o in range(MG_NUM_OPS)] for l in range(num_levels)]
+
+
+def mg_get_timing_records(ctx):
+    """[(level, op, ms)] of every timed op since mg_set_timing (issue order)."""
+    n = ctypes.c_int32()
+    check(lib().mg_get_timing_records(ctx, None, None, 0, ctypes.byref(n)), "mg_get_timing_records")
+    cap = n.value
+    slots = (ctypes.c_int32 * max(cap, 1))()
+    ms = (ctypes.c_double * max(cap, 1))()
+    check(lib().mg_get_timing_records(ctx, slots, ms, cap, ctypes.byref(n)), "mg_get_timing_records")
+    return [(slots[i] // MG_NUM_OPS, slots[i] % MG_NUM_OPS, ms[i]) for i in range(min(cap, n.value))]
 
 
 def mg_vcycle_launches(ctx) -> int:

@@ -126,6 +126,10 @@ class Multigrid:
     def set_timing(self, on: bool):
         mg.mg_set_timing(self.ctx, on)
 
+    def timing_records(self):
+        """[(level, op, ms)] of every op timed since set_timing(True)."""
+        return mg.mg_get_timing_records(self.ctx)
+
     def launches_per_vcycle(self) -> int:
         return mg.mg_vcycle_launches(self.ctx)
 
