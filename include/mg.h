@@ -86,8 +86,12 @@ enum {
 /* transport */
 enum { MG_TRANSPORT_AUTO = 0, MG_TRANSPORT_NCCL = 1, MG_TRANSPORT_LOCAL = 2 };
 
-/* bottom_mode */
-enum { MG_BOTTOM_AUTO = 0, MG_BOTTOM_SWEEPS = 1, MG_BOTTOM_RESIDENT = 2 };
+/* bottom_mode.  AUTO: the deepest levels without ghosts that fit (<= 64 bricks per level,
+ * <= 200 KB of fields) run as ONE cluster-resident launch (coarse.cu: pre-sweeps, restriction,
+ * initZero, bottom, interpolation, post-sweeps of those levels); a lone
+ * bottom level of <= 8 bricks runs in one CTA; otherwise per-sweep launches.  All modes are
+ * bitwise identical. */
+enum { MG_BOTTOM_AUTO = 0, MG_BOTTOM_SWEEPS = 1, MG_BOTTOM_RESIDENT = 2, MG_BOTTOM_CLUSTER = 3 };
 
 typedef struct {
   int32_t n_local[3];            /* cells per rank per axis (x,y,z); each divisible by 8*2^(num_levels-1) */
@@ -102,7 +106,8 @@ typedef struct {
   int32_t transport;             /* MG_TRANSPORT_*: auto = NCCL when world_size > 1 or a
                                     self-exchange is needed and an NCCL id is given, else local */
   int32_t use_graph;             /* 1 = replay the V-cycle as one CUDA graph (default 1) */
-  int32_t bottom_mode;           /* MG_BOTTOM_* (resident = one CTA runs all bottom sweeps in smem) */
+  int32_t bottom_mode;           /* MG_BOTTOM_* (resident = one CTA runs all bottom sweeps in smem,
+                                    cluster = the coarse levels run in one cluster launch) */
   int32_t overlap;               /* 1 = sweep interior bricks while the exchange is in flight */
   int32_t sweep_kernel;          /* 0 = auto (streaming column kernel on levels >= 16384 bricks),
                                     1 = one-brick-per-CTA kernel only, 2 = streaming kernel on every level */

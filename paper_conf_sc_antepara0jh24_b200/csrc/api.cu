@@ -225,7 +225,7 @@ mg_status check_params(const mg_params& p) {
   if (p.num_levels > 1 && p.pre_smooths < 1)
     return set_err(MG_ERR_INVALID_ARG, "pre_smooths must be >= 1 when num_levels > 1 (restriction reads its r)");
   if (p.transport < 0 || p.transport > MG_TRANSPORT_LOCAL) return set_err(MG_ERR_INVALID_ARG, "bad transport");
-  if (p.bottom_mode < 0 || p.bottom_mode > MG_BOTTOM_RESIDENT) return set_err(MG_ERR_INVALID_ARG, "bad bottom_mode");
+  if (p.bottom_mode < 0 || p.bottom_mode > MG_BOTTOM_CLUSTER) return set_err(MG_ERR_INVALID_ARG, "bad bottom_mode");
   return MG_OK;
 }
 
@@ -400,6 +400,23 @@ mg_status exec_op(mg_ctx* c, const Op& o, cudaStream_t s) {
       CKS(do_exchange(c, o.level, o.field, o.src, s));
       CKS(timer_end(c, s, t0, o.level, o.timer));
       return MG_OK;
+    case OP_COARSE: {
+      CoarseArgs a{};
+      a.nlev = c->lay.L - o.level;
+      for (int l = o.level; l < c->lay.L; ++l) {
+        const DevLevel& dl = c->dl[l];
+        a.lv[l - o.level] = {(int)c->lay.lv[l].n_owned, dl.adj, dl.parent, dl.c};
+      }
+      a.b0 = d.b;
+      a.x0 = d.x[o.dst];
+      a.pre = c->lay.p.pre_smooths;
+      a.post = c->lay.p.post_smooths;
+      a.bottom = c->lay.p.bottom_smooths;
+      CKS(timer_begin(c, s, &t0));
+      CKC(c, launch_coarse(a, s));
+      CKS(timer_end(c, s, t0, o.level, o.timer));
+      return MG_OK;
+    }
     case OP_BOTTOM_RES:
       CKS(timer_begin(c, s, &t0));
       CKC(c, launch_bottom_resident(d.x[o.src], d.x[o.dst], d.b, d.adj, (int)L.n_stored, o.n, o.zero, d.c, s));

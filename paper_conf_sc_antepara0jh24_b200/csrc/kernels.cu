@@ -696,7 +696,9 @@ cudaError_t kernels_init() {
   if (e != cudaSuccess) return e;
   e = pair_kernels_init();
   if (e != cudaSuccess) return e;
-  return pairw_kernels_init();
+  e = pairw_kernels_init();
+  if (e != cudaSuccess) return e;
+  return coarse_kernels_init();
 }
 
 }  // namespace mgb

@@ -122,6 +122,29 @@ struct CopyRun {
   int64_t n;
 };
 cudaError_t launch_copy_runs(const CopyRun* runs, int nruns, int64_t max_n, cudaStream_t s);
+// Resident coarse solver (coarse.cu): levels l0 .. L-1 of one V-cycle (pre-sweeps + fused
+// restriction, initZero, bottom, interpolation, post-sweeps) in one launch of a cluster of
+// kCoarseCtas CTAs holding every field of those levels in shared memory.  No ghosts.
+constexpr int kCoarseCtas = 8;
+constexpr int kCoarseThreads = 512;
+constexpr int kCoarseMaxLevels = 8;
+constexpr size_t kCoarseMaxSmem = 200 * 1024;
+struct CoarseLevel {
+  int nb;                 // bricks (owned == stored: no ghosts)
+  const int32_t* adj;     // [nb][8]
+  const int32_t* parent;  // [nb] coarse brick * 8 + octant (levels < last)
+  Coeffs c;
+};
+struct CoarseArgs {
+  int nlev;  // levels l0 .. l0 + nlev - 1; the last one is the bottom
+  CoarseLevel lv[kCoarseMaxLevels];
+  const double* b0;  // b of level l0 (restricted by the level above)
+  double* x0;        // out: x of level l0 after its post-sweeps
+  int pre, post, bottom;
+};
+size_t coarse_smem_bytes(const CoarseArgs& a);
+cudaError_t launch_coarse(const CoarseArgs& a, cudaStream_t s);
+cudaError_t coarse_kernels_init();
 cudaError_t kernels_init();  // one-time attribute setup
 
 }  // namespace mgb

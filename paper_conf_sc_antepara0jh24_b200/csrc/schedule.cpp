@@ -161,7 +161,8 @@ void Builder::bottom(int l, int n, bool zero) {
   const LevelLayout& L = lay.lv[l];
   const int bm = lay.p.bottom_mode;
   const bool can_res = !ghosts(l) && L.n_stored <= kResidentMaxBricks;
-  const bool res = can_res && (bm == MG_BOTTOM_RESIDENT || (bm == MG_BOTTOM_AUTO && fusion(l) != MG_FUSION_PAPER));
+  const bool res = can_res && (bm == MG_BOTTOM_RESIDENT ||
+                                ((bm == MG_BOTTOM_AUTO || bm == MG_BOTTOM_CLUSTER) && fusion(l) != MG_FUSION_PAPER));
   const bool fold_zero = zero && fusion(l) == MG_FUSION_FULL;
   if (res) {
     Op o;
@@ -180,9 +181,35 @@ void Builder::bottom(int l, int n, bool zero) {
   phase(l, n, fold_zero, 0, false, MG_OP_BOTTOM);
 }
 
+int Builder::coarse_start() const {
+  const int L = lay.L;
+  const int bm = lay.p.bottom_mode;
+  if (L < 2 || !(bm == MG_BOTTOM_AUTO || bm == MG_BOTTOM_CLUSTER)) return -1;
+  if (lay.p.pre_smooths < 1) return -1;
+  // the deepest run of levels >= 1 without ghosts, paper kernel set excluded, whose first level
+  // fits the cluster (<= 8 bricks per CTA) and whose fields fit its shared memory
+  int l0 = L;
+  while (l0 - 1 >= 1 && !ghosts(l0 - 1) && fusion(l0 - 1) != MG_FUSION_PAPER &&
+         lay.lv[l0 - 1].n_owned <= 8 * kCoarseCtas && L - (l0 - 1) <= kCoarseMaxLevels)
+    --l0;
+  if (l0 >= L || ghosts(L - 1) || fusion(L - 1) == MG_FUSION_PAPER) return -1;
+  CoarseArgs a{};
+  a.nlev = L - l0;
+  for (int l = l0; l < L; ++l) a.lv[l - l0].nb = (int)lay.lv[l].n_owned;
+  while (a.nlev > 1 && coarse_smem_bytes(a) > kCoarseMaxSmem) {  // drop the largest level
+    for (int i = 0; i + 1 < a.nlev; ++i) a.lv[i] = a.lv[i + 1];
+    --a.nlev;
+    ++l0;
+  }
+  if (coarse_smem_bytes(a) > kCoarseMaxSmem) return -1;
+  if (l0 == L - 1 && bm == MG_BOTTOM_AUTO && lay.lv[L - 1].n_stored <= kResidentMaxBricks) return -1;  // one CTA does
+  return l0;
+}
+
 void Builder::vcycle() {
   const int L = lay.L;
   const mg_params& p = lay.p;
+  const int lc = coarse_start();  // levels lc .. L-1 run in one cluster launch (-1: none)
   // Coarse x is dead at the start of a cycle (zeroed below): normalise its buffer.
   for (int l = 1; l < L; ++l) {
     st[l].cur = 0;
@@ -197,7 +224,8 @@ void Builder::vcycle() {
     bottom(0, p.bottom_smooths, false);
     return;
   }
-  for (int l = 0; l + 1 < L; ++l) {  // Alg 2 steps 1-8
+  const int top = lc > 0 ? lc : L;  // levels handled one op at a time: 0 .. top-1
+  for (int l = 0; l + 1 < top || (lc > 0 && l + 1 == top); ++l) {  // Alg 2 steps 1-8
     const bool full = fusion(l) == MG_FUSION_FULL;
     const bool zero_first = l > 0 && full;
     phase(l, p.pre_smooths, zero_first, full ? 2 : 1, false, MG_OP_SWEEP);
@@ -205,6 +233,7 @@ void Builder::vcycle() {
       exchange_b(l + 1);  // restriction fused into the last pre-sweep
     else
       restrict_op(l);
+    if (l + 1 == lc) break;  // the cluster solve zeroes its own levels
     // the fold needs a first coarse sweep to absorb it (pre_smooths >= 1 is validated)
     const bool fold = fusion(l + 1) == MG_FUSION_FULL && (l + 2 < L || p.bottom_smooths > 0);
     if (!fold)  // initZero as its own kernel (Alg 2 step 8)
@@ -214,8 +243,19 @@ void Builder::vcycle() {
       st[l + 1].since = 0;
     }
   }
-  bottom(L - 1, p.bottom_smooths, true);  // steps 10-15
-  for (int l = L - 2; l >= 0; --l) {       // steps 16-23
+  if (lc > 0) {  // steps 1-23 of levels lc .. L-1 in one launch
+    Op o;
+    o.kind = OP_COARSE;
+    o.level = lc;
+    o.src = o.dst = 0;
+    o.timer = MG_OP_BOTTOM;
+    ops.push_back(o);
+    st[lc].cur = 0;
+    st[lc].dx = 0;
+  } else {
+    bottom(L - 1, p.bottom_smooths, true);  // steps 10-15
+  }
+  for (int l = top - (lc > 0 ? 1 : 2); l >= 0; --l) {  // steps 16-23
     const bool fuse_i = fusion(l) == MG_FUSION_FULL && !ghosts(l) && p.post_smooths > 0;
     if (!fuse_i) interp_op(l);
     phase(l, p.post_smooths, false, 0, fuse_i, MG_OP_SWEEP);
@@ -234,6 +274,7 @@ int64_t op_launches(const Op& o, const Layout& lay, bool overlap) {
     case OP_INTERP:
     case OP_ZERO:
     case OP_BOTTOM_RES:
+    case OP_COARSE:
       return 1;
     default:
       return 0;

@@ -16,7 +16,9 @@
 
 namespace mgb {
 
-enum OpKind { OP_SWEEP = 0, OP_RESTRICT, OP_INTERP, OP_ZERO, OP_EXCH, OP_BOTTOM_RES, OP_SWEEP2 };
+enum OpKind { OP_SWEEP = 0, OP_RESTRICT, OP_INTERP, OP_ZERO, OP_EXCH, OP_BOTTOM_RES, OP_SWEEP2, OP_COARSE };
+// OP_COARSE: levels `level` .. L-1 of the cycle in one cluster launch (coarse.cu); x of `level`
+// ends in buffer `dst`.
 // OP_SWEEP2: two consecutive plain sweeps in one pass (sweep2.cu); `flags` are the
 // second sweep's (r / restriction); owned bricks only; needs ghost depth >= 2.
 
@@ -62,6 +64,7 @@ struct Builder {
   void interp_op(int l);
   void bottom(int l, int n, bool zero);
   void exchange_b(int l);
+  int coarse_start() const;  // first level of the cluster-resident coarse solve, or -1
   void vcycle();
 };
 

@@ -231,6 +231,27 @@ def test_solve_matches_oracle(oracle_mod):
     m.close()
 
 
+@pytest.mark.parametrize("bottom_mode", [0, 1, 2, 3])
+@pytest.mark.parametrize("shape,L,pre,post,bottom", [
+    ((64, 64, 64), 4, 12, 12, 100),   # config 1: levels 1-3 (64, 8, 1 bricks) in the cluster
+    ((32, 96, 64), 3, 3, 2, 20),      # non-cubic, ragged brick counts per CTA (48 -> 6 bricks)
+    ((64, 32, 96), 3, 2, 0, 5),       # post = 0
+    ((32, 32, 32), 3, 1, 1, 0),       # bottom = 0
+    ((64, 64, 64), 2, 2, 2, 7),       # coarsest level alone (64 bricks) in the cluster
+])
+def test_coarse_cluster_solver_bitwise(oracle_mod, bottom_mode, shape, L, pre, post, bottom):
+    """The cluster-resident coarse solve (coarse.cu, bottom_mode auto / cluster: the deepest
+    ghost-free levels in one launch, neighbours through DSMEM) against per-level launches
+    (sweeps / resident) and the oracle, bit for bit, 2 cycles."""
+    b = mg_inputs.random_rhs(shape, 31)
+    xs, ns = oracle_cycles(oracle_mod, b, L, 2, pre, post, bottom)
+    m = new(shape, L, pre=pre, post=post, bottom=bottom, bottom_mode=bottom_mode)
+    m.set_rhs(dev(b))
+    m.set_solution(None)
+    check_cycles(m, xs, ns)
+    m.close()
+
+
 def test_edge_cases_single_level_and_minimal_sweeps(oracle_mod):
     """L = 1 (bottom only), pre = 1, post = 0, bottom = 0."""
     for shape, L, pre, post, bottom in [((16, 8, 24), 1, 1, 1, 7), ((32, 32, 32), 3, 1, 0, 0),
