@@ -96,6 +96,10 @@ __global__ void __launch_bounds__(P2_THREADS, kPairCtasPerSm)
   const bool isW = i0 == 0, isE = i0 == 6, isS = j == 0, isN = j == 7;
   const int sWE = isW ? j : 8 + j;                     // face lane holding my W / E face cell
   const int sSN = (isS ? 16 : 24) + i0;                // face lanes holding my S / N face pair
+  // my W / E face x0 (row j) and S / N face x0 pair (i0, i0+1) in the slab stage at plane 0 (lanes
+  // inside the brick read the same words as a boundary lane: broadcasts, no extra wavefronts)
+  const int fwo = isE ? OXWE + 128 + 2 * j : OXWE + 2 * j + 1;
+  const int fsno = isN ? OXSN + 128 + i0 : OXSN + 8 + i0;
   // ---- face-cell role: face ff (0 W, 1 E, 2 S, 3 N), in-face coordinate c8 ----
   const int ff = l >> 3, c8 = l & 7;
   int oc0, oo0, ob0, obk, olo, ohi;  // stage offsets (doubles) at plane 0; slabs step 16 / plane
@@ -112,6 +116,7 @@ __global__ void __launch_bounds__(P2_THREADS, kPairCtasPerSm)
     oc0 = OXSN + 128 + c8, oo0 = OXSN + 128 + 8 + c8, ob0 = OBSN + 64 + c8, obk = 8;
     olo = OCOR + 1 * 16 + 1, ohi = OCOR + 3 * 16 + 0;  // NW (i=7), NE (i=0)
   }
+  const int ocr = c8 == 7 ? ohi : olo;  // the one diagonal-corner value this face lane needs
   // the own-brick cell next to the face cell lives in lane srcOwn's register pair
   const int srcOwn = ff == 0 ? 4 * c8 : ff == 1 ? 4 * c8 + 3 : ff == 2 ? (c8 >> 1) : 28 + (c8 >> 1);
   const bool ownY = ff == 1 || (ff >= 2 && (c8 & 1));
@@ -236,16 +241,15 @@ __global__ void __launch_bounds__(P2_THREADS, kPairCtasPerSm)
         const double ownx = __shfl_sync(FULL, xc.x, srcOwn), owny = __shfl_sync(FULL, xc.y, srcOwn);
         const double own = ownY ? owny : ownx;
         const double up = __shfl_up_sync(FULL, c, 1), dn = __shfl_down_sync(FULL, c, 1);
-        const double lo = c8 > 0 ? up : G[olo + 2 * k];
-        const double hi = c8 < 7 ? dn : G[ohi + 2 * k];
+        const double corner = G[ocr + 2 * k];
+        const double lo = c8 > 0 ? up : corner;
+        const double hi = c8 < 7 ? dn : corner;
         const double sum = DADD(DADD(DADD(o, own), DADD(lo, hi)), DADD(bt, tp));
         const double af = DADD(DMUL(alpha, c), DMUL(beta, sum));
         const double fx1 = DADD(c, DMUL(gamma, DSUB(af, bf)));
-        // -- deliver face x0 / face x1 to the own lanes next to the faces
-        const double vwe = __shfl_sync(FULL, c, sWE);
-        double2 vsn;
-        vsn.x = __shfl_sync(FULL, c, sSN);
-        vsn.y = __shfl_sync(FULL, c, sSN + 1);
+        // -- face x0 next to my cells from the slab; face x1 delivered by the face lanes
+        const double vwe = G[fwo + 16 * k];
+        const double2 vsn = lds2(G + fsno + 16 * k);
         fweq[cur][kk] = __shfl_sync(FULL, fx1, sWE);
         fsnq[cur][kk].x = __shfl_sync(FULL, fx1, sSN);
         fsnq[cur][kk].y = __shfl_sync(FULL, fx1, sSN + 1);
