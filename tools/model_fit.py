@@ -38,6 +38,8 @@ def samples(runs):
             elif name == "bottom":
                 if nbot > 1:  # one record per bottom sweep (launched sweeps)
                     name, x = "bottom_sweep", float(nl ** 3)
+                elif lvl < r["levels"] - 1:  # the cluster coarse solve of levels lvl .. L-1
+                    name, x = "coarse_cluster", float(nl ** 3)
                 else:  # the resident kernel: all sweeps in one launch
                     x = nl ** 3 * float(r.get("bottom", 100))
             else:
@@ -78,6 +80,8 @@ def main():
                                                    s[6] != 1 and s[3] in ("c2", "c3_fusion") and s[1] <= 128 ** 3],
         "bottom sweep, launched (paper set)": [s for s in S if s[0] == "bottom_sweep" and s[3] == "fit_paper"],
         "bottom, 100 sweeps in one resident CTA": [s for s in S if s[0] == "bottom"],
+        "coarse levels <= 64 bricks, one cluster launch (x = cells of its top level)":
+            [s for s in S if s[0] == "coarse_cluster"],
         "exchange, self (local copies)": [s for s in S if s[0] == "exchange" and s[3] == "c3"],
     }
     fits = {}
@@ -96,7 +100,7 @@ def main():
                "bottom": 24}.get(key)
         if name.startswith("exchange"):
             lines.append(f"| {name} | {len(ss)} | {a * 1e3:.1f} | — | {b / 1e6:.1f} (bytes) | {mis:.2f} |")
-        elif name.startswith("bottom, 100"):
+        elif name.startswith("bottom, 100") or name.startswith("coarse levels"):
             lines.append(f"| {name} | {len(ss)} | {a * 1e3:.1f} | {b / 1e6:.2f} (pt-sweeps) | — | {mis:.2f} |")
         else:
             gbs = f"{b / 1e6 * bpp:.0f}" if bpp else "—"
