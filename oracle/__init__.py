@@ -56,6 +56,10 @@ def _load():
             "oracle_get_threads": (I, []),
             "oracle_apply_op": (None, [I, I, I, D, P, P]),
             "oracle_smooth": (None, [S, D, P, P, P]),
+            "oracle_smooth_gamma": (None, [S, D, P, P, P]),
+            "oracle_smooth_residual_gamma": (None, [S, D, P, P, P, P]),
+            "oracle_chebyshev_gamma": (D, [D, I, I, I]),
+            "oracle_mg_set_smoother": (None, [P, I, I]),
             "oracle_smooth_residual": (None, [S, D, P, P, P, P]),
             "oracle_restriction": (None, [I, I, I, P, P]),
             "oracle_init_zero": (None, [S, P]),
@@ -126,6 +130,19 @@ def smooth_residual(x: np.ndarray, Ax: np.ndarray, b: np.ndarray, h: float):
     return x, r
 
 
+def smooth_gamma(x: np.ndarray, Ax: np.ndarray, b: np.ndarray, gamma: float) -> np.ndarray:
+    """x + gamma*(Ax - b) with an explicit step (the Chebyshev smoother's sweeps)."""
+    x = _f64(x).copy()
+    Ax, b = _f64(Ax), _f64(b)
+    _load().oracle_smooth_gamma(x.size, float(gamma), _ptr(x), _ptr(Ax), _ptr(b))
+    return x
+
+
+def chebyshev_gamma(h: float, s: int, k: int, rho: int) -> float:
+    """Step of sweep k of an s-sweep Chebyshev smoother over mu in [mu_max/rho, mu_max] (reading A19)."""
+    return float(_load().oracle_chebyshev_gamma(float(h), int(s), int(k), int(rho)))
+
+
 def restriction(r: np.ndarray) -> np.ndarray:
     r = _f64(r)
     nz, ny, nx = r.shape
@@ -164,7 +181,8 @@ def sweep_points(x: np.ndarray, b: np.ndarray, h: float, pts: np.ndarray):
 class OracleMG:
     """Alg 1 / Alg 2 on a global periodic grid of shape (nz, ny, nx)."""
 
-    def __init__(self, shape, levels: int, pre: int = 12, post: int = 12, bottom: int = 100, h0: float | None = None):
+    def __init__(self, shape, levels: int, pre: int = 12, post: int = 12, bottom: int = 100, h0: float | None = None,
+                 smoother: int = 0, cheby_ratio: int = 6):
         nz, ny, nx = (int(s) for s in shape)
         self.shape = (nz, ny, nx)
         self.levels = int(levels)
@@ -173,6 +191,7 @@ class OracleMG:
         self._h = self._lib.oracle_mg_create(nx, ny, nz, self.levels, self.h0, int(pre), int(post), int(bottom))
         if not self._h:
             raise ValueError(f"oracle_mg_create failed for shape={shape} levels={levels}")
+        self._lib.oracle_mg_set_smoother(self._h, int(smoother), int(cheby_ratio))
 
     def close(self):
         if getattr(self, "_h", None):

@@ -20,6 +20,9 @@
  *   interpolation+incr.   P:L69, L123, L135  x^h = x^h + I(x^2h), piecewise constant
  *   V-cycle               P:L144-146 (Alg 2), readings A1-A3 of DESIGN.md
  *   maxNormRes            P:L139-141 (Alg 1), P:L148 (max residual, 1e-10)
+ *   Chebyshev smoother    variant (N4, reading A19): per-sweep steps gamma_k, see
+ *                         oracle_chebyshev_gamma; pinned by the Chebyshev-polynomial
+ *                         error factor on eigenmodes (tests/test_oracle_pins.py)
  *
  * Readings of garbled / silent passages:
  *   - expression order (A8): neighbour sum pairwise by axis
@@ -84,22 +87,46 @@ void oracle_apply_op(int nx, int ny, int nz, double h, const double *x, double *
   }
 }
 
-/* smooth (P:L118, L148): point Jacobi x := x + gamma*(Ax - b), gamma = h^2/12. */
-void oracle_smooth(size_t n, double h, double *x, const double *Ax, const double *b) {
-  const double gamma = (h * h) / 12.0;
+/* smooth with an explicit step: x := x + gamma*(Ax - b) (P:L118, L148 with gamma given). */
+void oracle_smooth_gamma(size_t n, double gamma, double *x, const double *Ax, const double *b) {
 #pragma omp parallel for schedule(static)
   for (size_t p = 0; p < n; ++p) x[p] = x[p] + gamma * (Ax[p] - b[p]);
 }
 
-/* smooth+residual (P:L119, L133, L148): the smooth above and r = b - Ax from the
- * SAME Ax ("simultaneously calculates the residual", P:L133). */
-void oracle_smooth_residual(size_t n, double h, double *x, const double *Ax, const double *b, double *r) {
-  const double gamma = (h * h) / 12.0;
+/* smooth+residual with an explicit step; r = b - Ax from the SAME Ax. */
+void oracle_smooth_residual_gamma(size_t n, double gamma, double *x, const double *Ax, const double *b, double *r) {
 #pragma omp parallel for schedule(static)
   for (size_t p = 0; p < n; ++p) {
     r[p] = b[p] - Ax[p];
     x[p] = x[p] + gamma * (Ax[p] - b[p]);
   }
+}
+
+/* smooth (P:L118, L148): point Jacobi x := x + gamma*(Ax - b), gamma = h^2/12. */
+void oracle_smooth(size_t n, double h, double *x, const double *Ax, const double *b) {
+  oracle_smooth_gamma(n, (h * h) / 12.0, x, Ax, b);
+}
+
+/* smooth+residual (P:L119, L133, L148): the smooth above and r = b - Ax from the
+ * SAME Ax ("simultaneously calculates the residual", P:L133). */
+void oracle_smooth_residual(size_t n, double h, double *x, const double *Ax, const double *b, double *r) {
+  oracle_smooth_residual_gamma(n, (h * h) / 12.0, x, Ax, b, r);
+}
+
+/* Chebyshev smoother variant (the paper names other smoothers as
+ * future work; not in its method).  Reading A19: s sweeps of
+ * non-stationary Richardson x := x + gamma_k (Ax - b) whose steps are the reciprocals of
+ * the Chebyshev nodes of the smoothing interval mu in [mu_max/rho, mu_max], mu = -lambda,
+ * mu_max = 12/h^2 (the damped-Jacobi bound):
+ *   nu_j = theta + delta*cos(pi*(2j+1)/(2s)), theta = (1+1/rho)/2, delta = (1-1/rho)/2,
+ *   gamma_k = h^2 / (12*nu_j(k)),  j(k) = k/2 for even k, s-1-(k-1)/2 for odd k
+ * (small and large steps interleaved).  After the s sweeps the error of every mode is
+ * multiplied by T_s((theta - mu/mu_max)/delta) / T_s(theta/delta). */
+double oracle_chebyshev_gamma(double h, int s, int k, int rho) {
+  const int j = (k % 2 == 0) ? k / 2 : s - 1 - (k - 1) / 2;
+  const double th = 0.5 * (1.0 + 1.0 / (double)rho), de = 0.5 * (1.0 - 1.0 / (double)rho);
+  const double nu = th + de * cos(3.14159265358979323846 * (double)(2 * j + 1) / (double)(2 * s));
+  return (h * h) / (12.0 * nu);
 }
 
 /* restriction: b^{2h} = average of the 8 fine cells of each coarse
@@ -159,6 +186,7 @@ double oracle_max_norm_residual(int nx, int ny, int nz, double h, const double *
 #define ORACLE_MAX_LEVELS 16
 typedef struct {
   int L, pre, post, bottom;
+  int smoother, rho; /* 0 = damped Jacobi (the paper); 1 = Chebyshev (oracle_chebyshev_gamma) on pre/post */
   int n[ORACLE_MAX_LEVELS][3];
   double h[ORACLE_MAX_LEVELS];
   double *x[ORACLE_MAX_LEVELS], *b[ORACLE_MAX_LEVELS], *Ax[ORACLE_MAX_LEVELS], *r[ORACLE_MAX_LEVELS];
@@ -210,6 +238,16 @@ oracle_mg *oracle_mg_create(int nx, int ny, int nz, int L, double h0, int pre, i
   return m;
 }
 
+void oracle_mg_set_smoother(oracle_mg *m, int smoother, int rho) {
+  m->smoother = smoother;
+  m->rho = rho;
+}
+
+/* step of sweep it of n at level l (pre / post smoothing) */
+static double step_gamma(const oracle_mg *m, int l, int n, int it) {
+  return m->smoother ? oracle_chebyshev_gamma(m->h[l], n, it, m->rho) : (m->h[l] * m->h[l]) / 12.0;
+}
+
 void oracle_mg_set_b(oracle_mg *m, const double *b) { memcpy(m->b[0], b, lvl_n(m, 0) * sizeof(double)); }
 void oracle_mg_set_x(oracle_mg *m, const double *x) {
   if (x)
@@ -233,7 +271,7 @@ void oracle_mg_vcycle(oracle_mg *m) {
     const int *n = m->n[l];
     for (int it = 0; it < m->pre; ++it) {                       /* steps 2-6 */
       oracle_apply_op(n[0], n[1], n[2], m->h[l], m->x[l], m->Ax[l]); /* exchange()+applyOp */
-      oracle_smooth_residual(lvl_n(m, l), m->h[l], m->x[l], m->Ax[l], m->b[l], m->r[l]);
+      oracle_smooth_residual_gamma(lvl_n(m, l), step_gamma(m, l, m->pre, it), m->x[l], m->Ax[l], m->b[l], m->r[l]);
     }
     oracle_restriction(n[0], n[1], n[2], m->r[l], m->b[l + 1]); /* step 7 */
     oracle_init_zero(lvl_n(m, l + 1), m->x[l + 1]);             /* step 8 */
@@ -251,7 +289,7 @@ void oracle_mg_vcycle(oracle_mg *m) {
     oracle_interpolation_increment(n[0], n[1], n[2], m->x[l + 1], m->x[l]);
     for (int it = 0; it < m->post; ++it) {
       oracle_apply_op(n[0], n[1], n[2], m->h[l], m->x[l], m->Ax[l]);
-      oracle_smooth_residual(lvl_n(m, l), m->h[l], m->x[l], m->Ax[l], m->b[l], m->r[l]);
+      oracle_smooth_residual_gamma(lvl_n(m, l), step_gamma(m, l, m->post, it), m->x[l], m->Ax[l], m->b[l], m->r[l]);
     }
   }
 }

@@ -330,3 +330,76 @@ def test_sweep_points_matches_full_sweep(oracle_mod):
     pts = np.arange(x.size)
     xn_p, r_p = oracle_mod.sweep_points(x, b, h, pts)
     assert np.array_equal(xn_p, xs.ravel()) and np.array_equal(r_p, r.ravel())
+
+
+# ------------------------------------------------ Chebyshev smoother (N4 variant, reading A19)
+def cheb_T(s, t):
+    """Chebyshev polynomial of the first kind T_s(t) for any real t (textbook closed forms)."""
+    if abs(t) <= 1.0:
+        return np.cos(s * np.arccos(t))
+    v = np.cosh(s * np.arccosh(abs(t)))
+    return v if t > 0 or s % 2 == 0 else -v
+
+
+@pytest.mark.parametrize("s,rho", [(12, 6), (4, 4), (7, 10)])
+def test_chebyshev_error_factor_on_modes(oracle_mod, s, rho):
+    """s Chebyshev sweeps multiply the error of an eigenmode (A u = -mu u) by
+    P(mu) = T_s((theta - mu/mu_max)/delta) / T_s(theta/delta), mu_max = 12/h^2,
+    theta = (1+1/rho)/2, delta = (1-1/rho)/2 -- the polynomial whose roots are the
+    Chebyshev nodes of [mu_max/rho, mu_max].  Computed here from the closed form of T_s,
+    not from the oracle's step formula; a wrong node, scaling or missing sweep fails."""
+    shape = (16, 16, 16)
+    h = 1.0 / 16
+    mu_max = 12.0 / h**2
+    th, de = 0.5 * (1 + 1 / rho), 0.5 * (1 - 1 / rho)
+    for k in [(1, 0, 0), (2, 3, 1), (4, 4, 4), (8, 8, 7)]:
+        u, lam, _ = mode(shape, h, k=k)
+        mu = -lam
+        b = lam * u  # x* = u
+        x = np.zeros(shape)
+        for it in range(s):
+            g = oracle_mod.chebyshev_gamma(h, s, it, rho)
+            x = oracle_mod.smooth_gamma(x, oracle_mod.apply_op(x, h), b, g)
+        P = cheb_T(s, (th - mu / mu_max) / de) / cheb_T(s, th / de)
+        err = x - u  # = P(mu) * (x0 - u) = -P u
+        assert np.abs(err + P * u).max() <= 1e-11 * max(1.0, abs(P)), (k, P)
+        if mu >= mu_max / rho:  # inside the smoothing interval: damped by 1/T_s(theta/delta)
+            assert abs(P) <= 1.0 / cheb_T(s, th / de) * (1 + 1e-9), (k, P)
+
+
+def test_chebyshev_steps_are_node_reciprocals(oracle_mod):
+    """The s steps are exactly the reciprocals of the s Chebyshev nodes (each used once),
+    interleaved small/large; s = 1 with rho -> 1 is the damped-Jacobi step h^2/12."""
+    h, s, rho = 1.0 / 32, 12, 6
+    mu_max = 12.0 / h**2
+    th, de = 0.5 * (1 + 1 / rho), 0.5 * (1 - 1 / rho)
+    nodes = sorted(mu_max * (th + de * np.cos(np.pi * (2 * j + 1) / (2 * s))) for j in range(s))
+    steps = [oracle_mod.chebyshev_gamma(h, s, k, rho) for k in range(s)]
+    assert np.allclose(sorted(1.0 / g for g in steps), nodes, rtol=1e-14)
+    assert steps[0] < steps[1] and steps[2] < steps[1]  # interleaved order
+    assert oracle_mod.chebyshev_gamma(h, 1, 0, 1) == h * h / 12.0
+
+
+def test_chebyshev_vcycle_converges_faster(oracle_mod):
+    """With the same sweep counts the Chebyshev-smoothed V-cycle contracts faster than the
+    paper's damped Jacobi (a property, not a value: the variant must not break the cycle),
+    and smoother = 0 is the paper's cycle bit for bit."""
+    N, L = 32, 3
+    b = mg_inputs.random_rhs((N, N, N), 0)
+    rj = _rho(oracle_mod, N, L, b)
+    mg = oracle_mod.OracleMG((N, N, N), L, smoother=1, cheby_ratio=6)
+    mg.set_b(b)
+    mg.set_x(None)
+    norms = [mg.norm()]
+    for _ in range(6):
+        mg.vcycle()
+        norms.append(mg.norm())
+    rc = float(np.exp(np.mean(np.log([norms[c] / norms[c - 1] for c in range(2, 7)]))))
+    assert rc < rj, (rc, rj)
+    a = oracle_mod.OracleMG((N, N, N), L, smoother=0)
+    c = oracle_mod.OracleMG((N, N, N), L)
+    for m in (a, c):
+        m.set_b(b)
+        m.set_x(None)
+        m.vcycle()
+    assert np.array_equal(a.get_x(), c.get_x())
