@@ -50,6 +50,8 @@ def parse():
     ap.add_argument("--no-graph", action="store_true")
     ap.add_argument("--no-overlap", action="store_true")
     ap.add_argument("--tb", type=int, default=1, help="temporal blocking: two sweeps per HBM pass (sweep2.cu)")
+    ap.add_argument("--smoother", type=int, default=0, help="0 damped Jacobi (the paper), 1 Chebyshev variant (N4)")
+    ap.add_argument("--cheby-ratio", type=int, default=0, help="Chebyshev smoothing interval [mu_max/ratio, mu_max]")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--ref-n", type=int, default=0, help="reference arm: grid side of the bounded sample")
@@ -238,7 +240,8 @@ def main():
     n = a.n
     m = Multigrid((n, n, n), pg, a.levels, a.pre, a.post, a.bottom, ca_period=a.ca_period, fusion=a.fusion,
                   ghost_mode=1 if a.ghost_all else 0, use_graph=not a.no_graph, overlap=not a.no_overlap,
-                  rank=rank, world_size=world, device=local, temporal_blocking=a.tb)
+                  rank=rank, world_size=world, device=local, temporal_blocking=a.tb, smoother=a.smoother,
+                  cheby_ratio=a.cheby_ratio)
     gshape = (n * pg[2], n * pg[1], n * pg[0])
     b_host = torch.from_numpy(mg_inputs.local_sin_rhs(gshape, rank, pg)).pin_memory()
     b_dev = b_host.to(dev)
@@ -358,6 +361,7 @@ def main():
                        "ca_period": a.ca_period or "auto(8)", "ghost_mode": "all" if a.ghost_all else "auto",
                        "cuda_graph": not a.no_graph, "overlap": not a.no_overlap,
                        "temporal_blocking": bool(a.tb),
+                       "smoother": "chebyshev" if a.smoother == 1 else "damped jacobi (paper)",
                        "l2": "no flush: every level-0 field is 1 GiB > 126 MB L2 (inputs larger than L2)",
                        "parallelism": f"3D domain decomposition {pg[0]}x{pg[1]}x{pg[2]}"},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",

@@ -113,7 +113,11 @@ typedef struct {
                                     1 = one-brick-per-CTA kernel only, 2 = streaming kernel on every level */
   int32_t temporal_blocking;     /* 1 = two Jacobi sweeps per HBM pass on streaming levels (sweep2.cu,
                                     bit-identical; default), 0 = one sweep per pass */
-  int32_t reserved[5];
+  int32_t smoother;              /* 0 = damped Jacobi (the paper); 1 = Chebyshev: the pre / post
+                                    sweeps of a level take the steps h^2/(12 nu_k) at the Chebyshev nodes nu_k of
+                                    [1/cheby_ratio, 1] (variant N4, reading A19); the bottom stays Jacobi */
+  int32_t cheby_ratio;           /* smoothing interval mu in [mu_max/cheby_ratio, mu_max]; 0 => 6 */
+  int32_t reserved[3];
   double h0;                     /* finest spacing; <= 0 => 1 / max_d(global N_d) (reading A7) */
 } mg_params;
 

@@ -218,6 +218,7 @@ mg_params normalized(const mg_params* p) {
     }
     q.h0 = m > 0 ? 1.0 / (double)m : 1.0;
   }
+  if (q.cheby_ratio <= 0) q.cheby_ratio = 6;
   return q;
 }
 
@@ -226,6 +227,7 @@ mg_status check_params(const mg_params& p) {
     return set_err(MG_ERR_INVALID_ARG, "pre_smooths must be >= 1 when num_levels > 1 (restriction reads its r)");
   if (p.transport < 0 || p.transport > MG_TRANSPORT_LOCAL) return set_err(MG_ERR_INVALID_ARG, "bad transport");
   if (p.bottom_mode < 0 || p.bottom_mode > MG_BOTTOM_CLUSTER) return set_err(MG_ERR_INVALID_ARG, "bad bottom_mode");
+  if (p.smoother < 0 || p.smoother > 1) return set_err(MG_ERR_INVALID_ARG, "smoother must be 0 (Jacobi) or 1 (Chebyshev)");
   return MG_OK;
 }
 
@@ -292,9 +294,11 @@ mg_status sweep_range(mg_ctx* c, const Op& o, int64_t b0, int64_t b1, cudaStream
   if (b1 <= b0) return MG_OK;
   DevLevel& d = c->dl[o.level];
   const int l = o.level;
+  Coeffs cc = d.c;  // the smoother's step for this sweep (Chebyshev variant) or the level's Jacobi step
+  if (o.g1 > 0) cc.gamma = o.g1;
   if (o.paper) {
-    CKC(c, launch_apply_op(d.x[o.src], d.Ax, d.adj, b0, b1 - b0, d.c, s));
-    CKC(c, launch_smooth(d.x[o.src], d.Ax, d.b, d.r, b0, b1 - b0, d.c, (o.flags & SW_WRITE_R) != 0, s));
+    CKC(c, launch_apply_op(d.x[o.src], d.Ax, d.adj, b0, b1 - b0, cc, s));
+    CKC(c, launch_smooth(d.x[o.src], d.Ax, d.b, d.r, b0, b1 - b0, cc, (o.flags & SW_WRITE_R) != 0, s));
     return MG_OK;
   }
   SweepArgs a{};
@@ -310,7 +314,8 @@ mg_status sweep_range(mg_ctx* c, const Op& o, int64_t b0, int64_t b1, cudaStream
   }
   a.brick0 = b0;
   a.nbricks = b1 - b0;
-  a.c = d.c;
+  a.c = cc;
+  a.gamma2 = o.g2 > 0 ? o.g2 : d.c.gamma;
   if (o.kind == OP_SWEEP2) {  // two sweeps in one pass: the builder only emits it where a plan exists
     for (const auto& pr : d.pairs) {
       if (pr.b0 == b0 && pr.b1 == b1) {
@@ -405,8 +410,12 @@ mg_status exec_op(mg_ctx* c, const Op& o, cudaStream_t s) {
       a.nlev = c->lay.L - o.level;
       for (int l = o.level; l < c->lay.L; ++l) {
         const DevLevel& dl = c->dl[l];
-        a.lv[l - o.level] = {(int)c->lay.lv[l].n_owned, dl.adj, dl.parent, dl.c};
+        a.lv[l - o.level] = {(int)c->lay.lv[l].n_owned, dl.adj, dl.parent, dl.c, dl.h};
       }
+      const mg_params& P = c->lay.p;
+      a.cheb = P.smoother == 1;
+      for (int k = 0; a.cheb && k < P.pre_smooths; ++k) a.nu_pre[k] = cheb_nu(P.pre_smooths, k, P.cheby_ratio);
+      for (int k = 0; a.cheb && k < P.post_smooths; ++k) a.nu_post[k] = cheb_nu(P.post_smooths, k, P.cheby_ratio);
       a.b0 = d.b;
       a.x0 = d.x[o.dst];
       a.pre = c->lay.p.pre_smooths;

@@ -87,8 +87,13 @@ __global__ void __cluster_dims__(kCoarseCtas, 1, 1) __launch_bounds__(kCoarseThr
   for (int l = 0; l < kCoarseMaxLevels; ++l) cur[l] = 0;
   cl.sync();
 
-  // one Jacobi sweep of level l (ping-pong), optionally with r = b - Ax
-  auto sweep = [&](int l, bool write_r) {
+  // step of a pre / post sweep: the level's Jacobi step or, for the Chebyshev variant,
+  // h^2 / (12 nu) with the host's node nu (same IEEE operations as the host's sweep_gamma)
+  auto step = [&](int l, const double* nu, int k) {
+    return a.cheb ? __ddiv_rn(DMUL(a.lv[l].h, a.lv[l].h), DMUL(12.0, nu[k])) : a.lv[l].c.gamma;
+  };
+  // one sweep of level l (ping-pong) with step g, optionally with r = b - Ax
+  auto sweep = [&](int l, bool write_r, double g) {
     const CoarseLevel& L = a.lv[l];
     double* xs = v.x[l][cur[l]];
     double* xd = v.x[l][cur[l] ^ 1];
@@ -108,7 +113,7 @@ __global__ void __cluster_dims__(kCoarseCtas, 1, 1) __launch_bounds__(kCoarseThr
       const double tp = k < 7 ? xs[e + 64] : *at(xs, __ldg(ad + 5), c - 448);
       const double av = stencil_a(xc, w, ee, s, n, bt, tp, L.c.alpha, L.c.beta);
       const double bb = bl[e];
-      xd[e] = DADD(xc, DMUL(L.c.gamma, DSUB(av, bb)));
+      xd[e] = DADD(xc, DMUL(g, DSUB(av, bb)));
       if (write_r) rl[e] = DSUB(bb, av);
     }
     cur[l] ^= 1;
@@ -148,13 +153,13 @@ __global__ void __cluster_dims__(kCoarseCtas, 1, 1) __launch_bounds__(kCoarseThr
 
   const int last = a.nlev - 1;
   for (int l = 0; l < last; ++l) {  // Alg 2 steps 1-8 on levels l0 .. L-2
-    for (int s = 0; s < a.pre; ++s) sweep(l, s == a.pre - 1);
+    for (int s = 0; s < a.pre; ++s) sweep(l, s == a.pre - 1, step(l, a.nu_pre, s));
     restrict_to(l);
   }
-  for (int s = 0; s < a.bottom; ++s) sweep(last, false);  // steps 10-15
-  for (int l = last - 1; l >= 0; --l) {                  // steps 16-23
+  for (int s = 0; s < a.bottom; ++s) sweep(last, false, a.lv[last].c.gamma);  // steps 10-15 (Jacobi)
+  for (int l = last - 1; l >= 0; --l) {                                       // steps 16-23
     interp_from(l);
-    for (int s = 0; s < a.post; ++s) sweep(l, false);
+    for (int s = 0; s < a.post; ++s) sweep(l, false, step(l, a.nu_post, s));
   }
   for (int e = threadIdx.x; e < v.slots[0] * 512; e += T) {  // x of level l0 for the level above
     const int q = (e >> 9) * C + (int)me;

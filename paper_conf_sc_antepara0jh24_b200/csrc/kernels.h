@@ -33,7 +33,8 @@ struct SweepArgs {
   double* bc;            // coarse b (SW_RESTRICT)
   const double* xc;      // coarse x (SW_INTERP)
   int64_t brick0, nbricks;
-  Coeffs c;
+  Coeffs c;        // c.gamma: the step of the (first) sweep
+  double gamma2;   // two-sweep kernels: the step of the second sweep
 };
 
 cudaError_t launch_sweep(const SweepArgs& a, unsigned flags, cudaStream_t s);
@@ -129,11 +130,13 @@ constexpr int kCoarseCtas = 8;
 constexpr int kCoarseThreads = 512;
 constexpr int kCoarseMaxLevels = 8;
 constexpr size_t kCoarseMaxSmem = 200 * 1024;
+constexpr int kCoarseMaxCheb = 32;  // Chebyshev smoother: pre / post sweeps the cluster solve supports
 struct CoarseLevel {
   int nb;                 // bricks (owned == stored: no ghosts)
   const int32_t* adj;     // [nb][8]
   const int32_t* parent;  // [nb] coarse brick * 8 + octant (levels < last)
-  Coeffs c;
+  Coeffs c;               // c.gamma: damped Jacobi step (bottom, and pre / post when cheb == 0)
+  double h;
 };
 struct CoarseArgs {
   int nlev;  // levels l0 .. l0 + nlev - 1; the last one is the bottom
@@ -141,6 +144,8 @@ struct CoarseArgs {
   const double* b0;  // b of level l0 (restricted by the level above)
   double* x0;        // out: x of level l0 after its post-sweeps
   int pre, post, bottom;
+  int cheb;                                          // 1: pre / post steps h^2 / (12 nu)
+  double nu_pre[kCoarseMaxCheb], nu_post[kCoarseMaxCheb];  // Chebyshev nodes in sweep order (host-computed)
 };
 size_t coarse_smem_bytes(const CoarseArgs& a);
 cudaError_t launch_coarse(const CoarseArgs& a, cudaStream_t s);

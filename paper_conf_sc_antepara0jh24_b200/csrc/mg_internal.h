@@ -12,6 +12,8 @@
 // (P:L156).
 #pragma once
 
+#include <cmath>
+
 #include <cstdint>
 #include <string>
 #include <vector>
@@ -77,6 +79,19 @@ struct LevelLayout {
   };
   std::vector<PairTable> pairs;
 };
+
+// Step of sweep k of an s-sweep pre / post phase at spacing h (reading A19): damped
+// Jacobi h^2/12, or the Chebyshev variant h^2/(12 nu_k) with nu_k the Chebyshev nodes of
+// [1/rho, 1], small and large steps interleaved.  Written out from the reading alone; the
+// same IEEE operations on the same host libm give the same bits.
+inline double cheb_nu(int s, int k, int rho) {
+  const int j = (k % 2 == 0) ? k / 2 : s - 1 - (k - 1) / 2;
+  const double th = 0.5 * (1.0 + 1.0 / (double)rho), de = 0.5 * (1.0 - 1.0 / (double)rho);
+  return th + de * std::cos(3.14159265358979323846 * (double)(2 * j + 1) / (double)(2 * s));
+}
+inline double sweep_gamma(const mg_params& p, double h, int s, int k) {
+  return p.smoother == 1 ? (h * h) / (12.0 * cheb_nu(s, k, p.cheby_ratio)) : (h * h) / 12.0;
+}
 
 constexpr int kPairMeta = 11;
 constexpr int kPairCtasPerSm = 4;                   // resident two-sweep CTAs per SM (shared-memory bound)

@@ -48,6 +48,9 @@ bool Builder::pair_ghosts_ok(int l) const {
 }
 
 void Builder::phase(int l, int n, bool zero_first, int last, bool interp_first, int timer) {
+  const double h = lay.p.h0 * (double)(1 << l);
+  // pre / post sweeps take the smoother's steps; the bottom stays damped Jacobi
+  auto step = [&](int s) { return timer == MG_OP_SWEEP ? sweep_gamma(lay.p, h, n, s) : (h * h) / 12.0; };
   const bool g = ghosts(l);
   const int k = period(l);
   const bool paper = fusion(l) == MG_FUSION_PAPER;
@@ -61,6 +64,8 @@ void Builder::phase(int l, int n, bool zero_first, int last, bool interp_first, 
       o.kind = OP_SWEEP2;
       o.level = l;
       o.timer = timer;
+      o.g1 = step(s);
+      o.g2 = step(s + 1);
       const bool ex = g && (S.dx < 2 || S.since + 2 > k);
       if (ex) {
         S.dx = MG_MAX_PERIOD;
@@ -88,6 +93,7 @@ void Builder::phase(int l, int n, bool zero_first, int last, bool interp_first, 
     o.level = l;
     o.paper = paper;
     o.timer = timer;
+    o.g1 = step(s);
     const bool zero = zero_first && s == 0;
     const bool ex = g && !zero && (S.dx < 1 || S.since >= k);
     if (ex) {
@@ -186,6 +192,7 @@ int Builder::coarse_start() const {
   const int bm = lay.p.bottom_mode;
   if (L < 2 || !(bm == MG_BOTTOM_AUTO || bm == MG_BOTTOM_CLUSTER)) return -1;
   if (lay.p.pre_smooths < 1) return -1;
+  if (lay.p.smoother == 1 && (lay.p.pre_smooths > kCoarseMaxCheb || lay.p.post_smooths > kCoarseMaxCheb)) return -1;
   // the deepest run of levels >= 1 without ghosts, paper kernel set excluded, whose first level
   // fits the cluster (<= 8 bricks per CTA) and whose fields fit its shared memory
   int l0 = L;

@@ -35,6 +35,7 @@ struct Op {
   int n = 0;                // OP_BOTTOM_RES: sweeps
   bool zero = false;        // OP_BOTTOM_RES: x == 0 on entry
   int timer = 0;            // MG_OP_*
+  double g1 = 0, g2 = 0;    // smoothing steps of the (first, second) sweep; 0 = the level's Jacobi h^2/12
 };
 
 struct LevelState {

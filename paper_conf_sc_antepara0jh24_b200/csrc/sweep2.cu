@@ -86,7 +86,7 @@ __global__ void __launch_bounds__(P2_THREADS, kPairCtasPerSm)
   const int2 cr = pa.ctas[blockIdx.x];
   const int64_t base = cr.x;
   const int cnt = cr.y;
-  const double alpha = p.c.alpha, beta = p.c.beta, gamma = p.c.gamma;
+  const double alpha = p.c.alpha, beta = p.c.beta, gamma = p.c.gamma, gamma2 = p.gamma2;
   const uint64_t pol_keep = l2_evict_last(), pol_stream = l2_evict_first();
 
   // ---- own-cell role: planes k0 = 2w, k0+1; cell pair (i0, i0+1) of row j ----
@@ -300,8 +300,8 @@ __global__ void __launch_bounds__(P2_THREADS, kPairCtasPerSm)
           const double a0 = stencil_a(xc.x, wv, xc.y, sv.x, nv.x, xb.x, xt.x, alpha, beta);
           const double a1 = stencil_a(xc.y, xc.x, ev, sv.y, nv.y, xb.y, xt.y, alpha, beta);
           double2 y, rv;
-          y.x = DADD(xc.x, DMUL(gamma, DSUB(a0, bb.x)));
-          y.y = DADD(xc.y, DMUL(gamma, DSUB(a1, bb.y)));
+          y.x = DADD(xc.x, DMUL(gamma2, DSUB(a0, bb.x)));
+          y.y = DADD(xc.y, DMUL(gamma2, DSUB(a1, bb.y)));
           rv.x = DSUB(bb.x, a0);
           rv.y = DSUB(bb.y, a1);
           st_hint2(p.xo + g + 64 * k, y, pol_stream);  // never re-read by this pass

@@ -123,7 +123,7 @@ __global__ void __launch_bounds__(32 * kW2WarpsPerSm, 1)
   int(*MT)[kW2Meta] = S.meta[h];
   double* SLb = &S.sl[h][0].xwe[0][0][0][0];
   uint64_t* BAR = S.bar[h];
-  const double alpha = p.c.alpha, beta = p.c.beta, gamma = p.c.gamma;
+  const double alpha = p.c.alpha, beta = p.c.beta, gamma = p.c.gamma, gamma2 = p.gamma2;
   const uint64_t pol_keep = l2_evict_last(), pol_stream = l2_evict_first();
 
   // ---- own footprint: cells (2ip + a, 2jp + c); rows at q0 and q0 + 8 of a plane
@@ -323,10 +323,10 @@ __global__ void __launch_bounds__(32 * kW2WarpsPerSm, 1)
     if (out_emit) {
       const double2 bp0 = B[rp][0], bp1 = B[rp][1];
       double2 z0, z1, r0, r1;
-      z0.x = DADD(yc0.x, DMUL(gamma, DSUB(a[0], bp0.x)));
-      z0.y = DADD(yc0.y, DMUL(gamma, DSUB(a[1], bp0.y)));
-      z1.x = DADD(yc1.x, DMUL(gamma, DSUB(a[2], bp1.x)));
-      z1.y = DADD(yc1.y, DMUL(gamma, DSUB(a[3], bp1.y)));
+      z0.x = DADD(yc0.x, DMUL(gamma2, DSUB(a[0], bp0.x)));
+      z0.y = DADD(yc0.y, DMUL(gamma2, DSUB(a[1], bp0.y)));
+      z1.x = DADD(yc1.x, DMUL(gamma2, DSUB(a[2], bp1.x)));
+      z1.y = DADD(yc1.y, DMUL(gamma2, DSUB(a[3], bp1.y)));
       r0.x = DSUB(bp0.x, a[0]);
       r0.y = DSUB(bp0.y, a[1]);
       r1.x = DSUB(bp1.x, a[2]);

@@ -443,3 +443,50 @@ def test_temporal_blocking_on_off_bitwise(oracle_mod, tb):
     m.set_solution(None)
     check_cycles(m, xs, ns)
     m.close()
+
+
+# ------------------------------------------------- Chebyshev smoother variant (N4, reading A19)
+@pytest.mark.parametrize("kw", [dict(), dict(temporal_blocking=0), dict(fusion=1), dict(temporal_blocking=2),
+                                dict(bottom_mode=1), dict(ghost_mode=1, ca_period=4), dict(sweep_kernel=2),
+                                dict(cheby_ratio=10)])
+def test_chebyshev_smoother_vcycle_bitwise(oracle_mod, kw):
+    """smoother = 1: per-sweep Chebyshev steps in every kernel that sweeps (single, two-sweep
+    passes, paper kernel set, cluster coarse solve, ghost sweeps), bit for bit with the oracle's
+    Chebyshev V-cycle; the bottom stays damped Jacobi."""
+    shape = (64, 64, 64)
+    rho = kw.get("cheby_ratio", 6)
+    b = mg_inputs.random_rhs(shape, 41)
+    orc = oracle_mod.OracleMG(shape, 4, 12, 12, 100, smoother=1, cheby_ratio=rho)
+    orc.set_b(b)
+    orc.set_x(None)
+    xs, ns = [], []
+    for _ in range(2):
+        orc.vcycle()
+        xs.append(orc.get_x())
+        ns.append(orc.norm())
+    m = new(shape, 4, smoother=1, **kw)
+    m.set_rhs(dev(b))
+    m.set_solution(None)
+    check_cycles(m, xs, ns)
+    m.close()
+    orc.close()
+
+
+def test_chebyshev_smoother_loopback_bitwise(oracle_mod):
+    _, solver = _mg()
+    pg, n_local = (2, 2, 1), (32, 32, 32)
+    gshape = (32, 64, 64)
+    b = mg_inputs.random_rhs(gshape, 42)
+    orc = oracle_mod.OracleMG(gshape, 3, 12, 12, 100, smoother=1, cheby_ratio=6)
+    orc.set_b(b)
+    orc.set_x(None)
+    orc.vcycle()
+    g = solver.LoopbackGroup(n_local, pg, num_levels=3, smoother=1)
+    g.set_rhs([dev(mg_inputs.local_block(b, r, pg)) for r in range(g.world_size)])
+    g.set_solution(None)
+    g.vcycle()
+    assert g.residual_norm() == orc.norm()
+    for r in range(g.world_size):
+        assert_bitwise(host(g.get_solution(r)), mg_inputs.local_block(orc.get_x(), r, pg), what=f"rank {r}")
+    g.close()
+    orc.close()

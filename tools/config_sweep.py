@@ -76,9 +76,10 @@ def main():
             json.dump(self, open(a.out, "w"))
 
     out = Out()
-    # config 1: 64^3, L = 4, solve to 1e-10; paper kernel set and fused
+    # config 1: 64^3, L = 4, solve to 1e-10; paper kernel set and fused; Chebyshev smoother variant
     for fu in (1, 3):
         out.append(run("c1", 64, 4, solve=True, fusion=[fu] * 16))
+    out.append(run("c1", 64, 4, solve=True, smoother=1))
     # config 2: 256^3, L = 6; paper kernel set / fused / fused + temporal blocking
     out.append(run("c2", 256, 6, fusion=[1] * 16, temporal_blocking=0))
     out.append(run("c2", 256, 6, fusion=[3] * 16, temporal_blocking=0))
@@ -101,6 +102,8 @@ def main():
     for fu in (1, 2, 3):
         out.append(run("c3_fusion", 512, 6, fusion=[fu] * 16, temporal_blocking=0))
     out.append(run("c3_fusion", 512, 6))
+    out.append(run("c3_fusion", 512, 6, solve=True))
+    out.append(run("c3_fusion", 512, 6, solve=True, smoother=1))
     # config 5 at P = 1: 1024^3, L = 7 (global coarsest 16^3)
     if not a.quick:
         out.append(run("c5", 1024, 7, cycles=3))

@@ -12,12 +12,14 @@ def desc(r):
     parts = []
     fu = r.get("fusion", [0])[0]
     parts.append({0: "fusion auto(full)", 1: "paper kernel set", 2: "fused sweep", 3: "full fusion"}[fu])
-    tb = r.get("temporal_blocking", 1)
+    tb = r.get("temporal_blocking", 1) if fu != 1 else 0
     parts.append({0: "1 sweep/pass", 1: "2 sweeps/pass", 2: "2 sweeps/pass (warp streams)"}[tb])
     if r.get("ghost_mode"):
         parts.append(f"self-exchange k={r['ca_period'][0]}")
     if r.get("pre") is not None:
         parts.append(f"s={r['pre']}")
+    if r.get("smoother") == 1:
+        parts.append("Chebyshev smoother")
     return ", ".join(parts)
 
 
