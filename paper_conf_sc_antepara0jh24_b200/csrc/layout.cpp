@@ -369,9 +369,9 @@ static LevelLayout::PairTable pair_table(const LevelLayout& L, int64_t b0, int64
     v.insert(v.end(), m, m + kPairMeta);
   };
   auto push_run = [&](std::vector<int32_t>& v, const int32_t* run, int64_t len) {
-    push_item(v, adj(run[0], 4), 0);  // warm-up
+    push_item(v, adj(run[0], 4), 2);  // warm-up (only its plane 7 of x1 is needed)
     for (int64_t q = 0; q < len; ++q) push_item(v, run[q], q > 0 ? 1 : 0);
-    push_item(v, adj(run[len - 1], 5), 1);  // cool-down
+    push_item(v, adj(run[len - 1], 5), 1 | 4);  // cool-down (only its plane 0 of x1 is needed)
   };
   const int64_t full = (nch / G) * G;  // chains dealt round-robin
   for (int64_t c = 0; c < full; ++c) push_run(stream[(size_t)(c % G)], chains[(size_t)c].data(), chains[(size_t)c].size());

@@ -63,7 +63,8 @@ struct LevelLayout {
   // range as z-chains, cut into near-equal CTA pieces; each piece is preceded by
   // its warm-up brick (the B neighbour of its first brick) and followed by its
   // cool-down brick (T neighbour of its last): item = (id, flags, W,E,S,N,
-  // SW,NW,SE,NE, parent), flags bit0 = "previous item is a range brick".
+  // SW,NW,SE,NE, parent), flags bit0 = "previous item is a range brick", bit1 = warm-up,
+  // bit2 = cool-down (the kernel computes only the x1 planes the run needs from those).
   //
   // kind 2 (sweep2w.cu): one stream per HALF-WARP, two streams per warp with
   // equal step counts.  A step is one z-plane; item = (id, emit | kb<<8 | ke<<16,

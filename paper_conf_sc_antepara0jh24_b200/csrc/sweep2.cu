@@ -215,62 +215,67 @@ __global__ void __launch_bounds__(P2_THREADS, kPairCtasPerSm)
         mbar_wait(&S.bx[(m + 1) % P2_NX], (uint32_t)(((m + 1) / P2_NX) & 1));
         mbar_wait(&S.bs[(m + 1) % P2_NS], (uint32_t)(((m + 1) / P2_NS) & 1));
       }
+      // a warm-up item contributes only its x1 plane 7 (warp 3), a cool-down item only plane 0 (warp 0)
+      const int fl = S.meta[m % P2_RING][1];
+      const bool idle = ((fl & 2) && w < P2_WARPS - 1) || ((fl & 4) && w > 0);
       const double* X = S.ownx[m % P2_NX];
       const double* NX = S.ownx[(m + 1) % P2_NX];  // stale if no next item (feeds only unused cells)
       const double* G = reinterpret_cast<const double*>(&S.sl[m % P2_NS]);
       const double* N = reinterpret_cast<const double*>(&S.sl[(m + 1) % P2_NS]);
-      const double2 xm = w > 0 ? lds2(X + 64 * (k0 - 1) + q) : lds2(S.cx0[prv] + q);
-      const double2 x0 = lds2(X + 64 * k0 + q);
-      const double2 x1 = lds2(X + 64 * (k0 + 1) + q);
-      const double2 x2 = w < P2_WARPS - 1 ? lds2(X + 64 * (k0 + 2) + q) : lds2(NX + q);
-      // face lane: its face cell's x0 on planes k0-1 .. k0+2
-      const double cm = w > 0 ? G[oc0 + 16 * (k0 - 1)] : S.cface[prv][l];
-      const double cf0 = G[oc0 + 16 * k0], cf1 = G[oc0 + 16 * (k0 + 1)];
-      const double cp = w < P2_WARPS - 1 ? G[oc0 + 16 * (k0 + 2)] : N[oc0];
-      double* Aw = S.A[cur];
+      if (!idle) {
+        const double2 xm = w > 0 ? lds2(X + 64 * (k0 - 1) + q) : lds2(S.cx0[prv] + q);
+        const double2 x0 = lds2(X + 64 * k0 + q);
+        const double2 x1 = lds2(X + 64 * (k0 + 1) + q);
+        const double2 x2 = w < P2_WARPS - 1 ? lds2(X + 64 * (k0 + 2) + q) : lds2(NX + q);
+        // face lane: its face cell's x0 on planes k0-1 .. k0+2
+        const double cm = w > 0 ? G[oc0 + 16 * (k0 - 1)] : S.cface[prv][l];
+        const double cf0 = G[oc0 + 16 * k0], cf1 = G[oc0 + 16 * (k0 + 1)];
+        const double cp = w < P2_WARPS - 1 ? G[oc0 + 16 * (k0 + 2)] : N[oc0];
+        double* Aw = S.A[cur];
 #pragma unroll
-      for (int kk = 0; kk < 2; ++kk) {
-        const int k = k0 + kk;
-        const double2 xc = kk ? x1 : x0, xb = kk ? x0 : xm, xt = kk ? x2 : x1;
-        // -- x1 of this lane's face cell.  Its W/E (or S/N) neighbour pair is {o, own} and the
-        //    other in-plane pair {lo, hi}; IEEE addition is commutative, so
-        //    ((o+own)+(lo+hi))+(b+t) is bit-identical to the canonical ((w+e)+(s+n))+(b+t).
-        const double c = kk ? cf1 : cf0, bt = kk ? cf0 : cm, tp = kk ? cp : cf1;
-        const double o = G[oo0 + 16 * k];
-        const double bf = G[ob0 + obk * k];
-        const double ownx = __shfl_sync(FULL, xc.x, srcOwn), owny = __shfl_sync(FULL, xc.y, srcOwn);
-        const double own = ownY ? owny : ownx;
-        const double up = __shfl_up_sync(FULL, c, 1), dn = __shfl_down_sync(FULL, c, 1);
-        const double corner = G[ocr + 2 * k];
-        const double lo = c8 > 0 ? up : corner;
-        const double hi = c8 < 7 ? dn : corner;
-        const double sum = DADD(DADD(DADD(o, own), DADD(lo, hi)), DADD(bt, tp));
-        const double af = DADD(DMUL(alpha, c), DMUL(beta, sum));
-        const double fx1 = DADD(c, DMUL(gamma, DSUB(af, bf)));
-        // -- face x0 next to my cells from the slab; face x1 delivered by the face lanes
-        const double vwe = G[fwo + 16 * k];
-        const double2 vsn = lds2(G + fsno + 16 * k);
-        fweq[cur][kk] = __shfl_sync(FULL, fx1, sWE);
-        fsnq[cur][kk].x = __shfl_sync(FULL, fx1, sSN);
-        fsnq[cur][kk].y = __shfl_sync(FULL, fx1, sSN + 1);
-        // -- x1 of the own cells
-        const double2 bb = bq[cur][kk];
-        double2 rs_, rn_;  // rows j-1, j+1 of the plane live in lanes l-4, l+4
-        rs_.x = __shfl_up_sync(FULL, xc.x, 4), rs_.y = __shfl_up_sync(FULL, xc.y, 4);
-        rn_.x = __shfl_down_sync(FULL, xc.x, 4), rn_.y = __shfl_down_sync(FULL, xc.y, 4);
-        const double wl = __shfl_up_sync(FULL, xc.y, 1), er = __shfl_down_sync(FULL, xc.x, 1);
-        const double wo = isW ? vwe : wl, eo = isE ? vwe : er;
-        const double2 so = isS ? vsn : rs_, no = isN ? vsn : rn_;
-        const double a0 = stencil_a(xc.x, wo, xc.y, so.x, no.x, xb.x, xt.x, alpha, beta);
-        const double a1 = stencil_a(xc.y, xc.x, eo, so.y, no.y, xb.y, xt.y, alpha, beta);
-        double2 y;
-        y.x = DADD(xc.x, DMUL(gamma, DSUB(a0, bb.x)));
-        y.y = DADD(xc.y, DMUL(gamma, DSUB(a1, bb.y)));
-        *reinterpret_cast<double2*>(Aw + 64 * k + q) = y;
-      }
-      if (w == P2_WARPS - 1) {  // plane 7 carries for the next item's plane 0
-        *reinterpret_cast<double2*>(S.cx0[cur] + q) = x1;
-        S.cface[cur][l] = cf1;
+        for (int kk = 0; kk < 2; ++kk) {
+          const int k = k0 + kk;
+          const double2 xc = kk ? x1 : x0, xb = kk ? x0 : xm, xt = kk ? x2 : x1;
+          // -- x1 of this lane's face cell.  Its W/E (or S/N) neighbour pair is {o, own} and the
+          //    other in-plane pair {lo, hi}; IEEE addition is commutative, so
+          //    ((o+own)+(lo+hi))+(b+t) is bit-identical to the canonical ((w+e)+(s+n))+(b+t).
+          const double c = kk ? cf1 : cf0, bt = kk ? cf0 : cm, tp = kk ? cp : cf1;
+          const double o = G[oo0 + 16 * k];
+          const double bf = G[ob0 + obk * k];
+          const double ownx = __shfl_sync(FULL, xc.x, srcOwn), owny = __shfl_sync(FULL, xc.y, srcOwn);
+          const double own = ownY ? owny : ownx;
+          const double up = __shfl_up_sync(FULL, c, 1), dn = __shfl_down_sync(FULL, c, 1);
+          const double corner = G[ocr + 2 * k];
+          const double lo = c8 > 0 ? up : corner;
+          const double hi = c8 < 7 ? dn : corner;
+          const double sum = DADD(DADD(DADD(o, own), DADD(lo, hi)), DADD(bt, tp));
+          const double af = DADD(DMUL(alpha, c), DMUL(beta, sum));
+          const double fx1 = DADD(c, DMUL(gamma, DSUB(af, bf)));
+          // -- face x0 next to my cells from the slab; face x1 delivered by the face lanes
+          const double vwe = G[fwo + 16 * k];
+          const double2 vsn = lds2(G + fsno + 16 * k);
+          fweq[cur][kk] = __shfl_sync(FULL, fx1, sWE);
+          fsnq[cur][kk].x = __shfl_sync(FULL, fx1, sSN);
+          fsnq[cur][kk].y = __shfl_sync(FULL, fx1, sSN + 1);
+          // -- x1 of the own cells
+          const double2 bb = bq[cur][kk];
+          double2 rs_, rn_;  // rows j-1, j+1 of the plane live in lanes l-4, l+4
+          rs_.x = __shfl_up_sync(FULL, xc.x, 4), rs_.y = __shfl_up_sync(FULL, xc.y, 4);
+          rn_.x = __shfl_down_sync(FULL, xc.x, 4), rn_.y = __shfl_down_sync(FULL, xc.y, 4);
+          const double wl = __shfl_up_sync(FULL, xc.y, 1), er = __shfl_down_sync(FULL, xc.x, 1);
+          const double wo = isW ? vwe : wl, eo = isE ? vwe : er;
+          const double2 so = isS ? vsn : rs_, no = isN ? vsn : rn_;
+          const double a0 = stencil_a(xc.x, wo, xc.y, so.x, no.x, xb.x, xt.x, alpha, beta);
+          const double a1 = stencil_a(xc.y, xc.x, eo, so.y, no.y, xb.y, xt.y, alpha, beta);
+          double2 y;
+          y.x = DADD(xc.x, DMUL(gamma, DSUB(a0, bb.x)));
+          y.y = DADD(xc.y, DMUL(gamma, DSUB(a1, bb.y)));
+          *reinterpret_cast<double2*>(Aw + 64 * k + q) = y;
+        }
+        if (w == P2_WARPS - 1) {  // plane 7 carries for the next item's plane 0
+          *reinterpret_cast<double2*>(S.cx0[cur] + q) = x1;
+          S.cface[cur][l] = cf1;
+        }
       }
     }
     __syncthreads();  // x1 of item m (plane 0 for phase B) and the carries are visible
