@@ -86,11 +86,12 @@ enum {
 /* transport */
 enum { MG_TRANSPORT_AUTO = 0, MG_TRANSPORT_NCCL = 1, MG_TRANSPORT_LOCAL = 2 };
 
-/* bottom_mode.  AUTO: the deepest levels without ghosts that fit (<= 64 bricks per level,
- * <= 200 KB of fields) run as ONE cluster-resident launch (coarse.cu: pre-sweeps, restriction,
- * initZero, bottom, interpolation, post-sweeps of those levels); a lone
- * bottom level of <= 8 bricks runs in one CTA; otherwise per-sweep launches.  All modes are
- * bitwise identical. */
+/* bottom_mode.  AUTO: a bottom level of <= 8 bricks without ghosts runs all its sweeps in one
+ * CTA (resident), otherwise per-sweep launches.  CLUSTER (opt-in): the deepest
+ * levels without ghosts that fit (<= 64 bricks per level, <= 200 KB of fields) run as ONE
+ * 8-CTA cluster launch (coarse.cu: pre-sweeps, restriction, initZero, bottom, interpolation,
+ * post-sweeps of those levels); measured no faster than graph-replayed launches (DESIGN.md
+ * §7.3).  All modes are bitwise identical. */
 enum { MG_BOTTOM_AUTO = 0, MG_BOTTOM_SWEEPS = 1, MG_BOTTOM_RESIDENT = 2, MG_BOTTOM_CLUSTER = 3 };
 
 typedef struct {

@@ -190,7 +190,8 @@ void Builder::bottom(int l, int n, bool zero) {
 int Builder::coarse_start() const {
   const int L = lay.L;
   const int bm = lay.p.bottom_mode;
-  if (L < 2 || !(bm == MG_BOTTOM_AUTO || bm == MG_BOTTOM_CLUSTER)) return -1;
+  // opt-in: measured slower than graph-replayed per-level launches below 512^3
+  if (L < 2 || bm != MG_BOTTOM_CLUSTER) return -1;
   if (lay.p.pre_smooths < 1) return -1;
   if (lay.p.smoother == 1 && (lay.p.pre_smooths > kCoarseMaxCheb || lay.p.post_smooths > kCoarseMaxCheb)) return -1;
   // the deepest run of levels >= 1 without ghosts, paper kernel set excluded, whose first level
@@ -209,7 +210,6 @@ int Builder::coarse_start() const {
     ++l0;
   }
   if (coarse_smem_bytes(a) > kCoarseMaxSmem) return -1;
-  if (l0 == L - 1 && bm == MG_BOTTOM_AUTO && lay.lv[L - 1].n_stored <= kResidentMaxBricks) return -1;  // one CTA does
   return l0;
 }
 

@@ -447,8 +447,8 @@ def test_temporal_blocking_on_off_bitwise(oracle_mod, tb):
 
 # ------------------------------------------------- Chebyshev smoother variant (N4, reading A19)
 @pytest.mark.parametrize("kw", [dict(), dict(temporal_blocking=0), dict(fusion=1), dict(temporal_blocking=2),
-                                dict(bottom_mode=1), dict(ghost_mode=1, ca_period=4), dict(sweep_kernel=2),
-                                dict(cheby_ratio=10)])
+                                dict(bottom_mode=1), dict(bottom_mode=3), dict(ghost_mode=1, ca_period=4),
+                                dict(sweep_kernel=2), dict(cheby_ratio=10)])
 def test_chebyshev_smoother_vcycle_bitwise(oracle_mod, kw):
     """smoother = 1: per-sweep Chebyshev steps in every kernel that sweeps (single, two-sweep
     passes, paper kernel set, cluster coarse solve, ghost sweeps), bit for bit with the oracle's
