@@ -59,6 +59,7 @@ def _load():
             "oracle_smooth_gamma": (None, [S, D, P, P, P]),
             "oracle_smooth_residual_gamma": (None, [S, D, P, P, P, P]),
             "oracle_chebyshev_gamma": (D, [D, I, I, I]),
+            "oracle_gsrb_half": (None, [I, I, I, D, I, P, P, P, P]),
             "oracle_mg_set_smoother": (None, [P, I, I]),
             "oracle_smooth_residual": (None, [S, D, P, P, P, P]),
             "oracle_restriction": (None, [I, I, I, P, P]),
@@ -136,6 +137,16 @@ def smooth_gamma(x: np.ndarray, Ax: np.ndarray, b: np.ndarray, gamma: float) -> 
     Ax, b = _f64(Ax), _f64(b)
     _load().oracle_smooth_gamma(x.size, float(gamma), _ptr(x), _ptr(Ax), _ptr(b))
     return x
+
+
+def gsrb_half(x: np.ndarray, Ax: np.ndarray, b: np.ndarray, h: float, colour: int):
+    """One red (colour 0) or black (1) Gauss-Seidel half-sweep (reading A20); returns (x', r)."""
+    x = _f64(x).copy()
+    Ax, b = _f64(Ax), _f64(b)
+    r = np.empty_like(x)
+    nz, ny, nx = x.shape
+    _load().oracle_gsrb_half(nx, ny, nz, float(h), int(colour), _ptr(x), _ptr(Ax), _ptr(b), _ptr(r))
+    return x, r
 
 
 def chebyshev_gamma(h: float, s: int, k: int, rho: int) -> float:

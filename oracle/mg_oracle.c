@@ -20,6 +20,8 @@
  *   interpolation+incr.   P:L69, L123, L135  x^h = x^h + I(x^2h), piecewise constant
  *   V-cycle               P:L144-146 (Alg 2), readings A1-A3 of DESIGN.md
  *   maxNormRes            P:L139-141 (Alg 1), P:L148 (max residual, 1e-10)
+ *   GSRB smoother         variant (N4, reading A20): red then black Gauss-Seidel half-sweeps,
+ *                         oracle_gsrb_half; pinned against a sparse triangular solve
  *   Chebyshev smoother    variant (N4, reading A19): per-sweep steps gamma_k, see
  *                         oracle_chebyshev_gamma; pinned by the Chebyshev-polynomial
  *                         error factor on eigenmodes (tests/test_oracle_pins.py)
@@ -113,6 +115,23 @@ void oracle_smooth_residual(size_t n, double h, double *x, const double *Ax, con
   oracle_smooth_residual_gamma(n, (h * h) / 12.0, x, Ax, b, r);
 }
 
+/* Red-black Gauss-Seidel half-sweep (GSRB smoother variant, reading A20): from
+ * the same Ax of the whole grid, cells of colour c = (i+j+k) mod 2 (global indices) take the
+ * Gauss-Seidel update x := x + (h^2/6)(Ax - b) (1/|diag| of P:L148's operator); the other colour
+ * keeps x.  If r != NULL, r = b - Ax on every cell (the residual of the x the half-sweep read). */
+void oracle_gsrb_half(int nx, int ny, int nz, double h, int colour, double *x, const double *Ax, const double *b,
+                      double *r) {
+  const double g = (h * h) / 6.0;
+#pragma omp parallel for schedule(static)
+  for (int k = 0; k < nz; ++k)
+    for (int j = 0; j < ny; ++j)
+      for (int i = 0; i < nx; ++i) {
+        const size_t p = IDX(i, j, k, nx, ny);
+        if (r) r[p] = b[p] - Ax[p];
+        if (((i + j + k) & 1) == colour) x[p] = x[p] + g * (Ax[p] - b[p]);
+      }
+}
+
 /* Chebyshev smoother variant (the paper names other smoothers as
  * future work; not in its method).  Reading A19: s sweeps of
  * non-stationary Richardson x := x + gamma_k (Ax - b) whose steps are the reciprocals of
@@ -186,7 +205,8 @@ double oracle_max_norm_residual(int nx, int ny, int nz, double h, const double *
 #define ORACLE_MAX_LEVELS 16
 typedef struct {
   int L, pre, post, bottom;
-  int smoother, rho; /* 0 = damped Jacobi (the paper); 1 = Chebyshev (oracle_chebyshev_gamma) on pre/post */
+  int smoother, rho; /* 0 = damped Jacobi (the paper); 1 = Chebyshev (oracle_chebyshev_gamma) on pre/post;
+                        2 = red-black Gauss-Seidel on pre/post (oracle_gsrb_half: red then black) */
   int n[ORACLE_MAX_LEVELS][3];
   double h[ORACLE_MAX_LEVELS];
   double *x[ORACLE_MAX_LEVELS], *b[ORACLE_MAX_LEVELS], *Ax[ORACLE_MAX_LEVELS], *r[ORACLE_MAX_LEVELS];
@@ -270,6 +290,13 @@ void oracle_mg_vcycle(oracle_mg *m) {
   for (int l = 0; l + 1 < L; ++l) {
     const int *n = m->n[l];
     for (int it = 0; it < m->pre; ++it) {                       /* steps 2-6 */
+      if (m->smoother == 2) {                                    /* GSRB: red half, then black half */
+        for (int c = 0; c < 2; ++c) {
+          oracle_apply_op(n[0], n[1], n[2], m->h[l], m->x[l], m->Ax[l]);
+          oracle_gsrb_half(n[0], n[1], n[2], m->h[l], c, m->x[l], m->Ax[l], m->b[l], m->r[l]);
+        }
+        continue;
+      }
       oracle_apply_op(n[0], n[1], n[2], m->h[l], m->x[l], m->Ax[l]); /* exchange()+applyOp */
       oracle_smooth_residual_gamma(lvl_n(m, l), step_gamma(m, l, m->pre, it), m->x[l], m->Ax[l], m->b[l], m->r[l]);
     }
@@ -288,6 +315,13 @@ void oracle_mg_vcycle(oracle_mg *m) {
     const int *n = m->n[l];
     oracle_interpolation_increment(n[0], n[1], n[2], m->x[l + 1], m->x[l]);
     for (int it = 0; it < m->post; ++it) {
+      if (m->smoother == 2) {
+        for (int c = 0; c < 2; ++c) {
+          oracle_apply_op(n[0], n[1], n[2], m->h[l], m->x[l], m->Ax[l]);
+          oracle_gsrb_half(n[0], n[1], n[2], m->h[l], c, m->x[l], m->Ax[l], m->b[l], m->r[l]);
+        }
+        continue;
+      }
       oracle_apply_op(n[0], n[1], n[2], m->h[l], m->x[l], m->Ax[l]);
       oracle_smooth_residual_gamma(lvl_n(m, l), step_gamma(m, l, m->post, it), m->x[l], m->Ax[l], m->b[l], m->r[l]);
     }
