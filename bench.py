@@ -50,7 +50,8 @@ def parse():
     ap.add_argument("--no-graph", action="store_true")
     ap.add_argument("--no-overlap", action="store_true")
     ap.add_argument("--tb", type=int, default=1, help="temporal blocking: two sweeps per HBM pass (sweep2.cu)")
-    ap.add_argument("--smoother", type=int, default=0, help="0 damped Jacobi (the paper), 1 Chebyshev variant (N4)")
+    ap.add_argument("--smoother", type=int, default=0,
+                    help="0 damped Jacobi (the paper), 1 Chebyshev, 2 red-black Gauss-Seidel (N4 variants)")
     ap.add_argument("--cheby-ratio", type=int, default=0, help="Chebyshev smoothing interval [mu_max/ratio, mu_max]")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
@@ -361,7 +362,7 @@ def main():
                        "ca_period": a.ca_period or "auto(8)", "ghost_mode": "all" if a.ghost_all else "auto",
                        "cuda_graph": not a.no_graph, "overlap": not a.no_overlap,
                        "temporal_blocking": bool(a.tb),
-                       "smoother": "chebyshev" if a.smoother == 1 else "damped jacobi (paper)",
+                       "smoother": {1: "chebyshev", 2: "red-black gauss-seidel"}.get(a.smoother, "damped jacobi (paper)"),
                        "l2": "no flush: every level-0 field is 1 GiB > 126 MB L2 (inputs larger than L2)",
                        "parallelism": f"3D domain decomposition {pg[0]}x{pg[1]}x{pg[2]}"},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",

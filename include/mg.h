@@ -116,7 +116,10 @@ typedef struct {
                                     bit-identical; default), 0 = one sweep per pass */
   int32_t smoother;              /* 0 = damped Jacobi (the paper); 1 = Chebyshev: the pre / post
                                     sweeps of a level take the steps h^2/(12 nu_k) at the Chebyshev nodes nu_k of
-                                    [1/cheby_ratio, 1] (variant N4, reading A19); the bottom stays Jacobi */
+                                    [1/cheby_ratio, 1] (variant N4, reading A19); 2 = red-black
+                                    Gauss-Seidel: each pre / post sweep is a red then a black half-sweep with step
+                                    h^2/6, colour (i+j+k) mod 2, r from the last (black) half-sweep (reading A20).
+                                    The bottom stays damped Jacobi. */
   int32_t cheby_ratio;           /* smoothing interval mu in [mu_max/cheby_ratio, mu_max]; 0 => 6 */
   int32_t reserved[3];
   double h0;                     /* finest spacing; <= 0 => 1 / max_d(global N_d) (reading A7) */

@@ -227,7 +227,8 @@ mg_status check_params(const mg_params& p) {
     return set_err(MG_ERR_INVALID_ARG, "pre_smooths must be >= 1 when num_levels > 1 (restriction reads its r)");
   if (p.transport < 0 || p.transport > MG_TRANSPORT_LOCAL) return set_err(MG_ERR_INVALID_ARG, "bad transport");
   if (p.bottom_mode < 0 || p.bottom_mode > MG_BOTTOM_CLUSTER) return set_err(MG_ERR_INVALID_ARG, "bad bottom_mode");
-  if (p.smoother < 0 || p.smoother > 1) return set_err(MG_ERR_INVALID_ARG, "smoother must be 0 (Jacobi) or 1 (Chebyshev)");
+  if (p.smoother < 0 || p.smoother > 2)
+    return set_err(MG_ERR_INVALID_ARG, "smoother must be 0 (Jacobi), 1 (Chebyshev) or 2 (red-black Gauss-Seidel)");
   return MG_OK;
 }
 
@@ -298,7 +299,7 @@ mg_status sweep_range(mg_ctx* c, const Op& o, int64_t b0, int64_t b1, cudaStream
   if (o.g1 > 0) cc.gamma = o.g1;
   if (o.paper) {
     CKC(c, launch_apply_op(d.x[o.src], d.Ax, d.adj, b0, b1 - b0, cc, s));
-    CKC(c, launch_smooth(d.x[o.src], d.Ax, d.b, d.r, b0, b1 - b0, cc, (o.flags & SW_WRITE_R) != 0, s));
+    CKC(c, launch_smooth(d.x[o.src], d.Ax, d.b, d.r, b0, b1 - b0, cc, (o.flags & SW_WRITE_R) != 0, s, o.c1));
     return MG_OK;
   }
   SweepArgs a{};
@@ -316,6 +317,8 @@ mg_status sweep_range(mg_ctx* c, const Op& o, int64_t b0, int64_t b1, cudaStream
   a.nbricks = b1 - b0;
   a.c = cc;
   a.gamma2 = o.g2 > 0 ? o.g2 : d.c.gamma;
+  a.colour = o.c1;
+  a.colour2 = o.c2;
   if (o.kind == OP_SWEEP2) {  // two sweeps in one pass: the builder only emits it where a plan exists
     for (const auto& pr : d.pairs) {
       if (pr.b0 == b0 && pr.b1 == b1) {

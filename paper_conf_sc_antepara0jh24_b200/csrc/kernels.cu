@@ -147,7 +147,7 @@ __global__ void __launch_bounds__(256) sweep_kernel(SweepArgs p, unsigned long l
       mx = nan_max(mx, fabs(DSUB(bb, a)));
     } else {
       res[ii] = DSUB(bb, a);
-      out[ii] = DADD(c, DMUL(p.c.gamma, DSUB(a, bb)));
+      out[ii] = keep_cell(p.colour, i, j, k) ? c : DADD(c, DMUL(p.c.gamma, DSUB(a, bb)));
     }
   }
 
@@ -351,8 +351,8 @@ __global__ void __launch_bounds__(COL_WARPS * 32, 6)
       const double a0 = stencil_a(xc.x, wv, xc.y, sv.x, nv.x, xm.x, xp.x, p.c.alpha, p.c.beta);
       const double a1 = stencil_a(xc.y, xc.x, ev, sv.y, nv.y, xm.y, xp.y, p.c.alpha, p.c.beta);
       double2 xn, rv;
-      xn.x = DADD(xc.x, DMUL(p.c.gamma, DSUB(a0, bb.x)));
-      xn.y = DADD(xc.y, DMUL(p.c.gamma, DSUB(a1, bb.y)));
+      xn.x = keep_cell(p.colour, i0, j, k) ? xc.x : DADD(xc.x, DMUL(p.c.gamma, DSUB(a0, bb.x)));
+      xn.y = keep_cell(p.colour, i0 + 1, j, k) ? xc.y : DADD(xc.y, DMUL(p.c.gamma, DSUB(a1, bb.y)));
       rv.x = DSUB(bb.x, a0);
       rv.y = DSUB(bb.y, a1);
       st_stream2(p.xo + gbase + 64 * k, xn);
@@ -467,17 +467,18 @@ cudaError_t launch_norm(const double* x, const double* b, const int32_t* adj, in
 template <bool WRITE_R>
 __global__ void __launch_bounds__(256) smooth_kernel(double* __restrict__ x, const double* __restrict__ Ax,
                                                      const double* __restrict__ b, double* __restrict__ r,
-                                                     int64_t base, int64_t n2, double gamma) {
+                                                     int64_t base, int64_t n2, double gamma, int colour) {
   for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < n2; q += (int64_t)gridDim.x * blockDim.x) {
     const int64_t o = base + 2 * q;
     const double2 xv = ldg2(x + o);
     const double2 av = ld_stream2(Ax + o);
     const double2 bv = ld_stream2(b + o);
+    const int c = (int)(o & 511), i = c & 7, j = (c >> 3) & 7, k = c >> 6;
     double2 xn, rv;
     rv.x = DSUB(bv.x, av.x);
     rv.y = DSUB(bv.y, av.y);
-    xn.x = DADD(xv.x, DMUL(gamma, DSUB(av.x, bv.x)));
-    xn.y = DADD(xv.y, DMUL(gamma, DSUB(av.y, bv.y)));
+    xn.x = keep_cell(colour, i, j, k) ? xv.x : DADD(xv.x, DMUL(gamma, DSUB(av.x, bv.x)));
+    xn.y = keep_cell(colour, i + 1, j, k) ? xv.y : DADD(xv.y, DMUL(gamma, DSUB(av.y, bv.y)));
     st_stream2(x + o, xn);
     if (WRITE_R) st_stream2(r + o, rv);
   }
@@ -492,13 +493,13 @@ static unsigned grid_for(int64_t n2) {
 }
 
 cudaError_t launch_smooth(double* x, const double* Ax, const double* b, double* r, int64_t brick0, int64_t nbricks,
-                          Coeffs c, bool write_r, cudaStream_t s) {
+                          Coeffs c, bool write_r, cudaStream_t s, int colour) {
   if (nbricks <= 0) return cudaSuccess;
   const int64_t n2 = nbricks * 256;
   if (write_r)
-    smooth_kernel<true><<<grid_for(n2), 256, 0, s>>>(x, Ax, b, r, brick0 * 512, n2, c.gamma);
+    smooth_kernel<true><<<grid_for(n2), 256, 0, s>>>(x, Ax, b, r, brick0 * 512, n2, c.gamma, colour);
   else
-    smooth_kernel<false><<<grid_for(n2), 256, 0, s>>>(x, Ax, b, r, brick0 * 512, n2, c.gamma);
+    smooth_kernel<false><<<grid_for(n2), 256, 0, s>>>(x, Ax, b, r, brick0 * 512, n2, c.gamma, colour);
   return cudaGetLastError();
 }
 

@@ -33,8 +33,10 @@ struct SweepArgs {
   double* bc;            // coarse b (SW_RESTRICT)
   const double* xc;      // coarse x (SW_INTERP)
   int64_t brick0, nbricks;
-  Coeffs c;        // c.gamma: the step of the (first) sweep
-  double gamma2;   // two-sweep kernels: the step of the second sweep
+  Coeffs c;          // c.gamma: the step of the (first) sweep
+  double gamma2;     // two-sweep kernels: the step of the second sweep
+  int colour = -1;   // red-black half-sweep (GSRB variant): update only cells with (i+j+k) mod 2 == colour,
+  int colour2 = -1;  // keep the others (r still on every cell); -1 = every cell.  colour2: second sweep
 };
 
 cudaError_t launch_sweep(const SweepArgs& a, unsigned flags, cudaStream_t s);
@@ -96,7 +98,7 @@ cudaError_t launch_apply_op(const double* x, double* Ax, const int32_t* adj, int
                             Coeffs c, cudaStream_t s);
 // smooth(+residual) pointwise (paper kernel set): x += gamma (Ax - b); r = b - Ax
 cudaError_t launch_smooth(double* x, const double* Ax, const double* b, double* r, int64_t brick0, int64_t nbricks,
-                          Coeffs c, bool write_r, cudaStream_t s);
+                          Coeffs c, bool write_r, cudaStream_t s, int colour = -1);
 // restriction over fine bricks [0, nfine): bc[parent octant] = avg8(r)
 cudaError_t launch_restrict(const double* r, double* bc, const int32_t* parent, int64_t nfine, cudaStream_t s);
 // interpolation+increment over fine bricks [0, nfine): x += xc(parent)

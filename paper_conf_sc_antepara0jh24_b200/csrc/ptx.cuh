@@ -21,6 +21,12 @@ __device__ __forceinline__ double stencil_a(double c, double w, double e, double
   return DADD(DMUL(alpha, c), DMUL(beta, sum));
 }
 
+// red-black half-sweep (GSRB variant): does the cell keep its x?  Brick edges are even, so the
+// colour of global cell (8 bx + i, ...) is (i + j + k) mod 2 with the in-brick coordinates.
+__device__ __forceinline__ bool keep_cell(int colour, int i, int j, int k) {
+  return colour >= 0 && ((i + j + k) & 1) != colour;
+}
+
 __device__ __forceinline__ double2 ldg2(const double* p) { return __ldg(reinterpret_cast<const double2*>(p)); }
 __device__ __forceinline__ double2 ld_stream2(const double* p) {
   double2 v;

@@ -49,16 +49,24 @@ bool Builder::pair_ghosts_ok(int l) const {
 
 void Builder::phase(int l, int n, bool zero_first, int last, bool interp_first, int timer) {
   const double h = lay.p.h0 * (double)(1 << l);
-  // pre / post sweeps take the smoother's steps; the bottom stays damped Jacobi
-  auto step = [&](int s) { return timer == MG_OP_SWEEP ? sweep_gamma(lay.p, h, n, s) : (h * h) / 12.0; };
+  // pre / post sweeps take the smoother's steps; the bottom stays damped Jacobi.  The red-black
+  // Gauss-Seidel variant (reading A20) turns each of the n sweeps into a red and a black
+  // half-sweep with the Gauss-Seidel step h^2/6; every half-sweep counts as a sweep below.
+  const bool gs = timer == MG_OP_SWEEP && lay.p.smoother == 2;
+  const int nh = gs ? 2 * n : n;
+  auto step = [&](int s) {
+    if (gs) return (h * h) / 6.0;
+    return timer == MG_OP_SWEEP ? sweep_gamma(lay.p, h, n, s) : (h * h) / 12.0;
+  };
+  auto colour = [&](int s) { return gs ? (s & 1) : -1; };
   const bool g = ghosts(l);
   const int k = period(l);
   const bool paper = fusion(l) == MG_FUSION_PAPER;
   const bool pairs = pair_ok(l);
   LevelState& S = st[l];
-  for (int s = 0; s < n; ++s) {
+  for (int s = 0; s < nh; ++s) {
     const bool single_only = (zero_first && s == 0) || (interp_first && s == 0);
-    if (pairs && !single_only && s + 1 < n) {
+    if (pairs && !single_only && s + 1 < nh) {
       // sweeps s and s+1 in one pass (temporal blocking); x1 never leaves the chip
       Op o;
       o.kind = OP_SWEEP2;
@@ -66,6 +74,8 @@ void Builder::phase(int l, int n, bool zero_first, int last, bool interp_first, 
       o.timer = timer;
       o.g1 = step(s);
       o.g2 = step(s + 1);
+      o.c1 = colour(s);
+      o.c2 = colour(s + 1);
       const bool ex = g && (S.dx < 2 || S.since + 2 > k);
       if (ex) {
         S.dx = MG_MAX_PERIOD;
@@ -75,7 +85,7 @@ void Builder::phase(int l, int n, bool zero_first, int last, bool interp_first, 
       // ghost validity after two sweeps over the ghost shell too (x1 needs x0 one cell further
       // out and b at its own depth; x2 likewise from x1): min(d_x - 2, d_b - 1)
       const int d_inc = std::min(S.dx - 2, S.db - 1);
-      const bool last_p = s + 1 == n - 1;
+      const bool last_p = s + 1 == nh - 1;
       o.ghosts = g && !last_p && d_inc >= 1 && (S.since + 2) < k && pair_ghosts_ok(l);
       if (last_p && last == 1) o.flags |= SW_WRITE_R;
       if (last_p && last == 2) o.flags |= SW_RESTRICT;
@@ -94,6 +104,7 @@ void Builder::phase(int l, int n, bool zero_first, int last, bool interp_first, 
     o.paper = paper;
     o.timer = timer;
     o.g1 = step(s);
+    o.c1 = colour(s);
     const bool zero = zero_first && s == 0;
     const bool ex = g && !zero && (S.dx < 1 || S.since >= k);
     if (ex) {
@@ -102,7 +113,7 @@ void Builder::phase(int l, int n, bool zero_first, int last, bool interp_first, 
     }
     o.exch_before = ex;
     const int d_inc = zero ? S.db : std::min(S.dx - 1, S.db);
-    const bool last_s = s == n - 1;
+    const bool last_s = s == nh - 1;
     o.ghosts = g && !last_s && d_inc >= 1 && (S.since + 1) < k;
     if (zero) o.flags |= SW_ZERO_X;
     if (interp_first && s == 0) {
@@ -194,6 +205,7 @@ int Builder::coarse_start() const {
   if (L < 2 || bm != MG_BOTTOM_CLUSTER) return -1;
   if (lay.p.pre_smooths < 1) return -1;
   if (lay.p.smoother == 1 && (lay.p.pre_smooths > kCoarseMaxCheb || lay.p.post_smooths > kCoarseMaxCheb)) return -1;
+  if (lay.p.smoother == 2) return -1;  // red-black half-sweeps: per-level kernels only
   // the deepest run of levels >= 1 without ghosts, paper kernel set excluded, whose first level
   // fits the cluster (<= 8 bricks per CTA) and whose fields fit its shared memory
   int l0 = L;

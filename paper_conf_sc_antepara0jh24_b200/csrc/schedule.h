@@ -36,6 +36,7 @@ struct Op {
   bool zero = false;        // OP_BOTTOM_RES: x == 0 on entry
   int timer = 0;            // MG_OP_*
   double g1 = 0, g2 = 0;    // smoothing steps of the (first, second) sweep; 0 = the level's Jacobi h^2/12
+  int c1 = -1, c2 = -1;     // red-black colour of the (first, second) half-sweep (GSRB); -1 = every cell
 };
 
 struct LevelState {

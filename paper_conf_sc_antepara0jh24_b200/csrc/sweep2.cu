@@ -102,6 +102,8 @@ __global__ void __launch_bounds__(P2_THREADS, kPairCtasPerSm)
   const int fsno = isN ? OXSN + 128 + i0 : OXSN + 8 + i0;
   // ---- face-cell role: face ff (0 W, 1 E, 2 S, 3 N), in-face coordinate c8 ----
   const int ff = l >> 3, c8 = l & 7;
+  // in-brick (i, j) of this lane's face cell in its neighbour brick (the red-black colour)
+  const int fci = ff == 0 ? 7 : ff == 1 ? 0 : c8, fcj = ff == 0 || ff == 1 ? c8 : ff == 2 ? 7 : 0;
   int oc0, oo0, ob0, obk, olo, ohi;  // stage offsets (doubles) at plane 0; slabs step 16 / plane
   if (ff == 0) {         // W brick, cell (7, c8, k): o = (6, c8), own = (0, c8) of my brick
     oc0 = OXWE + 2 * c8 + 1, oo0 = OXWE + 2 * c8, ob0 = OBWE + 2 * c8 + 1, obk = 16;
@@ -250,7 +252,7 @@ __global__ void __launch_bounds__(P2_THREADS, kPairCtasPerSm)
           const double hi = c8 < 7 ? dn : corner;
           const double sum = DADD(DADD(DADD(o, own), DADD(lo, hi)), DADD(bt, tp));
           const double af = DADD(DMUL(alpha, c), DMUL(beta, sum));
-          const double fx1 = DADD(c, DMUL(gamma, DSUB(af, bf)));
+          const double fx1 = keep_cell(p.colour, fci, fcj, k) ? c : DADD(c, DMUL(gamma, DSUB(af, bf)));
           // -- face x0 next to my cells from the slab; face x1 delivered by the face lanes
           const double vwe = G[fwo + 16 * k];
           const double2 vsn = lds2(G + fsno + 16 * k);
@@ -268,8 +270,8 @@ __global__ void __launch_bounds__(P2_THREADS, kPairCtasPerSm)
           const double a0 = stencil_a(xc.x, wo, xc.y, so.x, no.x, xb.x, xt.x, alpha, beta);
           const double a1 = stencil_a(xc.y, xc.x, eo, so.y, no.y, xb.y, xt.y, alpha, beta);
           double2 y;
-          y.x = DADD(xc.x, DMUL(gamma, DSUB(a0, bb.x)));
-          y.y = DADD(xc.y, DMUL(gamma, DSUB(a1, bb.y)));
+          y.x = keep_cell(p.colour, i0, j, k) ? xc.x : DADD(xc.x, DMUL(gamma, DSUB(a0, bb.x)));
+          y.y = keep_cell(p.colour, i0 + 1, j, k) ? xc.y : DADD(xc.y, DMUL(gamma, DSUB(a1, bb.y)));
           *reinterpret_cast<double2*>(Aw + 64 * k + q) = y;
         }
         if (w == P2_WARPS - 1) {  // plane 7 carries for the next item's plane 0
@@ -305,8 +307,8 @@ __global__ void __launch_bounds__(P2_THREADS, kPairCtasPerSm)
           const double a0 = stencil_a(xc.x, wv, xc.y, sv.x, nv.x, xb.x, xt.x, alpha, beta);
           const double a1 = stencil_a(xc.y, xc.x, ev, sv.y, nv.y, xb.y, xt.y, alpha, beta);
           double2 y, rv;
-          y.x = DADD(xc.x, DMUL(gamma2, DSUB(a0, bb.x)));
-          y.y = DADD(xc.y, DMUL(gamma2, DSUB(a1, bb.y)));
+          y.x = keep_cell(p.colour2, i0, j, k) ? xc.x : DADD(xc.x, DMUL(gamma2, DSUB(a0, bb.x)));
+          y.y = keep_cell(p.colour2, i0 + 1, j, k) ? xc.y : DADD(xc.y, DMUL(gamma2, DSUB(a1, bb.y)));
           rv.x = DSUB(bb.x, a0);
           rv.y = DSUB(bb.y, a1);
           st_hint2(p.xo + g + 64 * k, y, pol_stream);  // never re-read by this pass

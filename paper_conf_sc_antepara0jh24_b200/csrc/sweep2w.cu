@@ -164,6 +164,9 @@ __global__ void __launch_bounds__(32 * kW2WarpsPerSm, 1)
   }
   const int bo1 = bo0 + (bks == 16 ? 2 : 1);
   const bool fWE = ff < 2, fswap = pr == 3;
+  // in-brick (i, j) of the two face cells (red-black colour): W (7, c8), E (0, c8), S (c8, 7), N (c8, 0)
+  const int fi0 = ff == 0 ? 7 : ff == 1 ? 0 : 2 * pr, fj0 = ff < 2 ? 2 * pr : ff == 2 ? 7 : 0;
+  const int fi1 = ff < 2 ? fi0 : fi0 + 1, fj1 = ff < 2 ? fj0 + 1 : fj0;
 
   // ---- meta ring (items 0..6) + the pending item 7; barriers; the first two slab stages
   for (int e = hl; e < 7 * kW2Meta / 4; e += 16)
@@ -297,8 +300,10 @@ __global__ void __launch_bounds__(32 * kW2WarpsPerSm, 1)
     const double cc0 = C[rp][0], cc1 = C[rp][1];
     const double up = __shfl_up_sync(FULL, cc1, 1, 16), dn = __shfl_down_sync(FULL, cc0, 1, 16);
     const double lo0 = pr > 0 ? up : corn, hi1 = pr < 3 ? dn : corn;
-    const double fx1a = face_x1(cc0, O[rp][0], own0, lo0, cc1, C[rq][0], C[r][0], bf0, alpha, beta, gamma);
-    const double fx1b = face_x1(cc1, O[rp][1], own1, cc0, hi1, C[rq][1], C[r][1], bf1, alpha, beta, gamma);
+    const double fx1a0 = face_x1(cc0, O[rp][0], own0, lo0, cc1, C[rq][0], C[r][0], bf0, alpha, beta, gamma);
+    const double fx1b0 = face_x1(cc1, O[rp][1], own1, cc0, hi1, C[rq][1], C[r][1], bf1, alpha, beta, gamma);
+    const double fx1a = keep_cell(p.colour, fi0, fj0, k) ? cc0 : fx1a0;
+    const double fx1b = keep_cell(p.colour, fi1, fj1, k) ? cc1 : fx1b0;
 
     // ---- sweep 1, my four cells of plane k
     double a[4];
@@ -306,10 +311,10 @@ __global__ void __launch_bounds__(32 * kW2WarpsPerSm, 1)
     // X[s-2] is dead: x0 of the plane after the next step goes there
     load_x(m1, k1, X[rq]);
     const double2 bc0 = B[r][0], bc1 = B[r][1];
-    Y[r][0].x = DADD(xc0.x, DMUL(gamma, DSUB(a[0], bc0.x)));
-    Y[r][0].y = DADD(xc0.y, DMUL(gamma, DSUB(a[1], bc0.y)));
-    Y[r][1].x = DADD(xc1.x, DMUL(gamma, DSUB(a[2], bc1.x)));
-    Y[r][1].y = DADD(xc1.y, DMUL(gamma, DSUB(a[3], bc1.y)));
+    Y[r][0].x = keep_cell(p.colour, 2 * ip, 2 * jp, k) ? xc0.x : DADD(xc0.x, DMUL(gamma, DSUB(a[0], bc0.x)));
+    Y[r][0].y = keep_cell(p.colour, 2 * ip + 1, 2 * jp, k) ? xc0.y : DADD(xc0.y, DMUL(gamma, DSUB(a[1], bc0.y)));
+    Y[r][1].x = keep_cell(p.colour, 2 * ip, 2 * jp + 1, k) ? xc1.x : DADD(xc1.x, DMUL(gamma, DSUB(a[2], bc1.x)));
+    Y[r][1].y = keep_cell(p.colour, 2 * ip + 1, 2 * jp + 1, k) ? xc1.y : DADD(xc1.y, DMUL(gamma, DSUB(a[3], bc1.y)));
     // face x1 of plane k for the lanes next to the faces (their x2 of plane k, next step)
     GW[r][0] = __shfl_sync(FULL, fx1a, src_we, 16);
     GW[r][1] = __shfl_sync(FULL, fx1b, src_we, 16);
@@ -323,10 +328,11 @@ __global__ void __launch_bounds__(32 * kW2WarpsPerSm, 1)
     if (out_emit) {
       const double2 bp0 = B[rp][0], bp1 = B[rp][1];
       double2 z0, z1, r0, r1;
-      z0.x = DADD(yc0.x, DMUL(gamma2, DSUB(a[0], bp0.x)));
-      z0.y = DADD(yc0.y, DMUL(gamma2, DSUB(a[1], bp0.y)));
-      z1.x = DADD(yc1.x, DMUL(gamma2, DSUB(a[2], bp1.x)));
-      z1.y = DADD(yc1.y, DMUL(gamma2, DSUB(a[3], bp1.y)));
+      const int ko = out_k;
+      z0.x = keep_cell(p.colour2, 2 * ip, 2 * jp, ko) ? yc0.x : DADD(yc0.x, DMUL(gamma2, DSUB(a[0], bp0.x)));
+      z0.y = keep_cell(p.colour2, 2 * ip + 1, 2 * jp, ko) ? yc0.y : DADD(yc0.y, DMUL(gamma2, DSUB(a[1], bp0.y)));
+      z1.x = keep_cell(p.colour2, 2 * ip, 2 * jp + 1, ko) ? yc1.x : DADD(yc1.x, DMUL(gamma2, DSUB(a[2], bp1.x)));
+      z1.y = keep_cell(p.colour2, 2 * ip + 1, 2 * jp + 1, ko) ? yc1.y : DADD(yc1.y, DMUL(gamma2, DSUB(a[3], bp1.y)));
       r0.x = DSUB(bp0.x, a[0]);
       r0.y = DSUB(bp0.y, a[1]);
       r1.x = DSUB(bp1.x, a[2]);

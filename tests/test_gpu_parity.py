@@ -490,3 +490,49 @@ def test_chebyshev_smoother_loopback_bitwise(oracle_mod):
         assert_bitwise(host(g.get_solution(r)), mg_inputs.local_block(orc.get_x(), r, pg), what=f"rank {r}")
     g.close()
     orc.close()
+
+
+# ------------------------------------------------- red-black Gauss-Seidel variant (N4, reading A20)
+@pytest.mark.parametrize("kw", [dict(), dict(temporal_blocking=0), dict(fusion=1), dict(fusion=2),
+                                dict(temporal_blocking=2), dict(bottom_mode=1), dict(ghost_mode=1, ca_period=3),
+                                dict(ghost_mode=1, ca_period=8), dict(sweep_kernel=2)])
+def test_gsrb_smoother_vcycle_bitwise(oracle_mod, kw):
+    """smoother = 2: every pre / post sweep is a red then a black half-sweep (step h^2/6) in the
+    single-sweep, two-sweep (red + black in one pass), paper-set and ghost-shell schedules; bit
+    for bit with the oracle's GSRB V-cycle."""
+    shape = (64, 64, 64)
+    b = mg_inputs.random_rhs(shape, 43)
+    orc = oracle_mod.OracleMG(shape, 4, 12, 12, 100, smoother=2)
+    orc.set_b(b)
+    orc.set_x(None)
+    xs, ns = [], []
+    for _ in range(2):
+        orc.vcycle()
+        xs.append(orc.get_x())
+        ns.append(orc.norm())
+    m = new(shape, 4, smoother=2, **kw)
+    m.set_rhs(dev(b))
+    m.set_solution(None)
+    check_cycles(m, xs, ns)
+    m.close()
+    orc.close()
+
+
+def test_gsrb_smoother_loopback_bitwise(oracle_mod):
+    _, solver = _mg()
+    pg, n_local = (2, 1, 2), (32, 32, 32)
+    gshape = (64, 32, 64)
+    b = mg_inputs.random_rhs(gshape, 44)
+    orc = oracle_mod.OracleMG(gshape, 3, 12, 12, 100, smoother=2)
+    orc.set_b(b)
+    orc.set_x(None)
+    orc.vcycle()
+    g = solver.LoopbackGroup(n_local, pg, num_levels=3, smoother=2)
+    g.set_rhs([dev(mg_inputs.local_block(b, r, pg)) for r in range(g.world_size)])
+    g.set_solution(None)
+    g.vcycle()
+    assert g.residual_norm() == orc.norm()
+    for r in range(g.world_size):
+        assert_bitwise(host(g.get_solution(r)), mg_inputs.local_block(orc.get_x(), r, pg), what=f"rank {r}")
+    g.close()
+    orc.close()

@@ -80,6 +80,7 @@ def main():
     for fu in (1, 3):
         out.append(run("c1", 64, 4, solve=True, fusion=[fu] * 16))
     out.append(run("c1", 64, 4, solve=True, smoother=1))
+    out.append(run("c1", 64, 4, solve=True, smoother=2))
     # config 2: 256^3, L = 6; paper kernel set / fused / fused + temporal blocking
     out.append(run("c2", 256, 6, fusion=[1] * 16, temporal_blocking=0))
     out.append(run("c2", 256, 6, fusion=[3] * 16, temporal_blocking=0))
@@ -104,6 +105,7 @@ def main():
     out.append(run("c3_fusion", 512, 6))
     out.append(run("c3_fusion", 512, 6, solve=True))
     out.append(run("c3_fusion", 512, 6, solve=True, smoother=1))
+    out.append(run("c3_fusion", 512, 6, solve=True, smoother=2))
     # config 5 at P = 1: 1024^3, L = 7 (global coarsest 16^3)
     if not a.quick:
         out.append(run("c5", 1024, 7, cycles=3))

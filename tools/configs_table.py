@@ -18,8 +18,8 @@ def desc(r):
         parts.append(f"self-exchange k={r['ca_period'][0]}")
     if r.get("pre") is not None:
         parts.append(f"s={r['pre']}")
-    if r.get("smoother") == 1:
-        parts.append("Chebyshev smoother")
+    if r.get("smoother") in (1, 2):
+        parts.append({1: "Chebyshev smoother", 2: "red-black Gauss-Seidel smoother"}[r["smoother"]])
     return ", ".join(parts)
 
 
