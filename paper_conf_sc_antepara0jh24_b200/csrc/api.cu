@@ -679,6 +679,7 @@ mg_status mg_workspace_bytes(const mg_params* p, int32_t rank, int32_t world_siz
   Layout lay;
   std::string msg;
   const mg_params q = normalized(p);
+  CKS(check_params(q));
   mg_status s = build_layout(q, rank, world_size, lay, msg);
   if (s != MG_OK) return set_err(s, msg);
   *out_bytes = carve(lay, nullptr, nullptr, nullptr, nullptr);

@@ -79,3 +79,26 @@ def test_workspace_bytes_scales_with_levels():
     a = mg.mg_workspace_bytes(mg.params((64, 64, 64), num_levels=1))
     b = mg.mg_workspace_bytes(mg.params((64, 64, 64), num_levels=4))
     assert b > a and a >= 5 * 64**3 * 8
+
+
+@pytest.mark.parametrize("bad", [dict(smoother=3), dict(smoother=-1), dict(bottom_mode=4), dict(transport=7),
+                                 dict(num_levels=2, pre=0)])
+def test_invalid_parameters_are_rejected_without_a_gpu(bad):
+    """Parameter validation (mg_workspace_bytes, the first call of a setup) rejects unknown
+    smoothers, bottom modes, transports and pre = 0 with more than one level (the restriction
+    reads the last pre-sweep's r) -- MG_ERR_INVALID_ARG with a message, no crash."""
+    from paper_conf_sc_antepara0jh24_b200 import mg
+
+    kw = dict(num_levels=3)
+    kw.update(bad)
+    with pytest.raises(mg.MGError) as e:
+        mg.mg_workspace_bytes(mg.params((64, 64, 64), **kw))
+    assert e.value.status == -1 and str(e.value)
+
+
+@pytest.mark.parametrize("smoother", [0, 1, 2])
+def test_smoother_variants_need_no_extra_workspace(smoother):
+    from paper_conf_sc_antepara0jh24_b200 import mg
+
+    base = mg.mg_workspace_bytes(mg.params((64, 64, 64), num_levels=3))
+    assert mg.mg_workspace_bytes(mg.params((64, 64, 64), num_levels=3, smoother=smoother)) == base
