@@ -21,6 +21,7 @@ enum SweepFlags : unsigned {
   SW_INTERP = 4u,      // read x as x_fine + x_coarse(parent) (interpolation+increment fused)
   SW_ZERO_X = 8u,      // x == 0 (initZero folded into the first coarse sweep)
   SW_NO_SMOOTH = 16u,  // do not write x' (restriction-only last sweep is never used; kept for tests)
+  SW_COLOUR = 32u,     // two-sweep kernel: red-black half-sweeps (colour masks compiled in only here)
 };
 
 struct SweepArgs {

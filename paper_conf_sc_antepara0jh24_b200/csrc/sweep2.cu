@@ -79,9 +79,11 @@ __global__ void __launch_bounds__(P2_THREADS, kPairCtasPerSm)
     sweep2_kernel(SweepArgs p, PairArgs pa, const __grid_constant__ PairMaps mp) {
   constexpr bool WRITE_R = (FLAGS & SW_WRITE_R) != 0;
   constexpr bool RESTRICT = (FLAGS & SW_RESTRICT) != 0;
+  constexpr bool COLOUR = (FLAGS & SW_COLOUR) != 0;  // red-black half-sweeps (GSRB variant)
   constexpr unsigned FULL = 0xffffffffu;
   extern __shared__ __align__(128) unsigned char smem_raw[];
   P2Smem& S = *reinterpret_cast<P2Smem*>(smem_raw);
+  const int col1 = COLOUR ? p.colour : -1, col2 = COLOUR ? p.colour2 : -1;
   const int t = threadIdx.x, w = t >> 5, l = t & 31;
   const int2 cr = pa.ctas[blockIdx.x];
   const int64_t base = cr.x;
@@ -252,7 +254,7 @@ __global__ void __launch_bounds__(P2_THREADS, kPairCtasPerSm)
           const double hi = c8 < 7 ? dn : corner;
           const double sum = DADD(DADD(DADD(o, own), DADD(lo, hi)), DADD(bt, tp));
           const double af = DADD(DMUL(alpha, c), DMUL(beta, sum));
-          const double fx1 = keep_cell(p.colour, fci, fcj, k) ? c : DADD(c, DMUL(gamma, DSUB(af, bf)));
+          const double fx1 = keep_cell(col1, fci, fcj, k) ? c : DADD(c, DMUL(gamma, DSUB(af, bf)));
           // -- face x0 next to my cells from the slab; face x1 delivered by the face lanes
           const double vwe = G[fwo + 16 * k];
           const double2 vsn = lds2(G + fsno + 16 * k);
@@ -270,8 +272,8 @@ __global__ void __launch_bounds__(P2_THREADS, kPairCtasPerSm)
           const double a0 = stencil_a(xc.x, wo, xc.y, so.x, no.x, xb.x, xt.x, alpha, beta);
           const double a1 = stencil_a(xc.y, xc.x, eo, so.y, no.y, xb.y, xt.y, alpha, beta);
           double2 y;
-          y.x = keep_cell(p.colour, i0, j, k) ? xc.x : DADD(xc.x, DMUL(gamma, DSUB(a0, bb.x)));
-          y.y = keep_cell(p.colour, i0 + 1, j, k) ? xc.y : DADD(xc.y, DMUL(gamma, DSUB(a1, bb.y)));
+          y.x = keep_cell(col1, i0, j, k) ? xc.x : DADD(xc.x, DMUL(gamma, DSUB(a0, bb.x)));
+          y.y = keep_cell(col1, i0 + 1, j, k) ? xc.y : DADD(xc.y, DMUL(gamma, DSUB(a1, bb.y)));
           *reinterpret_cast<double2*>(Aw + 64 * k + q) = y;
         }
         if (w == P2_WARPS - 1) {  // plane 7 carries for the next item's plane 0
@@ -307,8 +309,8 @@ __global__ void __launch_bounds__(P2_THREADS, kPairCtasPerSm)
           const double a0 = stencil_a(xc.x, wv, xc.y, sv.x, nv.x, xb.x, xt.x, alpha, beta);
           const double a1 = stencil_a(xc.y, xc.x, ev, sv.y, nv.y, xb.y, xt.y, alpha, beta);
           double2 y, rv;
-          y.x = keep_cell(p.colour2, i0, j, k) ? xc.x : DADD(xc.x, DMUL(gamma2, DSUB(a0, bb.x)));
-          y.y = keep_cell(p.colour2, i0 + 1, j, k) ? xc.y : DADD(xc.y, DMUL(gamma2, DSUB(a1, bb.y)));
+          y.x = keep_cell(col2, i0, j, k) ? xc.x : DADD(xc.x, DMUL(gamma2, DSUB(a0, bb.x)));
+          y.y = keep_cell(col2, i0 + 1, j, k) ? xc.y : DADD(xc.y, DMUL(gamma2, DSUB(a1, bb.y)));
           rv.x = DSUB(bb.x, a0);
           rv.y = DSUB(bb.y, a1);
           st_hint2(p.xo + g + 64 * k, y, pol_stream);  // never re-read by this pass
@@ -352,19 +354,25 @@ cudaError_t launch_sweep2(const SweepArgs& a, const PairArgs& pa, const PairMaps
   if (pa.nctas <= 0) return cudaSuccess;
   const unsigned g = (unsigned)pa.nctas;
   const size_t sm = sizeof(P2Smem);
-  switch (flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP | SW_ZERO_X)) {
+  const unsigned col = (a.colour >= 0 || a.colour2 >= 0) ? SW_COLOUR : 0u;
+  switch ((flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP | SW_ZERO_X)) | col) {
     case 0: sweep2_kernel<0><<<g, P2_THREADS, sm, s>>>(a, pa, pm); break;
     case SW_WRITE_R: sweep2_kernel<SW_WRITE_R><<<g, P2_THREADS, sm, s>>>(a, pa, pm); break;
     case SW_RESTRICT: sweep2_kernel<SW_RESTRICT><<<g, P2_THREADS, sm, s>>>(a, pa, pm); break;
+    case SW_COLOUR: sweep2_kernel<SW_COLOUR><<<g, P2_THREADS, sm, s>>>(a, pa, pm); break;
+    case SW_WRITE_R | SW_COLOUR: sweep2_kernel<SW_WRITE_R | SW_COLOUR><<<g, P2_THREADS, sm, s>>>(a, pa, pm); break;
+    case SW_RESTRICT | SW_COLOUR: sweep2_kernel<SW_RESTRICT | SW_COLOUR><<<g, P2_THREADS, sm, s>>>(a, pa, pm); break;
     default: return cudaErrorInvalidValue;
   }
   return cudaGetLastError();
 }
 
 cudaError_t pair_kernels_init() {
-  const void* k[3] = {(const void*)sweep2_kernel<0>, (const void*)sweep2_kernel<SW_WRITE_R>,
-                      (const void*)sweep2_kernel<SW_RESTRICT>};
-  for (int i = 0; i < 3; ++i) {
+  const void* k[6] = {(const void*)sweep2_kernel<0>, (const void*)sweep2_kernel<SW_WRITE_R>,
+                      (const void*)sweep2_kernel<SW_RESTRICT>, (const void*)sweep2_kernel<SW_COLOUR>,
+                      (const void*)sweep2_kernel<SW_WRITE_R | SW_COLOUR>,
+                      (const void*)sweep2_kernel<SW_RESTRICT | SW_COLOUR>};
+  for (int i = 0; i < 6; ++i) {
     cudaError_t e = cudaFuncSetAttribute(k[i], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(P2Smem));
     if (e != cudaSuccess) return e;
     e = cudaFuncSetAttribute(k[i], cudaFuncAttributePreferredSharedMemoryCarveout, 100);
