@@ -49,7 +49,9 @@ def parse():
     ap.add_argument("--ghost-all", action="store_true", help="self-exchange ghost shell on every axis")
     ap.add_argument("--no-graph", action="store_true")
     ap.add_argument("--no-overlap", action="store_true")
-    ap.add_argument("--tb", type=int, default=1, help="temporal blocking: two sweeps per HBM pass (sweep2.cu)")
+    ap.add_argument("--tb", type=int, default=3,
+                    help="temporal blocking (two sweeps per HBM pass): 3 = 2x2-brick pencils (sweep2p.cu, default), "
+                         "1 = one-brick CTA streams (sweep2.cu), 2 = warp plane streams (sweep2w.cu), 0 = off")
     ap.add_argument("--smoother", type=int, default=0,
                     help="0 damped Jacobi (the paper), 1 Chebyshev, 2 red-black Gauss-Seidel (N4 variants)")
     ap.add_argument("--cheby-ratio", type=int, default=0, help="Chebyshev smoothing interval [mu_max/ratio, mu_max]")
@@ -130,14 +132,15 @@ def measured_peaks():
     return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
 
 
-def ncu_traffic(n):
-    """Per-launch DRAM bytes of the level-0 sweep from the committed ncu --set full summary."""
+def ncu_traffic(n, kernel):
+    """Per-launch DRAM bytes of the level-0 pass kernel from the committed ncu --set full summary
+    (None unless that summary is of the same kernel at the same size)."""
     path = os.path.join(ROOT, "profiles", "ncu_sweep_summary.json")
     if not os.path.exists(path):
         return None
     try:
         d = json.load(open(path))
-        if int(d.get("n", -1)) == n:
+        if int(d.get("n", -1)) == n and d.get("kernel", "").split("<")[0].split()[-1] == kernel:
             return float(d["dram_bytes_per_launch"])
     except Exception:
         pass
@@ -311,7 +314,7 @@ def main():
     # the same level-0 work expressed as one-sweep-per-pass traffic (what the sweeps would move unblocked)
     sweep_equiv = pts * (B_SWEEP * nsweep0 + 2 * B_COARSE_PER_FINE) / (sweep0_ms / 1e3) / 1e9
     peak, peak_src = measured_peaks()
-    traffic = ncu_traffic(n)
+    traffic = ncu_traffic(n, {0: "sweep_col_kernel", 1: "sweep2_kernel", 2: "sweep2w_kernel"}.get(a.tb, "sweep2p_kernel"))
     levels = []
     total_inst = sum(sum(r) for r in tm) / ninst
     for l, row in enumerate(tm):
@@ -361,14 +364,16 @@ def main():
                        "fusion": "auto(full)" if not a.fusion else a.fusion,
                        "ca_period": a.ca_period or "auto(8)", "ghost_mode": "all" if a.ghost_all else "auto",
                        "cuda_graph": not a.no_graph, "overlap": not a.no_overlap,
-                       "temporal_blocking": bool(a.tb),
+                       "temporal_blocking": {0: "off", 1: "one-brick CTA streams", 2: "warp plane streams"}.get(
+                           a.tb, "2x2-brick pencils"),
                        "smoother": {1: "chebyshev", 2: "red-black gauss-seidel"}.get(a.smoother, "damped jacobi (paper)"),
                        "l2": "no flush: every level-0 field is 1 GiB > 126 MB L2 (inputs larger than L2)",
                        "parallelism": f"3D domain decomposition {pg[0]}x{pg[1]}x{pg[2]}"},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic,
-                         "kernel": ("level-0 passes: sweep2_kernel (two sweeps per pass) + sweep_col_kernel / "
-                                    "interp-fused sweep_kernel" if a.tb else
+                         "kernel": ("level-0 passes: %s (two sweeps per pass) + sweep_col_kernel / "
+                                    "interp-fused sweep_kernel" % {1: "sweep2_kernel", 2: "sweep2w_kernel"}.get(
+                                        a.tb, "sweep2p_kernel") if a.tb else
                                     "level-0 sweeps: sweep_col_kernel + interp-fused sweep_kernel"),
                          "passes_per_vcycle": npass0, "launch_ms": launch_ms,
                          "bytes_per_point_per_pass": bytes0 / pts / npass0,

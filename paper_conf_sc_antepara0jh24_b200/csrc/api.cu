@@ -56,6 +56,7 @@ struct DevLevel {
   };
   std::vector<Pair> pairs;  // two-sweep item streams per brick range
   PairMaps pmaps[2];        // tensor maps for the two-sweep kernel reading x[0] / x[1]
+  PairMaps nmaps[2];        // the same with 4-plane boxes for the pencil kernel (sweep2p.cu)
   // local-transport exchange: [x[0] | x[1] | b][recv run] copy descriptors (device), one launch
   CopyRun* cruns = nullptr;
   int ncruns = 0;
@@ -189,6 +190,7 @@ size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double**
       pr.args.nctas = (int64_t)pt.ctas.size() / 2;
       pr.args.warps = (const int4*)take(pt.warps.size() * sizeof(int32_t));
       pr.args.nwarps = (int64_t)pt.warps.size() / 4;
+      pr.args.chunks = (const int32_t*)take(pt.chunks.size() * sizeof(int32_t));
       d.pairs.push_back(pr);
     }
     d.ncruns = (int)L.recvs.size();
@@ -322,7 +324,9 @@ mg_status sweep_range(mg_ctx* c, const Op& o, int64_t b0, int64_t b1, cudaStream
   if (o.kind == OP_SWEEP2) {  // two sweeps in one pass: the builder only emits it where a plan exists
     for (const auto& pr : d.pairs) {
       if (pr.b0 == b0 && pr.b1 == b1) {
-        if (pr.args.kind == 2)
+        if (pr.args.kind == 3)
+          CKC(c, launch_sweep2p(a, pr.args, d.nmaps[o.src], o.flags, s));
+        else if (pr.args.kind == 2)
           CKC(c, launch_sweep2w(a, pr.args, d.pmaps[o.src], o.flags, s));
         else
           CKC(c, launch_sweep2(a, pr.args, d.pmaps[o.src], o.flags, s));
@@ -586,9 +590,14 @@ mg_status init_ctx(mg_ctx* c, const mg_params& p, int rank, int world, int devic
       CKC(c, cudaMemcpyAsync((void*)pa.meta, pt.meta.data(), pt.meta.size() * 4, cudaMemcpyHostToDevice, stream));
       CKC(c, cudaMemcpyAsync((void*)pa.ctas, pt.ctas.data(), pt.ctas.size() * 4, cudaMemcpyHostToDevice, stream));
       CKC(c, cudaMemcpyAsync((void*)pa.warps, pt.warps.data(), pt.warps.size() * 4, cudaMemcpyHostToDevice, stream));
+      CKC(c, cudaMemcpyAsync((void*)pa.chunks, pt.chunks.data(), pt.chunks.size() * 4, cudaMemcpyHostToDevice,
+                             stream));
     }
     if (!L.pairs.empty())
-      for (int xb = 0; xb < 2; ++xb) CKC(c, encode_pair_maps(d.x[xb], d.b, L.n_alloc, &d.pmaps[xb]));
+      for (int xb = 0; xb < 2; ++xb) {
+        CKC(c, encode_pair_maps(d.x[xb], d.b, L.n_alloc, &d.pmaps[xb]));
+        CKC(c, encode_pencil_maps(d.x[xb], d.b, L.n_alloc, &d.nmaps[xb]));
+      }
   }
   CKC(c, cudaStreamSynchronize(stream));  // host vectors above are temporaries
   CKC(c, cudaStreamCreateWithFlags(&c->comm, cudaStreamNonBlocking));
@@ -670,7 +679,7 @@ void mg_params_default(mg_params* p) {
   p->bottom_smooths = 100;
   p->use_graph = 1;
   p->overlap = 1;
-  p->temporal_blocking = 1;
+  p->temporal_blocking = 3;
   p->h0 = 0.0;
 }
 

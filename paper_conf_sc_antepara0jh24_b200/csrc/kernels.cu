@@ -697,6 +697,8 @@ cudaError_t kernels_init() {
   if (e != cudaSuccess) return e;
   e = pair_kernels_init();
   if (e != cudaSuccess) return e;
+  e = pencil_kernels_init();
+  if (e != cudaSuccess) return e;
   e = pairw_kernels_init();
   if (e != cudaSuccess) return e;
   return coarse_kernels_init();

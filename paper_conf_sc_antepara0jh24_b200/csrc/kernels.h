@@ -72,6 +72,7 @@ struct PairArgs {
   int64_t nctas;
   const int4* warps;    // kind 2: (first item half 0, first item half 1, steps, items0 | items1<<16) per warp
   int64_t nwarps;
+  const int32_t* chunks;  // kind 3: chunk codes (item row << 3 | type << 1 | half); ctas = (first chunk, count)
 };
 struct PairMaps {
   CUtensorMap xwe;   // x boxes {2,8,8}: W (i=6,7) / E (i=0,1) face slabs
@@ -89,6 +90,13 @@ cudaError_t pair_kernels_init();
 cudaError_t launch_sweep2w(const SweepArgs& a, const PairArgs& pa, const PairMaps& pm, unsigned flags,
                            cudaStream_t s);
 cudaError_t pairw_kernels_init();
+// 2x2-brick pencil two-sweep kernel (sweep2p.cu): maps with 4-plane boxes ({2,8,4}, {8,2,4},
+// {2,1,4}; b {2,8,4}, {8,1,4}) in the PairMaps fields
+cudaError_t encode_pencil_maps(const double* x, const double* b, int64_t n_alloc, PairMaps* out);
+bool pencil_supports(unsigned flags);
+cudaError_t launch_sweep2p(const SweepArgs& a, const PairArgs& pa, const PairMaps& pm, unsigned flags,
+                           cudaStream_t s);
+cudaError_t pencil_kernels_init();
 
 // true if the streaming kernel implements `flags` (plain, +r, +restriction)
 bool col_supports(unsigned flags);

@@ -265,7 +265,8 @@ mg_status build_layout(const mg_params& p, int rank, int world, Layout& out, std
   for (int l = 0; l < out.L; ++l) build_col_tables(out.lv[l], min_b);
   for (int l = 0; l + 1 < out.L; ++l) build_parents(out.lv[l], out.lv[l + 1]);
   if (p.temporal_blocking != 0)
-    for (int l = 0; l < out.L; ++l) build_pair_tables(out.lv[l], min_b, p.temporal_blocking == 1 ? 1 : 2);
+    for (int l = 0; l < out.L; ++l)
+      build_pair_tables(out.lv[l], min_b, p.temporal_blocking == 2 ? 2 : p.temporal_blocking == 3 ? 3 : 1);
   return MG_OK;
 }
 
@@ -403,6 +404,114 @@ static LevelLayout::PairTable pair_table(const LevelLayout& L, int64_t b0, int64
   return t;
 }
 
+// Chunk streams for the pencil two-sweep kernel (sweep2p.cu), one per resident CTA
+// (G = kPenCtas).  Only for the owned range of a level whose x / y brick counts are even: the
+// owned bricks are cut into 2x2-brick tiles aligned to even owned coordinates (so a tile layer
+// is one coarse brick's x-y extent and the kernel's restriction writes whole coarse columns);
+// a tile column (its z-chain of layers along T) plays the role of a brick chain in pair_table:
+// runs of its layers are dealt round-robin (below).  A run of layers
+// becomes chunks [warm-up layer half 1, (layer half 0, half 1)..., cool-down layer half 0];
+// warm-up / cool-down are the B / T neighbour layers (their x1 planes 7 / 0 are the k-halos of
+// the run's second sweep).  Returns kind 0 if the range does not tile.
+static LevelLayout::PairTable pencil_table(const LevelLayout& L, int64_t b0, int64_t b1) {
+  LevelLayout::PairTable t;
+  t.kind = 0;
+  if (b0 != 0 || b1 != L.n_owned || (L.nb[0] & 1) || (L.nb[1] & 1) || L.n_owned <= 0) return t;
+  auto adj = [&](int64_t id, int f) -> int32_t {
+    return id >= L.n_stored ? (int32_t)L.zero_brick : L.adj[(size_t)id * 8 + f];
+  };
+  auto par = [&](int64_t id) -> int32_t {
+    return (id < L.n_stored && !L.parent.empty()) ? L.parent[(size_t)id] : -1;
+  };
+  const int tx = L.nb[0] / 2, ty = L.nb[1] / 2, nz = L.nb[2];
+  // items of every tile layer: [tile][z]
+  std::vector<std::array<int32_t, kPenMeta>> layers((size_t)tx * ty * nz);
+  auto make_item = [&](int32_t b00) -> std::array<int32_t, kPenMeta> {
+    std::array<int32_t, kPenMeta> m{};
+    const int32_t b10 = adj(b00, 1), b01 = adj(b00, 3), b11 = adj(b10, 3);
+    const int32_t W0 = adj(b00, 0), W1 = adj(b01, 0), E0 = adj(b10, 1), E1 = adj(b11, 1);
+    const int32_t S0 = adj(b00, 2), S1 = adj(b10, 2), N0 = adj(b01, 3), N1 = adj(b11, 3);
+    const int32_t v[17] = {b00, b10, b01, b11, W0, W1, E0, E1, S0, S1, N0, N1,
+                           adj(W0, 2), adj(W1, 3), adj(E0, 2), adj(E1, 3), par(b00)};
+    for (int f = 0; f < 17; ++f) m[(size_t)f] = v[f];
+    return m;
+  };
+  for (int py = 0; py < ty; ++py)
+    for (int px = 0; px < tx; ++px)
+      for (int z = 0; z < nz; ++z) {
+        const int64_t b00 = L.ext_index(2 * px, 2 * py, z);
+        if (b00 < 0 || b00 >= L.n_owned) return t;
+        auto m = make_item((int32_t)b00);
+        // the tile must be the 2x2 block of owned bricks at (2px.., 2py..) and (for restriction)
+        // one coarse brick's octants 0..3 (+4 for odd z)
+        if (m[1] != L.ext_index(2 * px + 1, 2 * py, z) || m[2] != L.ext_index(2 * px, 2 * py + 1, z) ||
+            m[3] != L.ext_index(2 * px + 1, 2 * py + 1, z) || adj(m[2], 1) != m[3])
+          return t;
+        if (m[16] >= 0)
+          for (int k = 1; k < 4; ++k)
+            if (par(m[(size_t)k]) != m[16] + k || (m[16] & 3) != 0) return t;
+        layers[((size_t)py * tx + px) * nz + z] = m;
+      }
+  t.kind = 3;
+  t.b0 = b0;
+  t.b1 = b1;
+  const int64_t ncol = (int64_t)tx * ty;
+  const int64_t G = std::max<int64_t>(1, std::min<int64_t>(kPenCtas, ncol * nz));
+  std::vector<std::vector<int32_t>> stream((size_t)G);  // per CTA: chunk codes (item rows filled below)
+  auto push_item = [&](const std::array<int32_t, kPenMeta>& m) -> int32_t {
+    const int32_t row = (int32_t)(t.meta.size() / kPenMeta);
+    t.meta.insert(t.meta.end(), m.begin(), m.end());
+    return row;
+  };
+  // the B / T neighbour layer of a tile layer (warm-up / cool-down): every brick's B / T link
+  auto shifted = [&](const std::array<int32_t, kPenMeta>& m, int f) {
+    return make_item(adj(m[0], f));
+  };
+  auto push_run = [&](std::vector<int32_t>& v, int64_t col, int z0, int len) {
+    const auto& first = layers[(size_t)col * nz + z0];
+    const auto& last = layers[(size_t)col * nz + ((z0 + len - 1) % nz)];
+    v.push_back((push_item(shifted(first, 4)) << 3) | (1 << 1) | 1);  // warm-up: half 1
+    for (int q = 0; q < len; ++q) {
+      const int32_t row = push_item(layers[(size_t)col * nz + ((z0 + q) % nz)]);
+      v.push_back(row << 3);
+      v.push_back((row << 3) | 1);
+    }
+    v.push_back((push_item(shifted(last, 5)) << 3) | (2 << 1));  // cool-down: half 0
+  };
+  // Units = (z-run, tile column): the column's layers cut into nzr near-equal runs.  Units are
+  // ordered z-run-major, column-minor (x fastest) and dealt round-robin, so the CTAs working at
+  // the same moment hold a compact band of columns at the same height: the side slabs they read
+  // are their neighbours' own bricks, fetched from HBM by the neighbour at about the same time
+  // (L2 hits).  nzr minimises the busiest CTA's work (the kernel is latency-bound, so a CTA's
+  // speed does not depend on how many CTAs share its SM: every CTA must get the same work), in
+  // quarter layers: a run of n layers costs 4n + 1 (its warm-up / cool-down steps).
+  auto zr0 = [&](int nzr, int r) { return (int)((int64_t)r * nz / nzr); };
+  int best = 1;
+  int64_t best_cost = INT64_MAX;
+  for (int nzr = 1; nzr <= nz; ++nzr) {
+    std::vector<int64_t> cta((size_t)G, 0);
+    for (int64_t u = 0; u < ncol * nzr; ++u) {
+      const int r = (int)(u / ncol);
+      cta[(size_t)(u % G)] += 4 * (zr0(nzr, r + 1) - zr0(nzr, r)) + 1;
+    }
+    const int64_t cost = *std::max_element(cta.begin(), cta.end());
+    if (cost < best_cost) best_cost = cost, best = nzr;
+  }
+  for (int64_t u = 0; u < ncol * best; ++u) {
+    const int r = (int)(u / ncol);
+    const int64_t col = u % ncol;
+    push_run(stream[(size_t)(u % G)], col, zr0(best, r), zr0(best, r + 1) - zr0(best, r));
+  }
+  for (int64_t g = 0; g < G; ++g) {
+    const auto& v = stream[(size_t)g];
+    if (v.empty()) continue;
+    t.ctas.push_back((int32_t)t.chunks.size());
+    t.ctas.push_back((int32_t)v.size());
+    t.chunks.insert(t.chunks.end(), v.begin(), v.end());
+  }
+  return t;
+}
+
 // Plane streams for the warp two-sweep kernel (sweep2w.cu), one per half-warp
 // (G = kW2Streams, even).  Chains are dealt round-robin and the remainder cut
 // into equal pieces exactly as in pair_table; each run becomes
@@ -508,7 +617,10 @@ void build_pair_tables(LevelLayout& L, int64_t min_bricks, int kind) {
     bool dup = false;
     for (auto& c : L.pairs) dup |= (c.b0 == r[0] && c.b1 == r[1]);
     if (dup) continue;
-    LevelLayout::PairTable t = kind == 2 ? warp_table(L, r[0], r[1]) : pair_table(L, r[0], r[1]);
+    LevelLayout::PairTable t;
+    t.kind = 0;
+    if (kind == 3) t = pencil_table(L, r[0], r[1]);
+    if (t.kind == 0) t = kind == 2 ? warp_table(L, r[0], r[1]) : pair_table(L, r[0], r[1]);
     if (t.kind != 0) L.pairs.push_back(std::move(t));
   }
 }

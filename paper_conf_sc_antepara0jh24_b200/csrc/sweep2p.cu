@@ -1,0 +1,391 @@
+// sweep2p.cu -- two Jacobi sweeps per HBM pass over 2x2-brick pencils (temporal blocking,
+// SURVEY §8(f) N1; third design).
+//
+// The paper deepens the ghost zone to a brick so several smooths run per exchange
+// (P:L156); this kernel applies the idea on chip: x0 -> x1 -> x2 in one pass over HBM
+// (read x0, b; write x2: 24 B per point for TWO sweeps).  Each sweep is exactly the
+// canonical smooth(+residual) of kernels.cu (reading A8), so x2 is bit-identical to two
+// separate sweeps.
+//
+// Data flow (why it is shaped like this: DESIGN.md §7.1).  A CTA of two warps walks a
+// stream of half-layer CHUNKS of 2x2-brick pencils (layout.cpp pencil_table):
+// [warm-up half, (layer half 0, half 1)..., cool-down half] per run of a tile column.
+//   * A chunk = 4 z-planes of the 16x16-cell tile.  Lanes 0-23 of warp 0 stage it by TMA
+//     into a 2-stage shared-memory ring (one mbarrier per stage): the four own x0 bricks'
+//     planes (1D bulk, 2 KB each), the 2-cell-deep x0 slabs of the 8 side neighbours
+//     (3D tensor boxes {2,8,4} / {8,2,4}), their b faces, the 4 diagonal corner columns.
+//   * The k-direction lives in registers: a lane owns a 2x2 cell footprint of the tile
+//     (pair column p = lane & 7, row pair jp = lane >> 3, warp = brick row), keeps x0 of
+//     planes g-1..g+1 and x1 of planes g-2..g, and per step g
+//       - sweep 1 on plane g: x1 of its 4 cells (S/N rows by LDS.128 from the staged bricks,
+//         W/E by shuffles, tile edges from the slabs), published to a 2-plane x1 buffer;
+//       - x1 of ONE ring cell (the redundant 1-cell ring around the tile the second sweep
+//         needs: warp 0 = W/E rows 0-7 + the S row, warp 1 = W/E rows 8-15 + the N row);
+//       - sweep 2 on plane g-1 from the x1 registers and the x1 buffer, streamed to HBM with
+//         r or the restricted coarse b (the 2x2 footprint is exactly one coarse column, so the
+//         2x2x2 restriction sum forms in registers).
+//   * b of the own cells by 128-bit loads two planes ahead; one CTA barrier per plane.
+// Every cell of a 2x2-brick tile moves 24 B per pass from HBM; through the SM's shared-memory
+// crossbar it moves about half of what sweep2.cu's one-brick items move (no k-plane
+// re-reads, no x1 round trip for own cells, a 25% instead of 50% redundant ring).
+#include <cudaTypedefs.h>
+
+#include <type_traits>
+
+#include "kernels.h"
+#include "mg_internal.h"
+#include "ptx.cuh"
+
+namespace mgb {
+
+namespace {
+
+constexpr int PN_ST = 2;          // TMA stages (half-layer chunks): chunk c+1 lands while chunk c is swept
+constexpr int PN_MINB = 6;        // resident CTAs per SM (37.4 KB of shared memory each; <= 168 registers)
+constexpr int PN_THREADS = 64;    // two warps: warp w = brick row w of the tile
+// stage layout, offsets in doubles.  Own bricks q = bx + 2 by at 264 q (2112 B apart: the two
+// bricks of a tile row sit 64 B apart modulo 128, so a quarter-warp's 128-bit loads of one tile
+// row hit all 32 banks); tensor-copy destinations 128-byte aligned.
+constexpr int OWN_STRIDE = 264;
+constexpr int XW = 1056, XE = 1184, XS = 1312, XN = 1440;  // 2 boxes of 64 each: x0 slabs
+constexpr int BW = 1568, BE = 1696;                        // 2 boxes of 64: b of the W / E bricks
+constexpr int BS = 1824, BN = 1888;                        // 2 boxes of 32: b of the S / N bricks
+constexpr int COR = 1952;                                  // 4 boxes of 8 (16 apart): SW, NW, SE, NE
+constexpr int STAGE = 2016;
+constexpr int CHUNK_BYTES = 4 * 2048 + 8 * 512 + 4 * 512 + 4 * 256 + 4 * 64;
+constexpr int PUB = 18 * 16;  // x1 of tile rows -1..16 (rows -1 / 16: the S / N ring)
+static_assert(STAGE * 8 % 128 == 0 && XW * 8 % 128 == 0 && BS * 8 % 128 == 0 && COR * 8 % 128 == 0, "align");
+static_assert(3 * OWN_STRIDE + 256 <= XW, "own bricks fit");
+__device__ __forceinline__ double2 lds_d2(const double* p) { return *reinterpret_cast<const double2*>(p); }
+constexpr size_t SMEM_BYTES = (size_t)(PN_ST * STAGE + 2 * PUB + 2 * 32) * 8 + PN_ST * 8;
+
+}  // namespace
+
+template <unsigned FLAGS>
+__global__ void __launch_bounds__(PN_THREADS, PN_MINB)
+    sweep2p_kernel(SweepArgs p, PairArgs pa, const __grid_constant__ PairMaps mp) {
+  constexpr bool WRITE_R = (FLAGS & SW_WRITE_R) != 0;
+  constexpr bool RESTRICT = (FLAGS & SW_RESTRICT) != 0;
+  constexpr bool COLOUR = (FLAGS & SW_COLOUR) != 0;  // red-black half-sweeps (GSRB variant)
+  constexpr unsigned FULL = 0xffffffffu;
+  constexpr int RANGE = 0, WARM = 1, COOL = 2;
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  double* const ST = reinterpret_cast<double*>(smem_raw);  // [PN_ST][STAGE]
+  double* const XP = ST + PN_ST * STAGE;                    // [2][PUB]  x1 of tile rows -1..16
+  double* const RWE = XP + 2 * PUB;                         // [2][2][16] x1 of the W / E ring columns
+  uint64_t* const BAR = reinterpret_cast<uint64_t*>(RWE + 64);
+  const int col1 = COLOUR ? p.colour : -1, col2 = COLOUR ? p.colour2 : -1;
+  const int t = threadIdx.x, w = t >> 5, l = t & 31;
+  const int2 cr = pa.ctas[blockIdx.x];
+  const int32_t* CH = pa.chunks + cr.x;  // chunk codes: item row << 3 | type << 1 | half
+  const int cnt = cr.y;
+  const double alpha = p.c.alpha, beta = p.c.beta, gamma = p.c.gamma, gamma2 = p.gamma2;
+  const uint64_t pol_keep = l2_evict_last(), pol_stream = l2_evict_first();
+
+  // ---- own-cell role: cells (2p + a, 8w + 2jp + r) of the tile ----
+  const int pc = l & 7, jp = l >> 3, bx = pc >> 2, ib = 2 * (pc & 3), jb = 2 * jp, q = bx + 2 * w;
+  const int oO = OWN_STRIDE * q + 8 * jb + ib;  // row jb of brick q at plane 0; row jb+1 at +8
+  int oS, sS, oN, sN;                           // S row (jb-1) / N row (jb+2) pair at plane 0, plane stride
+  if (jb > 0) oS = oO - 8, sS = 64;
+  else if (w == 1) oS = OWN_STRIDE * (q - 2) + 56 + ib, sS = 64;
+  else oS = XS + 64 * bx + 8 + ib, sS = 16;  // S slab row j = 7
+  if (jb < 6) oN = oO + 16, sN = 64;
+  else if (w == 0) oN = OWN_STRIDE * (q + 2) + ib, sN = 64;
+  else oN = XN + 64 * bx + ib, sN = 16;  // N slab row j = 0
+  const bool edW = pc == 0, edE = pc == 7;
+  const int oEd = edW ? XW + 64 * w + 2 * jb + 1 : XE + 64 * w + 2 * jb;  // tile-edge W / E x0 (rows jb, jb+1: +2)
+  const int R0 = 8 * w + jb;                                              // tile row of my row 0
+  const int pO = (R0 + 1) * 16 + 2 * pc;                                  // my row 0 in the x1 buffer
+  const int oRwe = (edW ? 0 : 16) + R0;                                   // ring x1 column, rows R0, R0+1
+
+  // ---- ring role: x1 of one cell of the 1-cell ring around the tile ----
+  int oc, oo, oown, olo, slo, ohi, shi, ob, sb, oout, rstr, rci, rcj;
+  if (l < 16) {  // W (lanes 0-7) / E (8-15) face, tile row 8w + j
+    const int side = l >> 3, j = l & 7, cc = side ? 0 : 1;
+    const int X = side ? XE : XW;
+    oc = X + 64 * w + 2 * j + cc;
+    oo = X + 64 * w + 2 * j + (cc ^ 1);
+    oown = OWN_STRIDE * (2 * w + side) + 8 * j + (side ? 7 : 0);
+    if (j > 0) olo = oc - 2, slo = 16;
+    else if (w == 1) olo = X + 14 + cc, slo = 16;
+    else olo = COR + (side ? 32 : 0) + cc, slo = 2;  // SW / SE corner
+    if (j < 7) ohi = oc + 2, shi = 16;
+    else if (w == 0) ohi = X + 64 + cc, shi = 16;
+    else ohi = COR + (side ? 48 : 16) + cc, shi = 2;  // NW / NE corner
+    ob = (side ? BE : BW) + 64 * w + 2 * j + cc, sb = 16;
+    oout = 2 * PUB + 16 * side + 8 * w + j, rstr = 32;  // RWE[par][side][row] (RWE = XP + 2 PUB)
+    rci = side ? 0 : 7, rcj = j;
+  } else {  // S (warp 0) / N (warp 1) row, tile column i
+    const int i = l - 16, i8 = i & 7, bxr = i >> 3;
+    const bool S = w == 0;
+    const int X = S ? XS : XN, rowc = S ? 8 : 0, rowo = S ? 0 : 8;
+    oc = X + 64 * bxr + rowc + i8;
+    oo = X + 64 * bxr + rowo + i8;
+    oown = S ? OWN_STRIDE * bxr + i8 : OWN_STRIDE * (2 + bxr) + 56 + i8;
+    if (i > 0) olo = X + 64 * ((i - 1) >> 3) + rowc + ((i - 1) & 7), slo = 16;
+    else olo = COR + (S ? 0 : 16) + 1, slo = 2;  // SW / NW corner (i = 7)
+    if (i < 15) ohi = X + 64 * ((i + 1) >> 3) + rowc + ((i + 1) & 7), shi = 16;
+    else ohi = COR + (S ? 32 : 48), shi = 2;  // SE / NE corner (i = 0)
+    ob = (S ? BS : BN) + 32 * bxr + i8, sb = 8;
+    oout = (S ? 0 : 17 * 16) + i, rstr = PUB;  // XP[par][row -1 / 16][i]
+    rci = i8, rcj = S ? 7 : 0;
+  }
+
+  if (t == 0) {
+    for (int s = 0; s < PN_ST; ++s) mbar_init(&BAR[s], 1);
+    mbar_fence_init();
+  }
+  __syncthreads();
+
+  // ---- producer: lanes 0-23 of warp 0, one TMA copy each per chunk ----
+  const int mi = l < 12 ? l : l - 8;  // meta field of my copy: own 0-3, W0..N1 4-11, corners 12-15
+  int issued = 0, ic = 0, ic1 = 0, im = 0;
+  if (w == 0 && cnt > 0) {
+    ic = CH[0];
+    ic1 = cnt > 1 ? CH[1] : 0;
+    im = l < 24 ? pa.meta[(int64_t)(ic >> 3) * kPenMeta + mi] : 0;
+  }
+  auto issue = [&]() {  // warp 0 (uniform): stage chunk `issued`
+    const int n = issued, s = n % PN_ST, half = ic & 1;
+    double* D = ST + s * STAGE;
+    fence_proxy_async();
+    if (l == 0) mbar_expect_tx(&BAR[s], CHUNK_BYTES);
+    __syncwarp();
+    const int kz = im * 8 + 4 * half;
+    if (l < 4) {
+      // evict_last: the neighbour tiles' slab copies read these bricks' faces shortly after
+      tma_load_1d_hint(D + OWN_STRIDE * l, p.x + (int64_t)im * 512 + 256 * half, 2048, &BAR[s], pol_keep);
+    } else if (l < 12) {
+      const bool xf = l < 8, lowside = ((l - 4) & 2) == 0;  // W / S boxes sit at the high face
+      tma_load_3d(D + XW + 64 * (l - 4), xf ? &mp.xwe : &mp.xsn, xf && lowside ? 6 : 0, !xf && lowside ? 6 : 0,
+                  kz, &BAR[s]);
+    } else if (l < 16) {
+      tma_load_3d(D + BW + 64 * (l - 12), &mp.bwe, l < 14 ? 6 : 0, 0, kz, &BAR[s]);
+    } else if (l < 20) {
+      tma_load_3d(D + BS + 32 * (l - 16), &mp.bsn, 0, l < 18 ? 7 : 0, kz, &BAR[s]);
+    } else if (l < 24) {  // SW (6,7), NW (6,0), SE (0,7), NE (0,0)
+      const int cc = l - 20;
+      tma_load_3d(D + COR + 16 * cc, &mp.xcor, cc < 2 ? 6 : 0, (cc & 1) ? 0 : 7, kz, &BAR[s]);
+    }
+    ++issued;
+    ic = ic1;
+    if (issued < cnt && l < 24) im = pa.meta[(int64_t)(ic >> 3) * kPenMeta + mi];
+    if (issued + 1 < cnt) ic1 = CH[issued + 1];
+  };
+  int nwait = 0;
+  auto need = [&](int n) {
+    while (nwait <= n) {
+      mbar_wait(&BAR[nwait % PN_ST], (uint32_t)((nwait / PN_ST) & 1));
+      ++nwait;
+    }
+  };
+
+  // ---- per-chunk metadata (uniform): code, my brick id, parent of b00; chunks c-1, c, c+1 ----
+  auto meta_at = [&](int code, int f) { return pa.meta[(int64_t)(code >> 3) * kPenMeta + f]; };
+  int codeP = 0, idP = 0, parP = 0;
+  int codeC = 0, idC = 0, parC = 0, codeN = 0, idN = 0, parN = 0, codeNN = 0;
+  if (cnt > 0) codeC = CH[0], idC = meta_at(codeC, q), parC = meta_at(codeC, 16);
+  if (cnt > 1) codeN = CH[1], idN = meta_at(codeN, q), parN = meta_at(codeN, 16);
+  if (cnt > 2) codeNN = CH[2];
+
+  // ---- registers: x0 planes g-1, g, g+1; x1 planes g-2, g-1, g; b of planes g-1 .. g+2 ----
+  double2 Xm[2], Xc[2], Xp[2], Ym[2], Yc[2], Y[2], B[4][2];
+  double rcm = 0.0, rc = 0.0, rcp = 0.0, rpart = 0.0;
+#pragma unroll
+  for (int r = 0; r < 2; ++r) {
+    Xm[r] = Xc[r] = Xp[r] = Ym[r] = Yc[r] = Y[r] = make_double2(0.0, 0.0);
+#pragma unroll
+    for (int s = 0; s < 4; ++s) B[s][r] = make_double2(0.0, 0.0);
+  }
+  auto load_b = [&](double2* dst, int id, int code, int kk) {
+    const double* bp = p.b + (int64_t)id * 512 + 64 * (4 * (code & 1) + kk) + 8 * jb + ib;
+    dst[0] = ld_hint2(bp, pol_keep);  // the neighbour tiles' b-face copies reuse these lines from L2
+    dst[1] = ld_hint2(bp + 8, pol_keep);
+  };
+
+  // one step: sweep 1 on plane g = 4c + kk, sweep 2 on plane g - 1 (if it is a range plane)
+  auto step = [&](const int c, auto kkc, const bool start, const bool sw2, const bool pref) {
+    constexpr int kk = decltype(kkc)::value;
+    const double* S0 = ST + (c % PN_ST) * STAGE;
+    need(c);
+    if (kk == 3) need(c + 1);
+    const double* S1 = kk == 3 ? ST + ((c + 1) % PN_ST) * STAGE : S0;  // stage of plane g+1
+    constexpr int kp = (kk + 1) & 3;                                   // its plane in that stage
+    if (start) {  // first step of a run (warm-up plane 7): prime the register windows
+      Xm[0] = lds_d2(S0 + oO + 64 * (kk - 1)), Xm[1] = lds_d2(S0 + oO + 8 + 64 * (kk - 1));
+      Xc[0] = lds_d2(S0 + oO + 64 * kk), Xc[1] = lds_d2(S0 + oO + 8 + 64 * kk);
+      rcm = S0[oc + 16 * (kk - 1)];
+      rc = S0[oc + 16 * kk];
+      load_b(B[kk], idC, codeC, kk);
+      load_b(B[(kk + 1) & 3], idN, codeN, 0);
+    }
+    if (pref) {  // b of plane g+2
+      if (kk < 2) load_b(B[(kk + 2) & 3], idC, codeC, kk + 2);
+      else load_b(B[(kk + 2) & 3], idN, codeN, kk - 2);
+    }
+    const int kz1 = 4 * (codeC & 1) + kk;  // in-brick plane of g (red-black colour)
+
+    // ---------------- sweep 1, own cells, plane g ----------------
+    Xp[0] = lds_d2(S1 + oO + 64 * kp);
+    Xp[1] = lds_d2(S1 + oO + 8 + 64 * kp);
+    {
+      const double2 xs = lds_d2(S0 + oS + sS * kk), xn = lds_d2(S0 + oN + sN * kk);
+      double e0 = 0.0, e1 = 0.0;
+      if (edW || edE) e0 = S0[oEd + 16 * kk], e1 = S0[oEd + 2 + 16 * kk];
+      const double wl0 = __shfl_up_sync(FULL, Xc[0].y, 1), er0 = __shfl_down_sync(FULL, Xc[0].x, 1);
+      const double wl1 = __shfl_up_sync(FULL, Xc[1].y, 1), er1 = __shfl_down_sync(FULL, Xc[1].x, 1);
+      const double W0 = edW ? e0 : wl0, E0 = edE ? e0 : er0, W1 = edW ? e1 : wl1, E1 = edE ? e1 : er1;
+      const double2 bb0 = B[kk][0], bb1 = B[kk][1];
+      const double a00 = stencil_a(Xc[0].x, W0, Xc[0].y, xs.x, Xc[1].x, Xm[0].x, Xp[0].x, alpha, beta);
+      const double a10 = stencil_a(Xc[0].y, Xc[0].x, E0, xs.y, Xc[1].y, Xm[0].y, Xp[0].y, alpha, beta);
+      const double a01 = stencil_a(Xc[1].x, W1, Xc[1].y, Xc[0].x, xn.x, Xm[1].x, Xp[1].x, alpha, beta);
+      const double a11 = stencil_a(Xc[1].y, Xc[1].x, E1, Xc[0].y, xn.y, Xm[1].y, Xp[1].y, alpha, beta);
+      Y[0].x = keep_cell(col1, ib, jb, kz1) ? Xc[0].x : DADD(Xc[0].x, DMUL(gamma, DSUB(a00, bb0.x)));
+      Y[0].y = keep_cell(col1, ib + 1, jb, kz1) ? Xc[0].y : DADD(Xc[0].y, DMUL(gamma, DSUB(a10, bb0.y)));
+      Y[1].x = keep_cell(col1, ib, jb + 1, kz1) ? Xc[1].x : DADD(Xc[1].x, DMUL(gamma, DSUB(a01, bb1.x)));
+      Y[1].y = keep_cell(col1, ib + 1, jb + 1, kz1) ? Xc[1].y : DADD(Xc[1].y, DMUL(gamma, DSUB(a11, bb1.y)));
+      double* P = XP + (kk & 1) * PUB;  // parity of plane g = 4c + kk
+      *reinterpret_cast<double2*>(P + pO) = Y[0];
+      *reinterpret_cast<double2*>(P + pO + 16) = Y[1];
+    }
+    // ---------------- sweep 1, ring cell, plane g ----------------
+    {
+      rcp = S1[oc + 16 * kp];
+      const double o = S0[oo + 16 * kk], own = S0[oown + 64 * kk];
+      const double lo = S0[olo + slo * kk], hi = S0[ohi + shi * kk], bv = S0[ob + sb * kk];
+      // ((o + own) + (lo + hi)) + (b + t): the canonical ((w+e)+(s+n))+(b+t) up to the order of
+      // the operands of single additions (IEEE addition is commutative, so bit for bit equal)
+      const double sum = DADD(DADD(DADD(o, own), DADD(lo, hi)), DADD(rcm, rcp));
+      const double a = DADD(DMUL(alpha, rc), DMUL(beta, sum));
+      const double y = keep_cell(col1, rci, rcj, kz1) ? rc : DADD(rc, DMUL(gamma, DSUB(a, bv)));
+      XP[oout + rstr * (kk & 1)] = y;
+    }
+    // ---------------- sweep 2, own cells, plane g-1 ----------------
+    if (sw2) {
+      constexpr int par = (kk + 1) & 1;  // parity of plane g - 1
+      const double* P = XP + par * PUB;
+      const double2 ys = lds_d2(P + pO - 16), yn = lds_d2(P + pO + 32);
+      double2 ed = make_double2(0.0, 0.0);
+      if (edW || edE) ed = lds_d2(RWE + 32 * par + oRwe);
+      const double wl0 = __shfl_up_sync(FULL, Yc[0].y, 1), er0 = __shfl_down_sync(FULL, Yc[0].x, 1);
+      const double wl1 = __shfl_up_sync(FULL, Yc[1].y, 1), er1 = __shfl_down_sync(FULL, Yc[1].x, 1);
+      const double W0 = edW ? ed.x : wl0, E0 = edE ? ed.x : er0, W1 = edW ? ed.y : wl1, E1 = edE ? ed.y : er1;
+      constexpr int km = (kk + 3) & 3;  // plane g-1 within its chunk
+      const double2 bb0 = B[km][0], bb1 = B[km][1];
+      const int code2 = kk > 0 ? codeC : codeP, id2 = kk > 0 ? idC : idP;
+      const int kz2 = 4 * (code2 & 1) + km;
+      const double a00 = stencil_a(Yc[0].x, W0, Yc[0].y, ys.x, Yc[1].x, Ym[0].x, Y[0].x, alpha, beta);
+      const double a10 = stencil_a(Yc[0].y, Yc[0].x, E0, ys.y, Yc[1].y, Ym[0].y, Y[0].y, alpha, beta);
+      const double a01 = stencil_a(Yc[1].x, W1, Yc[1].y, Yc[0].x, yn.x, Ym[1].x, Y[1].x, alpha, beta);
+      const double a11 = stencil_a(Yc[1].y, Yc[1].x, E1, Yc[0].y, yn.y, Ym[1].y, Y[1].y, alpha, beta);
+      double2 z0, z1, r0, r1;
+      z0.x = keep_cell(col2, ib, jb, kz2) ? Yc[0].x : DADD(Yc[0].x, DMUL(gamma2, DSUB(a00, bb0.x)));
+      z0.y = keep_cell(col2, ib + 1, jb, kz2) ? Yc[0].y : DADD(Yc[0].y, DMUL(gamma2, DSUB(a10, bb0.y)));
+      z1.x = keep_cell(col2, ib, jb + 1, kz2) ? Yc[1].x : DADD(Yc[1].x, DMUL(gamma2, DSUB(a01, bb1.x)));
+      z1.y = keep_cell(col2, ib + 1, jb + 1, kz2) ? Yc[1].y : DADD(Yc[1].y, DMUL(gamma2, DSUB(a11, bb1.y)));
+      r0.x = DSUB(bb0.x, a00), r0.y = DSUB(bb0.y, a10), r1.x = DSUB(bb1.x, a01), r1.y = DSUB(bb1.y, a11);
+      const int64_t go = (int64_t)id2 * 512 + 64 * kz2 + 8 * jb + ib;
+      st_hint2(p.xo + go, z0, pol_stream);  // never re-read by this pass
+      st_hint2(p.xo + go + 8, z1, pol_stream);
+      if (WRITE_R) {
+        st_hint2(p.r + go, r0, pol_stream);
+        st_hint2(p.r + go + 8, r1, pol_stream);
+      }
+      if (RESTRICT) {
+        // this lane's 2x2 footprint x 2 planes is one coarse cell: canonical order
+        // ((r000+r100)+(r010+r110)) + ((r001+r101)+(r011+r111))
+        const double s = DADD(DADD(r0.x, r0.y), DADD(r1.x, r1.y));
+        if ((km & 1) == 0) {
+          rpart = s;
+        } else {
+          const int pr = kk > 0 ? parC : parP;
+          const int K = 4 * ((pr >> 2) & 1) + (kz2 >> 1);
+          p.bc[(int64_t)(pr >> 3) * 512 + pc + 8 * (4 * w + jp) + 64 * K] = DMUL(0.125, DADD(rpart, s));
+        }
+      }
+    }
+    __syncthreads();  // x1 of plane g published; stage c (and c+1) reads of this step done
+#pragma unroll
+    for (int r = 0; r < 2; ++r) {
+      Xm[r] = Xc[r], Xc[r] = Xp[r];
+      Ym[r] = Yc[r], Yc[r] = Y[r];
+    }
+    rcm = rc, rc = rcp;
+  };
+
+  for (int c = 0; c < cnt; ++c) {
+    if (w == 0)
+      while (issued < cnt && issued <= c + PN_ST - 1) issue();
+    const int type = (codeC >> 1) & 3, typeP = (codeP >> 1) & 3, typeN = (codeN >> 1) & 3;
+    using I0 = std::integral_constant<int, 0>;
+    using I1 = std::integral_constant<int, 1>;
+    using I2 = std::integral_constant<int, 2>;
+    using I3 = std::integral_constant<int, 3>;
+    if (type == WARM) {
+      step(c, I3{}, true, false, true);
+    } else if (type == RANGE) {
+      step(c, I0{}, false, c > 0 && typeP == RANGE, true);
+      step(c, I1{}, false, true, true);
+      step(c, I2{}, false, true, typeN == RANGE || typeN == COOL);
+      step(c, I3{}, false, true, typeN == RANGE);
+    } else {
+      step(c, I0{}, false, true, false);
+    }
+    codeP = codeC, idP = idC, parP = parC;
+    codeC = codeN, idC = idN, parC = parN;
+    codeN = codeNN;
+    if (c + 2 < cnt) idN = meta_at(codeN, q), parN = meta_at(codeN, 16);
+    if (c + 3 < cnt) codeNN = CH[c + 3];
+  }
+}
+
+bool pencil_supports(unsigned flags) {
+  const unsigned fl = flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP | SW_ZERO_X);
+  return fl == 0 || fl == SW_WRITE_R || fl == SW_RESTRICT;
+}
+
+cudaError_t encode_pencil_maps(const double* x, const double* b, int64_t n_alloc, PairMaps* out) {
+  const unsigned we[3] = {2, 8, 4}, sn2[3] = {8, 2, 4}, cor[3] = {2, 1, 4}, sn1[3] = {8, 1, 4};
+  cudaError_t e;
+  if ((e = encode_box_map(x, n_alloc, we, &out->xwe)) != cudaSuccess) return e;
+  if ((e = encode_box_map(x, n_alloc, sn2, &out->xsn)) != cudaSuccess) return e;
+  if ((e = encode_box_map(x, n_alloc, cor, &out->xcor)) != cudaSuccess) return e;
+  if ((e = encode_box_map(b, n_alloc, we, &out->bwe)) != cudaSuccess) return e;
+  return encode_box_map(b, n_alloc, sn1, &out->bsn);
+}
+
+cudaError_t launch_sweep2p(const SweepArgs& a, const PairArgs& pa, const PairMaps& pm, unsigned flags,
+                           cudaStream_t s) {
+  if (pa.nctas <= 0) return cudaSuccess;
+  const unsigned g = (unsigned)pa.nctas;
+  const size_t sm = SMEM_BYTES;
+  const unsigned col = (a.colour >= 0 || a.colour2 >= 0) ? SW_COLOUR : 0u;
+  switch ((flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP | SW_ZERO_X)) | col) {
+    case 0: sweep2p_kernel<0><<<g, PN_THREADS, sm, s>>>(a, pa, pm); break;
+    case SW_WRITE_R: sweep2p_kernel<SW_WRITE_R><<<g, PN_THREADS, sm, s>>>(a, pa, pm); break;
+    case SW_RESTRICT: sweep2p_kernel<SW_RESTRICT><<<g, PN_THREADS, sm, s>>>(a, pa, pm); break;
+    case SW_COLOUR: sweep2p_kernel<SW_COLOUR><<<g, PN_THREADS, sm, s>>>(a, pa, pm); break;
+    case SW_WRITE_R | SW_COLOUR: sweep2p_kernel<SW_WRITE_R | SW_COLOUR><<<g, PN_THREADS, sm, s>>>(a, pa, pm); break;
+    case SW_RESTRICT | SW_COLOUR:
+      sweep2p_kernel<SW_RESTRICT | SW_COLOUR><<<g, PN_THREADS, sm, s>>>(a, pa, pm);
+      break;
+    default: return cudaErrorInvalidValue;
+  }
+  return cudaGetLastError();
+}
+
+cudaError_t pencil_kernels_init() {
+  const void* k[6] = {(const void*)sweep2p_kernel<0>, (const void*)sweep2p_kernel<SW_WRITE_R>,
+                      (const void*)sweep2p_kernel<SW_RESTRICT>, (const void*)sweep2p_kernel<SW_COLOUR>,
+                      (const void*)sweep2p_kernel<SW_WRITE_R | SW_COLOUR>,
+                      (const void*)sweep2p_kernel<SW_RESTRICT | SW_COLOUR>};
+  for (int i = 0; i < 6; ++i) {
+    cudaError_t e = cudaFuncSetAttribute(k[i], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM_BYTES);
+    if (e != cudaSuccess) return e;
+    e = cudaFuncSetAttribute(k[i], cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
+}
+
+}  // namespace mgb
