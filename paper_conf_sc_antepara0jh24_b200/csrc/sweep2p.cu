@@ -10,7 +10,7 @@
 // Data flow (why it is shaped like this: DESIGN.md §7.1).  A CTA of two warps walks a
 // stream of half-layer CHUNKS of 2x2-brick pencils (layout.cpp pencil_table):
 // [warm-up half, (layer half 0, half 1)..., cool-down half] per run of a tile column.
-//   * A chunk = 4 z-planes of the 16x16-cell tile.  Lanes 0-23 of warp 0 stage it by TMA
+//   * A chunk = 4 z-planes of the 16x16-cell tile.  Lanes 0-11 of both warps stage it by TMA
 //     into a 2-stage shared-memory ring (one mbarrier per stage): the four own x0 bricks'
 //     planes (1D bulk, 2 KB each), the 2-cell-deep x0 slabs of the 8 side neighbours
 //     (3D tensor boxes {2,8,4} / {8,2,4}), their b faces, the 4 diagonal corner columns.
@@ -93,10 +93,10 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
   else if (w == 0) oN = OWN_STRIDE * (q + 2) + ib, sN = 64;
   else oN = XN + 64 * bx + ib, sN = 16;  // N slab row j = 0
   const bool edW = pc == 0, edE = pc == 7;
-  const int oEd = edW ? XW + 64 * w + 2 * jb + 1 : XE + 64 * w + 2 * jb;  // tile-edge W / E x0 (rows jb, jb+1: +2)
+  const int oEd = edE ? XE + 64 * w + 2 * jb : XW + 64 * w + 2 * jb + 1;  // tile-edge W / E x0 (rows jb, jb+1: +2)
   const int R0 = 8 * w + jb;                                              // tile row of my row 0
   const int pO = (R0 + 1) * 16 + 2 * pc;                                  // my row 0 in the x1 buffer
-  const int oRwe = (edW ? 0 : 16) + R0;                                   // ring x1 column, rows R0, R0+1
+  const int oRwe = (edE ? 16 : 0) + R0;                                   // ring x1 column, rows R0, R0+1
 
   // ---- ring role: x1 of one cell of the 1-cell ring around the tile ----
   int oc, oo, oown, olo, slo, ohi, shi, ob, sb, oout, rstr, rci, rcj;
@@ -132,61 +132,63 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
   }
 
   if (t == 0) {
-    for (int s = 0; s < PN_ST; ++s) mbar_init(&BAR[s], 1);
+    for (int s = 0; s < PN_ST; ++s) mbar_init(&BAR[s], 2);  // one arrive.expect_tx per warp
     mbar_fence_init();
   }
   __syncthreads();
 
-  // ---- producer: lanes 0-23 of warp 0, one TMA copy each per chunk ----
-  const int mi = l < 12 ? l : l - 8;  // meta field of my copy: own 0-3, W0..N1 4-11, corners 12-15
+  // ---- producer: lanes 0-11 of each warp, one TMA copy each per chunk.  Warp 0: the four own
+  // bricks' half (1D bulk) and the 8 x0 side slabs; warp 1: the 8 b faces and 4 corner columns ----
+  const int mi = w == 0 ? l : l + 4;  // meta field of my copy
   int issued = 0, ic = 0, ic1 = 0, im = 0;
-  if (w == 0 && cnt > 0) {
+  if (cnt > 0) {
     ic = CH[0];
     ic1 = cnt > 1 ? CH[1] : 0;
-    im = l < 24 ? pa.meta[(int64_t)(ic >> 3) * kPenMeta + mi] : 0;
+    im = l < 12 ? pa.meta[(int64_t)(ic >> 3) * kPenMeta + mi] : 0;
   }
-  auto issue = [&]() {  // warp 0 (uniform): stage chunk `issued`
+  auto issue = [&]() {  // both warps (uniform): stage chunk `issued`
     const int n = issued, s = n % PN_ST, half = ic & 1;
     double* D = ST + s * STAGE;
     fence_proxy_async();
-    if (l == 0) mbar_expect_tx(&BAR[s], CHUNK_BYTES);
+    if (l == 0) mbar_expect_tx(&BAR[s], w == 0 ? 4 * 2048 + 8 * 512 : 4 * 512 + 4 * 256 + 4 * 64);
     __syncwarp();
     const int kz = im * 8 + 4 * half;
-    if (l < 4) {
-      // evict_last: the neighbour tiles' slab copies read these bricks' faces shortly after
-      tma_load_1d_hint(D + OWN_STRIDE * l, p.x + (int64_t)im * 512 + 256 * half, 2048, &BAR[s], pol_keep);
-    } else if (l < 12) {
-      const bool xf = l < 8, lowside = ((l - 4) & 2) == 0;  // W / S boxes sit at the high face
-      tma_load_3d(D + XW + 64 * (l - 4), xf ? &mp.xwe : &mp.xsn, xf && lowside ? 6 : 0, !xf && lowside ? 6 : 0,
-                  kz, &BAR[s]);
-    } else if (l < 16) {
-      tma_load_3d(D + BW + 64 * (l - 12), &mp.bwe, l < 14 ? 6 : 0, 0, kz, &BAR[s]);
-    } else if (l < 20) {
-      tma_load_3d(D + BS + 32 * (l - 16), &mp.bsn, 0, l < 18 ? 7 : 0, kz, &BAR[s]);
-    } else if (l < 24) {  // SW (6,7), NW (6,0), SE (0,7), NE (0,0)
-      const int cc = l - 20;
-      tma_load_3d(D + COR + 16 * cc, &mp.xcor, cc < 2 ? 6 : 0, (cc & 1) ? 0 : 7, kz, &BAR[s]);
+    if (w == 0) {
+      if (l < 4) {
+        // evict_last: the neighbour tiles' slab copies read these bricks' faces shortly after
+        tma_load_1d_hint(D + OWN_STRIDE * l, p.x + (int64_t)im * 512 + 256 * half, 2048, &BAR[s], pol_keep);
+      } else if (l < 12) {
+        const bool xf = l < 8, lowside = ((l - 4) & 2) == 0;  // W / S boxes sit at the high face
+        tma_load_3d(D + XW + 64 * (l - 4), xf ? &mp.xwe : &mp.xsn, xf && lowside ? 6 : 0,
+                    !xf && lowside ? 6 : 0, kz, &BAR[s]);
+      }
+    } else {
+      if (l < 4) {
+        tma_load_3d(D + BW + 64 * l, &mp.bwe, l < 2 ? 6 : 0, 0, kz, &BAR[s]);
+      } else if (l < 8) {
+        tma_load_3d(D + BS + 32 * (l - 4), &mp.bsn, 0, l < 6 ? 7 : 0, kz, &BAR[s]);
+      } else if (l < 12) {  // SW (6,7), NW (6,0), SE (0,7), NE (0,0)
+        const int cc = l - 8;
+        tma_load_3d(D + COR + 16 * cc, &mp.xcor, cc < 2 ? 6 : 0, (cc & 1) ? 0 : 7, kz, &BAR[s]);
+      }
     }
     ++issued;
     ic = ic1;
-    if (issued < cnt && l < 24) im = pa.meta[(int64_t)(ic >> 3) * kPenMeta + mi];
+    if (issued < cnt && l < 12) im = pa.meta[(int64_t)(ic >> 3) * kPenMeta + mi];
     if (issued + 1 < cnt) ic1 = CH[issued + 1];
   };
-  int nwait = 0;
-  auto need = [&](int n) {
-    while (nwait <= n) {
-      mbar_wait(&BAR[nwait % PN_ST], (uint32_t)((nwait / PN_ST) & 1));
-      ++nwait;
-    }
-  };
+  // every chunk is waited for exactly once, in order: at its run's warm-up step or at step kk = 3
+  // of the chunk before it
+  auto wait_chunk = [&](int n) { mbar_wait(&BAR[n % PN_ST], (uint32_t)((n / PN_ST) & 1)); };
 
-  // ---- per-chunk metadata (uniform): code, my brick id, parent of b00; chunks c-1, c, c+1 ----
+  // ---- per-chunk metadata (uniform, loaded two chunks ahead): code, my brick id, parent of b00 ----
   auto meta_at = [&](int code, int f) { return pa.meta[(int64_t)(code >> 3) * kPenMeta + f]; };
-  int codeP = 0, idP = 0, parP = 0;
-  int codeC = 0, idC = 0, parC = 0, codeN = 0, idN = 0, parN = 0, codeNN = 0;
+  int codeP = 0, idP = 0, parP = 0, codeC = 0, idC = 0, parC = 0, codeN = 0, idN = 0, parN = 0;
+  int codeNN = 0, idNN = 0, parNN = 0, code3 = 0;
   if (cnt > 0) codeC = CH[0], idC = meta_at(codeC, q), parC = meta_at(codeC, 16);
   if (cnt > 1) codeN = CH[1], idN = meta_at(codeN, q), parN = meta_at(codeN, 16);
-  if (cnt > 2) codeNN = CH[2];
+  if (cnt > 2) codeNN = CH[2], idNN = meta_at(codeNN, q), parNN = meta_at(codeNN, 16);
+  if (cnt > 3) code3 = CH[3];
 
   // ---- registers: x0 planes g-1, g, g+1; x1 planes g-2, g-1, g; b of planes g-1 .. g+2 ----
   double2 Xm[2], Xc[2], Xp[2], Ym[2], Yc[2], Y[2], B[4][2];
@@ -197,6 +199,7 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
 #pragma unroll
     for (int s = 0; s < 4; ++s) B[s][r] = make_double2(0.0, 0.0);
   }
+  // b rows jb, jb+1 of my brick (always a valid brick id: unused chunks read brick 0)
   auto load_b = [&](double2* dst, int id, int code, int kk) {
     const double* bp = p.b + (int64_t)id * 512 + 64 * (4 * (code & 1) + kk) + 8 * jb + ib;
     dst[0] = ld_hint2(bp, pol_keep);  // the neighbour tiles' b-face copies reuse these lines from L2
@@ -207,8 +210,8 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
   auto step = [&](const int c, auto kkc, const bool start, const bool sw2, const bool pref) {
     constexpr int kk = decltype(kkc)::value;
     const double* S0 = ST + (c % PN_ST) * STAGE;
-    need(c);
-    if (kk == 3) need(c + 1);
+    if (start) wait_chunk(c);
+    if (kk == 3) wait_chunk(c + 1);
     const double* S1 = kk == 3 ? ST + ((c + 1) % PN_ST) * STAGE : S0;  // stage of plane g+1
     constexpr int kp = (kk + 1) & 3;                                   // its plane in that stage
     if (start) {  // first step of a run (warm-up plane 7): prime the register windows
@@ -219,10 +222,11 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
       load_b(B[kk], idC, codeC, kk);
       load_b(B[(kk + 1) & 3], idN, codeN, 0);
     }
-    if (pref) {  // b of plane g+2
-      if (kk < 2) load_b(B[(kk + 2) & 3], idC, codeC, kk + 2);
-      else load_b(B[(kk + 2) & 3], idN, codeN, kk - 2);
-    }
+    // b of plane g+2 into registers (harmless when that plane is not swept: `pref` only says it is
+    // needed).  (An L2 prefetch of plane g+4 on top measured slower: +0.9 GB of DRAM reads.)
+    (void)pref;
+    if (kk < 2) load_b(B[(kk + 2) & 3], idC, codeC, kk + 2);
+    else load_b(B[(kk + 2) & 3], idN, codeN, kk - 2);
     const int kz1 = 4 * (codeC & 1) + kk;  // in-brick plane of g (red-black colour)
 
     // ---------------- sweep 1, own cells, plane g ----------------
@@ -230,8 +234,8 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     Xp[1] = lds_d2(S1 + oO + 8 + 64 * kp);
     {
       const double2 xs = lds_d2(S0 + oS + sS * kk), xn = lds_d2(S0 + oN + sN * kk);
-      double e0 = 0.0, e1 = 0.0;
-      if (edW || edE) e0 = S0[oEd + 16 * kk], e1 = S0[oEd + 2 + 16 * kk];
+      // tile-edge x0 (inner lanes read the W edge lane's words: broadcasts, no extra wavefronts)
+      const double e0 = S0[oEd + 16 * kk], e1 = S0[oEd + 2 + 16 * kk];
       const double wl0 = __shfl_up_sync(FULL, Xc[0].y, 1), er0 = __shfl_down_sync(FULL, Xc[0].x, 1);
       const double wl1 = __shfl_up_sync(FULL, Xc[1].y, 1), er1 = __shfl_down_sync(FULL, Xc[1].x, 1);
       const double W0 = edW ? e0 : wl0, E0 = edE ? e0 : er0, W1 = edW ? e1 : wl1, E1 = edE ? e1 : er1;
@@ -261,12 +265,13 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
       XP[oout + rstr * (kk & 1)] = y;
     }
     // ---------------- sweep 2, own cells, plane g-1 ----------------
-    if (sw2) {
+    // computed on every step (one basic block with sweep 1 and the ring: the scheduler interleaves
+    // the three dependency chains); only the stores depend on sw2
+    {
       constexpr int par = (kk + 1) & 1;  // parity of plane g - 1
       const double* P = XP + par * PUB;
       const double2 ys = lds_d2(P + pO - 16), yn = lds_d2(P + pO + 32);
-      double2 ed = make_double2(0.0, 0.0);
-      if (edW || edE) ed = lds_d2(RWE + 32 * par + oRwe);
+      const double2 ed = lds_d2(RWE + 32 * par + oRwe);
       const double wl0 = __shfl_up_sync(FULL, Yc[0].y, 1), er0 = __shfl_down_sync(FULL, Yc[0].x, 1);
       const double wl1 = __shfl_up_sync(FULL, Yc[1].y, 1), er1 = __shfl_down_sync(FULL, Yc[1].x, 1);
       const double W0 = edW ? ed.x : wl0, E0 = edE ? ed.x : er0, W1 = edW ? ed.y : wl1, E1 = edE ? ed.y : er1;
@@ -285,9 +290,11 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
       z1.y = keep_cell(col2, ib + 1, jb + 1, kz2) ? Yc[1].y : DADD(Yc[1].y, DMUL(gamma2, DSUB(a11, bb1.y)));
       r0.x = DSUB(bb0.x, a00), r0.y = DSUB(bb0.y, a10), r1.x = DSUB(bb1.x, a01), r1.y = DSUB(bb1.y, a11);
       const int64_t go = (int64_t)id2 * 512 + 64 * kz2 + 8 * jb + ib;
-      st_hint2(p.xo + go, z0, pol_stream);  // never re-read by this pass
-      st_hint2(p.xo + go + 8, z1, pol_stream);
-      if (WRITE_R) {
+      if (sw2) {
+        st_hint2(p.xo + go, z0, pol_stream);  // never re-read by this pass
+        st_hint2(p.xo + go + 8, z1, pol_stream);
+      }
+      if (WRITE_R && sw2) {
         st_hint2(p.r + go, r0, pol_stream);
         st_hint2(p.r + go + 8, r1, pol_stream);
       }
@@ -297,7 +304,7 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
         const double s = DADD(DADD(r0.x, r0.y), DADD(r1.x, r1.y));
         if ((km & 1) == 0) {
           rpart = s;
-        } else {
+        } else if (sw2) {
           const int pr = kk > 0 ? parC : parP;
           const int K = 4 * ((pr >> 2) & 1) + (kz2 >> 1);
           p.bc[(int64_t)(pr >> 3) * 512 + pc + 8 * (4 * w + jp) + 64 * K] = DMUL(0.125, DADD(rpart, s));
@@ -314,8 +321,7 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
   };
 
   for (int c = 0; c < cnt; ++c) {
-    if (w == 0)
-      while (issued < cnt && issued <= c + PN_ST - 1) issue();
+    while (issued < cnt && issued <= c + PN_ST - 1) issue();
     const int type = (codeC >> 1) & 3, typeP = (codeP >> 1) & 3, typeN = (codeN >> 1) & 3;
     using I0 = std::integral_constant<int, 0>;
     using I1 = std::integral_constant<int, 1>;
@@ -333,9 +339,10 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     }
     codeP = codeC, idP = idC, parP = parC;
     codeC = codeN, idC = idN, parC = parN;
-    codeN = codeNN;
-    if (c + 2 < cnt) idN = meta_at(codeN, q), parN = meta_at(codeN, 16);
-    if (c + 3 < cnt) codeNN = CH[c + 3];
+    codeN = codeNN, idN = idNN, parN = parNN;
+    codeNN = code3;
+    if (c + 3 < cnt) idNN = meta_at(codeNN, q), parNN = meta_at(codeNN, 16);
+    if (c + 4 < cnt) code3 = CH[c + 4];
   }
 }
 
