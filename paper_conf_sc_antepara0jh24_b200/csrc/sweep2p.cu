@@ -57,7 +57,8 @@ constexpr int PUB = 18 * 16;  // x1 of tile rows -1..16 (rows -1 / 16: the S / N
 static_assert(STAGE * 8 % 128 == 0 && XW * 8 % 128 == 0 && BS * 8 % 128 == 0 && COR * 8 % 128 == 0, "align");
 static_assert(3 * OWN_STRIDE + 256 <= XW, "own bricks fit");
 __device__ __forceinline__ double2 lds_d2(const double* p) { return *reinterpret_cast<const double2*>(p); }
-constexpr size_t SMEM_BYTES = (size_t)(PN_ST * STAGE + 2 * PUB + 2 * 32) * 8 + PN_ST * 8;
+constexpr int MRS = 4;  // chunk metadata ring slots: code, ids of b00..b11, parent of b00
+constexpr size_t SMEM_BYTES = (size_t)(PN_ST * STAGE + 2 * PUB + 2 * 32) * 8 + PN_ST * 8 + MRS * 8 * 4;
 
 }  // namespace
 
@@ -74,12 +75,14 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
   double* const XP = ST + PN_ST * STAGE;                    // [2][PUB]  x1 of tile rows -1..16
   double* const RWE = XP + 2 * PUB;                         // [2][2][16] x1 of the W / E ring columns
   uint64_t* const BAR = reinterpret_cast<uint64_t*>(RWE + 64);
+  int* const MR = reinterpret_cast<int*>(BAR + PN_ST);  // [MRS][8]: code, id b00..b11, parent (chunk n: slot n % 4)
   const int col1 = COLOUR ? p.colour : -1, col2 = COLOUR ? p.colour2 : -1;
   const int t = threadIdx.x, w = t >> 5, l = t & 31;
   const int2 cr = pa.ctas[blockIdx.x];
   const int32_t* CH = pa.chunks + cr.x;  // chunk codes: item row << 3 | type << 1 | half
   const int cnt = cr.y;
   const double alpha = p.c.alpha, beta = p.c.beta, gamma = p.c.gamma, gamma2 = p.gamma2;
+  // L2 policies (evict_normal for x0, b or x2 measured no different: DESIGN.md §7.1)
   const uint64_t pol_keep = l2_evict_last(), pol_stream = l2_evict_first();
 
   // ---- own-cell role: cells (2p + a, 8w + 2jp + r) of the tile ----
@@ -139,12 +142,14 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
 
   // ---- producer: lanes 0-11 of each warp, one TMA copy each per chunk.  Warp 0: the four own
   // bricks' half (1D bulk) and the 8 x0 side slabs; warp 1: the 8 b faces and 4 corner columns ----
-  const int mi = w == 0 ? l : l + 4;  // meta field of my copy
+  // meta field of my copy; lane 12 of warp 0 fetches the parent for the metadata ring
+  const int mi = w == 0 ? (l < 12 ? l : 16) : l + 4;
+  const bool mload = l < 12 || (w == 0 && l == 12);
   int issued = 0, ic = 0, ic1 = 0, im = 0;
   if (cnt > 0) {
     ic = CH[0];
     ic1 = cnt > 1 ? CH[1] : 0;
-    im = l < 12 ? pa.meta[(int64_t)(ic >> 3) * kPenMeta + mi] : 0;
+    im = mload ? pa.meta[(int64_t)(ic >> 3) * kPenMeta + mi] : 0;
   }
   auto issue = [&]() {  // both warps (uniform): stage chunk `issued`
     const int n = issued, s = n % PN_ST, half = ic & 1;
@@ -154,6 +159,11 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     __syncwarp();
     const int kz = im * 8 + 4 * half;
     if (w == 0) {
+      // metadata ring (read by both warps after the next barrier; slot n % 4 is chunk n - 4's,
+      // long consumed)
+      if (l == 0) MR[(n % MRS) * 8] = ic;
+      if (l < 4) MR[(n % MRS) * 8 + 1 + l] = im;
+      if (l == 12) MR[(n % MRS) * 8 + 5] = im;
       if (l < 4) {
         // evict_last: the neighbour tiles' slab copies read these bricks' faces shortly after
         tma_load_1d_hint(D + OWN_STRIDE * l, p.x + (int64_t)im * 512 + 256 * half, 2048, &BAR[s], pol_keep);
@@ -174,21 +184,17 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     }
     ++issued;
     ic = ic1;
-    if (issued < cnt && l < 12) im = pa.meta[(int64_t)(ic >> 3) * kPenMeta + mi];
+    if (issued < cnt && mload) im = pa.meta[(int64_t)(ic >> 3) * kPenMeta + mi];
     if (issued + 1 < cnt) ic1 = CH[issued + 1];
   };
   // every chunk is waited for exactly once, in order: at its run's warm-up step or at step kk = 3
   // of the chunk before it
   auto wait_chunk = [&](int n) { mbar_wait(&BAR[n % PN_ST], (uint32_t)((n / PN_ST) & 1)); };
 
-  // ---- per-chunk metadata (uniform, loaded two chunks ahead): code, my brick id, parent of b00 ----
+  // ---- per-chunk metadata from the ring (chunk c+1's entry is written when it is issued, at the
+  // start of chunk c, so it is visible from chunk c's second step on) ----
   auto meta_at = [&](int code, int f) { return pa.meta[(int64_t)(code >> 3) * kPenMeta + f]; };
-  int codeP = 0, idP = 0, parP = 0, codeC = 0, idC = 0, parC = 0, codeN = 0, idN = 0, parN = 0;
-  int codeNN = 0, idNN = 0, parNN = 0, code3 = 0;
-  if (cnt > 0) codeC = CH[0], idC = meta_at(codeC, q), parC = meta_at(codeC, 16);
-  if (cnt > 1) codeN = CH[1], idN = meta_at(codeN, q), parN = meta_at(codeN, 16);
-  if (cnt > 2) codeNN = CH[2], idNN = meta_at(codeNN, q), parNN = meta_at(codeNN, 16);
-  if (cnt > 3) code3 = CH[3];
+  auto mr = [&](int n, int f) { return MR[(n % MRS) * 8 + f]; };
 
   // ---- registers: x0 planes g-1, g, g+1; x1 planes g-2, g-1, g; b of planes g-1 .. g+2 ----
   double2 Xm[2], Xc[2], Xp[2], Ym[2], Yc[2], Y[2], B[4][2];
@@ -214,6 +220,12 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     if (kk == 3) wait_chunk(c + 1);
     const double* S1 = kk == 3 ? ST + ((c + 1) % PN_ST) * STAGE : S0;  // stage of plane g+1
     constexpr int kp = (kk + 1) & 3;                                   // its plane in that stage
+    const int codeC = mr(c, 0), idC = mr(c, 1 + q);
+    // chunk c+1 (b prefetch from step kk = 2 on): its ring entry, except on a run's warm-up step,
+    // where chunk c+1 was issued at the start of this very step (not visible yet): from global
+    int codeN = 0, idN = 0;
+    if (start) codeN = CH[c + 1], idN = meta_at(codeN, q);
+    else if (kk >= 2) codeN = mr(c + 1, 0), idN = mr(c + 1, 1 + q);
     if (start) {  // first step of a run (warm-up plane 7): prime the register windows
       Xm[0] = lds_d2(S0 + oO + 64 * (kk - 1)), Xm[1] = lds_d2(S0 + oO + 8 + 64 * (kk - 1));
       Xc[0] = lds_d2(S0 + oO + 64 * kk), Xc[1] = lds_d2(S0 + oO + 8 + 64 * kk);
@@ -277,7 +289,7 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
       const double W0 = edW ? ed.x : wl0, E0 = edE ? ed.x : er0, W1 = edW ? ed.y : wl1, E1 = edE ? ed.y : er1;
       constexpr int km = (kk + 3) & 3;  // plane g-1 within its chunk
       const double2 bb0 = B[km][0], bb1 = B[km][1];
-      const int code2 = kk > 0 ? codeC : codeP, id2 = kk > 0 ? idC : idP;
+      const int code2 = kk > 0 ? codeC : mr(c + MRS - 1, 0), id2 = kk > 0 ? idC : mr(c + MRS - 1, 1 + q);
       const int kz2 = 4 * (code2 & 1) + km;
       const double a00 = stencil_a(Yc[0].x, W0, Yc[0].y, ys.x, Yc[1].x, Ym[0].x, Y[0].x, alpha, beta);
       const double a10 = stencil_a(Yc[0].y, Yc[0].x, E0, ys.y, Yc[1].y, Ym[0].y, Y[0].y, alpha, beta);
@@ -305,7 +317,7 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
         if ((km & 1) == 0) {
           rpart = s;
         } else if (sw2) {
-          const int pr = kk > 0 ? parC : parP;
+          const int pr = mr(kk > 0 ? c : c + MRS - 1, 5);
           const int K = 4 * ((pr >> 2) & 1) + (kz2 >> 1);
           p.bc[(int64_t)(pr >> 3) * 512 + pc + 8 * (4 * w + jp) + 64 * K] = DMUL(0.125, DADD(rpart, s));
         }
@@ -320,9 +332,11 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     rcm = rc, rc = rcp;
   };
 
+  while (issued < cnt && issued < PN_ST) issue();
+  __syncthreads();  // ring entries of chunks 0, 1
   for (int c = 0; c < cnt; ++c) {
     while (issued < cnt && issued <= c + PN_ST - 1) issue();
-    const int type = (codeC >> 1) & 3, typeP = (codeP >> 1) & 3, typeN = (codeN >> 1) & 3;
+    const int type = (mr(c, 0) >> 1) & 3, typeP = c > 0 ? (mr(c + MRS - 1, 0) >> 1) & 3 : WARM;
     using I0 = std::integral_constant<int, 0>;
     using I1 = std::integral_constant<int, 1>;
     using I2 = std::integral_constant<int, 2>;
@@ -330,19 +344,13 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     if (type == WARM) {
       step(c, I3{}, true, false, true);
     } else if (type == RANGE) {
-      step(c, I0{}, false, c > 0 && typeP == RANGE, true);
+      step(c, I0{}, false, typeP == RANGE, true);
       step(c, I1{}, false, true, true);
-      step(c, I2{}, false, true, typeN == RANGE || typeN == COOL);
-      step(c, I3{}, false, true, typeN == RANGE);
+      step(c, I2{}, false, true, true);
+      step(c, I3{}, false, true, true);
     } else {
       step(c, I0{}, false, true, false);
     }
-    codeP = codeC, idP = idC, parP = parC;
-    codeC = codeN, idC = idN, parC = parN;
-    codeN = codeNN, idN = idNN, parN = parNN;
-    codeNN = code3;
-    if (c + 3 < cnt) idNN = meta_at(codeNN, q), parNN = meta_at(codeNN, 16);
-    if (c + 4 < cnt) code3 = CH[c + 4];
   }
 }
 
