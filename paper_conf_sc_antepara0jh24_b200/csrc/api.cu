@@ -190,7 +190,6 @@ size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double**
       pr.args.nctas = (int64_t)pt.ctas.size() / 2;
       pr.args.warps = (const int4*)take(pt.warps.size() * sizeof(int32_t));
       pr.args.nwarps = (int64_t)pt.warps.size() / 4;
-      pr.args.chunks = (const int32_t*)take(pt.chunks.size() * sizeof(int32_t));
       d.pairs.push_back(pr);
     }
     d.ncruns = (int)L.recvs.size();
@@ -590,8 +589,6 @@ mg_status init_ctx(mg_ctx* c, const mg_params& p, int rank, int world, int devic
       CKC(c, cudaMemcpyAsync((void*)pa.meta, pt.meta.data(), pt.meta.size() * 4, cudaMemcpyHostToDevice, stream));
       CKC(c, cudaMemcpyAsync((void*)pa.ctas, pt.ctas.data(), pt.ctas.size() * 4, cudaMemcpyHostToDevice, stream));
       CKC(c, cudaMemcpyAsync((void*)pa.warps, pt.warps.data(), pt.warps.size() * 4, cudaMemcpyHostToDevice, stream));
-      CKC(c, cudaMemcpyAsync((void*)pa.chunks, pt.chunks.data(), pt.chunks.size() * 4, cudaMemcpyHostToDevice,
-                             stream));
     }
     if (!L.pairs.empty())
       for (int xb = 0; xb < 2; ++xb) {

@@ -67,12 +67,12 @@ cudaError_t encode_box_map(const double* base, int64_t n_alloc, const unsigned b
 // Two-sweep (temporally blocked) streaming kernel, sweep2.cu.
 struct PairArgs {
   int kind;             // 1: CTA item streams (sweep2.cu), 2: half-warp plane streams (sweep2w.cu)
-  const int32_t* meta;  // kind 1: [items][11] id, flags, W,E,S,N, SW,NW,SE,NE, parent; kind 2: [items][12]
+  const int32_t* meta;  // kind 1: [items][11] id, flags, W,E,S,N, SW,NW,SE,NE, parent; kind 2: [items][12];
+                        // kind 3: [chunks][20] chunk records (mg_internal.h kPenRec)
   const int2* ctas;     // kind 1: (first item, item count) per CTA
   int64_t nctas;
   const int4* warps;    // kind 2: (first item half 0, first item half 1, steps, items0 | items1<<16) per warp
   int64_t nwarps;
-  const int32_t* chunks;  // kind 3: chunk codes (item row << 3 | type << 1 | half); ctas = (first chunk, count)
 };
 struct PairMaps {
   CUtensorMap xwe;   // x boxes {2,8,8}: W (i=6,7) / E (i=0,1) face slabs

@@ -410,7 +410,8 @@ static LevelLayout::PairTable pair_table(const LevelLayout& L, int64_t b0, int64
 // is one coarse brick's x-y extent and the kernel's restriction writes whole coarse columns);
 // a tile column (its z-chain of layers along T) plays the role of a brick chain in pair_table:
 // runs of its layers are dealt round-robin (below).  A run of layers
-// becomes chunks [warm-up layer half 1, (layer half 0, half 1)..., cool-down layer half 0];
+// becomes chunks [warm-up layer half 1, (layer half 0, half 1)..., cool-down layer half 0], each
+// a record of kPenRec ints (code, the tile layer's 16 brick ids, parent);
 // warm-up / cool-down are the B / T neighbour layers (their x1 planes 7 / 0 are the k-halos of
 // the run's second sweep).  Returns kind 0 if the range does not tile.
 static LevelLayout::PairTable pencil_table(const LevelLayout& L, int64_t b0, int64_t b1) {
@@ -457,11 +458,13 @@ static LevelLayout::PairTable pencil_table(const LevelLayout& L, int64_t b0, int
   t.b1 = b1;
   const int64_t ncol = (int64_t)tx * ty;
   const int64_t G = std::max<int64_t>(1, std::min<int64_t>(kPenCtas, ncol * nz));
-  std::vector<std::vector<int32_t>> stream((size_t)G);  // per CTA: chunk codes (item rows filled below)
-  auto push_item = [&](const std::array<int32_t, kPenMeta>& m) -> int32_t {
-    const int32_t row = (int32_t)(t.meta.size() / kPenMeta);
-    t.meta.insert(t.meta.end(), m.begin(), m.end());
-    return row;
+  std::vector<std::vector<int32_t>> stream((size_t)G);  // per CTA: its chunk records
+  // one 20-int record per chunk: code (type << 1 | half), the 16 brick ids, parent of b00
+  auto push_chunk = [&](std::vector<int32_t>& v, const std::array<int32_t, kPenMeta>& m, int type, int half) {
+    v.push_back((type << 1) | half);
+    v.insert(v.end(), m.begin(), m.begin() + 17);
+    v.push_back(0);
+    v.push_back(0);
   };
   // the B / T neighbour layer of a tile layer (warm-up / cool-down): every brick's B / T link
   auto shifted = [&](const std::array<int32_t, kPenMeta>& m, int f) {
@@ -470,13 +473,12 @@ static LevelLayout::PairTable pencil_table(const LevelLayout& L, int64_t b0, int
   auto push_run = [&](std::vector<int32_t>& v, int64_t col, int z0, int len) {
     const auto& first = layers[(size_t)col * nz + z0];
     const auto& last = layers[(size_t)col * nz + ((z0 + len - 1) % nz)];
-    v.push_back((push_item(shifted(first, 4)) << 3) | (1 << 1) | 1);  // warm-up: half 1
+    push_chunk(v, shifted(first, 4), 1, 1);  // warm-up: half 1
     for (int q = 0; q < len; ++q) {
-      const int32_t row = push_item(layers[(size_t)col * nz + ((z0 + q) % nz)]);
-      v.push_back(row << 3);
-      v.push_back((row << 3) | 1);
+      push_chunk(v, layers[(size_t)col * nz + ((z0 + q) % nz)], 0, 0);
+      push_chunk(v, layers[(size_t)col * nz + ((z0 + q) % nz)], 0, 1);
     }
-    v.push_back((push_item(shifted(last, 5)) << 3) | (2 << 1));  // cool-down: half 0
+    push_chunk(v, shifted(last, 5), 2, 0);  // cool-down: half 0
   };
   // Units = (z-run, tile column): the column's layers cut into nzr near-equal runs.  Units are
   // ordered z-run-major, column-minor (x fastest) and dealt round-robin, so the CTAs working at
@@ -505,9 +507,9 @@ static LevelLayout::PairTable pencil_table(const LevelLayout& L, int64_t b0, int
   for (int64_t g = 0; g < G; ++g) {
     const auto& v = stream[(size_t)g];
     if (v.empty()) continue;
-    t.ctas.push_back((int32_t)t.chunks.size());
-    t.ctas.push_back((int32_t)v.size());
-    t.chunks.insert(t.chunks.end(), v.begin(), v.end());
+    t.ctas.push_back((int32_t)(t.meta.size() / kPenRec));
+    t.ctas.push_back((int32_t)(v.size() / kPenRec));
+    t.meta.insert(t.meta.end(), v.begin(), v.end());
   }
   return t;
 }

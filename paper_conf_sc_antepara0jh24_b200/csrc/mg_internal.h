@@ -77,8 +77,6 @@ struct LevelLayout {
     std::vector<int32_t> meta;   // [items][kPairMeta] (kind 1) / [items][kW2Meta] (kind 2)
     std::vector<int32_t> ctas;   // kind 1: [nctas][2] offset (items), count
     std::vector<int32_t> warps;  // kind 2: [nwarps][4] first item of half 0, of half 1, steps, items0 | items1<<16
-    std::vector<int32_t> chunks; // kind 3: chunk codes item row << 3 | type << 1 | half (type 0 range,
-                                 // 1 warm-up, 2 cool-down); ctas = (first chunk, chunk count)
   };
   std::vector<PairTable> pairs;
 };
@@ -99,10 +97,12 @@ inline double sweep_gamma(const mg_params& p, double h, int s, int k) {
 constexpr int kPairMeta = 11;
 constexpr int kPairCtasPerSm = 4;                   // resident two-sweep CTAs per SM (shared-memory bound)
 constexpr int64_t kPairCtas = 148 * kPairCtasPerSm;  // one item stream per resident two-sweep CTA
-// kind 3 (sweep2p.cu): 2x2-brick pencils.  item = one z-layer of a tile: b00, b10, b01, b11 (own
-// bricks, x then y), W0, W1 (W of b00, b01), E0, E1 (E of b10, b11), S0, S1 (S of b00, b10),
-// N0, N1 (N of b01, b11), SW, NW, SE, NE (diagonal corners), parent of b00, 0, 0, 0.
-constexpr int kPenMeta = 20;
+// kind 3 (sweep2p.cu): 2x2-brick pencils.  meta = one record per half-layer chunk: code (type << 1 |
+// half; type 0 range, 1 warm-up, 2 cool-down), the tile layer's bricks b00, b10, b01, b11 (own, x then
+// y), W0, W1 (W of b00, b01), E0, E1 (E of b10, b11), S0, S1 (S of b00, b10), N0, N1 (N of b01, b11),
+// SW, NW, SE, NE (diagonal corners), parent of b00, 0, 0; ctas = (first record, record count).
+constexpr int kPenMeta = 20;  // host-side tile-layer item: the 16 ids, parent, 0, 0, 0
+constexpr int kPenRec = 20;   // chunk record (80 bytes: one 1D bulk copy)
 constexpr int kPenCtasPerSm = 6;                    // resident pencil CTAs per SM (shared-memory bound)
 constexpr int64_t kPenCtas = 148 * kPenCtasPerSm;
 constexpr int kW2Meta = 12;

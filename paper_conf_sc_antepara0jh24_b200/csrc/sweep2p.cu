@@ -57,8 +57,8 @@ constexpr int PUB = 18 * 16;  // x1 of tile rows -1..16 (rows -1 / 16: the S / N
 static_assert(STAGE * 8 % 128 == 0 && XW * 8 % 128 == 0 && BS * 8 % 128 == 0 && COR * 8 % 128 == 0, "align");
 static_assert(3 * OWN_STRIDE + 256 <= XW, "own bricks fit");
 __device__ __forceinline__ double2 lds_d2(const double* p) { return *reinterpret_cast<const double2*>(p); }
-constexpr int MRS = 4;  // chunk metadata ring slots: code, ids of b00..b11, parent of b00
-constexpr size_t SMEM_BYTES = (size_t)(PN_ST * STAGE + 2 * PUB + 2 * 32) * 8 + PN_ST * 8 + MRS * 8 * 4;
+constexpr int MRS = 4;  // chunk record ring slots (record n in slot n % 4)
+constexpr size_t SMEM_BYTES = (size_t)(PN_ST * STAGE + 2 * PUB + 2 * 32) * 8 + 16 + MRS * kPenRec * 4;
 
 }  // namespace
 
@@ -75,11 +75,11 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
   double* const XP = ST + PN_ST * STAGE;                    // [2][PUB]  x1 of tile rows -1..16
   double* const RWE = XP + 2 * PUB;                         // [2][2][16] x1 of the W / E ring columns
   uint64_t* const BAR = reinterpret_cast<uint64_t*>(RWE + 64);
-  int* const MR = reinterpret_cast<int*>(BAR + PN_ST);  // [MRS][8]: code, id b00..b11, parent (chunk n: slot n % 4)
+  int* const MR = reinterpret_cast<int*>(BAR + 2);  // [MRS][kPenRec] chunk records, 16-byte aligned slots
   const int col1 = COLOUR ? p.colour : -1, col2 = COLOUR ? p.colour2 : -1;
   const int t = threadIdx.x, w = t >> 5, l = t & 31;
   const int2 cr = pa.ctas[blockIdx.x];
-  const int32_t* CH = pa.chunks + cr.x;  // chunk codes: item row << 3 | type << 1 | half
+  const int32_t* REC = pa.meta + (int64_t)cr.x * kPenRec;  // chunk records: code, 16 brick ids, parent
   const int cnt = cr.y;
   const double alpha = p.c.alpha, beta = p.c.beta, gamma = p.c.gamma, gamma2 = p.gamma2;
   // L2 policies (evict_normal for x0, b or x2 measured no different: DESIGN.md §7.1)
@@ -140,33 +140,30 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
   }
   __syncthreads();
 
+  // ---- chunk records: record n lands in ring slot n % 4 with chunk n-1's TMA (records 0 and 1 by
+  // plain loads here), so it is in shared memory once chunk n-1 has been waited for ----
+  auto mr = [&](int n, int f) { return MR[(n % MRS) * kPenRec + f]; };
+  for (int e = t; e < 2 * kPenRec; e += PN_THREADS)
+    if (e < cnt * kPenRec) MR[e] = REC[e];
+
   // ---- producer: lanes 0-11 of each warp, one TMA copy each per chunk.  Warp 0: the four own
-  // bricks' half (1D bulk) and the 8 x0 side slabs; warp 1: the 8 b faces and 4 corner columns ----
-  // meta field of my copy; lane 12 of warp 0 fetches the parent for the metadata ring
-  const int mi = w == 0 ? (l < 12 ? l : 16) : l + 4;
-  const bool mload = l < 12 || (w == 0 && l == 12);
-  int issued = 0, ic = 0, ic1 = 0, im = 0;
-  if (cnt > 0) {
-    ic = CH[0];
-    ic1 = cnt > 1 ? CH[1] : 0;
-    im = mload ? pa.meta[(int64_t)(ic >> 3) * kPenMeta + mi] : 0;
-  }
+  // bricks' half (1D bulk) and the 8 x0 side slabs; warp 1: the 8 b faces, the 4 corner columns
+  // and (lane 12) the record of the chunk after ----
+  int issued = 0;
   auto issue = [&]() {  // both warps (uniform): stage chunk `issued`
-    const int n = issued, s = n % PN_ST, half = ic & 1;
+    const int n = issued, s = n % PN_ST, code = mr(n, 0), half = code & 1;
+    const bool rec = n + 1 >= 2 && n + 1 < cnt;
+    const int id = l < 12 ? mr(n, 1 + (w == 0 ? l : l + 4)) : 0;
     double* D = ST + s * STAGE;
     fence_proxy_async();
-    if (l == 0) mbar_expect_tx(&BAR[s], w == 0 ? 4 * 2048 + 8 * 512 : 4 * 512 + 4 * 256 + 4 * 64);
+    if (l == 0)
+      mbar_expect_tx(&BAR[s], w == 0 ? 4 * 2048 + 8 * 512 : 4 * 512 + 4 * 256 + 4 * 64 + (rec ? kPenRec * 4 : 0));
     __syncwarp();
-    const int kz = im * 8 + 4 * half;
+    const int kz = id * 8 + 4 * half;
     if (w == 0) {
-      // metadata ring (read by both warps after the next barrier; slot n % 4 is chunk n - 4's,
-      // long consumed)
-      if (l == 0) MR[(n % MRS) * 8] = ic;
-      if (l < 4) MR[(n % MRS) * 8 + 1 + l] = im;
-      if (l == 12) MR[(n % MRS) * 8 + 5] = im;
       if (l < 4) {
         // evict_last: the neighbour tiles' slab copies read these bricks' faces shortly after
-        tma_load_1d_hint(D + OWN_STRIDE * l, p.x + (int64_t)im * 512 + 256 * half, 2048, &BAR[s], pol_keep);
+        tma_load_1d_hint(D + OWN_STRIDE * l, p.x + (int64_t)id * 512 + 256 * half, 2048, &BAR[s], pol_keep);
       } else if (l < 12) {
         const bool xf = l < 8, lowside = ((l - 4) & 2) == 0;  // W / S boxes sit at the high face
         tma_load_3d(D + XW + 64 * (l - 4), xf ? &mp.xwe : &mp.xsn, xf && lowside ? 6 : 0,
@@ -180,21 +177,20 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
       } else if (l < 12) {  // SW (6,7), NW (6,0), SE (0,7), NE (0,0)
         const int cc = l - 8;
         tma_load_3d(D + COR + 16 * cc, &mp.xcor, cc < 2 ? 6 : 0, (cc & 1) ? 0 : 7, kz, &BAR[s]);
+      } else if (l == 12 && rec) {  // slot (n+1) % 4 held record n-3, consumed long ago
+        tma_load_1d(MR + ((n + 1) % MRS) * kPenRec, REC + (int64_t)(n + 1) * kPenRec, kPenRec * 4, &BAR[s]);
       }
     }
     ++issued;
-    ic = ic1;
-    if (issued < cnt && mload) im = pa.meta[(int64_t)(ic >> 3) * kPenMeta + mi];
-    if (issued + 1 < cnt) ic1 = CH[issued + 1];
   };
-  // every chunk is waited for exactly once, in order: at its run's warm-up step or at step kk = 3
-  // of the chunk before it
-  auto wait_chunk = [&](int n) { mbar_wait(&BAR[n % PN_ST], (uint32_t)((n / PN_ST) & 1)); };
-
-  // ---- per-chunk metadata from the ring (chunk c+1's entry is written when it is issued, at the
-  // start of chunk c, so it is visible from chunk c's second step on) ----
-  auto meta_at = [&](int code, int f) { return pa.meta[(int64_t)(code >> 3) * kPenMeta + f]; };
-  auto mr = [&](int n, int f) { return MR[(n % MRS) * 8 + f]; };
+  // chunks are waited for in order (uniform counter)
+  int nwait = 0;
+  auto wait_upto = [&](int n) {
+    while (nwait <= n) {
+      mbar_wait(&BAR[nwait % PN_ST], (uint32_t)((nwait / PN_ST) & 1));
+      ++nwait;
+    }
+  };
 
   // ---- registers: x0 planes g-1, g, g+1; x1 planes g-2, g-1, g; b of planes g-1 .. g+2 ----
   double2 Xm[2], Xc[2], Xp[2], Ym[2], Yc[2], Y[2], B[4][2];
@@ -216,16 +212,12 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
   auto step = [&](const int c, auto kkc, const bool start, const bool sw2, const bool pref) {
     constexpr int kk = decltype(kkc)::value;
     const double* S0 = ST + (c % PN_ST) * STAGE;
-    if (start) wait_chunk(c);
-    if (kk == 3) wait_chunk(c + 1);
+    if (kk == 3) wait_upto(c + 1);
     const double* S1 = kk == 3 ? ST + ((c + 1) % PN_ST) * STAGE : S0;  // stage of plane g+1
     constexpr int kp = (kk + 1) & 3;                                   // its plane in that stage
     const int codeC = mr(c, 0), idC = mr(c, 1 + q);
-    // chunk c+1 (b prefetch from step kk = 2 on): its ring entry, except on a run's warm-up step,
-    // where chunk c+1 was issued at the start of this very step (not visible yet): from global
-    int codeN = 0, idN = 0;
-    if (start) codeN = CH[c + 1], idN = meta_at(codeN, q);
-    else if (kk >= 2) codeN = mr(c + 1, 0), idN = mr(c + 1, 1 + q);
+    // chunk c+1 (b prefetch from step kk = 2 on; its record came with chunk c)
+    const int codeN = (start || kk >= 2) ? mr(c + 1, 0) : 0, idN = (start || kk >= 2) ? mr(c + 1, 1 + q) : 0;
     if (start) {  // first step of a run (warm-up plane 7): prime the register windows
       Xm[0] = lds_d2(S0 + oO + 64 * (kk - 1)), Xm[1] = lds_d2(S0 + oO + 8 + 64 * (kk - 1));
       Xc[0] = lds_d2(S0 + oO + 64 * kk), Xc[1] = lds_d2(S0 + oO + 8 + 64 * kk);
@@ -317,7 +309,7 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
         if ((km & 1) == 0) {
           rpart = s;
         } else if (sw2) {
-          const int pr = mr(kk > 0 ? c : c + MRS - 1, 5);
+          const int pr = mr(kk > 0 ? c : c + MRS - 1, 17);
           const int K = 4 * ((pr >> 2) & 1) + (kz2 >> 1);
           p.bc[(int64_t)(pr >> 3) * 512 + pc + 8 * (4 * w + jp) + 64 * K] = DMUL(0.125, DADD(rpart, s));
         }
@@ -332,9 +324,10 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     rcm = rc, rc = rcp;
   };
 
-  while (issued < cnt && issued < PN_ST) issue();
-  __syncthreads();  // ring entries of chunks 0, 1
+  __syncthreads();  // records 0, 1
   for (int c = 0; c < cnt; ++c) {
+    // chunk c (and with it record c+1) before issuing chunk c+1 into the stage chunk c-1 used
+    if (c > 0) wait_upto(c);
     while (issued < cnt && issued <= c + PN_ST - 1) issue();
     const int type = (mr(c, 0) >> 1) & 3, typeP = c > 0 ? (mr(c + MRS - 1, 0) >> 1) & 3 : WARM;
     using I0 = std::integral_constant<int, 0>;
