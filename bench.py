@@ -294,20 +294,19 @@ def main():
     tm = m.timings()
     m.set_timing(False)
     nsweep0 = a.pre + a.post
-    sweep0_ms = tm[0][mg.OP_NAMES.index("sweep")] / ninst
-    # HBM passes over level 0 per V-cycle: with temporal blocking every pass is two sweeps except the
-    # interpolation-fused first post-sweep and an odd leftover (pre 12 -> 6 pairs; post 1 + 11 -> 1 + 5 + 1)
-    fusion0 = a.fusion or mg.MG_FUSION_FULL
-    if a.tb:
-        post_rest = a.post - (1 if fusion0 == mg.MG_FUSION_FULL else 0)
-        npass0 = (a.pre + 1) // 2 + (1 if fusion0 == mg.MG_FUSION_FULL else 0) + (post_rest + 1) // 2
-    else:
-        npass0 = nsweep0
+    # every level-0 pass of the instrumented cycles, from the per-op records (two-sweep passes and any
+    # single sweeps alike; the interpolation is its own op where the pencil passes run)
+    recs = m.timing_records()
+    passes0 = [ms for (lv, op, ms) in recs if lv == 0 and op == mg.OP_NAMES.index("sweep")]
+    sweep0_ms = sum(passes0) / ninst
+    npass0 = round(len(passes0) / ninst)
     launch_ms = sweep0_ms / npass0
+    interp_fused = tm[0][mg.OP_NAMES.index("interpolation")] == 0
     # algorithmic bytes of the level-0 passes of one V-cycle (24 B/pt each: read x, b; write x'),
-    # + 1 B/pt for the fused restriction output and the fused interpolation input
+    # + 1 B/pt for the fused restriction output (and the fused interpolation input, if fused)
+    fusion0 = a.fusion or mg.MG_FUSION_FULL
     pts = n**3
-    bytes0 = pts * (B_SWEEP * npass0 + 2 * B_COARSE_PER_FINE)
+    bytes0 = pts * (B_SWEEP * npass0 + (2 if interp_fused else 1) * B_COARSE_PER_FINE)
     if fusion0 != mg.MG_FUSION_FULL:
         bytes0 = pts * (B_SWEEP * (npass0 - 1) + B_SWEEP_R)
     achieved = bytes0 / (sweep0_ms / 1e3) / 1e9

@@ -28,6 +28,12 @@ bool Builder::has_pair_table(int l, int64_t b0, int64_t b1) const {
   return false;
 }
 
+bool Builder::pencil_table(int l) const {
+  for (const auto& pt : lay.lv[l].pairs)
+    if (pt.b0 == 0 && pt.b1 == lay.lv[l].n_owned) return pt.kind == 3;
+  return false;
+}
+
 bool Builder::pair_ok(int l) const {
   if (!lay.p.temporal_blocking || fusion(l) == MG_FUSION_PAPER) return false;
   const LevelLayout& L = lay.lv[l];
@@ -275,7 +281,11 @@ void Builder::vcycle() {
     bottom(L - 1, p.bottom_smooths, true);  // steps 10-15
   }
   for (int l = top - (lc > 0 ? 1 : 2); l >= 0; --l) {  // steps 16-23
-    const bool fuse_i = fusion(l) == MG_FUSION_FULL && !ghosts(l) && p.post_smooths > 0;
+    // interpolation fused into the first post-sweep -- except where pencil passes run (their
+    // kernel has no interpolation input): a separate interpolation then lets all post-sweeps pair
+    // up (measured faster: one-brick interp-fused sweeps are the slowest single sweeps)
+    const bool pencil_pairs = pair_ok(l) && pencil_table(l) && p.post_smooths % 2 == 0 && lay.p.smoother != 2;
+    const bool fuse_i = fusion(l) == MG_FUSION_FULL && !ghosts(l) && p.post_smooths > 0 && !pencil_pairs;
     if (!fuse_i) interp_op(l);
     phase(l, p.post_smooths, false, 0, fuse_i, MG_OP_SWEEP);
   }

@@ -57,6 +57,7 @@ struct Builder {
   int fusion(int l) const;
   int period(int l) const;
   bool pair_ok(int l) const;  // two-sweep passes possible at level l
+  bool pencil_table(int l) const;  // the owned range of level l has a 2x2-brick pencil plan (kind 3)
   bool pair_ghosts_ok(int l) const;  // two-sweep passes may include the ghost shell at level l
   bool has_pair_table(int l, int64_t b0, int64_t b1) const;
   // `n` smooth(+residual) sweeps at level l.  last: 0 none, 1 write r, 2 fused restriction.

@@ -41,7 +41,7 @@ namespace mgb {
 namespace {
 
 constexpr int PN_ST = 2;          // TMA stages (half-layer chunks): chunk c+1 lands while chunk c is swept
-constexpr int PN_MINB = 6;        // resident CTAs per SM (37.4 KB of shared memory each; <= 168 registers)
+constexpr int PN_MINB = 4;        // resident CTAs per SM (53.3 KB of shared memory each)
 constexpr int PN_THREADS = 64;    // two warps: warp w = brick row w of the tile
 // stage layout, offsets in doubles.  Own bricks q = bx + 2 by at 264 q (2112 B apart: the two
 // bricks of a tile row sit 64 B apart modulo 128, so a quarter-warp's 128-bit loads of one tile
@@ -51,10 +51,11 @@ constexpr int XW = 1056, XE = 1184, XS = 1312, XN = 1440;  // 2 boxes of 64 each
 constexpr int BW = 1568, BE = 1696;                        // 2 boxes of 64: b of the W / E bricks
 constexpr int BS = 1824, BN = 1888;                        // 2 boxes of 32: b of the S / N bricks
 constexpr int COR = 1952;                                  // 4 boxes of 8 (16 apart): SW, NW, SE, NE
-constexpr int STAGE = 2016;
-constexpr int CHUNK_BYTES = 4 * 2048 + 8 * 512 + 4 * 512 + 4 * 256 + 4 * 64;
+constexpr int BOWN = 2016;  // b of the own bricks' half, same layout as the x0 bricks
+constexpr int STAGE = 3072;
 constexpr int PUB = 18 * 16;  // x1 of tile rows -1..16 (rows -1 / 16: the S / N ring)
 static_assert(STAGE * 8 % 128 == 0 && XW * 8 % 128 == 0 && BS * 8 % 128 == 0 && COR * 8 % 128 == 0, "align");
+static_assert(BOWN + 3 * OWN_STRIDE + 256 <= STAGE, "own b fits");
 static_assert(3 * OWN_STRIDE + 256 <= XW, "own bricks fit");
 __device__ __forceinline__ double2 lds_d2(const double* p) { return *reinterpret_cast<const double2*>(p); }
 constexpr int MRS = 4;  // chunk record ring slots (record n in slot n % 4)
@@ -154,10 +155,11 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     const int n = issued, s = n % PN_ST, code = mr(n, 0), half = code & 1;
     const bool rec = n + 1 >= 2 && n + 1 < cnt;
     const int id = l < 12 ? mr(n, 1 + (w == 0 ? l : l + 4)) : 0;
+    const int bid = (w == 0 && l >= 12 && l < 16) ? mr(n, 1 + l - 12) : 0;
     double* D = ST + s * STAGE;
     fence_proxy_async();
     if (l == 0)
-      mbar_expect_tx(&BAR[s], w == 0 ? 4 * 2048 + 8 * 512 : 4 * 512 + 4 * 256 + 4 * 64 + (rec ? kPenRec * 4 : 0));
+      mbar_expect_tx(&BAR[s], w == 0 ? 8 * 2048 + 8 * 512 : 4 * 512 + 4 * 256 + 4 * 64 + (rec ? kPenRec * 4 : 0));
     __syncwarp();
     const int kz = id * 8 + 4 * half;
     if (w == 0) {
@@ -168,6 +170,9 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
         const bool xf = l < 8, lowside = ((l - 4) & 2) == 0;  // W / S boxes sit at the high face
         tma_load_3d(D + XW + 64 * (l - 4), xf ? &mp.xwe : &mp.xsn, xf && lowside ? 6 : 0,
                     !xf && lowside ? 6 : 0, kz, &BAR[s]);
+      } else if (l < 16) {  // b of the own bricks (lanes 12-15 hold ids 0-3 too: see bid)
+        tma_load_1d_hint(D + BOWN + OWN_STRIDE * (l - 12), p.b + (int64_t)bid * 512 + 256 * half, 2048, &BAR[s],
+                         pol_keep);
       }
     } else {
       if (l < 4) {
@@ -193,21 +198,14 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
   };
 
   // ---- registers: x0 planes g-1, g, g+1; x1 planes g-2, g-1, g; b of planes g-1 .. g+2 ----
-  double2 Xm[2], Xc[2], Xp[2], Ym[2], Yc[2], Y[2], B[4][2];
+  double2 Xm[2], Xc[2], Xp[2], Ym[2], Yc[2], Y[2], Bm[2], Bc[2];
   double rcm = 0.0, rc = 0.0, rcp = 0.0, rpart = 0.0;
 #pragma unroll
   for (int r = 0; r < 2; ++r) {
     Xm[r] = Xc[r] = Xp[r] = Ym[r] = Yc[r] = Y[r] = make_double2(0.0, 0.0);
 #pragma unroll
-    for (int s = 0; s < 4; ++s) B[s][r] = make_double2(0.0, 0.0);
+    Bm[r] = Bc[r] = make_double2(0.0, 0.0);
   }
-  // b rows jb, jb+1 of my brick (always a valid brick id: unused chunks read brick 0)
-  auto load_b = [&](double2* dst, int id, int code, int kk) {
-    const double* bp = p.b + (int64_t)id * 512 + 64 * (4 * (code & 1) + kk) + 8 * jb + ib;
-    dst[0] = ld_hint2(bp, pol_keep);  // the neighbour tiles' b-face copies reuse these lines from L2
-    dst[1] = ld_hint2(bp + 8, pol_keep);
-  };
-
   // one step: sweep 1 on plane g = 4c + kk, sweep 2 on plane g - 1 (if it is a range plane)
   auto step = [&](const int c, auto kkc, const bool start, const bool sw2, const bool pref) {
     constexpr int kk = decltype(kkc)::value;
@@ -216,21 +214,14 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     const double* S1 = kk == 3 ? ST + ((c + 1) % PN_ST) * STAGE : S0;  // stage of plane g+1
     constexpr int kp = (kk + 1) & 3;                                   // its plane in that stage
     const int codeC = mr(c, 0), idC = mr(c, 1 + q);
-    // chunk c+1 (b prefetch from step kk = 2 on; its record came with chunk c)
-    const int codeN = (start || kk >= 2) ? mr(c + 1, 0) : 0, idN = (start || kk >= 2) ? mr(c + 1, 1 + q) : 0;
     if (start) {  // first step of a run (warm-up plane 7): prime the register windows
       Xm[0] = lds_d2(S0 + oO + 64 * (kk - 1)), Xm[1] = lds_d2(S0 + oO + 8 + 64 * (kk - 1));
       Xc[0] = lds_d2(S0 + oO + 64 * kk), Xc[1] = lds_d2(S0 + oO + 8 + 64 * kk);
       rcm = S0[oc + 16 * (kk - 1)];
       rc = S0[oc + 16 * kk];
-      load_b(B[kk], idC, codeC, kk);
-      load_b(B[(kk + 1) & 3], idN, codeN, 0);
     }
-    // b of plane g+2 into registers (harmless when that plane is not swept: `pref` only says it is
-    // needed).  (An L2 prefetch of plane g+4 on top measured slower: +0.9 GB of DRAM reads.)
     (void)pref;
-    if (kk < 2) load_b(B[(kk + 2) & 3], idC, codeC, kk + 2);
-    else load_b(B[(kk + 2) & 3], idN, codeN, kk - 2);
+    (void)idC;
     const int kz1 = 4 * (codeC & 1) + kk;  // in-brick plane of g (red-black colour)
 
     // ---------------- sweep 1, own cells, plane g ----------------
@@ -243,7 +234,8 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
       const double wl0 = __shfl_up_sync(FULL, Xc[0].y, 1), er0 = __shfl_down_sync(FULL, Xc[0].x, 1);
       const double wl1 = __shfl_up_sync(FULL, Xc[1].y, 1), er1 = __shfl_down_sync(FULL, Xc[1].x, 1);
       const double W0 = edW ? e0 : wl0, E0 = edE ? e0 : er0, W1 = edW ? e1 : wl1, E1 = edE ? e1 : er1;
-      const double2 bb0 = B[kk][0], bb1 = B[kk][1];
+      Bc[0] = lds_d2(S0 + BOWN + oO + 64 * kk), Bc[1] = lds_d2(S0 + BOWN + oO + 8 + 64 * kk);
+      const double2 bb0 = Bc[0], bb1 = Bc[1];
       const double a00 = stencil_a(Xc[0].x, W0, Xc[0].y, xs.x, Xc[1].x, Xm[0].x, Xp[0].x, alpha, beta);
       const double a10 = stencil_a(Xc[0].y, Xc[0].x, E0, xs.y, Xc[1].y, Xm[0].y, Xp[0].y, alpha, beta);
       const double a01 = stencil_a(Xc[1].x, W1, Xc[1].y, Xc[0].x, xn.x, Xm[1].x, Xp[1].x, alpha, beta);
@@ -280,7 +272,7 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
       const double wl1 = __shfl_up_sync(FULL, Yc[1].y, 1), er1 = __shfl_down_sync(FULL, Yc[1].x, 1);
       const double W0 = edW ? ed.x : wl0, E0 = edE ? ed.x : er0, W1 = edW ? ed.y : wl1, E1 = edE ? ed.y : er1;
       constexpr int km = (kk + 3) & 3;  // plane g-1 within its chunk
-      const double2 bb0 = B[km][0], bb1 = B[km][1];
+      const double2 bb0 = Bm[0], bb1 = Bm[1];  // b of plane g-1 (its stage may be refilled by now)
       const int code2 = kk > 0 ? codeC : mr(c + MRS - 1, 0), id2 = kk > 0 ? idC : mr(c + MRS - 1, 1 + q);
       const int kz2 = 4 * (code2 & 1) + km;
       const double a00 = stencil_a(Yc[0].x, W0, Yc[0].y, ys.x, Yc[1].x, Ym[0].x, Y[0].x, alpha, beta);
@@ -320,6 +312,7 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     for (int r = 0; r < 2; ++r) {
       Xm[r] = Xc[r], Xc[r] = Xp[r];
       Ym[r] = Yc[r], Yc[r] = Y[r];
+      Bm[r] = Bc[r];
     }
     rcm = rc, rc = rcp;
   };

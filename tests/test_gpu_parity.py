@@ -345,6 +345,28 @@ def test_full_size_512_sweep_sampled(oracle_mod):
     m.close()
 
 
+def test_full_size_512_pencil_pass_bitwise(oracle_mod):
+    """512^3 (the bench workload, launch configuration of bench.py: the 2x2-brick pencil pass over
+    592 CTAs): one two-sweep pass with r, every point against the oracle's two sweeps."""
+    mg, _ = _mg()
+    shape = (512, 512, 512)
+    m = new(shape, 6)
+    h = mg_inputs.default_h0(shape)
+    x = mg_inputs.random_field(shape, 26)
+    b = mg_inputs.sin_rhs(shape)
+    m.level_set(0, mg.MG_FIELD_X, dev(x))
+    m.level_set(0, mg.MG_FIELD_B, dev(b))
+    mg.mg_op_smooth(m.ctx, 0, 2, 1, 2)
+    gx = host(m.level_get(0, mg.MG_FIELD_X))
+    gr = host(m.level_get(0, mg.MG_FIELD_R))
+    m.close()
+    xo, ro = x, None
+    for _ in range(2):
+        xo, ro = oracle_mod.smooth_residual(xo, oracle_mod.apply_op(xo, h), b, h)
+    assert_bitwise(gx, xo, what="x")
+    assert_bitwise(gr, ro, what="r")
+
+
 @pytest.mark.slow
 def test_full_size_512_vcycle_bitwise(oracle_mod):
     """512^3, L = 6, 12/12/100 (bench configuration): one full V-cycle bitwise + norm."""
