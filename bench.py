@@ -292,11 +292,11 @@ def main():
         m.vcycle()
     torch.cuda.synchronize()
     tm = m.timings()
+    recs = m.timing_records()  # (mg_set_timing clears them)
     m.set_timing(False)
     nsweep0 = a.pre + a.post
     # every level-0 pass of the instrumented cycles, from the per-op records (two-sweep passes and any
     # single sweeps alike; the interpolation is its own op where the pencil passes run)
-    recs = m.timing_records()
     passes0 = [ms for (lv, op, ms) in recs if lv == 0 and op == mg.OP_NAMES.index("sweep")]
     sweep0_ms = sum(passes0) / ninst
     npass0 = round(len(passes0) / ninst)
