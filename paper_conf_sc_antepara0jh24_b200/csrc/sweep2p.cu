@@ -59,7 +59,10 @@ static_assert(BOWN + 3 * OWN_STRIDE + 256 <= STAGE, "own b fits");
 static_assert(3 * OWN_STRIDE + 256 <= XW, "own bricks fit");
 __device__ __forceinline__ double2 lds_d2(const double* p) { return *reinterpret_cast<const double2*>(p); }
 constexpr int MRS = 4;  // chunk record ring slots (record n in slot n % 4)
-constexpr size_t SMEM_BYTES = (size_t)(PN_ST * STAGE + 2 * PUB + 2 * 32) * 8 + 16 + MRS * kPenRec * 4;
+// ring x1 columns per parity: W rows 0-15 at 0, E rows at 18 (the two columns' rows sit in
+// different banks, so the edge lanes' 128-bit loads of a quarter-warp do not conflict)
+constexpr int RWE_E = 18, RWE_PAR = 36;
+constexpr size_t SMEM_BYTES = (size_t)(PN_ST * STAGE + 2 * PUB + 2 * RWE_PAR) * 8 + 16 + MRS * kPenRec * 4;
 
 }  // namespace
 
@@ -74,8 +77,8 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
   extern __shared__ __align__(128) unsigned char smem_raw[];
   double* const ST = reinterpret_cast<double*>(smem_raw);  // [PN_ST][STAGE]
   double* const XP = ST + PN_ST * STAGE;                    // [2][PUB]  x1 of tile rows -1..16
-  double* const RWE = XP + 2 * PUB;                         // [2][2][16] x1 of the W / E ring columns
-  uint64_t* const BAR = reinterpret_cast<uint64_t*>(RWE + 64);
+  double* const RWE = XP + 2 * PUB;                         // [2][RWE_PAR] x1 of the W / E ring columns
+  uint64_t* const BAR = reinterpret_cast<uint64_t*>(RWE + 2 * RWE_PAR);
   int* const MR = reinterpret_cast<int*>(BAR + 2);  // [MRS][kPenRec] chunk records, 16-byte aligned slots
   const int col1 = COLOUR ? p.colour : -1, col2 = COLOUR ? p.colour2 : -1;
   const int t = threadIdx.x, w = t >> 5, l = t & 31;
@@ -100,7 +103,7 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
   const int oEd = edE ? XE + 64 * w + 2 * jb : XW + 64 * w + 2 * jb + 1;  // tile-edge W / E x0 (rows jb, jb+1: +2)
   const int R0 = 8 * w + jb;                                              // tile row of my row 0
   const int pO = (R0 + 1) * 16 + 2 * pc;                                  // my row 0 in the x1 buffer
-  const int oRwe = (edE ? 16 : 0) + R0;                                   // ring x1 column, rows R0, R0+1
+  const int oRwe = (edE ? RWE_E : 0) + R0;                                // ring x1 column, rows R0, R0+1
 
   // ---- ring role: x1 of one cell of the 1-cell ring around the tile ----
   int oc, oo, oown, olo, slo, ohi, shi, ob, sb, oout, rstr, rci, rcj;
@@ -117,7 +120,7 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     else if (w == 0) ohi = X + 64 + cc, shi = 16;
     else ohi = COR + (side ? 48 : 16) + cc, shi = 2;  // NW / NE corner
     ob = (side ? BE : BW) + 64 * w + 2 * j + cc, sb = 16;
-    oout = 2 * PUB + 16 * side + 8 * w + j, rstr = 32;  // RWE[par][side][row] (RWE = XP + 2 PUB)
+    oout = 2 * PUB + RWE_E * side + 8 * w + j, rstr = RWE_PAR;  // RWE[par][side col + row] (RWE = XP + 2 PUB)
     rci = side ? 0 : 7, rcj = j;
   } else {  // S (warp 0) / N (warp 1) row, tile column i
     const int i = l - 16, i8 = i & 7, bxr = i >> 3;
@@ -267,7 +270,7 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
       constexpr int par = (kk + 1) & 1;  // parity of plane g - 1
       const double* P = XP + par * PUB;
       const double2 ys = lds_d2(P + pO - 16), yn = lds_d2(P + pO + 32);
-      const double2 ed = lds_d2(RWE + 32 * par + oRwe);
+      const double2 ed = lds_d2(RWE + RWE_PAR * par + oRwe);
       const double wl0 = __shfl_up_sync(FULL, Yc[0].y, 1), er0 = __shfl_down_sync(FULL, Yc[0].x, 1);
       const double wl1 = __shfl_up_sync(FULL, Yc[1].y, 1), er1 = __shfl_down_sync(FULL, Yc[1].x, 1);
       const double W0 = edW ? ed.x : wl0, E0 = edE ? ed.x : er0, W1 = edW ? ed.y : wl1, E1 = edE ? ed.y : er1;
