@@ -248,6 +248,13 @@ mg_status mg_group_destroy(mg_group* g);
  * parent: int32 [stored] = coarse brick index*8 + octant (-1 if none).
  * plan: int64 [runs][6] = peer, direction(0..26), run index, local brick offset,
  * remote brick offset, brick count.
+ * pass plan: the two-sweep (temporal blocking) plan number `idx` of a level (one per swept brick
+ * range).  info[0] kind (1 one-brick CTA streams, 2 warp plane streams, 3 2x2-brick pencil chunk
+ * streams), [1] b0, [2] b1 (brick range), [3] ints of meta, [4] ints of ctas; MG_ERR_INVALID_ARG
+ * if idx is past the last plan.  meta / ctas (may be NULL: sizes only) receive copies of the
+ * tables the kernel reads; for kind 3, meta = int32 [chunks][20] = code (type << 1 | half; type 0
+ * range, 1 warm-up, 2 cool-down), ids of b00, b10, b01, b11, W0, W1, E0, E1, S0, S1, N0, N1, SW,
+ * NW, SE, NE, parent of b00, 0, 0; ctas = int32 [ctas][2] = first chunk, chunk count.
  * -------------------------------------------------------------------------- */
 mg_status mg_layout_create(const mg_params* p, int32_t rank, int32_t world_size, mg_layout** out);
 mg_status mg_layout_level_info(const mg_layout* lay, int32_t level, int64_t info[16]);
@@ -255,6 +262,8 @@ mg_status mg_layout_adjacency(const mg_layout* lay, int32_t level, int32_t* out)
 mg_status mg_layout_coords(const mg_layout* lay, int32_t level, int32_t* out);
 mg_status mg_layout_parent(const mg_layout* lay, int32_t level, int32_t* out);
 mg_status mg_layout_plan(const mg_layout* lay, int32_t level, int32_t which /*0 send,1 recv*/, int64_t* out);
+mg_status mg_layout_pass_plan(const mg_layout* lay, int32_t level, int32_t idx, int64_t info[5], int32_t* meta,
+                              int32_t* ctas);
 mg_status mg_layout_destroy(mg_layout* lay);
 
 #ifdef __cplusplus

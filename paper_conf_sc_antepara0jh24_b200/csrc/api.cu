@@ -1215,6 +1215,23 @@ mg_status mg_layout_plan(const mg_layout* m, int32_t level, int32_t which, int64
   return MG_OK;
 }
 
+mg_status mg_layout_pass_plan(const mg_layout* m, int32_t level, int32_t idx, int64_t info[5], int32_t* meta,
+                              int32_t* ctas) {
+  const LevelLayout* L = nullptr;
+  CKS(lay_level(m, level, &L));
+  if (!info) return set_err(MG_ERR_INVALID_ARG, "null info");
+  if (idx < 0 || idx >= (int32_t)L->pairs.size()) return set_err(MG_ERR_INVALID_ARG, "no such pass plan");
+  const auto& t = L->pairs[(size_t)idx];
+  info[0] = t.kind;
+  info[1] = t.b0;
+  info[2] = t.b1;
+  info[3] = (int64_t)t.meta.size();
+  info[4] = (int64_t)t.ctas.size();
+  if (meta) std::copy(t.meta.begin(), t.meta.end(), meta);
+  if (ctas) std::copy(t.ctas.begin(), t.ctas.end(), ctas);
+  return MG_OK;
+}
+
 mg_status mg_layout_destroy(mg_layout* m) {
   delete m;
   return MG_OK;

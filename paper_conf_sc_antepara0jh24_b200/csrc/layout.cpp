@@ -266,7 +266,8 @@ mg_status build_layout(const mg_params& p, int rank, int world, Layout& out, std
   for (int l = 0; l + 1 < out.L; ++l) build_parents(out.lv[l], out.lv[l + 1]);
   if (p.temporal_blocking != 0)
     for (int l = 0; l < out.L; ++l)
-      build_pair_tables(out.lv[l], min_b, p.temporal_blocking == 2 ? 2 : p.temporal_blocking == 3 ? 3 : 1);
+      build_pair_tables(out.lv[l], p.sweep_kernel == 0 ? kPairMinBricks : min_b,
+                        p.temporal_blocking == 2 ? 2 : p.temporal_blocking == 3 ? 3 : 1);
   return MG_OK;
 }
 

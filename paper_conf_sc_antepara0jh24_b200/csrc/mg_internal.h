@@ -116,6 +116,10 @@ void build_pair_tables(LevelLayout& L, int64_t min_bricks, int kind);
 
 constexpr int kColSeg = 16;             // bricks per streamed segment
 constexpr int64_t kColMinBricks = 16384;  // levels smaller than this use the one-brick-per-CTA kernel
+// two-sweep passes (auto kernel choice) from this level size on: at 512^3 levels 0-2 (level 2 =
+// 128^3, 4096 bricks: pencil passes 0.29 vs 0.43 ms of single sweeps per cycle; 512 bricks measured
+// no better in graph replay)
+constexpr int64_t kPairMinBricks = 4096;
 void build_col_tables(LevelLayout& L, int64_t min_bricks);
 
 struct Layout {

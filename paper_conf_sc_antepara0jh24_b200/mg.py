@@ -110,6 +110,8 @@ _SIGS = {
     "mg_layout_coords": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_void_p]),
     "mg_layout_parent": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_void_p]),
     "mg_layout_plan": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32, ctypes.c_void_p]),
+    "mg_layout_pass_plan": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32, ctypes.c_void_p,
+                                           ctypes.c_void_p, ctypes.c_void_p]),
     "mg_layout_destroy": (ctypes.c_int, [ctypes.c_void_p]),
 }
 
@@ -377,6 +379,21 @@ class Layout:
         a = self._np.zeros(inf["owned"] + inf["nghost"], dtype=self._np.int32)
         check(lib().mg_layout_parent(self.h, level, a.ctypes.data), "mg_layout_parent")
         return a
+
+    def pass_plans(self, level):
+        """Two-sweep pass plans of a level: [(kind, b0, b1, meta int32 array, ctas int32 [n][2])]."""
+        np = self._np
+        out = []
+        for idx in range(64):
+            info = (ctypes.c_int64 * 5)()
+            if lib().mg_layout_pass_plan(self.h, level, idx, info, None, None) != 0:
+                break
+            meta = np.zeros(max(info[3], 1), dtype=np.int32)
+            ctas = np.zeros(max(info[4], 2), dtype=np.int32)
+            check(lib().mg_layout_pass_plan(self.h, level, idx, info, meta.ctypes.data, ctas.ctypes.data),
+                  "mg_layout_pass_plan")
+            out.append((info[0], info[1], info[2], meta[:info[3]], ctas[:info[4]].reshape(-1, 2)))
+        return out
 
     def plan(self, level, which):
         inf = self.info(level)

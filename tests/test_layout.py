@@ -178,3 +178,62 @@ def test_invalid_params_rejected():
     p = mg.params((32, 32, 32), num_levels=2, ca_period=9)
     with pytest.raises(mg.MGError):
         mg.Layout(p, 0, 1)
+
+
+# ------------------------------------------------- two-sweep pencil plans (sweep2p.cu, kind 3)
+W_, E_, S_, N_, B_, T_ = range(6)
+
+
+@pytest.mark.parametrize("n_local,pg,L,gm", [((128, 128, 128), (1, 1, 1), 3, 0), ((256, 128, 64), (1, 1, 1), 2, 0),
+                                            ((128, 128, 128), (1, 1, 1), 2, 1), ((128, 128, 128), (2, 1, 1), 2, 0),
+                                            ((512, 512, 512), (1, 1, 1), 2, 0)])
+def test_pencil_plan_covers_owned_bricks(n_local, pg, L, gm):
+    """Every owned brick is swept exactly once per half by the pencil chunk streams; each record's
+    16 ids are the tile layer's bricks and neighbours by the adjacency table; tiles sit on even
+    brick coordinates (one coarse brick's x-y octants 0-3); runs are [warm-up, layers linked by T,
+    cool-down] with the B / T neighbour layers; every CTA gets the same work to within a run."""
+    p, lays = layouts(n_local, pg, L, gm)
+    lay = lays[0]
+    inf = lay.info(0)
+    adj, crd = lay.adjacency(0), lay.coords(0)
+    par = lay.parent(0) if L > 1 else None
+    plans = [pl for pl in lay.pass_plans(0) if pl[0] == 3]
+    assert len(plans) == 1 and plans[0][1] == 0 and plans[0][2] == inf["owned"]
+    _, _, _, meta, ctas = plans[0]
+    rec = meta.reshape(-1, 20)
+    seen = np.zeros((inf["owned"], 2), dtype=np.int64)
+    work = []
+    for first, count in ctas:
+        chunks = rec[first:first + count]
+        types = (chunks[:, 0] >> 1) & 3
+        halves = chunks[:, 0] & 1
+        w, m = 0, 0
+        while m < count:
+            assert types[m] == 1 and halves[m] == 1  # warm-up half 1
+            e = m + 1
+            while types[e] == 0:
+                e += 1
+            assert types[e] == 2 and halves[e] == 0  # cool-down half 0
+            rng = chunks[m + 1:e]
+            assert len(rng) % 2 == 0 and (halves[m + 1:e] == np.tile([0, 1], len(rng) // 2)).all()
+            layers = rng[::2, 1]
+            assert chunks[m, 1] == adj[layers[0], B_] and chunks[e, 1] == adj[layers[-1], T_]
+            assert all(adj[a, T_] == b for a, b in zip(layers[:-1], layers[1:]))
+            w += 4 * len(layers) + 1
+            m = e + 1
+        work.append(w)
+        for r in chunks:
+            b00, b10, b01, b11, W0, W1, E0, E1, S0, S1, N0, N1, SW, NW, SE, NE, pa = r[1:18]
+            assert (b10, b01, b11) == (adj[b00, E_], adj[b00, N_], adj[b10, N_]) and adj[b01, E_] == b11
+            assert (W0, W1, E0, E1) == (adj[b00, W_], adj[b01, W_], adj[b10, E_], adj[b11, E_])
+            assert (S0, S1, N0, N1) == (adj[b00, S_], adj[b10, S_], adj[b01, N_], adj[b11, N_])
+            assert (SW, NW, SE, NE) == (adj[W0, S_], adj[W1, N_], adj[E0, S_], adj[E1, N_])
+            if (r[0] >> 1) & 3 == 0:
+                assert crd[b00, 0] % 2 == 0 and crd[b00, 1] % 2 == 0
+                for k, b in enumerate((b00, b10, b01, b11)):
+                    seen[b, r[0] & 1] += 1
+                    if par is not None:
+                        assert pa % 4 == 0 and par[b] == pa + k
+    assert (seen == 1).all()
+    ideal = sum(work) / len(work)
+    assert max(work) <= ideal * 1.15 + 8
