@@ -369,7 +369,7 @@ mg_status exec_op(mg_ctx* c, const Op& o, cudaStream_t s) {
     case OP_SWEEP2: {
       const int64_t end = o.ghosts ? L.n_stored : L.n_owned;
       if (o.exch_before) {
-        const bool split = c->lay.p.overlap && L.n_interior > 0;
+        const bool split = c->lay.p.overlap && L.n_interior > 0 && !o.nosplit;
         if (split) {
           CKS(timer_begin(c, s, &t0));
           CKC(c, cudaEventRecord(c->ev_fork, s));

@@ -414,18 +414,26 @@ static LevelLayout::PairTable pair_table(const LevelLayout& L, int64_t b0, int64
 // becomes chunks [warm-up layer half 1, (layer half 0, half 1)..., cool-down layer half 0], each
 // a record of kPenRec ints (code, the tile layer's 16 brick ids, parent);
 // warm-up / cool-down are the B / T neighbour layers (their x1 planes 7 / 0 are the k-halos of
-// the run's second sweep).  Returns kind 0 if the range does not tile.
+// the run's second sweep).  Also for the whole stored range of a level with a ghost shell
+// (two-sweep passes that sweep the ghosts redundantly, so one exchange serves several passes):
+// there the tiles cover the extended box (owned + ghost layer), aligned to its origin, and no
+// restriction runs.  Returns kind 0 if the range does not tile.
 static LevelLayout::PairTable pencil_table(const LevelLayout& L, int64_t b0, int64_t b1) {
   LevelLayout::PairTable t;
   t.kind = 0;
-  if (b0 != 0 || b1 != L.n_owned || (L.nb[0] & 1) || (L.nb[1] & 1) || L.n_owned <= 0) return t;
+  const bool owned = b0 == 0 && b1 == L.n_owned;
+  const bool stored = b0 == 0 && b1 == L.n_stored && L.n_ghost > 0;
+  if ((!owned && !stored) || L.n_owned <= 0) return t;
+  const int gx = stored ? L.g[0] : 0, gy = stored ? L.g[1] : 0, gz = stored ? L.g[2] : 0;
+  const int ex = L.nb[0] + 2 * gx, ey = L.nb[1] + 2 * gy;
+  if ((ex & 1) || (ey & 1)) return t;
   auto adj = [&](int64_t id, int f) -> int32_t {
     return id >= L.n_stored ? (int32_t)L.zero_brick : L.adj[(size_t)id * 8 + f];
   };
   auto par = [&](int64_t id) -> int32_t {
     return (id < L.n_stored && !L.parent.empty()) ? L.parent[(size_t)id] : -1;
   };
-  const int tx = L.nb[0] / 2, ty = L.nb[1] / 2, nz = L.nb[2];
+  const int tx = ex / 2, ty = ey / 2, nz = L.nb[2] + 2 * gz;
   // items of every tile layer: [tile][z]
   std::vector<std::array<int32_t, kPenMeta>> layers((size_t)tx * ty * nz);
   auto make_item = [&](int32_t b00) -> std::array<int32_t, kPenMeta> {
@@ -441,15 +449,16 @@ static LevelLayout::PairTable pencil_table(const LevelLayout& L, int64_t b0, int
   for (int py = 0; py < ty; ++py)
     for (int px = 0; px < tx; ++px)
       for (int z = 0; z < nz; ++z) {
-        const int64_t b00 = L.ext_index(2 * px, 2 * py, z);
-        if (b00 < 0 || b00 >= L.n_owned) return t;
+        const int X = 2 * px - gx, Y = 2 * py - gy, Z = z - gz;
+        const int64_t b00 = L.ext_index(X, Y, Z);
+        if (b00 < 0 || b00 >= b1) return t;
         auto m = make_item((int32_t)b00);
-        // the tile must be the 2x2 block of owned bricks at (2px.., 2py..) and (for restriction)
-        // one coarse brick's octants 0..3 (+4 for odd z)
-        if (m[1] != L.ext_index(2 * px + 1, 2 * py, z) || m[2] != L.ext_index(2 * px, 2 * py + 1, z) ||
-            m[3] != L.ext_index(2 * px + 1, 2 * py + 1, z) || adj(m[2], 1) != m[3])
+        // the tile must be the 2x2 block of bricks at (X.., Y..) and (owned range, for the fused
+        // restriction) one coarse brick's octants 0..3 (+4 for odd z)
+        if (m[1] != L.ext_index(X + 1, Y, Z) || m[2] != L.ext_index(X, Y + 1, Z) ||
+            m[3] != L.ext_index(X + 1, Y + 1, Z) || adj(m[2], 1) != m[3])
           return t;
-        if (m[16] >= 0)
+        if (owned && m[16] >= 0)
           for (int k = 1; k < 4; ++k)
             if (par(m[(size_t)k]) != m[16] + k || (m[16] & 3) != 0) return t;
         layers[((size_t)py * tx + px) * nz + z] = m;

@@ -34,6 +34,14 @@ bool Builder::pencil_table(int l) const {
   return false;
 }
 
+bool Builder::pencil_ghosts(int l) const {
+  const LevelLayout& L = lay.lv[l];
+  if (L.n_ghost == 0) return false;
+  for (const auto& pt : L.pairs)
+    if (pt.b0 == 0 && pt.b1 == L.n_stored) return pt.kind == 3;
+  return false;
+}
+
 bool Builder::pair_ok(int l) const {
   if (!lay.p.temporal_blocking || fusion(l) == MG_FUSION_PAPER) return false;
   const LevelLayout& L = lay.lv[l];
@@ -50,6 +58,7 @@ bool Builder::pair_ok(int l) const {
 bool Builder::pair_ghosts_ok(int l) const {
   const LevelLayout& L = lay.lv[l];
   if (!has_pair_table(l, 0, L.n_stored)) return false;
+  if (pencil_table(l) && pencil_ghosts(l)) return true;  // pencil passes run unsplit
   return !(lay.p.overlap && L.n_interior > 0) || has_pair_table(l, L.n_interior, L.n_stored);
 }
 
@@ -88,6 +97,9 @@ void Builder::phase(int l, int n, bool zero_first, int last, bool interp_first, 
         S.since = 0;
       }
       o.exch_before = ex;
+      // pencil passes exchange first and then sweep the whole range (they do not tile the surface
+      // shell, so there is no interior / surface overlap split)
+      o.nosplit = pencil_table(l);
       // ghost validity after two sweeps over the ghost shell too (x1 needs x0 one cell further
       // out and b at its own depth; x2 likewise from x1): min(d_x - 2, d_b - 1)
       const int d_inc = std::min(S.dx - 2, S.db - 1);
@@ -284,7 +296,8 @@ void Builder::vcycle() {
     // interpolation fused into the first post-sweep -- except where pencil passes run (their
     // kernel has no interpolation input): a separate interpolation then lets all post-sweeps pair
     // up (measured faster: one-brick interp-fused sweeps are the slowest single sweeps)
-    const bool pencil_pairs = pair_ok(l) && pencil_table(l) && p.post_smooths % 2 == 0 && lay.p.smoother != 2;
+    const int nh = lay.p.smoother == 2 ? 2 * p.post_smooths : p.post_smooths;  // (half-)sweeps
+    const bool pencil_pairs = pair_ok(l) && pencil_table(l) && nh % 2 == 0;
     const bool fuse_i = fusion(l) == MG_FUSION_FULL && !ghosts(l) && p.post_smooths > 0 && !pencil_pairs;
     if (!fuse_i) interp_op(l);
     phase(l, p.post_smooths, false, 0, fuse_i, MG_OP_SWEEP);
@@ -296,7 +309,7 @@ int64_t op_launches(const Op& o, const Layout& lay, bool overlap) {
     case OP_SWEEP:
     case OP_SWEEP2: {
       const int per = o.paper ? 2 : 1;
-      const bool split = o.exch_before && overlap && lay.lv[o.level].n_interior > 0;
+      const bool split = o.exch_before && overlap && lay.lv[o.level].n_interior > 0 && !o.nosplit;
       return per * (split ? 2 : 1);
     }
     case OP_RESTRICT:

@@ -37,6 +37,7 @@ struct Op {
   int timer = 0;            // MG_OP_*
   double g1 = 0, g2 = 0;    // smoothing steps of the (first, second) sweep; 0 = the level's Jacobi h^2/12
   int c1 = -1, c2 = -1;     // red-black colour of the (first, second) half-sweep (GSRB); -1 = every cell
+  bool nosplit = false;     // exchange before the whole sweep (pencil passes: no interior / surface split)
 };
 
 struct LevelState {
@@ -58,6 +59,7 @@ struct Builder {
   int period(int l) const;
   bool pair_ok(int l) const;  // two-sweep passes possible at level l
   bool pencil_table(int l) const;  // the owned range of level l has a 2x2-brick pencil plan (kind 3)
+  bool pencil_ghosts(int l) const;  // ... and so has its whole stored range (owned + ghost shell)
   bool pair_ghosts_ok(int l) const;  // two-sweep passes may include the ghost shell at level l
   bool has_pair_table(int l, int64_t b0, int64_t b1) const;
   // `n` smooth(+residual) sweeps at level l.  last: 0 none, 1 write r, 2 fused restriction.

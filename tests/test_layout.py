@@ -198,10 +198,22 @@ def test_pencil_plan_covers_owned_bricks(n_local, pg, L, gm):
     adj, crd = lay.adjacency(0), lay.coords(0)
     par = lay.parent(0) if L > 1 else None
     plans = [pl for pl in lay.pass_plans(0) if pl[0] == 3]
-    assert len(plans) == 1 and plans[0][1] == 0 and plans[0][2] == inf["owned"]
-    _, _, _, meta, ctas = plans[0]
+    # the owned range (tiles on even owned coordinates: restriction), and with a ghost shell the
+    # whole stored range (tiles on the extended box, ghost-sweeping passes)
+    want = [(0, inf["owned"])] + ([(0, inf["owned"] + inf["nghost"])] if inf["nghost"] else [])
+    assert [(pl[1], pl[2]) for pl in plans] == want
+    for _, b0, b1, meta, ctas in plans:
+        owned = b1 == inf["owned"]
+        g = np.array(inf["ghost"][:2]) * (0 if owned else 1)
+        _check_pencil_plan(meta, ctas, b1, adj, crd, par if owned else None, g)
+
+
+def _check_pencil_plan(meta, ctas, nrange, adj, crd, par, g):
+    # neighbours past the outermost ghosts are the zero brick (index = stored count), whose own
+    # neighbours are the zero brick again
+    adj = np.vstack([adj, np.full((1, 8), adj.shape[0], dtype=adj.dtype)])
     rec = meta.reshape(-1, 20)
-    seen = np.zeros((inf["owned"], 2), dtype=np.int64)
+    seen = np.zeros((nrange, 2), dtype=np.int64)
     work = []
     for first, count in ctas:
         chunks = rec[first:first + count]
@@ -229,7 +241,7 @@ def test_pencil_plan_covers_owned_bricks(n_local, pg, L, gm):
             assert (S0, S1, N0, N1) == (adj[b00, S_], adj[b10, S_], adj[b01, N_], adj[b11, N_])
             assert (SW, NW, SE, NE) == (adj[W0, S_], adj[W1, N_], adj[E0, S_], adj[E1, N_])
             if (r[0] >> 1) & 3 == 0:
-                assert crd[b00, 0] % 2 == 0 and crd[b00, 1] % 2 == 0
+                assert (crd[b00, 0] + g[0]) % 2 == 0 and (crd[b00, 1] + g[1]) % 2 == 0
                 for k, b in enumerate((b00, b10, b01, b11)):
                     seen[b, r[0] & 1] += 1
                     if par is not None:
