@@ -91,12 +91,12 @@ def main():
         out.append(run("fit_paper", n, lv, fusion=[1] * 16, temporal_blocking=0))
         out.append(run("fit_default", n, lv))
     # config 3: 512^3 in self-exchange mode (ghost shell on every axis, local copies):
-    # CA period k and smooth count s; temporal blocking on / off
+    # CA period k and smooth count s; temporal blocking off / one-brick kernel / pencils (default)
     ks = (1, 2, 4, 8)
     ss = (12,) if a.quick else (4, 8, 12, 16)
     for s in ss:
         for k in ks:
-            for tb in ((1,) if s != 12 else (0, 1)):
+            for tb in ((3,) if s != 12 else (0, 1, 3)):
                 out.append(run("c3", 512, 6, pre=s, post=s, ghost_mode=1, transport=2, ca_period=[k] * 16,
                                temporal_blocking=tb))
     # config 3: fusion variants (no ghosts)

@@ -12,8 +12,9 @@ def desc(r):
     parts = []
     fu = r.get("fusion", [0])[0]
     parts.append({0: "fusion auto(full)", 1: "paper kernel set", 2: "fused sweep", 3: "full fusion"}[fu])
-    tb = r.get("temporal_blocking", 1) if fu != 1 else 0
-    parts.append({0: "1 sweep/pass", 1: "2 sweeps/pass", 2: "2 sweeps/pass (warp streams)"}[tb])
+    tb = r.get("temporal_blocking", 3) if fu != 1 else 0
+    parts.append({0: "1 sweep/pass", 1: "2 sweeps/pass (one-brick CTA streams)", 2: "2 sweeps/pass (warp streams)",
+                  3: "2 sweeps/pass (2x2-brick pencils)"}[tb])
     if r.get("ghost_mode"):
         parts.append(f"self-exchange k={r['ca_period'][0]}")
     if r.get("pre") is not None:

@@ -45,7 +45,7 @@ def samples(runs):
             else:
                 x = float(nl ** 3)
             if x:
-                out.append((name, x, ms, r["tag"], r.get("temporal_blocking", 1), lvl, r.get("fusion", [0])[0]))
+                out.append((name, x, ms, r["tag"], r.get("temporal_blocking", 3), lvl, r.get("fusion", [0])[0]))
     return out
 
 
