@@ -201,13 +201,14 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
   };
 
   // ---- registers: x0 planes g-1, g, g+1; x1 planes g-2, g-1, g; b of planes g-1 .. g+2 ----
-  double2 Xm[2], Xc[2], Xp[2], Ym[2], Yc[2], Y[2], Bm[2], Bc[2];
-  double rcm = 0.0, rc = 0.0, rcp = 0.0, rpart = 0.0;
+  // rings indexed by plane mod 4 (= the step's kk, a compile-time constant: no register moves
+  // between steps): x0 (planes g-1..g+1), x1 (g-2..g), b (g-1, g), the ring cell's x0 (g-1..g+1)
+  double2 XR[4][2], YR[4][2], BR[4][2];
+  double RR[4] = {0.0, 0.0, 0.0, 0.0}, rpart = 0.0;
 #pragma unroll
   for (int r = 0; r < 2; ++r) {
-    Xm[r] = Xc[r] = Xp[r] = Ym[r] = Yc[r] = Y[r] = make_double2(0.0, 0.0);
 #pragma unroll
-    Bm[r] = Bc[r] = make_double2(0.0, 0.0);
+    for (int s = 0; s < 4; ++s) XR[s][r] = YR[s][r] = BR[s][r] = make_double2(0.0, 0.0);
   }
   // one step: sweep 1 on plane g = 4c + kk, sweep 2 on plane g - 1 (if it is a range plane)
   auto step = [&](const int c, auto kkc, const bool start, const bool sw2, const bool pref) {
@@ -216,6 +217,18 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     if (kk == 3) wait_upto(c + 1);
     const double* S1 = kk == 3 ? ST + ((c + 1) % PN_ST) * STAGE : S0;  // stage of plane g+1
     constexpr int kp = (kk + 1) & 3;                                   // its plane in that stage
+    constexpr int km1 = (kk + 3) & 3, km2 = (kk + 2) & 3;              // ring slots of planes g-1, g-2
+    double2(&Xm)[2] = XR[km1];
+    double2(&Xc)[2] = XR[kk];
+    double2(&Xp)[2] = XR[kp];
+    double2(&Ym)[2] = YR[km2];
+    double2(&Yc)[2] = YR[km1];
+    double2(&Y)[2] = YR[kk];
+    double2(&Bm)[2] = BR[km1];
+    double2(&Bc)[2] = BR[kk];
+    double& rcm = RR[km1];
+    double& rc = RR[kk];
+    double& rcp = RR[kp];
     const int codeC = mr(c, 0), idC = mr(c, 1 + q);
     if (start) {  // first step of a run (warm-up plane 7): prime the register windows
       Xm[0] = lds_d2(S0 + oO + 64 * (kk - 1)), Xm[1] = lds_d2(S0 + oO + 8 + 64 * (kk - 1));
@@ -311,13 +324,6 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
       }
     }
     __syncthreads();  // x1 of plane g published; stage c (and c+1) reads of this step done
-#pragma unroll
-    for (int r = 0; r < 2; ++r) {
-      Xm[r] = Xc[r], Xc[r] = Xp[r];
-      Ym[r] = Yc[r], Yc[r] = Y[r];
-      Bm[r] = Bc[r];
-    }
-    rcm = rc, rc = rcp;
   };
 
   __syncthreads();  // records 0, 1
