@@ -103,7 +103,7 @@ constexpr int64_t kPairCtas = 148 * kPairCtasPerSm;  // one item stream per resi
 // SW, NW, SE, NE (diagonal corners), parent of b00, 0, 0; ctas = (first record, record count).
 constexpr int kPenMeta = 20;  // host-side tile-layer item: the 16 ids, parent, 0, 0, 0
 constexpr int kPenRec = 20;   // chunk record (80 bytes: one 1D bulk copy)
-constexpr int kPenCtasPerSm = 4;                    // resident pencil CTAs per SM (shared-memory bound)
+constexpr int kPenCtasPerSm = 6;                    // resident pencil CTAs per SM (shared-memory bound)
 constexpr int64_t kPenCtas = 148 * kPenCtasPerSm;
 constexpr int kW2Meta = 12;
 constexpr int kW2WarpsPerSm = 7;                    // resident one-warp CTAs per SM (shared-memory bound)

@@ -41,7 +41,7 @@ namespace mgb {
 namespace {
 
 constexpr int PN_ST = 2;          // TMA stages (half-layer chunks): chunk c+1 lands while chunk c is swept
-constexpr int PN_MINB = 4;        // resident CTAs per SM (53.3 KB of shared memory each)
+constexpr int PN_MINB = 6;        // resident CTAs per SM (37.8 KB of shared memory each, <= 168 registers)
 constexpr int PN_THREADS = 64;    // two warps: warp w = brick row w of the tile
 // stage layout, offsets in doubles.  Own bricks q = bx + 2 by at 264 q (2112 B apart: the two
 // bricks of a tile row sit 64 B apart modulo 128, so a quarter-warp's 128-bit loads of one tile
@@ -51,11 +51,9 @@ constexpr int XW = 1056, XE = 1184, XS = 1312, XN = 1440;  // 2 boxes of 64 each
 constexpr int BW = 1568, BE = 1696;                        // 2 boxes of 64: b of the W / E bricks
 constexpr int BS = 1824, BN = 1888;                        // 2 boxes of 32: b of the S / N bricks
 constexpr int COR = 1952;                                  // 4 boxes of 8 (16 apart): SW, NW, SE, NE
-constexpr int BOWN = 2016;  // b of the own bricks' half, same layout as the x0 bricks
-constexpr int STAGE = 3072;
+constexpr int STAGE = 2016;
 constexpr int PUB = 18 * 16;  // x1 of tile rows -1..16 (rows -1 / 16: the S / N ring)
 static_assert(STAGE * 8 % 128 == 0 && XW * 8 % 128 == 0 && BS * 8 % 128 == 0 && COR * 8 % 128 == 0, "align");
-static_assert(BOWN + 3 * OWN_STRIDE + 256 <= STAGE, "own b fits");
 static_assert(3 * OWN_STRIDE + 256 <= XW, "own bricks fit");
 __device__ __forceinline__ double2 lds_d2(const double* p) { return *reinterpret_cast<const double2*>(p); }
 constexpr int MRS = 4;  // chunk record ring slots (record n in slot n % 4)
@@ -158,11 +156,10 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     const int n = issued, s = n % PN_ST, code = mr(n, 0), half = code & 1;
     const bool rec = n + 1 >= 2 && n + 1 < cnt;
     const int id = l < 12 ? mr(n, 1 + (w == 0 ? l : l + 4)) : 0;
-    const int bid = (w == 0 && l >= 12 && l < 16) ? mr(n, 1 + l - 12) : 0;
     double* D = ST + s * STAGE;
     fence_proxy_async();
     if (l == 0)
-      mbar_expect_tx(&BAR[s], w == 0 ? 8 * 2048 + 8 * 512 : 4 * 512 + 4 * 256 + 4 * 64 + (rec ? kPenRec * 4 : 0));
+      mbar_expect_tx(&BAR[s], w == 0 ? 4 * 2048 + 8 * 512 : 4 * 512 + 4 * 256 + 4 * 64 + (rec ? kPenRec * 4 : 0));
     __syncwarp();
     const int kz = id * 8 + 4 * half;
     if (w == 0) {
@@ -173,9 +170,6 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
         const bool xf = l < 8, lowside = ((l - 4) & 2) == 0;  // W / S boxes sit at the high face
         tma_load_3d(D + XW + 64 * (l - 4), xf ? &mp.xwe : &mp.xsn, xf && lowside ? 6 : 0,
                     !xf && lowside ? 6 : 0, kz, &BAR[s]);
-      } else if (l < 16) {  // b of the own bricks (lanes 12-15 hold ids 0-3 too: see bid)
-        tma_load_1d_hint(D + BOWN + OWN_STRIDE * (l - 12), p.b + (int64_t)bid * 512 + 256 * half, 2048, &BAR[s],
-                         pol_keep);
       }
     } else {
       if (l < 4) {
@@ -203,16 +197,24 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
   // ---- registers: x0 planes g-1, g, g+1; x1 planes g-2, g-1, g; b of planes g-1 .. g+2 ----
   // rings indexed by plane mod 4 (= the step's kk, a compile-time constant: no register moves
   // between steps): x0 (planes g-1..g+1), x1 (g-2..g), b (g-1, g), the ring cell's x0 (g-1..g+1)
-  double2 XR[4][2], YR[4][2], BR[4][2];
+  // b of the own cells: plane-mod-8 ring of 128-bit loads issued four planes ahead (slot of plane
+  // g = g mod 8 = 4 (c mod 2) + kk; a run has an even number of chunks and starts at an even c,
+  // so c's parity is known from the chunk's type and half: compile-time slots)
+  double2 XR[4][2], YR[4][2], BR[8][2];
   double RR[4] = {0.0, 0.0, 0.0, 0.0}, rpart = 0.0;
 #pragma unroll
   for (int r = 0; r < 2; ++r) {
 #pragma unroll
-    for (int s = 0; s < 4; ++s) XR[s][r] = YR[s][r] = BR[s][r] = make_double2(0.0, 0.0);
+    for (int s = 0; s < 4; ++s) XR[s][r] = YR[s][r] = BR[s][r] = BR[s + 4][r] = make_double2(0.0, 0.0);
   }
   // one step: sweep 1 on plane g = 4c + kk, sweep 2 on plane g - 1 (if it is a range plane)
-  auto step = [&](const int c, auto kkc, const bool start, const bool sw2, const bool pref) {
-    constexpr int kk = decltype(kkc)::value;
+  auto load_b = [&](double2* dst, int id, int code, int kk) {  // rows jb, jb+1 (always a valid brick)
+    const double* bp = p.b + (int64_t)id * 512 + 64 * (4 * (code & 1) + kk) + 8 * jb + ib;
+    dst[0] = ld_hint2(bp, pol_keep);  // the neighbour tiles' b-face copies reuse these lines from L2
+    dst[1] = ld_hint2(bp + 8, pol_keep);
+  };
+  auto step = [&](const int c, auto kkc, auto parc, const bool start, const bool sw2) {
+    constexpr int kk = decltype(kkc)::value, par = decltype(parc)::value;  // par = c mod 2
     const double* S0 = ST + (c % PN_ST) * STAGE;
     if (kk == 3) wait_upto(c + 1);
     const double* S1 = kk == 3 ? ST + ((c + 1) % PN_ST) * STAGE : S0;  // stage of plane g+1
@@ -224,20 +226,26 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     double2(&Ym)[2] = YR[km2];
     double2(&Yc)[2] = YR[km1];
     double2(&Y)[2] = YR[kk];
-    double2(&Bm)[2] = BR[km1];
-    double2(&Bc)[2] = BR[kk];
+    constexpr int bc = 4 * par + kk, bm = kk > 0 ? bc - 1 : 4 * (par ^ 1) + 3, bn = 4 * (par ^ 1) + kk;
+    double2(&Bm)[2] = BR[bm];  // b of plane g-1
+    double2(&Bc)[2] = BR[bc];  // b of plane g
     double& rcm = RR[km1];
     double& rc = RR[kk];
     double& rcp = RR[kp];
     const int codeC = mr(c, 0), idC = mr(c, 1 + q);
+    const int codeN = mr(c + 1, 0), idN = mr(c + 1, 1 + q);  // record c+1 came with chunk c
     if (start) {  // first step of a run (warm-up plane 7): prime the register windows
       Xm[0] = lds_d2(S0 + oO + 64 * (kk - 1)), Xm[1] = lds_d2(S0 + oO + 8 + 64 * (kk - 1));
       Xc[0] = lds_d2(S0 + oO + 64 * kk), Xc[1] = lds_d2(S0 + oO + 8 + 64 * kk);
       rcm = S0[oc + 16 * (kk - 1)];
       rc = S0[oc + 16 * kk];
+      // b of this plane and of the next chunk's planes 0-2 (plane 3 follows below)
+      load_b(BR[bc], idC, codeC, kk);
+#pragma unroll
+      for (int k2 = 0; k2 < 3; ++k2) load_b(BR[4 * (par ^ 1) + k2], idN, codeN, k2);
     }
-    (void)pref;
-    (void)idC;
+    // b of plane g+4 (the next chunk's plane kk; harmless where that plane is not swept)
+    load_b(BR[bn], idN, codeN, kk);
     const int kz1 = 4 * (codeC & 1) + kk;  // in-brick plane of g (red-black colour)
 
     // ---------------- sweep 1, own cells, plane g ----------------
@@ -250,7 +258,6 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
       const double wl0 = __shfl_up_sync(FULL, Xc[0].y, 1), er0 = __shfl_down_sync(FULL, Xc[0].x, 1);
       const double wl1 = __shfl_up_sync(FULL, Xc[1].y, 1), er1 = __shfl_down_sync(FULL, Xc[1].x, 1);
       const double W0 = edW ? e0 : wl0, E0 = edE ? e0 : er0, W1 = edW ? e1 : wl1, E1 = edE ? e1 : er1;
-      Bc[0] = lds_d2(S0 + BOWN + oO + 64 * kk), Bc[1] = lds_d2(S0 + BOWN + oO + 8 + 64 * kk);
       const double2 bb0 = Bc[0], bb1 = Bc[1];
       const double a00 = stencil_a(Xc[0].x, W0, Xc[0].y, xs.x, Xc[1].x, Xm[0].x, Xp[0].x, alpha, beta);
       const double a10 = stencil_a(Xc[0].y, Xc[0].x, E0, xs.y, Xc[1].y, Xm[0].y, Xp[0].y, alpha, beta);
@@ -288,7 +295,7 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
       const double wl1 = __shfl_up_sync(FULL, Yc[1].y, 1), er1 = __shfl_down_sync(FULL, Yc[1].x, 1);
       const double W0 = edW ? ed.x : wl0, E0 = edE ? ed.x : er0, W1 = edW ? ed.y : wl1, E1 = edE ? ed.y : er1;
       constexpr int km = (kk + 3) & 3;  // plane g-1 within its chunk
-      const double2 bb0 = Bm[0], bb1 = Bm[1];  // b of plane g-1 (its stage may be refilled by now)
+      const double2 bb0 = Bm[0], bb1 = Bm[1];
       const int code2 = kk > 0 ? codeC : mr(c + MRS - 1, 0), id2 = kk > 0 ? idC : mr(c + MRS - 1, 1 + q);
       const int kz2 = 4 * (code2 & 1) + km;
       const double a00 = stencil_a(Yc[0].x, W0, Yc[0].y, ys.x, Yc[1].x, Ym[0].x, Y[0].x, alpha, beta);
@@ -336,15 +343,22 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     using I1 = std::integral_constant<int, 1>;
     using I2 = std::integral_constant<int, 2>;
     using I3 = std::integral_constant<int, 3>;
+    using P0 = std::integral_constant<int, 0>;  // chunk parity: warm-up and half 1 even,
+    using P1 = std::integral_constant<int, 1>;  // half 0 and cool-down odd
     if (type == WARM) {
-      step(c, I3{}, true, false, true);
+      step(c, I3{}, P0{}, true, false);
+    } else if (type == RANGE && (mr(c, 0) & 1) == 0) {
+      step(c, I0{}, P1{}, false, typeP == RANGE);
+      step(c, I1{}, P1{}, false, true);
+      step(c, I2{}, P1{}, false, true);
+      step(c, I3{}, P1{}, false, true);
     } else if (type == RANGE) {
-      step(c, I0{}, false, typeP == RANGE, true);
-      step(c, I1{}, false, true, true);
-      step(c, I2{}, false, true, true);
-      step(c, I3{}, false, true, true);
+      step(c, I0{}, P0{}, false, true);
+      step(c, I1{}, P0{}, false, true);
+      step(c, I2{}, P0{}, false, true);
+      step(c, I3{}, P0{}, false, true);
     } else {
-      step(c, I0{}, false, true, false);
+      step(c, I0{}, P1{}, false, true);
     }
   }
 }
