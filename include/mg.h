@@ -121,7 +121,11 @@ typedef struct {
                                     h^2/6, colour (i+j+k) mod 2, r from the last (black) half-sweep (reading A20).
                                     The bottom stays damped Jacobi. */
   int32_t cheby_ratio;           /* smoothing interval mu in [mu_max/cheby_ratio, mu_max]; 0 => 6 */
-  int32_t reserved[3];
+  int32_t launch_pdl;            /* programmatic dependent launch of every library kernel: 0 = auto (on),
+                                    1 = on, 2 = off.  A kernel's CTAs may be scheduled while the previous
+                                    kernel of the stream drains; each waits for it before touching memory
+                                    (griddepcontrol), so results are bitwise unchanged */
+  int32_t reserved[2];
   double h0;                     /* finest spacing; <= 0 => 1 / max_d(global N_d) (reading A7) */
 } mg_params;
 

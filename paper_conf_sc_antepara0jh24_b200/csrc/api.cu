@@ -228,6 +228,7 @@ mg_status check_params(const mg_params& p) {
     return set_err(MG_ERR_INVALID_ARG, "pre_smooths must be >= 1 when num_levels > 1 (restriction reads its r)");
   if (p.transport < 0 || p.transport > MG_TRANSPORT_LOCAL) return set_err(MG_ERR_INVALID_ARG, "bad transport");
   if (p.bottom_mode < 0 || p.bottom_mode > MG_BOTTOM_CLUSTER) return set_err(MG_ERR_INVALID_ARG, "bad bottom_mode");
+  if (p.launch_pdl < 0 || p.launch_pdl > 2) return set_err(MG_ERR_INVALID_ARG, "launch_pdl must be 0, 1 or 2");
   if (p.smoother < 0 || p.smoother > 2)
     return set_err(MG_ERR_INVALID_ARG, "smoother must be 0 (Jacobi), 1 (Chebyshev) or 2 (red-black Gauss-Seidel)");
   return MG_OK;
@@ -479,6 +480,7 @@ mg_status check_ctx(mg_ctx* c) {
   if (!c) return set_err(MG_ERR_INVALID_ARG, "null context");
   if (c->poisoned) return set_err(MG_ERR_STATE, "context poisoned by an earlier CUDA/NCCL error");
   if (cudaSetDevice(c->device) != cudaSuccess) return set_err(MG_ERR_CUDA, "cudaSetDevice failed");
+  g_launch_pdl = c->lay.p.launch_pdl != 2;  // kernels enqueued or captured by this call
   return MG_OK;
 }
 

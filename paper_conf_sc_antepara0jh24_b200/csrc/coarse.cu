@@ -74,6 +74,7 @@ size_t coarse_smem_bytes(const CoarseArgs& a) {
 
 __global__ void __cluster_dims__(kCoarseCtas, 1, 1) __launch_bounds__(kCoarseThreads, 1)
     coarse_cluster_kernel(const __grid_constant__ CoarseArgs a) {
+  pdl_begin();
   cg::cluster_group cl = cg::this_cluster();
   const unsigned me = cl.block_rank();
   extern __shared__ __align__(16) double sm[];

@@ -26,6 +26,8 @@
 
 namespace mgb {
 
+bool g_launch_pdl = true;
+
 Coeffs level_coeffs(double h) {
   const double inv = 1.0 / (h * h);
   Coeffs c;
@@ -55,6 +57,7 @@ enum { MODE_SWEEP = 0, MODE_APPLY = 1, MODE_NORM = 2 };
 
 template <int MODE, unsigned FLAGS>
 __global__ void __launch_bounds__(256) sweep_kernel(SweepArgs p, unsigned long long* acc) {
+  pdl_begin();
   constexpr bool WRITE_R = (FLAGS & SW_WRITE_R) != 0;
   constexpr bool RESTRICT = (FLAGS & SW_RESTRICT) != 0;
   constexpr bool INTERP = (FLAGS & SW_INTERP) != 0;
@@ -193,7 +196,7 @@ __global__ void __launch_bounds__(256) sweep_kernel(SweepArgs p, unsigned long l
 template <unsigned FLAGS>
 static cudaError_t launch_sweep_t(const SweepArgs& a, cudaStream_t s) {
   if (a.nbricks <= 0) return cudaSuccess;
-  sweep_kernel<MODE_SWEEP, FLAGS><<<(unsigned)a.nbricks, 256, 0, s>>>(a, nullptr);
+  launch_k(sweep_kernel<MODE_SWEEP, FLAGS>, (unsigned)a.nbricks, 256, 0, s, a, nullptr);
   return cudaGetLastError();
 }
 
@@ -258,6 +261,7 @@ constexpr int COL_WARPS = 4;  // warp w streams planes 2w, 2w+1 of every brick
 template <unsigned FLAGS>
 __global__ void __launch_bounds__(COL_WARPS * 32, 6)
     sweep_col_kernel(SweepArgs p, ColArgs ca, const __grid_constant__ FaceMaps fm) {
+  pdl_wait();
   constexpr bool WRITE_R = (FLAGS & SW_WRITE_R) != 0;
   constexpr bool RESTRICT = (FLAGS & SW_RESTRICT) != 0;
   extern __shared__ __align__(128) unsigned char smem_raw[];
@@ -375,6 +379,7 @@ __global__ void __launch_bounds__(COL_WARPS * 32, 6)
       p.bc[(int64_t)(pr >> 3) * 512 + (4 * ox + I) + 8 * (4 * oy + J) + 64 * (4 * oz + K)] = v;
     }
   }
+  pdl_trigger();
 }
 
 bool col_supports(unsigned flags) {
@@ -388,9 +393,9 @@ cudaError_t launch_sweep_col(const SweepArgs& a, const ColArgs& c, const FaceMap
   const size_t sm = sizeof(ColSmem<false>), smr = sizeof(ColSmem<true>);
   const unsigned g = (unsigned)c.nseg, b = COL_WARPS * 32;
   switch (flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP | SW_ZERO_X)) {
-    case 0: sweep_col_kernel<0><<<g, b, sm, s>>>(a, c, fm); break;
-    case SW_WRITE_R: sweep_col_kernel<SW_WRITE_R><<<g, b, sm, s>>>(a, c, fm); break;
-    case SW_RESTRICT: sweep_col_kernel<SW_RESTRICT><<<g, b, smr, s>>>(a, c, fm); break;
+    case 0: launch_plain(sweep_col_kernel<0>, g, b, sm, s, a, c, fm); break;
+    case SW_WRITE_R: launch_plain(sweep_col_kernel<SW_WRITE_R>, g, b, sm, s, a, c, fm); break;
+    case SW_RESTRICT: launch_plain(sweep_col_kernel<SW_RESTRICT>, g, b, smr, s, a, c, fm); break;
     default: return cudaErrorInvalidValue;
   }
   return cudaGetLastError();
@@ -443,7 +448,7 @@ cudaError_t launch_apply_op(const double* x, double* Ax, const int32_t* adj, int
   a.brick0 = brick0;
   a.nbricks = nbricks;
   a.c = c;
-  sweep_kernel<MODE_APPLY, 0><<<(unsigned)nbricks, 256, 0, s>>>(a, nullptr);
+  launch_k(sweep_kernel<MODE_APPLY, 0>, (unsigned)nbricks, 256, 0, s, a, nullptr);
   return cudaGetLastError();
 }
 
@@ -457,7 +462,7 @@ cudaError_t launch_norm(const double* x, const double* b, const int32_t* adj, in
   a.brick0 = 0;
   a.nbricks = nbricks;
   a.c = c;
-  sweep_kernel<MODE_NORM, 0><<<(unsigned)nbricks, 256, 0, s>>>(a, acc);
+  launch_k(sweep_kernel<MODE_NORM, 0>, (unsigned)nbricks, 256, 0, s, a, acc);
   return cudaGetLastError();
 }
 
@@ -468,6 +473,7 @@ template <bool WRITE_R>
 __global__ void __launch_bounds__(256) smooth_kernel(double* __restrict__ x, const double* __restrict__ Ax,
                                                      const double* __restrict__ b, double* __restrict__ r,
                                                      int64_t base, int64_t n2, double gamma, int colour) {
+  pdl_begin();
   for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < n2; q += (int64_t)gridDim.x * blockDim.x) {
     const int64_t o = base + 2 * q;
     const double2 xv = ldg2(x + o);
@@ -497,9 +503,9 @@ cudaError_t launch_smooth(double* x, const double* Ax, const double* b, double* 
   if (nbricks <= 0) return cudaSuccess;
   const int64_t n2 = nbricks * 256;
   if (write_r)
-    smooth_kernel<true><<<grid_for(n2), 256, 0, s>>>(x, Ax, b, r, brick0 * 512, n2, c.gamma, colour);
+    launch_k(smooth_kernel<true>, grid_for(n2), 256, 0, s, x, Ax, b, r, brick0 * 512, n2, c.gamma, colour);
   else
-    smooth_kernel<false><<<grid_for(n2), 256, 0, s>>>(x, Ax, b, r, brick0 * 512, n2, c.gamma, colour);
+    launch_k(smooth_kernel<false>, grid_for(n2), 256, 0, s, x, Ax, b, r, brick0 * 512, n2, c.gamma, colour);
   return cudaGetLastError();
 }
 
@@ -509,6 +515,7 @@ cudaError_t launch_smooth(double* x, const double* Ax, const double* b, double* 
 // ---------------------------------------------------------------------------
 __global__ void __launch_bounds__(128) restrict_kernel(const double* __restrict__ r, double* __restrict__ bc,
                                                        const int32_t* __restrict__ parent) {
+  pdl_begin();
   __shared__ __align__(16) double rs[512];
   const int64_t f = blockIdx.x;
   const int t = threadIdx.x;
@@ -530,13 +537,14 @@ __global__ void __launch_bounds__(128) restrict_kernel(const double* __restrict_
 
 cudaError_t launch_restrict(const double* r, double* bc, const int32_t* parent, int64_t nfine, cudaStream_t s) {
   if (nfine <= 0) return cudaSuccess;
-  restrict_kernel<<<(unsigned)nfine, 128, 0, s>>>(r, bc, parent);
+  launch_k(restrict_kernel, (unsigned)nfine, 128, 0, s, r, bc, parent);
   return cudaGetLastError();
 }
 
 // interpolation+increment: one CTA (256 threads) per fine brick, 2 cells each.
 __global__ void __launch_bounds__(256) interp_kernel(double* __restrict__ x, const double* __restrict__ xc,
                                                      const int32_t* __restrict__ parent) {
+  pdl_begin();
   const int64_t f = blockIdx.x;
   const int t = threadIdx.x;
   const int i0 = 2 * (t & 3), j = (t >> 2) & 7, k = t >> 5;
@@ -551,11 +559,12 @@ __global__ void __launch_bounds__(256) interp_kernel(double* __restrict__ x, con
 
 cudaError_t launch_interp(double* x, const double* xc, const int32_t* parent, int64_t nfine, cudaStream_t s) {
   if (nfine <= 0) return cudaSuccess;
-  interp_kernel<<<(unsigned)nfine, 256, 0, s>>>(x, xc, parent);
+  launch_k(interp_kernel, (unsigned)nfine, 256, 0, s, x, xc, parent);
   return cudaGetLastError();
 }
 
 __global__ void __launch_bounds__(256) zero_kernel(double* __restrict__ x, int64_t base, int64_t n2) {
+  pdl_begin();
   for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < n2; q += (int64_t)gridDim.x * blockDim.x)
     reinterpret_cast<double2*>(x + base)[q] = make_double2(0.0, 0.0);
 }
@@ -563,7 +572,7 @@ __global__ void __launch_bounds__(256) zero_kernel(double* __restrict__ x, int64
 cudaError_t launch_zero(double* x, int64_t brick0, int64_t nbricks, cudaStream_t s) {
   if (nbricks <= 0) return cudaSuccess;
   const int64_t n2 = nbricks * 256;
-  zero_kernel<<<grid_for(n2), 256, 0, s>>>(x, brick0 * 512, n2);
+  launch_k(zero_kernel, grid_for(n2), 256, 0, s, x, brick0 * 512, n2);
   return cudaGetLastError();
 }
 
@@ -576,6 +585,7 @@ __global__ void __launch_bounds__(1024) bottom_resident_kernel(const double* __r
                                                                const double* __restrict__ b,
                                                                const int32_t* __restrict__ adj, int nbricks,
                                                                int sweeps, int zero_x, Coeffs c) {
+  pdl_begin();
   // A thread owns a k-column of 4 cells (i, j, k0..k0+3) of one brick: its x lives in registers,
   // the in-plane neighbours come from the shared copy of the previous sweep (ping-pong), the two
   // k-halos too; every neighbour offset is resolved through the adjacency table once, up front.
@@ -636,7 +646,7 @@ cudaError_t launch_bottom_resident(const double* x, double* xo, const double* b,
                                    int sweeps, bool zero_x, Coeffs c, cudaStream_t s) {
   if (nbricks <= 0 || nbricks > kResidentMaxBricks) return cudaErrorInvalidValue;
   const size_t smem = (size_t)nbricks * 512 * 2 * sizeof(double);
-  bottom_resident_kernel<<<1, 128 * nbricks, smem, s>>>(x, xo, b, adj, nbricks, sweeps, zero_x ? 1 : 0, c);
+  launch_k(bottom_resident_kernel, 1, 128 * nbricks, smem, s, x, xo, b, adj, nbricks, sweeps, zero_x ? 1 : 0, c);
   return cudaGetLastError();
 }
 
@@ -645,6 +655,7 @@ cudaError_t launch_bottom_resident(const double* x, double* xo, const double* b,
 // ---------------------------------------------------------------------------
 __global__ void __launch_bounds__(256) lex_to_brick_kernel(const double* __restrict__ lex, double* __restrict__ br,
                                                            const int32_t* __restrict__ coord, int nx, int ny) {
+  pdl_begin();
   const int64_t bI = blockIdx.x;
   const int t = threadIdx.x;
   const int i0 = 2 * (t & 3), j = (t >> 2) & 7, k = t >> 5;
@@ -655,6 +666,7 @@ __global__ void __launch_bounds__(256) lex_to_brick_kernel(const double* __restr
 
 __global__ void __launch_bounds__(256) brick_to_lex_kernel(const double* __restrict__ br, double* __restrict__ lex,
                                                            const int32_t* __restrict__ coord, int nx, int ny) {
+  pdl_begin();
   const int64_t bI = blockIdx.x;
   const int t = threadIdx.x;
   const int i0 = 2 * (t & 3), j = (t >> 2) & 7, k = t >> 5;
@@ -666,19 +678,20 @@ __global__ void __launch_bounds__(256) brick_to_lex_kernel(const double* __restr
 cudaError_t launch_lex_to_brick(const double* lex, double* bricks, const int32_t* coord, int64_t nowned, int nx,
                                 int ny, cudaStream_t s) {
   if (nowned <= 0) return cudaSuccess;
-  lex_to_brick_kernel<<<(unsigned)nowned, 256, 0, s>>>(lex, bricks, coord, nx, ny);
+  launch_k(lex_to_brick_kernel, (unsigned)nowned, 256, 0, s, lex, bricks, coord, nx, ny);
   return cudaGetLastError();
 }
 
 cudaError_t launch_brick_to_lex(const double* bricks, double* lex, const int32_t* coord, int64_t nowned, int nx,
                                 int ny, cudaStream_t s) {
   if (nowned <= 0) return cudaSuccess;
-  brick_to_lex_kernel<<<(unsigned)nowned, 256, 0, s>>>(bricks, lex, coord, nx, ny);
+  launch_k(brick_to_lex_kernel, (unsigned)nowned, 256, 0, s, bricks, lex, coord, nx, ny);
   return cudaGetLastError();
 }
 
 // blockIdx.y = run; the x-blocks stride over its 16-byte words
 __global__ void __launch_bounds__(256) copy_runs_kernel(const CopyRun* __restrict__ runs) {
+  pdl_begin();
   const CopyRun r = runs[blockIdx.y];
   const double2* src = reinterpret_cast<const double2*>(r.src);
   double2* dst = reinterpret_cast<double2*>(r.dst);
@@ -693,7 +706,7 @@ cudaError_t launch_copy_runs(const CopyRun* runs, int nruns, int64_t max_n, cuda
   const int64_t words = max_n / 2;
   const int64_t want = (int64_t)148 * 8 * 4 / nruns;
   const unsigned gx = (unsigned)std::max<int64_t>(1, std::min<int64_t>((words + 255) / 256, std::max<int64_t>(1, want)));
-  copy_runs_kernel<<<dim3(gx, (unsigned)nruns), 256, 0, s>>>(runs);
+  launch_k(copy_runs_kernel, dim3(gx, (unsigned)nruns), 256, 0, s, runs);
   return cudaGetLastError();
 }
 

@@ -163,4 +163,36 @@ cudaError_t launch_coarse(const CoarseArgs& a, cudaStream_t s);
 cudaError_t coarse_kernels_init();
 cudaError_t kernels_init();  // one-time attribute setup
 
+// Programmatic dependent launch for every kernel the library enqueues: set by the
+// API from mg_params.launch_pdl before it enqueues or captures work.  The kernels begin with
+// pdl_begin() (ptx.cuh), so the attribute only lets a kernel's CTAs be scheduled while the
+// previous kernel of the stream drains; results are unchanged.
+extern bool g_launch_pdl;
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_ex(bool pdl, void (*k)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s,
+                             Args... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = pdl ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, k, static_cast<KArgs>(args)...);
+}
+// short kernels: PDL attribute when enabled
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_k(void (*k)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s, Args... args) {
+  return launch_ex(g_launch_pdl, k, grid, block, smem, s, args...);
+}
+// persistent streaming kernels: never launched early (they still wait and trigger, see ptx.cuh)
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_plain(void (*k)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s,
+                                Args... args) {
+  return launch_ex(false, k, grid, block, smem, s, args...);
+}
+
 }  // namespace mgb

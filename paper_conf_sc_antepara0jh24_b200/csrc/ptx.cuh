@@ -27,6 +27,21 @@ __device__ __forceinline__ bool keep_cell(int colour, int i, int j, int k) {
   return colour >= 0 && ((i + j + k) & 1) != colour;
 }
 
+// Programmatic dependent launch (PDL).  Every kernel of the library waits (pdl_wait) until the
+// grids it depends on have completed and their writes are visible before it touches memory; the
+// wait is unconditional in every CTA, so completion stays transitive along the stream, and it is
+// a no-op for a kernel launched without the PDL attribute.  pdl_trigger lets the next kernel of
+// the stream start scheduling its CTAs (they park in their own pdl_wait): the short kernels of the
+// coarse levels trigger at once (pdl_begin); the persistent streaming kernels trigger after their
+// work loop and are themselves launched without the attribute, so their CTAs are placed on a
+// drained GPU (an early-launched persistent grid lands unevenly on the SMs: measured slower).
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+__device__ __forceinline__ void pdl_begin() {
+  pdl_wait();
+  pdl_trigger();
+}
+
 __device__ __forceinline__ double2 ldg2(const double* p) { return __ldg(reinterpret_cast<const double2*>(p)); }
 __device__ __forceinline__ double2 ld_stream2(const double* p) {
   double2 v;

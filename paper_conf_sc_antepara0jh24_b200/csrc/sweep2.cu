@@ -77,6 +77,7 @@ __device__ __forceinline__ double2 lds2(const double* p) { return *reinterpret_c
 template <unsigned FLAGS>
 __global__ void __launch_bounds__(P2_THREADS, kPairCtasPerSm)
     sweep2_kernel(SweepArgs p, PairArgs pa, const __grid_constant__ PairMaps mp) {
+  pdl_wait();
   constexpr bool WRITE_R = (FLAGS & SW_WRITE_R) != 0;
   constexpr bool RESTRICT = (FLAGS & SW_RESTRICT) != 0;
   constexpr bool COLOUR = (FLAGS & SW_COLOUR) != 0;  // red-black half-sweeps (GSRB variant)
@@ -342,6 +343,7 @@ __global__ void __launch_bounds__(P2_THREADS, kPairCtasPerSm)
     step(m, std::integral_constant<int, 0>{});
     if (m + 1 < cnt) step(m + 1, std::integral_constant<int, 1>{});
   }
+  pdl_trigger();
 }
 
 bool pair_supports(unsigned flags) {
@@ -356,12 +358,12 @@ cudaError_t launch_sweep2(const SweepArgs& a, const PairArgs& pa, const PairMaps
   const size_t sm = sizeof(P2Smem);
   const unsigned col = (a.colour >= 0 || a.colour2 >= 0) ? SW_COLOUR : 0u;
   switch ((flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP | SW_ZERO_X)) | col) {
-    case 0: sweep2_kernel<0><<<g, P2_THREADS, sm, s>>>(a, pa, pm); break;
-    case SW_WRITE_R: sweep2_kernel<SW_WRITE_R><<<g, P2_THREADS, sm, s>>>(a, pa, pm); break;
-    case SW_RESTRICT: sweep2_kernel<SW_RESTRICT><<<g, P2_THREADS, sm, s>>>(a, pa, pm); break;
-    case SW_COLOUR: sweep2_kernel<SW_COLOUR><<<g, P2_THREADS, sm, s>>>(a, pa, pm); break;
-    case SW_WRITE_R | SW_COLOUR: sweep2_kernel<SW_WRITE_R | SW_COLOUR><<<g, P2_THREADS, sm, s>>>(a, pa, pm); break;
-    case SW_RESTRICT | SW_COLOUR: sweep2_kernel<SW_RESTRICT | SW_COLOUR><<<g, P2_THREADS, sm, s>>>(a, pa, pm); break;
+    case 0: launch_plain(sweep2_kernel<0>, g, P2_THREADS, sm, s, a, pa, pm); break;
+    case SW_WRITE_R: launch_plain(sweep2_kernel<SW_WRITE_R>, g, P2_THREADS, sm, s, a, pa, pm); break;
+    case SW_RESTRICT: launch_plain(sweep2_kernel<SW_RESTRICT>, g, P2_THREADS, sm, s, a, pa, pm); break;
+    case SW_COLOUR: launch_plain(sweep2_kernel<SW_COLOUR>, g, P2_THREADS, sm, s, a, pa, pm); break;
+    case SW_WRITE_R | SW_COLOUR: launch_plain(sweep2_kernel<SW_WRITE_R | SW_COLOUR>, g, P2_THREADS, sm, s, a, pa, pm); break;
+    case SW_RESTRICT | SW_COLOUR: launch_plain(sweep2_kernel<SW_RESTRICT | SW_COLOUR>, g, P2_THREADS, sm, s, a, pa, pm); break;
     default: return cudaErrorInvalidValue;
   }
   return cudaGetLastError();

@@ -67,6 +67,7 @@ constexpr size_t SMEM_BYTES = (size_t)(PN_ST * STAGE + 2 * PUB + 2 * RWE_PAR) * 
 template <unsigned FLAGS>
 __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     sweep2p_kernel(SweepArgs p, PairArgs pa, const __grid_constant__ PairMaps mp) {
+  pdl_wait();
   constexpr bool WRITE_R = (FLAGS & SW_WRITE_R) != 0;
   constexpr bool RESTRICT = (FLAGS & SW_RESTRICT) != 0;
   constexpr bool COLOUR = (FLAGS & SW_COLOUR) != 0;  // red-black half-sweeps (GSRB variant)
@@ -361,6 +362,7 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
       step(c, I0{}, P1{}, false, true);
     }
   }
+  pdl_trigger();
 }
 
 bool pencil_supports(unsigned flags) {
@@ -385,13 +387,13 @@ cudaError_t launch_sweep2p(const SweepArgs& a, const PairArgs& pa, const PairMap
   const size_t sm = SMEM_BYTES;
   const unsigned col = (a.colour >= 0 || a.colour2 >= 0) ? SW_COLOUR : 0u;
   switch ((flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP | SW_ZERO_X)) | col) {
-    case 0: sweep2p_kernel<0><<<g, PN_THREADS, sm, s>>>(a, pa, pm); break;
-    case SW_WRITE_R: sweep2p_kernel<SW_WRITE_R><<<g, PN_THREADS, sm, s>>>(a, pa, pm); break;
-    case SW_RESTRICT: sweep2p_kernel<SW_RESTRICT><<<g, PN_THREADS, sm, s>>>(a, pa, pm); break;
-    case SW_COLOUR: sweep2p_kernel<SW_COLOUR><<<g, PN_THREADS, sm, s>>>(a, pa, pm); break;
-    case SW_WRITE_R | SW_COLOUR: sweep2p_kernel<SW_WRITE_R | SW_COLOUR><<<g, PN_THREADS, sm, s>>>(a, pa, pm); break;
+    case 0: launch_plain(sweep2p_kernel<0>, g, PN_THREADS, sm, s, a, pa, pm); break;
+    case SW_WRITE_R: launch_plain(sweep2p_kernel<SW_WRITE_R>, g, PN_THREADS, sm, s, a, pa, pm); break;
+    case SW_RESTRICT: launch_plain(sweep2p_kernel<SW_RESTRICT>, g, PN_THREADS, sm, s, a, pa, pm); break;
+    case SW_COLOUR: launch_plain(sweep2p_kernel<SW_COLOUR>, g, PN_THREADS, sm, s, a, pa, pm); break;
+    case SW_WRITE_R | SW_COLOUR: launch_plain(sweep2p_kernel<SW_WRITE_R | SW_COLOUR>, g, PN_THREADS, sm, s, a, pa, pm); break;
     case SW_RESTRICT | SW_COLOUR:
-      sweep2p_kernel<SW_RESTRICT | SW_COLOUR><<<g, PN_THREADS, sm, s>>>(a, pa, pm);
+      launch_plain(sweep2p_kernel<SW_RESTRICT | SW_COLOUR>, g, PN_THREADS, sm, s, a, pa, pm);
       break;
     default: return cudaErrorInvalidValue;
   }

@@ -104,6 +104,7 @@ __device__ __forceinline__ double face_x1(double c, double o, double own, double
 template <unsigned FLAGS>
 __global__ void __launch_bounds__(32 * kW2WarpsPerSm, 1)
     sweep2w_kernel(SweepArgs p, PairArgs pa, const __grid_constant__ PairMaps mp) {
+  pdl_wait();
   constexpr bool WRITE_R = (FLAGS & SW_WRITE_R) != 0;
   constexpr bool RESTRICT = (FLAGS & SW_RESTRICT) != 0;
   constexpr unsigned FULL = 0xffffffffu;
@@ -379,6 +380,7 @@ __global__ void __launch_bounds__(32 * kW2WarpsPerSm, 1)
     if (s + 1 < nsteps) step(std::integral_constant<int, 1>{});
     if (s + 2 < nsteps) step(std::integral_constant<int, 2>{});
   }
+  pdl_trigger();
 }
 
 cudaError_t launch_sweep2w(const SweepArgs& a, const PairArgs& pa, const PairMaps& pm, unsigned flags,
@@ -388,9 +390,9 @@ cudaError_t launch_sweep2w(const SweepArgs& a, const PairArgs& pa, const PairMap
   const size_t sm = sizeof(W2Smem) * kW2WarpsPerSm;
   constexpr unsigned kThreads = 32 * kW2WarpsPerSm;
   switch (flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP | SW_ZERO_X)) {
-    case 0: sweep2w_kernel<0><<<g, kThreads, sm, s>>>(a, pa, pm); break;
-    case SW_WRITE_R: sweep2w_kernel<SW_WRITE_R><<<g, kThreads, sm, s>>>(a, pa, pm); break;
-    case SW_RESTRICT: sweep2w_kernel<SW_RESTRICT><<<g, kThreads, sm, s>>>(a, pa, pm); break;
+    case 0: launch_plain(sweep2w_kernel<0>, g, kThreads, sm, s, a, pa, pm); break;
+    case SW_WRITE_R: launch_plain(sweep2w_kernel<SW_WRITE_R>, g, kThreads, sm, s, a, pa, pm); break;
+    case SW_RESTRICT: launch_plain(sweep2w_kernel<SW_RESTRICT>, g, kThreads, sm, s, a, pa, pm); break;
     default: return cudaErrorInvalidValue;
   }
   return cudaGetLastError();
