@@ -52,15 +52,21 @@ constexpr int BW = 1568, BE = 1696;                        // 2 boxes of 64: b o
 constexpr int BS = 1824, BN = 1888;                        // 2 boxes of 32: b of the S / N bricks
 constexpr int COR = 1952;                                  // 4 boxes of 8 (16 apart): SW, NW, SE, NE
 constexpr int STAGE = 2016;
-constexpr int PUB = 18 * 16;  // x1 of tile rows -1..16 (rows -1 / 16: the S / N ring)
+// x1 buffers (offsets from XP, in doubles): per parity p, tile rows -1..15 at PUB p (row -1: the S ring);
+// the N ring rows (tile row 16) at NROW + 16 p, 64 B off the S rows modulo 128, so the S and N ring
+// stores of one brick column (one half-warp) fall in complementary banks; the W / E ring columns at
+// RWE_OFF (W rows 0-15 at 16 p, E rows at RWE_E + 16 p: the W and E ring stores of a half-warp and
+// the edge lanes' 128-bit loads of a quarter-warp are conflict-free)
+constexpr int PUB = 17 * 16;
+constexpr int NROW = 2 * PUB + 8;
+constexpr int RWE_OFF = NROW + 32, RWE_E = 40, RWE_PAR = 16;
+constexpr int XP_SIZE = RWE_OFF + RWE_E + 2 * RWE_PAR;  // 656
 static_assert(STAGE * 8 % 128 == 0 && XW * 8 % 128 == 0 && BS * 8 % 128 == 0 && COR * 8 % 128 == 0, "align");
 static_assert(3 * OWN_STRIDE + 256 <= XW, "own bricks fit");
 __device__ __forceinline__ double2 lds_d2(const double* p) { return *reinterpret_cast<const double2*>(p); }
 constexpr int MRS = 4;  // chunk record ring slots (record n in slot n % 4)
-// ring x1 columns per parity: W rows 0-15 at 0, E rows at 18 (the two columns' rows sit in
-// different banks, so the edge lanes' 128-bit loads of a quarter-warp do not conflict)
-constexpr int RWE_E = 18, RWE_PAR = 36;
-constexpr size_t SMEM_BYTES = (size_t)(PN_ST * STAGE + 2 * PUB + 2 * RWE_PAR) * 8 + 16 + MRS * kPenRec * 4;
+constexpr size_t SMEM_BYTES = (size_t)(PN_ST * STAGE + XP_SIZE) * 8 + 16 + MRS * kPenRec * 4;
+static_assert(SMEM_BYTES + 1024 <= 233472 / PN_MINB, "PN_MINB CTAs per SM must fit in shared memory");
 
 }  // namespace
 
@@ -75,9 +81,9 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
   constexpr int RANGE = 0, WARM = 1, COOL = 2;
   extern __shared__ __align__(128) unsigned char smem_raw[];
   double* const ST = reinterpret_cast<double*>(smem_raw);  // [PN_ST][STAGE]
-  double* const XP = ST + PN_ST * STAGE;                    // [2][PUB]  x1 of tile rows -1..16
-  double* const RWE = XP + 2 * PUB;                         // [2][RWE_PAR] x1 of the W / E ring columns
-  uint64_t* const BAR = reinterpret_cast<uint64_t*>(RWE + 2 * RWE_PAR);
+  double* const XP = ST + PN_ST * STAGE;                    // x1 of tile rows -1..16 (layout above)
+  double* const RWE = XP + RWE_OFF;                         // x1 of the W / E ring columns
+  uint64_t* const BAR = reinterpret_cast<uint64_t*>(XP + XP_SIZE);
   int* const MR = reinterpret_cast<int*>(BAR + 2);  // [MRS][kPenRec] chunk records, 16-byte aligned slots
   const int col1 = COLOUR ? p.colour : -1, col2 = COLOUR ? p.colour2 : -1;
   const int t = threadIdx.x, w = t >> 5, l = t & 31;
@@ -102,6 +108,8 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
   const int oEd = edE ? XE + 64 * w + 2 * jb : XW + 64 * w + 2 * jb + 1;  // tile-edge W / E x0 (rows jb, jb+1: +2)
   const int R0 = 8 * w + jb;                                              // tile row of my row 0
   const int pO = (R0 + 1) * 16 + 2 * pc;                                  // my row 0 in the x1 buffer
+  const bool nrow = R0 + 2 == 16;                                         // row R0 + 2 is the N ring row
+  const int pN = nrow ? NROW + 2 * pc : pO + 32, sPN = nrow ? RWE_PAR : PUB;  // its offset, parity stride
   const int oRwe = (edE ? RWE_E : 0) + R0;                                // ring x1 column, rows R0, R0+1
 
   // ---- ring role: x1 of one cell of the 1-cell ring around the tile ----
@@ -119,11 +127,12 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     else if (w == 0) ohi = X + 64 + cc, shi = 16;
     else ohi = COR + (side ? 48 : 16) + cc, shi = 2;  // NW / NE corner
     ob = (side ? BE : BW) + 64 * w + 2 * j + cc, sb = 16;
-    oout = 2 * PUB + RWE_E * side + 8 * w + j, rstr = RWE_PAR;  // RWE[par][side col + row] (RWE = XP + 2 PUB)
+    oout = RWE_OFF + RWE_E * side + 8 * w + j, rstr = RWE_PAR;  // RWE[side col + row] + 16 par
     rci = side ? 0 : 7, rcj = j;
-  } else {  // S (warp 0) / N (warp 1) row, tile column i
-    const int i = l - 16, i8 = i & 7, bxr = i >> 3;
-    const bool S = w == 0;
+  } else {  // S (lanes 16-23) / N (24-31) ring rows over brick column bxr = w (tile columns 8w + i8):
+            // the S and N slab rows of one brick column sit in complementary banks
+    const int i8 = l & 7, bxr = w, i = 8 * w + i8;
+    const bool S = l < 24;
     const int X = S ? XS : XN, rowc = S ? 8 : 0, rowo = S ? 0 : 8;
     oc = X + 64 * bxr + rowc + i8;
     oo = X + 64 * bxr + rowo + i8;
@@ -133,7 +142,7 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     if (i < 15) ohi = X + 64 * ((i + 1) >> 3) + rowc + ((i + 1) & 7), shi = 16;
     else ohi = COR + (S ? 32 : 48), shi = 2;  // SE / NE corner (i = 0)
     ob = (S ? BS : BN) + 32 * bxr + i8, sb = 8;
-    oout = (S ? 0 : 17 * 16) + i, rstr = PUB;  // XP[par][row -1 / 16][i]
+    oout = S ? i : NROW + i, rstr = S ? PUB : RWE_PAR;  // row -1 / 16, column i
     rci = i8, rcj = S ? 7 : 0;
   }
 
@@ -214,6 +223,9 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     dst[0] = ld_hint2(bp, pol_keep);  // the neighbour tiles' b-face copies reuse these lines from L2
     dst[1] = ld_hint2(bp + 8, pol_keep);
   };
+  // this chunk's records, read from the record ring once per chunk (the step reads registers):
+  // code / own brick id of chunk c, c + 1 and c - 1 (plane g - 1 of step kk = 0), parent of c and c - 1
+  int codeC = 0, idC = 0, codeN = 0, idN = 0, codeP = 0, idP = 0, parC = 0, parP = 0;
   auto step = [&](const int c, auto kkc, auto parc, const bool start, const bool sw2) {
     constexpr int kk = decltype(kkc)::value, par = decltype(parc)::value;  // par = c mod 2
     const double* S0 = ST + (c % PN_ST) * STAGE;
@@ -233,8 +245,6 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     double& rcm = RR[km1];
     double& rc = RR[kk];
     double& rcp = RR[kp];
-    const int codeC = mr(c, 0), idC = mr(c, 1 + q);
-    const int codeN = mr(c + 1, 0), idN = mr(c + 1, 1 + q);  // record c+1 came with chunk c
     if (start) {  // first step of a run (warm-up plane 7): prime the register windows
       Xm[0] = lds_d2(S0 + oO + 64 * (kk - 1)), Xm[1] = lds_d2(S0 + oO + 8 + 64 * (kk - 1));
       Xc[0] = lds_d2(S0 + oO + 64 * kk), Xc[1] = lds_d2(S0 + oO + 8 + 64 * kk);
@@ -290,14 +300,14 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     {
       constexpr int par = (kk + 1) & 1;  // parity of plane g - 1
       const double* P = XP + par * PUB;
-      const double2 ys = lds_d2(P + pO - 16), yn = lds_d2(P + pO + 32);
+      const double2 ys = lds_d2(P + pO - 16), yn = lds_d2(XP + pN + sPN * par);
       const double2 ed = lds_d2(RWE + RWE_PAR * par + oRwe);
       const double wl0 = __shfl_up_sync(FULL, Yc[0].y, 1), er0 = __shfl_down_sync(FULL, Yc[0].x, 1);
       const double wl1 = __shfl_up_sync(FULL, Yc[1].y, 1), er1 = __shfl_down_sync(FULL, Yc[1].x, 1);
       const double W0 = edW ? ed.x : wl0, E0 = edE ? ed.x : er0, W1 = edW ? ed.y : wl1, E1 = edE ? ed.y : er1;
       constexpr int km = (kk + 3) & 3;  // plane g-1 within its chunk
       const double2 bb0 = Bm[0], bb1 = Bm[1];
-      const int code2 = kk > 0 ? codeC : mr(c + MRS - 1, 0), id2 = kk > 0 ? idC : mr(c + MRS - 1, 1 + q);
+      const int code2 = kk > 0 ? codeC : codeP, id2 = kk > 0 ? idC : idP;
       const int kz2 = 4 * (code2 & 1) + km;
       const double a00 = stencil_a(Yc[0].x, W0, Yc[0].y, ys.x, Yc[1].x, Ym[0].x, Y[0].x, alpha, beta);
       const double a10 = stencil_a(Yc[0].y, Yc[0].x, E0, ys.y, Yc[1].y, Ym[0].y, Y[0].y, alpha, beta);
@@ -325,7 +335,7 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
         if ((km & 1) == 0) {
           rpart = s;
         } else if (sw2) {
-          const int pr = mr(kk > 0 ? c : c + MRS - 1, 17);
+          const int pr = kk > 0 ? parC : parP;
           const int K = 4 * ((pr >> 2) & 1) + (kz2 >> 1);
           p.bc[(int64_t)(pr >> 3) * 512 + pc + 8 * (4 * w + jp) + 64 * K] = DMUL(0.125, DADD(rpart, s));
         }
@@ -339,7 +349,11 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     // chunk c (and with it record c+1) before issuing chunk c+1 into the stage chunk c-1 used
     if (c > 0) wait_upto(c);
     while (issued < cnt && issued <= c + PN_ST - 1) issue();
-    const int type = (mr(c, 0) >> 1) & 3, typeP = c > 0 ? (mr(c + MRS - 1, 0) >> 1) & 3 : WARM;
+    codeP = codeC, idP = idC, parP = parC;
+    codeC = mr(c, 0), idC = mr(c, 1 + q);
+    codeN = mr(c + 1, 0), idN = mr(c + 1, 1 + q);  // record c+1 came with chunk c
+    if (RESTRICT) parC = mr(c, 17);
+    const int type = (codeC >> 1) & 3, typeP = c > 0 ? (codeP >> 1) & 3 : WARM;
     using I0 = std::integral_constant<int, 0>;
     using I1 = std::integral_constant<int, 1>;
     using I2 = std::integral_constant<int, 2>;
@@ -348,7 +362,7 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     using P1 = std::integral_constant<int, 1>;  // half 0 and cool-down odd
     if (type == WARM) {
       step(c, I3{}, P0{}, true, false);
-    } else if (type == RANGE && (mr(c, 0) & 1) == 0) {
+    } else if (type == RANGE && (codeC & 1) == 0) {
       step(c, I0{}, P1{}, false, typeP == RANGE);
       step(c, I1{}, P1{}, false, true);
       step(c, I2{}, P1{}, false, true);

@@ -8,7 +8,7 @@ if [ -z "$NOTEST" ]; then
   timeout 1200 python -m pytest tests -m gpu -q -x ${PYTEST_K:+-k "$PYTEST_K"} > gpurun_out/pt_ab.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pt_ab.log
   tail -3 gpurun_out/pt_ab.log
 fi
-IFS=';' read -ra SETS <<< "${AB:-}"
+IFS=";" read -ra SETS <<< "${AB:-}"; [ ${#SETS[@]} -eq 0 ] && SETS=("")
 i=0
 for rep in ${REPS:-1 2}; do
 for args in "${SETS[@]}"; do
