@@ -490,6 +490,22 @@ def test_temporal_blocking_on_off_bitwise(oracle_mod, tb):
     m.close()
 
 
+@pytest.mark.parametrize("launch_pdl", [1, 2])
+@pytest.mark.parametrize("use_graph", [True, False])
+def test_programmatic_dependent_launch_on_off_bitwise(oracle_mod, launch_pdl, use_graph):
+    """Programmatic dependent launch on (1) and off (2), captured in the V-cycle graph or launched
+    op by op, gives the oracle's bits: 128^3, L = 5 (pencil passes on levels 0-1, one-brick kernels,
+    the resident bottom), 12/12/100, two cycles."""
+    shape = (128, 128, 128)
+    b = mg_inputs.random_rhs(shape, 29)
+    xs, ns = oracle_cycles(oracle_mod, b, 5, 2)
+    m = new(shape, 5, launch_pdl=launch_pdl, use_graph=use_graph)
+    m.set_rhs(dev(b))
+    m.set_solution(None)
+    check_cycles(m, xs, ns)
+    m.close()
+
+
 # ------------------------------------------------- Chebyshev smoother variant (N4, reading A19)
 @pytest.mark.parametrize("kw", [dict(), dict(temporal_blocking=0), dict(fusion=1), dict(temporal_blocking=2),
                                 dict(bottom_mode=1), dict(bottom_mode=3), dict(ghost_mode=1, ca_period=4),
