@@ -56,6 +56,8 @@ def parse():
                     help="0 damped Jacobi (the paper), 1 Chebyshev, 2 red-black Gauss-Seidel (N4 variants)")
     ap.add_argument("--cheby-ratio", type=int, default=0, help="Chebyshev smoothing interval [mu_max/ratio, mu_max]")
     ap.add_argument("--no-pdl", action="store_true", help="launch kernels without programmatic dependent launch")
+    ap.add_argument("--bottom-mode", type=int, default=0,
+                    help="0 auto, 1 per-sweep launches, 2 resident bottom, 3 cluster coarse solve, 4 grid coarse solve")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--ref-n", type=int, default=0, help="reference arm: grid side of the bounded sample")
@@ -246,7 +248,8 @@ def main():
     m = Multigrid((n, n, n), pg, a.levels, a.pre, a.post, a.bottom, ca_period=a.ca_period, fusion=a.fusion,
                   ghost_mode=1 if a.ghost_all else 0, use_graph=not a.no_graph, overlap=not a.no_overlap,
                   rank=rank, world_size=world, device=local, temporal_blocking=a.tb, smoother=a.smoother,
-                  cheby_ratio=a.cheby_ratio, launch_pdl=2 if a.no_pdl else 0)
+                  cheby_ratio=a.cheby_ratio, launch_pdl=2 if a.no_pdl else 0,
+                  bottom_mode=a.bottom_mode)
     gshape = (n * pg[2], n * pg[1], n * pg[0])
     b_host = torch.from_numpy(mg_inputs.local_sin_rhs(gshape, rank, pg)).pin_memory()
     b_dev = b_host.to(dev)
@@ -364,6 +367,8 @@ def main():
                        "fusion": "auto(full)" if not a.fusion else a.fusion,
                        "ca_period": a.ca_period or "auto(8)", "ghost_mode": "all" if a.ghost_all else "auto",
                        "cuda_graph": not a.no_graph, "overlap": not a.no_overlap, "pdl": not a.no_pdl,
+                       "coarse": {0: "auto", 1: "per-sweep launches", 2: "resident bottom", 3: "cluster solve",
+                                  4: "grid solve"}[a.bottom_mode],
                        "temporal_blocking": {0: "off", 1: "one-brick CTA streams", 2: "warp plane streams"}.get(
                            a.tb, "2x2-brick pencils"),
                        "smoother": {1: "chebyshev", 2: "red-black gauss-seidel"}.get(a.smoother, "damped jacobi (paper)"),

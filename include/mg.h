@@ -92,7 +92,7 @@ enum { MG_TRANSPORT_AUTO = 0, MG_TRANSPORT_NCCL = 1, MG_TRANSPORT_LOCAL = 2 };
  * 8-CTA cluster launch (coarse.cu: pre-sweeps, restriction, initZero, bottom, interpolation,
  * post-sweeps of those levels); measured no faster than graph-replayed launches (DESIGN.md
  * §7.3).  All modes are bitwise identical. */
-enum { MG_BOTTOM_AUTO = 0, MG_BOTTOM_SWEEPS = 1, MG_BOTTOM_RESIDENT = 2, MG_BOTTOM_CLUSTER = 3 };
+enum { MG_BOTTOM_AUTO = 0, MG_BOTTOM_SWEEPS = 1, MG_BOTTOM_RESIDENT = 2, MG_BOTTOM_CLUSTER = 3, MG_BOTTOM_GRID = 4 };
 
 typedef struct {
   int32_t n_local[3];            /* cells per rank per axis (x,y,z); each divisible by 8*2^(num_levels-1) */
@@ -108,7 +108,9 @@ typedef struct {
                                     self-exchange is needed and an NCCL id is given, else local */
   int32_t use_graph;             /* 1 = replay the V-cycle as one CUDA graph (default 1) */
   int32_t bottom_mode;           /* MG_BOTTOM_* (resident = one CTA runs all bottom sweeps in smem,
-                                    cluster = the coarse levels run in one cluster launch) */
+                                    cluster = the coarse levels run in one cluster launch, grid = the
+                                    ghost-free levels of <= 512 bricks run in one launch of one CTA per
+                                    SM with grid barriers between dependent steps) */
   int32_t overlap;               /* 1 = sweep interior bricks while the exchange is in flight */
   int32_t sweep_kernel;          /* 0 = auto (streaming column kernel on levels >= 16384 bricks),
                                     1 = one-brick-per-CTA kernel only, 2 = streaming kernel on every level */

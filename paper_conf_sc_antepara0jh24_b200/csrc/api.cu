@@ -204,7 +204,8 @@ size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double**
     double* st = (double*)take((size_t)lay.lv[0].n_owned * kBV * sizeof(double));
     if (stage) stage[k] = st;
   }
-  unsigned long long* ac = (unsigned long long*)take(256);
+  // norm accumulator (word 0) and the grid coarse solve's barrier words (from byte 64, kGridBarWords)
+  unsigned long long* ac = (unsigned long long*)take(64 + kGridBarWords * sizeof(unsigned));
   if (acc) *acc = ac;
   return align256(off);
 }
@@ -227,7 +228,7 @@ mg_status check_params(const mg_params& p) {
   if (p.num_levels > 1 && p.pre_smooths < 1)
     return set_err(MG_ERR_INVALID_ARG, "pre_smooths must be >= 1 when num_levels > 1 (restriction reads its r)");
   if (p.transport < 0 || p.transport > MG_TRANSPORT_LOCAL) return set_err(MG_ERR_INVALID_ARG, "bad transport");
-  if (p.bottom_mode < 0 || p.bottom_mode > MG_BOTTOM_CLUSTER) return set_err(MG_ERR_INVALID_ARG, "bad bottom_mode");
+  if (p.bottom_mode < 0 || p.bottom_mode > MG_BOTTOM_GRID) return set_err(MG_ERR_INVALID_ARG, "bad bottom_mode");
   if (p.launch_pdl < 0 || p.launch_pdl > 2) return set_err(MG_ERR_INVALID_ARG, "launch_pdl must be 0, 1 or 2");
   if (p.smoother < 0 || p.smoother > 2)
     return set_err(MG_ERR_INVALID_ARG, "smoother must be 0 (Jacobi), 1 (Chebyshev) or 2 (red-black Gauss-Seidel)");
@@ -413,6 +414,26 @@ mg_status exec_op(mg_ctx* c, const Op& o, cudaStream_t s) {
       CKS(timer_end(c, s, t0, o.level, o.timer));
       return MG_OK;
     case OP_COARSE: {
+      if (c->lay.p.bottom_mode == MG_BOTTOM_GRID) {
+        GridCoarseArgs a{};
+        a.nlev = c->lay.L - o.level;
+        for (int l = o.level; l < c->lay.L; ++l) {
+          const DevLevel& dl = c->dl[l];
+          a.lv[l - o.level] = {c->lay.lv[l].n_owned, dl.adj, dl.parent, {dl.x[0], dl.x[1]}, dl.b, dl.c, dl.h};
+        }
+        const mg_params& P = c->lay.p;
+        a.cheb = P.smoother == 1;
+        for (int k = 0; a.cheb && k < P.pre_smooths; ++k) a.nu_pre[k] = cheb_nu(P.pre_smooths, k, P.cheby_ratio);
+        for (int k = 0; a.cheb && k < P.post_smooths; ++k) a.nu_post[k] = cheb_nu(P.post_smooths, k, P.cheby_ratio);
+        a.pre = P.pre_smooths;
+        a.post = P.post_smooths;
+        a.bottom = P.bottom_smooths;
+        a.bar = reinterpret_cast<unsigned*>(c->acc + 8);  // zeroed at setup; consistent after every launch
+        CKS(timer_begin(c, s, &t0));
+        CKC(c, launch_coarse_grid(a, s));
+        CKS(timer_end(c, s, t0, o.level, o.timer));
+        return MG_OK;
+      }
       CoarseArgs a{};
       a.nlev = c->lay.L - o.level;
       for (int l = o.level; l < c->lay.L; ++l) {

@@ -23,6 +23,7 @@
 
 #include "kernels.h"
 #include "ptx.cuh"
+#include "resident.cuh"
 
 namespace mgb {
 
@@ -581,65 +582,14 @@ cudaError_t launch_zero(double* x, int64_t brick0, int64_t nbricks, cudaStream_t
 // ghosts, <= 8 bricks) in one CTA's shared memory; `sweeps` Jacobi sweeps with
 // a CTA barrier between sweeps instead of `sweeps` kernel launches.
 // ---------------------------------------------------------------------------
+
 __global__ void __launch_bounds__(1024) bottom_resident_kernel(const double* __restrict__ x, double* __restrict__ xo,
                                                                const double* __restrict__ b,
                                                                const int32_t* __restrict__ adj, int nbricks,
                                                                int sweeps, int zero_x, Coeffs c) {
   pdl_begin();
-  // A thread owns a k-column of 4 cells (i, j, k0..k0+3) of one brick: its x lives in registers,
-  // the in-plane neighbours come from the shared copy of the previous sweep (ping-pong), the two
-  // k-halos too; every neighbour offset is resolved through the adjacency table once, up front.
   extern __shared__ __align__(16) double sm[];
-  const int n = nbricks * 512;
-  double* xa = sm;
-  double* xb = sm + n;
-  const int t = threadIdx.x, br = t >> 7, q = t & 127;
-  const int i = q & 7, j = (q >> 3) & 7, k0 = 4 * (q >> 6);
-  const bool act = br < nbricks;
-  const int o = br * 512 + i + 8 * j + 64 * k0;  // my cell k0
-  int oW = 0, oE = 0, oS = 0, oN = 0, oB = 0, oT = 0;
-  double xv[4] = {0.0, 0.0, 0.0, 0.0}, bv[4] = {0.0, 0.0, 0.0, 0.0};
-  if (act) {
-    const int32_t* a = adj + br * 8;
-    oW = i > 0 ? o - 1 : a[0] * 512 + 7 + 8 * j + 64 * k0;
-    oE = i < 7 ? o + 1 : a[1] * 512 + 0 + 8 * j + 64 * k0;
-    oS = j > 0 ? o - 8 : a[2] * 512 + i + 56 + 64 * k0;
-    oN = j < 7 ? o + 8 : a[3] * 512 + i + 0 + 64 * k0;
-    oB = k0 > 0 ? o - 64 : a[4] * 512 + i + 8 * j + 448;
-    oT = k0 < 4 ? o + 256 : a[5] * 512 + i + 8 * j;
-#pragma unroll
-    for (int kk = 0; kk < 4; ++kk) {
-      xv[kk] = zero_x ? 0.0 : x[o + 64 * kk];
-      bv[kk] = b[o + 64 * kk];
-      xa[o + 64 * kk] = xv[kk];
-    }
-  }
-  __syncthreads();
-  for (int s = 0; s < sweeps; ++s) {
-    if (act) {
-      double nx[4];
-#pragma unroll
-      for (int kk = 0; kk < 4; ++kk) {
-        const double bt = kk > 0 ? xv[kk - 1] : xa[oB];
-        const double tp = kk < 3 ? xv[kk + 1] : xa[oT];
-        const double av = stencil_a(xv[kk], xa[oW + 64 * kk], xa[oE + 64 * kk], xa[oS + 64 * kk],
-                                    xa[oN + 64 * kk], bt, tp, c.alpha, c.beta);
-        nx[kk] = DADD(xv[kk], DMUL(c.gamma, DSUB(av, bv[kk])));
-      }
-#pragma unroll
-      for (int kk = 0; kk < 4; ++kk) {
-        xv[kk] = nx[kk];
-        xb[o + 64 * kk] = nx[kk];
-      }
-    }
-    __syncthreads();
-    double* tmp = xa;
-    xa = xb;
-    xb = tmp;
-  }
-  if (act)
-#pragma unroll
-    for (int kk = 0; kk < 4; ++kk) xo[o + 64 * kk] = xv[kk];
+  bottom_resident_body(x, xo, b, adj, nbricks, sweeps, zero_x, c, sm);
 }
 
 cudaError_t launch_bottom_resident(const double* x, double* xo, const double* b, const int32_t* adj, int nbricks,
@@ -735,7 +685,9 @@ cudaError_t kernels_init() {
   if (e != cudaSuccess) return e;
   e = pairw_kernels_init();
   if (e != cudaSuccess) return e;
-  return coarse_kernels_init();
+  e = coarse_kernels_init();
+  if (e != cudaSuccess) return e;
+  return coarse_grid_init();
 }
 
 }  // namespace mgb

@@ -159,6 +159,33 @@ struct CoarseArgs {
   double nu_pre[kCoarseMaxCheb], nu_post[kCoarseMaxCheb];  // Chebyshev nodes in sweep order (host-computed)
 };
 size_t coarse_smem_bytes(const CoarseArgs& a);
+// Grid-resident coarse solver (coarse_grid.cu): the same levels l0 .. L-1 in one launch of one
+// kGridCoarseThreads-thread CTA per SM (cooperative: all co-resident), fields in the level buffers,
+// a grid barrier between dependent steps; the bottom (<= kResidentMaxBricks bricks) in CTA 0.
+// x of every level starts at 0; x of level l0 ends in lv[0].x[0].  No ghosts.
+constexpr int kGridCoarseThreads = 1024;
+constexpr int64_t kGridCoarseMaxBricks = 512;  // largest level handed to it (512^3: levels 3 .. 5; measured)
+struct GridLevel {
+  int64_t nb;             // bricks (owned == stored: no ghosts)
+  const int32_t* adj;     // [nb][8]
+  const int32_t* parent;  // [nb] coarse brick * 8 + octant (levels < last)
+  double* x[2];           // ping-pong x (x[0] holds x at entry and, for level l0, at exit)
+  double* b;              // b (level l0: restricted by the level above; deeper: written here)
+  Coeffs c;
+  double h;
+};
+struct GridCoarseArgs {
+  int nlev;
+  GridLevel lv[kCoarseMaxLevels];
+  int pre, post, bottom;
+  int cheb;
+  double nu_pre[kCoarseMaxCheb], nu_post[kCoarseMaxCheb];
+  unsigned* bar;  // kGridBarWords words of zeroed device memory: arrive count, generation
+};
+constexpr int kGridBarWords = 16;
+cudaError_t launch_coarse_grid(const GridCoarseArgs& a, cudaStream_t s);
+cudaError_t coarse_grid_init();
+
 cudaError_t launch_coarse(const CoarseArgs& a, cudaStream_t s);
 cudaError_t coarse_kernels_init();
 cudaError_t kernels_init();  // one-time attribute setup

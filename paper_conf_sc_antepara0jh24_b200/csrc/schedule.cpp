@@ -1,6 +1,8 @@
 // schedule.cpp -- compiles Alg 2 into device ops; see schedule.h.
 #include "schedule.h"
 
+#include <cstdlib>
+
 #include <algorithm>
 
 #include "kernels.h"
@@ -197,7 +199,7 @@ void Builder::bottom(int l, int n, bool zero) {
   const int bm = lay.p.bottom_mode;
   const bool can_res = !ghosts(l) && L.n_stored <= kResidentMaxBricks;
   const bool res = can_res && (bm == MG_BOTTOM_RESIDENT ||
-                                ((bm == MG_BOTTOM_AUTO || bm == MG_BOTTOM_CLUSTER) && fusion(l) != MG_FUSION_PAPER));
+                                ((bm == MG_BOTTOM_AUTO || bm == MG_BOTTOM_CLUSTER || bm == MG_BOTTOM_GRID) && fusion(l) != MG_FUSION_PAPER));
   const bool fold_zero = zero && fusion(l) == MG_FUSION_FULL;
   if (res) {
     Op o;
@@ -220,10 +222,20 @@ int Builder::coarse_start() const {
   const int L = lay.L;
   const int bm = lay.p.bottom_mode;
   // opt-in: measured slower than graph-replayed per-level launches below 512^3
-  if (L < 2 || bm != MG_BOTTOM_CLUSTER) return -1;
+  if (L < 2 || (bm != MG_BOTTOM_CLUSTER && bm != MG_BOTTOM_GRID)) return -1;
   if (lay.p.pre_smooths < 1) return -1;
   if (lay.p.smoother == 1 && (lay.p.pre_smooths > kCoarseMaxCheb || lay.p.post_smooths > kCoarseMaxCheb)) return -1;
   if (lay.p.smoother == 2) return -1;  // red-black half-sweeps: per-level kernels only
+  if (bm == MG_BOTTOM_GRID) {  // grid-resident solve: the deepest ghost-free run of levels >= 1
+    int l0 = L;                // with <= kGridCoarseMaxBricks bricks (fields stay in HBM / L2)
+    static const int64_t maxb = getenv("MG_GRID_MAX_BRICKS") ? atoll(getenv("MG_GRID_MAX_BRICKS"))
+                                                              : kGridCoarseMaxBricks;  // (experiments)
+    while (l0 - 1 >= 1 && !ghosts(l0 - 1) && fusion(l0 - 1) != MG_FUSION_PAPER &&
+           lay.lv[l0 - 1].n_owned <= maxb && L - (l0 - 1) <= kCoarseMaxLevels)
+      --l0;
+    if (l0 >= L || ghosts(L - 1) || fusion(L - 1) == MG_FUSION_PAPER) return -1;
+    return l0;
+  }
   // the deepest run of levels >= 1 without ghosts, paper kernel set excluded, whose first level
   // fits the cluster (<= 8 bricks per CTA) and whose fields fit its shared memory
   int l0 = L;

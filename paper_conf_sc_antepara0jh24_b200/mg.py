@@ -19,7 +19,7 @@ MG_MAX_LEVELS = 16
 MG_FUSION_AUTO, MG_FUSION_PAPER, MG_FUSION_SWEEP, MG_FUSION_FULL = 0, 1, 2, 3
 MG_GHOST_AUTO, MG_GHOST_ALL = 0, 1
 MG_TRANSPORT_AUTO, MG_TRANSPORT_NCCL, MG_TRANSPORT_LOCAL = 0, 1, 2
-MG_BOTTOM_AUTO, MG_BOTTOM_SWEEPS, MG_BOTTOM_RESIDENT, MG_BOTTOM_CLUSTER = 0, 1, 2, 3
+MG_BOTTOM_AUTO, MG_BOTTOM_SWEEPS, MG_BOTTOM_RESIDENT, MG_BOTTOM_CLUSTER, MG_BOTTOM_GRID = 0, 1, 2, 3, 4
 MG_FIELD_X, MG_FIELD_B, MG_FIELD_R = 0, 1, 2
 OP_NAMES = ["sweep", "applyOp", "smooth", "restriction", "interpolation", "initZero", "exchange", "bottom"]
 MG_NUM_OPS = len(OP_NAMES)

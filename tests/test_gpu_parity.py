@@ -231,18 +231,22 @@ def test_solve_matches_oracle(oracle_mod):
     m.close()
 
 
-@pytest.mark.parametrize("bottom_mode", [0, 1, 2, 3])
+@pytest.mark.parametrize("bottom_mode", [0, 1, 2, 3, 4])
 @pytest.mark.parametrize("shape,L,pre,post,bottom", [
     ((64, 64, 64), 4, 12, 12, 100),   # config 1: levels 1-3 (64, 8, 1 bricks) in the cluster
     ((32, 96, 64), 3, 3, 2, 20),      # non-cubic, ragged brick counts per CTA (48 -> 6 bricks)
     ((64, 32, 96), 3, 2, 0, 5),       # post = 0
     ((32, 32, 32), 3, 1, 1, 0),       # bottom = 0
     ((64, 64, 64), 2, 2, 2, 7),       # coarsest level alone (64 bricks) in the cluster
+    ((128, 64, 64), 3, 1, 2, 3),      # pre = 1 (the first sweep is the restriction sweep)
+    ((128, 128, 128), 5, 12, 12, 100),  # grid solve: levels 1-4 (512 .. 1 bricks)
+    ((96, 128, 64), 2, 3, 3, 9),      # coarsest level of 48 bricks: the bottom as grid sweeps
 ])
 def test_coarse_cluster_solver_bitwise(oracle_mod, bottom_mode, shape, L, pre, post, bottom):
-    """The cluster-resident coarse solve (coarse.cu, bottom_mode auto / cluster: the deepest
-    ghost-free levels in one launch, neighbours through DSMEM) against per-level launches
-    (sweeps / resident) and the oracle, bit for bit, 2 cycles."""
+    """The cluster-resident coarse solve (coarse.cu, bottom_mode cluster: the deepest ghost-free
+    levels in one launch, neighbours through DSMEM) and the grid-resident one (coarse_grid.cu,
+    bottom_mode grid: one CTA per SM, grid barriers) against per-level launches (auto / sweeps /
+    resident) and the oracle, bit for bit, 2 cycles."""
     b = mg_inputs.random_rhs(shape, 31)
     xs, ns = oracle_cycles(oracle_mod, b, L, 2, pre, post, bottom)
     m = new(shape, L, pre=pre, post=post, bottom=bottom, bottom_mode=bottom_mode)
@@ -476,6 +480,27 @@ def test_pencil_pass_work_splits(oracle_mod, n, shape, ghost_mode):
     m.close()
 
 
+def test_vcycle_512_grid_coarse_bitwise(oracle_mod):
+    """At the bench size (512^3, L = 6) the grid-resident coarse solve (levels 2-5) and the
+    per-level launches give identical x after one V-cycle (bitwise over the whole field) and the
+    same residual norm."""
+    import torch
+
+    shape = (512, 512, 512)
+    b = mg_inputs.sin_rhs(shape)
+    out = []
+    for bm in (0, 4):
+        m = new(shape, 6, bottom_mode=bm)
+        m.set_rhs(dev(b))
+        m.set_solution(None)
+        m.vcycle()
+        out.append((m.get_solution(), m.residual_norm()))
+        m.close()
+        torch.cuda.empty_cache()
+    assert torch.equal(out[0][0], out[1][0])
+    assert out[0][1] == out[1][1]
+
+
 @pytest.mark.parametrize("tb", [0, 1, 2, 3])
 def test_temporal_blocking_on_off_bitwise(oracle_mod, tb):
     """The V-cycle with and without temporal blocking gives the oracle's bits (256^3, L = 6,
@@ -508,7 +533,8 @@ def test_programmatic_dependent_launch_on_off_bitwise(oracle_mod, launch_pdl, us
 
 # ------------------------------------------------- Chebyshev smoother variant (N4, reading A19)
 @pytest.mark.parametrize("kw", [dict(), dict(temporal_blocking=0), dict(fusion=1), dict(temporal_blocking=2),
-                                dict(bottom_mode=1), dict(bottom_mode=3), dict(ghost_mode=1, ca_period=4),
+                                dict(bottom_mode=1), dict(bottom_mode=3), dict(bottom_mode=4),
+                                dict(ghost_mode=1, ca_period=4),
                                 dict(sweep_kernel=2), dict(cheby_ratio=10), dict(temporal_blocking=3),
                                 dict(temporal_blocking=3, sweep_kernel=2)])
 def test_chebyshev_smoother_vcycle_bitwise(oracle_mod, kw):
