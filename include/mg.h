@@ -256,7 +256,9 @@ mg_status mg_group_destroy(mg_group* g);
  * remote brick offset, brick count.
  * pass plan: the two-sweep (temporal blocking) plan number `idx` of a level (one per swept brick
  * range).  info[0] kind (1 one-brick CTA streams, 2 warp plane streams, 3 2x2-brick pencil chunk
- * streams), [1] b0, [2] b1 (brick range), [3] ints of meta, [4] ints of ctas; MG_ERR_INVALID_ARG
+ * streams), [1] b0, [2] b1 (brick range), [3] ints of meta, [4] ints of ctas, [5] part (kind 3
+ * on a level with a ghost shell: 0 every unit of the range, 1 the units whose records name no
+ * ghost brick -- swept while an exchange fills the ghosts --, 2 the others); MG_ERR_INVALID_ARG
  * if idx is past the last plan.  meta / ctas (may be NULL: sizes only) receive copies of the
  * tables the kernel reads; for kind 3, meta = int32 [chunks][20] = code (type << 1 | half; type 0
  * range, 1 warm-up, 2 cool-down), ids of b00, b10, b01, b11, W0, W1, E0, E1, S0, S1, N0, N1, SW,
@@ -268,7 +270,7 @@ mg_status mg_layout_adjacency(const mg_layout* lay, int32_t level, int32_t* out)
 mg_status mg_layout_coords(const mg_layout* lay, int32_t level, int32_t* out);
 mg_status mg_layout_parent(const mg_layout* lay, int32_t level, int32_t* out);
 mg_status mg_layout_plan(const mg_layout* lay, int32_t level, int32_t which /*0 send,1 recv*/, int64_t* out);
-mg_status mg_layout_pass_plan(const mg_layout* lay, int32_t level, int32_t idx, int64_t info[5], int32_t* meta,
+mg_status mg_layout_pass_plan(const mg_layout* lay, int32_t level, int32_t idx, int64_t info[6], int32_t* meta,
                               int32_t* ctas);
 mg_status mg_layout_destroy(mg_layout* lay);
 

@@ -52,6 +52,7 @@ struct DevLevel {
   FaceMaps fmaps[2];      // TMA face-halo tensor maps over x[0], x[1] (levels with column plans)
   struct Pair {
     int64_t b0, b1;
+    int part;  // LevelLayout::PairTable::part
     PairArgs args;
   };
   std::vector<Pair> pairs;  // two-sweep item streams per brick range
@@ -103,6 +104,11 @@ struct mg_ctx {
   bool poisoned = false;
   bool timing = false;
   bool use_col = true;  // streaming column kernel where a plan exists (sweep_kernel == 1 disables)
+  // pencil passes on ghost-shell levels: the units that read no ghost brick overlap the exchange.
+  // Default: only for exchanges with other processes (NCCL, world_size > 1); measured slower with a
+  // local self-exchange (0.16 ms of copies per cycle do not pay for the split).
+  // MG_PENCIL_OVERLAP=0/1 overrides (tests, measurements).
+  bool pencil_overlap = false;
   std::vector<double> tm;
   std::vector<TimerRec> trec;
   std::vector<std::pair<int, double>> recs;  // (level*MG_NUM_OPS + op, ms) per timed op, since mg_set_timing
@@ -184,6 +190,7 @@ size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double**
       DevLevel::Pair pr;
       pr.b0 = pt.b0;
       pr.b1 = pt.b1;
+      pr.part = pt.part;
       pr.args.kind = pt.kind;
       pr.args.meta = (const int32_t*)take(pt.meta.size() * sizeof(int32_t));
       pr.args.ctas = (const int2*)take(pt.ctas.size() * sizeof(int32_t));
@@ -294,7 +301,8 @@ mg_status fill_copy_tables(mg_ctx* c) {
 }
 
 // ------------------------------------------------------------- executor
-mg_status sweep_range(mg_ctx* c, const Op& o, int64_t b0, int64_t b1, cudaStream_t s) {
+// part: for OP_SWEEP2, which units of the range's pencil plan (LevelLayout::PairTable::part)
+mg_status sweep_range(mg_ctx* c, const Op& o, int64_t b0, int64_t b1, cudaStream_t s, int part = 0) {
   if (b1 <= b0) return MG_OK;
   DevLevel& d = c->dl[o.level];
   const int l = o.level;
@@ -324,7 +332,7 @@ mg_status sweep_range(mg_ctx* c, const Op& o, int64_t b0, int64_t b1, cudaStream
   a.colour2 = o.c2;
   if (o.kind == OP_SWEEP2) {  // two sweeps in one pass: the builder only emits it where a plan exists
     for (const auto& pr : d.pairs) {
-      if (pr.b0 == b0 && pr.b1 == b1) {
+      if (pr.b0 == b0 && pr.b1 == b1 && pr.part == part) {
         if (pr.args.kind == 3)
           CKC(c, launch_sweep2p(a, pr.args, d.nmaps[o.src], o.flags, s));
         else if (pr.args.kind == 2)
@@ -371,6 +379,22 @@ mg_status exec_op(mg_ctx* c, const Op& o, cudaStream_t s) {
     case OP_SWEEP2: {
       const int64_t end = o.ghosts ? L.n_stored : L.n_owned;
       if (o.exch_before) {
+        // pencil passes: the units that read no ghost brick overlap the exchange, the rest follow
+        bool pen_split = false;
+        if (o.kind == OP_SWEEP2 && c->lay.p.overlap && c->pencil_overlap)
+          for (const auto& pr : d.pairs) pen_split |= pr.b0 == 0 && pr.b1 == end && pr.part == 1;
+        if (pen_split) {
+          CKS(timer_begin(c, s, &t0));
+          CKC(c, cudaEventRecord(c->ev_fork, s));
+          CKC(c, cudaStreamWaitEvent(c->comm, c->ev_fork, 0));
+          CKS(do_exchange(c, o.level, 0, o.src, c->comm));
+          CKC(c, cudaEventRecord(c->ev_join, c->comm));
+          CKS(sweep_range(c, o, 0, end, s, 1));
+          CKC(c, cudaStreamWaitEvent(s, c->ev_join, 0));
+          CKS(sweep_range(c, o, 0, end, s, 2));
+          CKS(timer_end(c, s, t0, o.level, o.timer));
+          return MG_OK;
+        }
         const bool split = c->lay.p.overlap && L.n_interior > 0 && !o.nosplit;
         if (split) {
           CKS(timer_begin(c, s, &t0));
@@ -463,11 +487,11 @@ mg_status exec_op(mg_ctx* c, const Op& o, cudaStream_t s) {
   return set_err(MG_ERR_STATE, "unknown op");
 }
 
-Plan make_plan(const Builder& b, const Layout& lay) {
+Plan make_plan(const Builder& b, const Layout& lay, bool pencil_overlap) {
   Plan p;
   p.ops = b.ops;
   for (int l = 0; l < MG_MAX_LEVELS; ++l) p.final_st[l] = b.st[l];
-  for (const Op& o : p.ops) p.launches += op_launches(o, lay, lay.p.overlap != 0);
+  for (const Op& o : p.ops) p.launches += op_launches(o, lay, lay.p.overlap != 0, pencil_overlap);
   return p;
 }
 
@@ -506,7 +530,7 @@ mg_status check_ctx(mg_ctx* c) {
 }
 
 mg_status build_and_run(mg_ctx* c, mg_group* g, bool vcycle_graph, Builder& b) {
-  const Plan p = make_plan(b, c->lay);
+  const Plan p = make_plan(b, c->lay, c->pencil_overlap);
   CKS(run_plan(c, g, p, g ? g->stream : c->stream));
   if (g) {
     for (mg_ctx* r : g->r)
@@ -532,7 +556,7 @@ mg_status vcycle_impl(mg_ctx* c, mg_group* g) {
     Builder b(c0->lay);
     for (int l = 0; l < MG_MAX_LEVELS; ++l) b.st[l] = c0->st[l];
     b.vcycle();
-    Plan p = make_plan(b, c0->lay);
+    Plan p = make_plan(b, c0->lay, c0->pencil_overlap);
     if (graph) {
       // capture on a private non-blocking stream; the graph is then launched on the caller's stream
       cudaStream_t cs = g ? g->cap : c->cap;
@@ -581,6 +605,8 @@ mg_status init_ctx(mg_ctx* c, const mg_params& p, int rank, int world, int devic
   c->device = device;
   c->stream = stream;
   c->use_col = p.sweep_kernel != 1;
+  c->pencil_overlap = world > 1 && p.transport != MG_TRANSPORT_LOCAL;
+  if (const char* e = getenv("MG_PENCIL_OVERLAP")) c->pencil_overlap = atoi(e) != 0;
   const size_t need = carve(c->lay, nullptr, nullptr, nullptr, nullptr);
   if (!workspace || ws_bytes < need)
     return set_err(MG_ERR_OOM, "workspace too small: need " + std::to_string(need) + " bytes");
@@ -937,7 +963,7 @@ mg_status mg_vcycle_launches(mg_ctx* c, int64_t* out) {
   Builder b(c->lay);
   for (int l = 0; l < MG_MAX_LEVELS; ++l) b.st[l] = c->st[l];
   b.vcycle();
-  *out = make_plan(b, c->lay).launches;
+  *out = make_plan(b, c->lay, c->pencil_overlap).launches;
   return MG_OK;
 }
 
@@ -1238,7 +1264,7 @@ mg_status mg_layout_plan(const mg_layout* m, int32_t level, int32_t which, int64
   return MG_OK;
 }
 
-mg_status mg_layout_pass_plan(const mg_layout* m, int32_t level, int32_t idx, int64_t info[5], int32_t* meta,
+mg_status mg_layout_pass_plan(const mg_layout* m, int32_t level, int32_t idx, int64_t info[6], int32_t* meta,
                               int32_t* ctas) {
   const LevelLayout* L = nullptr;
   CKS(lay_level(m, level, &L));
@@ -1250,6 +1276,7 @@ mg_status mg_layout_pass_plan(const mg_layout* m, int32_t level, int32_t idx, in
   info[2] = t.b1;
   info[3] = (int64_t)t.meta.size();
   info[4] = (int64_t)t.ctas.size();
+  info[5] = t.part;
   if (meta) std::copy(t.meta.begin(), t.meta.end(), meta);
   if (ctas) std::copy(t.ctas.begin(), t.ctas.end(), ctas);
   return MG_OK;

@@ -12,6 +12,7 @@
 //    order ("optimal brick layout", "packing- and unpacking-free
 //    communication buffers").  The order of the 26 surface regions below was
 //    found by tools/region_order_search.py: 42 runs for 26 neighbours.
+#include <cstdlib>
 #include <algorithm>
 #include <array>
 #include <cstdio>
@@ -418,7 +419,10 @@ static LevelLayout::PairTable pair_table(const LevelLayout& L, int64_t b0, int64
 // (two-sweep passes that sweep the ghosts redundantly, so one exchange serves several passes):
 // there the tiles cover the extended box (owned + ghost layer), aligned to its origin, and no
 // restriction runs.  Returns kind 0 if the range does not tile.
-static LevelLayout::PairTable pencil_table(const LevelLayout& L, int64_t b0, int64_t b1) {
+// part 1 / 2 (levels with a ghost shell): only the units whose records name no ghost brick /
+// the others, so the first can run while an exchange fills the ghost bricks (part 1 on one CTA
+// slot per SM fewer, which the exchange's kernels then find free).
+static LevelLayout::PairTable pencil_table(const LevelLayout& L, int64_t b0, int64_t b1, int part = 0) {
   LevelLayout::PairTable t;
   t.kind = 0;
   const bool owned = b0 == 0 && b1 == L.n_owned;
@@ -466,8 +470,10 @@ static LevelLayout::PairTable pencil_table(const LevelLayout& L, int64_t b0, int
   t.kind = 3;
   t.b0 = b0;
   t.b1 = b1;
+  t.part = part;
   const int64_t ncol = (int64_t)tx * ty;
-  const int64_t G = std::max<int64_t>(1, std::min<int64_t>(kPenCtas, ncol * nz));
+  static const int64_t gmax = getenv("MG_PEN_CTAS") ? atoll(getenv("MG_PEN_CTAS")) : kPenCtas;  // (experiments)
+  const int64_t G = std::max<int64_t>(1, std::min<int64_t>(gmax, ncol * nz));
   std::vector<std::vector<int32_t>> stream((size_t)G);  // per CTA: its chunk records
   // one 20-int record per chunk: code (type << 1 | half), the 16 brick ids, parent of b00
   auto push_chunk = [&](std::vector<int32_t>& v, const std::array<int32_t, kPenMeta>& m, int type, int half) {
@@ -509,10 +515,32 @@ static LevelLayout::PairTable pencil_table(const LevelLayout& L, int64_t b0, int
     const int64_t cost = *std::max_element(cta.begin(), cta.end());
     if (cost < best_cost) best_cost = cost, best = nzr;
   }
-  for (int64_t u = 0; u < ncol * best; ++u) {
-    const int r = (int)(u / ncol);
-    const int64_t col = u % ncol;
-    push_run(stream[(size_t)(u % G)], col, zr0(best, r), zr0(best, r + 1) - zr0(best, r));
+  if (part == 0) {
+    for (int64_t u = 0; u < ncol * best; ++u) {
+      const int r = (int)(u / ncol);
+      const int64_t col = u % ncol;
+      push_run(stream[(size_t)(u % G)], col, zr0(best, r), zr0(best, r + 1) - zr0(best, r));
+    }
+  } else {  // the units of one part, in the same order, dealt round-robin over Gp CTAs
+    const int64_t Gp = std::max<int64_t>(1, part == 1 ? G - G / kPenCtasPerSm : G);
+    int64_t k = 0;
+    std::vector<int32_t> run;
+    for (int64_t u = 0; u < ncol * best; ++u) {
+      const int r = (int)(u / ncol);
+      const int64_t col = u % ncol;
+      run.clear();
+      push_run(run, col, zr0(best, r), zr0(best, r + 1) - zr0(best, r));
+      bool ghost = false;
+      for (size_t e = 0; e < run.size(); e += kPenRec)
+        for (int f = 1; f <= 16; ++f) {
+          const int32_t id = run[e + (size_t)f];
+          ghost |= id >= L.n_owned && id < L.n_stored;
+        }
+      if (ghost != (part == 2)) continue;
+      auto& v = stream[(size_t)(k++ % Gp)];
+      v.insert(v.end(), run.begin(), run.end());
+    }
+    if (k == 0) t.kind = 0;
   }
   for (int64_t g = 0; g < G; ++g) {
     const auto& v = stream[(size_t)g];
@@ -635,6 +663,18 @@ void build_pair_tables(LevelLayout& L, int64_t min_bricks, int kind) {
     if (t.kind == 0) t = kind == 2 ? warp_table(L, r[0], r[1]) : pair_table(L, r[0], r[1]);
     if (t.kind != 0) L.pairs.push_back(std::move(t));
   }
+  // pencil passes over a level with a ghost shell: the units split by whether they read a ghost
+  // brick, for the overlap of the exchange with the interior units (both parts or neither)
+  if (kind == 3 && L.n_ghost > 0)
+    for (const int64_t b1 : {L.n_owned, L.n_stored}) {
+      bool have = false;
+      for (const auto& c : L.pairs) have |= c.kind == 3 && c.part == 0 && c.b0 == 0 && c.b1 == b1;
+      if (!have) continue;
+      LevelLayout::PairTable p1 = pencil_table(L, 0, b1, 1), p2 = pencil_table(L, 0, b1, 2);
+      if (p1.kind != 3 || p2.kind != 3) continue;
+      L.pairs.push_back(std::move(p1));
+      L.pairs.push_back(std::move(p2));
+    }
 }
 
 }  // namespace mgb

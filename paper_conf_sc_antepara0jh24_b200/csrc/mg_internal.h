@@ -74,6 +74,9 @@ struct LevelLayout {
   struct PairTable {
     int kind = 1;
     int64_t b0 = 0, b1 = 0;
+    // kind 3 on a level with a ghost shell: 0 = every unit of the range; 1 = the units that read
+    // no ghost brick (swept while the exchange fills the ghosts), 2 = the others (after it)
+    int part = 0;
     std::vector<int32_t> meta;   // [items][kPairMeta] (kind 1) / [items][kW2Meta] (kind 2)
     std::vector<int32_t> ctas;   // kind 1: [nctas][2] offset (items), count
     std::vector<int32_t> warps;  // kind 2: [nwarps][4] first item of half 0, of half 1, steps, items0 | items1<<16

@@ -26,13 +26,13 @@ int Builder::period(int l) const {
 
 bool Builder::has_pair_table(int l, int64_t b0, int64_t b1) const {
   for (const auto& pt : lay.lv[l].pairs)
-    if (pt.b0 == b0 && pt.b1 == b1) return true;
+    if (pt.b0 == b0 && pt.b1 == b1 && pt.part == 0) return true;
   return false;
 }
 
 bool Builder::pencil_table(int l) const {
   for (const auto& pt : lay.lv[l].pairs)
-    if (pt.b0 == 0 && pt.b1 == lay.lv[l].n_owned) return pt.kind == 3;
+    if (pt.b0 == 0 && pt.b1 == lay.lv[l].n_owned && pt.part == 0) return pt.kind == 3;
   return false;
 }
 
@@ -40,7 +40,7 @@ bool Builder::pencil_ghosts(int l) const {
   const LevelLayout& L = lay.lv[l];
   if (L.n_ghost == 0) return false;
   for (const auto& pt : L.pairs)
-    if (pt.b0 == 0 && pt.b1 == L.n_stored) return pt.kind == 3;
+    if (pt.b0 == 0 && pt.b1 == L.n_stored && pt.part == 0) return pt.kind == 3;
   return false;
 }
 
@@ -316,11 +316,17 @@ void Builder::vcycle() {
   }
 }
 
-int64_t op_launches(const Op& o, const Layout& lay, bool overlap) {
+int64_t op_launches(const Op& o, const Layout& lay, bool overlap, bool pencil_overlap) {
   switch (o.kind) {
     case OP_SWEEP:
     case OP_SWEEP2: {
       const int per = o.paper ? 2 : 1;
+      const LevelLayout& L = lay.lv[o.level];
+      const int64_t end = o.ghosts ? L.n_stored : L.n_owned;
+      bool pen_split = false;
+      if (o.kind == OP_SWEEP2 && o.exch_before && overlap && pencil_overlap)
+        for (const auto& pt : L.pairs) pen_split |= pt.b0 == 0 && pt.b1 == end && pt.part == 1;
+      if (pen_split) return 2;
       const bool split = o.exch_before && overlap && lay.lv[o.level].n_interior > 0 && !o.nosplit;
       return per * (split ? 2 : 1);
     }

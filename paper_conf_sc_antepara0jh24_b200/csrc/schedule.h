@@ -73,6 +73,6 @@ struct Builder {
   void vcycle();
 };
 
-int64_t op_launches(const Op& o, const Layout& lay, bool overlap);
+int64_t op_launches(const Op& o, const Layout& lay, bool overlap, bool pencil_overlap);
 
 }  // namespace mgb

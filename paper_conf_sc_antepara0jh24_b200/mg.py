@@ -383,18 +383,18 @@ class Layout:
         return a
 
     def pass_plans(self, level):
-        """Two-sweep pass plans of a level: [(kind, b0, b1, meta int32 array, ctas int32 [n][2])]."""
+        """Two-sweep pass plans of a level: [(kind, b0, b1, meta int32 array, ctas int32 [n][2], part)]."""
         np = self._np
         out = []
         for idx in range(64):
-            info = (ctypes.c_int64 * 5)()
+            info = (ctypes.c_int64 * 6)()
             if lib().mg_layout_pass_plan(self.h, level, idx, info, None, None) != 0:
                 break
             meta = np.zeros(max(info[3], 1), dtype=np.int32)
             ctas = np.zeros(max(info[4], 2), dtype=np.int32)
             check(lib().mg_layout_pass_plan(self.h, level, idx, info, meta.ctypes.data, ctas.ctypes.data),
                   "mg_layout_pass_plan")
-            out.append((info[0], info[1], info[2], meta[:info[3]], ctas[:info[4]].reshape(-1, 2)))
+            out.append((info[0], info[1], info[2], meta[:info[3]], ctas[:info[4]].reshape(-1, 2), info[5]))
         return out
 
     def plan(self, level, which):

@@ -515,6 +515,38 @@ def test_temporal_blocking_on_off_bitwise(oracle_mod, tb):
     m.close()
 
 
+@pytest.mark.parametrize("mode", ["loopback", "self"])
+def test_pencil_exchange_overlap_bitwise(oracle_mod, mode, monkeypatch):
+    """Pencil passes on ghost-shell levels with the exchange overlapped (MG_PENCIL_OVERLAP=1: the
+    units that read no ghost brick run while the exchange fills the ghosts, the rest after it):
+    oracle bits for a 2x2x2 loopback decomposition and for the self-exchanged ghost shell."""
+    monkeypatch.setenv("MG_PENCIL_OVERLAP", "1")
+    mg, solver = _mg()
+    if mode == "self":
+        shape = (128, 128, 128)
+        b = mg_inputs.random_rhs(shape, 37)
+        xs, ns = oracle_cycles(oracle_mod, b, 4, 2)
+        m = new(shape, 4, ghost_mode=1, ca_period=8)
+        m.set_rhs(dev(b))
+        m.set_solution(None)
+        check_cycles(m, xs, ns)
+        m.close()
+        return
+    pg, n_local = (2, 2, 2), (64, 64, 64)
+    gshape = (n_local[2] * pg[2], n_local[1] * pg[1], n_local[0] * pg[0])
+    b = mg_inputs.random_rhs(gshape, 38)
+    xs, ns = oracle_cycles(oracle_mod, b, 3, 2)
+    g = solver.LoopbackGroup(n_local, pg, num_levels=3)
+    g.set_rhs([dev(mg_inputs.local_block(b, r, pg)) for r in range(g.world_size)])
+    g.set_solution(None)
+    for c in range(2):
+        g.vcycle()
+        assert g.residual_norm() == ns[c]
+        for r in range(g.world_size):
+            assert_bitwise(host(g.get_solution(r)), mg_inputs.local_block(xs[c], r, pg), what=f"rank {r}")
+    g.close()
+
+
 @pytest.mark.parametrize("launch_pdl", [1, 2])
 @pytest.mark.parametrize("use_graph", [True, False])
 def test_programmatic_dependent_launch_on_off_bitwise(oracle_mod, launch_pdl, use_graph):

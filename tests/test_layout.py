@@ -197,15 +197,28 @@ def test_pencil_plan_covers_owned_bricks(n_local, pg, L, gm):
     inf = lay.info(0)
     adj, crd = lay.adjacency(0), lay.coords(0)
     par = lay.parent(0) if L > 1 else None
-    plans = [pl for pl in lay.pass_plans(0) if pl[0] == 3]
+    allp = [pl for pl in lay.pass_plans(0) if pl[0] == 3]
+    plans = [pl for pl in allp if pl[5] == 0]
     # the owned range (tiles on even owned coordinates: restriction), and with a ghost shell the
     # whole stored range (tiles on the extended box, ghost-sweeping passes)
     want = [(0, inf["owned"])] + ([(0, inf["owned"] + inf["nghost"])] if inf["nghost"] else [])
     assert [(pl[1], pl[2]) for pl in plans] == want
-    for _, b0, b1, meta, ctas in plans:
+    for _, b0, b1, meta, ctas, _ in plans:
         owned = b1 == inf["owned"]
         g = np.array(inf["ghost"][:2]) * (0 if owned else 1)
-        _check_pencil_plan(meta, ctas, b1, adj, crd, par if owned else None, g)
+        assert (_check_pencil_plan(meta, ctas, b1, adj, crd, par if owned else None, g) == 1).all()
+        # with a ghost shell: the same units split into those that read no ghost brick (swept while
+        # the exchange fills the ghosts) and the rest; together they cover every brick once per half
+        parts = {pl[5]: pl for pl in allp if pl[5] and (pl[1], pl[2]) == (b0, b1)}
+        assert sorted(parts) == ([1, 2] if inf["nghost"] else [])
+        if parts:
+            seen = sum(_check_pencil_plan(parts[k][3], parts[k][4], b1, adj, crd, par if owned else None, g)
+                       for k in (1, 2))
+            assert (seen == 1).all()
+            ids = parts[1][3].reshape(-1, 20)[:, 1:17]
+            assert not ((ids >= inf["owned"]) & (ids < inf["owned"] + inf["nghost"])).any()
+            ids2 = parts[2][3].reshape(-1, 20)[:, 1:17]
+            assert ((ids2 >= inf["owned"]) & (ids2 < inf["owned"] + inf["nghost"])).any()
 
 
 def _check_pencil_plan(meta, ctas, nrange, adj, crd, par, g):
@@ -246,6 +259,6 @@ def _check_pencil_plan(meta, ctas, nrange, adj, crd, par, g):
                     seen[b, r[0] & 1] += 1
                     if par is not None:
                         assert pa % 4 == 0 and par[b] == pa + k
-    assert (seen == 1).all()
     ideal = sum(work) / len(work)
     assert max(work) <= ideal * 1.15 + 8
+    return seen
