@@ -109,6 +109,17 @@ struct mg_ctx {
   // local self-exchange (0.16 ms of copies per cycle do not pay for the split).
   // MG_PENCIL_OVERLAP=0/1 overrides (tests, measurements).
   bool pencil_overlap = false;
+  // replicated bottom (Layout::repl): the global coarsest level's fields and the copy tables that
+  // gather b into it and scatter this rank's owned x out of it
+  struct Repl {
+    double* x[2] = {nullptr, nullptr};
+    double* b = nullptr;
+    int32_t* adj = nullptr;
+    double* gbuf = nullptr;  // all-gather landing buffer [world][n_owned bricks] (NCCL)
+    CopyRun* gather = nullptr;
+    CopyRun* scatter = nullptr;  // [2][n_owned]: into x[0] / x[1] of the coarsest level
+    bool allgather = false;
+  } rp;
   std::vector<double> tm;
   std::vector<TimerRec> trec;
   std::vector<std::pair<int, double>> recs;  // (level*MG_NUM_OPS + op, ms) per timed op, since mg_set_timing
@@ -156,7 +167,8 @@ struct mg_group {
 namespace {
 
 // ------------------------------------------------------------- workspace
-size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double** stage, unsigned long long** acc) {
+size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double** stage, unsigned long long** acc,
+             mg_ctx::Repl* rp = nullptr) {
   size_t off = 0;
   auto take = [&](size_t bytes) -> char* {
     const size_t o = align256(off);
@@ -210,6 +222,19 @@ size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double**
   for (int k = 0; k < 2; ++k) {
     double* st = (double*)take((size_t)lay.lv[0].n_owned * kBV * sizeof(double));
     if (stage) stage[k] = st;
+  }
+  if (lay.repl) {  // replicated bottom
+    const size_t gfb = (size_t)lay.gb.n_alloc * kBV * sizeof(double);
+    const int64_t nown = lay.lv[(size_t)lay.L - 1].n_owned;
+    mg_ctx::Repl r;
+    r.x[0] = (double*)take(gfb);
+    r.x[1] = (double*)take(gfb);
+    r.b = (double*)take(gfb);
+    r.adj = (int32_t*)take((size_t)lay.gb.n_stored * 8 * sizeof(int32_t));
+    r.gbuf = lay.world > 1 ? (double*)take((size_t)lay.world * nown * kBV * sizeof(double)) : nullptr;
+    r.gather = (CopyRun*)take((size_t)lay.gb.n_owned * sizeof(CopyRun));
+    r.scatter = (CopyRun*)take((size_t)2 * nown * sizeof(CopyRun));
+    if (rp) *rp = r;
   }
   // norm accumulator (word 0) and the grid coarse solve's barrier words (from byte 64, kGridBarWords)
   unsigned long long* ac = (unsigned long long*)take(64 + kGridBarWords * sizeof(unsigned));
@@ -271,6 +296,39 @@ mg_status do_exchange(mg_ctx* c, int l, int field, int xbuf, cudaStream_t s) {
     const int fv = field ? 2 : xbuf;
     CKC(c, launch_copy_runs(d.cruns + (size_t)fv * d.ncruns, d.ncruns, d.cmax, s));
   }
+  return MG_OK;
+}
+
+// Replicated bottom tables: global brick q <- its owner's owned b brick (from the all-gather
+// buffer on NCCL, straight from the owner's field in a loopback group or a one-rank run), and this
+// rank's owned coarsest bricks <- their global bricks (the solve leaves x in rp.x[1]).
+mg_status fill_repl_tables(mg_ctx* c) {
+  const Layout& lay = c->lay;
+  if (!lay.repl) return MG_OK;
+  const int lb = lay.L - 1;
+  const int64_t nown = lay.lv[(size_t)lb].n_owned;
+  const size_t bb = (size_t)kBV;
+  c->rp.allgather = c->use_nccl && lay.world > 1;
+  std::vector<CopyRun> g((size_t)lay.gb.n_owned), sc((size_t)2 * nown);
+  for (int64_t q = 0; q < lay.gb.n_owned; ++q) {
+    const int32_t src = lay.gb_src[(size_t)q];
+    const int r = (int)(src / nown);
+    const int64_t i = src % nown;
+    const double* from;
+    if (c->rp.allgather)
+      from = c->rp.gbuf + (size_t)src * bb;
+    else if (c->group)
+      from = c->group->r[(size_t)r]->dl[(size_t)lb].b + (size_t)i * bb;
+    else
+      from = c->dl[(size_t)lb].b + (size_t)i * bb;
+    g[(size_t)q] = {from, c->rp.b + (size_t)q * bb, (int64_t)bb};
+  }
+  for (int xb = 0; xb < 2; ++xb)
+    for (int64_t i = 0; i < nown; ++i)
+      sc[(size_t)xb * nown + i] = {c->rp.x[1] + (size_t)lay.gb_mine[(size_t)i] * bb,
+                                   c->dl[(size_t)lb].x[xb] + (size_t)i * bb, (int64_t)bb};
+  CKC(c, cudaMemcpy(c->rp.gather, g.data(), g.size() * sizeof(CopyRun), cudaMemcpyHostToDevice));
+  CKC(c, cudaMemcpy(c->rp.scatter, sc.data(), sc.size() * sizeof(CopyRun), cudaMemcpyHostToDevice));
   return MG_OK;
 }
 
@@ -478,6 +536,29 @@ mg_status exec_op(mg_ctx* c, const Op& o, cudaStream_t s) {
       CKS(timer_end(c, s, t0, o.level, o.timer));
       return MG_OK;
     }
+    case OP_BOTTOM_REPL: {
+      const Layout& lay = c->lay;
+      const int64_t ng = lay.gb.n_owned;
+      CKS(timer_begin(c, s, &t0));
+      if (c->rp.allgather)
+        CKN(c, ncclAllGather(d.b, c->rp.gbuf, (size_t)L.n_owned * kBV, ncclFloat64, c->nccl, s));
+      CKC(c, launch_copy_runs(c->rp.gather, (int)ng, kBV, s));
+      if (ng <= kResidentMaxBricks) {
+        CKC(c, launch_bottom_resident(c->rp.x[0], c->rp.x[1], c->rp.b, c->rp.adj, (int)ng, o.n, true, d.c, s));
+      } else {
+        CoarseArgs a{};
+        a.nlev = 1;
+        a.lv[0] = {(int)ng, c->rp.adj, nullptr, d.c, d.h};
+        a.b0 = c->rp.b;
+        a.x0 = c->rp.x[1];
+        a.pre = a.post = 0;
+        a.bottom = o.n;
+        CKC(c, launch_coarse(a, s));
+      }
+      CKC(c, launch_copy_runs(c->rp.scatter + (size_t)o.dst * L.n_owned, (int)L.n_owned, kBV, s));
+      CKS(timer_end(c, s, t0, o.level, o.timer));
+      return MG_OK;
+    }
     case OP_BOTTOM_RES:
       CKS(timer_begin(c, s, &t0));
       CKC(c, launch_bottom_resident(d.x[o.src], d.x[o.dst], d.b, d.adj, (int)L.n_stored, o.n, o.zero, d.c, s));
@@ -611,7 +692,7 @@ mg_status init_ctx(mg_ctx* c, const mg_params& p, int rank, int world, int devic
   if (!workspace || ws_bytes < need)
     return set_err(MG_ERR_OOM, "workspace too small: need " + std::to_string(need) + " bytes");
   if (((uintptr_t)workspace & 255) != 0) return set_err(MG_ERR_INVALID_ARG, "workspace must be 256-byte aligned");
-  carve(c->lay, (char*)workspace, &c->dl, c->stage, &c->acc);
+  carve(c->lay, (char*)workspace, &c->dl, c->stage, &c->acc, &c->rp);
   (void)tables_only_upload;
   CKC(c, cudaMemsetAsync(workspace, 0, need, stream));
   for (int l = 0; l < c->lay.L; ++l) {
@@ -645,6 +726,9 @@ mg_status init_ctx(mg_ctx* c, const mg_params& p, int rank, int world, int devic
         CKC(c, encode_pencil_maps(d.x[xb], d.b, L.n_alloc, &d.nmaps[xb]));
       }
   }
+  if (c->lay.repl)
+    CKC(c, cudaMemcpyAsync(c->rp.adj, c->lay.gb.adj.data(), c->lay.gb.adj.size() * sizeof(int32_t),
+                           cudaMemcpyHostToDevice, stream));
   CKC(c, cudaStreamSynchronize(stream));  // host vectors above are temporaries
   CKC(c, cudaStreamCreateWithFlags(&c->comm, cudaStreamNonBlocking));
   CKC(c, cudaStreamCreateWithFlags(&c->cap, cudaStreamNonBlocking));
@@ -808,6 +892,11 @@ mg_status mg_setup(const mg_params* p, int32_t rank, int32_t world_size, const u
       free_ctx(c);
       return s;
     }
+  }
+  s = fill_repl_tables(c);
+  if (s != MG_OK) {
+    free_ctx(c);
+    return s;
   }
   *out = c;
   return MG_OK;
@@ -1107,6 +1196,7 @@ mg_status mg_group_setup(const mg_params* p, int32_t world_size, int32_t device,
   }
   for (mg_ctx* c : g->r) {  // every rank's fields exist now: the cross-rank copy tables
     mg_status s = fill_copy_tables(c);
+    if (s == MG_OK) s = fill_repl_tables(c);
     if (s != MG_OK) {
       mg_group_destroy(g);
       return s;

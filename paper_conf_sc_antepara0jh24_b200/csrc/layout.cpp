@@ -269,6 +269,37 @@ mg_status build_layout(const mg_params& p, int rank, int world, Layout& out, std
     for (int l = 0; l < out.L; ++l)
       build_pair_tables(out.lv[l], p.sweep_kernel == 0 ? kPairMinBricks : min_b,
                         p.temporal_blocking == 2 ? 2 : p.temporal_blocking == 3 ? 3 : 1);
+  // replicated bottom: the global coarsest level as one rank would store it
+  const LevelLayout& B = out.lv[(size_t)out.L - 1];
+  out.repl = false;
+  if (out.L >= 2 && B.n_ghost > 0 && p.bottom_smooths > 0 && p.bottom_mode != MG_BOTTOM_SWEEPS) {
+    Layout g;
+    g.p = p;
+    for (int a = 0; a < 3; ++a) {
+      g.p.n_local[a] = p.n_local[a] * p.proc_grid[a];
+      g.p.proc_grid[a] = 1;
+    }
+    g.p.ghost_mode = MG_GHOST_AUTO;
+    g.L = out.L;
+    LevelLayout G;
+    build_level(g, out.L - 1, G);
+    if (G.n_owned <= kReplMaxBricks) {
+      out.gb = std::move(G);
+      const int nbx = B.nb[0], nby = B.nb[1], nbz = B.nb[2];
+      out.gb_src.assign((size_t)out.gb.n_owned, -1);
+      for (int64_t q = 0; q < out.gb.n_owned; ++q) {
+        const int X = out.gb.coord[(size_t)q * 3], Y = out.gb.coord[(size_t)q * 3 + 1], Z = out.gb.coord[(size_t)q * 3 + 2];
+        const int r = X / nbx + p.proc_grid[0] * (Y / nby + p.proc_grid[1] * (Z / nbz));
+        out.gb_src[(size_t)q] = (int32_t)(r * B.n_owned + B.ext_index(X % nbx, Y % nby, Z % nbz));
+      }
+      out.gb_mine.assign((size_t)B.n_owned, -1);
+      for (int64_t i = 0; i < B.n_owned; ++i)
+        out.gb_mine[(size_t)i] = (int32_t)out.gb.ext_index(B.coord[(size_t)i * 3] + out.coords[0] * nbx,
+                                                           B.coord[(size_t)i * 3 + 1] + out.coords[1] * nby,
+                                                           B.coord[(size_t)i * 3 + 2] + out.coords[2] * nbz);
+      out.repl = true;
+    }
+  }
   return MG_OK;
 }
 

@@ -125,12 +125,23 @@ constexpr int64_t kColMinBricks = 16384;  // levels smaller than this use the on
 constexpr int64_t kPairMinBricks = 4096;
 void build_col_tables(LevelLayout& L, int64_t min_bricks);
 
+// Replicated bottom: when the coarsest level has a ghost shell (decomposed, or self-exchange) and
+// the global coarsest grid is small, every rank gathers the owned b bricks of all ranks and runs the
+// bottom sweeps on the whole periodic coarsest grid itself -- the same per-cell expressions on the
+// same values as the decomposed sweeps, without the ghost exchange every 8 sweeps (the
+// bottom's communication dominates).
+constexpr int64_t kReplMaxBricks = 64;  // global coarsest bricks (the cluster solve's capacity)
+
 struct Layout {
   mg_params p{};
   int rank = 0, world = 1;
   int coords[3] = {0, 0, 0};
   int L = 0;
   std::vector<LevelLayout> lv;
+  bool repl = false;             // replicated bottom in use
+  LevelLayout gb;                // the global coarsest level (one rank: periodic wrap, no ghosts)
+  std::vector<int32_t> gb_src;   // [gb.n_owned] source of each global brick: rank * n_owned + owned index
+  std::vector<int32_t> gb_mine;  // [n_owned of the coarsest level] global index of each owned brick
 };
 
 // Validates params and builds every level.  Returns MG_OK or an error with msg.

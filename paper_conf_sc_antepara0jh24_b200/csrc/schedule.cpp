@@ -153,6 +153,7 @@ void Builder::phase(int l, int n, bool zero_first, int last, bool interp_first, 
 
 void Builder::exchange_b(int l) {
   if (!ghosts(l)) return;
+  if (lay.repl && l == lay.L - 1) return;  // the replicated bottom gathers owned b only
   Op o;
   o.kind = OP_EXCH;
   o.level = l;
@@ -195,6 +196,19 @@ void Builder::interp_op(int l) {
 
 void Builder::bottom(int l, int n, bool zero) {
   if (n <= 0) return;
+  if (lay.repl && l == lay.L - 1 && zero && fusion(l) != MG_FUSION_PAPER) {  // replicated bottom
+    Op o;
+    o.kind = OP_BOTTOM_REPL;
+    o.level = l;
+    o.src = st[l].cur;
+    o.dst = 1 - st[l].cur;
+    o.n = n;
+    o.timer = MG_OP_BOTTOM;
+    ops.push_back(o);
+    st[l].cur = o.dst;
+    st[l].dx = 0;  // ghosts not filled: the interpolation reads owned coarse bricks only
+    return;
+  }
   const LevelLayout& L = lay.lv[l];
   const int bm = lay.p.bottom_mode;
   const bool can_res = !ghosts(l) && L.n_stored <= kResidentMaxBricks;
@@ -333,6 +347,8 @@ int64_t op_launches(const Op& o, const Layout& lay, bool overlap, bool pencil_ov
     case OP_RESTRICT:
     case OP_INTERP:
     case OP_ZERO:
+    case OP_BOTTOM_REPL:
+      return 3;  // gather copies, the solve, the scatter copies (+ an all-gather on NCCL)
     case OP_BOTTOM_RES:
     case OP_COARSE:
       return 1;
