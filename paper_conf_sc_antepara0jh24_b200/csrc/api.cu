@@ -231,7 +231,7 @@ size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double**
     r.x[1] = (double*)take(gfb);
     r.b = (double*)take(gfb);
     r.adj = (int32_t*)take((size_t)lay.gb.n_stored * 8 * sizeof(int32_t));
-    r.gbuf = lay.world > 1 ? (double*)take((size_t)lay.world * nown * kBV * sizeof(double)) : nullptr;
+    r.gbuf = (double*)take((size_t)lay.world * nown * kBV * sizeof(double));
     r.gather = (CopyRun*)take((size_t)lay.gb.n_owned * sizeof(CopyRun));
     r.scatter = (CopyRun*)take((size_t)2 * nown * sizeof(CopyRun));
     if (rp) *rp = r;
@@ -308,7 +308,7 @@ mg_status fill_repl_tables(mg_ctx* c) {
   const int lb = lay.L - 1;
   const int64_t nown = lay.lv[(size_t)lb].n_owned;
   const size_t bb = (size_t)kBV;
-  c->rp.allgather = c->use_nccl && lay.world > 1;
+  c->rp.allgather = c->use_nccl;  // (a one-rank NCCL run too: the self-exchange tests cover the path)
   std::vector<CopyRun> g((size_t)lay.gb.n_owned), sc((size_t)2 * nown);
   for (int64_t q = 0; q < lay.gb.n_owned; ++q) {
     const int32_t src = lay.gb_src[(size_t)q];

@@ -515,18 +515,20 @@ def test_temporal_blocking_on_off_bitwise(oracle_mod, tb):
     m.close()
 
 
-@pytest.mark.parametrize("mode", ["loopback", "self"])
+@pytest.mark.parametrize("mode", ["loopback", "self-local", "self-nccl"])
 def test_pencil_exchange_overlap_bitwise(oracle_mod, mode, monkeypatch):
     """Pencil passes on ghost-shell levels with the exchange overlapped (MG_PENCIL_OVERLAP=1: the
     units that read no ghost brick run while the exchange fills the ghosts, the rest after it):
-    oracle bits for a 2x2x2 loopback decomposition and for the self-exchanged ghost shell."""
+    oracle bits for a 2x2x2 loopback decomposition and for the self-exchanged ghost shell over local
+    copies and over NCCL (send/recv on the comm stream inside the captured graph; the replicated
+    bottom's ncclAllGather)."""
     monkeypatch.setenv("MG_PENCIL_OVERLAP", "1")
     mg, solver = _mg()
-    if mode == "self":
+    if mode.startswith("self"):
         shape = (128, 128, 128)
         b = mg_inputs.random_rhs(shape, 37)
         xs, ns = oracle_cycles(oracle_mod, b, 4, 2)
-        m = new(shape, 4, ghost_mode=1, ca_period=8)
+        m = new(shape, 4, ghost_mode=1, ca_period=8, transport=1 if mode == "self-nccl" else 2)
         m.set_rhs(dev(b))
         m.set_solution(None)
         check_cycles(m, xs, ns)
