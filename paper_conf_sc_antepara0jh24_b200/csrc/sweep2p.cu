@@ -372,7 +372,8 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
       step(c, I1{}, P0{}, false, true);
       step(c, I2{}, P0{}, false, true);
       step(c, I3{}, P0{}, false, true);
-    } else {
+    } else {  // COOL: plane 0 of the layer above (sweep 1), the run's last plane (sweep 2)
+      static_assert(COOL == 2, "chunk type codes (layout.cpp pencil_table)");
       step(c, I0{}, P1{}, false, true);
     }
   }
