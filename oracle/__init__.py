@@ -61,6 +61,9 @@ def _load():
             "oracle_chebyshev_gamma": (D, [D, I, I, I]),
             "oracle_gsrb_half": (None, [I, I, I, D, I, P, P, P, P]),
             "oracle_mg_set_smoother": (None, [P, I, I]),
+            "oracle_mg_set_bottom_solver": (None, [P, I]),
+            "oracle_dot_tree": (D, [S, P, P]),
+            "oracle_cg": (None, [I, I, I, D, I, P, P]),
             "oracle_smooth_residual": (None, [S, D, P, P, P, P]),
             "oracle_restriction": (None, [I, I, I, P, P]),
             "oracle_init_zero": (None, [S, P]),
@@ -154,6 +157,22 @@ def chebyshev_gamma(h: float, s: int, k: int, rho: int) -> float:
     return float(_load().oracle_chebyshev_gamma(float(h), int(s), int(k), int(rho)))
 
 
+def dot_tree(a: np.ndarray, b: np.ndarray) -> float:
+    """Fixed-order dot product of reading A21 (stride-doubling pairwise tree, lexicographic)."""
+    a, b = _f64(a), _f64(b)
+    assert a.size == b.size
+    return float(_load().oracle_dot_tree(a.size, _ptr(a), _ptr(b)))
+
+
+def cg(b: np.ndarray, h: float, iters: int) -> np.ndarray:
+    """`iters` CG iterations on A x = b from x = 0 (reading A21, the CG bottom variant)."""
+    b = _f64(b)
+    x = np.zeros_like(b)
+    nz, ny, nx = b.shape
+    _load().oracle_cg(nx, ny, nz, h, int(iters), _ptr(x), _ptr(b))
+    return x
+
+
 def restriction(r: np.ndarray) -> np.ndarray:
     r = _f64(r)
     nz, ny, nx = r.shape
@@ -193,7 +212,7 @@ class OracleMG:
     """Alg 1 / Alg 2 on a global periodic grid of shape (nz, ny, nx)."""
 
     def __init__(self, shape, levels: int, pre: int = 12, post: int = 12, bottom: int = 100, h0: float | None = None,
-                 smoother: int = 0, cheby_ratio: int = 6):
+                 smoother: int = 0, cheby_ratio: int = 6, bottom_solver: int = 0):
         nz, ny, nx = (int(s) for s in shape)
         self.shape = (nz, ny, nx)
         self.levels = int(levels)
@@ -203,6 +222,7 @@ class OracleMG:
         if not self._h:
             raise ValueError(f"oracle_mg_create failed for shape={shape} levels={levels}")
         self._lib.oracle_mg_set_smoother(self._h, int(smoother), int(cheby_ratio))
+        self._lib.oracle_mg_set_bottom_solver(self._h, int(bottom_solver))
 
     def close(self):
         if getattr(self, "_h", None):

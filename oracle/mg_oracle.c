@@ -25,6 +25,11 @@
  *   Chebyshev smoother    variant (N4, reading A19): per-sweep steps gamma_k, see
  *                         oracle_chebyshev_gamma; pinned by the Chebyshev-polynomial
  *                         error factor on eigenmodes (tests/test_oracle_pins.py)
+ *   CG bottom solver      variant (N4 "other bottom solvers", reading A21): `bottom`
+ *                         iterations of conjugate gradients on A x = b from x = 0 with a
+ *                         fixed-order (stride-doubling pairwise tree, lexicographic) dot
+ *                         product, oracle_cg / oracle_dot_tree; pinned by Krylov optimality
+ *                         against a dense projection and by finite termination
  *
  * Readings of garbled / silent passages:
  *   - expression order (A8): neighbour sum pairwise by axis
@@ -199,6 +204,62 @@ double oracle_max_norm_residual(int nx, int ny, int nz, double h, const double *
   return m;
 }
 
+/* Fixed-order dot product (reading A21): v_i = a_i * b_i over the lexicographic index, then for
+ * s = 1, 2, 4, ...: v_i = v_i + v_{i+s} for every i that is a multiple of 2s with i + s < n; the
+ * result is v_0 (a pairwise tree; every operation separately rounded).  Sequential (test oracle). */
+double oracle_dot_tree(size_t n, const double *a, const double *b) {
+  if (n == 0) return 0.0;
+  double *v = (double *)malloc(n * sizeof(double));
+  if (!v) return NAN;
+  for (size_t i = 0; i < n; ++i) v[i] = a[i] * b[i];
+  for (size_t s = 1; s < n; s *= 2)
+    for (size_t i = 0; i + s < n; i += 2 * s) v[i] = v[i] + v[i + s];
+  const double d = v[0];
+  free(v);
+  return d;
+}
+
+/* CG bottom solver (variant, reading A21; SURVEY §8(f) N4 "other bottom solvers"; the paper's
+ * bottom is `bottom` smooths): `iters` iterations of unpreconditioned conjugate
+ * gradients on A x = b (A = the level's applyOp, symmetric negative semi-definite on the periodic
+ * grid; b of zero mean) from x = 0:
+ *   r = b;  p = r;  rr = <r, r>
+ *   repeat iters times:  q = A p;  d = <p, q>;  if d == 0: stop
+ *                        alpha = rr / d;  x = x + alpha p;  r = r - alpha q
+ *                        rr' = <r, r>;  beta = rr' / rr;  p = r + beta p;  rr = rr'
+ * <.,.> = oracle_dot_tree; every operation separately rounded (CG's formulas hold for a definite
+ * operator of either sign: alpha < 0 here). */
+void oracle_cg(int nx, int ny, int nz, double h, int iters, double *x, const double *b) {
+  const size_t n = (size_t)nx * ny * nz;
+  double *r = (double *)malloc(n * sizeof(double)), *p = (double *)malloc(n * sizeof(double));
+  double *q = (double *)malloc(n * sizeof(double));
+  if (!r || !p || !q) {
+    free(r), free(p), free(q);
+    return;
+  }
+  for (size_t i = 0; i < n; ++i) {
+    x[i] = 0.0;
+    r[i] = b[i];
+    p[i] = b[i];
+  }
+  double rr = oracle_dot_tree(n, r, r);
+  for (int it = 0; it < iters; ++it) {
+    oracle_apply_op(nx, ny, nz, h, p, q);
+    const double d = oracle_dot_tree(n, p, q);
+    if (d == 0.0) break;
+    const double alpha = rr / d;
+    for (size_t i = 0; i < n; ++i) {
+      x[i] = x[i] + alpha * p[i];
+      r[i] = r[i] - alpha * q[i];
+    }
+    const double rr2 = oracle_dot_tree(n, r, r);
+    const double beta = rr2 / rr;
+    for (size_t i = 0; i < n; ++i) p[i] = r[i] + beta * p[i];
+    rr = rr2;
+  }
+  free(r), free(p), free(q);
+}
+
 /* ---------------------------------------------------------------------------
  * V-cycle hierarchy (Alg 2)
  * ------------------------------------------------------------------------- */
@@ -207,6 +268,7 @@ typedef struct {
   int L, pre, post, bottom;
   int smoother, rho; /* 0 = damped Jacobi (the paper); 1 = Chebyshev (oracle_chebyshev_gamma) on pre/post;
                         2 = red-black Gauss-Seidel on pre/post (oracle_gsrb_half: red then black) */
+  int bottom_solver;  /* 0 = `bottom` damped Jacobi smooths (the paper); 1 = `bottom` CG iterations (oracle_cg) */
   int n[ORACLE_MAX_LEVELS][3];
   double h[ORACLE_MAX_LEVELS];
   double *x[ORACLE_MAX_LEVELS], *b[ORACLE_MAX_LEVELS], *Ax[ORACLE_MAX_LEVELS], *r[ORACLE_MAX_LEVELS];
@@ -262,6 +324,7 @@ void oracle_mg_set_smoother(oracle_mg *m, int smoother, int rho) {
   m->smoother = smoother;
   m->rho = rho;
 }
+void oracle_mg_set_bottom_solver(oracle_mg *m, int solver) { m->bottom_solver = solver; }
 
 /* step of sweep it of n at level l (pre / post smoothing) */
 static double step_gamma(const oracle_mg *m, int l, int n, int it) {
@@ -306,6 +369,9 @@ void oracle_mg_vcycle(oracle_mg *m) {
   {                                                             /* steps 10-15: bottom */
     const int l = L - 1;
     const int *n = m->n[l];
+    if (m->bottom_solver == 1) /* reading A21: x = 0 (initZero) and `bottom` CG iterations */
+      oracle_cg(n[0], n[1], n[2], m->h[l], m->bottom, m->x[l], m->b[l]);
+    else
     for (int it = 0; it < m->bottom; ++it) {
       oracle_apply_op(n[0], n[1], n[2], m->h[l], m->x[l], m->Ax[l]);
       oracle_smooth(lvl_n(m, l), m->h[l], m->x[l], m->Ax[l], m->b[l]);

@@ -451,3 +451,95 @@ def test_gsrb_vcycle_converges_faster(oracle_mod):
         norms.append(mg.norm())
     rg = float(np.exp(np.mean(np.log([norms[c] / norms[c - 1] for c in range(2, 7)]))))
     assert rg < rj, (rg, rj)
+
+
+# ------------------------------------------------ CG bottom solver (N4 variant, reading A21)
+def test_dot_tree_order_and_accuracy(oracle_mod):
+    """The fixed-order dot product: exact on integer-valued data (any n, powers of two or not), within
+    the pairwise-summation bound of the exactly rounded sum (math.fsum) on random data, and
+    dependent on the order it states: a value whose sum cancels only in the pairwise pairing."""
+    import math
+    rng = np.random.default_rng(3)
+    for n in (1, 2, 3, 7, 8, 100, 512, 4096, 4097):
+        a = rng.integers(-50, 50, n).astype(np.float64)
+        b = rng.integers(-50, 50, n).astype(np.float64)
+        assert oracle_mod.dot_tree(a, b) == float(np.dot(a.astype(np.int64), b.astype(np.int64)))
+        a, b = rng.standard_normal(n), rng.standard_normal(n)
+        exact = math.fsum(a * b)
+        bound = (math.ceil(math.log2(max(n, 2))) + 1) * 2.0**-53 * float(np.sum(np.abs(a * b)))
+        assert abs(oracle_mod.dot_tree(a, b) - exact) <= bound
+    # the tree pairs (v0 + v1) + (v2 + v3) = (1e16 + 1) + (-1e16 + 1) = 1e16 + (-1e16) = 0 (each
+    # inner sum rounds the 1 away); left to right gives 1.0
+    v = np.array([1e16, 1.0, -1e16, 1.0])
+    assert oracle_mod.dot_tree(v, np.ones(4)) == 0.0
+    assert ((1e16 + 1.0) + -1e16) + 1.0 == 1.0
+
+
+def _fft_solution(b, h):
+    """Exact solution of the periodic discrete Poisson problem A x = b (zero-mean x) by the FFT."""
+    nz, ny, nx = b.shape
+    s = [np.sin(np.pi * np.arange(n) / n) ** 2 for n in (nz, ny, nx)]
+    lam = -(4.0 / h**2) * (s[0][:, None, None] + s[1][None, :, None] + s[2][None, None, :])
+    bh = np.fft.fftn(b)
+    lam[0, 0, 0] = 1.0
+    xh = bh / lam
+    xh[0, 0, 0] = 0.0
+    return np.real(np.fft.ifftn(xh))
+
+
+def test_cg_is_krylov_optimal(oracle_mod):
+    """CG's k-th iterate is the A-orthogonal (Galerkin) projection of the solution onto the Krylov
+    space span{b, Ab, ..., A^(k-1) b}: computed independently with the Kronecker-sum matrix and a QR
+    basis of the Krylov vectors, for k = 1..5 on a non-cubic grid."""
+    shape, h = (8, 16, 8), 1.0 / 16
+    b = mg_inputs.random_rhs(shape, 11)
+    A = kron_laplacian(shape, h).toarray()
+    K = [b.ravel()]
+    for k in range(1, 6):
+        V, _ = np.linalg.qr(np.stack(K, axis=1))
+        y = np.linalg.solve(V.T @ A @ V, V.T @ b.ravel())
+        want = V @ y
+        got = oracle_mod.cg(b, h, k).ravel()
+        assert np.abs(got - want).max() <= 1e-9 * np.abs(want).max(), k
+        K.append(A @ K[-1])
+
+
+def test_cg_converges_to_the_discrete_solution(oracle_mod):
+    """The A-norm error of the CG iterates decreases monotonically and 100 iterations reach the
+    exact discrete solution (FFT) on an 8x16x16 grid to 1e-7 relative (the coarsest grids the CG
+    bottom is built for have <= 4096 cells)."""
+    shape, h = (8, 16, 16), 1.0 / 16
+    b = mg_inputs.random_rhs(shape, 12)
+    xs = _fft_solution(b, h)
+    A = kron_laplacian(shape, h)
+    errs = []
+    for k in (2, 5, 10, 20, 40):
+        e = (oracle_mod.cg(b, h, k) - xs).ravel()
+        errs.append(float(-(e @ (A @ e))))  # -A is positive semi-definite
+    assert all(errs[i + 1] < errs[i] for i in range(len(errs) - 1)), errs
+    x = oracle_mod.cg(b, h, 100)
+    assert np.abs((x - x.mean()) - xs).max() <= 1e-7 * np.abs(xs).max()
+
+
+def test_cg_bottom_vcycle_contracts_faster_with_a_large_coarsest_grid(oracle_mod):
+    """With a 32^3 coarsest grid, 100 Jacobi smooths barely reduce the coarse error (survey: rho ~
+    0.36 per V-cycle), 100 CG iterations solve it: the CG-bottom V-cycle contracts much faster.
+    bottom_solver = 0 is the paper's cycle bit for bit."""
+    N, L = 64, 2
+    b = mg_inputs.sin_rhs((N, N, N))
+
+    def rho(**kw):
+        m = oracle_mod.OracleMG((N, N, N), L, **kw)
+        m.set_b(b)
+        m.set_x(None)
+        norms = [m.norm()]
+        for _ in range(4):
+            m.vcycle()
+            norms.append(m.norm())
+        return float(np.exp(np.mean(np.log([norms[c] / norms[c - 1] for c in range(2, 5)])))), m
+
+    rj, mj = rho()
+    rc, _ = rho(bottom_solver=1)
+    assert rj > 0.2 and rc < 0.1, (rj, rc)
+    r0, m0 = rho(bottom_solver=0)
+    assert np.array_equal(m0.get_x(), mj.get_x())
