@@ -56,6 +56,7 @@ def parse():
                     help="0 damped Jacobi (the paper), 1 Chebyshev, 2 red-black Gauss-Seidel (N4 variants)")
     ap.add_argument("--cheby-ratio", type=int, default=0, help="Chebyshev smoothing interval [mu_max/ratio, mu_max]")
     ap.add_argument("--no-pdl", action="store_true", help="launch kernels without programmatic dependent launch")
+    ap.add_argument("--bottom-solver", type=int, default=0, help="0 Jacobi smooths (the paper), 1 CG (variant)")
     ap.add_argument("--bottom-mode", type=int, default=0,
                     help="0 auto, 1 per-sweep launches, 2 resident bottom, 3 cluster coarse solve, 4 grid coarse solve")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -249,7 +250,7 @@ def main():
                   ghost_mode=1 if a.ghost_all else 0, use_graph=not a.no_graph, overlap=not a.no_overlap,
                   rank=rank, world_size=world, device=local, temporal_blocking=a.tb, smoother=a.smoother,
                   cheby_ratio=a.cheby_ratio, launch_pdl=2 if a.no_pdl else 0,
-                  bottom_mode=a.bottom_mode)
+                  bottom_mode=a.bottom_mode, bottom_solver=a.bottom_solver)
     gshape = (n * pg[2], n * pg[1], n * pg[0])
     b_host = torch.from_numpy(mg_inputs.local_sin_rhs(gshape, rank, pg)).pin_memory()
     b_dev = b_host.to(dev)
@@ -369,6 +370,7 @@ def main():
                        "cuda_graph": not a.no_graph, "overlap": not a.no_overlap, "pdl": not a.no_pdl,
                        "coarse": {0: "auto", 1: "per-sweep launches", 2: "resident bottom", 3: "cluster solve",
                                   4: "grid solve"}[a.bottom_mode],
+                       "bottom_solver": "conjugate gradients" if a.bottom_solver else "damped jacobi (paper)",
                        "temporal_blocking": {0: "off", 1: "one-brick CTA streams", 2: "warp plane streams"}.get(
                            a.tb, "2x2-brick pencils"),
                        "smoother": {1: "chebyshev", 2: "red-black gauss-seidel"}.get(a.smoother, "damped jacobi (paper)"),

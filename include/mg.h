@@ -127,7 +127,11 @@ typedef struct {
                                     1 = on, 2 = off.  A kernel's CTAs may be scheduled while the previous
                                     kernel of the stream drains; each waits for it before touching memory
                                     (griddepcontrol), so results are bitwise unchanged */
-  int32_t reserved[2];
+  int32_t bottom_solver;         /* 0 = `bottom_smooths` damped-Jacobi smooths (the paper);
+                                    1 = `bottom_smooths` conjugate-gradient iterations from x = 0 with a
+                                    fixed-order dot product (variant N4, reading A21; needs a
+                                    coarsest grid of <= 8 bricks, globally when decomposed) */
+  int32_t reserved[1];
   double h0;                     /* finest spacing; <= 0 => 1 / max_d(global N_d) (reading A7) */
 } mg_params;
 

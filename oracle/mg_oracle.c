@@ -220,15 +220,18 @@ double oracle_dot_tree(size_t n, const double *a, const double *b) {
 }
 
 /* CG bottom solver (variant, reading A21; SURVEY §8(f) N4 "other bottom solvers"; the paper's
- * bottom is `bottom` smooths): `iters` iterations of unpreconditioned conjugate
- * gradients on A x = b (A = the level's applyOp, symmetric negative semi-definite on the periodic
- * grid; b of zero mean) from x = 0:
- *   r = b;  p = r;  rr = <r, r>
- *   repeat iters times:  q = A p;  d = <p, q>;  if d == 0: stop
- *                        alpha = rr / d;  x = x + alpha p;  r = r - alpha q
- *                        rr' = <r, r>;  beta = rr' / rr;  p = r + beta p;  rr = rr'
- * <.,.> = oracle_dot_tree; every operation separately rounded (CG's formulas hold for a definite
- * operator of either sign: alpha < 0 here). */
+ * bottom is `bottom` smooths): at most `iters` iterations of unpreconditioned
+ * conjugate gradients on A x = b - m from x = 0.  A = the level's applyOp is symmetric negative
+ * semi-definite on the periodic grid with the constants as null space (reading A12), so CG runs on
+ * the consistent system: m = <b, 1> / N removes b's mean (rounding leaves a tiny one after the
+ * restrictions; left in, CG divides by p.Ap ~ 0 once the rest has converged and blows x up):
+ *   r = b - m;  p = r;  rr0 = rr = <r, r>
+ *   repeat:  q = A p;  d = <p, q>;  if not d < 0: stop            (breakdown / converged)
+ *            alpha = rr / d;  x = x + alpha p;  r = r - alpha q;  rr' = <r, r>
+ *            if rr' <= 1e-24 rr0: stop                               (relative residual 1e-12)
+ *            beta = rr' / rr;  p = r + beta p;  rr = rr'
+ * <.,.> = oracle_dot_tree (<b, 1> sums b itself); every operation separately rounded (CG's
+ * formulas hold for a definite operator of either sign: alpha < 0 here). */
 void oracle_cg(int nx, int ny, int nz, double h, int iters, double *x, const double *b) {
   const size_t n = (size_t)nx * ny * nz;
   double *r = (double *)malloc(n * sizeof(double)), *p = (double *)malloc(n * sizeof(double));
@@ -237,22 +240,26 @@ void oracle_cg(int nx, int ny, int nz, double h, int iters, double *x, const dou
     free(r), free(p), free(q);
     return;
   }
+  for (size_t i = 0; i < n; ++i) q[i] = 1.0;
+  const double m = oracle_dot_tree(n, b, q) / (double)n;
   for (size_t i = 0; i < n; ++i) {
     x[i] = 0.0;
-    r[i] = b[i];
-    p[i] = b[i];
+    r[i] = b[i] - m;
+    p[i] = r[i];
   }
   double rr = oracle_dot_tree(n, r, r);
+  const double rr0 = rr;
   for (int it = 0; it < iters; ++it) {
     oracle_apply_op(nx, ny, nz, h, p, q);
     const double d = oracle_dot_tree(n, p, q);
-    if (d == 0.0) break;
+    if (!(d < 0.0)) break;
     const double alpha = rr / d;
     for (size_t i = 0; i < n; ++i) {
       x[i] = x[i] + alpha * p[i];
       r[i] = r[i] - alpha * q[i];
     }
     const double rr2 = oracle_dot_tree(n, r, r);
+    if (rr2 <= 1e-24 * rr0) break;
     const double beta = rr2 / rr;
     for (size_t i = 0; i < n; ++i) p[i] = r[i] + beta * p[i];
     rr = rr2;

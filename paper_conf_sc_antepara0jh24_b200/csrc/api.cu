@@ -115,6 +115,7 @@ struct mg_ctx {
     double* x[2] = {nullptr, nullptr};
     double* b = nullptr;
     int32_t* adj = nullptr;
+    int32_t* coord = nullptr;  // global brick coords (the CG bottom's lexicographic order)
     double* gbuf = nullptr;  // all-gather landing buffer [world][n_owned bricks] (NCCL)
     CopyRun* gather = nullptr;
     CopyRun* scatter = nullptr;  // [2][n_owned]: into x[0] / x[1] of the coarsest level
@@ -231,6 +232,7 @@ size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double**
     r.x[1] = (double*)take(gfb);
     r.b = (double*)take(gfb);
     r.adj = (int32_t*)take((size_t)lay.gb.n_stored * 8 * sizeof(int32_t));
+    r.coord = (int32_t*)take((size_t)lay.gb.n_stored * 3 * sizeof(int32_t));
     r.gbuf = (double*)take((size_t)lay.world * nown * kBV * sizeof(double));
     r.gather = (CopyRun*)take((size_t)lay.gb.n_owned * sizeof(CopyRun));
     r.scatter = (CopyRun*)take((size_t)2 * nown * sizeof(CopyRun));
@@ -262,6 +264,8 @@ mg_status check_params(const mg_params& p) {
   if (p.transport < 0 || p.transport > MG_TRANSPORT_LOCAL) return set_err(MG_ERR_INVALID_ARG, "bad transport");
   if (p.bottom_mode < 0 || p.bottom_mode > MG_BOTTOM_GRID) return set_err(MG_ERR_INVALID_ARG, "bad bottom_mode");
   if (p.launch_pdl < 0 || p.launch_pdl > 2) return set_err(MG_ERR_INVALID_ARG, "launch_pdl must be 0, 1 or 2");
+  if (p.bottom_solver < 0 || p.bottom_solver > 1)
+    return set_err(MG_ERR_INVALID_ARG, "bottom_solver must be 0 (Jacobi smooths) or 1 (CG)");
   if (p.smoother < 0 || p.smoother > 2)
     return set_err(MG_ERR_INVALID_ARG, "smoother must be 0 (Jacobi), 1 (Chebyshev) or 2 (red-black Gauss-Seidel)");
   return MG_OK;
@@ -543,7 +547,10 @@ mg_status exec_op(mg_ctx* c, const Op& o, cudaStream_t s) {
       if (c->rp.allgather)
         CKN(c, ncclAllGather(d.b, c->rp.gbuf, (size_t)L.n_owned * kBV, ncclFloat64, c->nccl, s));
       CKC(c, launch_copy_runs(c->rp.gather, (int)ng, kBV, s));
-      if (ng <= kResidentMaxBricks) {
+      if (lay.p.bottom_solver == 1) {
+        CKC(c, launch_bottom_cg(c->rp.x[1], c->rp.b, c->rp.adj, c->rp.coord, (int)ng, lay.gb.n[0], lay.gb.n[1], o.n,
+                                d.c, s));
+      } else if (ng <= kResidentMaxBricks) {
         CKC(c, launch_bottom_resident(c->rp.x[0], c->rp.x[1], c->rp.b, c->rp.adj, (int)ng, o.n, true, d.c, s));
       } else {
         CoarseArgs a{};
@@ -559,6 +566,11 @@ mg_status exec_op(mg_ctx* c, const Op& o, cudaStream_t s) {
       CKS(timer_end(c, s, t0, o.level, o.timer));
       return MG_OK;
     }
+    case OP_BOTTOM_CG:
+      CKS(timer_begin(c, s, &t0));
+      CKC(c, launch_bottom_cg(d.x[o.dst], d.b, d.adj, d.coord, (int)L.n_owned, L.n[0], L.n[1], o.n, d.c, s));
+      CKS(timer_end(c, s, t0, o.level, o.timer));
+      return MG_OK;
     case OP_BOTTOM_RES:
       CKS(timer_begin(c, s, &t0));
       CKC(c, launch_bottom_resident(d.x[o.src], d.x[o.dst], d.b, d.adj, (int)L.n_stored, o.n, o.zero, d.c, s));
@@ -726,9 +738,12 @@ mg_status init_ctx(mg_ctx* c, const mg_params& p, int rank, int world, int devic
         CKC(c, encode_pencil_maps(d.x[xb], d.b, L.n_alloc, &d.nmaps[xb]));
       }
   }
-  if (c->lay.repl)
+  if (c->lay.repl) {
     CKC(c, cudaMemcpyAsync(c->rp.adj, c->lay.gb.adj.data(), c->lay.gb.adj.size() * sizeof(int32_t),
                            cudaMemcpyHostToDevice, stream));
+    CKC(c, cudaMemcpyAsync(c->rp.coord, c->lay.gb.coord.data(), c->lay.gb.coord.size() * sizeof(int32_t),
+                           cudaMemcpyHostToDevice, stream));
+  }
   CKC(c, cudaStreamSynchronize(stream));  // host vectors above are temporaries
   CKC(c, cudaStreamCreateWithFlags(&c->comm, cudaStreamNonBlocking));
   CKC(c, cudaStreamCreateWithFlags(&c->cap, cudaStreamNonBlocking));

@@ -687,6 +687,8 @@ cudaError_t kernels_init() {
   if (e != cudaSuccess) return e;
   e = coarse_kernels_init();
   if (e != cudaSuccess) return e;
+  e = cg_kernels_init();
+  if (e != cudaSuccess) return e;
   return coarse_grid_init();
 }
 

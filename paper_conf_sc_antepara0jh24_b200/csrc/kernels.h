@@ -189,6 +189,12 @@ cudaError_t coarse_grid_init();
 cudaError_t launch_coarse(const CoarseArgs& a, cudaStream_t s);
 cudaError_t coarse_kernels_init();
 cudaError_t kernels_init();  // one-time attribute setup
+// CG bottom solver (cg.cu, variant: reading A21): `iters` CG iterations on A x = b from x = 0 on the
+// coarsest level (no ghosts, <= kResidentMaxBricks bricks, one CTA); coord = brick coords [nb][3],
+// nx, ny = cells per axis (the lexicographic order of the fixed-order dot product).
+cudaError_t launch_bottom_cg(double* xo, const double* b, const int32_t* adj, const int32_t* coord, int nbricks,
+                             int nx, int ny, int iters, Coeffs c, cudaStream_t s);
+cudaError_t cg_kernels_init();
 
 // Programmatic dependent launch for every kernel the library enqueues: set by the
 // API from mg_params.launch_pdl before it enqueues or captures work.  The kernels begin with

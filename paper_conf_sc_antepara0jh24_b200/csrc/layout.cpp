@@ -300,6 +300,14 @@ mg_status build_layout(const mg_params& p, int rank, int world, Layout& out, std
       out.repl = true;
     }
   }
+  if (p.bottom_solver == 1) {  // CG bottom (reading A21): one CTA holds the whole coarsest grid
+    const int64_t nb = out.repl ? out.gb.n_owned : (B.n_ghost > 0 ? -1 : B.n_owned);
+    if (nb < 0 || nb > 8) {
+      msg = "bottom_solver = 1 (CG) needs a coarsest grid of <= 8 bricks (globally when decomposed), "
+            "without bottom_mode = sweeps on a ghost-shell level";
+      return MG_ERR_INVALID_ARG;
+    }
+  }
   return MG_OK;
 }
 

@@ -196,7 +196,21 @@ void Builder::interp_op(int l) {
 
 void Builder::bottom(int l, int n, bool zero) {
   if (n <= 0) return;
-  if (lay.repl && l == lay.L - 1 && zero && fusion(l) != MG_FUSION_PAPER) {  // replicated bottom
+  if (lay.p.bottom_solver == 1 && !(lay.repl && l == lay.L - 1)) {  // CG bottom (reading A21), from x = 0
+    Op o;
+    o.kind = OP_BOTTOM_CG;
+    o.level = l;
+    o.src = st[l].cur;
+    o.dst = 1 - st[l].cur;
+    o.n = n;
+    o.timer = MG_OP_BOTTOM;
+    ops.push_back(o);
+    st[l].cur = o.dst;
+    st[l].dx = 0;
+    return;
+  }
+  if (lay.repl && l == lay.L - 1 && (zero || lay.p.bottom_solver == 1) && fusion(l) != MG_FUSION_PAPER) {
+    // replicated bottom
     Op o;
     o.kind = OP_BOTTOM_REPL;
     o.level = l;
@@ -237,6 +251,7 @@ int Builder::coarse_start() const {
   const int bm = lay.p.bottom_mode;
   // opt-in: measured slower than graph-replayed per-level launches below 512^3
   if (L < 2 || (bm != MG_BOTTOM_CLUSTER && bm != MG_BOTTOM_GRID)) return -1;
+  if (lay.p.bottom_solver != 0) return -1;  // their bottoms are Jacobi smooths
   if (lay.p.pre_smooths < 1) return -1;
   if (lay.p.smoother == 1 && (lay.p.pre_smooths > kCoarseMaxCheb || lay.p.post_smooths > kCoarseMaxCheb)) return -1;
   if (lay.p.smoother == 2) return -1;  // red-black half-sweeps: per-level kernels only
@@ -348,7 +363,9 @@ int64_t op_launches(const Op& o, const Layout& lay, bool overlap, bool pencil_ov
     case OP_INTERP:
     case OP_ZERO:
     case OP_BOTTOM_REPL:
-      return 3;  // gather copies, the solve, the scatter copies (+ an all-gather on NCCL)
+      return 3;
+    case OP_BOTTOM_CG:
+      return 1;  // gather copies, the solve, the scatter copies (+ an all-gather on NCCL)
     case OP_BOTTOM_RES:
     case OP_COARSE:
       return 1;

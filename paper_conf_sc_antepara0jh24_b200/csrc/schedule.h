@@ -17,7 +17,8 @@
 namespace mgb {
 
 enum OpKind { OP_SWEEP = 0, OP_RESTRICT, OP_INTERP, OP_ZERO, OP_EXCH, OP_BOTTOM_RES, OP_SWEEP2, OP_COARSE,
-              OP_BOTTOM_REPL };
+              OP_BOTTOM_REPL, OP_BOTTOM_CG };
+// OP_BOTTOM_CG: `n` CG iterations from x = 0 on the (ghost-free) coarsest level into buffer `dst`.
 // OP_BOTTOM_REPL: the replicated bottom (Layout::repl): all-gather the owned b bricks of the
 // coarsest level, `n` sweeps from x = 0 on the global coarsest grid, owned x into buffer `dst`.
 // OP_COARSE: levels `level` .. L-1 of the cycle in one cluster launch (coarse.cu); x of `level`

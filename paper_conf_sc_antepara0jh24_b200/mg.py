@@ -51,7 +51,8 @@ class mg_params(ctypes.Structure):
         ("smoother", ctypes.c_int32),
         ("cheby_ratio", ctypes.c_int32),
         ("launch_pdl", ctypes.c_int32),
-        ("reserved", ctypes.c_int32 * 2),
+        ("bottom_solver", ctypes.c_int32),
+        ("reserved", ctypes.c_int32 * 1),
         ("h0", ctypes.c_double),
     ]
 
@@ -149,7 +150,7 @@ def check(status: int, where: str) -> int:
 
 def params(n_local, proc_grid=(1, 1, 1), num_levels=6, pre=12, post=12, bottom=100, ca_period=None, fusion=None,
            ghost_mode=MG_GHOST_AUTO, transport=MG_TRANSPORT_AUTO, use_graph=1, bottom_mode=MG_BOTTOM_AUTO,
-           overlap=1, h0=0.0, sweep_kernel=0, temporal_blocking=3, smoother=0, cheby_ratio=0, launch_pdl=0) -> mg_params:
+           overlap=1, h0=0.0, sweep_kernel=0, temporal_blocking=3, smoother=0, cheby_ratio=0, launch_pdl=0, bottom_solver=0) -> mg_params:
     p = mg_params()
     lib().mg_params_default(ctypes.byref(p))
     p.n_local[:] = [int(v) for v in n_local]
@@ -166,6 +167,7 @@ def params(n_local, proc_grid=(1, 1, 1), num_levels=6, pre=12, post=12, bottom=1
     p.temporal_blocking = int(temporal_blocking)
     p.smoother, p.cheby_ratio = int(smoother), int(cheby_ratio)
     p.launch_pdl = int(launch_pdl)
+    p.bottom_solver = int(bottom_solver)
     return p
 
 

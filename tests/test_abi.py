@@ -81,7 +81,7 @@ def test_workspace_bytes_scales_with_levels():
     assert b > a and a >= 5 * 64**3 * 8
 
 
-@pytest.mark.parametrize("bad", [dict(smoother=3), dict(launch_pdl=3), dict(smoother=-1), dict(bottom_mode=5), dict(transport=7),
+@pytest.mark.parametrize("bad", [dict(smoother=3), dict(launch_pdl=3), dict(bottom_solver=2), dict(smoother=-1), dict(bottom_mode=5), dict(transport=7),
                                  dict(num_levels=2, pre=0)])
 def test_invalid_parameters_are_rejected_without_a_gpu(bad):
     """Parameter validation (mg_workspace_bytes, the first call of a setup) rejects unknown

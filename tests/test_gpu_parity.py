@@ -515,6 +515,53 @@ def test_temporal_blocking_on_off_bitwise(oracle_mod, tb):
     m.close()
 
 
+@pytest.mark.parametrize("shape,L,pre,post,bottom", [
+    ((64, 64, 64), 4, 12, 12, 100),   # coarsest 8^3: one brick
+    ((128, 128, 128), 4, 12, 12, 100),  # coarsest 16^3: 8 bricks, the paper's bottom size
+    ((24, 16, 8), 1, 0, 0, 37),       # bottom only, 6 bricks: a non-power-of-two dot-product length
+    ((64, 32, 16), 2, 3, 2, 60),      # non-cubic, 8 bricks
+])
+def test_cg_bottom_vcycle_bitwise(oracle_mod, shape, L, pre, post, bottom):
+    """bottom_solver = 1: CG bottom (reading A21) from x = 0 with the fixed-order dot product, bit for
+    bit with the oracle's CG V-cycle (2 cycles)."""
+    b = mg_inputs.random_rhs(shape, 43)
+    orc = oracle_mod.OracleMG(shape, L, pre, post, bottom, bottom_solver=1)
+    orc.set_b(b)
+    orc.set_x(None)
+    xs, ns = [], []
+    for _ in range(2):
+        orc.vcycle()
+        xs.append(orc.get_x())
+        ns.append(orc.norm())
+    m = new(shape, L, pre=pre, post=post, bottom=bottom, bottom_solver=1)
+    m.set_rhs(dev(b))
+    m.set_solution(None)
+    check_cycles(m, xs, ns)
+    m.close()
+
+
+def test_cg_bottom_replicated_loopback_bitwise(oracle_mod):
+    """CG bottom on the replicated global coarsest grid of a 2x2x2 loopback decomposition (8^3 per
+    rank: 16^3 globally, 8 bricks), bit for bit with the undecomposed oracle."""
+    _, solver = _mg()
+    pg, n_local, L = (2, 2, 2), (32, 32, 32), 3
+    gshape = (n_local[2] * pg[2], n_local[1] * pg[1], n_local[0] * pg[0])
+    b = mg_inputs.random_rhs(gshape, 44)
+    orc = oracle_mod.OracleMG(gshape, L, bottom_solver=1)
+    orc.set_b(b)
+    orc.set_x(None)
+    g = solver.LoopbackGroup(n_local, pg, num_levels=L, bottom_solver=1)
+    g.set_rhs([dev(mg_inputs.local_block(b, r, pg)) for r in range(g.world_size)])
+    g.set_solution(None)
+    for c in range(2):
+        orc.vcycle()
+        g.vcycle()
+        assert g.residual_norm() == orc.norm()
+        for r in range(g.world_size):
+            assert_bitwise(host(g.get_solution(r)), mg_inputs.local_block(orc.get_x(), r, pg), what=f"rank {r}")
+    g.close()
+
+
 @pytest.mark.parametrize("mode", ["loopback", "self-local", "self-nccl"])
 def test_pencil_exchange_overlap_bitwise(oracle_mod, mode, monkeypatch):
     """Pencil passes on ghost-shell levels with the exchange overlapped (MG_PENCIL_OVERLAP=1: the

@@ -178,6 +178,12 @@ def test_invalid_params_rejected():
     p = mg.params((32, 32, 32), num_levels=2, ca_period=9)
     with pytest.raises(mg.MGError):
         mg.Layout(p, 0, 1)
+    # CG bottom (reading A21) needs a coarsest grid of <= 8 bricks (here 64, and 64 globally)
+    for pg in ((1, 1, 1), (2, 2, 2)):
+        p = mg.params((64, 64, 64), pg, num_levels=2, bottom_solver=1)
+        with pytest.raises(mg.MGError):
+            mg.Layout(p, 0, pg[0] * pg[1] * pg[2])
+    mg.Layout(mg.params((64, 64, 64), num_levels=4, bottom_solver=1), 0, 1)  # 8^3 coarsest: accepted
 
 
 # ------------------------------------------------- two-sweep pencil plans (sweep2p.cu, kind 3)

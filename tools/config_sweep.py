@@ -106,6 +106,7 @@ def main():
     out.append(run("c3_fusion", 512, 6, solve=True))
     out.append(run("c3_fusion", 512, 6, solve=True, smoother=1))
     out.append(run("c3_fusion", 512, 6, solve=True, smoother=2))
+    out.append(run("c3_fusion", 512, 6, solve=True, bottom_solver=1))
     # config 5 at P = 1: 1024^3, L = 7 (global coarsest 16^3)
     if not a.quick:
         out.append(run("c5", 1024, 7, cycles=3))
