@@ -17,6 +17,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstdint>
 
 #include <cudaTypedefs.h>
@@ -558,9 +559,41 @@ __global__ void __launch_bounds__(256) interp_kernel(double* __restrict__ x, con
   *px = v;
 }
 
+// the same, four fine bricks per CTA (one per 64-thread quarter, 8 cells per thread): all loads of
+// a thread (parent, coarse value, four 16-byte x pieces) are issued before its adds and stores, so
+// more bytes are in flight per thread; stores stream past L1 (the next pass re-reads x from HBM)
+__global__ void __launch_bounds__(256) interp4_kernel(double* __restrict__ x, const double* __restrict__ xc,
+                                                      const int32_t* __restrict__ parent, int64_t nfine) {
+  pdl_begin();
+  const int t = threadIdx.x, qb = t >> 6, u = t & 63;
+  const int64_t f = (int64_t)blockIdx.x * 4 + qb;
+  if (f >= nfine) return;
+  // pieces e = u + 64 m, m = 0..3: the double2 at cells 2e, 2e + 1 of the brick (one coarse cell)
+  const int pr = __ldg(parent + f);
+  double2* px = reinterpret_cast<double2*>(x + f * 512);
+  double2 v[4];
+  double cv[4];
+#pragma unroll
+  for (int m = 0; m < 4; ++m) {
+    const int e = u + 64 * m, c = 2 * e, i0 = c & 7, j = (c >> 3) & 7, k = c >> 6;
+    v[m] = px[e];
+    cv[m] = __ldg(xc + (int64_t)(pr >> 3) * 512 + coarse_off(pr & 7, i0, j, k));
+  }
+#pragma unroll
+  for (int m = 0; m < 4; ++m) {
+    v[m].x = DADD(v[m].x, cv[m]);
+    v[m].y = DADD(v[m].y, cv[m]);
+    st_stream2(x + f * 512 + 2 * (u + 64 * m), v[m]);
+  }
+}
+
 cudaError_t launch_interp(double* x, const double* xc, const int32_t* parent, int64_t nfine, cudaStream_t s) {
   if (nfine <= 0) return cudaSuccess;
-  launch_k(interp_kernel, (unsigned)nfine, 256, 0, s, x, xc, parent);
+  static const bool one = getenv("MG_INTERP1") != nullptr;  // (measurement switch: one brick per CTA)
+  if (one)
+    launch_k(interp_kernel, (unsigned)nfine, 256, 0, s, x, xc, parent);
+  else
+    launch_k(interp4_kernel, (unsigned)((nfine + 3) / 4), 256, 0, s, x, xc, parent, nfine);
   return cudaGetLastError();
 }
 
