@@ -543,3 +543,31 @@ def test_cg_bottom_vcycle_contracts_faster_with_a_large_coarsest_grid(oracle_mod
     assert rj > 0.2 and rc < 0.1, (rj, rc)
     r0, m0 = rho(bottom_solver=0)
     assert np.array_equal(m0.get_x(), mj.get_x())
+
+
+def test_cg_solves_the_consistent_system(oracle_mod):
+    """The periodic operator annihilates constants (reading A12), so CG runs on b - mean(b) (reading
+    A21): a constant added to b changes nothing beyond rounding, and the converged residual is b's
+    mean (b - A x = mean(b) to 1e-10 relative)."""
+    shape, h = (16, 16, 8), 1.0 / 16
+    b = mg_inputs.random_rhs(shape, 13)
+    x0 = oracle_mod.cg(b, h, 100)
+    x1 = oracle_mod.cg(b + 0.25, h, 100)
+    assert np.abs(x1 - x0).max() <= 1e-10 * np.abs(x0).max()
+    r = (b + 0.25) - oracle_mod.apply_op(x1, h)
+    assert np.abs(r - 0.25).max() <= 1e-10 * np.abs(b).max()
+
+
+def test_cg_bottom_vcycle_converges_with_a_16_cube_bottom(oracle_mod):
+    """128^3, L = 4 (the paper's 16^3 coarsest): the CG-bottom V-cycle contracts every cycle down to
+    the paper's tolerance (with b's rounding-level mean left in CG, this cycle diverged)."""
+    N = 128
+    m = oracle_mod.OracleMG((N, N, N), 4, bottom_solver=1)
+    m.set_b(mg_inputs.sin_rhs((N, N, N)))
+    m.set_x(None)
+    norms = [m.norm()]
+    for _ in range(7):
+        m.vcycle()
+        norms.append(m.norm())
+    assert all(norms[c + 1] < 0.2 * norms[c] for c in range(len(norms) - 1)), norms
+    assert norms[-1] < 1e-10

@@ -2,7 +2,7 @@
 
 Applies one plausible slip at a time to oracle/mg_oracle.c, rebuilds, runs
 tests/test_oracle_pins.py and reports whether some pin catches it.  The
-source is restored afterwards.  Last run: every mutation below CAUGHT.
+source is restored afterwards.  Last run: every mutation below CAUGHT (12 of 12).
 """
 import os
 import subprocess
@@ -20,6 +20,14 @@ MUTATIONS = {
     "dropped_neighbour": ("(xb + xt)", "(xb + xb)"),
     "residual_sign": ("r[p] = b[p] - Ax[p];", "r[p] = Ax[p] - b[p];"),
     "bottom_without_smooth": ("      oracle_smooth(lvl_n(m, l), m->h[l], m->x[l], m->Ax[l], m->b[l]);", ""),
+    # CG bottom variant (reading A21)
+    "cg_beta_inverted": ("const double beta = rr2 / rr;", "const double beta = rr / rr2;"),
+    "cg_residual_sign": ("r[i] = r[i] - alpha * q[i];", "r[i] = r[i] + alpha * q[i];"),
+    "cg_mean_not_removed": ("r[i] = b[i] - m;", "r[i] = b[i];"),
+    "dot_tree_left_to_right": ("for (size_t i = 0; i + s < n; i += 2 * s) v[i] = v[i] + v[i + s];",
+                               "for (size_t i = 0; i + s < n; i += 2 * s) v[i] = v[i] + v[i + s];\n"
+                               "  if (n > 1) { double t = v[0]; v[0] = a[0] * b[0];"
+                               " for (size_t i = 1; i < n; ++i) v[0] = v[0] + a[i] * b[i]; (void)t; }"),
 }
 
 
