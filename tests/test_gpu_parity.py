@@ -384,6 +384,54 @@ def test_full_size_512_vcycle_bitwise(oracle_mod):
     m.close()
 
 
+@pytest.mark.parametrize("pg", [(2, 1, 1), (2, 2, 1), (2, 2, 2)])
+def test_config5_1024_decomposition_invariant(pg):
+    """Config 5 at its full size (1024^3 total, L = 7, global coarsest 16^3 for every P): one V-cycle on
+    one rank and on the P = 2 / 4 / 8 loopback decompositions (down to 512^3 per rank: ghost shells,
+    local exchanges
+    through the NCCL plans, pencil passes over the stored box, the replicated bottom) give bit-identical
+    x and the same residual norm (decomposition invariance; the oracle's own cycle at this
+    size is checked by the 512^3 tests and the invariance chain)."""
+    import torch
+
+    _, solver = _mg()
+    torch.cuda.empty_cache()  # (the previous case's cached blocks)
+    G = (1024, 1024, 1024)
+    P = pg[0] * pg[1] * pg[2]
+    nl = (1024 // pg[0], 1024 // pg[1], 1024 // pg[2])  # (nx, ny, nz) per rank
+    blocks = [torch.from_numpy(mg_inputs.local_sin_rhs(G, r, pg)) for r in range(P)]
+
+    def sl(r):
+        cx, cy, cz = mg_inputs.rank_coords(r, pg)
+        return (slice(cz * nl[2], (cz + 1) * nl[2]), slice(cy * nl[1], (cy + 1) * nl[1]),
+                slice(cx * nl[0], (cx + 1) * nl[0]))
+
+    b = torch.empty(G, dtype=torch.float64, device="cuda")
+    for r, blk in enumerate(blocks):
+        b[sl(r)] = blk.cuda()
+    m = new(G, 7)
+    m.set_rhs(b)
+    m.set_solution(None)
+    m.vcycle()
+    n1 = m.residual_norm()
+    x1 = m.get_solution()
+    m.close()
+    del b
+    torch.cuda.empty_cache()
+    g = solver.LoopbackGroup(nl, pg, num_levels=7)
+    g.set_rhs([blk.cuda() for blk in blocks])
+    g.set_solution(None)
+    g.vcycle()
+    assert g.residual_norm() == n1
+    try:
+        for r in range(P):
+            assert torch.equal(g.get_solution(r), x1[sl(r)]), f"rank {r}"
+    finally:
+        g.close()
+        del g, x1
+        torch.cuda.empty_cache()
+
+
 # ------------------------------------------------- streaming (column) kernel
 @pytest.mark.parametrize("tb", [0, 1, 2, 3])
 @pytest.mark.parametrize("fusion", [2, 3])
