@@ -276,6 +276,13 @@ mg_status mg_layout_parent(const mg_layout* lay, int32_t level, int32_t* out);
 mg_status mg_layout_plan(const mg_layout* lay, int32_t level, int32_t which /*0 send,1 recv*/, int64_t* out);
 mg_status mg_layout_pass_plan(const mg_layout* lay, int32_t level, int32_t idx, int64_t info[6], int32_t* meta,
                               int32_t* ctas);
+/* Replicated bottom (the coarsest level has a ghost shell and the global coarsest grid <= 64
+ * bricks): info[0] = global coarsest bricks (0: not replicated), info[1] = this rank's owned
+ * coarsest bricks; gb_src int32 [info[0]] = rank * info[1] + owned index of the brick each global
+ * brick is gathered from (the all-gather's rank-major order), gb_mine int32 [info[1]] = the global
+ * brick of each owned brick, gb_adj int32 [info[0]][8] = the global level's adjacency (periodic
+ * wrap).  Any array may be NULL. */
+mg_status mg_layout_repl(const mg_layout* lay, int64_t info[2], int32_t* gb_src, int32_t* gb_mine, int32_t* gb_adj);
 mg_status mg_layout_destroy(mg_layout* lay);
 
 #ifdef __cplusplus

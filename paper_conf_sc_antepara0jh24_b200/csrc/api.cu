@@ -1333,6 +1333,18 @@ mg_status mg_layout_level_info(const mg_layout* m, int32_t level, int64_t info[1
   return MG_OK;
 }
 
+mg_status mg_layout_repl(const mg_layout* m, int64_t info[2], int32_t* gb_src, int32_t* gb_mine, int32_t* gb_adj) {
+  if (!m || !info) return set_err(MG_ERR_INVALID_ARG, "null argument");
+  const Layout& lay = m->lay;
+  info[0] = lay.repl ? lay.gb.n_owned : 0;
+  info[1] = lay.lv[(size_t)lay.L - 1].n_owned;
+  if (!lay.repl) return MG_OK;
+  if (gb_src) std::copy(lay.gb_src.begin(), lay.gb_src.end(), gb_src);
+  if (gb_mine) std::copy(lay.gb_mine.begin(), lay.gb_mine.end(), gb_mine);
+  if (gb_adj) std::copy(lay.gb.adj.begin(), lay.gb.adj.end(), gb_adj);
+  return MG_OK;
+}
+
 mg_status mg_layout_adjacency(const mg_layout* m, int32_t level, int32_t* out) {
   const LevelLayout* L = nullptr;
   CKS(lay_level(m, level, &L));

@@ -114,6 +114,8 @@ _SIGS = {
     "mg_layout_plan": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32, ctypes.c_void_p]),
     "mg_layout_pass_plan": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32, ctypes.c_void_p,
                                            ctypes.c_void_p, ctypes.c_void_p]),
+    "mg_layout_repl": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
+                                      ctypes.c_void_p]),
     "mg_layout_destroy": (ctypes.c_int, [ctypes.c_void_p]),
 }
 
@@ -365,6 +367,19 @@ class Layout:
         v = list(buf)
         return {"n": v[0:3], "nb": v[3:6], "ghost": v[6:9], "owned": v[9], "interior": v[10], "nghost": v[11],
                 "alloc": v[12], "send_runs": v[13], "recv_runs": v[14], "zero_brick": v[15]}
+
+    def repl(self):
+        """Replicated bottom maps: None, or (gb_src, gb_mine, gb_adj) (see mg_layout_repl)."""
+        np = self._np
+        info = (ctypes.c_int64 * 2)()
+        check(lib().mg_layout_repl(self.h, info, None, None, None), "mg_layout_repl")
+        if info[0] == 0:
+            return None
+        src = np.zeros(info[0], dtype=np.int32)
+        mine = np.zeros(info[1], dtype=np.int32)
+        adj = np.zeros((info[0], 8), dtype=np.int32)
+        check(lib().mg_layout_repl(self.h, info, src.ctypes.data, mine.ctypes.data, adj.ctypes.data), "mg_layout_repl")
+        return src, mine, adj
 
     def adjacency(self, level):
         inf = self.info(level)

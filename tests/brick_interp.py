@@ -111,10 +111,23 @@ def exchange_local(fields, levels):
     return out
 
 
-def vcycle_ranks(xs, bs, ranks, L, h0, pre, post, bottom, exchange=exchange_local):
+def replicated_bottom(b_own, gathered_fn, src, mine, gadj, h, bottom):
+    """The library's replicated bottom (Layout::repl): all-gather the owned coarsest b bricks
+    (rank-major), permute them into the global coarsest level by `src`, `bottom` sweeps from x = 0 on
+    that periodic grid, this rank's owned x by `mine`.  gathered_fn(b_own) -> [world * n_own] bricks."""
+    gb = gathered_fn(b_own)[src]
+    ng = len(src)
+    x = np.zeros((ng, 8, 8, 8))
+    for _ in range(bottom):
+        x, _ = sweep(x, gb, gadj, ng, h)
+    return x[mine]
+
+
+def vcycle_ranks(xs, bs, ranks, L, h0, pre, post, bottom, exchange=exchange_local, bottom_fn=None):
     """One V-cycle (Alg 2) over every rank's brick fields.  ranks[r][l] = RankLevel.
     xs, bs: per-rank lists of per-level arrays (level-0 b must already hold valid ghosts).
-    `exchange(fields, levels)` fills ghost bricks (in-process or over torch.distributed)."""
+    `exchange(fields, levels)` fills ghost bricks (in-process or over torch.distributed).
+    bottom_fn(xs, bs, h) (optional) replaces the exchanged bottom sweeps."""
     R = len(ranks)
     own = lambda r, l: ranks[r][l].n_owned  # noqa: E731
     rs = [[None] * L for _ in range(R)]
@@ -132,6 +145,9 @@ def vcycle_ranks(xs, bs, ranks, L, h0, pre, post, bottom, exchange=exchange_loca
         for r in range(R):
             bs[r][l + 1] = bl[r]
     h = h0 * 2 ** (L - 1)
+    if bottom_fn is not None:
+        bottom_fn(xs, bs, h)
+        bottom = 0
     for s in range(bottom):
         xl = exchange([xs[r][L - 1] for r in range(R)], [ranks[r][L - 1] for r in range(R)])
         for r in range(R):

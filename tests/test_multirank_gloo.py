@@ -24,7 +24,7 @@ def _free_port():
     return port
 
 
-def _worker(rank, world, port, n_local, pg, L, out_dir):
+def _worker(rank, world, port, n_local, pg, L, out_dir, replicated):
     import sys
 
     sys.path.insert(0, ROOT)
@@ -68,18 +68,36 @@ def _worker(rank, world, port, n_local, pg, L, out_dir):
         xs = [[levels[l].zeros() for l in range(L)]]
         bs = [[None] * L]
         bs[0][0] = exchange([levels[0].to_bricks(mg_inputs.local_block(b, rank, pg))], [levels[0]])[0]
-        xs = bi.vcycle_ranks(xs, bs, [levels], L, h0, 2, 2, 10, exchange=exchange)
+        rep = lay.repl()
+        assert rep is not None  # decomposed coarsest level with a ghost shell, tiny global grid
+
+        def gathered(b_own):  # the all-gather the library does with ncclAllGather, rank-major
+            n_own = b_own.shape[0]
+            parts = [torch.empty(n_own * 512, dtype=torch.float64) for _ in range(world)]
+            dist.all_gather(parts, torch.from_numpy(np.ascontiguousarray(b_own).ravel()))
+            return torch.cat(parts).numpy().reshape(world * n_own, 8, 8, 8)
+
+        def bottom_fn(xs_, bs_, h):
+            n_own = levels[L - 1].n_owned
+            xs_[0][L - 1][:n_own] = bi.replicated_bottom(bs_[0][L - 1][:n_own], gathered, rep[0], rep[1], rep[2], h, 10)
+
+        xs = bi.vcycle_ranks(xs, bs, [levels], L, h0, 2, 2, 10, exchange=exchange,
+                             bottom_fn=bottom_fn if replicated else None)
         np.save(os.path.join(out_dir, f"x{rank}.npy"), levels[0].from_bricks(xs[0][0]))
     finally:
         dist.destroy_process_group()
 
 
+@pytest.mark.parametrize("replicated", [False, True])
 @pytest.mark.parametrize("n_local,pg,L", [((16, 16, 16), (2, 1, 1), 2), ((16, 16, 16), (2, 2, 1), 2)])
-def test_gloo_multirank_vcycle_bitwise(oracle_mod, tmp_path, n_local, pg, L):
+def test_gloo_multirank_vcycle_bitwise(oracle_mod, tmp_path, n_local, pg, L, replicated):
+    """Per-rank layouts and plans from the C ABI, real gloo point-to-point exchanges, the bottom either
+    swept with ghost exchanges or replicated as the library does it (all-gather of the owned coarsest
+    b over gloo, the library's gather / scatter maps and global adjacency): the oracle's bits."""
     import mg_inputs
 
     world = pg[0] * pg[1] * pg[2]
-    mp.start_processes(_worker, args=(world, _free_port(), n_local, pg, L, str(tmp_path)), nprocs=world,
+    mp.start_processes(_worker, args=(world, _free_port(), n_local, pg, L, str(tmp_path), replicated), nprocs=world,
                        join=True, start_method="spawn")
     gshape = (n_local[2] * pg[2], n_local[1] * pg[1], n_local[0] * pg[0])
     b = mg_inputs.random_rhs(gshape, 11)
