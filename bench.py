@@ -352,6 +352,20 @@ def main():
         te = max_over_ranks((time.perf_counter() - t0) * 1e3)
         e2e = {"value": world * n**3 * ke / (te / 1e3), "unit": "DOF/s", "h2d_bytes_per_step": int(b_host.numel() * 8),
                "d2h_bytes_per_step": 8, "steps": ke, "ms_per_step": te / ke}
+        # (informational) the same metric over whole solves through mg_solve (Alg 1): one upload of b
+        # per solve, V-cycles until max|b - Ax| < 1e-10 with the norm read back after every cycle
+        ks, cyc_tot = 3, 0
+        barrier()
+        t0 = time.perf_counter()
+        for _ in range(ks):
+            m.set_rhs_host(b_host)
+            m.set_solution(None)
+            _, cyc, _ = m.solve(1e-10, 20)
+            cyc_tot += cyc
+        ts = max_over_ranks((time.perf_counter() - t0) * 1e3)
+        e2e["solve"] = {"value": world * n**3 * cyc_tot / (ts / 1e3), "unit": "DOF/s", "solves": ks,
+                        "vcycles_per_solve": cyc_tot / ks, "ms_per_solve": ts / ks,
+                        "h2d_bytes_per_solve": int(b_host.numel() * 8)}
 
     launches = m.launches_per_vcycle()
     xbytes, xmsgs = m.exchange_stats()
