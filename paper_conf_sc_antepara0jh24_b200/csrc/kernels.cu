@@ -403,7 +403,8 @@ cudaError_t launch_sweep_col(const SweepArgs& a, const ColArgs& c, const FaceMap
   return cudaGetLastError();
 }
 
-cudaError_t encode_box_map(const double* base, int64_t n_alloc, const unsigned box[3], CUtensorMap* out) {
+cudaError_t encode_box_map(const double* base, int64_t n_alloc, const unsigned box[3], CUtensorMap* out,
+                           bool swizzle64) {
   static PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
   if (!encode) {
     void* fn = nullptr;
@@ -418,7 +419,8 @@ cudaError_t encode_box_map(const double* base, int64_t n_alloc, const unsigned b
   const cuuint32_t estr[3] = {1, 1, 1};
   const cuuint32_t bx[3] = {box[0], box[1], box[2]};
   const CUresult r = encode(out, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, const_cast<double*>(base), dims, strides, bx,
-                            estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                            estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                            swizzle64 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_NONE,
                             CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
 }

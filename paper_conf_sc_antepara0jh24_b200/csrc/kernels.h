@@ -62,7 +62,8 @@ struct FaceMaps {
 cudaError_t encode_face_maps(const double* x, int64_t n_alloc, FaceMaps* out);
 // One TMA tensor map over a brick field seen as [n_alloc*8 planes][8 j][8 i]
 // doubles with the given box {i, j, planes}.
-cudaError_t encode_box_map(const double* base, int64_t n_alloc, const unsigned box[3], CUtensorMap* out);
+cudaError_t encode_box_map(const double* base, int64_t n_alloc, const unsigned box[3], CUtensorMap* out,
+                           bool swizzle64 = false);  // swizzle64: 16-byte chunk c of row r lands at chunk c ^ ((r >> 1) & 3)
 
 // Two-sweep (temporally blocked) streaming kernel, sweep2.cu.
 struct PairArgs {
@@ -80,6 +81,7 @@ struct PairMaps {
   CUtensorMap xcor;  // x boxes {2,1,8}: the four diagonal-corner columns
   CUtensorMap bwe;   // b boxes {2,8,8}
   CUtensorMap bsn;   // b boxes {8,1,8}
+  CUtensorMap xown;  // pencil kernel: x boxes {8,8,4} (an own brick's half), 64-byte swizzle
 };
 cudaError_t encode_pair_maps(const double* x, const double* b, int64_t n_alloc, PairMaps* out);
 // flags apply to the SECOND sweep of the pair: plain, +r, +restriction
