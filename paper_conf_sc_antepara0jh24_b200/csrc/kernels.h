@@ -81,7 +81,6 @@ struct PairMaps {
   CUtensorMap xcor;  // x boxes {2,1,8}: the four diagonal-corner columns
   CUtensorMap bwe;   // b boxes {2,8,8}
   CUtensorMap bsn;   // b boxes {8,1,8}
-  CUtensorMap xown;  // pencil kernel: x boxes {8,8,4} (an own brick's half), 64-byte swizzle
 };
 cudaError_t encode_pair_maps(const double* x, const double* b, int64_t n_alloc, PairMaps* out);
 // flags apply to the SECOND sweep of the pair: plain, +r, +restriction
