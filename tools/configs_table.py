@@ -21,6 +21,8 @@ def desc(r):
         parts.append(f"s={r['pre']}")
     if r.get("smoother") in (1, 2):
         parts.append({1: "Chebyshev smoother", 2: "red-black Gauss-Seidel smoother"}[r["smoother"]])
+    if r.get("bottom_solver") == 1:
+        parts.append("CG bottom")
     return ", ".join(parts)
 
 
