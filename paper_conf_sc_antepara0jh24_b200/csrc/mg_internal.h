@@ -120,8 +120,9 @@ void build_pair_tables(LevelLayout& L, int64_t min_bricks, int kind);
 constexpr int kColSeg = 16;             // bricks per streamed segment
 constexpr int64_t kColMinBricks = 16384;  // levels smaller than this use the one-brick-per-CTA kernel
 // two-sweep passes (auto kernel choice) from this level size on: at 512^3 levels 0-2 (level 2 =
-// 128^3, 4096 bricks: pencil passes 0.29 vs 0.43 ms of single sweeps per cycle; 512 bricks measured
-// no better in graph replay)
+// 128^3, 4096 bricks: pencil passes 0.29 vs 0.43 ms of single sweeps per cycle; pencil passes on
+// levels 3-4 too (512 / 64 bricks) measured 0.16 vs 0.19 ms instrumented at level 3 but within the
+// box noise in graph replay: 10.17-10.19 vs 10.12-10.22 ms)
 constexpr int64_t kPairMinBricks = 4096;
 void build_col_tables(LevelLayout& L, int64_t min_bricks);
 
