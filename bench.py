@@ -67,6 +67,14 @@ def parse():
     return ap.parse_args()
 
 
+def host_cores():
+    """Cores this process may run on (the oracle's OpenMP threads for the CPU legs)."""
+    try:
+        return len(os.sched_getaffinity(0))
+    except AttributeError:
+        return os.cpu_count() or 1
+
+
 def dist_env():
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -158,6 +166,7 @@ def oracle_dofs(n, levels, pre, post, bottom, seconds, min_cycles=1, max_cycles=
     import oracle
 
     oracle.build()
+    oracle.set_threads(host_cores())  # the host's cores (torchrun sets OMP_NUM_THREADS=1 per process)
     b = mg_inputs.sin_rhs((n, n, n))
     m = oracle.OracleMG((n, n, n), levels, pre, post, bottom)
     m.set_b(b)
@@ -196,6 +205,7 @@ def run_reference(a, rank, world):
     import oracle
 
     oracle.build()
+    oracle.set_threads(host_cores())
     n = a.ref_n or min(a.n, 256)
     lv = max(1, min(a.levels, (n // 8).bit_length()))
     import mg_inputs
