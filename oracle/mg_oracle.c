@@ -188,17 +188,27 @@ void oracle_interpolation_increment(int nx, int ny, int nz, const double *xc, do
 }
 
 /* maxNormRes (Alg 1): max over the domain of |b - Ax|, with a
- * fresh applyOp on the current x (reading A6). */
+ * fresh applyOp on the current x (reading A6).  A NaN anywhere makes the max NaN (a diverged
+ * iterate must not pass the 1e-10 test): each thread keeps a NaN once it saw one, and so does the
+ * combination of the threads' maxima. */
 double oracle_max_norm_residual(int nx, int ny, int nz, double h, const double *x, const double *b) {
   const size_t n = (size_t)nx * ny * nz;
   double *Ax = (double *)malloc(n * sizeof(double));
   if (!Ax) return NAN;
   oracle_apply_op(nx, ny, nz, h, x, Ax);
   double m = 0.0;
-#pragma omp parallel for schedule(static) reduction(max : m)
-  for (size_t p = 0; p < n; ++p) {
-    const double a = fabs(b[p] - Ax[p]);
-    if (a > m) m = a;
+#pragma omp parallel
+  {
+    double mt = 0.0;
+#pragma omp for schedule(static)
+    for (size_t p = 0; p < n; ++p) {
+      const double a = fabs(b[p] - Ax[p]);
+      if (a > mt || a != a) mt = a;
+    }
+#pragma omp critical
+    {
+      if (mt > m || mt != mt) m = mt;
+    }
   }
   free(Ax);
   return m;

@@ -196,33 +196,104 @@ def prolong_1d(nf):
     return P.tocsr()
 
 
-def matrix_vcycle(b0, x0, L, h0, pre, post, bottom):
+def chebyshev_steps(h, s, rho):
+    """The s steps of the Chebyshev smoother (reading A19) built from the textbook nodes, not from
+    the oracle's index formula: the reciprocals of the Chebyshev nodes of [mu_max/rho, mu_max]
+    (mu_max = 12/h^2), sorted ascending, then taken smallest, largest, second smallest, second
+    largest, ... (small and large steps interleaved)."""
+    mu_max = 12.0 / h**2
+    lo = mu_max / rho
+    nodes = [0.5 * (mu_max + lo) + 0.5 * (mu_max - lo) * np.cos(np.pi * (2 * j + 1) / (2 * s)) for j in range(s)]
+    asc = sorted(1.0 / mu for mu in nodes)
+    out, i, j = [], 0, s - 1
+    while i <= j:
+        out.append(asc[i])
+        i += 1
+        if i <= j:
+            out.append(asc[j])
+            j -= 1
+    return out
+
+
+def red_black_gs(A, shape):
+    """One Gauss-Seidel step in red-black ordering ((i+j+k) mod 2 = 0 first) as sparse matrices:
+    returns step(x, b) -> (x after the red half, x after both halves), the red half being the
+    exact solve of the red rows for the red unknowns with black fixed (the 7-point stencil couples
+    red only to black), the full step a sparse lower-triangular solve (D + L) x' = b - U x."""
+    import scipy.sparse.linalg as spla
+    nz, ny, nx = shape
+    K, J, I = np.meshgrid(np.arange(nz), np.arange(ny), np.arange(nx), indexing="ij")
+    colour = ((I + J + K) & 1).ravel()
+    perm = np.concatenate([np.flatnonzero(colour == 0), np.flatnonzero(colour == 1)])
+    nred = int(np.count_nonzero(colour == 0))
+    Ap = A.tocsr()[perm][:, perm]
+    lower = sp.tril(Ap, 0, format="csr")
+    upper = sp.triu(Ap, 1, format="csr")
+
+    def step(x, b):
+        y = spla.spsolve_triangular(lower, b[perm] - upper @ x[perm], lower=True)
+        full = np.empty_like(x)
+        full[perm] = y
+        half = x.copy()
+        half[perm[:nred]] = y[:nred]
+        return half, full
+
+    return step
+
+
+def matrix_vcycle(b0, x0, L, h0, pre, post, bottom, smoother=0, rho=6, bottom_solver=0):
     """Alg 2 written with SciPy sparse matrices: A_l Kronecker sum at h_l = 2^l h0,
     P_l = piecewise-constant prolongation, R_l = P_l^T / 8.  An independent
-    formulation (different summation order) of the same algorithm."""
+    formulation (different summation order) of the same algorithm.
+
+    Variants, each in its own matrix form:
+      smoother 1 (Chebyshev, reading A19): the pre / post sweeps of a level take the steps of
+        `chebyshev_steps(h_l, pre|post, rho)` in order; the restricted residual is the lagged one of
+        the last sweep (A5);
+      smoother 2 (GSRB, reading A20): each sweep is one red-black ordered Gauss-Seidel step (sparse
+        triangular solve); the restricted residual is b - A x of the x after the last red half;
+      bottom_solver 1 (CG, reading A21): the coarsest problem solved exactly, x = A^+ (b - mean b)
+        (dense pseudo-inverse; CG from x = 0 converges to it on the tiny coarsest grids used here).
+    The bottom of the smoother variants stays damped Jacobi."""
     shapes = [tuple(s >> l for s in b0.shape) for l in range(L)]
-    A = [kron_laplacian(shapes[l], h0 * 2**l) for l in range(L)]
+    hs = [h0 * 2**l for l in range(L)]
+    A = [kron_laplacian(shapes[l], hs[l]) for l in range(L)]
     P = [sp.kron(prolong_1d(shapes[l][0]), sp.kron(prolong_1d(shapes[l][1]), prolong_1d(shapes[l][2]))).tocsr()
          for l in range(L - 1)]
-    g = [(h0 * 2**l) ** 2 / 12.0 for l in range(L)]
+    g = [hs[l] ** 2 / 12.0 for l in range(L)]
+    gs = [red_black_gs(A[l], shapes[l]) for l in range(L - 1)] if smoother == 2 else None
+
+    def smooth(l, n):
+        """n sweeps at level l; returns the residual the last one writes."""
+        steps = chebyshev_steps(hs[l], n, rho) if smoother == 1 else [g[l]] * n
+        r = None
+        for it in range(n):
+            if smoother == 2:
+                half, x[l] = gs[l](x[l], b[l])
+                r = b[l] - A[l] @ half
+                continue
+            Ax = A[l] @ x[l]
+            r = b[l] - Ax
+            x[l] = x[l] + steps[it] * (Ax - b[l])
+        return r
+
     x = [None] * L
     b = [None] * L
     x[0], b[0] = x0.ravel().copy(), b0.ravel().copy()
     for l in range(L - 1):
-        for _ in range(pre):
-            Ax = A[l] @ x[l]
-            r = b[l] - Ax
-            x[l] = x[l] + g[l] * (Ax - b[l])
+        r = smooth(l, pre)
         b[l + 1] = (P[l].T @ r) / 8.0
         x[l + 1] = np.zeros_like(b[l + 1])
-    for _ in range(bottom):
-        Ax = A[L - 1] @ x[L - 1]
-        x[L - 1] = x[L - 1] + g[L - 1] * (Ax - b[L - 1])
+    if bottom_solver == 1:
+        bb = b[L - 1] - b[L - 1].mean()
+        x[L - 1] = np.linalg.pinv(A[L - 1].toarray()) @ bb
+    else:
+        for _ in range(bottom):
+            Ax = A[L - 1] @ x[L - 1]
+            x[L - 1] = x[L - 1] + g[L - 1] * (Ax - b[L - 1])
     for l in range(L - 2, -1, -1):
         x[l] = x[l] + P[l] @ x[l + 1]
-        for _ in range(post):
-            Ax = A[l] @ x[l]
-            x[l] = x[l] + g[l] * (Ax - b[l])
+        smooth(l, post)
     return x[0].reshape(b0.shape)
 
 
@@ -243,6 +314,66 @@ def test_vcycle_matches_sparse_matrix_vcycle(oracle_mod, shape, L, sweeps):
         xm = matrix_vcycle(b, xm, L, h0, pre, post, bottom)
         xo = mg.get_x()
         assert np.abs(xo - xm).max() <= 1e-12 * np.abs(xm).max()
+
+
+@pytest.mark.parametrize("smoother,shape,L,sweeps", [
+    (1, (16, 32, 24), 3, (5, 3, 20)),   # Chebyshev, pre != post
+    (1, (16, 16, 32), 2, (2, 7, 10)),
+    (2, (16, 32, 24), 3, (3, 2, 20)),   # red-black Gauss-Seidel, pre != post
+    (2, (8, 16, 16), 2, (1, 4, 10)),
+])
+def test_variant_vcycle_matches_sparse_matrix_vcycle(oracle_mod, smoother, shape, L, sweeps):
+    """The smoother variants' V-cycles (readings A19, A20) equal the sparse-matrix V-cycle written
+    with the textbook Chebyshev nodes resp. a red-black ordered Gauss-Seidel triangular solve, after 1
+    and 2 cycles, on non-cubic grids with pre != post: a swapped colour order, a reversed or
+    mis-counted step list, or the wrong lagged residual fails."""
+    pre, post, bottom = sweeps
+    h0 = mg_inputs.default_h0(shape)
+    b = mg_inputs.random_rhs(shape, 1)
+    mg = oracle_mod.OracleMG(shape, L, pre, post, bottom, h0, smoother=smoother, cheby_ratio=6)
+    mg.set_b(b)
+    mg.set_x(None)
+    xm = np.zeros(shape)
+    for _ in range(2):
+        mg.vcycle()
+        xm = matrix_vcycle(b, xm, L, h0, pre, post, bottom, smoother=smoother, rho=6)
+        xo = mg.get_x()
+        assert np.abs(xo - xm).max() <= 1e-11 * np.abs(xm).max()
+
+
+@pytest.mark.parametrize("shape,L", [((16, 32, 24), 3), ((16, 16, 16), 3)])
+def test_cg_bottom_vcycle_matches_matrix_vcycle_with_exact_bottom(oracle_mod, shape, L):
+    """The CG-bottom V-cycle (reading A21) equals the matrix V-cycle whose coarsest problem is solved
+    exactly (pseudo-inverse of the consistent system): 100 CG iterations from x = 0 on a <= 4x8x6
+    coarsest grid reach the discrete solution (finite termination), so a wrong start, a skipped mean
+    removal or a bottom that is not the CG solve fails."""
+    pre, post, bottom = 3, 4, 100
+    h0 = mg_inputs.default_h0(shape)
+    b = mg_inputs.random_rhs(shape, 2)
+    mg = oracle_mod.OracleMG(shape, L, pre, post, bottom, h0, bottom_solver=1)
+    mg.set_b(b)
+    mg.set_x(None)
+    xm = np.zeros(shape)
+    for _ in range(2):
+        mg.vcycle()
+        xm = matrix_vcycle(b, xm, L, h0, pre, post, bottom, bottom_solver=1)
+        xo = mg.get_x()
+        assert np.abs(xo - xm).max() <= 1e-9 * np.abs(xm).max()
+
+
+def test_max_norm_propagates_nan(oracle_mod):
+    """maxNormRes of a residual with a NaN is NaN (a diverged solve must not look
+    converged: max over a set containing NaN is taken as NaN, as the GPU's bit-pattern max does),
+    wherever the NaN sits (first / last cell, any thread's chunk); finite values are unaffected."""
+    shape = (8, 8, 16)
+    h = 1.0 / 16
+    x = np.zeros(shape)
+    for p in (0, 5, x.size // 2, x.size - 1):
+        b = mg_inputs.random_field(shape, 7)
+        b.ravel()[p] = np.nan
+        assert np.isnan(oracle_mod.max_norm_residual(x, b, h)), p
+    b = mg_inputs.random_field(shape, 7)
+    assert oracle_mod.max_norm_residual(x, b, h) == np.abs(b).max()
 
 
 def _rho(oracle_mod, N, L, b):

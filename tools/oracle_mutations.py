@@ -2,7 +2,7 @@
 
 Applies one plausible slip at a time to oracle/mg_oracle.c, rebuilds, runs
 tests/test_oracle_pins.py and reports whether some pin catches it.  The
-source is restored afterwards.  Last run: every mutation below CAUGHT (12 of 12).
+source is restored afterwards.  Last run: every mutation below CAUGHT (17 of 17).
 """
 import os
 import subprocess
@@ -28,6 +28,14 @@ MUTATIONS = {
                                "for (size_t i = 0; i + s < n; i += 2 * s) v[i] = v[i] + v[i + s];\n"
                                "  if (n > 1) { double t = v[0]; v[0] = a[0] * b[0];"
                                " for (size_t i = 1; i < n; ++i) v[0] = v[0] + a[i] * b[i]; (void)t; }"),
+    # smoother variants in the V-cycle (readings A19, A20)
+    "gsrb_pre_black_before_red": ("oracle_gsrb_half(n[0], n[1], n[2], m->h[l], c, m->x[l], m->Ax[l], m->b[l], m->r[l]);\n        }\n        continue;\n      }\n      oracle_apply_op(n[0], n[1], n[2], m->h[l], m->x[l], m->Ax[l]); /* exchange()+applyOp */",
+                                  "oracle_gsrb_half(n[0], n[1], n[2], m->h[l], 1 - c, m->x[l], m->Ax[l], m->b[l], m->r[l]);\n        }\n        continue;\n      }\n      oracle_apply_op(n[0], n[1], n[2], m->h[l], m->x[l], m->Ax[l]); /* exchange()+applyOp */"),
+    "gsrb_post_black_before_red": ("oracle_gsrb_half(n[0], n[1], n[2], m->h[l], c, m->x[l], m->Ax[l], m->b[l], m->r[l]);\n        }\n        continue;\n      }\n      oracle_apply_op(n[0], n[1], n[2], m->h[l], m->x[l], m->Ax[l]);\n      oracle_smooth_residual_gamma(lvl_n(m, l), step_gamma(m, l, m->post, it)",
+                                   "oracle_gsrb_half(n[0], n[1], n[2], m->h[l], 1 - c, m->x[l], m->Ax[l], m->b[l], m->r[l]);\n        }\n        continue;\n      }\n      oracle_apply_op(n[0], n[1], n[2], m->h[l], m->x[l], m->Ax[l]);\n      oracle_smooth_residual_gamma(lvl_n(m, l), step_gamma(m, l, m->post, it)"),
+    "chebyshev_pre_uses_post_count": ("step_gamma(m, l, m->pre, it)", "step_gamma(m, l, m->post, it)"),
+    "chebyshev_step_order_reversed": ("oracle_chebyshev_gamma(m->h[l], n, it, m->rho)", "oracle_chebyshev_gamma(m->h[l], n, n - 1 - it, m->rho)"),
+    "norm_drops_nan": ("if (a > mt || a != a) mt = a;", "if (a > mt) mt = a;"),
 }
 
 
