@@ -160,13 +160,14 @@ def ncu_traffic(n, kernel):
 
 
 # ------------------------------------------------------------------ oracle timing
-def oracle_dofs(n, levels, pre, post, bottom, seconds, min_cycles=1, max_cycles=1000):
+def oracle_dofs(n, levels, pre, post, bottom, seconds, min_cycles=1, max_cycles=1000, threads=None):
     """Time the CPU oracle (as it stands) running V-cycles on an n^3 grid."""
     import mg_inputs
     import oracle
 
     oracle.build()
-    oracle.set_threads(host_cores())  # the host's cores (torchrun sets OMP_NUM_THREADS=1 per process)
+    # the host's cores by default (torchrun sets OMP_NUM_THREADS=1 per process)
+    oracle.set_threads(threads or host_cores())
     b = mg_inputs.sin_rhs((n, n, n))
     m = oracle.OracleMG((n, n, n), levels, pre, post, bottom)
     m.set_b(b)
@@ -195,7 +196,12 @@ def cpu_baseline(a):
         v, c2, dt2, cores = oracle_dofs(small, lv, a.pre, a.post, a.bottom, a.cpu_seconds)
         sample = (f"{c2} oracle V-cycle(s) on a {small}^3 grid (L={lv}, same sweeps), {dt2:.1f} s; "
                   f"DOF/s of that sample")
-    return {"value": v, "unit": "DOF/s", "cores": cores, "kind": "oracle", "sample": sample}
+    # the same oracle on one core (both core counts), on a 256^3 sample (one cycle
+    # of the 512^3 workload would take ~30 s on one core)
+    v1, c1, dt1, _ = oracle_dofs(small, lv_small, a.pre, a.post, a.bottom, 0.0, threads=1)
+    single = {"value": v1, "unit": "DOF/s", "cores": 1,
+              "sample": f"{c1} oracle V-cycle(s) on a {small}^3 grid (L={lv_small}) on one thread, {dt1:.1f} s"}
+    return {"value": v, "unit": "DOF/s", "cores": cores, "kind": "oracle", "sample": sample, "single_thread": single}
 
 
 def run_reference(a, rank, world):
@@ -206,15 +212,29 @@ def run_reference(a, rank, world):
 
     oracle.build()
     oracle.set_threads(host_cores())
-    n = a.ref_n or min(a.n, 256)
-    lv = max(1, min(a.levels, (n // 8).bit_length()))
     import mg_inputs
 
-    b = mg_inputs.sin_rhs((n, n, n))
-    m = oracle.OracleMG((n, n, n), lv, a.pre, a.post, a.bottom)
-    m.set_b(b)
-    m.set_x(None)
-    for _ in range(a.warmup):
+    def setup(n, lv):
+        m = oracle.OracleMG((n, n, n), lv, a.pre, a.post, a.bottom)
+        m.set_b(mg_inputs.sin_rhs((n, n, n)))
+        m.set_x(None)
+        return m
+
+    # the workload itself (512^3 per rank, L = 6: about 2 s per oracle cycle on 16 cores); a 256^3
+    # sample only if the first (warm-up) cycle says the run would not end within ~5 minutes
+    n = a.ref_n or a.n
+    lv = a.levels if n == a.n else max(1, min(a.levels, (n // 8).bit_length()))
+    m = setup(n, lv)
+    t0 = time.perf_counter()
+    m.vcycle()
+    t1 = time.perf_counter() - t0
+    if not a.ref_n and t1 * (a.steps + a.warmup) > 300.0 and n > 256:
+        m.close()
+        n = 256
+        lv = max(1, min(a.levels, (n // 8).bit_length()))
+        m = setup(n, lv)
+        m.vcycle()
+    for _ in range(a.warmup - 1):
         m.vcycle()
     t0 = time.perf_counter()
     for _ in range(a.steps):
@@ -222,11 +242,14 @@ def run_reference(a, rank, world):
     dt = time.perf_counter() - t0
     value = n**3 * a.steps / dt
     pg = PROC_GRIDS.get(a.gpus, (1, 1, 1))
-    sample = f"each step = one oracle V-cycle on a {n}^3 grid (L={lv}, {a.pre}/{a.post}/{a.bottom}), bounded sample"
+    sample = (f"each step = one oracle V-cycle of the {n}^3 workload (L={lv}, {a.pre}/{a.post}/{a.bottom})"
+              if n == a.n and lv == a.levels else
+              f"each step = one oracle V-cycle on a {n}^3 grid (L={lv}, {a.pre}/{a.post}/{a.bottom}), bounded sample")
     line = {"metric": METRIC, "value": value, "unit": "DOF/s", "n_gpus": a.gpus, "steps": a.steps,
             "warmup": a.warmup, "ms_per_step": dt / a.steps * 1e3, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
-            "config": {"workload": workload_name(a, pg), "sample_grid": n, "levels": lv},
+            "config": {"workload": workload_name(a, pg) if n == a.n else
+                       f"{n}^3 sample of: " + workload_name(a, pg), "sample_grid": n, "levels": lv},
             "cpu_baseline": {"value": value, "unit": "DOF/s", "cores": oracle.get_threads(), "kind": "oracle",
                              "sample": sample},
             "e2e": {"value": value, "unit": "DOF/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
@@ -363,19 +386,23 @@ def main():
         e2e = {"value": world * n**3 * ke / (te / 1e3), "unit": "DOF/s", "h2d_bytes_per_step": int(b_host.numel() * 8),
                "d2h_bytes_per_step": 8, "steps": ke, "ms_per_step": te / ke}
         # (informational) the same metric over whole solves through mg_solve (Alg 1): one upload of b
-        # per solve, V-cycles until max|b - Ax| < 1e-10 with the norm read back after every cycle
+        # per solve, V-cycles until max|b - Ax| < 1e-10 with the norm read back after every cycle,
+        # then the solution x downloaded into pinned host memory (mg_get_solution_host)
         ks, cyc_tot = 3, 0
+        x_host = torch.empty(m.shape, dtype=torch.float64, pin_memory=True)
         barrier()
         t0 = time.perf_counter()
         for _ in range(ks):
             m.set_rhs_host(b_host)
             m.set_solution(None)
             _, cyc, _ = m.solve(1e-10, 20)
+            m.get_solution_host(x_host)
             cyc_tot += cyc
         ts = max_over_ranks((time.perf_counter() - t0) * 1e3)
         e2e["solve"] = {"value": world * n**3 * cyc_tot / (ts / 1e3), "unit": "DOF/s", "solves": ks,
                         "vcycles_per_solve": cyc_tot / ks, "ms_per_solve": ts / ks,
-                        "h2d_bytes_per_solve": int(b_host.numel() * 8)}
+                        "h2d_bytes_per_solve": int(b_host.numel() * 8),
+                        "d2h_bytes_per_solve": int(x_host.numel() * 8 + 8 * (cyc_tot / ks + 1))}
 
     launches = m.launches_per_vcycle()
     xbytes, xmsgs = m.exchange_stats()

@@ -104,8 +104,9 @@ typedef struct {
   int32_t ca_period[MG_MAX_LEVELS]; /* sweeps per x-exchange per level, 1..8; 0 = auto (8) */
   int32_t fusion[MG_MAX_LEVELS];    /* MG_FUSION_*; 0 = auto */
   int32_t ghost_mode;            /* MG_GHOST_* */
-  int32_t transport;             /* MG_TRANSPORT_*: auto = NCCL when world_size > 1 or a
-                                    self-exchange is needed and an NCCL id is given, else local */
+  int32_t transport;             /* MG_TRANSPORT_*: auto = NCCL when world_size > 1, else local device
+                                    copies (a one-rank MG_GHOST_ALL self-exchange goes through NCCL only
+                                    with MG_TRANSPORT_NCCL; nccl_id may then be NULL) */
   int32_t use_graph;             /* 1 = replay the V-cycle as one CUDA graph (default 1) */
   int32_t bottom_mode;           /* MG_BOTTOM_* (resident = one CTA runs all bottom sweeps in smem,
                                     cluster = the coarse levels run in one cluster launch, grid = the
@@ -161,7 +162,9 @@ mg_status mg_setup(const mg_params* p, int32_t rank, int32_t world_size, const u
  * the context's stream (e.g. the V-cycle of the previous right-hand side); the
  * conversion into bricks is ordered on the context's stream.  b_host must not
  * be modified until the next synchronising call returns; pinned memory gives a
- * truly asynchronous copy. */
+ * truly asynchronous copy.  The first host-buffer call (mg_set_rhs_host or
+ * mg_get_solution_host) allocates the two level-0 staging fields with cudaMalloc
+ * (library-owned, freed by mg_destroy; not part of mg_workspace_bytes). */
 mg_status mg_set_rhs(mg_ctx* c, const double* b_dev);
 mg_status mg_set_rhs_host(mg_ctx* c, const double* b_host);
 /* Initial guess; NULL => x = 0 (reading A9). */
@@ -183,7 +186,9 @@ mg_status mg_residual_norm_async(mg_ctx* c);
 mg_status mg_residual_norm_wait(mg_ctx* c, double* out_max_abs);
 
 /* Alg 1: while norm > tol and cycles < max_cycles: V-cycle.
- * Returns MG_NOT_CONVERGED (1) if the cap was hit. */
+ * Returns MG_OK when the final norm is <= tol, MG_NOT_CONVERGED (1) if the cap was
+ * hit or the norm is not finite (a NaN stops the loop at once; mg_last_error says
+ * "not finite"). */
 mg_status mg_solve(mg_ctx* c, double tol, int32_t max_cycles, int32_t* cycles_done, double* final_norm);
 
 /* Per (level, op) device times in ms of the last mg_vcycle run with
@@ -283,6 +288,10 @@ mg_status mg_layout_pass_plan(const mg_layout* lay, int32_t level, int32_t idx, 
  * brick of each owned brick, gb_adj int32 [info[0]][8] = the global level's adjacency (periodic
  * wrap).  Any array may be NULL. */
 mg_status mg_layout_repl(const mg_layout* lay, int64_t info[2], int32_t* gb_src, int32_t* gb_mine, int32_t* gb_adj);
+/* Kernel launches of this library one V-cycle issues from a fresh context's state, the count
+ * mg_vcycle_launches gives on a GPU (exchanges: one copy kernel each if local_exchange, none of
+ * ours over NCCL). */
+mg_status mg_layout_vcycle_launches(const mg_layout* lay, int32_t local_exchange, int64_t* out);
 mg_status mg_layout_destroy(mg_layout* lay);
 
 #ifdef __cplusplus

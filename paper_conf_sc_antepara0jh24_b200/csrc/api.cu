@@ -15,6 +15,7 @@
 #include <cuda_runtime.h>
 #include <nccl.h>
 
+#include <cmath>
 #include <cstdio>
 #include <cstring>
 #include <string>
@@ -121,6 +122,7 @@ struct mg_ctx {
     CopyRun* scatter = nullptr;  // [2][n_owned]: into x[0] / x[1] of the coarsest level
     bool allgather = false;
   } rp;
+  std::vector<void*> allocs;  // library-owned device buffers allocated on first use (freed by mg_destroy)
   std::vector<double> tm;
   std::vector<TimerRec> trec;
   std::vector<std::pair<int, double>> recs;  // (level*MG_NUM_OPS + op, ms) per timed op, since mg_set_timing
@@ -185,7 +187,9 @@ size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double**
     d.x[1] = (double*)take(fb);
     d.b = (double*)take(fb);
     d.r = (double*)take(fb);
-    d.Ax = (double*)take(fb);
+    // Ax only for the paper's kernel set (MG_FUSION_PAPER: applyOp writes it, smooth+residual reads
+    // it); a per-op call that asks for the paper set on another level allocates it lazily (ensure_ax)
+    if (lay.p.fusion[l] == MG_FUSION_PAPER) d.Ax = (double*)take(fb);
     d.adj = (int32_t*)take((size_t)L.n_stored * 8 * sizeof(int32_t));
     d.parent = (int32_t*)take((size_t)L.n_alloc * sizeof(int32_t));
     d.coord = (int32_t*)take((size_t)L.n_stored * 3 * sizeof(int32_t));
@@ -218,12 +222,9 @@ size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double**
     d.c = level_coeffs(d.h);
     if (out) (*out)[l] = d;
   }
-  // two staging fields for host uploads (double-buffered: the upload of the next right-hand
-  // side overlaps the current V-cycle)
-  for (int k = 0; k < 2; ++k) {
-    double* st = (double*)take((size_t)lay.lv[0].n_owned * kBV * sizeof(double));
-    if (stage) stage[k] = st;
-  }
+  // (the two host-upload staging fields are allocated on first use of the host-buffer calls,
+  // ensure_stage: a device-only caller does not pay 2 level-0 fields for them)
+  (void)stage;
   if (lay.repl) {  // replicated bottom
     const size_t gfb = (size_t)lay.gb.n_alloc * kBV * sizeof(double);
     const int64_t nown = lay.lv[(size_t)lay.L - 1].n_owned;
@@ -278,6 +279,41 @@ cudaEvent_t pool_event(mg_ctx* c) {
     c->evpool.push_back(e);
   }
   return c->evpool[c->evnext++];
+}
+
+// buffers allocated on first use (outside graph capture: callers run these before a plan executes)
+mg_status ensure_ax(mg_ctx* c, int l) {
+  DevLevel& d = c->dl[l];
+  if (d.Ax) return MG_OK;
+  void* p = nullptr;
+  CKC(c, cudaMalloc(&p, (size_t)c->lay.lv[l].n_alloc * kBV * sizeof(double)));
+  c->allocs.push_back(p);
+  d.Ax = (double*)p;
+  return MG_OK;
+}
+
+mg_status ensure_stage(mg_ctx* c) {
+  if (c->stage[0]) return MG_OK;
+  for (int k = 0; k < 2; ++k) {
+    void* p = nullptr;
+    CKC(c, cudaMalloc(&p, (size_t)c->lay.lv[0].n_owned * kBV * sizeof(double)));
+    c->allocs.push_back(p);
+    c->stage[k] = (double*)p;
+  }
+  return MG_OK;
+}
+
+// every buffer a plan's ops need exists (Ax of the levels that run the paper's kernel set)
+mg_status prepare_plan(mg_ctx* c, mg_group* g, const std::vector<Op>& ops) {
+  for (const Op& o : ops)
+    if (o.paper) {
+      if (g) {
+        for (mg_ctx* r : g->r) CKS(ensure_ax(r, o.level));
+      } else {
+        CKS(ensure_ax(c, o.level));
+      }
+    }
+  return MG_OK;
 }
 
 // ------------------------------------------------------------- exchange
@@ -580,11 +616,11 @@ mg_status exec_op(mg_ctx* c, const Op& o, cudaStream_t s) {
   return set_err(MG_ERR_STATE, "unknown op");
 }
 
-Plan make_plan(const Builder& b, const Layout& lay, bool pencil_overlap) {
+Plan make_plan(const Builder& b, const Layout& lay, bool pencil_overlap, bool local_exchange) {
   Plan p;
   p.ops = b.ops;
   for (int l = 0; l < MG_MAX_LEVELS; ++l) p.final_st[l] = b.st[l];
-  for (const Op& o : p.ops) p.launches += op_launches(o, lay, lay.p.overlap != 0, pencil_overlap);
+  for (const Op& o : p.ops) p.launches += op_launches(o, lay, lay.p.overlap != 0, pencil_overlap, local_exchange);
   return p;
 }
 
@@ -623,7 +659,8 @@ mg_status check_ctx(mg_ctx* c) {
 }
 
 mg_status build_and_run(mg_ctx* c, mg_group* g, bool vcycle_graph, Builder& b) {
-  const Plan p = make_plan(b, c->lay, c->pencil_overlap);
+  const Plan p = make_plan(b, c->lay, c->pencil_overlap, !c->use_nccl);
+  CKS(prepare_plan(c, g, p.ops));
   CKS(run_plan(c, g, p, g ? g->stream : c->stream));
   if (g) {
     for (mg_ctx* r : g->r)
@@ -649,7 +686,8 @@ mg_status vcycle_impl(mg_ctx* c, mg_group* g) {
     Builder b(c0->lay);
     for (int l = 0; l < MG_MAX_LEVELS; ++l) b.st[l] = c0->st[l];
     b.vcycle();
-    Plan p = make_plan(b, c0->lay, c0->pencil_overlap);
+    Plan p = make_plan(b, c0->lay, c0->pencil_overlap, !c0->use_nccl);
+    CKS(prepare_plan(c0, g, p.ops));
     if (graph) {
       // capture on a private non-blocking stream; the graph is then launched on the caller's stream
       cudaStream_t cs = g ? g->cap : c->cap;
@@ -782,6 +820,7 @@ void free_ctx(mg_ctx* c) {
   if (c->ev_join) cudaEventDestroy(c->ev_join);
   for (cudaEvent_t e : c->evpool) cudaEventDestroy(e);
   if (c->h_pinned) cudaFreeHost(c->h_pinned);
+  for (void* a : c->allocs) cudaFree(a);
   delete c;
 }
 
@@ -926,6 +965,7 @@ mg_status mg_set_rhs(mg_ctx* c, const double* b_dev) {
 mg_status mg_set_rhs_host(mg_ctx* c, const double* b_host) {
   CKS(check_ctx(c));
   if (!b_host) return set_err(MG_ERR_INVALID_ARG, "null b");
+  CKS(ensure_stage(c));
   const size_t bytes = (size_t)c->lay.lv[0].n_owned * kBV * sizeof(double);
   // Upload on the copy stream into staging field k (free once its previous conversion ran), so
   // the transfer overlaps whatever the caller's stream is still executing (the V-cycle of the
@@ -963,6 +1003,7 @@ mg_status mg_get_solution(mg_ctx* c, double* x_dev) {
 mg_status mg_get_solution_host(mg_ctx* c, double* x_host) {
   CKS(check_ctx(c));
   if (!x_host) return set_err(MG_ERR_INVALID_ARG, "null x");
+  CKS(ensure_stage(c));
   const int k = c->stage_k;  // every upload into it is already ordered before its conversion
   CKS(mg_get_solution(c, c->stage[k]));
   const size_t bytes = (size_t)c->lay.lv[0].n_owned * kBV * sizeof(double);
@@ -1028,7 +1069,10 @@ mg_status mg_solve(mg_ctx* c, double tol, int32_t max_cycles, int32_t* cycles_do
   }
   if (cycles_done) *cycles_done = k;
   if (final_norm) *final_norm = nr;
-  return nr > tol ? MG_NOT_CONVERGED : MG_OK;
+  // a NaN norm fails `nr > tol` as well as `nr <= tol`: the loop stops at once and the solve reports
+  // that it did not converge (a diverged iteration must never look converged)
+  if (!std::isfinite(nr)) return set_err(MG_NOT_CONVERGED, "residual norm is not finite: the iteration diverged");
+  return nr <= tol ? MG_OK : MG_NOT_CONVERGED;
 }
 
 mg_status mg_set_timing(mg_ctx* c, int32_t enabled) {
@@ -1067,7 +1111,7 @@ mg_status mg_vcycle_launches(mg_ctx* c, int64_t* out) {
   Builder b(c->lay);
   for (int l = 0; l < MG_MAX_LEVELS; ++l) b.st[l] = c->st[l];
   b.vcycle();
-  *out = make_plan(b, c->lay, c->pencil_overlap).launches;
+  *out = make_plan(b, c->lay, c->pencil_overlap, !c->use_nccl).launches;
   return MG_OK;
 }
 
@@ -1396,6 +1440,17 @@ mg_status mg_layout_pass_plan(const mg_layout* m, int32_t level, int32_t idx, in
   info[5] = t.part;
   if (meta) std::copy(t.meta.begin(), t.meta.end(), meta);
   if (ctas) std::copy(t.ctas.begin(), t.ctas.end(), ctas);
+  return MG_OK;
+}
+
+mg_status mg_layout_vcycle_launches(const mg_layout* m, int32_t local_exchange, int64_t* out) {
+  if (!m || !out) return set_err(MG_ERR_INVALID_ARG, "null argument");
+  Builder b(m->lay);
+  b.vcycle();  // from the state of a fresh context (every level's ghosts stale)
+  const bool pencil_overlap = m->lay.world > 1 && m->lay.p.transport != MG_TRANSPORT_LOCAL;
+  int64_t n = 0;
+  for (const Op& o : b.ops) n += op_launches(o, m->lay, m->lay.p.overlap != 0, pencil_overlap, local_exchange != 0);
+  *out = n;
   return MG_OK;
 }
 

@@ -345,30 +345,35 @@ void Builder::vcycle() {
   }
 }
 
-int64_t op_launches(const Op& o, const Layout& lay, bool overlap, bool pencil_overlap) {
+int64_t op_launches(const Op& o, const Layout& lay, bool overlap, bool pencil_overlap, bool local_exchange) {
+  // kernels of this library one op launches (NCCL's own kernels not counted); an exchange over the
+  // local transport is one copy kernel (copy_runs_kernel), over NCCL none of ours
+  const int64_t ex = local_exchange ? 1 : 0;
   switch (o.kind) {
     case OP_SWEEP:
     case OP_SWEEP2: {
-      const int per = o.paper ? 2 : 1;
+      const int per = o.paper ? 2 : 1;  // applyOp + smooth(+residual)
       const LevelLayout& L = lay.lv[o.level];
       const int64_t end = o.ghosts ? L.n_stored : L.n_owned;
+      const int64_t x = o.exch_before ? ex : 0;
       bool pen_split = false;
       if (o.kind == OP_SWEEP2 && o.exch_before && overlap && pencil_overlap)
         for (const auto& pt : L.pairs) pen_split |= pt.b0 == 0 && pt.b1 == end && pt.part == 1;
-      if (pen_split) return 2;
+      if (pen_split) return 2 + x;
       const bool split = o.exch_before && overlap && lay.lv[o.level].n_interior > 0 && !o.nosplit;
-      return per * (split ? 2 : 1);
+      return per * (split ? 2 : 1) + x;
     }
-    case OP_RESTRICT:
-    case OP_INTERP:
-    case OP_ZERO:
-    case OP_BOTTOM_REPL:
-      return 3;
-    case OP_BOTTOM_CG:
-      return 1;  // gather copies, the solve, the scatter copies (+ an all-gather on NCCL)
-    case OP_BOTTOM_RES:
-    case OP_COARSE:
+    case OP_RESTRICT:  // restrict_kernel
+    case OP_INTERP:    // interp4_kernel / interp_kernel
+    case OP_ZERO:      // zero_kernel
+    case OP_BOTTOM_CG:  // bottom_cg_kernel
+    case OP_BOTTOM_RES:  // bottom_resident_kernel
+    case OP_COARSE:      // one cluster / grid launch
       return 1;
+    case OP_BOTTOM_REPL:  // gather copies, the solve, the scatter copies (+ NCCL's all-gather)
+      return 3;
+    case OP_EXCH:
+      return ex;
     default:
       return 0;
   }

@@ -77,6 +77,7 @@ struct Builder {
   void vcycle();
 };
 
-int64_t op_launches(const Op& o, const Layout& lay, bool overlap, bool pencil_overlap);
+// own kernel launches of one op (local_exchange: exchanges run as one copy kernel, else NCCL)
+int64_t op_launches(const Op& o, const Layout& lay, bool overlap, bool pencil_overlap, bool local_exchange);
 
 }  // namespace mgb

@@ -116,6 +116,7 @@ _SIGS = {
                                            ctypes.c_void_p, ctypes.c_void_p]),
     "mg_layout_repl": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
                                       ctypes.c_void_p]),
+    "mg_layout_vcycle_launches": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.POINTER(ctypes.c_int64)]),
     "mg_layout_destroy": (ctypes.c_int, [ctypes.c_void_p]),
 }
 
@@ -413,6 +414,13 @@ class Layout:
                   "mg_layout_pass_plan")
             out.append((info[0], info[1], info[2], meta[:info[3]], ctas[:info[4]].reshape(-1, 2), info[5]))
         return out
+
+    def vcycle_launches(self, local_exchange=True) -> int:
+        """Own kernel launches of one V-cycle (mg_layout_vcycle_launches)."""
+        out = ctypes.c_int64()
+        check(lib().mg_layout_vcycle_launches(self.h, 1 if local_exchange else 0, ctypes.byref(out)),
+              "mg_layout_vcycle_launches")
+        return out.value
 
     def plan(self, level, which):
         inf = self.info(level)

@@ -90,7 +90,13 @@ class Multigrid:
         mg.mg_get_solution(self.ctx, _ptr(out))
         return out
 
-    def get_solution_host(self, out: torch.Tensor):
+    def get_solution_host(self, out: torch.Tensor | None = None) -> torch.Tensor:
+        """x (local lexicographic) into a host fp64 tensor (pinned if allocated here); synchronises."""
+        if out is None:
+            out = torch.empty(self.shape, dtype=torch.float64, pin_memory=True)
+        assert out.dtype == torch.float64 and not out.is_cuda and out.is_contiguous(), \
+            "fp64 contiguous host tensor expected"
+        assert tuple(out.shape) == self.shape, (tuple(out.shape), self.shape)
         mg.mg_get_solution_host(self.ctx, _ptr(out))
         return out
 
@@ -176,12 +182,15 @@ class LoopbackGroup:
 
     def set_rhs(self, blocks):
         for r, b in enumerate(blocks):
-            assert tuple(b.shape) == self.shape and b.is_cuda and b.dtype == torch.float64
+            assert tuple(b.shape) == self.shape and b.is_cuda and b.dtype == torch.float64 and b.is_contiguous()
             mg.mg_group_set_rhs(self.g, r, _ptr(b))
         mg.mg_group_commit_rhs(self.g)
 
     def set_solution(self, blocks=None):
         for r in range(self.world_size):
+            if blocks is not None:
+                b = blocks[r]
+                assert tuple(b.shape) == self.shape and b.is_cuda and b.dtype == torch.float64 and b.is_contiguous()
             mg.mg_group_set_solution(self.g, r, None if blocks is None else _ptr(blocks[r]))
 
     def vcycle(self):

@@ -78,7 +78,28 @@ def test_product_package_never_imports_oracle():
 def test_workspace_bytes_scales_with_levels():
     a = mg.mg_workspace_bytes(mg.params((64, 64, 64), num_levels=1))
     b = mg.mg_workspace_bytes(mg.params((64, 64, 64), num_levels=4))
-    assert b > a and a >= 5 * 64**3 * 8
+    assert b > a and a >= 4 * 64**3 * 8  # x, x' (ping-pong), b, r
+
+
+def test_workspace_holds_ax_only_for_the_paper_kernel_set():
+    """Ax (applyOp's output) exists only on levels that run the paper's kernel set (fusion 1); the
+    host-upload staging fields are allocated on first use, outside the workspace."""
+    n = 64
+    fused = mg.mg_workspace_bytes(mg.params((n, n, n), num_levels=1))
+    paper = mg.mg_workspace_bytes(mg.params((n, n, n), num_levels=1, fusion=[1] + [0] * 15))
+    assert paper - fused >= n**3 * 8 and paper - fused <= n**3 * 8 + 4096 + 256  # + the zero brick, alignment
+    assert fused < 5 * n**3 * 8
+
+
+@pytest.mark.parametrize("n,L,launches", [(512, 6, 90), (256, 6, 100), (64, 4, 73)])
+def test_vcycle_launch_count(n, L, launches):
+    """Launches of one V-cycle (the bench's launches_per_step): at 512^3, L = 6 level 0
+    runs 6 pencil passes + 1 interpolation + 6 passes (13), levels 1 and 2 a zero-folded single
+    sweep, 5 passes and a restricting single sweep, then an interpolation and 6 passes (14 each),
+    levels 3 and 4 24 single sweeps each (the first post-sweep with the interpolation fused), the
+    bottom 1 resident launch: 90."""
+    lay = mg.Layout(mg.params((n, n, n), num_levels=L))
+    assert lay.vcycle_launches() == launches
 
 
 @pytest.mark.parametrize("bad", [dict(smoother=3), dict(launch_pdl=3), dict(bottom_solver=2), dict(smoother=-1), dict(bottom_mode=5), dict(transport=7),

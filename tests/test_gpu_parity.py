@@ -231,6 +231,31 @@ def test_solve_matches_oracle(oracle_mod):
     m.close()
 
 
+@pytest.mark.parametrize("where", ["nan", "inf"])
+def test_solve_reports_nonfinite_norm(oracle_mod, where):
+    """A non-finite residual never looks converged (Alg 1 loops while norm > tol; a NaN fails
+    both norm > tol and norm <= tol): mg_solve stops and returns MG_NOT_CONVERGED with the non-finite
+    norm, as the oracle's NaN-propagating max does.  Cases: a NaN in b (norm NaN before any cycle);
+    an inf in b (norm inf, the V-cycle turns x into inf - inf = NaN, the loop stops on the NaN)."""
+    mg, _ = _mg()
+    shape = (32, 32, 32)
+    b = mg_inputs.random_rhs(shape, 1)
+    b[3, 4, 5] = np.nan if where == "nan" else np.inf
+    orc = oracle_mod.OracleMG(shape, 3)
+    orc.set_b(b)
+    orc.set_x(None)
+    assert not np.isfinite(orc.norm())
+    m = new(shape, 3)
+    m.set_rhs(dev(b))
+    m.set_solution(None)
+    st, cyc, fin = m.solve(1e-10, 20)
+    assert st == mg.MG_NOT_CONVERGED and not np.isfinite(fin), (st, cyc, fin)
+    assert cyc < 20
+    if where == "nan":
+        assert cyc == 0 and np.isnan(fin)
+    m.close()
+
+
 @pytest.mark.parametrize("bottom_mode", [0, 1, 2, 3, 4])
 @pytest.mark.parametrize("shape,L,pre,post,bottom", [
     ((64, 64, 64), 4, 12, 12, 100),   # config 1: levels 1-3 (64, 8, 1 bricks) in the cluster
