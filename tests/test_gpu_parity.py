@@ -409,6 +409,35 @@ def test_full_size_512_vcycle_bitwise(oracle_mod):
     m.close()
 
 
+@pytest.mark.slow
+def test_full_size_decomposed_2x1x1_vs_oracle(oracle_mod):
+    """Config 4's per-rank size in a decomposition, against the oracle itself: 1024 x 512 x 512 global
+    as a 2x1x1 loopback (512^3 per rank, L = 6: ghost shells on x, exchanges through the NCCL plans,
+    pencil passes over the stored box, the replicated bottom), one V-cycle: x of every rank and the
+    residual norm bit for bit equal to the undecomposed oracle (about 5 s of oracle time)."""
+    import torch
+
+    _, solver = _mg()
+    torch.cuda.empty_cache()
+    pg, L = (2, 1, 1), 6
+    nl = (512, 512, 512)
+    G = (512, 512, 1024)  # (nz, ny, nx)
+    b = mg_inputs.sin_rhs(G)
+    xs, ns = oracle_cycles(oracle_mod, b, L, 1)
+    g = solver.LoopbackGroup(nl, pg, num_levels=L)
+    try:
+        g.set_rhs([dev(mg_inputs.local_block(b, r, pg)) for r in range(2)])
+        g.set_solution(None)
+        g.vcycle()
+        assert g.residual_norm() == ns[0]
+        for r in range(2):
+            assert_bitwise(host(g.get_solution(r)), mg_inputs.local_block(xs[0], r, pg), what=f"rank {r}")
+    finally:
+        g.close()
+        del g
+        torch.cuda.empty_cache()
+
+
 @pytest.mark.parametrize("pg", [(2, 1, 1), (2, 2, 1), (2, 2, 2)])
 def test_config5_1024_decomposition_invariant(pg):
     """Config 5 at its full size (1024^3 total, L = 7, global coarsest 16^3 for every P): one V-cycle on
