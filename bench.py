@@ -49,9 +49,10 @@ def parse():
     ap.add_argument("--ghost-all", action="store_true", help="self-exchange ghost shell on every axis")
     ap.add_argument("--no-graph", action="store_true")
     ap.add_argument("--no-overlap", action="store_true")
-    ap.add_argument("--tb", type=int, default=3,
-                    help="temporal blocking (two sweeps per HBM pass): 3 = 2x2-brick pencils (sweep2p.cu, default), "
-                         "1 = one-brick CTA streams (sweep2.cu), 2 = warp plane streams (sweep2w.cu), 0 = off")
+    ap.add_argument("--tb", type=int, default=4,
+                    help="temporal blocking (two sweeps per HBM pass): 4 = 2x2-brick pencils, one warp per tile "
+                         "(sweep2q.cu, default), 3 = 2x2-brick pencils, two-warp CTAs (sweep2p.cu), 1 = one-brick "
+                         "CTA streams (sweep2.cu), 2 = warp plane streams (sweep2w.cu), 0 = off")
     ap.add_argument("--smoother", type=int, default=0,
                     help="0 damped Jacobi (the paper), 1 Chebyshev, 2 red-black Gauss-Seidel (N4 variants)")
     ap.add_argument("--cheby-ratio", type=int, default=0, help="Chebyshev smoothing interval [mu_max/ratio, mu_max]")
@@ -351,7 +352,9 @@ def main():
     # the same level-0 work expressed as one-sweep-per-pass traffic (what the sweeps would move unblocked)
     sweep_equiv = pts * (B_SWEEP * nsweep0 + 2 * B_COARSE_PER_FINE) / (sweep0_ms / 1e3) / 1e9
     peak, peak_src = measured_peaks()
-    traffic = ncu_traffic(n, {0: "sweep_col_kernel", 1: "sweep2_kernel", 2: "sweep2w_kernel"}.get(a.tb, "sweep2p_kernel"))
+    pass_kernel = {0: "sweep_col_kernel", 1: "sweep2_kernel", 2: "sweep2w_kernel", 3: "sweep2p_kernel"}.get(
+        a.tb, "sweep2q_kernel")
+    traffic = ncu_traffic(n, pass_kernel)
     levels = []
     total_inst = sum(sum(r) for r in tm) / ninst
     for l, row in enumerate(tm):
@@ -422,16 +425,15 @@ def main():
                        "coarse": {0: "auto", 1: "per-sweep launches", 2: "resident bottom", 3: "cluster solve",
                                   4: "grid solve"}[a.bottom_mode],
                        "bottom_solver": "conjugate gradients" if a.bottom_solver else "damped jacobi (paper)",
-                       "temporal_blocking": {0: "off", 1: "one-brick CTA streams", 2: "warp plane streams"}.get(
-                           a.tb, "2x2-brick pencils"),
+                       "temporal_blocking": {0: "off", 1: "one-brick CTA streams", 2: "warp plane streams",
+                                             3: "2x2-brick pencils, two-warp CTAs"}.get(
+                           a.tb, "2x2-brick pencils, one warp per tile"),
                        "smoother": {1: "chebyshev", 2: "red-black gauss-seidel"}.get(a.smoother, "damped jacobi (paper)"),
                        "l2": "no flush: every level-0 field is 1 GiB > 126 MB L2 (inputs larger than L2)",
                        "parallelism": f"3D domain decomposition {pg[0]}x{pg[1]}x{pg[2]}"},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic,
-                         "kernel": ("level-0 passes: %s (two sweeps per pass) + sweep_col_kernel / "
-                                    "interp-fused sweep_kernel" % {1: "sweep2_kernel", 2: "sweep2w_kernel"}.get(
-                                        a.tb, "sweep2p_kernel") if a.tb else
+                         "kernel": ("level-0 passes: %s (two sweeps per pass)" % pass_kernel if a.tb else
                                     "level-0 sweeps: sweep_col_kernel + interp-fused sweep_kernel"),
                          "passes_per_vcycle": npass0, "launch_ms": launch_ms,
                          "bytes_per_point_per_pass": bytes0 / pts / npass0,

@@ -59,6 +59,7 @@ struct DevLevel {
   std::vector<Pair> pairs;  // two-sweep item streams per brick range
   PairMaps pmaps[2];        // tensor maps for the two-sweep kernel reading x[0] / x[1]
   PairMaps nmaps[2];        // the same with 4-plane boxes for the pencil kernel (sweep2p.cu)
+  PairMaps qmaps[2];        // 2-plane boxes for the one-warp pencil kernel (sweep2q.cu)
   // local-transport exchange: [x[0] | x[1] | b][recv run] copy descriptors (device), one launch
   CopyRun* cruns = nullptr;
   int ncruns = 0;
@@ -431,7 +432,9 @@ mg_status sweep_range(mg_ctx* c, const Op& o, int64_t b0, int64_t b1, cudaStream
   if (o.kind == OP_SWEEP2) {  // two sweeps in one pass: the builder only emits it where a plan exists
     for (const auto& pr : d.pairs) {
       if (pr.b0 == b0 && pr.b1 == b1 && pr.part == part) {
-        if (pr.args.kind == 3)
+        if (pr.args.kind == 4)
+          CKC(c, launch_sweep2q(a, pr.args, d.qmaps[o.src], o.flags | (o.zero ? SW_ZERO_X : 0u), s));
+        else if (pr.args.kind == 3)
           CKC(c, launch_sweep2p(a, pr.args, d.nmaps[o.src], o.flags, s));
         else if (pr.args.kind == 2)
           CKC(c, launch_sweep2w(a, pr.args, d.pmaps[o.src], o.flags, s));
@@ -774,6 +777,7 @@ mg_status init_ctx(mg_ctx* c, const mg_params& p, int rank, int world, int devic
       for (int xb = 0; xb < 2; ++xb) {
         CKC(c, encode_pair_maps(d.x[xb], d.b, L.n_alloc, &d.pmaps[xb]));
         CKC(c, encode_pencil_maps(d.x[xb], d.b, L.n_alloc, &d.nmaps[xb]));
+        CKC(c, encode_quad_maps(d.x[xb], d.b, L.n_alloc, &d.qmaps[xb]));
       }
   }
   if (c->lay.repl) {
@@ -863,7 +867,7 @@ void mg_params_default(mg_params* p) {
   p->bottom_smooths = 100;
   p->use_graph = 1;
   p->overlap = 1;
-  p->temporal_blocking = 3;
+  p->temporal_blocking = 4;
   p->h0 = 0.0;
 }
 

@@ -718,6 +718,8 @@ cudaError_t kernels_init() {
   if (e != cudaSuccess) return e;
   e = pencil_kernels_init();
   if (e != cudaSuccess) return e;
+  e = quad_kernels_init();
+  if (e != cudaSuccess) return e;
   e = pairw_kernels_init();
   if (e != cudaSuccess) return e;
   e = coarse_kernels_init();

@@ -98,6 +98,14 @@ bool pencil_supports(unsigned flags);
 cudaError_t launch_sweep2p(const SweepArgs& a, const PairArgs& pa, const PairMaps& pm, unsigned flags,
                            cudaStream_t s);
 cudaError_t pencil_kernels_init();
+// one-warp 2x2-brick pencil two-sweep kernel (sweep2q.cu, plan kind 4: the kind-3 chunk records dealt
+// to kQuadCtas CTAs): maps with 2-plane boxes (x {2,8,2}, {8,2,2}, {2,1,2}; b {2,8,2}, {8,2,2}); the
+// flags of the SECOND sweep (plain, +r, +restriction) | SW_ZERO_X (the FIRST sweep reads x0 == 0)
+cudaError_t encode_quad_maps(const double* x, const double* b, int64_t n_alloc, PairMaps* out);
+bool quad_supports(unsigned flags);
+cudaError_t launch_sweep2q(const SweepArgs& a, const PairArgs& pa, const PairMaps& pm, unsigned flags,
+                           cudaStream_t s);
+cudaError_t quad_kernels_init();
 
 // true if the streaming kernel implements `flags` (plain, +r, +restriction)
 bool col_supports(unsigned flags);

@@ -268,7 +268,7 @@ mg_status build_layout(const mg_params& p, int rank, int world, Layout& out, std
   if (p.temporal_blocking != 0)
     for (int l = 0; l < out.L; ++l)
       build_pair_tables(out.lv[l], p.sweep_kernel == 0 ? kPairMinBricks : min_b,
-                        p.temporal_blocking == 2 ? 2 : p.temporal_blocking == 3 ? 3 : 1);
+                        p.temporal_blocking >= 2 && p.temporal_blocking <= 4 ? p.temporal_blocking : 1);
   // replicated bottom: the global coarsest level as one rank would store it
   const LevelLayout& B = out.lv[(size_t)out.L - 1];
   out.repl = false;
@@ -461,7 +461,10 @@ static LevelLayout::PairTable pair_table(const LevelLayout& L, int64_t b0, int64
 // part 1 / 2 (levels with a ghost shell): only the units whose records name no ghost brick /
 // the others, so the first can run while an exchange fills the ghost bricks (part 1 on one CTA
 // slot per SM fewer, which the exchange's kernels then find free).
-static LevelLayout::PairTable pencil_table(const LevelLayout& L, int64_t b0, int64_t b1, int part = 0) {
+// kind 3: G = kPenCtas (sweep2p.cu, two-warp CTAs); kind 4: the same records dealt to G = kQuadCtas
+// one-warp CTAs (sweep2q.cu).
+static LevelLayout::PairTable pencil_table(const LevelLayout& L, int64_t b0, int64_t b1, int part = 0,
+                                           int kind = 3) {
   LevelLayout::PairTable t;
   t.kind = 0;
   const bool owned = b0 == 0 && b1 == L.n_owned;
@@ -506,12 +509,15 @@ static LevelLayout::PairTable pencil_table(const LevelLayout& L, int64_t b0, int
             if (par(m[(size_t)k]) != m[16] + k || (m[16] & 3) != 0) return t;
         layers[((size_t)py * tx + px) * nz + z] = m;
       }
-  t.kind = 3;
+  t.kind = kind;
   t.b0 = b0;
   t.b1 = b1;
   t.part = part;
   const int64_t ncol = (int64_t)tx * ty;
-  static const int64_t gmax = getenv("MG_PEN_CTAS") ? atoll(getenv("MG_PEN_CTAS")) : kPenCtas;  // (experiments)
+  static const int64_t gpen = getenv("MG_PEN_CTAS") ? atoll(getenv("MG_PEN_CTAS")) : kPenCtas;  // (experiments)
+  static const int64_t gquad = getenv("MG_QUAD_CTAS") ? atoll(getenv("MG_QUAD_CTAS")) : kQuadCtas;
+  const int64_t gmax = kind == 4 ? gquad : gpen;
+  const int64_t per_sm = kind == 4 ? kQuadCtasPerSm : kPenCtasPerSm;
   const int64_t G = std::max<int64_t>(1, std::min<int64_t>(gmax, ncol * nz));
   std::vector<std::vector<int32_t>> stream((size_t)G);  // per CTA: its chunk records
   // one 20-int record per chunk: code (type << 1 | half), the 16 brick ids, parent of b00
@@ -561,7 +567,7 @@ static LevelLayout::PairTable pencil_table(const LevelLayout& L, int64_t b0, int
       push_run(stream[(size_t)(u % G)], col, zr0(best, r), zr0(best, r + 1) - zr0(best, r));
     }
   } else {  // the units of one part, in the same order, dealt round-robin over Gp CTAs
-    const int64_t Gp = std::max<int64_t>(1, part == 1 ? G - G / kPenCtasPerSm : G);
+    const int64_t Gp = std::max<int64_t>(1, part == 1 ? G - G / per_sm : G);
     int64_t k = 0;
     std::vector<int32_t> run;
     for (int64_t u = 0; u < ncol * best; ++u) {
@@ -698,19 +704,19 @@ void build_pair_tables(LevelLayout& L, int64_t min_bricks, int kind) {
     if (dup) continue;
     LevelLayout::PairTable t;
     t.kind = 0;
-    if (kind == 3) t = pencil_table(L, r[0], r[1]);
+    if (kind == 3 || kind == 4) t = pencil_table(L, r[0], r[1], 0, kind);
     if (t.kind == 0) t = kind == 2 ? warp_table(L, r[0], r[1]) : pair_table(L, r[0], r[1]);
     if (t.kind != 0) L.pairs.push_back(std::move(t));
   }
   // pencil passes over a level with a ghost shell: the units split by whether they read a ghost
   // brick, for the overlap of the exchange with the interior units (both parts or neither)
-  if (kind == 3 && L.n_ghost > 0)
+  if ((kind == 3 || kind == 4) && L.n_ghost > 0)
     for (const int64_t b1 : {L.n_owned, L.n_stored}) {
       bool have = false;
-      for (const auto& c : L.pairs) have |= c.kind == 3 && c.part == 0 && c.b0 == 0 && c.b1 == b1;
+      for (const auto& c : L.pairs) have |= c.kind == kind && c.part == 0 && c.b0 == 0 && c.b1 == b1;
       if (!have) continue;
-      LevelLayout::PairTable p1 = pencil_table(L, 0, b1, 1), p2 = pencil_table(L, 0, b1, 2);
-      if (p1.kind != 3 || p2.kind != 3) continue;
+      LevelLayout::PairTable p1 = pencil_table(L, 0, b1, 1, kind), p2 = pencil_table(L, 0, b1, 2, kind);
+      if (p1.kind != kind || p2.kind != kind) continue;
       L.pairs.push_back(std::move(p1));
       L.pairs.push_back(std::move(p2));
     }

@@ -108,6 +108,9 @@ constexpr int kPenMeta = 20;  // host-side tile-layer item: the 16 ids, parent, 
 constexpr int kPenRec = 20;   // chunk record (80 bytes: one 1D bulk copy)
 constexpr int kPenCtasPerSm = 6;                    // resident pencil CTAs per SM (shared-memory bound)
 constexpr int64_t kPenCtas = 148 * kPenCtasPerSm;
+// kind 4 (sweep2q.cu): the same chunk records for one-warp CTAs
+constexpr int kQuadCtasPerSm = 8;                   // resident one-warp pencil CTAs per SM (27.5 KB each)
+constexpr int64_t kQuadCtas = 148 * kQuadCtasPerSm;
 constexpr int kW2Meta = 12;
 constexpr int kW2WarpsPerSm = 7;                    // resident one-warp CTAs per SM (shared-memory bound)
 constexpr int64_t kW2Streams = 148 * kW2WarpsPerSm * 2;

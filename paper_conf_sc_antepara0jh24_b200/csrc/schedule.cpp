@@ -32,7 +32,13 @@ bool Builder::has_pair_table(int l, int64_t b0, int64_t b1) const {
 
 bool Builder::pencil_table(int l) const {
   for (const auto& pt : lay.lv[l].pairs)
-    if (pt.b0 == 0 && pt.b1 == lay.lv[l].n_owned && pt.part == 0) return pt.kind == 3;
+    if (pt.b0 == 0 && pt.b1 == lay.lv[l].n_owned && pt.part == 0) return pt.kind == 3 || pt.kind == 4;
+  return false;
+}
+
+bool Builder::pair_zero_ok(int l) const {
+  for (const auto& pt : lay.lv[l].pairs)
+    if (pt.b0 == 0 && pt.b1 == lay.lv[l].n_owned && pt.part == 0) return pt.kind == 4;
   return false;
 }
 
@@ -40,7 +46,7 @@ bool Builder::pencil_ghosts(int l) const {
   const LevelLayout& L = lay.lv[l];
   if (L.n_ghost == 0) return false;
   for (const auto& pt : L.pairs)
-    if (pt.b0 == 0 && pt.b1 == L.n_stored && pt.part == 0) return pt.kind == 3;
+    if (pt.b0 == 0 && pt.b1 == L.n_stored && pt.part == 0) return pt.kind == 3 || pt.kind == 4;
   return false;
 }
 
@@ -81,8 +87,11 @@ void Builder::phase(int l, int n, bool zero_first, int last, bool interp_first, 
   const bool paper = fusion(l) == MG_FUSION_PAPER;
   const bool pairs = pair_ok(l);
   LevelState& S = st[l];
+  // the one-warp pencil kernel folds initZero into its first sweep (x0 == 0): the first pair of a
+  // coarse level's pre-smoothing needs no single sweep
+  const bool zero_pair = pairs && pair_zero_ok(l);
   for (int s = 0; s < nh; ++s) {
-    const bool single_only = (zero_first && s == 0) || (interp_first && s == 0);
+    const bool single_only = (zero_first && s == 0 && !zero_pair) || (interp_first && s == 0);
     if (pairs && !single_only && s + 1 < nh) {
       // sweeps s and s+1 in one pass (temporal blocking); x1 never leaves the chip
       Op o;
@@ -93,7 +102,8 @@ void Builder::phase(int l, int n, bool zero_first, int last, bool interp_first, 
       o.g2 = step(s + 1);
       o.c1 = colour(s);
       o.c2 = colour(s + 1);
-      const bool ex = g && (S.dx < 2 || S.since + 2 > k);
+      o.zero = zero_first && s == 0;  // the first sweep reads x0 == 0 (SW_ZERO_X)
+      const bool ex = g && !o.zero && (S.dx < 2 || S.since + 2 > k);
       if (ex) {
         S.dx = MG_MAX_PERIOD;
         S.since = 0;

@@ -37,7 +37,7 @@ struct Op {
   bool exch_before = false; // exchange x[src] ghosts before the sweep
   int field = 0;            // OP_EXCH: 0 = x[src], 1 = b
   int n = 0;                // OP_BOTTOM_RES: sweeps
-  bool zero = false;        // OP_BOTTOM_RES: x == 0 on entry
+  bool zero = false;        // OP_BOTTOM_RES: x == 0 on entry; OP_SWEEP2: the first sweep reads x0 == 0
   int timer = 0;            // MG_OP_*
   double g1 = 0, g2 = 0;    // smoothing steps of the (first, second) sweep; 0 = the level's Jacobi h^2/12
   int c1 = -1, c2 = -1;     // red-black colour of the (first, second) half-sweep (GSRB); -1 = every cell
@@ -63,7 +63,8 @@ struct Builder {
   int period(int l) const;
   bool pair_ok(int l) const;  // two-sweep passes possible at level l
   bool pencil_table(int l) const;  // the owned range of level l has a 2x2-brick pencil plan (kind 3)
-  bool pencil_ghosts(int l) const;  // ... and so has its whole stored range (owned + ghost shell)
+  bool pencil_ghosts(int l) const;
+  bool pair_zero_ok(int l) const;  // the owned range's pencil kernel folds x0 == 0 into a pair (kind 4)  // ... and so has its whole stored range (owned + ghost shell)
   bool pair_ghosts_ok(int l) const;  // two-sweep passes may include the ghost shell at level l
   bool has_pair_table(int l, int64_t b0, int64_t b1) const;
   // `n` smooth(+residual) sweeps at level l.  last: 0 none, 1 write r, 2 fused restriction.

@@ -13,8 +13,8 @@ from tests import brick_interp as bi
 FACE = [(-1, 0, 0), (1, 0, 0), (0, -1, 0), (0, 1, 0), (0, 0, -1), (0, 0, 1)]
 
 
-def layouts(n_local, proc_grid, L, ghost_mode=0):
-    p = mg.params(n_local, proc_grid, num_levels=L, ghost_mode=ghost_mode)
+def layouts(n_local, proc_grid, L, ghost_mode=0, **kw):
+    p = mg.params(n_local, proc_grid, num_levels=L, ghost_mode=ghost_mode, **kw)
     world = proc_grid[0] * proc_grid[1] * proc_grid[2]
     return p, [mg.Layout(p, r, world) for r in range(world)]
 
@@ -193,17 +193,19 @@ W_, E_, S_, N_, B_, T_ = range(6)
 @pytest.mark.parametrize("n_local,pg,L,gm", [((128, 128, 128), (1, 1, 1), 3, 0), ((256, 128, 64), (1, 1, 1), 2, 0),
                                             ((128, 128, 128), (1, 1, 1), 2, 1), ((128, 128, 128), (2, 1, 1), 2, 0),
                                             ((512, 512, 512), (1, 1, 1), 2, 0)])
-def test_pencil_plan_covers_owned_bricks(n_local, pg, L, gm):
+@pytest.mark.parametrize("tb", [3, 4])
+def test_pencil_plan_covers_owned_bricks(n_local, pg, L, gm, tb):
     """Every owned brick is swept exactly once per half by the pencil chunk streams; each record's
     16 ids are the tile layer's bricks and neighbours by the adjacency table; tiles sit on even
     brick coordinates (one coarse brick's x-y octants 0-3); runs are [warm-up, layers linked by T,
-    cool-down] with the B / T neighbour layers; every CTA gets the same work to within a run."""
-    p, lays = layouts(n_local, pg, L, gm)
+    cool-down] with the B / T neighbour layers; every CTA gets the same work to within a run.
+    tb = 3: two-warp CTAs (sweep2p.cu), tb = 4: the same records for one-warp CTAs (sweep2q.cu)."""
+    p, lays = layouts(n_local, pg, L, gm, temporal_blocking=tb)
     lay = lays[0]
     inf = lay.info(0)
     adj, crd = lay.adjacency(0), lay.coords(0)
     par = lay.parent(0) if L > 1 else None
-    allp = [pl for pl in lay.pass_plans(0) if pl[0] == 3]
+    allp = [pl for pl in lay.pass_plans(0) if pl[0] == tb]
     plans = [pl for pl in allp if pl[5] == 0]
     # the owned range (tiles on even owned coordinates: restriction), and with a ghost shell the
     # whole stored range (tiles on the extended box, ghost-sweeping passes)
