@@ -22,8 +22,8 @@
 //     commutative the canonical ((w+e)+(s+n))+(b+t) comes out bit for bit.
 //   * Stages are 2-plane units (the own x0 planes by 1D bulk copies, the 2-cell slabs of the 8 side
 //     neighbours, their b faces and the 4 diagonal corner columns by 3D tensor boxes) in a QD_ST-deep
-//     ring, one mbarrier per stage; b of the own cells by 128-bit loads two planes ahead into a
-//     plane-mod-4 register ring; the chunk records (brick ids) are read from global memory one record
+//     ring, one mbarrier per stage, b of the own cells with them (kept in registers for one more plane:
+//     the second sweep's b); the chunk records (brick ids) are read from global memory two records
 //     ahead (the issue side keeps one field per lane: lane l issues copy l).  No CTA barrier: the
 //     warp synchronises with __syncwarp.
 //   * initZero folded into the first sweep (SW_ZERO_X: x0 == 0, only b is staged), so the first
@@ -41,29 +41,34 @@ namespace mgb {
 
 namespace {
 
-constexpr int QD_ST = 3;    // stage ring depth (2-plane units): two units of lead
-constexpr int QD_MINB = 8;  // resident one-warp CTAs per SM (27.5 KB of shared memory each)
+constexpr int QD_ST = 2;    // stage ring depth (2-plane units): one unit (two planes) of lead
+constexpr int QD_MINB = 8;  // resident one-warp CTAs per SM (27 KB of shared memory each)
 // stage layout, offsets in doubles (tensor-copy destinations 128-byte aligned).  Own brick q (2
-// planes x 64) at qb(q): bricks 1 and 3 sit 16 B off modulo 128 from bricks 0 and 2.
-__host__ __device__ constexpr int qb(int q) { return 128 * q + 2 * (q & 1); }
-constexpr int QXW = 528, QXE = 592, QXS = 656, QXN = 720;  // x0 slabs, 2 boxes of 32 each (W0 W1 ...)
-constexpr int QBW = 784, QBE = 848, QBS = 912, QBN = 976;  // b faces, 2 boxes of 32 each
-constexpr int QCOR = 1040;                                 // SW, NW, SE, NE corner columns at +16 k
-constexpr int QSTAGE = 1104;
+// planes x 64) of x0 at qb(q), of b at QOB + qb(q): bricks 1 and 3 sit 16 B off modulo 128 from
+// bricks 0 and 2.
+__host__ __device__ constexpr int qb(int q) { return 272 * (q >> 1) + 130 * (q & 1); }
+constexpr int QOB = 544;                                    // own b bricks
+constexpr int QXW = 1088, QXE = 1152, QXS = 1216, QXN = 1280;  // x0 slabs, 2 boxes of 32 each (W0 W1 ...)
+constexpr int QBW = 1344, QBE = 1408, QBS = 1472, QBN = 1536;  // b faces, 2 boxes of 32 each
+constexpr int QCOR = 1600;                                     // SW, NW, SE, NE corner columns at +16 k
+constexpr int QSTAGE = 1664;
 // ring buffer of the ring cells' x1, per plane parity: W column rows j at RW + j, E rows at
 // RE + (j ^ 9), S row columns i at RS + i, N columns at RN + (i ^ 10).  The permutations make both
 // the ring stores (W rows 0-7 with E rows 0-7 per half warp) and the edge lanes' loads (rows of one
 // set, resp. the 128-bit column pairs) conflict-free.
 constexpr int QRW = 0, QRE = 16, QRS = 32, QRN = 48, QRPAR = 64;
 constexpr size_t QSMEM = (size_t)(QD_ST * QSTAGE + 2 * QRPAR) * 8 + QD_ST * 8;
-static_assert(QXW >= qb(3) + 128 && QXW % 16 == 0 && QBW % 16 == 0 && QCOR % 16 == 0 && QSTAGE % 16 == 0,
+static_assert(qb(1) >= qb(0) + 128 && qb(2) >= qb(1) + 128 && qb(3) >= qb(2) + 128 && qb(1) % 16 == 2 &&
+                  qb(2) % 16 == 0 && qb(3) % 16 == 2,
+              "own bricks: disjoint, bricks 1 and 3 16 B off modulo 128");
+static_assert(QOB >= qb(3) + 128 && QOB % 16 == 0 && QXW >= QOB + qb(3) + 128 && QXW % 16 == 0 && QBW % 16 == 0 && QCOR % 16 == 0 && QSTAGE % 16 == 0,
               "stage layout");
 static_assert(QXE == QXW + 64 && QXS == QXW + 128 && QXN == QXW + 192 && QBE == QBW + 64 && QBS == QBW + 128 &&
                   QBN == QBW + 192,
               "slab k lands at QXW + 32 k, b face k at QBW + 32 k");
 static_assert(QSMEM + 1024 <= 233472 / QD_MINB, "QD_MINB CTAs per SM must fit in shared memory");
-constexpr uint32_t QTX_X = 4 * 1024 + 8 * 256 + 4 * 32;  // own x0, x0 slabs, corners
-constexpr uint32_t QTX_B = 4 * 256 + 4 * 256;            // b faces W/E, S/N
+constexpr uint32_t QTX_X = 4 * 1024 + 8 * 256 + 4 * 32;           // own x0, x0 slabs, corners
+constexpr uint32_t QTX_B = 4 * 1024 + 4 * 256 + 4 * 256;            // own b, b faces W/E, S/N
 
 __device__ __forceinline__ double2 lds2(const double* p) { return *reinterpret_cast<const double2*>(p); }
 __device__ __forceinline__ int ldgi(const int32_t* p) { return __ldg(p); }
@@ -144,16 +149,19 @@ __global__ void __launch_bounds__(32, QD_MINB)
   const int oBr = sB ? QRN + (iB ^ 10) : QRS + iB;
   const int rcjB = sB ? 0 : 7;
 
-  // ---- producer: lane l issues copy l of a unit; it keeps field fld of the record it issues from ----
-  const int fld = l < 4 ? 1 + l : l < 12 ? l + 1 : l < 24 ? l - 7 : l == 24 ? 0 : 17;
+  // ---- producer: lane l issues copy l of a unit; it keeps field fld of the record it issues from
+  // (lanes 0-3 own x0, 4-11 x0 slabs, 12-19 b faces, 20-23 corners, 24-27 own b; lane 28 the code) ----
+  const int fld = l < 4 ? 1 + l : l < 12 ? l + 1 : l < 24 ? l - 7 : l < 28 ? l - 23 : l == 28 ? 0 : 17;
   if (l == 0) {
     for (int s = 0; s < QD_ST; ++s) mbar_init(&BAR[s], 1);
     mbar_fence_init();
   }
   __syncwarp();
   int irec = 0, isub = 0, issued = 0;
+  // this lane's field of the record being issued and of the two after it (loaded two records ahead)
   int fcur = ldgi(REC + fld), fnext = cnt > 1 ? ldgi(REC + kPenRec + fld) : 0;
-  int icode = __shfl_sync(FULL, fcur, 24);
+  int fnext2 = cnt > 2 ? ldgi(REC + 2 * kPenRec + fld) : 0;
+  int icode = __shfl_sync(FULL, fcur, 28);
   isub = ((icode >> 1) & 3) == WARM ? 1 : 0;
   auto issue_next = [&]() {  // uniform: stage unit (irec, isub) into stage issued % QD_ST
     const int s = issued % QD_ST, pl0 = 4 * (icode & 1) + 2 * isub;
@@ -179,6 +187,8 @@ __global__ void __launch_bounds__(32, QD_MINB)
     } else if (l < 24) {
       const int k = l - 20;  // SW (6,7), NW (6,0), SE (0,7), NE (0,0)
       if (!ZX) tma_load_3d(D + QCOR + 16 * k, &mp.xcor, k < 2 ? 6 : 0, (k & 1) ? 0 : 7, kz, &BAR[s]);
+    } else if (l < 28) {
+      tma_load_1d_hint(D + QOB + qb(l - 24), p.b + (int64_t)fcur * 512 + 64 * pl0, 1024, &BAR[s], pol_keep);
     }
     ++issued;
     if (((icode >> 1) & 3) == RANGE && isub == 0) {
@@ -186,8 +196,9 @@ __global__ void __launch_bounds__(32, QD_MINB)
     } else {
       ++irec;
       fcur = fnext;
-      fnext = irec + 1 < cnt ? ldgi(REC + (int64_t)(irec + 1) * kPenRec + fld) : 0;
-      icode = __shfl_sync(FULL, fcur, 24);
+      fnext = fnext2;
+      fnext2 = irec + 2 < cnt ? ldgi(REC + (int64_t)(irec + 2) * kPenRec + fld) : 0;
+      icode = __shfl_sync(FULL, fcur, 28);
       isub = ((icode >> 1) & 3) == WARM ? 1 : 0;
     }
   };
@@ -196,7 +207,7 @@ __global__ void __launch_bounds__(32, QD_MINB)
   auto wait_unit = [&](int u) { mbar_wait(&BAR[u % QD_ST], (uint32_t)((u / QD_ST) & 1)); };
 
   // ---- registers: rings indexed by plane mod 4 (the step's kk, compile-time) ----
-  double2 XR[4][2][2], YR[4][2][2], BR[4][2][2];  // [plane slot][set][column pair]
+  double2 XR[4][2][2], YR[4][2][2], BR[2][2][2];  // [plane slot (b: plane parity)][set][column pair]
   double RA[4], RBc[4];                           // ring cells' x0 windows
   double rpart[2] = {0.0, 0.0};
 #pragma unroll
@@ -205,18 +216,11 @@ __global__ void __launch_bounds__(32, QD_MINB)
 #pragma unroll
     for (int s = 0; s < 2; ++s)
 #pragma unroll
-      for (int h = 0; h < 2; ++h) XR[k][s][h] = YR[k][s][h] = BR[k][s][h] = make_double2(0.0, 0.0);
+      for (int h = 0; h < 2; ++h) XR[k][s][h] = YR[k][s][h] = BR[k & 1][s][h] = make_double2(0.0, 0.0);
   }
-  auto load_b = [&](double2(&dst)[2][2], int id, int code, int kk2) {
-    const double* bp = p.b + (int64_t)id * 512 + 64 * (4 * (code & 1) + kk2) + ib;
-#pragma unroll
-    for (int s = 0; s < 2; ++s) {
-      dst[s][0] = ld_hint2(bp + 8 * jb[s], pol_keep);  // the neighbour tiles' b-face copies reuse these lines
-      dst[s][1] = ld_hint2(bp + 8 * jb[s] + 2, pol_keep);
-    }
-  };
   // compute-side records: current, next, the one after (prefetched), previous
   int codeC = 0, idC = 0, parC = 0, codeN = 0, idN = 0, parN = 0, codeN2 = 0, idN2 = 0, parN2 = 0;
+  (void)idN;
   int codeP = 0, idP = 0, parP = 0;
   auto ldrec = [&](int n, int& code, int& id, int& par) {
     if (n < cnt) {
@@ -256,14 +260,12 @@ __global__ void __launch_bounds__(32, QD_MINB)
       RA[kk] = ZX ? 0.0 : S0[oAc + 16];
       RBc[km1] = ZX ? 0.0 : S0[oBc];
       RBc[kk] = ZX ? 0.0 : S0[oBc + 16];
-      load_b(BR[kk], idC, codeC, kk);
-      load_b(BR[kp], idN, codeN, 0);
     }
-    // b of plane g + 2
-    if (!cool) {
-      if (kk + 2 < 4) load_b(BR[km2], idC, codeC, kk + 2);
-      else load_b(BR[km2], idN, codeN, kk - 2);
-    }
+    // b of the own cells, plane g (kept for sweep 2 of the next step)
+#pragma unroll
+    for (int s = 0; s < 2; ++s)
+#pragma unroll
+      for (int h = 0; h < 2; ++h) BR[kk & 1][s][h] = lds2(S0 + QOB + oOwn[s] + 64 * pl0 + 2 * h);
     const int kz1 = 4 * (codeC & 1) + kk;  // in-brick plane of g (red-black colour)
 
     // ---------------- sweep 1, own cells, plane g ----------------
@@ -286,7 +288,7 @@ __global__ void __launch_bounds__(32, QD_MINB)
         const double wl = __shfl_up_sync(FULL, X[s][1].y, 1), er = __shfl_down_sync(FULL, X[s][0].x, 1);
         const double W = edW ? ed[s] : wl, E = edE ? ed[s] : er;
         const double c0 = X[s][0].x, c1 = X[s][0].y, c2 = X[s][1].x, c3 = X[s][1].y;
-        const double2 o0 = X[s ^ 1][0], o1 = X[s ^ 1][1], b0 = BR[kk][s][0], b1 = BR[kk][s][1];
+        const double2 o0 = X[s ^ 1][0], o1 = X[s ^ 1][1], b0 = BR[kk & 1][s][0], b1 = BR[kk & 1][s][1];
         // (s, n) = (outside, other set): for an odd row that is (n, s) -- same bits (a + b == b + a)
         const double a0 = stencil_a(c0, W, c1, xo[s][0].x, o0.x, Xm[s][0].x, Xp[s][0].x, alpha, beta);
         const double a1 = stencil_a(c1, c0, c2, xo[s][0].y, o0.y, Xm[s][0].y, Xp[s][0].y, alpha, beta);
@@ -357,7 +359,7 @@ __global__ void __launch_bounds__(32, QD_MINB)
         const double wl = __shfl_up_sync(FULL, Yc[s][1].y, 1), er = __shfl_down_sync(FULL, Yc[s][0].x, 1);
         const double W = edW ? e2[s] : wl, E = edE ? e2[s] : er;
         const double c0 = Yc[s][0].x, c1 = Yc[s][0].y, c2 = Yc[s][1].x, c3 = Yc[s][1].y;
-        const double2 o0 = Yc[s ^ 1][0], o1 = Yc[s ^ 1][1], b0 = BR[km1][s][0], b1 = BR[km1][s][1];
+        const double2 o0 = Yc[s ^ 1][0], o1 = Yc[s ^ 1][1], b0 = BR[(kk + 1) & 1][s][0], b1 = BR[(kk + 1) & 1][s][1];
         const double a0 = stencil_a(c0, W, c1, yo[s][0].x, o0.x, Ym[s][0].x, Y[s][0].x, alpha, beta);
         const double a1 = stencil_a(c1, c0, c2, yo[s][0].y, o0.y, Ym[s][0].y, Y[s][0].y, alpha, beta);
         const double a2 = stencil_a(c2, c1, c3, yo[s][1].x, o1.x, Ym[s][1].x, Y[s][1].x, alpha, beta);
