@@ -149,47 +149,49 @@ __global__ void __launch_bounds__(32, QD_MINB)
   const int oBr = sB ? QRN + (iB ^ 10) : QRS + iB;
   const int rcjB = sB ? 0 : 7;
 
-  // ---- producer: lane l issues copy l of a unit; it keeps field fld of the record it issues from
-  // (lanes 0-3 own x0, 4-11 x0 slabs, 12-19 b faces, 20-23 corners, 24-27 own b; lane 28 the code) ----
-  const int fld = l < 4 ? 1 + l : l < 12 ? l + 1 : l < 24 ? l - 7 : l < 28 ? l - 23 : l == 28 ? 0 : 17;
+  // ---- producer: lane 0 issues every copy of a unit in straight-line code (per-lane operands of
+  // the TMA instructions would make the compiler loop over the issuing lanes); lane f keeps field
+  // f + 1 of the record being issued (f < 17: the 16 brick ids and the parent), lane 17 the code,
+  // prefetched two records ahead ----
+  const int fld = l < 17 ? l + 1 : 0;
   if (l == 0) {
     for (int s = 0; s < QD_ST; ++s) mbar_init(&BAR[s], 1);
     mbar_fence_init();
   }
   __syncwarp();
   int irec = 0, isub = 0, issued = 0;
-  // this lane's field of the record being issued and of the two after it (loaded two records ahead)
   int fcur = ldgi(REC + fld), fnext = cnt > 1 ? ldgi(REC + kPenRec + fld) : 0;
   int fnext2 = cnt > 2 ? ldgi(REC + 2 * kPenRec + fld) : 0;
-  int icode = __shfl_sync(FULL, fcur, 28);
+  int icode = __shfl_sync(FULL, fcur, 17);
   isub = ((icode >> 1) & 3) == WARM ? 1 : 0;
   auto issue_next = [&]() {  // uniform: stage unit (irec, isub) into stage issued % QD_ST
     const int s = issued % QD_ST, pl0 = 4 * (icode & 1) + 2 * isub;
     double* D = ST + s * QSTAGE;
+    int id[16];
+#pragma unroll
+    for (int f = 0; f < 16; ++f) id[f] = __shfl_sync(FULL, fcur, f);  // b00 b10 b01 b11 W0 W1 E0 E1 S0 S1 N0 N1 SW NW SE NE
     fence_proxy_async();  // this lane's generic reads of the stage are ordered before the refill
     __syncwarp();
-    if (l == 0) mbar_expect_tx(&BAR[s], ZX ? QTX_B : QTX_X + QTX_B);
-    __syncwarp();
-    const int kz = fcur * 8 + pl0;
-    if (l < 4) {
-      // evict_last: the neighbour tiles' slab copies read these bricks' faces shortly after
-      if (!ZX) tma_load_1d_hint(D + qb(l), p.x + (int64_t)fcur * 512 + 64 * pl0, 1024, &BAR[s], pol_keep);
-    } else if (l < 12) {
-      const int k = l - 4;  // W0 W1 E0 E1 S0 S1 N0 N1: the W / S boxes sit at the neighbour's high face
-      const bool xf = k < 4, low = (k & 2) == 0;
-      if (!ZX) tma_load_3d(D + QXW + 32 * k, xf ? &mp.xwe : &mp.xsn, xf && low ? 6 : 0, !xf && low ? 6 : 0, kz, &BAR[s]);
-    } else if (l < 16) {
-      const int k = l - 12;
-      tma_load_3d(D + QBW + 32 * k, &mp.bwe, k < 2 ? 6 : 0, 0, kz, &BAR[s]);
-    } else if (l < 20) {
-      const int k = l - 16;
-      tma_load_3d(D + QBS + 32 * k, &mp.bsn, 0, k < 2 ? 6 : 0, kz, &BAR[s]);
-    } else if (l < 24) {
-      const int k = l - 20;  // SW (6,7), NW (6,0), SE (0,7), NE (0,0)
-      if (!ZX) tma_load_3d(D + QCOR + 16 * k, &mp.xcor, k < 2 ? 6 : 0, (k & 1) ? 0 : 7, kz, &BAR[s]);
-    } else if (l < 28) {
-      tma_load_1d_hint(D + QOB + qb(l - 24), p.b + (int64_t)fcur * 512 + 64 * pl0, 1024, &BAR[s], pol_keep);
+    if (l == 0) {
+      mbar_expect_tx(&BAR[s], ZX ? QTX_B : QTX_X + QTX_B);
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        // evict_last: the neighbour tiles' slab copies read these bricks' faces shortly after
+        if (!ZX) tma_load_1d_hint(D + qb(q), p.x + (int64_t)id[q] * 512 + 64 * pl0, 1024, &BAR[s], pol_keep);
+        tma_load_1d_hint(D + QOB + qb(q), p.b + (int64_t)id[q] * 512 + 64 * pl0, 1024, &BAR[s], pol_keep);
+      }
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {  // W0 W1 E0 E1 S0 S1 N0 N1: the W / S boxes sit at the neighbour's high face
+        const bool xf = k < 4, low = (k & 2) == 0;
+        const int kz = id[4 + k] * 8 + pl0;
+        if (!ZX) tma_load_3d(D + QXW + 32 * k, xf ? &mp.xwe : &mp.xsn, xf && low ? 6 : 0, !xf && low ? 6 : 0, kz, &BAR[s]);
+        tma_load_3d(D + QBW + 32 * k, xf ? &mp.bwe : &mp.bsn, xf && low ? 6 : 0, !xf && low ? 6 : 0, kz, &BAR[s]);
+      }
+#pragma unroll
+      for (int k = 0; k < 4; ++k)  // SW (6,7), NW (6,0), SE (0,7), NE (0,0)
+        if (!ZX) tma_load_3d(D + QCOR + 16 * k, &mp.xcor, k < 2 ? 6 : 0, (k & 1) ? 0 : 7, id[12 + k] * 8 + pl0, &BAR[s]);
     }
+    __syncwarp();
     ++issued;
     if (((icode >> 1) & 3) == RANGE && isub == 0) {
       isub = 1;
@@ -198,7 +200,7 @@ __global__ void __launch_bounds__(32, QD_MINB)
       fcur = fnext;
       fnext = fnext2;
       fnext2 = irec + 2 < cnt ? ldgi(REC + (int64_t)(irec + 2) * kPenRec + fld) : 0;
-      icode = __shfl_sync(FULL, fcur, 28);
+      icode = __shfl_sync(FULL, fcur, 17);
       isub = ((icode >> 1) & 3) == WARM ? 1 : 0;
     }
   };
