@@ -49,9 +49,9 @@ def parse():
     ap.add_argument("--ghost-all", action="store_true", help="self-exchange ghost shell on every axis")
     ap.add_argument("--no-graph", action="store_true")
     ap.add_argument("--no-overlap", action="store_true")
-    ap.add_argument("--tb", type=int, default=4,
-                    help="temporal blocking (two sweeps per HBM pass): 4 = 2x2-brick pencils, one warp per tile "
-                         "(sweep2q.cu, default), 3 = 2x2-brick pencils, two-warp CTAs (sweep2p.cu), 1 = one-brick "
+    ap.add_argument("--tb", type=int, default=3,
+                    help="temporal blocking (two sweeps per HBM pass): 3 = 2x2-brick pencils, two-warp CTAs (sweep2p.cu, "
+                         "default), 4 = 2x2-brick pencils, one warp per tile (sweep2q.cu), 1 = one-brick "
                          "CTA streams (sweep2.cu), 2 = warp plane streams (sweep2w.cu), 0 = off")
     ap.add_argument("--smoother", type=int, default=0,
                     help="0 damped Jacobi (the paper), 1 Chebyshev, 2 red-black Gauss-Seidel (N4 variants)")
@@ -352,8 +352,8 @@ def main():
     # the same level-0 work expressed as one-sweep-per-pass traffic (what the sweeps would move unblocked)
     sweep_equiv = pts * (B_SWEEP * nsweep0 + 2 * B_COARSE_PER_FINE) / (sweep0_ms / 1e3) / 1e9
     peak, peak_src = measured_peaks()
-    pass_kernel = {0: "sweep_col_kernel", 1: "sweep2_kernel", 2: "sweep2w_kernel", 3: "sweep2p_kernel"}.get(
-        a.tb, "sweep2q_kernel")
+    pass_kernel = {0: "sweep_col_kernel", 1: "sweep2_kernel", 2: "sweep2w_kernel", 4: "sweep2q_kernel"}.get(
+        a.tb, "sweep2p_kernel")
     traffic = ncu_traffic(n, pass_kernel)
     levels = []
     total_inst = sum(sum(r) for r in tm) / ninst
@@ -426,8 +426,8 @@ def main():
                                   4: "grid solve"}[a.bottom_mode],
                        "bottom_solver": "conjugate gradients" if a.bottom_solver else "damped jacobi (paper)",
                        "temporal_blocking": {0: "off", 1: "one-brick CTA streams", 2: "warp plane streams",
-                                             3: "2x2-brick pencils, two-warp CTAs"}.get(
-                           a.tb, "2x2-brick pencils, one warp per tile"),
+                                             4: "2x2-brick pencils, one warp per tile"}.get(
+                           a.tb, "2x2-brick pencils, two-warp CTAs"),
                        "smoother": {1: "chebyshev", 2: "red-black gauss-seidel"}.get(a.smoother, "damped jacobi (paper)"),
                        "l2": "no flush: every level-0 field is 1 GiB > 126 MB L2 (inputs larger than L2)",
                        "parallelism": f"3D domain decomposition {pg[0]}x{pg[1]}x{pg[2]}"},

@@ -435,7 +435,7 @@ mg_status sweep_range(mg_ctx* c, const Op& o, int64_t b0, int64_t b1, cudaStream
         if (pr.args.kind == 4)
           CKC(c, launch_sweep2q(a, pr.args, d.qmaps[o.src], o.flags | (o.zero ? SW_ZERO_X : 0u), s));
         else if (pr.args.kind == 3)
-          CKC(c, launch_sweep2p(a, pr.args, d.nmaps[o.src], o.flags, s));
+          CKC(c, launch_sweep2p(a, pr.args, d.nmaps[o.src], o.flags | (o.zero ? SW_ZERO_X : 0u), s));
         else if (pr.args.kind == 2)
           CKC(c, launch_sweep2w(a, pr.args, d.pmaps[o.src], o.flags, s));
         else
@@ -867,7 +867,7 @@ void mg_params_default(mg_params* p) {
   p->bottom_smooths = 100;
   p->use_graph = 1;
   p->overlap = 1;
-  p->temporal_blocking = 4;
+  p->temporal_blocking = 3;
   p->h0 = 0.0;
 }
 

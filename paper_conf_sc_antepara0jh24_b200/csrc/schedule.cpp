@@ -38,7 +38,7 @@ bool Builder::pencil_table(int l) const {
 
 bool Builder::pair_zero_ok(int l) const {
   for (const auto& pt : lay.lv[l].pairs)
-    if (pt.b0 == 0 && pt.b1 == lay.lv[l].n_owned && pt.part == 0) return pt.kind == 4;
+    if (pt.b0 == 0 && pt.b1 == lay.lv[l].n_owned && pt.part == 0) return pt.kind == 3 || pt.kind == 4;
   return false;
 }
 

@@ -63,8 +63,8 @@ struct Builder {
   int period(int l) const;
   bool pair_ok(int l) const;  // two-sweep passes possible at level l
   bool pencil_table(int l) const;  // the owned range of level l has a 2x2-brick pencil plan (kind 3)
-  bool pencil_ghosts(int l) const;
-  bool pair_zero_ok(int l) const;  // the owned range's pencil kernel folds x0 == 0 into a pair (kind 4)  // ... and so has its whole stored range (owned + ghost shell)
+  bool pencil_ghosts(int l) const;  // ... and so has its whole stored range (owned + ghost shell)
+  bool pair_zero_ok(int l) const;   // the owned range's pencil kernel folds x0 == 0 into a pair (SW_ZERO_X)
   bool pair_ghosts_ok(int l) const;  // two-sweep passes may include the ghost shell at level l
   bool has_pair_table(int l, int64_t b0, int64_t b1) const;
   // `n` smooth(+residual) sweeps at level l.  last: 0 none, 1 write r, 2 fused restriction.

@@ -77,8 +77,13 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
   constexpr bool WRITE_R = (FLAGS & SW_WRITE_R) != 0;
   constexpr bool RESTRICT = (FLAGS & SW_RESTRICT) != 0;
   constexpr bool COLOUR = (FLAGS & SW_COLOUR) != 0;  // red-black half-sweeps (GSRB variant)
+  constexpr bool ZX = (FLAGS & SW_ZERO_X) != 0;      // x0 == 0: initZero folded into the first sweep
   constexpr unsigned FULL = 0xffffffffu;
   constexpr int RANGE = 0, WARM = 1, COOL = 2;
+  // x0 read from the stage, or 0 (ZX: nothing of x0 is staged; every sweep-1 operand is +0, so the
+  // first sweep computes the canonical expression on zeros, exactly what initZero + a sweep compute)
+  auto x0d = [&](const double* a) { return ZX ? 0.0 : *a; };
+  auto x0d2 = [&](const double* a) { return ZX ? make_double2(0.0, 0.0) : lds_d2(a); };
   extern __shared__ __align__(128) unsigned char smem_raw[];
   double* const ST = reinterpret_cast<double*>(smem_raw);  // [PN_ST][STAGE]
   double* const XP = ST + PN_ST * STAGE;                    // x1 of tile rows -1..16 (layout above)
@@ -169,11 +174,14 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     double* D = ST + s * STAGE;
     fence_proxy_async();
     if (l == 0)
-      mbar_expect_tx(&BAR[s], w == 0 ? 4 * 2048 + 8 * 512 : 4 * 512 + 4 * 256 + 4 * 64 + (rec ? kPenRec * 4 : 0));
+      mbar_expect_tx(&BAR[s], w == 0 ? (ZX ? 0 : 4 * 2048 + 8 * 512)
+                                     : 4 * 512 + 4 * 256 + (ZX ? 0 : 4 * 64) + (rec ? kPenRec * 4 : 0));
     __syncwarp();
     const int kz = id * 8 + 4 * half;
     if (w == 0) {
-      if (l < 4) {
+      if (ZX) {
+        // nothing of x0 is staged
+      } else if (l < 4) {
         // evict_last: the neighbour tiles' slab copies read these bricks' faces shortly after
         tma_load_1d_hint(D + OWN_STRIDE * l, p.x + (int64_t)id * 512 + 256 * half, 2048, &BAR[s], pol_keep);
       } else if (l < 12) {
@@ -188,7 +196,7 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
         tma_load_3d(D + BS + 32 * (l - 4), &mp.bsn, 0, l < 6 ? 7 : 0, kz, &BAR[s]);
       } else if (l < 12) {  // SW (6,7), NW (6,0), SE (0,7), NE (0,0)
         const int cc = l - 8;
-        tma_load_3d(D + COR + 16 * cc, &mp.xcor, cc < 2 ? 6 : 0, (cc & 1) ? 0 : 7, kz, &BAR[s]);
+        if (!ZX) tma_load_3d(D + COR + 16 * cc, &mp.xcor, cc < 2 ? 6 : 0, (cc & 1) ? 0 : 7, kz, &BAR[s]);
       } else if (l == 12 && rec) {  // slot (n+1) % 4 held record n-3, consumed long ago
         tma_load_1d(MR + ((n + 1) % MRS) * kPenRec, REC + (int64_t)(n + 1) * kPenRec, kPenRec * 4, &BAR[s]);
       }
@@ -246,10 +254,10 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     double& rc = RR[kk];
     double& rcp = RR[kp];
     if (start) {  // first step of a run (warm-up plane 7): prime the register windows
-      Xm[0] = lds_d2(S0 + oO + 64 * (kk - 1)), Xm[1] = lds_d2(S0 + oO + 8 + 64 * (kk - 1));
-      Xc[0] = lds_d2(S0 + oO + 64 * kk), Xc[1] = lds_d2(S0 + oO + 8 + 64 * kk);
-      rcm = S0[oc + 16 * (kk - 1)];
-      rc = S0[oc + 16 * kk];
+      Xm[0] = x0d2(S0 + oO + 64 * (kk - 1)), Xm[1] = x0d2(S0 + oO + 8 + 64 * (kk - 1));
+      Xc[0] = x0d2(S0 + oO + 64 * kk), Xc[1] = x0d2(S0 + oO + 8 + 64 * kk);
+      rcm = x0d(S0 + oc + 16 * (kk - 1));
+      rc = x0d(S0 + oc + 16 * kk);
       // b of this plane and of the next chunk's planes 0-2 (plane 3 follows below)
       load_b(BR[bc], idC, codeC, kk);
 #pragma unroll
@@ -260,12 +268,12 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     const int kz1 = 4 * (codeC & 1) + kk;  // in-brick plane of g (red-black colour)
 
     // ---------------- sweep 1, own cells, plane g ----------------
-    Xp[0] = lds_d2(S1 + oO + 64 * kp);
-    Xp[1] = lds_d2(S1 + oO + 8 + 64 * kp);
+    Xp[0] = x0d2(S1 + oO + 64 * kp);
+    Xp[1] = x0d2(S1 + oO + 8 + 64 * kp);
     {
-      const double2 xs = lds_d2(S0 + oS + sS * kk), xn = lds_d2(S0 + oN + sN * kk);
+      const double2 xs = x0d2(S0 + oS + sS * kk), xn = x0d2(S0 + oN + sN * kk);
       // tile-edge x0 (inner lanes read the W edge lane's words: broadcasts, no extra wavefronts)
-      const double e0 = S0[oEd + 16 * kk], e1 = S0[oEd + 2 + 16 * kk];
+      const double e0 = x0d(S0 + oEd + 16 * kk), e1 = x0d(S0 + oEd + 2 + 16 * kk);
       const double wl0 = __shfl_up_sync(FULL, Xc[0].y, 1), er0 = __shfl_down_sync(FULL, Xc[0].x, 1);
       const double wl1 = __shfl_up_sync(FULL, Xc[1].y, 1), er1 = __shfl_down_sync(FULL, Xc[1].x, 1);
       const double W0 = edW ? e0 : wl0, E0 = edE ? e0 : er0, W1 = edW ? e1 : wl1, E1 = edE ? e1 : er1;
@@ -284,9 +292,9 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
     }
     // ---------------- sweep 1, ring cell, plane g ----------------
     {
-      rcp = S1[oc + 16 * kp];
-      const double o = S0[oo + 16 * kk], own = S0[oown + 64 * kk];
-      const double lo = S0[olo + slo * kk], hi = S0[ohi + shi * kk], bv = S0[ob + sb * kk];
+      rcp = x0d(S1 + oc + 16 * kp);
+      const double o = x0d(S0 + oo + 16 * kk), own = x0d(S0 + oown + 64 * kk);
+      const double lo = x0d(S0 + olo + slo * kk), hi = x0d(S0 + ohi + shi * kk), bv = S0[ob + sb * kk];
       // ((o + own) + (lo + hi)) + (b + t): the canonical ((w+e)+(s+n))+(b+t) up to the order of
       // the operands of single additions (IEEE addition is commutative, so bit for bit equal)
       const double sum = DADD(DADD(DADD(o, own), DADD(lo, hi)), DADD(rcm, rcp));
@@ -381,7 +389,7 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
 }
 
 bool pencil_supports(unsigned flags) {
-  const unsigned fl = flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP | SW_ZERO_X);
+  const unsigned fl = flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP);
   return fl == 0 || fl == SW_WRITE_R || fl == SW_RESTRICT;
 }
 
@@ -395,6 +403,12 @@ cudaError_t encode_pencil_maps(const double* x, const double* b, int64_t n_alloc
   return encode_box_map(b, n_alloc, sn1, &out->bsn);
 }
 
+// every supported flag combination: {plain, +r, +restriction} x {colour} x {x0 == 0 in the first sweep}
+#define PENCIL_FLAG_LIST(X)                                                                              \
+  X(0) X(SW_WRITE_R) X(SW_RESTRICT) X(SW_COLOUR) X(SW_WRITE_R | SW_COLOUR) X(SW_RESTRICT | SW_COLOUR)   \
+  X(SW_ZERO_X) X(SW_ZERO_X | SW_WRITE_R) X(SW_ZERO_X | SW_RESTRICT) X(SW_ZERO_X | SW_COLOUR)             \
+  X(SW_ZERO_X | SW_WRITE_R | SW_COLOUR) X(SW_ZERO_X | SW_RESTRICT | SW_COLOUR)
+
 cudaError_t launch_sweep2p(const SweepArgs& a, const PairArgs& pa, const PairMaps& pm, unsigned flags,
                            cudaStream_t s) {
   if (pa.nctas <= 0) return cudaSuccess;
@@ -402,31 +416,30 @@ cudaError_t launch_sweep2p(const SweepArgs& a, const PairArgs& pa, const PairMap
   const size_t sm = SMEM_BYTES;
   const unsigned col = (a.colour >= 0 || a.colour2 >= 0) ? SW_COLOUR : 0u;
   switch ((flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP | SW_ZERO_X)) | col) {
-    case 0: launch_plain(sweep2p_kernel<0>, g, PN_THREADS, sm, s, a, pa, pm); break;
-    case SW_WRITE_R: launch_plain(sweep2p_kernel<SW_WRITE_R>, g, PN_THREADS, sm, s, a, pa, pm); break;
-    case SW_RESTRICT: launch_plain(sweep2p_kernel<SW_RESTRICT>, g, PN_THREADS, sm, s, a, pa, pm); break;
-    case SW_COLOUR: launch_plain(sweep2p_kernel<SW_COLOUR>, g, PN_THREADS, sm, s, a, pa, pm); break;
-    case SW_WRITE_R | SW_COLOUR: launch_plain(sweep2p_kernel<SW_WRITE_R | SW_COLOUR>, g, PN_THREADS, sm, s, a, pa, pm); break;
-    case SW_RESTRICT | SW_COLOUR:
-      launch_plain(sweep2p_kernel<SW_RESTRICT | SW_COLOUR>, g, PN_THREADS, sm, s, a, pa, pm);
-      break;
-    default: return cudaErrorInvalidValue;
+#define PENCIL_CASE(F)                                                      \
+  case (F):                                                                 \
+    launch_plain(sweep2p_kernel<(F)>, g, PN_THREADS, sm, s, a, pa, pm); \
+    break;
+    PENCIL_FLAG_LIST(PENCIL_CASE)
+#undef PENCIL_CASE
+    default:
+      return cudaErrorInvalidValue;
   }
   return cudaGetLastError();
 }
 
 cudaError_t pencil_kernels_init() {
-  const void* k[6] = {(const void*)sweep2p_kernel<0>, (const void*)sweep2p_kernel<SW_WRITE_R>,
-                      (const void*)sweep2p_kernel<SW_RESTRICT>, (const void*)sweep2p_kernel<SW_COLOUR>,
-                      (const void*)sweep2p_kernel<SW_WRITE_R | SW_COLOUR>,
-                      (const void*)sweep2p_kernel<SW_RESTRICT | SW_COLOUR>};
-  for (int i = 0; i < 6; ++i) {
-    cudaError_t e = cudaFuncSetAttribute(k[i], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM_BYTES);
-    if (e != cudaSuccess) return e;
-    e = cudaFuncSetAttribute(k[i], cudaFuncAttributePreferredSharedMemoryCarveout, 100);
-    if (e != cudaSuccess) return e;
-  }
-  return cudaSuccess;
+  cudaError_t e = cudaSuccess;
+#define PENCIL_ATTR(F)                                                                                      \
+  if ((e = cudaFuncSetAttribute(sweep2p_kernel<(F)>, cudaFuncAttributeMaxDynamicSharedMemorySize,          \
+                                (int)SMEM_BYTES)) != cudaSuccess)                                           \
+    return e;                                                                                               \
+  if ((e = cudaFuncSetAttribute(sweep2p_kernel<(F)>, cudaFuncAttributePreferredSharedMemoryCarveout, 100)) != \
+      cudaSuccess)                                                                                          \
+    return e;
+  PENCIL_FLAG_LIST(PENCIL_ATTR)
+#undef PENCIL_ATTR
+  return e;
 }
 
 }  // namespace mgb

@@ -153,7 +153,7 @@ def check(status: int, where: str) -> int:
 
 def params(n_local, proc_grid=(1, 1, 1), num_levels=6, pre=12, post=12, bottom=100, ca_period=None, fusion=None,
            ghost_mode=MG_GHOST_AUTO, transport=MG_TRANSPORT_AUTO, use_graph=1, bottom_mode=MG_BOTTOM_AUTO,
-           overlap=1, h0=0.0, sweep_kernel=0, temporal_blocking=4, smoother=0, cheby_ratio=0, launch_pdl=0, bottom_solver=0) -> mg_params:
+           overlap=1, h0=0.0, sweep_kernel=0, temporal_blocking=3, smoother=0, cheby_ratio=0, launch_pdl=0, bottom_solver=0) -> mg_params:
     p = mg_params()
     lib().mg_params_default(ctypes.byref(p))
     p.n_local[:] = [int(v) for v in n_local]

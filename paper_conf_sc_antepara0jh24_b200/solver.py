@@ -24,7 +24,7 @@ class Multigrid:
     def __init__(self, n_local, proc_grid=(1, 1, 1), num_levels=6, pre=12, post=12, bottom=100, ca_period=None,
                  fusion=None, ghost_mode=mg.MG_GHOST_AUTO, transport=mg.MG_TRANSPORT_AUTO, use_graph=True,
                  bottom_mode=mg.MG_BOTTOM_AUTO, overlap=True, h0=0.0, rank=0, world_size=1, device=None,
-                 stream: torch.cuda.Stream | None = None, sweep_kernel=0, temporal_blocking=4, smoother=0,
+                 stream: torch.cuda.Stream | None = None, sweep_kernel=0, temporal_blocking=3, smoother=0,
                  cheby_ratio=0, launch_pdl=0, bottom_solver=0):
         if not torch.cuda.is_available():
             raise RuntimeError("Multigrid needs a CUDA device (the library has no CPU fallback)")
@@ -149,7 +149,7 @@ class LoopbackGroup:
 
     def __init__(self, n_local, proc_grid, num_levels=6, pre=12, post=12, bottom=100, ca_period=None, fusion=None,
                  ghost_mode=mg.MG_GHOST_AUTO, use_graph=True, bottom_mode=mg.MG_BOTTOM_AUTO, overlap=True, h0=0.0,
-                 device=None, sweep_kernel=0, temporal_blocking=4, smoother=0, cheby_ratio=0, launch_pdl=0, bottom_solver=0):
+                 device=None, sweep_kernel=0, temporal_blocking=3, smoother=0, cheby_ratio=0, launch_pdl=0, bottom_solver=0):
         self.device = torch.device("cuda", torch.cuda.current_device() if device is None else int(device))
         torch.cuda.set_device(self.device)
         self.n_local = tuple(int(v) for v in n_local)
