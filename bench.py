@@ -47,6 +47,9 @@ def parse():
     ap.add_argument("--ca-period", type=int, default=0)
     ap.add_argument("--fusion", type=int, default=0)
     ap.add_argument("--ghost-all", action="store_true", help="self-exchange ghost shell on every axis")
+    ap.add_argument("--transport", choices=["auto", "nccl", "local"], default="auto",
+                    help="ghost exchange transport (auto: NCCL between processes, device copies for a one-rank "
+                         "self-exchange; nccl: NCCL send/recv even to itself)")
     ap.add_argument("--no-graph", action="store_true")
     ap.add_argument("--no-overlap", action="store_true")
     ap.add_argument("--tb", type=int, default=3,
@@ -257,6 +260,45 @@ def run_reference(a, rank, world):
     print(json.dumps(line), flush=True)
 
 
+# ------------------------------------------------------------------ exchanges
+NVLINK_GBS = 900.0  # NVLink 5: 900 GB/s per direction per GPU (B200_PROFILING.md; SURVEY §8(d))
+
+
+def exchange_block(m, a, world, max_over_ranks, tm, ninst):
+    """Per level: ghost exchanges per V-cycle, bytes per exchange, device time of one exchange (the
+    V-cycle's own transport, back to back, max over ranks), achieved GB/s and its fraction of the
+    NVLink per-direction bandwidth (between processes) -- plus the latency / bandwidth fit
+    t = alpha + bytes / beta over the levels (P:L216-236, N3) and the Table-II-style share of the
+    exchanges in the level time (P:L198-206)."""
+    counts, nbytes = m.exchange_plan()
+    if not any(nbytes):
+        return {"levels": [], "note": "no ghost shell (one rank, periodic wrap): no exchanges"}
+    transport = ("nccl" if (world > 1 or a.transport == "nccl") else "local device copies")
+    out = []
+    for l, (c, b) in enumerate(zip(counts, nbytes)):
+        if b <= 0:
+            continue
+        t = max_over_ranks(m.exchange_time(l, 20))
+        gbs = b / (t / 1e3) / 1e9 if t > 0 else None
+        lvl_ms = sum(tm[l]) / ninst if l < len(tm) else None
+        out.append({"level": l, "exchanges_per_cycle": c, "bytes_per_exchange": b, "ms_per_exchange": t,
+                    "gbs": gbs, "frac_of_nvlink_900": (gbs / NVLINK_GBS) if (gbs and world > 1) else None,
+                    "ms_per_cycle_if_serial": c * t,
+                    "share_of_level_time": (c * t / lvl_ms) if lvl_ms else None})
+    fit = None
+    pts = [(d["bytes_per_exchange"], d["ms_per_exchange"]) for d in out if d["ms_per_exchange"] > 0]
+    if len(pts) >= 2:
+        import numpy as np
+
+        X = np.array([[1.0, p[0]] for p in pts])
+        y = np.array([p[1] for p in pts])
+        (alpha, inv_beta), *_ = np.linalg.lstsq(X, y, rcond=None)
+        fit = {"alpha_us": alpha * 1e3, "beta_gbs": (1.0 / inv_beta / 1e6) if inv_beta > 0 else None,
+               "points": len(pts)}
+    return {"transport": transport, "levels": out, "fit": fit,
+            "link": "NVLink 5, 900 GB/s per direction" if world > 1 else "self-exchange on one GPU (no link)"}
+
+
 # ------------------------------------------------------------------ GPU arm
 def main():
     a = parse()
@@ -284,7 +326,9 @@ def main():
                   ghost_mode=1 if a.ghost_all else 0, use_graph=not a.no_graph, overlap=not a.no_overlap,
                   rank=rank, world_size=world, device=local, temporal_blocking=a.tb, smoother=a.smoother,
                   cheby_ratio=a.cheby_ratio, launch_pdl=2 if a.no_pdl else 0,
-                  bottom_mode=a.bottom_mode, bottom_solver=a.bottom_solver)
+                  bottom_mode=a.bottom_mode, bottom_solver=a.bottom_solver,
+                  transport={"auto": mg.MG_TRANSPORT_AUTO, "nccl": mg.MG_TRANSPORT_NCCL,
+                             "local": mg.MG_TRANSPORT_LOCAL}[a.transport])
     gshape = (n * pg[2], n * pg[1], n * pg[0])
     b_host = torch.from_numpy(mg_inputs.local_sin_rhs(gshape, rank, pg)).pin_memory()
     b_dev = b_host.to(dev)
@@ -409,6 +453,7 @@ def main():
 
     launches = m.launches_per_vcycle()
     xbytes, xmsgs = m.exchange_stats()
+    exchange = exchange_block(m, a, world, max_over_ranks, tm, ninst)
     cpu = None
     if rank == 0 and world == 1 and not a.no_cpu_baseline:
         cpu = cpu_baseline(a)
@@ -422,6 +467,7 @@ def main():
                        "fusion": "auto(full)" if not a.fusion else a.fusion,
                        "ca_period": a.ca_period or "auto(8)", "ghost_mode": "all" if a.ghost_all else "auto",
                        "cuda_graph": not a.no_graph, "overlap": not a.no_overlap, "pdl": not a.no_pdl,
+                       "transport": a.transport,
                        "coarse": {0: "auto", 1: "per-sweep launches", 2: "resident bottom", 3: "cluster solve",
                                   4: "grid solve"}[a.bottom_mode],
                        "bottom_solver": "conjugate gradients" if a.bottom_solver else "damped jacobi (paper)",
@@ -445,7 +491,7 @@ def main():
             "launches_per_step": launches,
             "clocks": clk,
             "final_residual_norm": norm,
-            "exchange": {"bytes_per_cycle_per_rank": xbytes, "messages_per_cycle_per_rank": xmsgs},
+            "exchange": dict(exchange, bytes_per_cycle_per_rank=xbytes, messages_per_cycle_per_rank=xmsgs),
             "levels": levels,
             "instrumented_ms_per_step": total_inst,
         }

@@ -211,6 +211,16 @@ mg_status mg_vcycle_launches(mg_ctx* c, int64_t* out);
 /* Exchange statistics: bytes this rank sends per V-cycle and message count. */
 mg_status mg_exchange_stats(mg_ctx* c, int64_t* bytes_per_cycle, int64_t* messages_per_cycle);
 
+/* Per level l < cap of the V-cycle mg_vcycle would run next: exchanges[l] = ghost exchanges (x before
+ * a sweep, b after the restriction), bytes[l] = bytes this rank sends in one exchange of the level
+ * (0 without a ghost shell).  Host-only, no device work. */
+mg_status mg_exchange_plan(mg_ctx* c, int32_t cap, int64_t* exchanges, int64_t* bytes);
+/* Device time of one ghost exchange of x at `level` (the V-cycle's transport: NCCL grouped
+ * send/recv of the brick runs, or the local copy kernel), averaged over `reps` back-to-back
+ * exchanges on the context's stream after one warm-up exchange (CUDA events; synchronises).
+ * Collective when the transport is NCCL.  0 for a level without a ghost shell.  Input of the
+ * bench's exchange block and of the exchange latency / bandwidth fit t = alpha + bytes / beta. */
+mg_status mg_exchange_time(mg_ctx* c, int32_t level, int32_t reps, double* ms_per_exchange);
 mg_status mg_destroy(mg_ctx* c);
 
 /* Thread-local description of the last error (never NULL). */

@@ -1138,6 +1138,45 @@ mg_status mg_exchange_stats(mg_ctx* c, int64_t* bytes_per_cycle, int64_t* messag
   return MG_OK;
 }
 
+mg_status mg_exchange_plan(mg_ctx* c, int32_t cap, int64_t* exchanges, int64_t* bytes) {
+  CKS(check_ctx(c));
+  if (cap < c->lay.L || !exchanges || !bytes) return set_err(MG_ERR_INVALID_ARG, "need cap >= num_levels and outputs");
+  Builder b(c->lay);
+  for (int l = 0; l < MG_MAX_LEVELS; ++l) b.st[l] = c->st[l];
+  b.vcycle();
+  for (int l = 0; l < c->lay.L; ++l) {
+    exchanges[l] = 0;
+    bytes[l] = 0;
+    for (const Run& r : c->lay.lv[l].sends) bytes[l] += r.count * kBV * (int64_t)sizeof(double);
+  }
+  for (const Op& o : b.ops)
+    if (o.kind == OP_EXCH || ((o.kind == OP_SWEEP || o.kind == OP_SWEEP2) && o.exch_before)) ++exchanges[o.level];
+  return MG_OK;
+}
+
+mg_status mg_exchange_time(mg_ctx* c, int32_t level, int32_t reps, double* ms_per_exchange) {
+  CKS(check_ctx(c));
+  if (c->group) return set_err(MG_ERR_STATE, "group member: not supported");
+  if (!ms_per_exchange || reps < 1 || level < 0 || level >= c->lay.L)
+    return set_err(MG_ERR_INVALID_ARG, "bad level / reps / output");
+  *ms_per_exchange = 0.0;
+  if (c->lay.lv[level].n_ghost == 0) return MG_OK;
+  // x of the level (its ghosts are refreshed: harmless for the V-cycle state, whose ghost validity
+  // only ever grows by an exchange)
+  const int xb = c->st[level].cur;
+  CKS(do_exchange(c, level, 0, xb, c->stream));  // warm-up (NCCL connection setup on first use)
+  cudaEvent_t e0 = pool_event(c), e1 = pool_event(c);
+  CKC(c, cudaEventRecord(e0, c->stream));
+  for (int i = 0; i < reps; ++i) CKS(do_exchange(c, level, 0, xb, c->stream));
+  CKC(c, cudaEventRecord(e1, c->stream));
+  CKC(c, cudaEventSynchronize(e1));
+  float ms = 0.f;
+  CKC(c, cudaEventElapsedTime(&ms, e0, e1));
+  c->evnext = 0;
+  *ms_per_exchange = (double)ms / reps;
+  return MG_OK;
+}
+
 mg_status mg_destroy(mg_ctx* c) {
   if (!c) return MG_OK;
   if (c->group) return set_err(MG_ERR_STATE, "group member: use mg_group_destroy");

@@ -86,6 +86,10 @@ _SIGS = {
     "mg_vcycle_launches": (ctypes.c_int, [ctypes.c_void_p, ctypes.POINTER(ctypes.c_int64)]),
     "mg_exchange_stats": (ctypes.c_int, [ctypes.c_void_p, ctypes.POINTER(ctypes.c_int64),
                                          ctypes.POINTER(ctypes.c_int64)]),
+    "mg_exchange_plan": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.POINTER(ctypes.c_int64),
+                                        ctypes.POINTER(ctypes.c_int64)]),
+    "mg_exchange_time": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32,
+                                        ctypes.POINTER(ctypes.c_double)]),
     "mg_destroy": (ctypes.c_int, [ctypes.c_void_p]),
     "mg_last_error": (ctypes.c_char_p, []),
     "mg_level_set": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32, ctypes.c_void_p]),
@@ -272,6 +276,19 @@ def mg_exchange_stats(ctx):
     b, m = ctypes.c_int64(), ctypes.c_int64()
     check(lib().mg_exchange_stats(ctx, ctypes.byref(b), ctypes.byref(m)), "mg_exchange_stats")
     return b.value, m.value
+
+
+def mg_exchange_plan(ctx, num_levels):
+    ex = (ctypes.c_int64 * num_levels)()
+    by = (ctypes.c_int64 * num_levels)()
+    check(lib().mg_exchange_plan(ctx, num_levels, ex, by), "mg_exchange_plan")
+    return list(ex), list(by)
+
+
+def mg_exchange_time(ctx, level, reps=20):
+    ms = ctypes.c_double()
+    check(lib().mg_exchange_time(ctx, level, reps, ctypes.byref(ms)), "mg_exchange_time")
+    return ms.value
 
 
 def mg_destroy(ctx):

@@ -143,6 +143,14 @@ class Multigrid:
     def exchange_stats(self):
         return mg.mg_exchange_stats(self.ctx)
 
+    def exchange_plan(self):
+        """([exchanges per V-cycle per level], [bytes this rank sends per exchange per level])."""
+        return mg.mg_exchange_plan(self.ctx, self.num_levels)
+
+    def exchange_time(self, level, reps=20) -> float:
+        """Device ms of one ghost exchange of x at `level` (collective over NCCL)."""
+        return mg.mg_exchange_time(self.ctx, level, reps)
+
 
 class LoopbackGroup:
     """world_size ranks of a proc_grid decomposition in one process on one GPU."""

@@ -811,3 +811,31 @@ def test_gsrb_smoother_loopback_bitwise(oracle_mod):
         assert_bitwise(host(g.get_solution(r)), mg_inputs.local_block(orc.get_x(), r, pg), what=f"rank {r}")
     g.close()
     orc.close()
+
+
+@pytest.mark.parametrize("transport", [2, 1])
+def test_exchange_plan_and_timing_keep_the_bits(oracle_mod, transport):
+    """mg_exchange_plan / mg_exchange_time (the bench's exchange block): a self-exchanged ghost shell
+    on every axis has exchanges on every level, the timing runs the V-cycle's own transport (local
+    copies / NCCL), and refreshing the ghosts in between leaves the V-cycle bitwise on the oracle."""
+    mg, _ = _mg()
+    shape = (64, 64, 64)
+    b = mg_inputs.random_rhs(shape, 41)
+    xs, ns = oracle_cycles(oracle_mod, b, 3, 2)
+    m = new(shape, 3, ghost_mode=1, transport=transport)
+    m.set_rhs(dev(b))
+    m.set_solution(None)
+    counts, nbytes = m.exchange_plan()
+    assert all(c > 0 for c in counts) and all(v > 0 for v in nbytes)
+    # one exchange of level 0 sends the whole surface shell: (8^3 - 6^3) bricks of 4 KiB
+    assert nbytes[0] == (8**3 - 6**3) * 4096
+    m.vcycle()
+    for l in range(3):
+        assert m.exchange_time(l, 3) > 0
+    nr = m.residual_norm()
+    assert nr == ns[0]
+    assert_bitwise(host(m.get_solution()), xs[0], what="x after cycle 1")
+    m.vcycle()
+    assert m.residual_norm() == ns[1]
+    assert_bitwise(host(m.get_solution()), xs[1], what="x after cycle 2")
+    m.close()
