@@ -827,8 +827,9 @@ def test_exchange_plan_and_timing_keep_the_bits(oracle_mod, transport):
     m.set_solution(None)
     counts, nbytes = m.exchange_plan()
     assert all(c > 0 for c in counts) and all(v > 0 for v in nbytes)
-    # one exchange of level 0 sends the whole surface shell: (8^3 - 6^3) bricks of 4 KiB
-    assert nbytes[0] == (8**3 - 6**3) * 4096
+    # one exchange of level 0 fills the whole one-brick ghost shell: 10^3 - 8^3 bricks of 4 KiB (a
+    # surface brick goes to every face / edge / corner direction it borders)
+    assert nbytes[0] == (10**3 - 8**3) * 4096
     m.vcycle()
     for l in range(3):
         assert m.exchange_time(l, 3) > 0
