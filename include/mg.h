@@ -84,7 +84,8 @@ enum {
 };
 
 /* transport */
-enum { MG_TRANSPORT_AUTO = 0, MG_TRANSPORT_NCCL = 1, MG_TRANSPORT_LOCAL = 2 };
+enum { MG_TRANSPORT_AUTO = 0, MG_TRANSPORT_NCCL = 1, MG_TRANSPORT_LOCAL = 2, MG_TRANSPORT_PEER = 3 };
+#define MG_PEER_BLOB_BYTES 128
 
 /* bottom_mode.  AUTO: a bottom level of <= 8 bricks without ghosts runs all its sweeps in one
  * CTA (resident), otherwise per-sweep launches.  CLUSTER (opt-in): the deepest
@@ -104,9 +105,14 @@ typedef struct {
   int32_t ca_period[MG_MAX_LEVELS]; /* sweeps per x-exchange per level, 1..8; 0 = auto (8) */
   int32_t fusion[MG_MAX_LEVELS];    /* MG_FUSION_*; 0 = auto */
   int32_t ghost_mode;            /* MG_GHOST_* */
-  int32_t transport;             /* MG_TRANSPORT_*: auto = NCCL when world_size > 1, else local device
-                                    copies (a one-rank MG_GHOST_ALL self-exchange goes through NCCL only
-                                    with MG_TRANSPORT_NCCL; nccl_id may then be NULL) */
+  int32_t transport;             /* MG_TRANSPORT_*.  Between processes (world_size > 1): auto / PEER = every
+                                    rank maps the others' workspaces (CUDA IPC, mg_peer_blob /
+                                    mg_peer_connect) and one device kernel per exchange copies the ghost
+                                    runs out of the neighbours' fields, ordered by device-side flags (no
+                                    NCCL; the norm's max and the replicated bottom's gather likewise);
+                                    NCCL = grouped ncclSend/ncclRecv + ncclAllReduce (needs nccl_id).  One
+                                    rank: local device copies, or NCCL self send/recv with
+                                    MG_TRANSPORT_NCCL (nccl_id may then be NULL) */
   int32_t use_graph;             /* 1 = replay the V-cycle as one CUDA graph (default 1) */
   int32_t bottom_mode;           /* MG_BOTTOM_* (resident = one CTA runs all bottom sweeps in smem,
                                     cluster = the coarse levels run in one cluster launch, grid = the
@@ -155,6 +161,18 @@ mg_status mg_nccl_unique_id(uint8_t out_id[128]);
  * workspace: device memory of >= mg_workspace_bytes, 256-byte aligned. */
 mg_status mg_setup(const mg_params* p, int32_t rank, int32_t world_size, const uint8_t* nccl_id,
                    int32_t device, void* cuda_stream, void* workspace, size_t ws_bytes, mg_ctx** out);
+
+/* Peer-memory transport (MG_TRANSPORT_PEER / AUTO with world_size > 1), after mg_setup and before
+ * the first exchange: every rank writes its blob (the CUDA IPC handle of the allocation holding its
+ * workspace, the workspace's offset in it, rank, world) with mg_peer_blob, the caller all-gathers
+ * the blobs in rank order (torch.distributed in the Python harness) and passes all of them
+ * (world_size * MG_PEER_BLOB_BYTES bytes) to mg_peer_connect, which maps the other workspaces
+ * (cudaIpcOpenMemHandle; closed by mg_destroy) and builds the exchange tables.  Every rank must use
+ * the same parameters (same workspace layout).  The workspace must come from cudaMalloc (e.g. the
+ * default torch caching allocator), not from a VMM / expandable-segments allocation.  Exchanges,
+ * norms and V-cycles before mg_peer_connect fail with MG_ERR_STATE. */
+mg_status mg_peer_blob(mg_ctx* c, uint8_t* out_blob);
+mg_status mg_peer_connect(mg_ctx* c, const uint8_t* all_blobs);
 
 /* Right-hand side b of level 0, local lexicographic, device / host.
  * mg_set_rhs_host does not block the host: the upload runs on an internal copy

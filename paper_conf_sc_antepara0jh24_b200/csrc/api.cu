@@ -12,9 +12,12 @@
 //                ncclGroup, or device copies for the in-process loopback group
 //   norm         fused applyOp + |b - Ax| + block max + atomicMax on the uint64
 //                bits (exact, order-free), ncclAllReduce(MAX) of 1 value
+#include <cuda.h>
 #include <cuda_runtime.h>
+#include <cudaTypedefs.h>
 #include <nccl.h>
 
+#include <algorithm>
 #include <cmath>
 #include <cstdio>
 #include <cstring>
@@ -100,6 +103,20 @@ struct mg_ctx {
   double* h_pinned = nullptr;
   ncclComm_t nccl = nullptr;
   bool use_nccl = false;
+  // peer-memory transport (MG_TRANSPORT_PEER, peer.cu): the other ranks' workspaces mapped by CUDA
+  // IPC; exchanges, the norm's global max and the replicated bottom's gather are device-side
+  bool use_peer = false, peer_ready = false;
+  std::vector<char*> peer_ws;     // [world] every rank's workspace in this address space
+  std::vector<void*> peer_open;   // IPC mappings to close
+  PeerSync ps_nb{}, ps_all{};     // participants: the neighbour ranks / every other rank
+  unsigned long long** d_remote_vals = nullptr;  // [world] the ranks' norm value slots (device array)
+  struct PeerArea {
+    unsigned long long* flags = nullptr;  // [world][2] slots of kPeerSlotU64
+    unsigned long long* vals = nullptr;   // [world] norm values
+    unsigned long long* epoch = nullptr;
+    unsigned* done = nullptr;
+    CopyRun* dummy = nullptr;
+  } pa;
   mg_group* group = nullptr;
   int grank = 0;
   LevelState st[MG_MAX_LEVELS];
@@ -172,7 +189,7 @@ namespace {
 
 // ------------------------------------------------------------- workspace
 size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double** stage, unsigned long long** acc,
-             mg_ctx::Repl* rp = nullptr) {
+             mg_ctx::Repl* rp = nullptr, mg_ctx::PeerArea* pa = nullptr) {
   size_t off = 0;
   auto take = [&](size_t bytes) -> char* {
     const size_t o = align256(off);
@@ -240,6 +257,19 @@ size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double**
     r.scatter = (CopyRun*)take((size_t)2 * nown * sizeof(CopyRun));
     if (rp) *rp = r;
   }
+  if (lay.world > 1 && pa) {  // peer-transport sync area (also carved for NCCL runs: a few KB)
+    pa->flags = (unsigned long long*)take((size_t)lay.world * 2 * kPeerSlotU64 * 8);
+    pa->vals = (unsigned long long*)take((size_t)lay.world * 8);
+    pa->epoch = (unsigned long long*)take(64);
+    pa->done = (unsigned*)take(64);
+    pa->dummy = (CopyRun*)take(sizeof(CopyRun));
+  } else if (lay.world > 1) {
+    take((size_t)lay.world * 2 * kPeerSlotU64 * 8);
+    take((size_t)lay.world * 8);
+    take(64);
+    take(64);
+    take(sizeof(CopyRun));
+  }
   // norm accumulator (word 0) and the grid coarse solve's barrier words (from byte 64, kGridBarWords)
   unsigned long long* ac = (unsigned long long*)take(64 + kGridBarWords * sizeof(unsigned));
   if (acc) *acc = ac;
@@ -263,7 +293,7 @@ mg_params normalized(const mg_params* p) {
 mg_status check_params(const mg_params& p) {
   if (p.num_levels > 1 && p.pre_smooths < 1)
     return set_err(MG_ERR_INVALID_ARG, "pre_smooths must be >= 1 when num_levels > 1 (restriction reads its r)");
-  if (p.transport < 0 || p.transport > MG_TRANSPORT_LOCAL) return set_err(MG_ERR_INVALID_ARG, "bad transport");
+  if (p.transport < 0 || p.transport > MG_TRANSPORT_PEER) return set_err(MG_ERR_INVALID_ARG, "bad transport");
   if (p.bottom_mode < 0 || p.bottom_mode > MG_BOTTOM_GRID) return set_err(MG_ERR_INVALID_ARG, "bad bottom_mode");
   if (p.launch_pdl < 0 || p.launch_pdl > 2) return set_err(MG_ERR_INVALID_ARG, "launch_pdl must be 0, 1 or 2");
   if (p.bottom_solver < 0 || p.bottom_solver > 1)
@@ -324,7 +354,12 @@ mg_status do_exchange(mg_ctx* c, int l, int field, int xbuf, cudaStream_t s) {
   const LevelLayout& L = c->lay.lv[l];
   double* f = field_ptr(c, l, field, xbuf);
   const size_t bb = (size_t)kBV;
-  if (c->use_nccl) {
+  if (c->use_peer) {
+    if (!c->peer_ready) return set_err(MG_ERR_STATE, "peer transport: call mg_peer_connect first");
+    const DevLevel& d = c->dl[l];
+    const int fv = field ? 2 : xbuf;
+    CKC(c, launch_peer_copy(d.cruns + (size_t)fv * d.ncruns, d.ncruns, d.cmax, c->ps_nb, s));
+  } else if (c->use_nccl) {
     CKN(c, ncclGroupStart());
     for (const Run& r : L.recvs)
       CKN(c, ncclRecv(f + r.local * bb, (size_t)r.count * bb, ncclFloat64, r.peer, c->nccl, s));
@@ -358,6 +393,9 @@ mg_status fill_repl_tables(mg_ctx* c) {
     const double* from;
     if (c->rp.allgather)
       from = c->rp.gbuf + (size_t)src * bb;
+    else if (c->use_peer)  // the owner's b field through its IPC mapping
+      from = (const double*)(c->peer_ws[(size_t)r] + ((const char*)c->dl[(size_t)lb].b - (const char*)c->peer_ws[(size_t)c->lay.rank])) +
+             (size_t)i * bb;
     else if (c->group)
       from = c->group->r[(size_t)r]->dl[(size_t)lb].b + (size_t)i * bb;
     else
@@ -389,8 +427,10 @@ mg_status fill_copy_tables(mg_ctx* c) {
       for (int i = 0; i < d.ncruns; ++i) {
         const Run& r = L.recvs[(size_t)i];
         mg_ctx* src = c->group ? c->group->r[r.peer] : c;
-        h[(size_t)fv * d.ncruns + i] = {field_ptr(src, l, field, xbuf) + r.remote * bb, f + r.local * bb,
-                                        (int64_t)r.count * (int64_t)bb};
+        const double* sf = field_ptr(src, l, field, xbuf);
+        if (c->use_peer)  // the sender's field at the same workspace offset, through its IPC mapping
+          sf = (const double*)(c->peer_ws[(size_t)r.peer] + ((const char*)f - (const char*)c->peer_ws[(size_t)c->lay.rank]));
+        h[(size_t)fv * d.ncruns + i] = {sf + r.remote * bb, f + r.local * bb, (int64_t)r.count * (int64_t)bb};
         d.cmax = std::max<int64_t>(d.cmax, (int64_t)r.count * (int64_t)bb);
       }
     }
@@ -585,7 +625,10 @@ mg_status exec_op(mg_ctx* c, const Op& o, cudaStream_t s) {
       CKS(timer_begin(c, s, &t0));
       if (c->rp.allgather)
         CKN(c, ncclAllGather(d.b, c->rp.gbuf, (size_t)L.n_owned * kBV, ncclFloat64, c->nccl, s));
-      CKC(c, launch_copy_runs(c->rp.gather, (int)ng, kBV, s));
+      if (c->use_peer)
+        CKC(c, launch_peer_copy(c->rp.gather, (int)ng, kBV, c->ps_all, s));
+      else
+        CKC(c, launch_copy_runs(c->rp.gather, (int)ng, kBV, s));
       if (lay.p.bottom_solver == 1) {
         CKC(c, launch_bottom_cg(c->rp.x[1], c->rp.b, c->rp.adj, c->rp.coord, (int)ng, lay.gb.n[0], lay.gb.n[1], o.n,
                                 d.c, s));
@@ -662,7 +705,7 @@ mg_status check_ctx(mg_ctx* c) {
 }
 
 mg_status build_and_run(mg_ctx* c, mg_group* g, bool vcycle_graph, Builder& b) {
-  const Plan p = make_plan(b, c->lay, c->pencil_overlap, !c->use_nccl);
+  const Plan p = make_plan(b, c->lay, c->pencil_overlap, !c->use_nccl);  // (peer: one copy kernel too)
   CKS(prepare_plan(c, g, p.ops));
   CKS(run_plan(c, g, p, g ? g->stream : c->stream));
   if (g) {
@@ -745,7 +788,9 @@ mg_status init_ctx(mg_ctx* c, const mg_params& p, int rank, int world, int devic
   if (!workspace || ws_bytes < need)
     return set_err(MG_ERR_OOM, "workspace too small: need " + std::to_string(need) + " bytes");
   if (((uintptr_t)workspace & 255) != 0) return set_err(MG_ERR_INVALID_ARG, "workspace must be 256-byte aligned");
-  carve(c->lay, (char*)workspace, &c->dl, c->stage, &c->acc, &c->rp);
+  carve(c->lay, (char*)workspace, &c->dl, c->stage, &c->acc, &c->rp, &c->pa);
+  c->peer_ws.assign((size_t)world, nullptr);
+  c->peer_ws[(size_t)rank] = (char*)workspace;
   (void)tables_only_upload;
   CKC(c, cudaMemsetAsync(workspace, 0, need, stream));
   for (int l = 0; l < c->lay.L; ++l) {
@@ -825,6 +870,7 @@ void free_ctx(mg_ctx* c) {
   for (cudaEvent_t e : c->evpool) cudaEventDestroy(e);
   if (c->h_pinned) cudaFreeHost(c->h_pinned);
   for (void* a : c->allocs) cudaFree(a);
+  for (void* a : c->peer_open) cudaIpcCloseMemHandle(a);
   delete c;
 }
 
@@ -916,7 +962,9 @@ mg_status mg_setup(const mg_params* p, int32_t rank, int32_t world_size, const u
   }
   bool any_ghost = false;
   for (const auto& L : c->lay.lv) any_ghost |= L.n_ghost > 0;
-  const bool want_nccl = world_size > 1 || q.transport == MG_TRANSPORT_NCCL;
+  // between processes: peer memory by default (MG_TRANSPORT_AUTO / PEER), NCCL when asked for
+  c->use_peer = world_size > 1 && (q.transport == MG_TRANSPORT_AUTO || q.transport == MG_TRANSPORT_PEER);
+  const bool want_nccl = q.transport == MG_TRANSPORT_NCCL;
   if (world_size > 1 && q.transport == MG_TRANSPORT_LOCAL) {
     free_ctx(c);
     return set_err(MG_ERR_INVALID_ARG, "multi-process runs need the NCCL transport (use mg_group_* for loopback)");
@@ -944,17 +992,19 @@ mg_status mg_setup(const mg_params* p, int32_t rank, int32_t world_size, const u
     c->use_nccl = true;
   }
   (void)any_ghost;
-  if (!c->use_nccl) {
+  if (!c->use_nccl && !c->use_peer) {  // (peer: at mg_peer_connect, once the mappings exist)
     s = fill_copy_tables(c);
     if (s != MG_OK) {
       free_ctx(c);
       return s;
     }
   }
-  s = fill_repl_tables(c);
-  if (s != MG_OK) {
-    free_ctx(c);
-    return s;
+  if (!c->use_peer) {
+    s = fill_repl_tables(c);
+    if (s != MG_OK) {
+      free_ctx(c);
+      return s;
+    }
   }
   *out = c;
   return MG_OK;
@@ -1038,6 +1088,10 @@ mg_status mg_residual_norm_async(mg_ctx* c) {
   CKC(c, launch_norm(d.x[c->st[0].cur], d.b, d.adj, L.n_owned, d.c, c->acc, c->stream));
   if (c->use_nccl && c->lay.world > 1)
     CKN(c, ncclAllReduce(c->acc, c->acc, 1, ncclUint64, ncclMax, c->nccl, c->stream));
+  if (c->use_peer && c->lay.world > 1) {
+    if (!c->peer_ready) return set_err(MG_ERR_STATE, "peer transport: call mg_peer_connect first");
+    CKC(c, launch_peer_allmax(c->acc, c->ps_all, c->d_remote_vals, c->pa.vals, c->lay.rank, c->lay.world, c->stream));
+  }
   CKC(c, cudaMemcpyAsync(c->h_pinned, c->acc, sizeof(unsigned long long), cudaMemcpyDeviceToHost, c->stream));
   CKC(c, cudaEventRecord(c->ev_norm, c->stream));
   c->norm_pending = true;
@@ -1174,6 +1228,109 @@ mg_status mg_exchange_time(mg_ctx* c, int32_t level, int32_t reps, double* ms_pe
   CKC(c, cudaEventElapsedTime(&ms, e0, e1));
   c->evnext = 0;
   *ms_per_exchange = (double)ms / reps;
+  return MG_OK;
+}
+
+namespace {
+struct PeerBlob {  // MG_PEER_BLOB_BYTES: what one rank publishes for the others to map it
+  cudaIpcMemHandle_t handle;  // of the allocation holding the workspace
+  int64_t ws_off;             // workspace pointer - allocation base
+  int32_t world, rank;
+  int64_t ws_bytes;
+};
+static_assert(sizeof(PeerBlob) <= MG_PEER_BLOB_BYTES, "peer blob");
+}  // namespace
+
+mg_status mg_peer_blob(mg_ctx* c, uint8_t* out) {
+  CKS(check_ctx(c));
+  if (!out) return set_err(MG_ERR_INVALID_ARG, "null out");
+  if (!c->use_peer) return set_err(MG_ERR_STATE, "not a peer-transport context");
+  static PFN_cuMemGetAddressRange_v3020 range = nullptr;
+  if (!range) {
+    void* fn = nullptr;
+    cudaDriverEntryPointQueryResult qr;
+    CKC(c, cudaGetDriverEntryPoint("cuMemGetAddressRange", &fn, cudaEnableDefault, &qr));
+    if (qr != cudaDriverEntryPointSuccess || !fn) return set_err(MG_ERR_CUDA, "cuMemGetAddressRange unavailable");
+    range = reinterpret_cast<PFN_cuMemGetAddressRange_v3020>(fn);
+  }
+  char* ws = c->peer_ws.empty() ? nullptr : c->peer_ws[(size_t)c->lay.rank];
+  CUdeviceptr base = 0;
+  size_t size = 0;
+  if (range(&base, &size, (CUdeviceptr)ws) != CUDA_SUCCESS) return set_err(MG_ERR_CUDA, "cuMemGetAddressRange failed");
+  PeerBlob b{};
+  CKC(c, cudaIpcGetMemHandle(&b.handle, (void*)base));
+  b.ws_off = (int64_t)((CUdeviceptr)ws - base);
+  b.world = c->lay.world;
+  b.rank = c->lay.rank;
+  b.ws_bytes = (int64_t)size;
+  std::memset(out, 0, MG_PEER_BLOB_BYTES);
+  std::memcpy(out, &b, sizeof(b));
+  return MG_OK;
+}
+
+mg_status mg_peer_connect(mg_ctx* c, const uint8_t* blobs) {
+  CKS(check_ctx(c));
+  if (!blobs) return set_err(MG_ERR_INVALID_ARG, "null blobs");
+  if (!c->use_peer) return set_err(MG_ERR_STATE, "not a peer-transport context");
+  if (c->peer_ready) return set_err(MG_ERR_STATE, "already connected");
+  const int W = c->lay.world, me = c->lay.rank;
+  char* mine = c->peer_ws[(size_t)me];
+  for (int r = 0; r < W; ++r) {
+    PeerBlob b;
+    std::memcpy(&b, blobs + (size_t)r * MG_PEER_BLOB_BYTES, sizeof(b));
+    if (b.world != W || b.rank != r) return set_err(MG_ERR_INVALID_ARG, "peer blobs out of order or from another run");
+    if (r == me) continue;
+    void* p = nullptr;
+    CKC(c, cudaIpcOpenMemHandle(&p, b.handle, cudaIpcMemLazyEnablePeerAccess));
+    c->peer_open.push_back(p);
+    c->peer_ws[(size_t)r] = (char*)p + b.ws_off;
+  }
+  // every rank carves the same workspace layout (same local geometry): rank r's object at offset o
+  // of its workspace is the object at offset o of this rank's
+  auto at = [&](int r, const void* local) { return c->peer_ws[(size_t)r] + ((const char*)local - mine); };
+  std::vector<unsigned long long*> remote((size_t)W * 2, nullptr), rvals((size_t)W, nullptr);
+  for (int r = 0; r < W; ++r) {
+    for (int k = 0; k < 2; ++k)  // THIS rank's slot (me, k) in rank r's flag array
+      remote[(size_t)r * 2 + k] = (unsigned long long*)at(r, c->pa.flags + ((size_t)me * 2 + k) * kPeerSlotU64);
+    rvals[(size_t)r] = (unsigned long long*)at(r, c->pa.vals);
+  }
+  std::vector<int> nb, all;
+  for (int r = 0; r < W; ++r)
+    if (r != me) all.push_back(r);
+  for (const auto& L : c->lay.lv)
+    for (const Run& r : L.recvs)
+      if (r.peer != me && std::find(nb.begin(), nb.end(), r.peer) == nb.end()) nb.push_back(r.peer);
+  std::sort(nb.begin(), nb.end());
+  // small device tables (library-owned)
+  auto upload = [&](const void* h, size_t bytes) -> void* {
+    void* d = nullptr;
+    if (cudaMalloc(&d, bytes) != cudaSuccess) return nullptr;
+    c->allocs.push_back(d);
+    if (cudaMemcpy(d, h, bytes, cudaMemcpyHostToDevice) != cudaSuccess) return nullptr;
+    return d;
+  };
+  void* d_remote = upload(remote.data(), remote.size() * sizeof(void*));
+  void* d_rvals = upload(rvals.data(), rvals.size() * sizeof(void*));
+  void* d_nb = upload(nb.empty() ? all.data() : nb.data(), std::max<size_t>(1, nb.size()) * sizeof(int));
+  void* d_all = upload(all.data(), std::max<size_t>(1, all.size()) * sizeof(int));
+  if (!d_remote || !d_rvals || !d_nb || !d_all) return set_err(MG_ERR_CUDA, "peer tables: cudaMalloc / cudaMemcpy failed");
+  c->d_remote_vals = (unsigned long long**)d_rvals;
+  PeerSync base{};
+  base.flags = c->pa.flags;
+  base.remote = (unsigned long long* const*)d_remote;
+  base.epoch = c->pa.epoch;
+  base.done = c->pa.done;
+  base.dummy_run = c->pa.dummy;
+  c->ps_nb = base;
+  c->ps_nb.part = (const int*)d_nb;
+  c->ps_nb.npart = (int)nb.size();
+  c->ps_all = base;
+  c->ps_all.part = (const int*)d_all;
+  c->ps_all.npart = (int)all.size();
+  c->peer_ready = true;
+  CKS(fill_copy_tables(c));
+  CKS(fill_repl_tables(c));
+  CKC(c, cudaDeviceSynchronize());
   return MG_OK;
 }
 

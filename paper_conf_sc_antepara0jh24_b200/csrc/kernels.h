@@ -143,6 +143,23 @@ struct CopyRun {
   int64_t n;
 };
 cudaError_t launch_copy_runs(const CopyRun* runs, int nruns, int64_t max_n, cudaStream_t s);
+// Exchange between processes over peer memory (peer.cu): the copy runs read other ranks' fields
+// through CUDA IPC mappings; device-side flags order them (ready / done per epoch, see peer.cu).
+constexpr int kPeerSlotU64 = 16;  // one flag per 128-byte slot
+struct PeerSync {
+  unsigned long long* flags;          // this rank's [world][2] slots (ready, done), kPeerSlotU64 apart
+  unsigned long long* const* remote;  // device [world * 2]: address of THIS rank's slot (kind) at rank n
+  const int* part;                    // device: the participant ranks (never this rank)
+  int npart;
+  unsigned long long* epoch;          // this rank's epoch counter (advanced by every peer kernel)
+  unsigned* done;                     // CTA completion counter (zero between kernels)
+  const CopyRun* dummy_run;           // a zero-length run (a rank without runs still takes part)
+};
+cudaError_t launch_peer_copy(const CopyRun* runs, int nruns, int64_t max_n, const PeerSync& s, cudaStream_t st);
+// global max of the uint64 bits at *acc over the participants (+ this rank): vals = this rank's
+// [world] value slots, remote_vals[n] = rank n's value slots
+cudaError_t launch_peer_allmax(unsigned long long* acc, const PeerSync& s, unsigned long long* const* remote_vals,
+                               unsigned long long* vals, int me, int world, cudaStream_t st);
 // Resident coarse solver (coarse.cu): levels l0 .. L-1 of one V-cycle (pre-sweeps + fused
 // restriction, initZero, bottom, interpolation, post-sweeps) in one launch of a cluster of
 // kCoarseCtas CTAs holding every field of those levels in shared memory.  No ghosts.

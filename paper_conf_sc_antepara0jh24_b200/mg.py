@@ -18,7 +18,8 @@ MG_OK, MG_NOT_CONVERGED = 0, 1
 MG_MAX_LEVELS = 16
 MG_FUSION_AUTO, MG_FUSION_PAPER, MG_FUSION_SWEEP, MG_FUSION_FULL = 0, 1, 2, 3
 MG_GHOST_AUTO, MG_GHOST_ALL = 0, 1
-MG_TRANSPORT_AUTO, MG_TRANSPORT_NCCL, MG_TRANSPORT_LOCAL = 0, 1, 2
+MG_TRANSPORT_AUTO, MG_TRANSPORT_NCCL, MG_TRANSPORT_LOCAL, MG_TRANSPORT_PEER = 0, 1, 2, 3
+MG_PEER_BLOB_BYTES = 128
 MG_BOTTOM_AUTO, MG_BOTTOM_SWEEPS, MG_BOTTOM_RESIDENT, MG_BOTTOM_CLUSTER, MG_BOTTOM_GRID = 0, 1, 2, 3, 4
 MG_FIELD_X, MG_FIELD_B, MG_FIELD_R = 0, 1, 2
 OP_NAMES = ["sweep", "applyOp", "smooth", "restriction", "interpolation", "initZero", "exchange", "bottom"]
@@ -86,6 +87,8 @@ _SIGS = {
     "mg_vcycle_launches": (ctypes.c_int, [ctypes.c_void_p, ctypes.POINTER(ctypes.c_int64)]),
     "mg_exchange_stats": (ctypes.c_int, [ctypes.c_void_p, ctypes.POINTER(ctypes.c_int64),
                                          ctypes.POINTER(ctypes.c_int64)]),
+    "mg_peer_blob": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_char_p]),
+    "mg_peer_connect": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_char_p]),
     "mg_exchange_plan": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.POINTER(ctypes.c_int64),
                                         ctypes.POINTER(ctypes.c_int64)]),
     "mg_exchange_time": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32,
@@ -276,6 +279,16 @@ def mg_exchange_stats(ctx):
     b, m = ctypes.c_int64(), ctypes.c_int64()
     check(lib().mg_exchange_stats(ctx, ctypes.byref(b), ctypes.byref(m)), "mg_exchange_stats")
     return b.value, m.value
+
+
+def mg_peer_blob(ctx) -> bytes:
+    buf = ctypes.create_string_buffer(MG_PEER_BLOB_BYTES)
+    check(lib().mg_peer_blob(ctx, buf), "mg_peer_blob")
+    return buf.raw
+
+
+def mg_peer_connect(ctx, blobs: bytes):
+    return check(lib().mg_peer_connect(ctx, blobs), "mg_peer_connect")
 
 
 def mg_exchange_plan(ctx, num_levels):

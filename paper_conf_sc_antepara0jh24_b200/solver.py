@@ -42,7 +42,9 @@ class Multigrid:
         self.ws_ptr = (base + 255) & ~255
         self.stream = stream if stream is not None else torch.cuda.current_stream(self.device)
         nccl_id = None
-        if self.world_size > 1:
+        self.transport = int(transport)
+        peer = self.world_size > 1 and self.transport in (mg.MG_TRANSPORT_AUTO, mg.MG_TRANSPORT_PEER)
+        if self.world_size > 1 and self.transport == mg.MG_TRANSPORT_NCCL:
             import torch.distributed as dist
 
             obj = [mg.mg_nccl_unique_id() if self.rank == 0 else None]
@@ -50,6 +52,12 @@ class Multigrid:
             nccl_id = obj[0]
         self.ctx = mg.mg_setup(self.p, self.rank, self.world_size, nccl_id, self.device.index,
                                self.stream.cuda_stream, self.ws_ptr, self.ws_bytes)
+        if peer:  # map every rank's workspace (CUDA IPC); blobs all-gathered in rank order
+            import torch.distributed as dist
+
+            blobs = [None] * self.world_size
+            dist.all_gather_object(blobs, mg.mg_peer_blob(self.ctx))
+            mg.mg_peer_connect(self.ctx, b"".join(blobs))
 
     @property
     def shape(self):  # numpy / torch order (nz, ny, nx)
