@@ -47,9 +47,9 @@ def parse():
     ap.add_argument("--ca-period", type=int, default=0)
     ap.add_argument("--fusion", type=int, default=0)
     ap.add_argument("--ghost-all", action="store_true", help="self-exchange ghost shell on every axis")
-    ap.add_argument("--transport", choices=["auto", "nccl", "local"], default="auto",
-                    help="ghost exchange transport (auto: NCCL between processes, device copies for a one-rank "
-                         "self-exchange; nccl: NCCL send/recv even to itself)")
+    ap.add_argument("--transport", choices=["auto", "peer", "nccl", "local"], default="auto",
+                    help="ghost exchange transport (auto: peer memory (CUDA IPC + device flags) between processes, "
+                         "device copies for a one-rank self-exchange; peer / nccl: that transport even to itself)")
     ap.add_argument("--no-graph", action="store_true")
     ap.add_argument("--no-overlap", action="store_true")
     ap.add_argument("--tb", type=int, default=3,
@@ -265,6 +265,8 @@ NVLINK_GBS = 900.0  # NVLink 5: 900 GB/s per direction per GPU (B200_PROFILING.m
 
 
 def exchange_block(m, a, world, max_over_ranks, tm, ninst):
+    from paper_conf_sc_antepara0jh24_b200 import mg
+
     """Per level: ghost exchanges per V-cycle, bytes per exchange, device time of one exchange (the
     V-cycle's own transport, back to back, max over ranks), achieved GB/s and its fraction of the
     NVLink per-direction bandwidth (between processes) -- plus the latency / bandwidth fit
@@ -273,7 +275,8 @@ def exchange_block(m, a, world, max_over_ranks, tm, ninst):
     counts, nbytes = m.exchange_plan()
     if not any(nbytes):
         return {"levels": [], "note": "no ghost shell (one rank, periodic wrap): no exchanges"}
-    transport = ("nccl" if (world > 1 or a.transport == "nccl") else "local device copies")
+    transport = {mg.MG_TRANSPORT_NCCL: "nccl", mg.MG_TRANSPORT_PEER: "peer memory (CUDA IPC, device flags)"}.get(
+        m.transport, "peer memory (CUDA IPC, device flags)" if world > 1 else "local device copies")
     out = []
     for l, (c, b) in enumerate(zip(counts, nbytes)):
         if b <= 0:
@@ -328,7 +331,7 @@ def main():
                   cheby_ratio=a.cheby_ratio, launch_pdl=2 if a.no_pdl else 0,
                   bottom_mode=a.bottom_mode, bottom_solver=a.bottom_solver,
                   transport={"auto": mg.MG_TRANSPORT_AUTO, "nccl": mg.MG_TRANSPORT_NCCL,
-                             "local": mg.MG_TRANSPORT_LOCAL}[a.transport])
+                             "local": mg.MG_TRANSPORT_LOCAL, "peer": mg.MG_TRANSPORT_PEER}[a.transport])
     gshape = (n * pg[2], n * pg[1], n * pg[0])
     b_host = torch.from_numpy(mg_inputs.local_sin_rhs(gshape, rank, pg)).pin_memory()
     b_dev = b_host.to(dev)

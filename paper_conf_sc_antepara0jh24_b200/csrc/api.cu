@@ -939,6 +939,8 @@ mg_status mg_nccl_unique_id(uint8_t out_id[128]) {
   return MG_OK;
 }
 
+static mg_status peer_connect_impl(mg_ctx* c, const uint8_t* blobs);
+
 mg_status mg_setup(const mg_params* p, int32_t rank, int32_t world_size, const uint8_t* nccl_id, int32_t device,
                    void* cuda_stream, void* workspace, size_t ws_bytes, mg_ctx** out) {
   if (!p || !out) return set_err(MG_ERR_INVALID_ARG, "null argument");
@@ -963,7 +965,7 @@ mg_status mg_setup(const mg_params* p, int32_t rank, int32_t world_size, const u
   bool any_ghost = false;
   for (const auto& L : c->lay.lv) any_ghost |= L.n_ghost > 0;
   // between processes: peer memory by default (MG_TRANSPORT_AUTO / PEER), NCCL when asked for
-  c->use_peer = world_size > 1 && (q.transport == MG_TRANSPORT_AUTO || q.transport == MG_TRANSPORT_PEER);
+  c->use_peer = (world_size > 1 && q.transport == MG_TRANSPORT_AUTO) || q.transport == MG_TRANSPORT_PEER;
   const bool want_nccl = q.transport == MG_TRANSPORT_NCCL;
   if (world_size > 1 && q.transport == MG_TRANSPORT_LOCAL) {
     free_ctx(c);
@@ -1001,6 +1003,12 @@ mg_status mg_setup(const mg_params* p, int32_t rank, int32_t world_size, const u
   }
   if (!c->use_peer) {
     s = fill_repl_tables(c);
+    if (s != MG_OK) {
+      free_ctx(c);
+      return s;
+    }
+  } else if (world_size == 1) {  // a one-rank self-exchange through the peer kernel (no participants)
+    s = peer_connect_impl(c, nullptr);
     if (s != MG_OK) {
       free_ctx(c);
       return s;
@@ -1268,14 +1276,10 @@ mg_status mg_peer_blob(mg_ctx* c, uint8_t* out) {
   return MG_OK;
 }
 
-mg_status mg_peer_connect(mg_ctx* c, const uint8_t* blobs) {
-  CKS(check_ctx(c));
-  if (!blobs) return set_err(MG_ERR_INVALID_ARG, "null blobs");
-  if (!c->use_peer) return set_err(MG_ERR_STATE, "not a peer-transport context");
-  if (c->peer_ready) return set_err(MG_ERR_STATE, "already connected");
+static mg_status peer_connect_impl(mg_ctx* c, const uint8_t* blobs) {
   const int W = c->lay.world, me = c->lay.rank;
   char* mine = c->peer_ws[(size_t)me];
-  for (int r = 0; r < W; ++r) {
+  for (int r = 0; r < W && W > 1; ++r) {
     PeerBlob b;
     std::memcpy(&b, blobs + (size_t)r * MG_PEER_BLOB_BYTES, sizeof(b));
     if (b.world != W || b.rank != r) return set_err(MG_ERR_INVALID_ARG, "peer blobs out of order or from another run");
@@ -1332,6 +1336,14 @@ mg_status mg_peer_connect(mg_ctx* c, const uint8_t* blobs) {
   CKS(fill_repl_tables(c));
   CKC(c, cudaDeviceSynchronize());
   return MG_OK;
+}
+
+mg_status mg_peer_connect(mg_ctx* c, const uint8_t* blobs) {
+  CKS(check_ctx(c));
+  if (!blobs) return set_err(MG_ERR_INVALID_ARG, "null blobs");
+  if (!c->use_peer) return set_err(MG_ERR_STATE, "not a peer-transport context");
+  if (c->peer_ready) return set_err(MG_ERR_STATE, "already connected");
+  return peer_connect_impl(c, blobs);
 }
 
 mg_status mg_destroy(mg_ctx* c) {

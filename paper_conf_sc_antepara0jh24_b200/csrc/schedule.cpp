@@ -21,7 +21,15 @@ int Builder::fusion(int l) const {
 
 int Builder::period(int l) const {
   const int k = lay.p.ca_period[l];
-  return k ? k : MG_MAX_PERIOD;
+  if (k) return k;
+  // auto (measured, one B200, self-exchanged ghost shell on every axis, profiles/r02_exchange.md):
+  // with exchanges as device copies on the same GPU (one rank, or a loopback group) an exchange of the
+  // finest level costs less than the redundant ghost-shell sweeping a longer period needs (period 2 at
+  // level 0: 8.42 vs 8.62 ms per cycle), the coarser levels are better at 8 (fewer launches); between
+  // processes an exchange crosses NVLink (~6x the bytes-time of a local copy, plus flag latency) and
+  // the brick-deep ghost zone's period 8 stays the default
+  const bool local = lay.world == 1 ? lay.p.transport != MG_TRANSPORT_NCCL : lay.p.transport == MG_TRANSPORT_LOCAL;
+  return (l == 0 && local) ? 2 : MG_MAX_PERIOD;
 }
 
 bool Builder::has_pair_table(int l, int64_t b0, int64_t b1) const {

@@ -56,8 +56,28 @@ class Multigrid:
             import torch.distributed as dist
 
             blobs = [None] * self.world_size
-            dist.all_gather_object(blobs, mg.mg_peer_blob(self.ctx))
-            mg.mg_peer_connect(self.ctx, b"".join(blobs))
+            try:
+                blob = mg.mg_peer_blob(self.ctx)
+            except mg.MGError:
+                blob = None
+            dist.all_gather_object(blobs, blob)
+            ok = all(b is not None for b in blobs)
+            if ok:
+                try:
+                    mg.mg_peer_connect(self.ctx, b"".join(blobs))
+                except mg.MGError:
+                    ok = False
+            oks = [None] * self.world_size
+            dist.all_gather_object(oks, ok)
+            if not all(oks):  # (e.g. no CUDA IPC between these devices): every rank falls back to NCCL
+                mg.mg_destroy(self.ctx)
+                self.ctx = None
+                self.transport = mg.MG_TRANSPORT_NCCL
+                self.p.transport = mg.MG_TRANSPORT_NCCL
+                obj = [mg.mg_nccl_unique_id() if self.rank == 0 else None]
+                dist.broadcast_object_list(obj, src=0)
+                self.ctx = mg.mg_setup(self.p, self.rank, self.world_size, obj[0], self.device.index,
+                                       self.stream.cuda_stream, self.ws_ptr, self.ws_bytes)
 
     @property
     def shape(self):  # numpy / torch order (nz, ny, nx)

@@ -178,11 +178,12 @@ def test_vcycle_fusion_variants_bitwise(oracle_mod, fusion, use_graph):
     m.close()
 
 
-@pytest.mark.parametrize("transport", [2, 1])
-@pytest.mark.parametrize("period", [1, 2, 4, 8])
+@pytest.mark.parametrize("transport", [2, 1, 3])
+@pytest.mark.parametrize("period", [0, 1, 2, 4, 8])
 def test_self_exchange_ca_periods_bitwise(oracle_mod, transport, period):
     """Ghost shell on every axis with self-exchange (communication avoiding on one
-    GPU): local copies and NCCL send/recv; any CA period gives the same bits."""
+    GPU): local copies, NCCL send/recv and the peer-memory kernel; any CA period (0: the
+    per-level auto choice) gives the same bits."""
     shape = (64, 64, 64)
     b = mg_inputs.random_rhs(shape, 4)
     xs, ns = oracle_cycles(oracle_mod, b, 3, 2, 12, 12, 100)
@@ -813,7 +814,7 @@ def test_gsrb_smoother_loopback_bitwise(oracle_mod):
     orc.close()
 
 
-@pytest.mark.parametrize("transport", [2, 1])
+@pytest.mark.parametrize("transport", [2, 1, 3])
 def test_exchange_plan_and_timing_keep_the_bits(oracle_mod, transport):
     """mg_exchange_plan / mg_exchange_time (the bench's exchange block): a self-exchanged ghost shell
     on every axis has exchanges on every level, the timing runs the V-cycle's own transport (local

@@ -4,10 +4,10 @@
 cd "${GRAFT_REPO_ROOT:-/root/repo}"
 mkdir -p gpurun_out/xs
 python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
-timeout 600 python -m pytest tests/test_gpu_parity.py -q -k "exchange_plan" 2>&1 | tail -2
+timeout 900 python -m pytest tests/test_gpu_parity.py -q -k "exchange_plan or self_exchange or peer_transport" 2>&1 | tail -2
 run() { timeout 600 python bench.py --steps 20 --warmup 5 --no-cpu-baseline --no-e2e "$@"; }
 run > gpurun_out/xs/base.json 2>/dev/null
-for t in local nccl; do for k in 8 4 2; do
+for t in local peer nccl; do for k in 0 8 4 2; do
   run --ghost-all --transport $t --ca-period $k > gpurun_out/xs/ga_${t}_k$k.json 2> gpurun_out/xs/ga_${t}_k$k.err
 done; done
 python - <<'PY'
