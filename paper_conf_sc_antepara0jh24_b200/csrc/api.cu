@@ -1315,8 +1315,11 @@ static mg_status peer_connect_impl(mg_ctx* c, const uint8_t* blobs) {
   };
   void* d_remote = upload(remote.data(), remote.size() * sizeof(void*));
   void* d_rvals = upload(rvals.data(), rvals.size() * sizeof(void*));
-  void* d_nb = upload(nb.empty() ? all.data() : nb.data(), std::max<size_t>(1, nb.size()) * sizeof(int));
-  void* d_all = upload(all.data(), std::max<size_t>(1, all.size()) * sizeof(int));
+  const int npart_nb = (int)nb.size(), npart_all = (int)all.size();
+  nb.push_back(0);  // (never read past npart: keeps the device arrays non-empty on one rank)
+  all.push_back(0);
+  void* d_nb = upload(nb.data(), nb.size() * sizeof(int));
+  void* d_all = upload(all.data(), all.size() * sizeof(int));
   if (!d_remote || !d_rvals || !d_nb || !d_all) return set_err(MG_ERR_CUDA, "peer tables: cudaMalloc / cudaMemcpy failed");
   c->d_remote_vals = (unsigned long long**)d_rvals;
   PeerSync base{};
@@ -1327,10 +1330,10 @@ static mg_status peer_connect_impl(mg_ctx* c, const uint8_t* blobs) {
   base.dummy_run = c->pa.dummy;
   c->ps_nb = base;
   c->ps_nb.part = (const int*)d_nb;
-  c->ps_nb.npart = (int)nb.size();
+  c->ps_nb.npart = npart_nb;
   c->ps_all = base;
   c->ps_all.part = (const int*)d_all;
-  c->ps_all.npart = (int)all.size();
+  c->ps_all.npart = npart_all;
   c->peer_ready = true;
   CKS(fill_copy_tables(c));
   CKS(fill_repl_tables(c));
