@@ -257,18 +257,13 @@ size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double**
     r.scatter = (CopyRun*)take((size_t)2 * nown * sizeof(CopyRun));
     if (rp) *rp = r;
   }
-  if (lay.world > 1 && pa) {  // peer-transport sync area (also carved for NCCL runs: a few KB)
-    pa->flags = (unsigned long long*)take((size_t)lay.world * 2 * kPeerSlotU64 * 8);
-    pa->vals = (unsigned long long*)take((size_t)lay.world * 8);
-    pa->epoch = (unsigned long long*)take(64);
-    pa->done = (unsigned*)take(64);
-    pa->dummy = (CopyRun*)take(sizeof(CopyRun));
-  } else if (lay.world > 1) {
-    take((size_t)lay.world * 2 * kPeerSlotU64 * 8);
-    take((size_t)lay.world * 8);
-    take(64);
-    take(64);
-    take(sizeof(CopyRun));
+  {  // peer-transport sync area (every run carves it: a few KB; a one-rank peer self-exchange uses it too)
+    unsigned long long* fl = (unsigned long long*)take((size_t)lay.world * 2 * kPeerSlotU64 * 8);
+    unsigned long long* vals = (unsigned long long*)take((size_t)lay.world * 8);
+    unsigned long long* ep = (unsigned long long*)take(64);
+    unsigned* dn = (unsigned*)take(64);
+    CopyRun* dm = (CopyRun*)take(sizeof(CopyRun));
+    if (pa) pa->flags = fl, pa->vals = vals, pa->epoch = ep, pa->done = dn, pa->dummy = dm;
   }
   // norm accumulator (word 0) and the grid coarse solve's barrier words (from byte 64, kGridBarWords)
   unsigned long long* ac = (unsigned long long*)take(64 + kGridBarWords * sizeof(unsigned));
