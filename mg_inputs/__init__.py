@@ -81,3 +81,28 @@ def local_sin_rhs(global_shape, rank: int, proc_grid, h0: float | None = None) -
     cx, cy, cz = rank_coords(rank, proc_grid)
     lz, ly, lx = gz // pz, gy // py, gx // px
     return sin_rhs(global_shape, h0, offset=(cz * lz, cy * ly, cx * lx), local_shape=(lz, ly, lx))
+
+
+def random_coef(shape, seed: int, lo: float = 0.5, hi: float = 2.0) -> np.ndarray:
+    """Cell coefficients c = U(lo, hi) > 0 of the variable-coefficient variant (reading A23): a rough
+    field (a factor 4 between neighbours at most), the hard case for the face averages."""
+    rng = np.random.default_rng(10_000 + seed)
+    return np.ascontiguousarray(rng.uniform(lo, hi, size=tuple(int(s) for s in shape)))
+
+
+def smooth_coef(global_shape, h0: float | None = None) -> np.ndarray:
+    """c = 1 + 0.5 prod_d sin(2 pi x_d / L_d) at the cell centres (in [0.5, 1.5]): the smooth
+    coefficient of the timing recipe for the variable-coefficient variant."""
+    return np.ascontiguousarray(1.0 + 0.5 * sin_rhs(global_shape, h0))
+
+
+def dirichlet_sin_rhs(global_shape, h0: float | None = None) -> np.ndarray:
+    """b = prod_d sin(pi x_d / L_d): the lowest Dirichlet mode (vanishes on the domain faces), the
+    timing right-hand side of the non-periodic variant (reading A22)."""
+    gz, gy, gx = (int(s) for s in global_shape)
+    h0 = default_h0(global_shape) if h0 is None else float(h0)
+
+    def ax(n):
+        return np.sin(np.pi * ((np.arange(n, dtype=np.float64) + 0.5) * h0) / (n * h0))
+
+    return np.ascontiguousarray((ax(gz)[:, None, None] * ax(gy)[None, :, None]) * ax(gx)[None, None, :])

@@ -11,6 +11,10 @@ follows.  This module only compiles it (gcc) and marshals numpy arrays via
 ctypes.  Grids are global, lexicographic, periodic, cell-centred, shaped
 ``(nz, ny, nx)`` in numpy (i fastest in memory).
 
+Variants beyond the paper: Chebyshev / red-black Gauss-Seidel smoothers, a CG
+bottom, homogeneous Dirichlet / Neumann boundaries (reading A22) and variable coefficients
+(reading A23) -- see ``OracleMG``'s arguments.
+
 Parity status: every function is pinned by a
 ``-m "not gpu"`` test in ``tests/test_oracle_pins.py`` against closed forms,
 invariants or an independent SciPy sparse-matrix V-cycle; nothing is
@@ -55,13 +59,20 @@ def _load():
             "oracle_set_threads": (None, [I]),
             "oracle_get_threads": (I, []),
             "oracle_apply_op": (None, [I, I, I, D, P, P]),
+            "oracle_apply_op_bc": (None, [I, I, I, D, I, P, P]),
+            "oracle_apply_op_vc": (None, [I, I, I, D, I, P, P, P]),
+            "oracle_vc_gamma": (None, [I, I, I, D, I, P, P]),
+            "oracle_smooth_residual_field": (None, [S, P, P, P, P, P]),
+            "oracle_max_norm_residual_ex": (D, [I, I, I, D, I, P, P, P]),
+            "oracle_mg_set_bc": (I, [P, I]),
+            "oracle_mg_set_coef": (I, [P, P]),
             "oracle_smooth": (None, [S, D, P, P, P]),
             "oracle_smooth_gamma": (None, [S, D, P, P, P]),
             "oracle_smooth_residual_gamma": (None, [S, D, P, P, P, P]),
             "oracle_chebyshev_gamma": (D, [D, I, I, I]),
             "oracle_gsrb_half": (None, [I, I, I, D, I, P, P, P, P]),
             "oracle_mg_set_smoother": (None, [P, I, I]),
-            "oracle_mg_set_bottom_solver": (None, [P, I]),
+            "oracle_mg_set_bottom_solver": (I, [P, I]),
             "oracle_dot_tree": (D, [S, P, P]),
             "oracle_cg": (None, [I, I, I, D, I, P, P]),
             "oracle_smooth_residual": (None, [S, D, P, P, P, P]),
@@ -111,12 +122,44 @@ def default_h0(shape) -> float:
 
 
 # ---------------------------------------------------------------- single ops
-def apply_op(x: np.ndarray, h: float) -> np.ndarray:
+def apply_op(x: np.ndarray, h: float, bc: int = 0) -> np.ndarray:
+    """The paper's 7-point operator; bc 1 / 2 = homogeneous Dirichlet / Neumann (reading A22)."""
     x = _f64(x)
     nz, ny, nx = x.shape
     out = np.empty_like(x)
-    _load().oracle_apply_op(nx, ny, nz, float(h), _ptr(x), _ptr(out))
+    if bc:
+        _load().oracle_apply_op_bc(nx, ny, nz, float(h), int(bc), _ptr(x), _ptr(out))
+    else:
+        _load().oracle_apply_op(nx, ny, nz, float(h), _ptr(x), _ptr(out))
     return out
+
+
+def apply_op_vc(x: np.ndarray, c: np.ndarray, h: float, bc: int = 0) -> np.ndarray:
+    """Variable-coefficient operator div(c grad x) with face values (c_p + c_n)/2 (reading A23)."""
+    x, c = _f64(x), _f64(c)
+    assert c.shape == x.shape
+    nz, ny, nx = x.shape
+    out = np.empty_like(x)
+    _load().oracle_apply_op_vc(nx, ny, nz, float(h), int(bc), _ptr(c), _ptr(x), _ptr(out))
+    return out
+
+
+def vc_gamma(c: np.ndarray, h: float, bc: int = 0) -> np.ndarray:
+    """Per-cell damped-Jacobi step (0.5 h^2) / (sum of the six face coefficients) (reading A23)."""
+    c = _f64(c)
+    nz, ny, nx = c.shape
+    out = np.empty_like(c)
+    _load().oracle_vc_gamma(nx, ny, nz, float(h), int(bc), _ptr(c), _ptr(out))
+    return out
+
+
+def smooth_residual_field(x: np.ndarray, Ax: np.ndarray, b: np.ndarray, gam: np.ndarray):
+    """x + gamma_p (Ax - b) and r = b - Ax with a step per cell (reading A23)."""
+    x = _f64(x).copy()
+    Ax, b, gam = _f64(Ax), _f64(b), _f64(gam)
+    r = np.empty_like(x)
+    _load().oracle_smooth_residual_field(x.size, _ptr(gam), _ptr(x), _ptr(Ax), _ptr(b), _ptr(r))
+    return x, r
 
 
 def smooth(x: np.ndarray, Ax: np.ndarray, b: np.ndarray, h: float) -> np.ndarray:
@@ -190,9 +233,12 @@ def interpolation_increment(xc: np.ndarray, x: np.ndarray) -> np.ndarray:
     return x
 
 
-def max_norm_residual(x: np.ndarray, b: np.ndarray, h: float) -> float:
+def max_norm_residual(x: np.ndarray, b: np.ndarray, h: float, bc: int = 0, c: np.ndarray | None = None) -> float:
     x, b = _f64(x), _f64(b)
     nz, ny, nx = x.shape
+    if bc or c is not None:
+        cp = None if c is None else _ptr(_f64(c))
+        return float(_load().oracle_max_norm_residual_ex(nx, ny, nz, float(h), int(bc), cp, _ptr(x), _ptr(b)))
     return float(_load().oracle_max_norm_residual(nx, ny, nz, float(h), _ptr(x), _ptr(b)))
 
 
@@ -212,7 +258,10 @@ class OracleMG:
     """Alg 1 / Alg 2 on a global periodic grid of shape (nz, ny, nx)."""
 
     def __init__(self, shape, levels: int, pre: int = 12, post: int = 12, bottom: int = 100, h0: float | None = None,
-                 smoother: int = 0, cheby_ratio: int = 6, bottom_solver: int = 0):
+                 smoother: int = 0, cheby_ratio: int = 6, bottom_solver: int = 0, bc: int = 0,
+                 coef: np.ndarray | None = None):
+        """bc: 0 periodic (the paper), 1 Dirichlet, 2 Neumann (reading A22); coef: level-0 cell
+        coefficients c > 0 of the variable-coefficient operator (reading A23), None = the paper's."""
         nz, ny, nx = (int(s) for s in shape)
         self.shape = (nz, ny, nx)
         self.levels = int(levels)
@@ -222,7 +271,15 @@ class OracleMG:
         if not self._h:
             raise ValueError(f"oracle_mg_create failed for shape={shape} levels={levels}")
         self._lib.oracle_mg_set_smoother(self._h, int(smoother), int(cheby_ratio))
-        self._lib.oracle_mg_set_bottom_solver(self._h, int(bottom_solver))
+        if self._lib.oracle_mg_set_bc(self._h, int(bc)) != 0:
+            raise ValueError(f"oracle: bc={bc} not supported")
+        if coef is not None:
+            coef = _f64(coef)
+            assert coef.shape == self.shape
+            if self._lib.oracle_mg_set_coef(self._h, _ptr(coef)) != 0:
+                raise ValueError("oracle: variable coefficients not supported with this configuration")
+        if self._lib.oracle_mg_set_bottom_solver(self._h, int(bottom_solver)) != 0:
+            raise ValueError("oracle: the CG bottom needs the periodic constant-coefficient operator")
 
     def close(self):
         if getattr(self, "_h", None):

@@ -25,6 +25,15 @@
  *   Chebyshev smoother    variant (N4, reading A19): per-sweep steps gamma_k, see
  *                         oracle_chebyshev_gamma; pinned by the Chebyshev-polynomial
  *                         error factor on eigenmodes (tests/test_oracle_pins.py)
+ *   boundary conditions   variant (N4 "non-periodic BCs", reading A22): homogeneous Dirichlet
+ *                         (bc = 1) or Neumann (bc = 2) on the domain faces of the cell-centred
+ *                         grid: the neighbour across a domain face is -x_p (Dirichlet: the linear
+ *                         extrapolation through 0 on the face) or +x_p (Neumann), on every level
+ *                         (rediscretised); oracle_apply_op_bc
+ *   variable coefficients variant (N4, reading A23): A x = div(c grad x) with a cell coefficient
+ *                         c > 0 and face values (c_p + c_n)/2, damped Jacobi with the local
+ *                         diagonal, coarse c = restriction of c; oracle_apply_op_vc,
+ *                         oracle_vc_gamma
  *   CG bottom solver      variant (N4 "other bottom solvers", reading A21): `bottom`
  *                         iterations of conjugate gradients on A x = b from x = 0 with a
  *                         fixed-order (stride-doubling pairwise tree, lexicographic) dot
@@ -71,26 +80,119 @@ int oracle_get_threads(void) {
 #endif
 }
 
+/* Neighbour of cell i on an axis of n cells (reading A22): the periodic wrap (bc 0, the paper,
+ * P:L148), or -1 when the neighbour lies outside a non-periodic domain (the caller then uses the
+ * boundary value: -x_p for homogeneous Dirichlet, +x_p for homogeneous Neumann). */
+static int nbr(int i, int d, int n, int bc) {
+  const int j = i + d;
+  if (j >= 0 && j < n) return j;
+  if (bc == 0) return (j + n) % n;
+  return -1;
+}
+
+/* value of x at neighbour (a, b, c) of cell p: inside, or the boundary image of x_p (reading A22) */
+static double nbv(const double *x, int a, int b, int c, int nx, int ny, int bc, double xp) {
+  if (a < 0 || b < 0 || c < 0) return bc == 1 ? -xp : xp;
+  return x[IDX(a, b, c, nx, ny)];
+}
+
 /* applyOp (Fig 1): Ax = alpha*x + beta*(6 neighbours),
- * alpha = -6/h^2, beta = 1/h^2, periodic wrap stands for exchange(). */
-void oracle_apply_op(int nx, int ny, int nz, double h, const double *x, double *Ax) {
+ * alpha = -6/h^2, beta = 1/h^2; periodic wrap stands for exchange() (bc = 0, the paper), or the
+ * homogeneous Dirichlet / Neumann boundary image of reading A22 (bc = 1 / 2). */
+void oracle_apply_op_bc(int nx, int ny, int nz, double h, int bc, const double *x, double *Ax) {
   const double inv = 1.0 / (h * h);
   const double alpha = -6.0 * inv;
   const double beta = inv;
 #pragma omp parallel for schedule(static)
   for (int k = 0; k < nz; ++k) {
-    const int kb = (k + nz - 1) % nz, kt = (k + 1) % nz;
+    const int kb = nbr(k, -1, nz, bc), kt = nbr(k, 1, nz, bc);
     for (int j = 0; j < ny; ++j) {
-      const int js = (j + ny - 1) % ny, jn = (j + 1) % ny;
+      const int js = nbr(j, -1, ny, bc), jn = nbr(j, 1, ny, bc);
       for (int i = 0; i < nx; ++i) {
-        const int iw = (i + nx - 1) % nx, ie = (i + 1) % nx;
-        const double xw = x[IDX(iw, j, k, nx, ny)], xe = x[IDX(ie, j, k, nx, ny)];
-        const double xs = x[IDX(i, js, k, nx, ny)], xn = x[IDX(i, jn, k, nx, ny)];
-        const double xb = x[IDX(i, j, kb, nx, ny)], xt = x[IDX(i, j, kt, nx, ny)];
+        const int iw = nbr(i, -1, nx, bc), ie = nbr(i, 1, nx, bc);
+        const double xp = x[IDX(i, j, k, nx, ny)];
+        const double xw = nbv(x, iw, j, k, nx, ny, bc, xp), xe = nbv(x, ie, j, k, nx, ny, bc, xp);
+        const double xs = nbv(x, i, js, k, nx, ny, bc, xp), xn = nbv(x, i, jn, k, nx, ny, bc, xp);
+        const double xb = nbv(x, i, j, kb, nx, ny, bc, xp), xt = nbv(x, i, j, kt, nx, ny, bc, xp);
         const double sum = ((xw + xe) + (xs + xn)) + (xb + xt);
-        Ax[IDX(i, j, k, nx, ny)] = alpha * x[IDX(i, j, k, nx, ny)] + beta * sum;
+        Ax[IDX(i, j, k, nx, ny)] = alpha * xp + beta * sum;
       }
     }
+  }
+}
+
+/* the paper's operator (periodic) */
+void oracle_apply_op(int nx, int ny, int nz, double h, const double *x, double *Ax) {
+  oracle_apply_op_bc(nx, ny, nz, h, 0, x, Ax);
+}
+
+/* Variable-coefficient operator (variant N4, reading A23; the paper's BrickLib "nonconstant
+ * coefficients"): (A x)_p = inv * sum_n beta_n (x_n - x_p), beta_n = (c_p + c_n) * 0.5 the
+ * face coefficient between p and neighbour n (arithmetic mean of the cell coefficients), inv = 1/h^2,
+ * terms t_n = beta_n * (x_n - x_p) summed ((tW+tE)+(tS+tN))+(tB+tT).  Across a non-periodic
+ * domain face (reading A22) the neighbour's x is the boundary image of x_p and its c is c_p (the
+ * face coefficient is then c_p).  With c = 1 this is the paper's operator up to rounding. */
+void oracle_apply_op_vc(int nx, int ny, int nz, double h, int bc, const double *c, const double *x, double *Ax) {
+  const double inv = 1.0 / (h * h);
+#pragma omp parallel for schedule(static)
+  for (int k = 0; k < nz; ++k) {
+    const int kb = nbr(k, -1, nz, bc), kt = nbr(k, 1, nz, bc);
+    for (int j = 0; j < ny; ++j) {
+      const int js = nbr(j, -1, ny, bc), jn = nbr(j, 1, ny, bc);
+      for (int i = 0; i < nx; ++i) {
+        const int iw = nbr(i, -1, nx, bc), ie = nbr(i, 1, nx, bc);
+        const size_t p = IDX(i, j, k, nx, ny);
+        const double xp = x[p], cp = c[p];
+        const int na[6][3] = {{iw, j, k}, {ie, j, k}, {i, js, k}, {i, jn, k}, {i, j, kb}, {i, j, kt}};
+        double t[6];
+        for (int q = 0; q < 6; ++q) {
+          const int a = na[q][0], b = na[q][1], cc = na[q][2];
+          const double xn = nbv(x, a, b, cc, nx, ny, bc, xp);
+          const double cn = (a < 0 || b < 0 || cc < 0) ? cp : c[IDX(a, b, cc, nx, ny)];
+          t[q] = ((cp + cn) * 0.5) * (xn - xp);
+        }
+        Ax[p] = inv * (((t[0] + t[1]) + (t[2] + t[3])) + (t[4] + t[5]));
+      }
+    }
+  }
+}
+
+/* Damped-Jacobi step of the variable-coefficient operator (reading A23): gamma_p = omega / |diag_p|
+ * with omega = 1/2 and diag_p = -inv * S_p, S_p = ((bW+bE)+(bS+bN))+(bB+bT) the sum of the six face
+ * coefficients, i.e. gamma_p = (0.5*h*h) / S_p (c = 1: S_p = 6, gamma = h^2/12, the paper's step,
+ * P:L148). */
+void oracle_vc_gamma(int nx, int ny, int nz, double h, int bc, const double *c, double *gam) {
+  const double g = 0.5 * (h * h);
+#pragma omp parallel for schedule(static)
+  for (int k = 0; k < nz; ++k) {
+    const int kb = nbr(k, -1, nz, bc), kt = nbr(k, 1, nz, bc);
+    for (int j = 0; j < ny; ++j) {
+      const int js = nbr(j, -1, ny, bc), jn = nbr(j, 1, ny, bc);
+      for (int i = 0; i < nx; ++i) {
+        const int iw = nbr(i, -1, nx, bc), ie = nbr(i, 1, nx, bc);
+        const size_t p = IDX(i, j, k, nx, ny);
+        const double cp = c[p];
+        const int na[6][3] = {{iw, j, k}, {ie, j, k}, {i, js, k}, {i, jn, k}, {i, j, kb}, {i, j, kt}};
+        double f[6];
+        for (int q = 0; q < 6; ++q) {
+          const int a = na[q][0], b = na[q][1], cc = na[q][2];
+          const double cn = (a < 0 || b < 0 || cc < 0) ? cp : c[IDX(a, b, cc, nx, ny)];
+          f[q] = (cp + cn) * 0.5;
+        }
+        gam[p] = g / (((f[0] + f[1]) + (f[2] + f[3])) + (f[4] + f[5]));
+      }
+    }
+  }
+}
+
+/* smooth(+residual) with a step per cell (variable coefficients, reading A23):
+ * r = b - Ax (if r != NULL), x := x + gamma_p (Ax - b). */
+void oracle_smooth_residual_field(size_t n, const double *gam, double *x, const double *Ax, const double *b,
+                                  double *r) {
+#pragma omp parallel for schedule(static)
+  for (size_t p = 0; p < n; ++p) {
+    if (r) r[p] = b[p] - Ax[p];
+    x[p] = x[p] + gam[p] * (Ax[p] - b[p]);
   }
 }
 
@@ -190,12 +292,17 @@ void oracle_interpolation_increment(int nx, int ny, int nz, const double *xc, do
 /* maxNormRes (Alg 1): max over the domain of |b - Ax|, with a
  * fresh applyOp on the current x (reading A6).  A NaN anywhere makes the max NaN (a diverged
  * iterate must not pass the 1e-10 test): each thread keeps a NaN once it saw one, and so does the
- * combination of the threads' maxima. */
-double oracle_max_norm_residual(int nx, int ny, int nz, double h, const double *x, const double *b) {
+ * combination of the threads' maxima.  _ex: under the boundary condition bc (reading A22) and,
+ * with c != NULL, the variable-coefficient operator (reading A23). */
+double oracle_max_norm_residual_ex(int nx, int ny, int nz, double h, int bc, const double *c, const double *x,
+                                   const double *b) {
   const size_t n = (size_t)nx * ny * nz;
   double *Ax = (double *)malloc(n * sizeof(double));
   if (!Ax) return NAN;
-  oracle_apply_op(nx, ny, nz, h, x, Ax);
+  if (c)
+    oracle_apply_op_vc(nx, ny, nz, h, bc, c, x, Ax);
+  else
+    oracle_apply_op_bc(nx, ny, nz, h, bc, x, Ax);
   double m = 0.0;
 #pragma omp parallel
   {
@@ -212,6 +319,11 @@ double oracle_max_norm_residual(int nx, int ny, int nz, double h, const double *
   }
   free(Ax);
   return m;
+}
+
+/* the paper's norm (periodic, constant coefficients) */
+double oracle_max_norm_residual(int nx, int ny, int nz, double h, const double *x, const double *b) {
+  return oracle_max_norm_residual_ex(nx, ny, nz, h, 0, NULL, x, b);
 }
 
 /* Fixed-order dot product (reading A21): v_i = a_i * b_i over the lexicographic index, then for
@@ -286,6 +398,8 @@ typedef struct {
   int smoother, rho; /* 0 = damped Jacobi (the paper); 1 = Chebyshev (oracle_chebyshev_gamma) on pre/post;
                         2 = red-black Gauss-Seidel on pre/post (oracle_gsrb_half: red then black) */
   int bottom_solver;  /* 0 = `bottom` damped Jacobi smooths (the paper); 1 = `bottom` CG iterations (oracle_cg) */
+  int bc;             /* 0 = periodic (the paper); 1 = homogeneous Dirichlet; 2 = homogeneous Neumann (A22) */
+  double *c[ORACLE_MAX_LEVELS], *gam[ORACLE_MAX_LEVELS]; /* variable coefficients (A23): NULL = constant */
   int n[ORACLE_MAX_LEVELS][3];
   double h[ORACLE_MAX_LEVELS];
   double *x[ORACLE_MAX_LEVELS], *b[ORACLE_MAX_LEVELS], *Ax[ORACLE_MAX_LEVELS], *r[ORACLE_MAX_LEVELS];
@@ -300,6 +414,8 @@ void oracle_mg_destroy(oracle_mg *m) {
     free(m->b[l]);
     free(m->Ax[l]);
     free(m->r[l]);
+    free(m->c[l]);
+    free(m->gam[l]);
   }
   free(m);
 }
@@ -341,11 +457,67 @@ void oracle_mg_set_smoother(oracle_mg *m, int smoother, int rho) {
   m->smoother = smoother;
   m->rho = rho;
 }
-void oracle_mg_set_bottom_solver(oracle_mg *m, int solver) { m->bottom_solver = solver; }
+/* CG bottom (A21) only for the periodic constant-coefficient operator: -1 otherwise */
+int oracle_mg_set_bottom_solver(oracle_mg *m, int solver) {
+  if (solver == 1 && (m->bc != 0 || m->c[0])) return -1;
+  m->bottom_solver = solver;
+  return 0;
+}
 
-/* step of sweep it of n at level l (pre / post smoothing) */
-static double step_gamma(const oracle_mg *m, int l, int n, int it) {
-  return m->smoother ? oracle_chebyshev_gamma(m->h[l], n, it, m->rho) : (m->h[l] * m->h[l]) / 12.0;
+/* boundary condition of every level (reading A22) */
+int oracle_mg_set_bc(oracle_mg *m, int bc) {
+  if (bc < 0 || bc > 2 || (bc != 0 && m->bottom_solver == 1)) return -1;
+  m->bc = bc;
+  for (int l = 0; l < m->L && m->c[l]; ++l)
+    oracle_vc_gamma(m->n[l][0], m->n[l][1], m->n[l][2], m->h[l], m->bc, m->c[l], m->gam[l]);
+  return 0;
+}
+
+/* Variable coefficients (reading A23): c of level 0 (lexicographic, c > 0); coarse levels take the
+ * restriction (volume average) of the level above; the Jacobi steps gamma_p of every
+ * level follow (oracle_vc_gamma).  c0 == NULL restores the paper's constant operator. */
+int oracle_mg_set_coef(oracle_mg *m, const double *c0) {
+  for (int l = 0; l < m->L; ++l) {
+    free(m->c[l]);
+    free(m->gam[l]);
+    m->c[l] = m->gam[l] = NULL;
+  }
+  if (!c0) return 0;
+  if (m->bottom_solver == 1) return -1;
+  for (int l = 0; l < m->L; ++l) {
+    m->c[l] = (double *)malloc(lvl_n(m, l) * sizeof(double));
+    m->gam[l] = (double *)malloc(lvl_n(m, l) * sizeof(double));
+    if (!m->c[l] || !m->gam[l]) return -1;
+    if (l == 0)
+      memcpy(m->c[0], c0, lvl_n(m, 0) * sizeof(double));
+    else
+      oracle_restriction(m->n[l - 1][0], m->n[l - 1][1], m->n[l - 1][2], m->c[l - 1], m->c[l]);
+    oracle_vc_gamma(m->n[l][0], m->n[l][1], m->n[l][2], m->h[l], m->bc, m->c[l], m->gam[l]);
+  }
+  return 0;
+}
+
+/* the level's operator: the paper's (under bc) or the variable-coefficient one */
+static void level_apply(const oracle_mg *m, int l, const double *x, double *Ax) {
+  const int *n = m->n[l];
+  if (m->c[l])
+    oracle_apply_op_vc(n[0], n[1], n[2], m->h[l], m->bc, m->c[l], x, Ax);
+  else
+    oracle_apply_op_bc(n[0], n[1], n[2], m->h[l], m->bc, x, Ax);
+}
+
+/* one smooth(+residual) of level l with the step of sweep it of n (pre / post), or the bottom's */
+static void level_smooth(oracle_mg *m, int l, int n, int it, int write_r) {
+  if (m->c[l]) {
+    oracle_smooth_residual_field(lvl_n(m, l), m->gam[l], m->x[l], m->Ax[l], m->b[l], write_r ? m->r[l] : NULL);
+    return;
+  }
+  const double g = n > 0 ? (m->smoother ? oracle_chebyshev_gamma(m->h[l], n, it, m->rho) : (m->h[l] * m->h[l]) / 12.0)
+                         : (m->h[l] * m->h[l]) / 12.0;
+  if (write_r)
+    oracle_smooth_residual_gamma(lvl_n(m, l), g, m->x[l], m->Ax[l], m->b[l], m->r[l]);
+  else
+    oracle_smooth_gamma(lvl_n(m, l), g, m->x[l], m->Ax[l], m->b[l]);
 }
 
 void oracle_mg_set_b(oracle_mg *m, const double *b) { memcpy(m->b[0], b, lvl_n(m, 0) * sizeof(double)); }
@@ -364,22 +536,29 @@ int oracle_mg_get_level(const oracle_mg *m, int l, int which, double *out) {
   return 0;
 }
 
+/* `n` pre / post sweeps of level l (Alg 2 steps 2-6, 18-21): exchange() + applyOp, then
+ * smooth+residual; the GSRB variant (A20) a red then a black half-sweep per sweep. */
+static void level_sweeps(oracle_mg *m, int l, int n) {
+  const int *d = m->n[l];
+  for (int it = 0; it < n; ++it) {
+    if (m->smoother == 2 && !m->c[l]) { /* GSRB: red half, then black half */
+      for (int c = 0; c < 2; ++c) {
+        level_apply(m, l, m->x[l], m->Ax[l]);
+        oracle_gsrb_half(d[0], d[1], d[2], m->h[l], c, m->x[l], m->Ax[l], m->b[l], m->r[l]);
+      }
+      continue;
+    }
+    level_apply(m, l, m->x[l], m->Ax[l]); /* exchange()+applyOp */
+    level_smooth(m, l, n, it, 1);
+  }
+}
+
 /* Alg 2, levels 0..L-1 with the bottom solver at L-1 (readings A1-A3). */
 void oracle_mg_vcycle(oracle_mg *m) {
   const int L = m->L;
   for (int l = 0; l + 1 < L; ++l) {
     const int *n = m->n[l];
-    for (int it = 0; it < m->pre; ++it) {                       /* steps 2-6 */
-      if (m->smoother == 2) {                                    /* GSRB: red half, then black half */
-        for (int c = 0; c < 2; ++c) {
-          oracle_apply_op(n[0], n[1], n[2], m->h[l], m->x[l], m->Ax[l]);
-          oracle_gsrb_half(n[0], n[1], n[2], m->h[l], c, m->x[l], m->Ax[l], m->b[l], m->r[l]);
-        }
-        continue;
-      }
-      oracle_apply_op(n[0], n[1], n[2], m->h[l], m->x[l], m->Ax[l]); /* exchange()+applyOp */
-      oracle_smooth_residual_gamma(lvl_n(m, l), step_gamma(m, l, m->pre, it), m->x[l], m->Ax[l], m->b[l], m->r[l]);
-    }
+    level_sweeps(m, l, m->pre);                                 /* steps 2-6 */
     oracle_restriction(n[0], n[1], n[2], m->r[l], m->b[l + 1]); /* step 7 */
     oracle_init_zero(lvl_n(m, l + 1), m->x[l + 1]);             /* step 8 */
   }
@@ -389,30 +568,20 @@ void oracle_mg_vcycle(oracle_mg *m) {
     if (m->bottom_solver == 1) /* reading A21: x = 0 (initZero) and `bottom` CG iterations */
       oracle_cg(n[0], n[1], n[2], m->h[l], m->bottom, m->x[l], m->b[l]);
     else
-    for (int it = 0; it < m->bottom; ++it) {
-      oracle_apply_op(n[0], n[1], n[2], m->h[l], m->x[l], m->Ax[l]);
-      oracle_smooth(lvl_n(m, l), m->h[l], m->x[l], m->Ax[l], m->b[l]);
-    }
+      for (int it = 0; it < m->bottom; ++it) {
+        level_apply(m, l, m->x[l], m->Ax[l]);
+        level_smooth(m, l, 0, it, 0); /* smooth (damped Jacobi) */
+      }
   }
   for (int l = L - 2; l >= 0; --l) {                            /* steps 16-23 */
     const int *n = m->n[l];
     oracle_interpolation_increment(n[0], n[1], n[2], m->x[l + 1], m->x[l]);
-    for (int it = 0; it < m->post; ++it) {
-      if (m->smoother == 2) {
-        for (int c = 0; c < 2; ++c) {
-          oracle_apply_op(n[0], n[1], n[2], m->h[l], m->x[l], m->Ax[l]);
-          oracle_gsrb_half(n[0], n[1], n[2], m->h[l], c, m->x[l], m->Ax[l], m->b[l], m->r[l]);
-        }
-        continue;
-      }
-      oracle_apply_op(n[0], n[1], n[2], m->h[l], m->x[l], m->Ax[l]);
-      oracle_smooth_residual_gamma(lvl_n(m, l), step_gamma(m, l, m->post, it), m->x[l], m->Ax[l], m->b[l], m->r[l]);
-    }
+    level_sweeps(m, l, m->post);
   }
 }
 
 double oracle_mg_norm(const oracle_mg *m) {
-  return oracle_max_norm_residual(m->n[0][0], m->n[0][1], m->n[0][2], m->h[0], m->x[0], m->b[0]);
+  return oracle_max_norm_residual_ex(m->n[0][0], m->n[0][1], m->n[0][2], m->h[0], m->bc, m->c[0], m->x[0], m->b[0]);
 }
 
 /* Alg 1: while maxNormRes > tol: V-cycle; maxNormRes.  The cycle
