@@ -83,6 +83,14 @@ enum {
                              (self-exchange: measures communication avoiding on 1 GPU) */
 };
 
+/* bc: domain boundary condition of every level (variant; reading A22).
+ * PERIODIC is the paper's model problem.  DIRICHLET / NEUMANN are homogeneous conditions on
+ * the faces of the cell-centred grid: the neighbour across a domain face is -x_p / +x_p.  The library
+ * gives every axis a one-brick ghost shell; the domain-face ghost bricks hold the reflected values
+ * (filled by a "mirror exchange" wherever an exchange runs: method of images), so every kernel and
+ * the communication-avoiding schedule run unchanged. */
+enum { MG_BC_PERIODIC = 0, MG_BC_DIRICHLET = 1, MG_BC_NEUMANN = 2 };
+
 /* transport */
 enum { MG_TRANSPORT_AUTO = 0, MG_TRANSPORT_NCCL = 1, MG_TRANSPORT_LOCAL = 2, MG_TRANSPORT_PEER = 3 };
 #define MG_PEER_BLOB_BYTES 128
@@ -138,6 +146,12 @@ typedef struct {
                                     1 = `bottom_smooths` conjugate-gradient iterations from x = 0 with a
                                     fixed-order dot product (variant N4, reading A21; needs a
                                     coarsest grid of <= 8 bricks, globally when decomposed) */
+  int32_t bc;                    /* MG_BC_* (variant, reading A22): not with smoother 2 (its colours do not
+                                    commute with the reflection) or bottom_solver 1 (periodic null space) */
+  int32_t var_coef;              /* 1 = variable coefficients A x = div(c grad x) (variant, reading A23):
+                                    the cell coefficients are set with mg_set_coefficients before the first
+                                    V-cycle; the one-brick kernels run every level; smoother 0 and
+                                    bottom_solver 0 only */
   int32_t reserved[1];
   double h0;                     /* finest spacing; <= 0 => 1 / max_d(global N_d) (reading A7) */
 } mg_params;
@@ -185,6 +199,14 @@ mg_status mg_peer_connect(mg_ctx* c, const uint8_t* all_blobs);
  * (library-owned, freed by mg_destroy; not part of mg_workspace_bytes). */
 mg_status mg_set_rhs(mg_ctx* c, const double* b_dev);
 mg_status mg_set_rhs_host(mg_ctx* c, const double* b_host);
+/* Variable-coefficient variant (params var_coef = 1, reading A23): the cell coefficients
+ * c > 0 of level 0, local lexicographic like b (device pointer, 16-byte aligned, caller-owned, read
+ * during the call's stream work only).  Coarse levels take the restriction of c (volume average, the
+ * restriction operator of P:L69, L120); ghost bricks are exchanged (reflected evenly on domain faces).
+ * Must be called before the first V-cycle / norm (MG_ERR_STATE otherwise); MG_ERR_STATE on a context
+ * with var_coef = 0.  Loopback groups: mg_group_set_coefficients per rank, then
+ * mg_group_commit_coefficients. */
+mg_status mg_set_coefficients(mg_ctx* c, const double* c_dev);
 /* Initial guess; NULL => x = 0 (reading A9). */
 mg_status mg_set_solution(mg_ctx* c, const double* x_dev);
 mg_status mg_get_solution(mg_ctx* c, double* x_dev);
@@ -277,7 +299,9 @@ mg_status mg_group_ctx(mg_group* g, int32_t rank, mg_ctx** out); /* per-rank vie
 mg_status mg_group_vcycle(mg_group* g);
 mg_status mg_group_residual_norm(mg_group* g, double* out_max_abs);
 mg_status mg_group_set_rhs(mg_group* g, int32_t rank, const double* b_dev); /* then mg_group_commit_rhs */
-mg_status mg_group_commit_rhs(mg_group* g); /* exchanges level-0 b ghosts of every rank */
+mg_status mg_group_commit_rhs(mg_group* g);
+mg_status mg_group_set_coefficients(mg_group* g, int32_t rank, const double* c_dev);
+mg_status mg_group_commit_coefficients(mg_group* g); /* exchanges level-0 b ghosts of every rank */
 mg_status mg_group_set_solution(mg_group* g, int32_t rank, const double* x_dev);
 mg_status mg_group_destroy(mg_group* g);
 
@@ -307,6 +331,11 @@ mg_status mg_layout_adjacency(const mg_layout* lay, int32_t level, int32_t* out)
 mg_status mg_layout_coords(const mg_layout* lay, int32_t level, int32_t* out);
 mg_status mg_layout_parent(const mg_layout* lay, int32_t level, int32_t* out);
 mg_status mg_layout_plan(const mg_layout* lay, int32_t level, int32_t which /*0 send,1 recv*/, int64_t* out);
+/* Mirror table of a level (non-periodic bc, reading A22): *count entries of int32 (ghost brick,
+ * source brick, mask of the reflected axes, bit a = axis a) into out (3 * count int32, or NULL to
+ * query the count).  The ghost brick's cell (i,j,k) is the source's cell with i -> 7-i etc. on the
+ * reflected axes, negated once per reflection for Dirichlet. */
+mg_status mg_layout_mirror(const mg_layout* lay, int32_t level, int64_t* count, int32_t* out);
 mg_status mg_layout_pass_plan(const mg_layout* lay, int32_t level, int32_t idx, int64_t info[6], int32_t* meta,
                               int32_t* ctas);
 /* Replicated bottom (the coarsest level has a ghost shell and the global coarsest grid <= 64

@@ -43,6 +43,7 @@ struct DevLevel {
   double* b = nullptr;
   double* r = nullptr;
   double* Ax = nullptr;
+  double* cf = nullptr;  // variable coefficients (reading A23): cell coefficients c, ghosts exchanged once
   int32_t* adj = nullptr;
   int32_t* parent = nullptr;
   int32_t* coord = nullptr;
@@ -67,6 +68,10 @@ struct DevLevel {
   CopyRun* cruns = nullptr;
   int ncruns = 0;
   int64_t cmax = 0;
+  // non-periodic bc (reading A22): domain-face ghost bricks <- reflected source bricks (int3 each)
+  int32_t* mirror = nullptr;
+  int nmirror = 0;
+  double mirror_sign = 1.0;
 };
 
 struct Plan {
@@ -99,6 +104,7 @@ struct mg_ctx {
   cudaEvent_t ev_h2d[2] = {nullptr, nullptr}, ev_free[2] = {nullptr, nullptr};
   cudaEvent_t ev_norm = nullptr;           // completion of the last enqueued residual norm
   bool norm_pending = false;
+  bool coef_ready = false;  // var_coef: mg_set_coefficients (+ the group commit) has run
   unsigned long long* acc = nullptr;
   double* h_pinned = nullptr;
   ncclComm_t nccl = nullptr;
@@ -208,6 +214,7 @@ size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double**
     // Ax only for the paper's kernel set (MG_FUSION_PAPER: applyOp writes it, smooth+residual reads
     // it); a per-op call that asks for the paper set on another level allocates it lazily (ensure_ax)
     if (lay.p.fusion[l] == MG_FUSION_PAPER) d.Ax = (double*)take(fb);
+    if (lay.p.var_coef) d.cf = (double*)take(fb);
     d.adj = (int32_t*)take((size_t)L.n_stored * 8 * sizeof(int32_t));
     d.parent = (int32_t*)take((size_t)L.n_alloc * sizeof(int32_t));
     d.coord = (int32_t*)take((size_t)L.n_stored * 3 * sizeof(int32_t));
@@ -234,8 +241,13 @@ size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double**
       pr.args.nwarps = (int64_t)pt.warps.size() / 4;
       d.pairs.push_back(pr);
     }
+    // (sized rank-independently: every rank of a run carves the same layout -- the loopback group and the
+    // peer transport address other ranks' objects at this rank's offsets)
     d.ncruns = (int)L.recvs.size();
-    d.cruns = (CopyRun*)take((size_t)d.ncruns * 3 * sizeof(CopyRun));
+    d.cruns = (CopyRun*)take((size_t)L.n_recv_slots * 4 * sizeof(CopyRun));
+    d.nmirror = (int)(L.mirror.size() / 3);
+    d.mirror = (int32_t*)take(lay.p.bc != MG_BC_PERIODIC ? (size_t)L.n_ghost * 3 * sizeof(int32_t) : 0);
+    d.mirror_sign = lay.p.bc == MG_BC_DIRICHLET ? -1.0 : 1.0;
     d.h = lay.p.h0 * (double)(1 << l);
     d.c = level_coeffs(d.h);
     if (out) (*out)[l] = d;
@@ -282,6 +294,11 @@ mg_params normalized(const mg_params* p) {
     q.h0 = m > 0 ? 1.0 / (double)m : 1.0;
   }
   if (q.cheby_ratio <= 0) q.cheby_ratio = 6;
+  if (q.var_coef) {  // reading A23: the one-brick kernels carry the coefficient variant
+    q.sweep_kernel = 1;
+    q.temporal_blocking = 0;
+    q.bottom_mode = MG_BOTTOM_SWEEPS;
+  }
   return q;
 }
 
@@ -295,6 +312,14 @@ mg_status check_params(const mg_params& p) {
     return set_err(MG_ERR_INVALID_ARG, "bottom_solver must be 0 (Jacobi smooths) or 1 (CG)");
   if (p.smoother < 0 || p.smoother > 2)
     return set_err(MG_ERR_INVALID_ARG, "smoother must be 0 (Jacobi), 1 (Chebyshev) or 2 (red-black Gauss-Seidel)");
+  if (p.var_coef < 0 || p.var_coef > 1) return set_err(MG_ERR_INVALID_ARG, "var_coef must be 0 or 1");
+  if (p.var_coef) {
+    if (p.smoother != 0 || p.bottom_solver != 0)
+      return set_err(MG_ERR_INVALID_ARG, "var_coef needs smoother 0 and bottom_solver 0 (reading A23)");
+    for (int l = 0; l < MG_MAX_LEVELS; ++l)
+      if (p.fusion[l] == MG_FUSION_PAPER)
+        return set_err(MG_ERR_INVALID_ARG, "var_coef: the paper's kernel set has no coefficient variant");
+  }
   return MG_OK;
 }
 
@@ -343,7 +368,10 @@ mg_status prepare_plan(mg_ctx* c, mg_group* g, const std::vector<Op>& ops) {
 }
 
 // ------------------------------------------------------------- exchange
-double* field_ptr(mg_ctx* c, int l, int field, int xbuf) { return field ? c->dl[l].b : c->dl[l].x[xbuf]; }
+// field 0: x[xbuf], 1: b, 2: the coefficients (variable-coefficient variant)
+double* field_ptr(mg_ctx* c, int l, int field, int xbuf) {
+  return field == 0 ? c->dl[l].x[xbuf] : field == 1 ? c->dl[l].b : c->dl[l].cf;
+}
 
 mg_status do_exchange(mg_ctx* c, int l, int field, int xbuf, cudaStream_t s) {
   const LevelLayout& L = c->lay.lv[l];
@@ -352,7 +380,7 @@ mg_status do_exchange(mg_ctx* c, int l, int field, int xbuf, cudaStream_t s) {
   if (c->use_peer) {
     if (!c->peer_ready) return set_err(MG_ERR_STATE, "peer transport: call mg_peer_connect first");
     const DevLevel& d = c->dl[l];
-    const int fv = field ? 2 : xbuf;
+    const int fv = field == 0 ? xbuf : field + 1;
     CKC(c, launch_peer_copy(d.cruns + (size_t)fv * d.ncruns, d.ncruns, d.cmax, c->ps_nb, s));
   } else if (c->use_nccl) {
     CKN(c, ncclGroupStart());
@@ -364,9 +392,14 @@ mg_status do_exchange(mg_ctx* c, int l, int field, int xbuf, cudaStream_t s) {
   } else {
     // every run of the exchange in one copy kernel (tables built by fill_copy_tables)
     const DevLevel& d = c->dl[l];
-    const int fv = field ? 2 : xbuf;
+    const int fv = field == 0 ? xbuf : field + 1;
     CKC(c, launch_copy_runs(d.cruns + (size_t)fv * d.ncruns, d.ncruns, d.cmax, s));
   }
+  // the domain-face ghosts (non-periodic bc, reading A22): reflections of owned / just received
+  // bricks, so after the receives on the same stream
+  const DevLevel& d = c->dl[l];
+  // (the coefficients are reflected evenly whatever the bc: the face coefficient at a domain face is c_p)
+  if (d.nmirror > 0) CKC(c, launch_mirror(f, d.mirror, d.nmirror, field == 2 ? 1.0 : d.mirror_sign, s));
   return MG_OK;
 }
 
@@ -414,11 +447,12 @@ mg_status fill_copy_tables(mg_ctx* c) {
     const LevelLayout& L = c->lay.lv[l];
     DevLevel& d = c->dl[l];
     if (d.ncruns == 0) continue;
-    std::vector<CopyRun> h((size_t)d.ncruns * 3);
+    std::vector<CopyRun> h((size_t)d.ncruns * 4, CopyRun{nullptr, nullptr, 0});
     d.cmax = 0;
-    for (int fv = 0; fv < 3; ++fv) {
-      const int field = fv == 2 ? 1 : 0, xbuf = fv == 2 ? 0 : fv;
+    for (int fv = 0; fv < 4; ++fv) {  // x[0], x[1], b, coefficients
+      const int field = fv < 2 ? 0 : fv - 1, xbuf = fv < 2 ? fv : 0;
       double* f = field_ptr(c, l, field, xbuf);
+      if (!f) continue;
       for (int i = 0; i < d.ncruns; ++i) {
         const Run& r = L.recvs[(size_t)i];
         mg_ctx* src = c->group ? c->group->r[r.peer] : c;
@@ -464,6 +498,14 @@ mg_status sweep_range(mg_ctx* c, const Op& o, int64_t b0, int64_t b1, cudaStream
   a.gamma2 = o.g2 > 0 ? o.g2 : d.c.gamma;
   a.colour = o.c1;
   a.colour2 = o.c2;
+  unsigned fl = o.flags;
+  if (d.cf) {  // variable coefficients (reading A23): the one-brick kernel only (normalized() forces it)
+    a.cf = d.cf;
+    a.vc_g = 0.5 * (d.h * d.h);
+    fl |= SW_VARCOEF;
+    CKC(c, launch_sweep(a, fl, s));
+    return MG_OK;
+  }
   if (o.kind == OP_SWEEP2) {  // two sweeps in one pass: the builder only emits it where a plan exists
     for (const auto& pr : d.pairs) {
       if (pr.b0 == b0 && pr.b1 == b1 && pr.part == part) {
@@ -717,6 +759,8 @@ mg_status build_and_run(mg_ctx* c, mg_group* g, bool vcycle_graph, Builder& b) {
 // V-cycle for a single context or a lockstep group, via a cached CUDA graph
 mg_status vcycle_impl(mg_ctx* c, mg_group* g) {
   mg_ctx* c0 = g ? g->r[0] : c;
+  if (c0->lay.p.var_coef && !c0->coef_ready)
+    return set_err(MG_ERR_STATE, "var_coef: set the coefficients (mg_set_coefficients) first");
   cudaStream_t s = g ? g->stream : c->stream;
   const int key = c0->st[0].cur & 1;
   const bool graph = c0->lay.p.use_graph && !c0->timing;
@@ -797,6 +841,9 @@ mg_status init_ctx(mg_ctx* c, const mg_params& p, int rank, int world, int devic
     CKC(c, cudaMemcpyAsync(d.parent, par.data(), par.size() * sizeof(int32_t), cudaMemcpyHostToDevice, stream));
     CKC(c, cudaMemcpyAsync(d.coord, L.coord.data(), L.coord.size() * sizeof(int32_t), cudaMemcpyHostToDevice,
                            stream));
+    if (!L.mirror.empty())
+      CKC(c, cudaMemcpyAsync(d.mirror, L.mirror.data(), L.mirror.size() * sizeof(int32_t), cudaMemcpyHostToDevice,
+                             stream));
     for (size_t k = 0; k < L.cols.size(); ++k) {
       const auto& ct = L.cols[k];
       const ColArgs& ca = d.cols[k].args;
@@ -1038,6 +1085,34 @@ mg_status mg_set_rhs_host(mg_ctx* c, const double* b_host) {
   return MG_OK;
 }
 
+// Variable coefficients (reading A23): level-0 c from a local lexicographic array, coarse c = the
+// restriction of the level above (restrict_kernel: the canonical volume average), then (one rank) the
+// ghost bricks of every level by exchange / mirror (c is reflected evenly).  Group members restrict
+// locally; mg_group_commit_coefficients exchanges once every rank has its c.
+static mg_status set_coefficients_impl(mg_ctx* c, const double* c_dev, cudaStream_t s) {
+  if (!c->lay.p.var_coef) return set_err(MG_ERR_STATE, "var_coef is 0: this context has the paper's constant operator");
+  if (!c_dev || ((uintptr_t)c_dev & 15)) return set_err(MG_ERR_INVALID_ARG, "c must be a 16-byte aligned device pointer");
+  const LevelLayout& L0 = c->lay.lv[0];
+  CKC(c, launch_lex_to_brick(c_dev, c->dl[0].cf, c->dl[0].coord, L0.n_owned, L0.n[0], L0.n[1], s));
+  for (int l = 0; l + 1 < c->lay.L; ++l)
+    CKC(c, launch_restrict(c->dl[l].cf, c->dl[l + 1].cf, c->dl[l].parent, c->lay.lv[l].n_owned, s));
+  return MG_OK;
+}
+
+static mg_status exchange_coefficients(mg_ctx* c, cudaStream_t s) {
+  for (int l = 0; l < c->lay.L; ++l)
+    if (c->lay.lv[l].n_ghost > 0) CKS(do_exchange(c, l, 2, 0, s));
+  c->coef_ready = true;
+  return MG_OK;
+}
+
+mg_status mg_set_coefficients(mg_ctx* c, const double* c_dev) {
+  CKS(check_ctx(c));
+  if (c->group) return set_err(MG_ERR_STATE, "group member: use mg_group_set_coefficients");
+  CKS(set_coefficients_impl(c, c_dev, c->stream));
+  return exchange_coefficients(c, c->stream);
+}
+
 mg_status mg_set_solution(mg_ctx* c, const double* x_dev) {
   CKS(check_ctx(c));
   if (!x_dev) {
@@ -1080,6 +1155,8 @@ mg_status mg_residual_norm_async(mg_ctx* c) {
   CKS(check_ctx(c));
   if (c->group) return set_err(MG_ERR_STATE, "group member: use mg_group_residual_norm");
   if (c->norm_pending) return set_err(MG_ERR_STATE, "a residual norm is already pending: call mg_residual_norm_wait");
+  if (c->lay.p.var_coef && !c->coef_ready)
+    return set_err(MG_ERR_STATE, "var_coef: set the coefficients (mg_set_coefficients) first");
   const LevelLayout& L = c->lay.lv[0];
   DevLevel& d = c->dl[0];
   if (L.n_ghost > 0) {
@@ -1088,7 +1165,7 @@ mg_status mg_residual_norm_async(mg_ctx* c) {
     c->st[0].since = 0;
   }
   CKC(c, cudaMemsetAsync(c->acc, 0, sizeof(unsigned long long), c->stream));
-  CKC(c, launch_norm(d.x[c->st[0].cur], d.b, d.adj, L.n_owned, d.c, c->acc, c->stream));
+  CKC(c, launch_norm(d.x[c->st[0].cur], d.b, d.adj, L.n_owned, d.c, c->acc, c->stream, d.cf));
   if (c->use_nccl && c->lay.world > 1)
     CKN(c, ncclAllReduce(c->acc, c->acc, 1, ncclUint64, ncclMax, c->nccl, c->stream));
   if (c->use_peer && c->lay.world > 1) {
@@ -1493,6 +1570,21 @@ mg_status mg_group_set_solution(mg_group* g, int32_t rank, const double* x_dev) 
   return mg_set_solution(c, x_dev);
 }
 
+mg_status mg_group_set_coefficients(mg_group* g, int32_t rank, const double* c_dev) {
+  mg_ctx* c = nullptr;
+  CKS(mg_group_ctx(g, rank, &c));
+  return set_coefficients_impl(c, c_dev, g->stream);
+}
+
+mg_status mg_group_commit_coefficients(mg_group* g) {
+  if (!g) return set_err(MG_ERR_INVALID_ARG, "null group");
+  for (mg_ctx* c : g->r) {
+    CKS(check_ctx(c));
+    CKS(exchange_coefficients(c, g->stream));
+  }
+  return MG_OK;
+}
+
 mg_status mg_group_commit_rhs(mg_group* g) {
   if (!g) return set_err(MG_ERR_INVALID_ARG, "null group");
   for (mg_ctx* c : g->r) {
@@ -1513,6 +1605,8 @@ mg_status mg_group_residual_norm(mg_group* g, double* out) {
   if (!g || !out) return set_err(MG_ERR_INVALID_ARG, "null argument");
   mg_ctx* c0 = g->r[0];
   CKS(check_ctx(c0));
+  if (c0->lay.p.var_coef && !c0->coef_ready)
+    return set_err(MG_ERR_STATE, "var_coef: set the coefficients (mg_group_set_coefficients + commit) first");
   for (mg_ctx* c : g->r) {
     if (c->lay.lv[0].n_ghost > 0) {
       CKS(do_exchange(c, 0, 0, c->st[0].cur, g->stream));
@@ -1526,7 +1620,7 @@ mg_status mg_group_residual_norm(mg_group* g, double* out) {
   for (mg_ctx* c : g->r) {
     const LevelLayout& L = c->lay.lv[0];
     DevLevel& d = c->dl[0];
-    CKC(c0, launch_norm(d.x[c->st[0].cur], d.b, d.adj, L.n_owned, d.c, c0->acc, g->stream));
+    CKC(c0, launch_norm(d.x[c->st[0].cur], d.b, d.adj, L.n_owned, d.c, c0->acc, g->stream, d.cf));
   }
   CKC(c0, cudaMemcpyAsync(c0->h_pinned, c0->acc, 8, cudaMemcpyDeviceToHost, g->stream));
   CKC(c0, cudaStreamSynchronize(g->stream));
@@ -1632,6 +1726,15 @@ mg_status mg_layout_plan(const mg_layout* m, int32_t level, int32_t which, int64
     out[i * 6 + 4] = v[i].remote;
     out[i * 6 + 5] = v[i].count;
   }
+  return MG_OK;
+}
+
+mg_status mg_layout_mirror(const mg_layout* m, int32_t level, int64_t* count, int32_t* out) {
+  const LevelLayout* L = nullptr;
+  CKS(lay_level(m, level, &L));
+  if (!count) return set_err(MG_ERR_INVALID_ARG, "null count");
+  *count = (int64_t)(L->mirror.size() / 3);
+  if (out) std::memcpy(out, L->mirror.data(), L->mirror.size() * sizeof(int32_t));
   return MG_OK;
 }
 

@@ -64,9 +64,13 @@ __global__ void __launch_bounds__(256) sweep_kernel(SweepArgs p, unsigned long l
   constexpr bool RESTRICT = (FLAGS & SW_RESTRICT) != 0;
   constexpr bool INTERP = (FLAGS & SW_INTERP) != 0;
   constexpr bool ZERO_X = (FLAGS & SW_ZERO_X) != 0;
+  constexpr bool VC = (FLAGS & SW_VARCOEF) != 0;  // variable coefficients (reading A23)
   __shared__ __align__(16) double xs[512];
   __shared__ double hw[64], he[64], hs[64], hn[64], hb[64], ht[64];
   __shared__ __align__(16) double rs[RESTRICT ? 512 : 1];
+  // VC: the coefficient brick and its six face halos (the face coefficients need c of both cells)
+  __shared__ __align__(16) double cs[VC ? 512 : 1];
+  __shared__ double ch[VC ? 6 : 1][VC ? 64 : 1];
 
   const int t = threadIdx.x;
   const int64_t brick = p.brick0 + blockIdx.x;
@@ -125,6 +129,22 @@ __global__ void __launch_bounds__(256) sweep_kernel(SweepArgs p, unsigned long l
     }
     __syncthreads();
   }
+  if (VC) {
+    const double2 cv = ldg2(p.cf + brick * 512 + 2 * t);
+    cs[2 * t] = cv.x;
+    cs[2 * t + 1] = cv.y;
+    {
+      const int f = t >> 6, m = t & 63;
+      const int nb = __ldg(adj + f);
+      const int ci = f < 2 ? (f == 0 ? 7 : 0) : (m & 7), cj = f < 2 ? (m & 7) : (f == 2 ? 7 : 0), ck = m >> 3;
+      ch[f][m] = __ldg(p.cf + (int64_t)nb * 512 + ci + 8 * cj + 64 * ck);
+    }
+    if (t < 128) {
+      const int f = 4 + (t >> 6), m = t & 63;
+      ch[f][m] = __ldg(p.cf + (int64_t)__ldg(adj + f) * 512 + m + 64 * (f == 4 ? 7 : 0));
+    }
+    __syncthreads();
+  }
 
   double out[2], res[2];
   double mx = 0.0;
@@ -144,7 +164,23 @@ __global__ void __launch_bounds__(256) sweep_kernel(SweepArgs p, unsigned long l
       bt = k > 0 ? xs[o - 64] : hb[i + 8 * j];
       tp = k < 7 ? xs[o + 64] : ht[i + 8 * j];
     }
-    const double a = stencil_a(c, w, e, s, n, bt, tp, p.c.alpha, p.c.beta);
+    double a, gam = p.c.gamma;
+    if (VC) {
+      // (A x)_p = inv * sum_n ((c_p + c_n) * 0.5) * (x_n - x_p), gamma_p = (0.5 h h) / sum_n face coefficient
+      const double cp = cs[o];
+      const double cw = i > 0 ? cs[o - 1] : ch[0][j + 8 * k], ce = i < 7 ? cs[o + 1] : ch[1][j + 8 * k];
+      const double cS = j > 0 ? cs[o - 8] : ch[2][i + 8 * k], cN = j < 7 ? cs[o + 8] : ch[3][i + 8 * k];
+      const double cB = k > 0 ? cs[o - 64] : ch[4][i + 8 * j], cT = k < 7 ? cs[o + 64] : ch[5][i + 8 * j];
+      const double fw = DMUL(DADD(cp, cw), 0.5), fe = DMUL(DADD(cp, ce), 0.5), fs = DMUL(DADD(cp, cS), 0.5);
+      const double fn = DMUL(DADD(cp, cN), 0.5), fb = DMUL(DADD(cp, cB), 0.5), ft = DMUL(DADD(cp, cT), 0.5);
+      const double sum = DADD(DADD(DADD(DMUL(fw, DSUB(w, c)), DMUL(fe, DSUB(e, c))),
+                                   DADD(DMUL(fs, DSUB(s, c)), DMUL(fn, DSUB(n, c)))),
+                              DADD(DMUL(fb, DSUB(bt, c)), DMUL(ft, DSUB(tp, c))));
+      a = DMUL(p.c.beta, sum);
+      gam = __ddiv_rn(p.vc_g, DADD(DADD(DADD(fw, fe), DADD(fs, fn)), DADD(fb, ft)));
+    } else {
+      a = stencil_a(c, w, e, s, n, bt, tp, p.c.alpha, p.c.beta);
+    }
     const double bb = ii ? bv.y : bv.x;
     if (MODE == MODE_APPLY) {
       out[ii] = a;
@@ -152,7 +188,7 @@ __global__ void __launch_bounds__(256) sweep_kernel(SweepArgs p, unsigned long l
       mx = nan_max(mx, fabs(DSUB(bb, a)));
     } else {
       res[ii] = DSUB(bb, a);
-      out[ii] = keep_cell(p.colour, i, j, k) ? c : DADD(c, DMUL(p.c.gamma, DSUB(a, bb)));
+      out[ii] = keep_cell(p.colour, i, j, k) ? c : DADD(c, DMUL(gam, DSUB(a, bb)));
     }
   }
 
@@ -203,6 +239,17 @@ static cudaError_t launch_sweep_t(const SweepArgs& a, cudaStream_t s) {
 }
 
 cudaError_t launch_sweep(const SweepArgs& a, unsigned flags, cudaStream_t s) {
+  if (flags & SW_VARCOEF) {
+    switch (flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP | SW_ZERO_X)) {
+#define VC_CASE(F) \
+  case (F): return launch_sweep_t<(F) | SW_VARCOEF>(a, s);
+      VC_CASE(0) VC_CASE(SW_WRITE_R) VC_CASE(SW_RESTRICT) VC_CASE(SW_INTERP) VC_CASE(SW_INTERP | SW_WRITE_R)
+      VC_CASE(SW_INTERP | SW_RESTRICT) VC_CASE(SW_ZERO_X) VC_CASE(SW_ZERO_X | SW_WRITE_R)
+      VC_CASE(SW_ZERO_X | SW_RESTRICT)
+#undef VC_CASE
+      default: return cudaErrorInvalidValue;
+    }
+  }
   switch (flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP | SW_ZERO_X)) {
     case 0: return launch_sweep_t<0>(a, s);
     case SW_WRITE_R: return launch_sweep_t<SW_WRITE_R>(a, s);
@@ -457,7 +504,7 @@ cudaError_t launch_apply_op(const double* x, double* Ax, const int32_t* adj, int
 }
 
 cudaError_t launch_norm(const double* x, const double* b, const int32_t* adj, int64_t nbricks, Coeffs c,
-                        unsigned long long* acc, cudaStream_t s) {
+                        unsigned long long* acc, cudaStream_t s, const double* cf) {
   if (nbricks <= 0) return cudaSuccess;
   SweepArgs a{};
   a.x = x;
@@ -466,7 +513,11 @@ cudaError_t launch_norm(const double* x, const double* b, const int32_t* adj, in
   a.brick0 = 0;
   a.nbricks = nbricks;
   a.c = c;
-  launch_k(sweep_kernel<MODE_NORM, 0>, (unsigned)nbricks, 256, 0, s, a, acc);
+  a.cf = cf;
+  if (cf)
+    launch_k(sweep_kernel<MODE_NORM, SW_VARCOEF>, (unsigned)nbricks, 256, 0, s, a, acc);
+  else
+    launch_k(sweep_kernel<MODE_NORM, 0>, (unsigned)nbricks, 256, 0, s, a, acc);
   return cudaGetLastError();
 }
 
@@ -675,6 +726,31 @@ cudaError_t launch_brick_to_lex(const double* bricks, double* lex, const int32_t
 }
 
 // blockIdx.y = run; the x-blocks stride over its 16-byte words
+// Mirror exchange (reading A22, method of images): one CTA per domain-face ghost brick, two cells per
+// thread; the cell (i, j, k) of the ghost brick takes cell (i', j', k') of its source brick, i' = 7 - i
+// on a reflected axis, negated once per reflection for Dirichlet (negation is exact).
+__global__ void __launch_bounds__(256) mirror_kernel(double* __restrict__ f, const int32_t* __restrict__ tab,
+                                                     double sign) {
+  pdl_begin();
+  const int e = blockIdx.x, t = threadIdx.x;
+  const int dst = __ldg(tab + 3 * e), src = __ldg(tab + 3 * e + 1), mask = __ldg(tab + 3 * e + 2);
+  const double s = (__popc(mask) & 1) ? sign : 1.0;
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {
+    const int c = t + 256 * h;
+    const int i = c & 7, j = (c >> 3) & 7, k = c >> 6;
+    const int is = (mask & 1) ? 7 - i : i, js = (mask & 2) ? 7 - j : j, ks = (mask & 4) ? 7 - k : k;
+    const double v = f[(int64_t)src * 512 + is + 8 * js + 64 * ks];
+    f[(int64_t)dst * 512 + c] = s < 0.0 ? -v : v;
+  }
+}
+
+cudaError_t launch_mirror(double* f, const int32_t* table, int n, double sign, cudaStream_t s) {
+  if (n <= 0) return cudaSuccess;
+  launch_k(mirror_kernel, (unsigned)n, 256, 0, s, f, table, sign);
+  return cudaGetLastError();
+}
+
 __global__ void __launch_bounds__(256) copy_runs_kernel(const CopyRun* __restrict__ runs) {
   pdl_begin();
   const CopyRun r = runs[blockIdx.y];

@@ -22,6 +22,7 @@ enum SweepFlags : unsigned {
   SW_ZERO_X = 8u,      // x == 0 (initZero folded into the first coarse sweep)
   SW_NO_SMOOTH = 16u,  // do not write x' (restriction-only last sweep is never used; kept for tests)
   SW_COLOUR = 32u,     // two-sweep kernel: red-black half-sweeps (colour masks compiled in only here)
+  SW_VARCOEF = 64u,    // one-brick kernel: variable coefficients div(c grad x) (reading A23), SweepArgs::cf
 };
 
 struct SweepArgs {
@@ -38,6 +39,8 @@ struct SweepArgs {
   double gamma2;     // two-sweep kernels: the step of the second sweep
   int colour = -1;   // red-black half-sweep (GSRB variant): update only cells with (i+j+k) mod 2 == colour,
   int colour2 = -1;  // keep the others (r still on every cell); -1 = every cell.  colour2: second sweep
+  const double* cf = nullptr;  // SW_VARCOEF: cell coefficients c (brick layout, ghosts valid)
+  double vc_g = 0.0;           // SW_VARCOEF: 0.5 * h * h (gamma_p = vc_g / sum of the face coefficients)
 };
 
 cudaError_t launch_sweep(const SweepArgs& a, unsigned flags, cudaStream_t s);
@@ -125,7 +128,7 @@ cudaError_t launch_interp(double* x, const double* xc, const int32_t* parent, in
 cudaError_t launch_zero(double* x, int64_t brick0, int64_t nbricks, cudaStream_t s);
 // max |b - Ax| over bricks [0, n) -> atomicMax on *acc (uint64 bits of a non-negative double)
 cudaError_t launch_norm(const double* x, const double* b, const int32_t* adj, int64_t nbricks, Coeffs c,
-                        unsigned long long* acc, cudaStream_t s);
+                        unsigned long long* acc, cudaStream_t s, const double* cf = nullptr);
 // resident bottom solve: all `nbricks` (<= kResidentMaxBricks, no ghosts) in one CTA's shared memory
 constexpr int kResidentMaxBricks = 8;
 cudaError_t launch_bottom_resident(const double* x, double* xo, const double* b, const int32_t* adj, int nbricks,
@@ -143,6 +146,10 @@ struct CopyRun {
   int64_t n;
 };
 cudaError_t launch_copy_runs(const CopyRun* runs, int nruns, int64_t max_n, cudaStream_t s);
+// Mirror exchange (non-periodic bc, reading A22): for each entry (dst, src, mask) of the
+// int32[n][3] table, brick dst = sign^popcount(mask) x brick src with the cells reversed on the axes
+// of mask (bit a: axis a).  sign = -1 (Dirichlet) or +1 (Neumann).
+cudaError_t launch_mirror(double* f, const int32_t* table, int n, double sign, cudaStream_t s);
 // Exchange between processes over peer memory (peer.cu): the copy runs read other ranks' fields
 // through CUDA IPC mappings; device-side flags order them (ready / done per epoch, see peer.cu).
 constexpr int kPeerSlotU64 = 16;  // one flag per 128-byte slot

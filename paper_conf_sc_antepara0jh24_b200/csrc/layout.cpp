@@ -38,6 +38,17 @@ int neighbour_rank(const Layout& lay, int dx, int dy, int dz) {
   return cx + P[0] * (cy + P[1] * cz);
 }
 
+// true if rank coords + (dx,dy,dz) leaves the global domain on an axis (non-periodic bc only)
+bool crosses_boundary(const Layout& lay, int dx, int dy, int dz) {
+  if (lay.p.bc == MG_BC_PERIODIC) return false;
+  const int d[3] = {dx, dy, dz};
+  for (int a = 0; a < 3; ++a) {
+    const int c = lay.coords[a] + d[a];
+    if (c < 0 || c >= lay.p.proc_grid[a]) return true;
+  }
+  return false;
+}
+
 int64_t LevelLayout::ext_index(int x, int y, int z) const {
   const int ex = nb[0] + 2 * g[0], ey = nb[1] + 2 * g[1];
   const int ez = nb[2] + 2 * g[2];
@@ -68,7 +79,9 @@ static void build_level(const Layout& lay, int l, LevelLayout& L) {
   for (int a = 0; a < 3; ++a) {
     L.n[a] = p.n_local[a] >> l;
     L.nb[a] = L.n[a] / kB;
-    L.g[a] = (p.ghost_mode == MG_GHOST_ALL || p.proc_grid[a] > 1) ? 1 : 0;
+    // a one-brick ghost shell on decomposed axes, on every axis in MG_GHOST_ALL, and on every axis
+    // with a non-periodic boundary (its domain-face ghosts hold the reflected values, reading A22)
+    L.g[a] = (p.ghost_mode == MG_GHOST_ALL || p.proc_grid[a] > 1 || p.bc != MG_BC_PERIODIC) ? 1 : 0;
   }
   const int nbx = L.nb[0], nby = L.nb[1], nbz = L.nb[2];
   const int ex = nbx + 2 * L.g[0], ey = nby + 2 * L.g[1], ez = nbz + 2 * L.g[2];
@@ -106,6 +119,7 @@ static void build_level(const Layout& lay, int l, LevelLayout& L) {
   // ---- ghost bricks, by receiver direction, in the sender's storage order ----
   L.sends.clear();
   L.recvs.clear();
+  L.n_recv_slots = 0;
   int64_t next = L.n_owned;
   for (int d = 0; d < 27; ++d) {
     int dx, dy, dz;
@@ -137,6 +151,9 @@ static void build_level(const Layout& lay, int l, LevelLayout& L) {
     std::sort(set.begin(), set.end());
     const int recv_peer = neighbour_rank(lay, dx, dy, dz);     // my ghost d comes from me+d
     const int send_peer = neighbour_rank(lay, -dx, -dy, -dz);  // my bricks go to me-d (its ghost d)
+    // non-periodic boundary (reading A22): nothing crosses a domain face -- ghosts beyond it are
+    // filled by the mirror table below, and a rank on the face sends nothing across it
+    const bool recv_cross = crosses_boundary(lay, dx, dy, dz), send_cross = crosses_boundary(lay, -dx, -dy, -dz);
     const int64_t gstart = next;
     int run = 0;
     for (size_t m = 0; m < set.size();) {
@@ -144,8 +161,9 @@ static void build_level(const Layout& lay, int l, LevelLayout& L) {
       while (e < set.size() && set[e].first == set[e - 1].first + 1) ++e;
       const int64_t cnt = (int64_t)(e - m);
       const int64_t goff = gstart + (int64_t)m;
-      L.recvs.push_back({recv_peer, d, run, goff, set[m].first, cnt});
-      L.sends.push_back({send_peer, d, run, set[m].first, goff, cnt});
+      ++L.n_recv_slots;  // (counted with the dropped ones: the workspace carve must not depend on the rank)
+      if (!recv_cross) L.recvs.push_back({recv_peer, d, run, goff, set[m].first, cnt});
+      if (!send_cross) L.sends.push_back({send_peer, d, run, set[m].first, goff, cnt});
       ++run;
       m = e;
     }
@@ -164,6 +182,26 @@ static void build_level(const Layout& lay, int l, LevelLayout& L) {
   }
   L.n_stored = next;
   L.n_ghost = next - L.n_owned;
+  // mirror table (reading A22, method of images): a ghost brick beyond a domain face is the owned (or
+  // received) brick reflected across every domain face it lies beyond, cells reversed on those axes,
+  // times -1 per reflection (Dirichlet) or +1 (Neumann); filled after the receives of an exchange
+  L.mirror.clear();
+  if (p.bc != MG_BC_PERIODIC) {
+    for (int64_t b = L.n_owned; b < L.n_stored; ++b) {
+      const int* e = &L.coord[(size_t)b * 3];
+      int q[3], mask = 0;
+      for (int a = 0; a < 3; ++a) {
+        q[a] = e[a];
+        if (e[a] < 0 && lay.coords[a] == 0) q[a] = 0, mask |= 1 << a;
+        if (e[a] >= L.nb[a] && lay.coords[a] == p.proc_grid[a] - 1) q[a] = L.nb[a] - 1, mask |= 1 << a;
+      }
+      if (!mask) continue;
+      const int64_t src = L.ext_index(q[0], q[1], q[2]);
+      L.mirror.push_back((int32_t)b);
+      L.mirror.push_back((int32_t)src);
+      L.mirror.push_back(mask);
+    }
+  }
   L.zero_brick = next;
   L.n_alloc = next + 1;
   // NCCL matches sends/recvs between a pair in posting order: sort both by (peer, dir, run)
@@ -249,6 +287,14 @@ mg_status build_layout(const mg_params& p, int rank, int world, Layout& out, std
       return MG_ERR_INVALID_ARG;
     }
   }
+  if (p.bc < MG_BC_PERIODIC || p.bc > MG_BC_NEUMANN) {
+    msg = "bc must be 0 (periodic), 1 (Dirichlet) or 2 (Neumann)";
+    return MG_ERR_INVALID_ARG;
+  }
+  if (p.bc != MG_BC_PERIODIC && (p.smoother == 2 || p.bottom_solver == 1)) {
+    msg = "a non-periodic bc needs smoother 0/1 and bottom_solver 0 (reading A22)";
+    return MG_ERR_INVALID_ARG;
+  }
   if (p.ghost_mode != MG_GHOST_AUTO && p.ghost_mode != MG_GHOST_ALL) {
     msg = "ghost_mode must be 0 or 1";
     return MG_ERR_INVALID_ARG;
@@ -272,7 +318,8 @@ mg_status build_layout(const mg_params& p, int rank, int world, Layout& out, std
   // replicated bottom: the global coarsest level as one rank would store it
   const LevelLayout& B = out.lv[(size_t)out.L - 1];
   out.repl = false;
-  if (out.L >= 2 && B.n_ghost > 0 && p.bottom_smooths > 0 && p.bottom_mode != MG_BOTTOM_SWEEPS) {
+  if (out.L >= 2 && B.n_ghost > 0 && p.bottom_smooths > 0 && p.bottom_mode != MG_BOTTOM_SWEEPS &&
+      p.bc == MG_BC_PERIODIC) {
     Layout g;
     g.p = p;
     for (int a = 0; a < 3; ++a) {

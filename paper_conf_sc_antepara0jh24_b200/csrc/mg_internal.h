@@ -47,6 +47,8 @@ struct LevelLayout {
   std::vector<int32_t> coord;   // [n_stored][3] extended brick coords
   std::vector<int32_t> parent;  // [n_stored] coarse brick * 8 + octant, -1 if none
   std::vector<Run> sends, recvs;
+  int64_t n_recv_slots = 0;     // receive runs before a non-periodic bc drops those across domain faces
+  std::vector<int32_t> mirror;  // [n][3] ghost brick, source brick, reflected-axes mask (bc != periodic)
   int64_t ext_index(int x, int y, int z) const;  // -1 if not stored
   std::vector<int32_t> ext2idx;  // dense map over the extended box
   // Column plans for the streaming sweep kernel: the bricks of a range [b0,b1)
@@ -159,5 +161,6 @@ inline void dir_from_index(int d, int& dx, int& dy, int& dz) {
   dz = d / 9 - 1;
 }
 int neighbour_rank(const Layout& lay, int dx, int dy, int dz);
+bool crosses_boundary(const Layout& lay, int dx, int dy, int dz);
 
 }  // namespace mgb

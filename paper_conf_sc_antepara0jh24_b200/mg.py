@@ -53,10 +53,14 @@ class mg_params(ctypes.Structure):
         ("cheby_ratio", ctypes.c_int32),
         ("launch_pdl", ctypes.c_int32),
         ("bottom_solver", ctypes.c_int32),
+        ("bc", ctypes.c_int32),
+        ("var_coef", ctypes.c_int32),
         ("reserved", ctypes.c_int32 * 1),
         ("h0", ctypes.c_double),
     ]
 
+
+MG_BC_PERIODIC, MG_BC_DIRICHLET, MG_BC_NEUMANN = 0, 1, 2
 
 _lib = None
 
@@ -71,6 +75,7 @@ _SIGS = {
     "mg_set_rhs": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
     "mg_set_rhs_host": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
     "mg_set_solution": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
+    "mg_set_coefficients": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
     "mg_get_solution": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
     "mg_get_solution_host": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
     "mg_vcycle": (ctypes.c_int, [ctypes.c_void_p]),
@@ -110,6 +115,8 @@ _SIGS = {
     "mg_group_residual_norm": (ctypes.c_int, [ctypes.c_void_p, ctypes.POINTER(ctypes.c_double)]),
     "mg_group_set_rhs": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_void_p]),
     "mg_group_commit_rhs": (ctypes.c_int, [ctypes.c_void_p]),
+    "mg_group_set_coefficients": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_void_p]),
+    "mg_group_commit_coefficients": (ctypes.c_int, [ctypes.c_void_p]),
     "mg_group_set_solution": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_void_p]),
     "mg_group_destroy": (ctypes.c_int, [ctypes.c_void_p]),
     "mg_layout_create": (ctypes.c_int, [ctypes.POINTER(mg_params), ctypes.c_int32, ctypes.c_int32,
@@ -119,6 +126,7 @@ _SIGS = {
     "mg_layout_coords": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_void_p]),
     "mg_layout_parent": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_void_p]),
     "mg_layout_plan": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32, ctypes.c_void_p]),
+    "mg_layout_mirror": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_void_p, ctypes.c_void_p]),
     "mg_layout_pass_plan": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32, ctypes.c_void_p,
                                            ctypes.c_void_p, ctypes.c_void_p]),
     "mg_layout_repl": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
@@ -160,7 +168,8 @@ def check(status: int, where: str) -> int:
 
 def params(n_local, proc_grid=(1, 1, 1), num_levels=6, pre=12, post=12, bottom=100, ca_period=None, fusion=None,
            ghost_mode=MG_GHOST_AUTO, transport=MG_TRANSPORT_AUTO, use_graph=1, bottom_mode=MG_BOTTOM_AUTO,
-           overlap=1, h0=0.0, sweep_kernel=0, temporal_blocking=3, smoother=0, cheby_ratio=0, launch_pdl=0, bottom_solver=0) -> mg_params:
+           overlap=1, h0=0.0, sweep_kernel=0, temporal_blocking=3, smoother=0, cheby_ratio=0, launch_pdl=0, bottom_solver=0,
+           bc=0, var_coef=0) -> mg_params:
     p = mg_params()
     lib().mg_params_default(ctypes.byref(p))
     p.n_local[:] = [int(v) for v in n_local]
@@ -178,6 +187,7 @@ def params(n_local, proc_grid=(1, 1, 1), num_levels=6, pre=12, post=12, bottom=1
     p.smoother, p.cheby_ratio = int(smoother), int(cheby_ratio)
     p.launch_pdl = int(launch_pdl)
     p.bottom_solver = int(bottom_solver)
+    p.bc, p.var_coef = int(bc), int(var_coef)
     return p
 
 
@@ -207,6 +217,10 @@ def mg_set_rhs(ctx, b_ptr):
 
 def mg_set_rhs_host(ctx, b_host_ptr):
     return check(lib().mg_set_rhs_host(ctx, b_host_ptr), "mg_set_rhs_host")
+
+
+def mg_set_coefficients(ctx, c_ptr):
+    return check(lib().mg_set_coefficients(ctx, c_ptr), "mg_set_coefficients")
 
 
 def mg_set_solution(ctx, x_ptr):
@@ -367,6 +381,14 @@ def mg_group_commit_rhs(g):
     return check(lib().mg_group_commit_rhs(g), "mg_group_commit_rhs")
 
 
+def mg_group_set_coefficients(g, rank, ptr):
+    return check(lib().mg_group_set_coefficients(g, rank, ptr), "mg_group_set_coefficients")
+
+
+def mg_group_commit_coefficients(g):
+    return check(lib().mg_group_commit_coefficients(g), "mg_group_commit_coefficients")
+
+
 def mg_group_set_solution(g, rank, ptr):
     return check(lib().mg_group_set_solution(g, rank, ptr), "mg_group_set_solution")
 
@@ -411,6 +433,16 @@ class Layout:
         adj = np.zeros((info[0], 8), dtype=np.int32)
         check(lib().mg_layout_repl(self.h, info, src.ctypes.data, mine.ctypes.data, adj.ctypes.data), "mg_layout_repl")
         return src, mine, adj
+
+    def mirror(self, level):
+        """[n][3] (ghost brick, source brick, reflected-axes mask) of a non-periodic bc (reading A22)."""
+        np = self._np
+        n = ctypes.c_int64()
+        check(lib().mg_layout_mirror(self.h, level, ctypes.byref(n), None), "mg_layout_mirror")
+        a = np.zeros((n.value, 3), dtype=np.int32)
+        if n.value:
+            check(lib().mg_layout_mirror(self.h, level, ctypes.byref(n), a.ctypes.data), "mg_layout_mirror")
+        return a
 
     def adjacency(self, level):
         inf = self.info(level)

@@ -27,6 +27,8 @@ class RankLevel:
         self.n_owned = self.info["owned"]
         self.n_alloc = self.info["alloc"]
         self.n = self.info["n"]  # x, y, z
+        self.mirror = lay.mirror(level)  # non-periodic bc (reading A22): (ghost, source, reflected axes)
+        self.mirror_sign = -1.0 if lay.p.bc == 1 else 1.0
 
     def zeros(self):
         return np.zeros((self.n_alloc, 8, 8, 8))  # [brick][k][j][i]
@@ -102,12 +104,24 @@ def interp(xf, fine: RankLevel, xc):
         xf[q] = xf[q] + np.repeat(np.repeat(np.repeat(blk, 2, 0), 2, 1), 2, 2)
 
 
+def apply_mirror(f, L: RankLevel):
+    """Domain-face ghost bricks from their reflected sources (after the receives)."""
+    for dst, src, mask in L.mirror:
+        blk = f[src]
+        for a, ax in ((0, 2), (1, 1), (2, 0)):  # brick array axes [k][j][i]
+            if mask >> a & 1:
+                blk = np.flip(blk, axis=ax)
+        f[dst] = blk * (L.mirror_sign ** bin(int(mask)).count("1"))
+
+
 def exchange_local(fields, levels):
     """In-process exchange of ghost bricks for all ranks (fields[r] is that rank's array)."""
     out = [f.copy() for f in fields]
     for r, L in enumerate(levels):
         for peer, d, run, local, remote, count in L.recvs:
             out[r][local:local + count] = fields[peer][remote:remote + count]
+    for r, L in enumerate(levels):
+        apply_mirror(out[r], L)
     return out
 
 

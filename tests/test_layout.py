@@ -168,6 +168,74 @@ def test_brick_interpreter_vcycle_bitwise_vs_oracle(oracle_mod, n_local, pg, L, 
     assert np.array_equal(got, want)
 
 
+BC_CASES = [((32, 32, 32), (1, 1, 1), 3, 1), ((16, 32, 16), (2, 1, 1), 2, 1), ((16, 16, 16), (2, 2, 2), 2, 2),
+            ((16, 16, 32), (1, 2, 3), 2, 1), ((32, 32, 32), (2, 1, 1), 3, 2)]
+
+
+@pytest.mark.parametrize("n_local,pg,L,bc", BC_CASES)
+def test_mirror_tables_and_dropped_runs(n_local, pg, L, bc):
+    """Non-periodic bc (reading A22): every axis has a ghost shell; no run crosses a domain face;
+    every ghost brick is filled exactly once, by a receive or by a mirror entry whose source is the
+    brick reflected across exactly the domain faces it lies beyond (owned or received)."""
+    _, lays = layouts(n_local, pg, L, bc=bc)
+    for r, lay in enumerate(lays):
+        cx, cy, cz = mg_inputs.rank_coords(r, pg)
+        rc = (cx, cy, cz)
+        for l in range(L):
+            inf = lay.info(l)
+            assert all(inf["ghost"])
+            co = lay.coords(l)
+            index = {tuple(c): q for q, c in enumerate(co)}
+            got = np.zeros(inf["owned"] + inf["nghost"], dtype=int)
+            for peer, d, run, local, remote, count in lay.plan(l, 1):
+                got[local:local + count] += 1
+                dd = (d % 3 - 1, (d // 3) % 3 - 1, d // 9 - 1)
+                assert all(0 <= rc[a] + dd[a] < pg[a] for a in range(3))  # never across a domain face
+            for peer, d, run, local, remote, count in lay.plan(l, 0):
+                dd = (d % 3 - 1, (d // 3) % 3 - 1, d // 9 - 1)
+                assert all(0 <= rc[a] - dd[a] < pg[a] for a in range(3))
+            for dst, src, mask in lay.mirror(l):
+                got[dst] += 1
+                e, q = list(co[dst]), list(co[src])
+                for a in range(3):
+                    beyond = (e[a] < 0 and rc[a] == 0) or (e[a] >= inf["nb"][a] and rc[a] == pg[a] - 1)
+                    assert bool(mask >> a & 1) == beyond
+                    assert q[a] == (min(max(e[a], 0), inf["nb"][a] - 1) if beyond else e[a])
+            assert np.all(got[inf["owned"]:] == 1) and np.all(got[:inf["owned"]] == 0)
+
+
+@pytest.mark.parametrize("n_local,pg,L,bc", BC_CASES)
+def test_brick_interpreter_bc_vcycle_bitwise_vs_oracle(oracle_mod, n_local, pg, L, bc):
+    """Dirichlet / Neumann (reading A22) on the library's layout tables: exchanges plus mirror
+    fills reproduce the oracle's V-cycle (3/3/20 sweeps) bit for bit, decomposed or not."""
+    p, lays = layouts(n_local, pg, L, bc=bc)
+    gshape = (n_local[2] * pg[2], n_local[1] * pg[1], n_local[0] * pg[0])
+    b = mg_inputs.random_field(gshape, 17)
+    pre, post, bottom = 3, 3, 20
+    h0 = mg_inputs.default_h0(gshape)
+    orc = oracle_mod.OracleMG(gshape, L, pre, post, bottom, h0, bc=bc)
+    orc.set_b(b)
+    orc.set_x(None)
+    orc.vcycle()
+    want = orc.get_x()
+    R = len(lays)
+    ranks = [[bi.RankLevel(lays[r], l) for l in range(L)] for r in range(R)]
+    xs = [[ranks[r][l].zeros() for l in range(L)] for r in range(R)]
+    bs = [[None] * L for _ in range(R)]
+    for r in range(R):
+        bs[r][0] = ranks[r][0].to_bricks(mg_inputs.local_block(b, r, pg))
+    b0 = bi.exchange_local([bs[r][0] for r in range(R)], [ranks[r][0] for r in range(R)])
+    for r in range(R):
+        bs[r][0] = b0[r]
+    xs = bi.vcycle_ranks(xs, bs, ranks, L, h0, pre, post, bottom)
+    got = np.zeros(gshape)
+    for r in range(R):
+        cx, cy, cz = mg_inputs.rank_coords(r, pg)
+        nx, ny, nz = n_local
+        got[cz * nz:(cz + 1) * nz, cy * ny:(cy + 1) * ny, cx * nx:(cx + 1) * nx] = ranks[r][0].from_bricks(xs[r][0])
+    assert np.array_equal(got, want)
+
+
 def test_invalid_params_rejected():
     bad = [mg.params((30, 32, 32), num_levels=1),  # not a multiple of 8
            mg.params((32, 32, 32), num_levels=4),  # 32 not a multiple of 8*2^3
@@ -270,3 +338,38 @@ def _check_pencil_plan(meta, ctas, nrange, adj, crd, par, g):
     ideal = sum(work) / len(work)
     assert max(work) <= ideal * 1.15 + 8
     return seen
+
+
+def test_variant_combinations_rejected():
+    """bc != periodic with GSRB / the CG bottom, var_coef with a smoother variant, the CG bottom or the
+    paper's kernel set, and out-of-range codes are refused at parameter validation (no GPU needed)."""
+    bad = [dict(bc=1, smoother=2), dict(bc=2, bottom_solver=1), dict(bc=3), dict(var_coef=1, smoother=1),
+           dict(var_coef=1, bottom_solver=1), dict(var_coef=1, fusion=1), dict(var_coef=2)]
+    for kw in bad:
+        p = mg.params((32, 32, 32), num_levels=2, **kw)
+        with pytest.raises(mg.MGError):
+            mg.mg_workspace_bytes(p, 0, 1)
+    for kw in (dict(bc=1), dict(bc=2, smoother=1), dict(var_coef=1, bc=1)):
+        assert mg.mg_workspace_bytes(mg.params((32, 32, 32), num_levels=2, **kw), 0, 1) > 0
+
+
+def test_var_coef_workspace_holds_a_coefficient_field():
+    """var_coef adds one field (n_alloc bricks) per level; bc adds the ghost shell on every axis."""
+    base = mg.mg_workspace_bytes(mg.params((32, 32, 32), num_levels=2, sweep_kernel=1, temporal_blocking=0,
+                                           bottom_mode=1), 0, 1)
+    vc = mg.mg_workspace_bytes(mg.params((32, 32, 32), num_levels=2, var_coef=1), 0, 1)
+    lay = mg.Layout(mg.params((32, 32, 32), num_levels=2), 0, 1)
+    field_bytes = sum(lay.info(l)["alloc"] * 512 * 8 for l in range(2))
+    assert field_bytes <= vc - base <= field_bytes + 4096 * 2
+
+
+@pytest.mark.parametrize("n_local,pg,L,bc", BC_CASES)
+def test_workspace_is_rank_independent(n_local, pg, L, bc):
+    """Every rank carves the same workspace layout (the loopback group and the peer transport address
+    other ranks' objects at their own offsets), also when a non-periodic bc drops the runs across
+    domain faces, which differ from rank to rank."""
+    world = pg[0] * pg[1] * pg[2]
+    for vc in (0, 1):
+        p = mg.params(n_local, pg, num_levels=L, bc=bc, var_coef=vc)
+        sizes = {mg.mg_workspace_bytes(p, r, world) for r in range(world)}
+        assert len(sizes) == 1, sizes
