@@ -62,8 +62,8 @@ typedef enum {
 } mg_status;
 
 #define MG_MAX_LEVELS 16
-#define MG_BRICK 8          /* brick edge: 8^3 bricks */
-#define MG_MAX_PERIOD 8     /* ghost depth in cells = brick edge */
+#define MG_BRICK 8          /* default brick edge: 8^3 bricks; params brick_edge = 4 selects 4^3 */
+#define MG_MAX_PERIOD 8     /* ghost depth in cells = brick edge; 4 with 4^3 bricks */
 
 /* fusion[l] variants.  Every variant produces bit-identical results. */
 enum {
@@ -152,7 +152,10 @@ typedef struct {
                                     the cell coefficients are set with mg_set_coefficients before the first
                                     V-cycle; the one-brick kernels run every level; smoother 0 and
                                     bottom_solver 0 only */
-  int32_t reserved[1];
+  int32_t brick_edge;            /* 0 or 8 = 8^3 bricks (the paper's NVIDIA / AMD choice); 4 = 4^3
+                                    bricks (the paper's Sunspot choice, variant N4): the one-brick kernel
+                                    family of generic.cu, per-sweep bottoms, ca_period <= 4, n_local a
+                                    multiple of 4*2^(num_levels-1) */
   double h0;                     /* finest spacing; <= 0 => 1 / max_d(global N_d) (reading A7) */
 } mg_params;
 

@@ -205,7 +205,7 @@ size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double**
   if (out) out->assign(lay.L, DevLevel());
   for (int l = 0; l < lay.L; ++l) {
     const LevelLayout& L = lay.lv[l];
-    const size_t fb = (size_t)L.n_alloc * kBV * sizeof(double);
+    const size_t fb = (size_t)L.n_alloc * lay.BV * sizeof(double);
     DevLevel d;
     d.x[0] = (double*)take(fb);
     d.x[1] = (double*)take(fb);
@@ -256,7 +256,7 @@ size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double**
   // ensure_stage: a device-only caller does not pay 2 level-0 fields for them)
   (void)stage;
   if (lay.repl) {  // replicated bottom
-    const size_t gfb = (size_t)lay.gb.n_alloc * kBV * sizeof(double);
+    const size_t gfb = (size_t)lay.gb.n_alloc * lay.BV * sizeof(double);
     const int64_t nown = lay.lv[(size_t)lay.L - 1].n_owned;
     mg_ctx::Repl r;
     r.x[0] = (double*)take(gfb);
@@ -264,7 +264,7 @@ size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double**
     r.b = (double*)take(gfb);
     r.adj = (int32_t*)take((size_t)lay.gb.n_stored * 8 * sizeof(int32_t));
     r.coord = (int32_t*)take((size_t)lay.gb.n_stored * 3 * sizeof(int32_t));
-    r.gbuf = (double*)take((size_t)lay.world * nown * kBV * sizeof(double));
+    r.gbuf = (double*)take((size_t)lay.world * nown * lay.BV * sizeof(double));
     r.gather = (CopyRun*)take((size_t)lay.gb.n_owned * sizeof(CopyRun));
     r.scatter = (CopyRun*)take((size_t)2 * nown * sizeof(CopyRun));
     if (rp) *rp = r;
@@ -294,7 +294,7 @@ mg_params normalized(const mg_params* p) {
     q.h0 = m > 0 ? 1.0 / (double)m : 1.0;
   }
   if (q.cheby_ratio <= 0) q.cheby_ratio = 6;
-  if (q.var_coef) {  // reading A23: the one-brick kernels carry the coefficient variant
+  if (q.var_coef || q.brick_edge == 4) {  // A23 / 4^3 bricks: the one-brick kernels carry the variant
     q.sweep_kernel = 1;
     q.temporal_blocking = 0;
     q.bottom_mode = MG_BOTTOM_SWEEPS;
@@ -313,6 +313,8 @@ mg_status check_params(const mg_params& p) {
   if (p.smoother < 0 || p.smoother > 2)
     return set_err(MG_ERR_INVALID_ARG, "smoother must be 0 (Jacobi), 1 (Chebyshev) or 2 (red-black Gauss-Seidel)");
   if (p.var_coef < 0 || p.var_coef > 1) return set_err(MG_ERR_INVALID_ARG, "var_coef must be 0 or 1");
+  if (p.brick_edge == 4 && p.bottom_solver != 0)
+    return set_err(MG_ERR_INVALID_ARG, "4^3 bricks: the CG bottom kernel holds 8^3 bricks (bottom_solver must be 0)");
   if (p.var_coef) {
     if (p.smoother != 0 || p.bottom_solver != 0)
       return set_err(MG_ERR_INVALID_ARG, "var_coef needs smoother 0 and bottom_solver 0 (reading A23)");
@@ -337,7 +339,7 @@ mg_status ensure_ax(mg_ctx* c, int l) {
   DevLevel& d = c->dl[l];
   if (d.Ax) return MG_OK;
   void* p = nullptr;
-  CKC(c, cudaMalloc(&p, (size_t)c->lay.lv[l].n_alloc * kBV * sizeof(double)));
+  CKC(c, cudaMalloc(&p, (size_t)c->lay.lv[l].n_alloc * c->lay.BV * sizeof(double)));
   c->allocs.push_back(p);
   d.Ax = (double*)p;
   return MG_OK;
@@ -347,7 +349,7 @@ mg_status ensure_stage(mg_ctx* c) {
   if (c->stage[0]) return MG_OK;
   for (int k = 0; k < 2; ++k) {
     void* p = nullptr;
-    CKC(c, cudaMalloc(&p, (size_t)c->lay.lv[0].n_owned * kBV * sizeof(double)));
+    CKC(c, cudaMalloc(&p, (size_t)c->lay.lv[0].n_owned * c->lay.BV * sizeof(double)));
     c->allocs.push_back(p);
     c->stage[k] = (double*)p;
   }
@@ -376,7 +378,7 @@ double* field_ptr(mg_ctx* c, int l, int field, int xbuf) {
 mg_status do_exchange(mg_ctx* c, int l, int field, int xbuf, cudaStream_t s) {
   const LevelLayout& L = c->lay.lv[l];
   double* f = field_ptr(c, l, field, xbuf);
-  const size_t bb = (size_t)kBV;
+  const size_t bb = (size_t)c->lay.BV;
   if (c->use_peer) {
     if (!c->peer_ready) return set_err(MG_ERR_STATE, "peer transport: call mg_peer_connect first");
     const DevLevel& d = c->dl[l];
@@ -399,7 +401,7 @@ mg_status do_exchange(mg_ctx* c, int l, int field, int xbuf, cudaStream_t s) {
   // bricks, so after the receives on the same stream
   const DevLevel& d = c->dl[l];
   // (the coefficients are reflected evenly whatever the bc: the face coefficient at a domain face is c_p)
-  if (d.nmirror > 0) CKC(c, launch_mirror(f, d.mirror, d.nmirror, field == 2 ? 1.0 : d.mirror_sign, s));
+  if (d.nmirror > 0) CKC(c, launch_mirror(f, d.mirror, d.nmirror, field == 2 ? 1.0 : d.mirror_sign, s, c->lay.E));
   return MG_OK;
 }
 
@@ -411,7 +413,7 @@ mg_status fill_repl_tables(mg_ctx* c) {
   if (!lay.repl) return MG_OK;
   const int lb = lay.L - 1;
   const int64_t nown = lay.lv[(size_t)lb].n_owned;
-  const size_t bb = (size_t)kBV;
+  const size_t bb = (size_t)c->lay.BV;
   c->rp.allgather = c->use_nccl;  // (a one-rank NCCL run too: the self-exchange tests cover the path)
   std::vector<CopyRun> g((size_t)lay.gb.n_owned), sc((size_t)2 * nown);
   for (int64_t q = 0; q < lay.gb.n_owned; ++q) {
@@ -442,7 +444,7 @@ mg_status fill_repl_tables(mg_ctx* c) {
 // Copy descriptors of the local transport: receiver ghost run <- sender surface run, for the
 // three exchanged fields (x[0], x[1], b).  Needs every rank's workspace carved (loopback groups).
 mg_status fill_copy_tables(mg_ctx* c) {
-  const size_t bb = (size_t)kBV;
+  const size_t bb = (size_t)c->lay.BV;
   for (int l = 0; l < c->lay.L; ++l) {
     const LevelLayout& L = c->lay.lv[l];
     DevLevel& d = c->dl[l];
@@ -470,15 +472,20 @@ mg_status fill_copy_tables(mg_ctx* c) {
 
 // ------------------------------------------------------------- executor
 // part: for OP_SWEEP2, which units of the range's pencil plan (LevelLayout::PairTable::part)
-mg_status sweep_range(mg_ctx* c, const Op& o, int64_t b0, int64_t b1, cudaStream_t s, int part = 0) {
+// paper_stage (the paper's kernel set, in-place smooth): 0 = applyOp then smooth, 1 = applyOp only,
+// 2 = smooth only -- a split sweep must finish every applyOp before the first in-place smooth
+mg_status sweep_range(mg_ctx* c, const Op& o, int64_t b0, int64_t b1, cudaStream_t s, int part = 0,
+                      int paper_stage = 0) {
   if (b1 <= b0) return MG_OK;
   DevLevel& d = c->dl[o.level];
   const int l = o.level;
   Coeffs cc = d.c;  // the smoother's step for this sweep (Chebyshev variant) or the level's Jacobi step
   if (o.g1 > 0) cc.gamma = o.g1;
   if (o.paper) {
-    CKC(c, launch_apply_op(d.x[o.src], d.Ax, d.adj, b0, b1 - b0, cc, s));
-    CKC(c, launch_smooth(d.x[o.src], d.Ax, d.b, d.r, b0, b1 - b0, cc, (o.flags & SW_WRITE_R) != 0, s, o.c1));
+    if (paper_stage != 2) CKC(c, launch_apply_op(d.x[o.src], d.Ax, d.adj, b0, b1 - b0, cc, s, c->lay.E));
+    if (paper_stage != 1)
+      CKC(c, launch_smooth(d.x[o.src], d.Ax, d.b, d.r, b0, b1 - b0, cc, (o.flags & SW_WRITE_R) != 0, s, o.c1,
+                           c->lay.E));
     return MG_OK;
   }
   SweepArgs a{};
@@ -498,6 +505,7 @@ mg_status sweep_range(mg_ctx* c, const Op& o, int64_t b0, int64_t b1, cudaStream
   a.gamma2 = o.g2 > 0 ? o.g2 : d.c.gamma;
   a.colour = o.c1;
   a.colour2 = o.c2;
+  a.E = c->lay.E;
   unsigned fl = o.flags;
   if (d.cf) {  // variable coefficients (reading A23): the one-brick kernel only (normalized() forces it)
     a.cf = d.cf;
@@ -580,9 +588,16 @@ mg_status exec_op(mg_ctx* c, const Op& o, cudaStream_t s) {
           CKC(c, cudaStreamWaitEvent(c->comm, c->ev_fork, 0));
           CKS(do_exchange(c, o.level, 0, o.src, c->comm));
           CKC(c, cudaEventRecord(c->ev_join, c->comm));
-          CKS(sweep_range(c, o, 0, L.n_interior, s));
-          CKC(c, cudaStreamWaitEvent(s, c->ev_join, 0));
-          CKS(sweep_range(c, o, L.n_interior, end, s));
+          if (o.paper) {  // in-place smooth: the surface bricks' applyOp must read the interior's old x
+            CKS(sweep_range(c, o, 0, L.n_interior, s, 0, 1));
+            CKC(c, cudaStreamWaitEvent(s, c->ev_join, 0));
+            CKS(sweep_range(c, o, L.n_interior, end, s, 0, 1));
+            CKS(sweep_range(c, o, 0, end, s, 0, 2));
+          } else {
+            CKS(sweep_range(c, o, 0, L.n_interior, s));
+            CKC(c, cudaStreamWaitEvent(s, c->ev_join, 0));
+            CKS(sweep_range(c, o, L.n_interior, end, s));
+          }
           CKS(timer_end(c, s, t0, o.level, o.timer));
           return MG_OK;
         }
@@ -597,17 +612,17 @@ mg_status exec_op(mg_ctx* c, const Op& o, cudaStream_t s) {
     }
     case OP_RESTRICT:
       CKS(timer_begin(c, s, &t0));
-      CKC(c, launch_restrict(d.r, c->dl[o.level + 1].b, d.parent, L.n_owned, s));
+      CKC(c, launch_restrict(d.r, c->dl[o.level + 1].b, d.parent, L.n_owned, s, c->lay.E));
       CKS(timer_end(c, s, t0, o.level, o.timer));
       return MG_OK;
     case OP_INTERP:
       CKS(timer_begin(c, s, &t0));
-      CKC(c, launch_interp(d.x[o.src], c->dl[o.level + 1].x[o.cbuf], d.parent, L.n_owned, s));
+      CKC(c, launch_interp(d.x[o.src], c->dl[o.level + 1].x[o.cbuf], d.parent, L.n_owned, s, c->lay.E));
       CKS(timer_end(c, s, t0, o.level, o.timer));
       return MG_OK;
     case OP_ZERO:
       CKS(timer_begin(c, s, &t0));
-      CKC(c, launch_zero(d.x[o.src], 0, L.n_stored, s));
+      CKC(c, launch_zero(d.x[o.src], 0, L.n_stored, s, c->lay.E));
       CKS(timer_end(c, s, t0, o.level, o.timer));
       return MG_OK;
     case OP_EXCH:
@@ -661,11 +676,11 @@ mg_status exec_op(mg_ctx* c, const Op& o, cudaStream_t s) {
       const int64_t ng = lay.gb.n_owned;
       CKS(timer_begin(c, s, &t0));
       if (c->rp.allgather)
-        CKN(c, ncclAllGather(d.b, c->rp.gbuf, (size_t)L.n_owned * kBV, ncclFloat64, c->nccl, s));
+        CKN(c, ncclAllGather(d.b, c->rp.gbuf, (size_t)L.n_owned * c->lay.BV, ncclFloat64, c->nccl, s));
       if (c->use_peer)
-        CKC(c, launch_peer_copy(c->rp.gather, (int)ng, kBV, c->ps_all, s));
+        CKC(c, launch_peer_copy(c->rp.gather, (int)ng, c->lay.BV, c->ps_all, s));
       else
-        CKC(c, launch_copy_runs(c->rp.gather, (int)ng, kBV, s));
+        CKC(c, launch_copy_runs(c->rp.gather, (int)ng, c->lay.BV, s));
       if (lay.p.bottom_solver == 1) {
         CKC(c, launch_bottom_cg(c->rp.x[1], c->rp.b, c->rp.adj, c->rp.coord, (int)ng, lay.gb.n[0], lay.gb.n[1], o.n,
                                 d.c, s));
@@ -681,7 +696,7 @@ mg_status exec_op(mg_ctx* c, const Op& o, cudaStream_t s) {
         a.bottom = o.n;
         CKC(c, launch_coarse(a, s));
       }
-      CKC(c, launch_copy_runs(c->rp.scatter + (size_t)o.dst * L.n_owned, (int)L.n_owned, kBV, s));
+      CKC(c, launch_copy_runs(c->rp.scatter + (size_t)o.dst * L.n_owned, (int)L.n_owned, c->lay.BV, s));
       CKS(timer_end(c, s, t0, o.level, o.timer));
       return MG_OK;
     }
@@ -922,7 +937,7 @@ mg_status set_level_field(mg_ctx* c, int l, int field, const double* src, bool e
   DevLevel& d = c->dl[l];
   const LevelLayout& L = c->lay.lv[l];
   double* dst = field == MG_FIELD_X ? d.x[c->st[l].cur] : field == MG_FIELD_B ? d.b : d.r;
-  CKC(c, launch_lex_to_brick(src, dst, d.coord, L.n_owned, L.n[0], L.n[1], c->stream));
+  CKC(c, launch_lex_to_brick(src, dst, d.coord, L.n_owned, L.n[0], L.n[1], c->stream, c->lay.E));
   if (field == MG_FIELD_X) {
     c->st[l].dx = 0;
     c->st[l].since = 1 << 20;
@@ -931,7 +946,7 @@ mg_status set_level_field(mg_ctx* c, int l, int field, const double* src, bool e
     c->st[l].db = 0;
     if (exchange_b && L.n_ghost > 0) {
       CKS(do_exchange(c, l, 1, 0, c->stream));
-      c->st[l].db = MG_MAX_PERIOD;
+      c->st[l].db = c->lay.E;
     }
   }
   return MG_OK;
@@ -1070,7 +1085,7 @@ mg_status mg_set_rhs_host(mg_ctx* c, const double* b_host) {
   CKS(check_ctx(c));
   if (!b_host) return set_err(MG_ERR_INVALID_ARG, "null b");
   CKS(ensure_stage(c));
-  const size_t bytes = (size_t)c->lay.lv[0].n_owned * kBV * sizeof(double);
+  const size_t bytes = (size_t)c->lay.lv[0].n_owned * c->lay.BV * sizeof(double);
   // Upload on the copy stream into staging field k (free once its previous conversion ran), so
   // the transfer overlaps whatever the caller's stream is still executing (the V-cycle of the
   // previous right-hand side); the conversion into bricks is ordered on the caller's stream.
@@ -1093,9 +1108,9 @@ static mg_status set_coefficients_impl(mg_ctx* c, const double* c_dev, cudaStrea
   if (!c->lay.p.var_coef) return set_err(MG_ERR_STATE, "var_coef is 0: this context has the paper's constant operator");
   if (!c_dev || ((uintptr_t)c_dev & 15)) return set_err(MG_ERR_INVALID_ARG, "c must be a 16-byte aligned device pointer");
   const LevelLayout& L0 = c->lay.lv[0];
-  CKC(c, launch_lex_to_brick(c_dev, c->dl[0].cf, c->dl[0].coord, L0.n_owned, L0.n[0], L0.n[1], s));
+  CKC(c, launch_lex_to_brick(c_dev, c->dl[0].cf, c->dl[0].coord, L0.n_owned, L0.n[0], L0.n[1], s, c->lay.E));
   for (int l = 0; l + 1 < c->lay.L; ++l)
-    CKC(c, launch_restrict(c->dl[l].cf, c->dl[l + 1].cf, c->dl[l].parent, c->lay.lv[l].n_owned, s));
+    CKC(c, launch_restrict(c->dl[l].cf, c->dl[l + 1].cf, c->dl[l].parent, c->lay.lv[l].n_owned, s, c->lay.E));
   return MG_OK;
 }
 
@@ -1117,7 +1132,7 @@ mg_status mg_set_solution(mg_ctx* c, const double* x_dev) {
   CKS(check_ctx(c));
   if (!x_dev) {
     const LevelLayout& L = c->lay.lv[0];
-    CKC(c, cudaMemsetAsync(c->dl[0].x[c->st[0].cur], 0, (size_t)L.n_stored * kBV * sizeof(double), c->stream));
+    CKC(c, cudaMemsetAsync(c->dl[0].x[c->st[0].cur], 0, (size_t)L.n_stored * c->lay.BV * sizeof(double), c->stream));
     c->st[0].dx = 0;
     return MG_OK;
   }
@@ -1128,7 +1143,7 @@ mg_status mg_get_solution(mg_ctx* c, double* x_dev) {
   CKS(check_ctx(c));
   if (!x_dev || ((uintptr_t)x_dev & 15)) return set_err(MG_ERR_INVALID_ARG, "x must be a 16-byte aligned pointer");
   const LevelLayout& L = c->lay.lv[0];
-  CKC(c, launch_brick_to_lex(c->dl[0].x[c->st[0].cur], x_dev, c->dl[0].coord, L.n_owned, L.n[0], L.n[1], c->stream));
+  CKC(c, launch_brick_to_lex(c->dl[0].x[c->st[0].cur], x_dev, c->dl[0].coord, L.n_owned, L.n[0], L.n[1], c->stream, c->lay.E));
   return MG_OK;
 }
 
@@ -1138,7 +1153,7 @@ mg_status mg_get_solution_host(mg_ctx* c, double* x_host) {
   CKS(ensure_stage(c));
   const int k = c->stage_k;  // every upload into it is already ordered before its conversion
   CKS(mg_get_solution(c, c->stage[k]));
-  const size_t bytes = (size_t)c->lay.lv[0].n_owned * kBV * sizeof(double);
+  const size_t bytes = (size_t)c->lay.lv[0].n_owned * c->lay.BV * sizeof(double);
   CKC(c, cudaMemcpyAsync(x_host, c->stage[k], bytes, cudaMemcpyDeviceToHost, c->stream));
   CKC(c, cudaEventRecord(c->ev_free[k], c->stream));
   CKC(c, cudaStreamSynchronize(c->stream));
@@ -1161,11 +1176,11 @@ mg_status mg_residual_norm_async(mg_ctx* c) {
   DevLevel& d = c->dl[0];
   if (L.n_ghost > 0) {
     CKS(do_exchange(c, 0, 0, c->st[0].cur, c->stream));
-    c->st[0].dx = MG_MAX_PERIOD;
+    c->st[0].dx = c->lay.E;
     c->st[0].since = 0;
   }
   CKC(c, cudaMemsetAsync(c->acc, 0, sizeof(unsigned long long), c->stream));
-  CKC(c, launch_norm(d.x[c->st[0].cur], d.b, d.adj, L.n_owned, d.c, c->acc, c->stream, d.cf));
+  CKC(c, launch_norm(d.x[c->st[0].cur], d.b, d.adj, L.n_owned, d.c, c->acc, c->stream, d.cf, c->lay.E));
   if (c->use_nccl && c->lay.world > 1)
     CKN(c, ncclAllReduce(c->acc, c->acc, 1, ncclUint64, ncclMax, c->nccl, c->stream));
   if (c->use_peer && c->lay.world > 1) {
@@ -1263,7 +1278,7 @@ mg_status mg_exchange_stats(mg_ctx* c, int64_t* bytes_per_cycle, int64_t* messag
     const bool ex = o.kind == OP_EXCH || ((o.kind == OP_SWEEP || o.kind == OP_SWEEP2) && o.exch_before);
     if (!ex) continue;
     for (const Run& r : c->lay.lv[o.level].sends) {
-      bytes += r.count * kBV * (int64_t)sizeof(double);
+      bytes += r.count * c->lay.BV * (int64_t)sizeof(double);
       ++msgs;
     }
   }
@@ -1281,7 +1296,7 @@ mg_status mg_exchange_plan(mg_ctx* c, int32_t cap, int64_t* exchanges, int64_t* 
   for (int l = 0; l < c->lay.L; ++l) {
     exchanges[l] = 0;
     bytes[l] = 0;
-    for (const Run& r : c->lay.lv[l].sends) bytes[l] += r.count * kBV * (int64_t)sizeof(double);
+    for (const Run& r : c->lay.lv[l].sends) bytes[l] += r.count * c->lay.BV * (int64_t)sizeof(double);
   }
   for (const Op& o : b.ops)
     if (o.kind == OP_EXCH || ((o.kind == OP_SWEEP || o.kind == OP_SWEEP2) && o.exch_before)) ++exchanges[o.level];
@@ -1446,7 +1461,7 @@ mg_status mg_level_get(mg_ctx* c, int32_t level, int32_t field, double* dst_dev)
   DevLevel& d = c->dl[level];
   const LevelLayout& L = c->lay.lv[level];
   const double* src = field == MG_FIELD_X ? d.x[c->st[level].cur] : field == MG_FIELD_B ? d.b : d.r;
-  CKC(c, launch_brick_to_lex(src, dst_dev, d.coord, L.n_owned, L.n[0], L.n[1], c->stream));
+  CKC(c, launch_brick_to_lex(src, dst_dev, d.coord, L.n_owned, L.n[0], L.n[1], c->stream, c->lay.E));
   return MG_OK;
 }
 
@@ -1590,7 +1605,7 @@ mg_status mg_group_commit_rhs(mg_group* g) {
   for (mg_ctx* c : g->r) {
     CKS(check_ctx(c));
     if (c->lay.lv[0].n_ghost > 0) CKS(do_exchange(c, 0, 1, 0, g->stream));
-    c->st[0].db = MG_MAX_PERIOD;
+    c->st[0].db = c->lay.E;
   }
   return MG_OK;
 }
@@ -1613,14 +1628,14 @@ mg_status mg_group_residual_norm(mg_group* g, double* out) {
     }
   }
   for (mg_ctx* c : g->r) {
-    c->st[0].dx = MG_MAX_PERIOD;
+    c->st[0].dx = c->lay.E;
     c->st[0].since = 0;
   }
   CKC(c0, cudaMemsetAsync(c0->acc, 0, sizeof(unsigned long long), g->stream));
   for (mg_ctx* c : g->r) {
     const LevelLayout& L = c->lay.lv[0];
     DevLevel& d = c->dl[0];
-    CKC(c0, launch_norm(d.x[c->st[0].cur], d.b, d.adj, L.n_owned, d.c, c0->acc, g->stream, d.cf));
+    CKC(c0, launch_norm(d.x[c->st[0].cur], d.b, d.adj, L.n_owned, d.c, c0->acc, g->stream, d.cf, c->lay.E));
   }
   CKC(c0, cudaMemcpyAsync(c0->h_pinned, c0->acc, 8, cudaMemcpyDeviceToHost, g->stream));
   CKC(c0, cudaStreamSynchronize(g->stream));

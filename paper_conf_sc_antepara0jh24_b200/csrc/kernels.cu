@@ -239,6 +239,7 @@ static cudaError_t launch_sweep_t(const SweepArgs& a, cudaStream_t s) {
 }
 
 cudaError_t launch_sweep(const SweepArgs& a, unsigned flags, cudaStream_t s) {
+  if (a.E != 8) return launch_gsweep(a, flags, 0, nullptr, s);
   if (flags & SW_VARCOEF) {
     switch (flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP | SW_ZERO_X)) {
 #define VC_CASE(F) \
@@ -490,7 +491,7 @@ cudaError_t encode_pair_maps(const double* x, const double* b, int64_t n_alloc, 
 }
 
 cudaError_t launch_apply_op(const double* x, double* Ax, const int32_t* adj, int64_t brick0, int64_t nbricks,
-                            Coeffs c, cudaStream_t s) {
+                            Coeffs c, cudaStream_t s, int E) {
   if (nbricks <= 0) return cudaSuccess;
   SweepArgs a{};
   a.x = x;
@@ -499,12 +500,14 @@ cudaError_t launch_apply_op(const double* x, double* Ax, const int32_t* adj, int
   a.brick0 = brick0;
   a.nbricks = nbricks;
   a.c = c;
+  a.E = E;
+  if (E != 8) return launch_gsweep(a, 0, 1, nullptr, s);
   launch_k(sweep_kernel<MODE_APPLY, 0>, (unsigned)nbricks, 256, 0, s, a, nullptr);
   return cudaGetLastError();
 }
 
 cudaError_t launch_norm(const double* x, const double* b, const int32_t* adj, int64_t nbricks, Coeffs c,
-                        unsigned long long* acc, cudaStream_t s, const double* cf) {
+                        unsigned long long* acc, cudaStream_t s, const double* cf, int E) {
   if (nbricks <= 0) return cudaSuccess;
   SweepArgs a{};
   a.x = x;
@@ -514,6 +517,8 @@ cudaError_t launch_norm(const double* x, const double* b, const int32_t* adj, in
   a.nbricks = nbricks;
   a.c = c;
   a.cf = cf;
+  a.E = E;
+  if (E != 8) return launch_gsweep(a, cf ? SW_VARCOEF : 0u, 2, acc, s);
   if (cf)
     launch_k(sweep_kernel<MODE_NORM, SW_VARCOEF>, (unsigned)nbricks, 256, 0, s, a, acc);
   else
@@ -554,8 +559,9 @@ static unsigned grid_for(int64_t n2) {
 }
 
 cudaError_t launch_smooth(double* x, const double* Ax, const double* b, double* r, int64_t brick0, int64_t nbricks,
-                          Coeffs c, bool write_r, cudaStream_t s, int colour) {
+                          Coeffs c, bool write_r, cudaStream_t s, int colour, int E) {
   if (nbricks <= 0) return cudaSuccess;
+  if (E != 8) return launch_gsmooth(x, Ax, b, r, brick0, nbricks, c, write_r, colour, E, s);
   const int64_t n2 = nbricks * 256;
   if (write_r)
     launch_k(smooth_kernel<true>, grid_for(n2), 256, 0, s, x, Ax, b, r, brick0 * 512, n2, c.gamma, colour);
@@ -590,8 +596,10 @@ __global__ void __launch_bounds__(128) restrict_kernel(const double* __restrict_
   }
 }
 
-cudaError_t launch_restrict(const double* r, double* bc, const int32_t* parent, int64_t nfine, cudaStream_t s) {
+cudaError_t launch_restrict(const double* r, double* bc, const int32_t* parent, int64_t nfine, cudaStream_t s,
+                            int E) {
   if (nfine <= 0) return cudaSuccess;
+  if (E != 8) return launch_grestrict(r, bc, parent, nfine, E, s);
   launch_k(restrict_kernel, (unsigned)nfine, 128, 0, s, r, bc, parent);
   return cudaGetLastError();
 }
@@ -640,8 +648,10 @@ __global__ void __launch_bounds__(256) interp4_kernel(double* __restrict__ x, co
   }
 }
 
-cudaError_t launch_interp(double* x, const double* xc, const int32_t* parent, int64_t nfine, cudaStream_t s) {
+cudaError_t launch_interp(double* x, const double* xc, const int32_t* parent, int64_t nfine, cudaStream_t s,
+                          int E) {
   if (nfine <= 0) return cudaSuccess;
+  if (E != 8) return launch_ginterp(x, xc, parent, nfine, E, s);
   static const bool one = getenv("MG_INTERP1") != nullptr;  // (measurement switch: one brick per CTA)
   if (one)
     launch_k(interp_kernel, (unsigned)nfine, 256, 0, s, x, xc, parent);
@@ -656,10 +666,10 @@ __global__ void __launch_bounds__(256) zero_kernel(double* __restrict__ x, int64
     reinterpret_cast<double2*>(x + base)[q] = make_double2(0.0, 0.0);
 }
 
-cudaError_t launch_zero(double* x, int64_t brick0, int64_t nbricks, cudaStream_t s) {
+cudaError_t launch_zero(double* x, int64_t brick0, int64_t nbricks, cudaStream_t s, int E) {
   if (nbricks <= 0) return cudaSuccess;
-  const int64_t n2 = nbricks * 256;
-  launch_k(zero_kernel, grid_for(n2), 256, 0, s, x, brick0 * 512, n2);
+  const int64_t bv = (int64_t)E * E * E, n2 = nbricks * bv / 2;
+  launch_k(zero_kernel, grid_for(n2), 256, 0, s, x, brick0 * bv, n2);
   return cudaGetLastError();
 }
 
@@ -712,15 +722,17 @@ __global__ void __launch_bounds__(256) brick_to_lex_kernel(const double* __restr
 }
 
 cudaError_t launch_lex_to_brick(const double* lex, double* bricks, const int32_t* coord, int64_t nowned, int nx,
-                                int ny, cudaStream_t s) {
+                                int ny, cudaStream_t s, int E) {
   if (nowned <= 0) return cudaSuccess;
+  if (E != 8) return launch_glex(lex, bricks, coord, nowned, nx, ny, 0, E, s);
   launch_k(lex_to_brick_kernel, (unsigned)nowned, 256, 0, s, lex, bricks, coord, nx, ny);
   return cudaGetLastError();
 }
 
 cudaError_t launch_brick_to_lex(const double* bricks, double* lex, const int32_t* coord, int64_t nowned, int nx,
-                                int ny, cudaStream_t s) {
+                                int ny, cudaStream_t s, int E) {
   if (nowned <= 0) return cudaSuccess;
+  if (E != 8) return launch_glex(bricks, lex, coord, nowned, nx, ny, 1, E, s);
   launch_k(brick_to_lex_kernel, (unsigned)nowned, 256, 0, s, bricks, lex, coord, nx, ny);
   return cudaGetLastError();
 }
@@ -745,8 +757,9 @@ __global__ void __launch_bounds__(256) mirror_kernel(double* __restrict__ f, con
   }
 }
 
-cudaError_t launch_mirror(double* f, const int32_t* table, int n, double sign, cudaStream_t s) {
+cudaError_t launch_mirror(double* f, const int32_t* table, int n, double sign, cudaStream_t s, int E) {
   if (n <= 0) return cudaSuccess;
+  if (E != 8) return launch_gmirror(f, table, n, sign, E, s);
   launch_k(mirror_kernel, (unsigned)n, 256, 0, s, f, table, sign);
   return cudaGetLastError();
 }

@@ -41,6 +41,7 @@ struct SweepArgs {
   int colour2 = -1;  // keep the others (r still on every cell); -1 = every cell.  colour2: second sweep
   const double* cf = nullptr;  // SW_VARCOEF: cell coefficients c (brick layout, ghosts valid)
   double vc_g = 0.0;           // SW_VARCOEF: 0.5 * h * h (gamma_p = vc_g / sum of the face coefficients)
+  int E = 8;                   // brick edge (8; 4: the generic kernels of generic.cu)
 };
 
 cudaError_t launch_sweep(const SweepArgs& a, unsigned flags, cudaStream_t s);
@@ -116,28 +117,30 @@ cudaError_t launch_sweep_col(const SweepArgs& a, const ColArgs& c, const FaceMap
                              cudaStream_t s);
 // applyOp (paper kernel set): Ax = alpha x + beta sum6
 cudaError_t launch_apply_op(const double* x, double* Ax, const int32_t* adj, int64_t brick0, int64_t nbricks,
-                            Coeffs c, cudaStream_t s);
+                            Coeffs c, cudaStream_t s, int E = 8);
 // smooth(+residual) pointwise (paper kernel set): x += gamma (Ax - b); r = b - Ax
 cudaError_t launch_smooth(double* x, const double* Ax, const double* b, double* r, int64_t brick0, int64_t nbricks,
-                          Coeffs c, bool write_r, cudaStream_t s, int colour = -1);
+                          Coeffs c, bool write_r, cudaStream_t s, int colour = -1, int E = 8);
 // restriction over fine bricks [0, nfine): bc[parent octant] = avg8(r)
-cudaError_t launch_restrict(const double* r, double* bc, const int32_t* parent, int64_t nfine, cudaStream_t s);
+cudaError_t launch_restrict(const double* r, double* bc, const int32_t* parent, int64_t nfine, cudaStream_t s,
+                            int E = 8);
 // interpolation+increment over fine bricks [0, nfine): x += xc(parent)
-cudaError_t launch_interp(double* x, const double* xc, const int32_t* parent, int64_t nfine, cudaStream_t s);
+cudaError_t launch_interp(double* x, const double* xc, const int32_t* parent, int64_t nfine, cudaStream_t s,
+                          int E = 8);
 // initZero over bricks [brick0, brick0+n)
-cudaError_t launch_zero(double* x, int64_t brick0, int64_t nbricks, cudaStream_t s);
+cudaError_t launch_zero(double* x, int64_t brick0, int64_t nbricks, cudaStream_t s, int E = 8);
 // max |b - Ax| over bricks [0, n) -> atomicMax on *acc (uint64 bits of a non-negative double)
 cudaError_t launch_norm(const double* x, const double* b, const int32_t* adj, int64_t nbricks, Coeffs c,
-                        unsigned long long* acc, cudaStream_t s, const double* cf = nullptr);
+                        unsigned long long* acc, cudaStream_t s, const double* cf = nullptr, int E = 8);
 // resident bottom solve: all `nbricks` (<= kResidentMaxBricks, no ghosts) in one CTA's shared memory
 constexpr int kResidentMaxBricks = 8;
 cudaError_t launch_bottom_resident(const double* x, double* xo, const double* b, const int32_t* adj, int nbricks,
                                    int sweeps, bool zero_x, Coeffs c, cudaStream_t s);
 // layout conversion (not part of the V-cycle): lexicographic local <-> bricks [0, nowned)
 cudaError_t launch_lex_to_brick(const double* lex, double* bricks, const int32_t* coord, int64_t nowned, int nx,
-                                int ny, cudaStream_t s);
+                                int ny, cudaStream_t s, int E = 8);
 cudaError_t launch_brick_to_lex(const double* bricks, double* lex, const int32_t* coord, int64_t nowned, int nx,
-                                int ny, cudaStream_t s);
+                                int ny, cudaStream_t s, int E = 8);
 // Local (self / loopback) ghost exchange: every run of one exchange in ONE launch instead of one
 // cudaMemcpyAsync per run (n doubles from src to dst, both 16-byte aligned, n even).
 struct CopyRun {
@@ -149,7 +152,17 @@ cudaError_t launch_copy_runs(const CopyRun* runs, int nruns, int64_t max_n, cuda
 // Mirror exchange (non-periodic bc, reading A22): for each entry (dst, src, mask) of the
 // int32[n][3] table, brick dst = sign^popcount(mask) x brick src with the cells reversed on the axes
 // of mask (bit a: axis a).  sign = -1 (Dirichlet) or +1 (Neumann).
-cudaError_t launch_mirror(double* f, const int32_t* table, int n, double sign, cudaStream_t s);
+cudaError_t launch_mirror(double* f, const int32_t* table, int n, double sign, cudaStream_t s, int E = 8);
+// generic.cu: the same operations for a brick edge E != 8 (E = 4; "4x4x4 on Sunspot").
+// mode 0 sweep (flags), 1 applyOp (x -> xo), 2 norm (atomicMax on *acc)
+cudaError_t launch_gsweep(const SweepArgs& a, unsigned flags, int mode, unsigned long long* acc, cudaStream_t s);
+cudaError_t launch_grestrict(const double* r, double* bc, const int32_t* parent, int64_t nfine, int E, cudaStream_t s);
+cudaError_t launch_ginterp(double* x, const double* xc, const int32_t* parent, int64_t nfine, int E, cudaStream_t s);
+cudaError_t launch_glex(const double* src, double* dst, const int32_t* coord, int64_t nowned, int nx, int ny,
+                        int dir, int E, cudaStream_t s);
+cudaError_t launch_gmirror(double* f, const int32_t* table, int n, double sign, int E, cudaStream_t s);
+cudaError_t launch_gsmooth(double* x, const double* Ax, const double* b, double* r, int64_t brick0, int64_t nbricks,
+                           Coeffs c, bool write_r, int colour, int E, cudaStream_t s);
 // Exchange between processes over peer memory (peer.cu): the copy runs read other ranks' fields
 // through CUDA IPC mappings; device-side flags order them (ready / done per epoch, see peer.cu).
 constexpr int kPeerSlotU64 = 16;  // one flag per 128-byte slot

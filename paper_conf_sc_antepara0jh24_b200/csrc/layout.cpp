@@ -78,7 +78,7 @@ static void build_level(const Layout& lay, int l, LevelLayout& L) {
   const mg_params& p = lay.p;
   for (int a = 0; a < 3; ++a) {
     L.n[a] = p.n_local[a] >> l;
-    L.nb[a] = L.n[a] / kB;
+    L.nb[a] = L.n[a] / lay.E;
     // a one-brick ghost shell on decomposed axes, on every axis in MG_GHOST_ALL, and on every axis
     // with a non-periodic boundary (its domain-face ghosts hold the reflected values, reading A22)
     L.g[a] = (p.ghost_mode == MG_GHOST_ALL || p.proc_grid[a] > 1 || p.bc != MG_BC_PERIODIC) ? 1 : 0;
@@ -264,11 +264,18 @@ mg_status build_layout(const mg_params& p, int rank, int world, Layout& out, std
     msg = "num_levels must be in [1, 16]";
     return MG_ERR_INVALID_ARG;
   }
-  const int64_t unit = (int64_t)kB << (p.num_levels - 1);
+  if (p.brick_edge != 0 && p.brick_edge != 4 && p.brick_edge != 8) {
+    msg = "brick_edge must be 0 / 8 (8^3 bricks) or 4 (4^3 bricks)";
+    return MG_ERR_INVALID_ARG;
+  }
+  const int E = p.brick_edge == 4 ? 4 : kB;
+  out.E = E;
+  out.BV = (int64_t)E * E * E;
+  const int64_t unit = (int64_t)E << (p.num_levels - 1);
   for (int a = 0; a < 3; ++a) {
     if (p.n_local[a] <= 0 || p.n_local[a] % unit != 0) {
-      snprintf(buf, sizeof buf, "n_local[%d]=%d must be a positive multiple of 8*2^(num_levels-1)=%lld", a,
-               p.n_local[a], (long long)unit);
+      snprintf(buf, sizeof buf, "n_local[%d]=%d must be a positive multiple of %d*2^(num_levels-1)=%lld", a,
+               p.n_local[a], E, (long long)unit);
       msg = buf;
       return MG_ERR_INVALID_ARG;
     }
@@ -278,8 +285,8 @@ mg_status build_layout(const mg_params& p, int rank, int world, Layout& out, std
     return MG_ERR_INVALID_ARG;
   }
   for (int l = 0; l < MG_MAX_LEVELS; ++l) {
-    if (p.ca_period[l] < 0 || p.ca_period[l] > MG_MAX_PERIOD) {
-      msg = "ca_period must be in [0, 8] (ghost depth = brick edge, P:L156)";
+    if (p.ca_period[l] < 0 || p.ca_period[l] > E) {
+      msg = "ca_period must be in [0, brick edge] (ghost depth = brick edge, P:L156)";
       return MG_ERR_INVALID_ARG;
     }
     if (p.fusion[l] < 0 || p.fusion[l] > MG_FUSION_FULL) {
@@ -322,6 +329,8 @@ mg_status build_layout(const mg_params& p, int rank, int world, Layout& out, std
       p.bc == MG_BC_PERIODIC) {
     Layout g;
     g.p = p;
+    g.E = out.E;
+    g.BV = out.BV;
     for (int a = 0; a < 3; ++a) {
       g.p.n_local[a] = p.n_local[a] * p.proc_grid[a];
       g.p.proc_grid[a] = 1;

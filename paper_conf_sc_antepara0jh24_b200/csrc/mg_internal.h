@@ -140,6 +140,8 @@ constexpr int64_t kReplMaxBricks = 64;  // global coarsest bricks (the cluster s
 
 struct Layout {
   mg_params p{};
+  int E = kB;     // brick edge (params brick_edge: 8, or 4 for the generic kernels)
+  int64_t BV = kBV;  // doubles per brick
   int rank = 0, world = 1;
   int coords[3] = {0, 0, 0};
   int L = 0;

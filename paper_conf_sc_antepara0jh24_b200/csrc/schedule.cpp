@@ -29,7 +29,7 @@ int Builder::period(int l) const {
   // processes an exchange crosses NVLink (~6x the bytes-time of a local copy, plus flag latency) and
   // the brick-deep ghost zone's period 8 stays the default
   const bool local = lay.world == 1 ? lay.p.transport != MG_TRANSPORT_NCCL : lay.p.transport == MG_TRANSPORT_LOCAL;
-  return (l == 0 && local) ? 2 : MG_MAX_PERIOD;
+  return (l == 0 && local) ? std::min(2, lay.E) : lay.E;
 }
 
 bool Builder::has_pair_table(int l, int64_t b0, int64_t b1) const {
@@ -113,7 +113,7 @@ void Builder::phase(int l, int n, bool zero_first, int last, bool interp_first, 
       o.zero = zero_first && s == 0;  // the first sweep reads x0 == 0 (SW_ZERO_X)
       const bool ex = g && !o.zero && (S.dx < 2 || S.since + 2 > k);
       if (ex) {
-        S.dx = MG_MAX_PERIOD;
+        S.dx = lay.E;
         S.since = 0;
       }
       o.exch_before = ex;
@@ -146,7 +146,7 @@ void Builder::phase(int l, int n, bool zero_first, int last, bool interp_first, 
     const bool zero = zero_first && s == 0;
     const bool ex = g && !zero && (S.dx < 1 || S.since >= k);
     if (ex) {
-      S.dx = MG_MAX_PERIOD;
+      S.dx = lay.E;
       S.since = 0;
     }
     o.exch_before = ex;
@@ -178,7 +178,7 @@ void Builder::exchange_b(int l) {
   o.field = 1;
   o.timer = MG_OP_EXCHANGE;
   ops.push_back(o);
-  st[l].db = MG_MAX_PERIOD;
+  st[l].db = lay.E;
 }
 
 void Builder::restrict_op(int l) {
@@ -197,7 +197,7 @@ void Builder::zero_op(int l) {
   o.src = o.dst = st[l].cur;
   o.timer = MG_OP_ZERO;
   ops.push_back(o);
-  st[l].dx = MG_MAX_PERIOD;  // zero is the true value of every ghost too
+  st[l].dx = lay.E;  // zero is the true value of every ghost too
   st[l].since = 0;
 }
 
@@ -335,7 +335,7 @@ void Builder::vcycle() {
     if (!fold)  // initZero as its own kernel (Alg 2 step 8)
       zero_op(l + 1);
     else {
-      st[l + 1].dx = MG_MAX_PERIOD;  // folded into the first coarse sweep
+      st[l + 1].dx = lay.E;  // folded into the first coarse sweep
       st[l + 1].since = 0;
     }
   }
@@ -365,13 +365,14 @@ void Builder::vcycle() {
 
 int64_t op_launches(const Op& o, const Layout& lay, bool overlap, bool pencil_overlap, bool local_exchange) {
   // kernels of this library one op launches (NCCL's own kernels not counted); an exchange over the
-  // local transport is one copy kernel (copy_runs_kernel), over NCCL none of ours
-  const int64_t ex = local_exchange ? 1 : 0;
+  // local (or peer) transport is one copy kernel (copy_runs_kernel) when the level has receives, over
+  // NCCL none of ours, plus the mirror kernel of a non-periodic bc
+  const LevelLayout& L = lay.lv[o.level];
+  const int64_t ex = (local_exchange && !L.recvs.empty() ? 1 : 0) + (L.mirror.empty() ? 0 : 1);
   switch (o.kind) {
     case OP_SWEEP:
     case OP_SWEEP2: {
       const int per = o.paper ? 2 : 1;  // applyOp + smooth(+residual)
-      const LevelLayout& L = lay.lv[o.level];
       const int64_t end = o.ghosts ? L.n_stored : L.n_owned;
       const int64_t x = o.exch_before ? ex : 0;
       bool pen_split = false;
@@ -379,7 +380,7 @@ int64_t op_launches(const Op& o, const Layout& lay, bool overlap, bool pencil_ov
         for (const auto& pt : L.pairs) pen_split |= pt.b0 == 0 && pt.b1 == end && pt.part == 1;
       if (pen_split) return 2 + x;
       const bool split = o.exch_before && overlap && lay.lv[o.level].n_interior > 0 && !o.nosplit;
-      return per * (split ? 2 : 1) + x;
+      return (split ? (o.paper ? 3 : 2) : per) + x;  // a split paper sweep: 2 applyOps, one smooth
     }
     case OP_RESTRICT:  // restrict_kernel
     case OP_INTERP:    // interp4_kernel / interp_kernel

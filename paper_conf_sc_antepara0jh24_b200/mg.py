@@ -55,7 +55,7 @@ class mg_params(ctypes.Structure):
         ("bottom_solver", ctypes.c_int32),
         ("bc", ctypes.c_int32),
         ("var_coef", ctypes.c_int32),
-        ("reserved", ctypes.c_int32 * 1),
+        ("brick_edge", ctypes.c_int32),
         ("h0", ctypes.c_double),
     ]
 
@@ -169,7 +169,7 @@ def check(status: int, where: str) -> int:
 def params(n_local, proc_grid=(1, 1, 1), num_levels=6, pre=12, post=12, bottom=100, ca_period=None, fusion=None,
            ghost_mode=MG_GHOST_AUTO, transport=MG_TRANSPORT_AUTO, use_graph=1, bottom_mode=MG_BOTTOM_AUTO,
            overlap=1, h0=0.0, sweep_kernel=0, temporal_blocking=3, smoother=0, cheby_ratio=0, launch_pdl=0, bottom_solver=0,
-           bc=0, var_coef=0) -> mg_params:
+           bc=0, var_coef=0, brick_edge=0) -> mg_params:
     p = mg_params()
     lib().mg_params_default(ctypes.byref(p))
     p.n_local[:] = [int(v) for v in n_local]
@@ -188,6 +188,7 @@ def params(n_local, proc_grid=(1, 1, 1), num_levels=6, pre=12, post=12, bottom=1
     p.launch_pdl = int(launch_pdl)
     p.bottom_solver = int(bottom_solver)
     p.bc, p.var_coef = int(bc), int(var_coef)
+    p.brick_edge = int(brick_edge)
     return p
 
 

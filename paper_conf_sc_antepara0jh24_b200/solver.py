@@ -25,7 +25,7 @@ class Multigrid:
                  fusion=None, ghost_mode=mg.MG_GHOST_AUTO, transport=mg.MG_TRANSPORT_AUTO, use_graph=True,
                  bottom_mode=mg.MG_BOTTOM_AUTO, overlap=True, h0=0.0, rank=0, world_size=1, device=None,
                  stream: torch.cuda.Stream | None = None, sweep_kernel=0, temporal_blocking=3, smoother=0,
-                 cheby_ratio=0, launch_pdl=0, bottom_solver=0, bc=0, var_coef=0):
+                 cheby_ratio=0, launch_pdl=0, bottom_solver=0, bc=0, var_coef=0, brick_edge=0):
         if not torch.cuda.is_available():
             raise RuntimeError("Multigrid needs a CUDA device (the library has no CPU fallback)")
         self.device = torch.device("cuda", torch.cuda.current_device() if device is None else int(device))
@@ -35,7 +35,8 @@ class Multigrid:
         self.rank, self.world_size = int(rank), int(world_size)
         self.p = mg.params(self.n_local, proc_grid, num_levels, pre, post, bottom, ca_period, fusion, ghost_mode,
                            transport, 1 if use_graph else 0, bottom_mode, 1 if overlap else 0, h0, sweep_kernel,
-                           temporal_blocking, smoother, cheby_ratio, launch_pdl, bottom_solver, bc, var_coef)
+                           temporal_blocking, smoother, cheby_ratio, launch_pdl, bottom_solver, bc, var_coef,
+                           brick_edge)
         self.ws_bytes = mg.mg_workspace_bytes(self.p, self.rank, self.world_size)
         self.ws = torch.empty(self.ws_bytes + 256, dtype=torch.uint8, device=self.device)
         base = _ptr(self.ws)
@@ -191,7 +192,7 @@ class LoopbackGroup:
     def __init__(self, n_local, proc_grid, num_levels=6, pre=12, post=12, bottom=100, ca_period=None, fusion=None,
                  ghost_mode=mg.MG_GHOST_AUTO, use_graph=True, bottom_mode=mg.MG_BOTTOM_AUTO, overlap=True, h0=0.0,
                  device=None, sweep_kernel=0, temporal_blocking=3, smoother=0, cheby_ratio=0, launch_pdl=0, bottom_solver=0,
-                 bc=0, var_coef=0):
+                 bc=0, var_coef=0, brick_edge=0):
         self.device = torch.device("cuda", torch.cuda.current_device() if device is None else int(device))
         torch.cuda.set_device(self.device)
         self.n_local = tuple(int(v) for v in n_local)
@@ -200,7 +201,7 @@ class LoopbackGroup:
         self.p = mg.params(self.n_local, proc_grid, num_levels, pre, post, bottom, ca_period, fusion, ghost_mode,
                            mg.MG_TRANSPORT_LOCAL, 1 if use_graph else 0, bottom_mode, 1 if overlap else 0, h0,
                            sweep_kernel, temporal_blocking, smoother, cheby_ratio, launch_pdl, bottom_solver, bc,
-                           var_coef)
+                           var_coef, brick_edge)
         per = (mg.mg_workspace_bytes(self.p, 0, self.world_size) + 255) & ~255
         self.ws = torch.empty(per * self.world_size + 256, dtype=torch.uint8, device=self.device)
         self.ws_ptr = (_ptr(self.ws) + 255) & ~255

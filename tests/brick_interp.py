@@ -27,18 +27,21 @@ class RankLevel:
         self.n_owned = self.info["owned"]
         self.n_alloc = self.info["alloc"]
         self.n = self.info["n"]  # x, y, z
+        self.E = self.n[0] // self.info["nb"][0]  # brick edge (8, or 4)
         self.mirror = lay.mirror(level)  # non-periodic bc (reading A22): (ghost, source, reflected axes)
         self.mirror_sign = -1.0 if lay.p.bc == 1 else 1.0
 
     def zeros(self):
-        return np.zeros((self.n_alloc, 8, 8, 8))  # [brick][k][j][i]
+        E = self.E
+        return np.zeros((self.n_alloc, E, E, E))  # [brick][k][j][i]
 
     def to_bricks(self, lex):  # lex (nz, ny, nx)
         out = self.zeros()
         c = self.coords[: self.n_owned]
         for q in range(self.n_owned):
             cx, cy, cz = c[q]
-            out[q] = lex[8 * cz:8 * cz + 8, 8 * cy:8 * cy + 8, 8 * cx:8 * cx + 8]
+            E = self.E
+            out[q] = lex[E * cz:E * cz + E, E * cy:E * cy + E, E * cx:E * cx + E]
         return out
 
     def from_bricks(self, br):
@@ -47,20 +50,23 @@ class RankLevel:
         c = self.coords[: self.n_owned]
         for q in range(self.n_owned):
             cx, cy, cz = c[q]
-            lex[8 * cz:8 * cz + 8, 8 * cy:8 * cy + 8, 8 * cx:8 * cx + 8] = br[q]
+            E = self.E
+            lex[E * cz:E * cz + E, E * cy:E * cy + E, E * cx:E * cx + E] = br[q]
         return lex
 
 
 def padded(x, adj, nb):
-    """(nb, 10, 10, 10) = each brick plus its 6 face halos via the adjacency table."""
-    X = np.zeros((nb, 10, 10, 10))
-    X[:, 1:9, 1:9, 1:9] = x[:nb]
-    X[:, 1:9, 1:9, 0] = x[adj[:nb, 0]][:, :, :, 7]  # W: neighbour's i = 7
-    X[:, 1:9, 1:9, 9] = x[adj[:nb, 1]][:, :, :, 0]  # E
-    X[:, 1:9, 0, 1:9] = x[adj[:nb, 2]][:, :, 7, :]  # S
-    X[:, 1:9, 9, 1:9] = x[adj[:nb, 3]][:, :, 0, :]  # N
-    X[:, 0, 1:9, 1:9] = x[adj[:nb, 4]][:, 7, :, :]  # B
-    X[:, 9, 1:9, 1:9] = x[adj[:nb, 5]][:, 0, :, :]  # T
+    """(nb, E+2, E+2, E+2) = each brick plus its 6 face halos via the adjacency table."""
+    E = x.shape[-1]
+    X = np.zeros((nb, E + 2, E + 2, E + 2))
+    m = slice(1, E + 1)
+    X[:, m, m, m] = x[:nb]
+    X[:, m, m, 0] = x[adj[:nb, 0]][:, :, :, E - 1]  # W: neighbour's i = E - 1
+    X[:, m, m, E + 1] = x[adj[:nb, 1]][:, :, :, 0]  # E
+    X[:, m, 0, m] = x[adj[:nb, 2]][:, :, E - 1, :]  # S
+    X[:, m, E + 1, m] = x[adj[:nb, 3]][:, :, 0, :]  # N
+    X[:, 0, m, m] = x[adj[:nb, 4]][:, E - 1, :, :]  # B
+    X[:, E + 1, m, m] = x[adj[:nb, 5]][:, 0, :, :]  # T
     return X
 
 
@@ -72,10 +78,11 @@ def coeffs(h):
 def sweep(x, b, adj, nb, h):
     """Returns (x', r) on bricks [0, nb): a = alpha x + beta sum6; r = b - a; x' = x + gamma (a - b)."""
     al, be, ga = coeffs(h)
+    E = x.shape[-1]
     X = padded(x, adj, nb)
-    c = X[:, 1:9, 1:9, 1:9]
-    s = ((X[:, 1:9, 1:9, 0:8] + X[:, 1:9, 1:9, 2:10]) + (X[:, 1:9, 0:8, 1:9] + X[:, 1:9, 2:10, 1:9])) + \
-        (X[:, 0:8, 1:9, 1:9] + X[:, 2:10, 1:9, 1:9])
+    m, lo, hi = slice(1, E + 1), slice(0, E), slice(2, E + 2)
+    c = X[:, m, m, m]
+    s = ((X[:, m, m, lo] + X[:, m, m, hi]) + (X[:, m, lo, m] + X[:, m, hi, m])) + (X[:, lo, m, m] + X[:, hi, m, m])
     a = al * c + be * s
     xn = x.copy()
     r = np.zeros_like(x)
@@ -85,6 +92,7 @@ def sweep(x, b, adj, nb, h):
 
 
 def restrict(rf, fine: RankLevel, bc):
+    H = fine.E // 2
     for q in range(fine.n_owned):
         pr = int(fine.parent[q])
         cb, o = pr >> 3, pr & 7
@@ -92,15 +100,16 @@ def restrict(rf, fine: RankLevel, bc):
         f = rf[q]
         v = 0.125 * (((f[0::2, 0::2, 0::2] + f[0::2, 0::2, 1::2]) + (f[0::2, 1::2, 0::2] + f[0::2, 1::2, 1::2]))
                      + ((f[1::2, 0::2, 0::2] + f[1::2, 0::2, 1::2]) + (f[1::2, 1::2, 0::2] + f[1::2, 1::2, 1::2])))
-        bc[cb, 4 * oz:4 * oz + 4, 4 * oy:4 * oy + 4, 4 * ox:4 * ox + 4] = v
+        bc[cb, H * oz:H * oz + H, H * oy:H * oy + H, H * ox:H * ox + H] = v
 
 
 def interp(xf, fine: RankLevel, xc):
+    H = fine.E // 2
     for q in range(fine.n_owned):
         pr = int(fine.parent[q])
         cb, o = pr >> 3, pr & 7
         ox, oy, oz = o & 1, (o >> 1) & 1, o >> 2
-        blk = xc[cb, 4 * oz:4 * oz + 4, 4 * oy:4 * oy + 4, 4 * ox:4 * ox + 4]
+        blk = xc[cb, H * oz:H * oz + H, H * oy:H * oy + H, H * ox:H * ox + H]
         xf[q] = xf[q] + np.repeat(np.repeat(np.repeat(blk, 2, 0), 2, 1), 2, 2)
 
 
@@ -131,7 +140,7 @@ def replicated_bottom(b_own, gathered_fn, src, mine, gadj, h, bottom):
     that periodic grid, this rank's owned x by `mine`.  gathered_fn(b_own) -> [world * n_own] bricks."""
     gb = gathered_fn(b_own)[src]
     ng = len(src)
-    x = np.zeros((ng, 8, 8, 8))
+    x = np.zeros((ng,) + b_own.shape[1:])
     for _ in range(bottom):
         x, _ = sweep(x, gb, gadj, ng, h)
     return x[mine]

@@ -5,7 +5,9 @@ against the CPU oracle (bitwise, and within the north-star tolerances):
     axis a ghost shell whose domain-face bricks are filled by the mirror exchange (method of images),
     so the paper's kernels, the communication-avoiding schedule and the decompositions run unchanged;
   * variable coefficients (reading A23): div(c grad x) with face averages of the cell coefficients,
-    damped Jacobi with the local diagonal, coarse c = restriction of c (one-brick kernels, SW_VARCOEF).
+    damped Jacobi with the local diagonal, coarse c = restriction of c (one-brick kernels, SW_VARCOEF);
+  * 4^3 bricks (brick_edge = 4, P:L154 Sunspot): the generic kernel family of generic.cu on the same
+    layout, exchange and schedule machinery.
 """
 import numpy as np
 import pytest
@@ -260,4 +262,81 @@ def test_var_coef_solve_and_state_errors(oracle_mod):
     m = new(shape, 4)
     with pytest.raises(mg.MGError):
         m.set_coefficients(dev(c))
+    m.close()
+
+
+# ------------------------------------------------------------ 4^3 bricks
+@pytest.mark.parametrize("shape,L", [((64, 64, 64), 4), ((32, 16, 48), 3), ((64, 64, 64), 5)])
+@pytest.mark.parametrize("variant", ["paper", "dirichlet", "varcoef"])
+def test_brick4_vcycle_bitwise(oracle_mod, shape, L, variant):
+    """4^3 bricks: V-cycles (12/12/100) bitwise equal to the oracle's after each of 2 cycles -- the
+    paper's problem, Dirichlet, and variable coefficients with a Neumann boundary (the oracle does not
+    know bricks: the brick edge must not change a bit)."""
+    bc = {"paper": 0, "dirichlet": 1, "varcoef": 2}[variant]
+    vc = variant == "varcoef"
+    b = mg_inputs.random_field(shape, 41) if bc == 1 else mg_inputs.random_rhs(shape, 41)
+    c = mg_inputs.random_coef(shape, 41) if vc else None
+    xs, ns = oracle_cycles(oracle_mod, b, L, 2, bc=bc, coef=c)
+    m = new(shape, L, bc=bc, var_coef=int(vc), brick_edge=4)
+    if vc:
+        m.set_coefficients(dev(c))
+    m.set_rhs(dev(b))
+    m.set_solution(None)
+    check_cycles(m, xs, ns)
+    m.close()
+
+
+@pytest.mark.parametrize("fusion", [1, 2, 3])
+@pytest.mark.parametrize("period", [1, 3, 4])
+@pytest.mark.parametrize("ghost_mode", [0, 1])
+@pytest.mark.parametrize("E", [4, 8])
+def test_brick4_fusion_ca_ghosts_bitwise(oracle_mod, fusion, period, ghost_mode, E):
+    """4^3 (and 8^3) bricks through the paper's kernel set (applyOp + smooth+residual + restriction +
+    initZero + interpolation), the fused sweep and full fusion; CA periods up to the 4-cell ghost
+    depth, with and without a self-exchanged ghost shell (the paper set's in-place smooth under the
+    interior / surface overlap split: every applyOp before the first smooth): the oracle's bits."""
+    shape = (32, 32, 64)
+    b = mg_inputs.random_rhs(shape, 42)
+    xs, ns = oracle_cycles(oracle_mod, b, 3, 2, 5, 4, 30)
+    m = new(shape, 3, pre=5, post=4, bottom=30, brick_edge=E, fusion=fusion, ca_period=period,
+            ghost_mode=ghost_mode)
+    m.set_rhs(dev(b))
+    m.set_solution(None)
+    check_cycles(m, xs, ns)
+    m.close()
+
+
+@pytest.mark.parametrize("pg,n_local,L,bc", [((2, 1, 1), (16, 16, 16), 3, 0), ((2, 2, 2), (16, 16, 16), 2, 1),
+                                             ((1, 2, 3), (8, 16, 8), 2, 0)])
+def test_brick4_loopback_decomposition_bitwise(oracle_mod, pg, n_local, L, bc):
+    """Decomposed 4^3-brick runs (one-brick-deep = 4-cell ghost shells exchanged through the same
+    packing-free plans) reproduce the undecomposed oracle bit for bit."""
+    _, solver = _mg()
+    gshape = (n_local[2] * pg[2], n_local[1] * pg[1], n_local[0] * pg[0])
+    b = mg_inputs.random_field(gshape, 43) if bc else mg_inputs.random_rhs(gshape, 43)
+    xs, ns = oracle_cycles(oracle_mod, b, L, 2, bc=bc)
+    g = solver.LoopbackGroup(n_local, pg, num_levels=L, bc=bc, brick_edge=4)
+    g.set_rhs([dev(mg_inputs.local_block(b, r, pg)) for r in range(g.world_size)])
+    g.set_solution(None)
+    for cyc in range(2):
+        g.vcycle()
+        assert g.residual_norm() == ns[cyc]
+        for r in range(g.world_size):
+            assert_bitwise(host(g.get_solution(r)), mg_inputs.local_block(xs[cyc], r, pg), what=f"rank {r}")
+    g.close()
+
+
+def test_brick4_solve_matches_oracle(oracle_mod):
+    """Alg 1 with 4^3 bricks: same cycle count and final norm as the oracle."""
+    shape = (64, 64, 64)
+    b = mg_inputs.sin_rhs(shape)
+    orc = oracle_mod.OracleMG(shape, 4)
+    orc.set_b(b)
+    orc.set_x(None)
+    c_o, norms = orc.solve(1e-10, 20)
+    m = new(shape, 4, brick_edge=4)
+    m.set_rhs(dev(b))
+    m.set_solution(None)
+    st, c_g, fin = m.solve(1e-10, 20)
+    assert st == 0 and c_g == c_o and fin == norms[-1] and fin < 1e-10
     m.close()

@@ -373,3 +373,71 @@ def test_workspace_is_rank_independent(n_local, pg, L, bc):
         p = mg.params(n_local, pg, num_levels=L, bc=bc, var_coef=vc)
         sizes = {mg.mg_workspace_bytes(p, r, world) for r in range(world)}
         assert len(sizes) == 1, sizes
+
+
+B4_CASES = [((16, 16, 16), (1, 1, 1), 3, 0, 0), ((16, 16, 16), (1, 1, 1), 2, 1, 0), ((8, 16, 8), (2, 1, 1), 2, 0, 0),
+            ((8, 8, 8), (2, 2, 2), 2, 0, 1), ((8, 8, 16), (1, 2, 3), 2, 0, 2), ((16, 8, 8), (2, 1, 1), 2, 0, 1)]
+
+
+@pytest.mark.parametrize("n_local,pg,L,gm,bc", B4_CASES)
+def test_brick4_layout_and_interpreter_bitwise_vs_oracle(oracle_mod, n_local, pg, L, gm, bc):
+    """4^3 bricks (brick_edge = 4, P:L154 Sunspot): the same layout machinery with a
+    4-cell brick -- adjacency consistent with the coords, every ghost brick filled exactly once --
+    and the host brick interpreter on those tables reproduces the oracle's V-cycle bit for bit
+    (periodic, self-exchanged ghost shells, decompositions, Dirichlet / Neumann)."""
+    p, lays = layouts(n_local, pg, L, gm, brick_edge=4, bc=bc)
+    for lay in lays:
+        for l in range(L):
+            inf = lay.info(l)
+            assert inf["nb"] == [n >> l >> 2 for n in n_local]
+            adj, co = lay.adjacency(l), lay.coords(l)
+            index = {tuple(c): q for q, c in enumerate(co)}
+            for q in range(inf["owned"]):
+                for f, d in enumerate(FACE):
+                    e = [int(co[q][a]) + d[a] for a in range(3)]
+                    for a in range(3):
+                        if not inf["ghost"][a]:
+                            e[a] %= inf["nb"][a]
+                    assert adj[q, f] == index[tuple(e)]
+            got = np.zeros(inf["owned"] + inf["nghost"], dtype=int)
+            for peer, d, run, local, remote, count in lay.plan(l, 1):
+                got[local:local + count] += 1
+            for dst, src, mask in lay.mirror(l):
+                got[dst] += 1
+            assert np.all(got[inf["owned"]:] == 1)
+    gshape = (n_local[2] * pg[2], n_local[1] * pg[1], n_local[0] * pg[0])
+    b = mg_inputs.random_field(gshape, 19) if bc == 1 else mg_inputs.random_rhs(gshape, 19)
+    pre, post, bottom = 3, 2, 15
+    h0 = mg_inputs.default_h0(gshape)
+    orc = oracle_mod.OracleMG(gshape, L, pre, post, bottom, h0, bc=bc)
+    orc.set_b(b)
+    orc.set_x(None)
+    orc.vcycle()
+    R = len(lays)
+    ranks = [[bi.RankLevel(lays[r], l) for l in range(L)] for r in range(R)]
+    assert ranks[0][0].E == 4
+    xs = [[ranks[r][l].zeros() for l in range(L)] for r in range(R)]
+    bs = [[None] * L for _ in range(R)]
+    for r in range(R):
+        bs[r][0] = ranks[r][0].to_bricks(mg_inputs.local_block(b, r, pg))
+    b0 = bi.exchange_local([bs[r][0] for r in range(R)], [ranks[r][0] for r in range(R)])
+    for r in range(R):
+        bs[r][0] = b0[r]
+    xs = bi.vcycle_ranks(xs, bs, ranks, L, h0, pre, post, bottom)
+    got = np.zeros(gshape)
+    for r in range(R):
+        cx, cy, cz = mg_inputs.rank_coords(r, pg)
+        nx, ny, nz = n_local
+        got[cz * nz:(cz + 1) * nz, cy * ny:(cy + 1) * ny, cx * nx:(cx + 1) * nx] = ranks[r][0].from_bricks(xs[r][0])
+    assert np.array_equal(got, orc.get_x())
+
+
+def test_brick4_params():
+    """brick_edge 4: n_local a multiple of 4*2^(L-1), ca_period <= 4, no CG bottom; 5 is refused."""
+    ok = mg.params((12, 8, 4), num_levels=1, brick_edge=4)
+    assert mg.mg_workspace_bytes(ok, 0, 1) > 0
+    for p in (mg.params((12, 8, 4), num_levels=2, brick_edge=4), mg.params((16, 16, 16), num_levels=2, brick_edge=5),
+              mg.params((16, 16, 16), num_levels=2, brick_edge=4, ca_period=5),
+              mg.params((16, 16, 16), num_levels=2, brick_edge=4, bottom_solver=1)):
+        with pytest.raises(mg.MGError):
+            mg.mg_workspace_bytes(p, 0, 1)
