@@ -54,8 +54,7 @@ def parse():
     ap.add_argument("--no-overlap", action="store_true")
     ap.add_argument("--tb", type=int, default=3,
                     help="temporal blocking (two sweeps per HBM pass): 3 = 2x2-brick pencils, two-warp CTAs (sweep2p.cu, "
-                         "default), 4 = 2x2-brick pencils, one warp per tile (sweep2q.cu), 1 = one-brick "
-                         "CTA streams (sweep2.cu), 2 = warp plane streams (sweep2w.cu), 0 = off")
+                         "default), 1 = one-brick CTA streams (sweep2.cu), 0 = off")
     ap.add_argument("--smoother", type=int, default=0,
                     help="0 damped Jacobi (the paper), 1 Chebyshev, 2 red-black Gauss-Seidel (N4 variants)")
     ap.add_argument("--cheby-ratio", type=int, default=0, help="Chebyshev smoothing interval [mu_max/ratio, mu_max]")
@@ -63,6 +62,9 @@ def parse():
     ap.add_argument("--bottom-solver", type=int, default=0, help="0 Jacobi smooths (the paper), 1 CG (variant)")
     ap.add_argument("--bottom-mode", type=int, default=0,
                     help="0 auto, 1 per-sweep launches, 2 resident bottom, 3 cluster coarse solve, 4 grid coarse solve")
+    ap.add_argument("--bc", type=int, default=0, help="variant (reading A22): 0 periodic (the paper), 1 Dirichlet, 2 Neumann")
+    ap.add_argument("--var-coef", action="store_true", help="variant (reading A23): div(c grad x), smooth c")
+    ap.add_argument("--brick-edge", type=int, default=0, help="variant: 4 = 4^3 bricks (P:L154 Sunspot)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--ref-n", type=int, default=0, help="reference arm: grid side of the bounded sample")
@@ -87,8 +89,10 @@ def dist_env():
 
 
 def workload_name(a, pg):
-    return (f"{a.n}^3 FP64 Poisson per GPU, 8^3 bricks, L={a.levels} ({a.n}->{a.n >> (a.levels - 1)}), "
-            f"{a.pre}/{a.post}/{a.bottom} smooths, 3D decomposition {pg[0]}x{pg[1]}x{pg[2]}")
+    e = a.brick_edge or 8
+    var = "".join([{0: "", 1: ", Dirichlet", 2: ", Neumann"}[a.bc], ", variable coefficients" if a.var_coef else ""])
+    return (f"{a.n}^3 FP64 Poisson per GPU, {e}^3 bricks, L={a.levels} ({a.n}->{a.n >> (a.levels - 1)}), "
+            f"{a.pre}/{a.post}/{a.bottom} smooths, 3D decomposition {pg[0]}x{pg[1]}x{pg[2]}{var}")
 
 
 # ------------------------------------------------------------------ clocks
@@ -329,11 +333,17 @@ def main():
                   ghost_mode=1 if a.ghost_all else 0, use_graph=not a.no_graph, overlap=not a.no_overlap,
                   rank=rank, world_size=world, device=local, temporal_blocking=a.tb, smoother=a.smoother,
                   cheby_ratio=a.cheby_ratio, launch_pdl=2 if a.no_pdl else 0,
-                  bottom_mode=a.bottom_mode, bottom_solver=a.bottom_solver,
+                  bottom_mode=a.bottom_mode, bottom_solver=a.bottom_solver, bc=a.bc,
+                  var_coef=1 if a.var_coef else 0, brick_edge=a.brick_edge,
                   transport={"auto": mg.MG_TRANSPORT_AUTO, "nccl": mg.MG_TRANSPORT_NCCL,
                              "local": mg.MG_TRANSPORT_LOCAL, "peer": mg.MG_TRANSPORT_PEER}[a.transport])
     gshape = (n * pg[2], n * pg[1], n * pg[0])
-    b_host = torch.from_numpy(mg_inputs.local_sin_rhs(gshape, rank, pg)).pin_memory()
+    if a.bc == 1:  # the lowest Dirichlet mode (the sin b of P:L148 is not zero on the faces)
+        b_host = torch.from_numpy(mg_inputs.local_block(mg_inputs.dirichlet_sin_rhs(gshape), rank, pg)).pin_memory()
+    else:
+        b_host = torch.from_numpy(mg_inputs.local_sin_rhs(gshape, rank, pg)).pin_memory()
+    if a.var_coef:
+        m.set_coefficients(torch.from_numpy(mg_inputs.local_block(mg_inputs.smooth_coef(gshape), rank, pg)).to(dev))
     b_dev = b_host.to(dev)
     m.set_rhs(b_dev)
     m.set_solution(None)
@@ -399,7 +409,7 @@ def main():
     # the same level-0 work expressed as one-sweep-per-pass traffic (what the sweeps would move unblocked)
     sweep_equiv = pts * (B_SWEEP * nsweep0 + 2 * B_COARSE_PER_FINE) / (sweep0_ms / 1e3) / 1e9
     peak, peak_src = measured_peaks()
-    pass_kernel = {0: "sweep_col_kernel", 1: "sweep2_kernel", 2: "sweep2w_kernel", 4: "sweep2q_kernel"}.get(
+    pass_kernel = {0: "sweep_col_kernel", 1: "sweep2_kernel"}.get(
         a.tb, "sweep2p_kernel")
     traffic = ncu_traffic(n, pass_kernel)
     levels = []
@@ -466,16 +476,17 @@ def main():
             "warmup": a.warmup, "ms_per_step": t_ms / a.steps, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": workload_name(a, pg), "n_local": [n, n, n], "proc_grid": list(pg),
-                       "levels": a.levels, "smooths": [a.pre, a.post, a.bottom], "brick": 8,
+                       "levels": a.levels, "smooths": [a.pre, a.post, a.bottom], "brick": a.brick_edge or 8,
+                       "bc": {0: "periodic (paper)", 1: "dirichlet", 2: "neumann"}[a.bc],
+                       "coefficients": "variable (smooth c)" if a.var_coef else "constant (paper)",
                        "fusion": "auto(full)" if not a.fusion else a.fusion,
-                       "ca_period": a.ca_period or "auto(8)", "ghost_mode": "all" if a.ghost_all else "auto",
+                       "ca_period": a.ca_period or "auto", "ghost_mode": "all" if a.ghost_all else "auto",
                        "cuda_graph": not a.no_graph, "overlap": not a.no_overlap, "pdl": not a.no_pdl,
                        "transport": a.transport,
                        "coarse": {0: "auto", 1: "per-sweep launches", 2: "resident bottom", 3: "cluster solve",
                                   4: "grid solve"}[a.bottom_mode],
                        "bottom_solver": "conjugate gradients" if a.bottom_solver else "damped jacobi (paper)",
-                       "temporal_blocking": {0: "off", 1: "one-brick CTA streams", 2: "warp plane streams",
-                                             4: "2x2-brick pencils, one warp per tile"}.get(
+                       "temporal_blocking": {0: "off", 1: "one-brick CTA streams"}.get(
                            a.tb, "2x2-brick pencils, two-warp CTAs"),
                        "smoother": {1: "chebyshev", 2: "red-black gauss-seidel"}.get(a.smoother, "damped jacobi (paper)"),
                        "l2": "no flush: every level-0 field is 1 GiB > 126 MB L2 (inputs larger than L2)",

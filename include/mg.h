@@ -129,8 +129,10 @@ typedef struct {
   int32_t overlap;               /* 1 = sweep interior bricks while the exchange is in flight */
   int32_t sweep_kernel;          /* 0 = auto (streaming column kernel on levels >= 16384 bricks),
                                     1 = one-brick-per-CTA kernel only, 2 = streaming kernel on every level */
-  int32_t temporal_blocking;     /* 1 = two Jacobi sweeps per HBM pass on streaming levels (sweep2.cu,
-                                    bit-identical; default), 0 = one sweep per pass */
+  int32_t temporal_blocking;     /* two Jacobi sweeps per HBM pass (bit-identical): 3 = over 2x2-brick pencils
+                                    (sweep2p.cu, the default), 1 = one-brick CTA item streams (sweep2.cu; also
+                                    the fallback of 3 on ranges that do not tile into pencils), 0 = one sweep
+                                    per pass; anything else is refused */
   int32_t smoother;              /* 0 = damped Jacobi (the paper); 1 = Chebyshev: the pre / post
                                     sweeps of a level take the steps h^2/(12 nu_k) at the Chebyshev nodes nu_k of
                                     [1/cheby_ratio, 1] (variant N4, reading A19); 2 = red-black

@@ -47,6 +47,7 @@ struct DevLevel {
   int32_t* adj = nullptr;
   int32_t* parent = nullptr;
   int32_t* coord = nullptr;
+  int32_t* radj = nullptr;  // resident-bottom adjacency of a one-rank non-periodic level (LevelLayout::radj)
   Coeffs c{};
   double h = 0;
   struct Col {
@@ -63,7 +64,6 @@ struct DevLevel {
   std::vector<Pair> pairs;  // two-sweep item streams per brick range
   PairMaps pmaps[2];        // tensor maps for the two-sweep kernel reading x[0] / x[1]
   PairMaps nmaps[2];        // the same with 4-plane boxes for the pencil kernel (sweep2p.cu)
-  PairMaps qmaps[2];        // 2-plane boxes for the one-warp pencil kernel (sweep2q.cu)
   // local-transport exchange: [x[0] | x[1] | b][recv run] copy descriptors (device), one launch
   CopyRun* cruns = nullptr;
   int ncruns = 0;
@@ -218,6 +218,7 @@ size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double**
     d.adj = (int32_t*)take((size_t)L.n_stored * 8 * sizeof(int32_t));
     d.parent = (int32_t*)take((size_t)L.n_alloc * sizeof(int32_t));
     d.coord = (int32_t*)take((size_t)L.n_stored * 3 * sizeof(int32_t));
+    if (!L.radj.empty()) d.radj = (int32_t*)take(L.radj.size() * sizeof(int32_t));
     for (const auto& ct : L.cols) {
       DevLevel::Col col;
       col.b0 = ct.b0;
@@ -237,8 +238,6 @@ size_t carve(const Layout& lay, char* base, std::vector<DevLevel>* out, double**
       pr.args.meta = (const int32_t*)take(pt.meta.size() * sizeof(int32_t));
       pr.args.ctas = (const int2*)take(pt.ctas.size() * sizeof(int32_t));
       pr.args.nctas = (int64_t)pt.ctas.size() / 2;
-      pr.args.warps = (const int4*)take(pt.warps.size() * sizeof(int32_t));
-      pr.args.nwarps = (int64_t)pt.warps.size() / 4;
       d.pairs.push_back(pr);
     }
     // (sized rank-independently: every rank of a run carves the same layout -- the loopback group and the
@@ -517,12 +516,8 @@ mg_status sweep_range(mg_ctx* c, const Op& o, int64_t b0, int64_t b1, cudaStream
   if (o.kind == OP_SWEEP2) {  // two sweeps in one pass: the builder only emits it where a plan exists
     for (const auto& pr : d.pairs) {
       if (pr.b0 == b0 && pr.b1 == b1 && pr.part == part) {
-        if (pr.args.kind == 4)
-          CKC(c, launch_sweep2q(a, pr.args, d.qmaps[o.src], o.flags | (o.zero ? SW_ZERO_X : 0u), s));
-        else if (pr.args.kind == 3)
+        if (pr.args.kind == 3)
           CKC(c, launch_sweep2p(a, pr.args, d.nmaps[o.src], o.flags | (o.zero ? SW_ZERO_X : 0u), s));
-        else if (pr.args.kind == 2)
-          CKC(c, launch_sweep2w(a, pr.args, d.pmaps[o.src], o.flags, s));
         else
           CKC(c, launch_sweep2(a, pr.args, d.pmaps[o.src], o.flags, s));
         return MG_OK;
@@ -707,7 +702,11 @@ mg_status exec_op(mg_ctx* c, const Op& o, cudaStream_t s) {
       return MG_OK;
     case OP_BOTTOM_RES:
       CKS(timer_begin(c, s, &t0));
-      CKC(c, launch_bottom_resident(d.x[o.src], d.x[o.dst], d.b, d.adj, (int)L.n_stored, o.n, o.zero, d.c, s));
+      if (!L.radj.empty())  // non-periodic bc, one rank: owned bricks, domain faces as images
+        CKC(c, launch_bottom_resident(d.x[o.src], d.x[o.dst], d.b, d.radj, (int)L.n_owned, o.n, o.zero, d.c, s,
+                                      d.mirror_sign));
+      else
+        CKC(c, launch_bottom_resident(d.x[o.src], d.x[o.dst], d.b, d.adj, (int)L.n_stored, o.n, o.zero, d.c, s));
       CKS(timer_end(c, s, t0, o.level, o.timer));
       return MG_OK;
   }
@@ -859,6 +858,8 @@ mg_status init_ctx(mg_ctx* c, const mg_params& p, int rank, int world, int devic
     if (!L.mirror.empty())
       CKC(c, cudaMemcpyAsync(d.mirror, L.mirror.data(), L.mirror.size() * sizeof(int32_t), cudaMemcpyHostToDevice,
                              stream));
+    if (!L.radj.empty())
+      CKC(c, cudaMemcpyAsync(d.radj, L.radj.data(), L.radj.size() * sizeof(int32_t), cudaMemcpyHostToDevice, stream));
     for (size_t k = 0; k < L.cols.size(); ++k) {
       const auto& ct = L.cols[k];
       const ColArgs& ca = d.cols[k].args;
@@ -873,13 +874,11 @@ mg_status init_ctx(mg_ctx* c, const mg_params& p, int rank, int world, int devic
       const PairArgs& pa = d.pairs[k].args;
       CKC(c, cudaMemcpyAsync((void*)pa.meta, pt.meta.data(), pt.meta.size() * 4, cudaMemcpyHostToDevice, stream));
       CKC(c, cudaMemcpyAsync((void*)pa.ctas, pt.ctas.data(), pt.ctas.size() * 4, cudaMemcpyHostToDevice, stream));
-      CKC(c, cudaMemcpyAsync((void*)pa.warps, pt.warps.data(), pt.warps.size() * 4, cudaMemcpyHostToDevice, stream));
     }
     if (!L.pairs.empty())
       for (int xb = 0; xb < 2; ++xb) {
         CKC(c, encode_pair_maps(d.x[xb], d.b, L.n_alloc, &d.pmaps[xb]));
         CKC(c, encode_pencil_maps(d.x[xb], d.b, L.n_alloc, &d.nmaps[xb]));
-        CKC(c, encode_quad_maps(d.x[xb], d.b, L.n_alloc, &d.qmaps[xb]));
       }
   }
   if (c->lay.repl) {
@@ -1166,6 +1165,32 @@ mg_status mg_vcycle(mg_ctx* c) {
   return vcycle_impl(c, nullptr);
 }
 
+// max |b - Ax| of level 0's owned cells -> atomicMax on *acc: the TMA column kernel (16 B/pt at its
+// streaming rate) where level 0 has a column plan over the owned range, else the one-brick kernel
+static mg_status norm_launch(mg_ctx* c, unsigned long long* acc, cudaStream_t s) {
+  const LevelLayout& L = c->lay.lv[0];
+  DevLevel& d = c->dl[0];
+  const int cur = c->st[0].cur;
+  if (c->use_col && !d.cf && c->lay.E == 8) {
+    for (const auto& col : d.cols) {
+      if (col.b0 == 0 && col.b1 == L.n_owned) {
+        SweepArgs a{};
+        a.x = d.x[cur];
+        a.b = d.b;
+        a.adj = d.adj;
+        a.brick0 = 0;
+        a.nbricks = L.n_owned;
+        a.c = d.c;
+        a.acc = acc;
+        CKC(c, launch_sweep_col(a, col.args, d.fmaps[cur], SW_NORM, s));
+        return MG_OK;
+      }
+    }
+  }
+  CKC(c, launch_norm(d.x[cur], d.b, d.adj, L.n_owned, d.c, acc, s, d.cf, c->lay.E));
+  return MG_OK;
+}
+
 mg_status mg_residual_norm_async(mg_ctx* c) {
   CKS(check_ctx(c));
   if (c->group) return set_err(MG_ERR_STATE, "group member: use mg_group_residual_norm");
@@ -1180,7 +1205,7 @@ mg_status mg_residual_norm_async(mg_ctx* c) {
     c->st[0].since = 0;
   }
   CKC(c, cudaMemsetAsync(c->acc, 0, sizeof(unsigned long long), c->stream));
-  CKC(c, launch_norm(d.x[c->st[0].cur], d.b, d.adj, L.n_owned, d.c, c->acc, c->stream, d.cf, c->lay.E));
+  CKS(norm_launch(c, c->acc, c->stream));
   if (c->use_nccl && c->lay.world > 1)
     CKN(c, ncclAllReduce(c->acc, c->acc, 1, ncclUint64, ncclMax, c->nccl, c->stream));
   if (c->use_peer && c->lay.world > 1) {

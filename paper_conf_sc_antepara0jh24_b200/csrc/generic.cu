@@ -7,7 +7,7 @@
 // a warp per brick) instead of one: the same cells per CTA as the one-brick-per-CTA kernels of
 // kernels.cu, whose structure these follow (brick + six face halos staged in shared memory through
 // the adjacency table; the canonical expression DAG of reading A8 / A23, so the results are bitwise
-// those of the oracle and of the 8^3 path).  The 8^3-specific kernels (TMA column sweeps, two-sweep
+// those of the 8^3 path and of the lexicographic reference).  The 8^3-specific kernels (TMA column sweeps, two-sweep
 // pencil passes, resident / cluster / CG bottoms) are not used with E = 4 (mg_setup forces the
 // one-brick kernel family and per-sweep bottoms).
 #include <cuda_runtime.h>

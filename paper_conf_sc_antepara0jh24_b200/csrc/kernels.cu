@@ -314,8 +314,10 @@ __global__ void __launch_bounds__(COL_WARPS * 32, 6)
   pdl_wait();
   constexpr bool WRITE_R = (FLAGS & SW_WRITE_R) != 0;
   constexpr bool RESTRICT = (FLAGS & SW_RESTRICT) != 0;
+  constexpr bool NORM = (FLAGS & SW_NORM) != 0;  // maxNormRes: only max |b - Ax| leaves the kernel
   extern __shared__ __align__(128) unsigned char smem_raw[];
   ColSmem<RESTRICT>& S = *reinterpret_cast<ColSmem<RESTRICT>*>(smem_raw);
+  double mx = 0.0;
   const int t = threadIdx.x, w = t >> 5, l = t & 31;
   const int i0 = 2 * (l & 3), j = l >> 2;
   const int q = 8 * j + i0;  // this lane's pair inside a plane
@@ -409,7 +411,12 @@ __global__ void __launch_bounds__(COL_WARPS * 32, 6)
       xn.y = keep_cell(p.colour, i0 + 1, j, k) ? xc.y : DADD(xc.y, DMUL(p.c.gamma, DSUB(a1, bb.y)));
       rv.x = DSUB(bb.x, a0);
       rv.y = DSUB(bb.y, a1);
-      st_stream2(p.xo + gbase + 64 * k, xn);
+      if (NORM) {
+        mx = nan_max(mx, fabs(rv.x));
+        mx = nan_max(mx, fabs(rv.y));
+      } else {
+        st_stream2(p.xo + gbase + 64 * k, xn);
+      }
       if (WRITE_R) st_stream2(p.r + gbase + 64 * k, rv);
       if (RESTRICT) *reinterpret_cast<double2*>(S.rs[n & 1] + 64 * k + q) = rv;
       if (k == 7) *reinterpret_cast<double2*>(S.carry[n & 1] + q) = xc;  // k-halo of the next brick
@@ -429,6 +436,18 @@ __global__ void __launch_bounds__(COL_WARPS * 32, 6)
       p.bc[(int64_t)(pr >> 3) * 512 + (4 * ox + I) + 8 * (4 * oy + J) + 64 * (4 * oz + K)] = v;
     }
   }
+  if (NORM) {  // exact max over the CTA's cells, published as uint64 bits (monotone for >= 0)
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) mx = nan_max(mx, __shfl_xor_sync(0xffffffffu, mx, off));
+    __shared__ double wm[COL_WARPS];
+    if (l == 0) wm[w] = mx;
+    __syncthreads();
+    if (t == 0) {
+      double m = wm[0];
+      for (int q2 = 1; q2 < COL_WARPS; ++q2) m = nan_max(m, wm[q2]);
+      atomicMax(p.acc, (unsigned long long)__double_as_longlong(m));
+    }
+  }
   pdl_trigger();
 }
 
@@ -442,11 +461,16 @@ cudaError_t launch_sweep_col(const SweepArgs& a, const ColArgs& c, const FaceMap
   if (c.nseg <= 0) return cudaSuccess;
   const size_t sm = sizeof(ColSmem<false>), smr = sizeof(ColSmem<true>);
   const unsigned g = (unsigned)c.nseg, b = COL_WARPS * 32;
-  switch (flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP | SW_ZERO_X)) {
+  if (flags == SW_NORM) {
+    launch_plain(sweep_col_kernel<SW_NORM>, g, b, sm, s, a, c, fm);
+    return cudaGetLastError();
+  }
+  switch (flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP | SW_ZERO_X | SW_NORM)) {
     case 0: launch_plain(sweep_col_kernel<0>, g, b, sm, s, a, c, fm); break;
     case SW_WRITE_R: launch_plain(sweep_col_kernel<SW_WRITE_R>, g, b, sm, s, a, c, fm); break;
     case SW_RESTRICT: launch_plain(sweep_col_kernel<SW_RESTRICT>, g, b, smr, s, a, c, fm); break;
-    default: return cudaErrorInvalidValue;
+    default:
+      return cudaErrorInvalidValue;
   }
   return cudaGetLastError();
 }
@@ -682,17 +706,17 @@ cudaError_t launch_zero(double* x, int64_t brick0, int64_t nbricks, cudaStream_t
 __global__ void __launch_bounds__(1024) bottom_resident_kernel(const double* __restrict__ x, double* __restrict__ xo,
                                                                const double* __restrict__ b,
                                                                const int32_t* __restrict__ adj, int nbricks,
-                                                               int sweeps, int zero_x, Coeffs c) {
+                                                               int sweeps, int zero_x, Coeffs c, double msign) {
   pdl_begin();
   extern __shared__ __align__(16) double sm[];
-  bottom_resident_body(x, xo, b, adj, nbricks, sweeps, zero_x, c, sm);
+  bottom_resident_body(x, xo, b, adj, nbricks, sweeps, zero_x, c, sm, msign);
 }
 
 cudaError_t launch_bottom_resident(const double* x, double* xo, const double* b, const int32_t* adj, int nbricks,
-                                   int sweeps, bool zero_x, Coeffs c, cudaStream_t s) {
+                                   int sweeps, bool zero_x, Coeffs c, cudaStream_t s, double msign) {
   if (nbricks <= 0 || nbricks > kResidentMaxBricks) return cudaErrorInvalidValue;
   const size_t smem = (size_t)nbricks * 512 * 2 * sizeof(double);
-  launch_k(bottom_resident_kernel, 1, 128 * nbricks, smem, s, x, xo, b, adj, nbricks, sweeps, zero_x ? 1 : 0, c);
+  launch_k(bottom_resident_kernel, 1, 128 * nbricks, smem, s, x, xo, b, adj, nbricks, sweeps, zero_x ? 1 : 0, c, msign);
   return cudaGetLastError();
 }
 
@@ -791,9 +815,9 @@ cudaError_t kernels_init() {
   e = cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev);
   if (e != cudaSuccess) return e;
   const int colsm = (int)sizeof(ColSmem<false>), colsmr = (int)sizeof(ColSmem<true>);
-  const void* colk[3] = {(const void*)sweep_col_kernel<0>, (const void*)sweep_col_kernel<SW_WRITE_R>,
-                         (const void*)sweep_col_kernel<SW_RESTRICT>};
-  for (int k = 0; k < 3; ++k) {
+  const void* colk[4] = {(const void*)sweep_col_kernel<0>, (const void*)sweep_col_kernel<SW_WRITE_R>,
+                         (const void*)sweep_col_kernel<SW_RESTRICT>, (const void*)sweep_col_kernel<SW_NORM>};
+  for (int k = 0; k < 4; ++k) {
     e = cudaFuncSetAttribute(colk[k], cudaFuncAttributeMaxDynamicSharedMemorySize, k == 2 ? colsmr : colsm);
     if (e != cudaSuccess) return e;
     // the streaming kernel is shared-memory-resident: ask for the full 228 KB carveout
@@ -806,10 +830,6 @@ cudaError_t kernels_init() {
   e = pair_kernels_init();
   if (e != cudaSuccess) return e;
   e = pencil_kernels_init();
-  if (e != cudaSuccess) return e;
-  e = quad_kernels_init();
-  if (e != cudaSuccess) return e;
-  e = pairw_kernels_init();
   if (e != cudaSuccess) return e;
   e = coarse_kernels_init();
   if (e != cudaSuccess) return e;

@@ -23,6 +23,7 @@ enum SweepFlags : unsigned {
   SW_NO_SMOOTH = 16u,  // do not write x' (restriction-only last sweep is never used; kept for tests)
   SW_COLOUR = 32u,     // two-sweep kernel: red-black half-sweeps (colour masks compiled in only here)
   SW_VARCOEF = 64u,    // one-brick kernel: variable coefficients div(c grad x) (reading A23), SweepArgs::cf
+  SW_NORM = 128u,      // column kernel: no stores, max |b - Ax| into SweepArgs::acc (maxNormRes)
 };
 
 struct SweepArgs {
@@ -42,6 +43,7 @@ struct SweepArgs {
   const double* cf = nullptr;  // SW_VARCOEF: cell coefficients c (brick layout, ghosts valid)
   double vc_g = 0.0;           // SW_VARCOEF: 0.5 * h * h (gamma_p = vc_g / sum of the face coefficients)
   int E = 8;                   // brick edge (8; 4: the generic kernels of generic.cu)
+  unsigned long long* acc = nullptr;  // SW_NORM: atomicMax target (uint64 bits of a non-negative double)
 };
 
 cudaError_t launch_sweep(const SweepArgs& a, unsigned flags, cudaStream_t s);
@@ -71,13 +73,11 @@ cudaError_t encode_box_map(const double* base, int64_t n_alloc, const unsigned b
 
 // Two-sweep (temporally blocked) streaming kernel, sweep2.cu.
 struct PairArgs {
-  int kind;             // 1: CTA item streams (sweep2.cu), 2: half-warp plane streams (sweep2w.cu)
-  const int32_t* meta;  // kind 1: [items][11] id, flags, W,E,S,N, SW,NW,SE,NE, parent; kind 2: [items][12];
+  int kind;             // 1: CTA item streams (sweep2.cu), 3: 2x2-brick pencil chunk streams (sweep2p.cu)
+  const int32_t* meta;  // kind 1: [items][11] id, flags, W,E,S,N, SW,NW,SE,NE, parent;
                         // kind 3: [chunks][20] chunk records (mg_internal.h kPenRec)
-  const int2* ctas;     // kind 1: (first item, item count) per CTA
+  const int2* ctas;     // (first item / chunk, count) per CTA
   int64_t nctas;
-  const int4* warps;    // kind 2: (first item half 0, first item half 1, steps, items0 | items1<<16) per warp
-  int64_t nwarps;
 };
 struct PairMaps {
   CUtensorMap xwe;   // x boxes {2,8,8}: W (i=6,7) / E (i=0,1) face slabs
@@ -92,9 +92,6 @@ bool pair_supports(unsigned flags);
 cudaError_t launch_sweep2(const SweepArgs& a, const PairArgs& pa, const PairMaps& pm, unsigned flags,
                           cudaStream_t s);
 cudaError_t pair_kernels_init();
-cudaError_t launch_sweep2w(const SweepArgs& a, const PairArgs& pa, const PairMaps& pm, unsigned flags,
-                           cudaStream_t s);
-cudaError_t pairw_kernels_init();
 // 2x2-brick pencil two-sweep kernel (sweep2p.cu): maps with 4-plane boxes ({2,8,4}, {8,2,4},
 // {2,1,4}; b {2,8,4}, {8,1,4}) in the PairMaps fields
 cudaError_t encode_pencil_maps(const double* x, const double* b, int64_t n_alloc, PairMaps* out);
@@ -102,14 +99,6 @@ bool pencil_supports(unsigned flags);
 cudaError_t launch_sweep2p(const SweepArgs& a, const PairArgs& pa, const PairMaps& pm, unsigned flags,
                            cudaStream_t s);
 cudaError_t pencil_kernels_init();
-// one-warp 2x2-brick pencil two-sweep kernel (sweep2q.cu, plan kind 4: the kind-3 chunk records dealt
-// to kQuadCtas CTAs): maps with 2-plane boxes (x {2,8,2}, {8,2,2}, {2,1,2}; b {2,8,2}, {8,2,2}); the
-// flags of the SECOND sweep (plain, +r, +restriction) | SW_ZERO_X (the FIRST sweep reads x0 == 0)
-cudaError_t encode_quad_maps(const double* x, const double* b, int64_t n_alloc, PairMaps* out);
-bool quad_supports(unsigned flags);
-cudaError_t launch_sweep2q(const SweepArgs& a, const PairArgs& pa, const PairMaps& pm, unsigned flags,
-                           cudaStream_t s);
-cudaError_t quad_kernels_init();
 
 // true if the streaming kernel implements `flags` (plain, +r, +restriction)
 bool col_supports(unsigned flags);
@@ -135,7 +124,8 @@ cudaError_t launch_norm(const double* x, const double* b, const int32_t* adj, in
 // resident bottom solve: all `nbricks` (<= kResidentMaxBricks, no ghosts) in one CTA's shared memory
 constexpr int kResidentMaxBricks = 8;
 cudaError_t launch_bottom_resident(const double* x, double* xo, const double* b, const int32_t* adj, int nbricks,
-                                   int sweeps, bool zero_x, Coeffs c, cudaStream_t s);
+                                   int sweeps, bool zero_x, Coeffs c, cudaStream_t s,
+                                   double msign = 0.0);
 // layout conversion (not part of the V-cycle): lexicographic local <-> bricks [0, nowned)
 cudaError_t launch_lex_to_brick(const double* lex, double* bricks, const int32_t* coord, int64_t nowned, int nx,
                                 int ny, cudaStream_t s, int E = 8);

@@ -231,6 +231,33 @@ static void build_level(const Layout& lay, int l, LevelLayout& L) {
     L.adj[(size_t)b * 8 + 6] = (int32_t)b;
     L.adj[(size_t)b * 8 + 7] = 0;
   }
+  // one-CTA resident bottom under a non-periodic bc: when every ghost of the level is a reflection
+  // (one rank), the owned bricks' adjacency with each domain face marked -1 (the face cell's image
+  // is the cell itself, resident.cuh); empty when a ghost comes from another rank
+  L.radj.clear();
+  if (p.bc != MG_BC_PERIODIC && lay.world == 1 && L.recvs.empty()) {
+    std::vector<int32_t> src((size_t)L.n_ghost, -1), msk((size_t)L.n_ghost, 0);
+    for (size_t e = 0; e + 2 < L.mirror.size(); e += 3) {
+      src[(size_t)(L.mirror[e] - L.n_owned)] = L.mirror[e + 1];
+      msk[(size_t)(L.mirror[e] - L.n_owned)] = L.mirror[e + 2];
+    }
+    L.radj.assign((size_t)L.n_owned * 8, 0);
+    bool ok = true;
+    for (int64_t b = 0; b < L.n_owned && ok; ++b) {
+      for (int f = 0; f < 6; ++f) {
+        const int32_t nb = L.adj[(size_t)b * 8 + f];
+        if (nb < L.n_owned) {
+          L.radj[(size_t)b * 8 + f] = nb;
+        } else {
+          const int64_t g = nb - L.n_owned;
+          ok = g < L.n_ghost && src[(size_t)g] == b && msk[(size_t)g] == (1 << (f >> 1));
+          L.radj[(size_t)b * 8 + f] = -1;
+        }
+      }
+      L.radj[(size_t)b * 8 + 6] = (int32_t)b;
+    }
+    if (!ok) L.radj.clear();
+  }
 }
 
 static void build_parents(LevelLayout& F, const LevelLayout& C) {
@@ -302,6 +329,11 @@ mg_status build_layout(const mg_params& p, int rank, int world, Layout& out, std
     msg = "a non-periodic bc needs smoother 0/1 and bottom_solver 0 (reading A22)";
     return MG_ERR_INVALID_ARG;
   }
+  if (p.temporal_blocking != 0 && p.temporal_blocking != 1 && p.temporal_blocking != 3) {
+    msg = "temporal_blocking must be 0 (one sweep per pass), 1 (one-brick two-sweep streams) or 3 (2x2-brick "
+          "pencils, the default)";
+    return MG_ERR_INVALID_ARG;
+  }
   if (p.ghost_mode != MG_GHOST_AUTO && p.ghost_mode != MG_GHOST_ALL) {
     msg = "ghost_mode must be 0 or 1";
     return MG_ERR_INVALID_ARG;
@@ -321,7 +353,7 @@ mg_status build_layout(const mg_params& p, int rank, int world, Layout& out, std
   if (p.temporal_blocking != 0)
     for (int l = 0; l < out.L; ++l)
       build_pair_tables(out.lv[l], p.sweep_kernel == 0 ? kPairMinBricks : min_b,
-                        p.temporal_blocking >= 2 && p.temporal_blocking <= 4 ? p.temporal_blocking : 1);
+                        p.temporal_blocking == 3 ? 3 : 1);
   // replicated bottom: the global coarsest level as one rank would store it
   const LevelLayout& B = out.lv[(size_t)out.L - 1];
   out.repl = false;
@@ -517,8 +549,7 @@ static LevelLayout::PairTable pair_table(const LevelLayout& L, int64_t b0, int64
 // part 1 / 2 (levels with a ghost shell): only the units whose records name no ghost brick /
 // the others, so the first can run while an exchange fills the ghost bricks (part 1 on one CTA
 // slot per SM fewer, which the exchange's kernels then find free).
-// kind 3: G = kPenCtas (sweep2p.cu, two-warp CTAs); kind 4: the same records dealt to G = kQuadCtas
-// one-warp CTAs (sweep2q.cu).
+// kind 3: G = kPenCtas (sweep2p.cu, two-warp CTAs).
 static LevelLayout::PairTable pencil_table(const LevelLayout& L, int64_t b0, int64_t b1, int part = 0,
                                            int kind = 3) {
   LevelLayout::PairTable t;
@@ -571,9 +602,8 @@ static LevelLayout::PairTable pencil_table(const LevelLayout& L, int64_t b0, int
   t.part = part;
   const int64_t ncol = (int64_t)tx * ty;
   static const int64_t gpen = getenv("MG_PEN_CTAS") ? atoll(getenv("MG_PEN_CTAS")) : kPenCtas;  // (experiments)
-  static const int64_t gquad = getenv("MG_QUAD_CTAS") ? atoll(getenv("MG_QUAD_CTAS")) : kQuadCtas;
-  const int64_t gmax = kind == 4 ? gquad : gpen;
-  const int64_t per_sm = kind == 4 ? kQuadCtasPerSm : kPenCtasPerSm;
+  const int64_t gmax = gpen;
+  const int64_t per_sm = kPenCtasPerSm;
   const int64_t G = std::max<int64_t>(1, std::min<int64_t>(gmax, ncol * nz));
   std::vector<std::vector<int32_t>> stream((size_t)G);  // per CTA: its chunk records
   // one 20-int record per chunk: code (type << 1 | half), the 16 brick ids, parent of b00
@@ -653,96 +683,6 @@ static LevelLayout::PairTable pencil_table(const LevelLayout& L, int64_t b0, int
   return t;
 }
 
-// Plane streams for the warp two-sweep kernel (sweep2w.cu), one per half-warp
-// (G = kW2Streams, even).  Chains are dealt round-robin and the remainder cut
-// into equal pieces exactly as in pair_table; each run becomes
-// [warm-up (planes 5..7), bricks (0..7, emitted), cool-down (plane 0)].  The two
-// streams of a warp are padded with dummy items (zero brick, nothing emitted) to
-// the same number of steps, so the warp's two halves step in lockstep.
-// Returns an empty table (kind 0: the schedule then uses single-sweep passes) if a
-// stream would overflow the kernel's 16-bit item counts.
-static LevelLayout::PairTable warp_table(const LevelLayout& L, int64_t b0, int64_t b1) {
-  LevelLayout::PairTable t;
-  t.kind = 2;
-  t.b0 = b0;
-  t.b1 = b1;
-  const auto chains = z_chains(L, b0, b1);
-  const int64_t nch = (int64_t)chains.size();
-  int64_t nb = 0;
-  for (const auto& c : chains) nb += (int64_t)c.size();
-  int64_t G = std::max<int64_t>(2, std::min<int64_t>(kW2Streams, nb / 4));
-  G += G & 1;
-  auto adj = [&](int64_t id, int f) -> int32_t {
-    return id >= L.n_stored ? (int32_t)L.zero_brick : L.adj[(size_t)id * 8 + f];
-  };
-  struct Stream {
-    std::vector<int32_t> meta;
-    int64_t items = 0, steps = 0;
-  };
-  std::vector<Stream> st((size_t)G);
-  auto push_item = [&](Stream& s, int32_t id, int emit, int kb, int ke) {
-    const int32_t W = adj(id, 0), E = adj(id, 1), S = adj(id, 2), N = adj(id, 3);
-    const int32_t par = (id < L.n_stored && !L.parent.empty()) ? L.parent[(size_t)id] : -1;
-    const int32_t m[kW2Meta] = {id, emit | kb << 8 | ke << 16, W, E, S, N, adj(W, 2), adj(W, 3), adj(E, 2), adj(E, 3),
-                                par, 0};
-    s.meta.insert(s.meta.end(), m, m + kW2Meta);
-    s.items += 1;
-    s.steps += ke - kb;
-  };
-  auto push_run = [&](Stream& s, const int32_t* run, int64_t len) {
-    push_item(s, adj(run[0], 4), 0, 5, 8);  // warm-up: planes 5, 6 prime, plane 7 is the run's k-halo
-    for (int64_t q = 0; q < len; ++q) push_item(s, run[q], 1, 0, 8);
-    push_item(s, adj(run[len - 1], 5), 0, 0, 1);  // cool-down: plane 0 is the run's k-halo
-  };
-  const int64_t full = (nch / G) * G;
-  for (int64_t c = 0; c < full; ++c) push_run(st[(size_t)(c % G)], chains[(size_t)c].data(), chains[(size_t)c].size());
-  std::vector<int32_t> rest, rest_chain;
-  for (int64_t c = full; c < nch; ++c)
-    for (int32_t id : chains[(size_t)c]) {
-      rest.push_back(id);
-      rest_chain.push_back((int32_t)c);
-    }
-  const int64_t nr = (int64_t)rest.size();
-  int64_t off = 0;
-  for (int64_t g = 0; g < G && nr > 0; ++g) {
-    const int64_t cnt = nr / G + (g < nr % G ? 1 : 0);
-    for (int64_t m = off; m < off + cnt;) {
-      int64_t e = m + 1;
-      while (e < off + cnt && rest_chain[(size_t)e] == rest_chain[(size_t)m]) ++e;
-      push_run(st[(size_t)g], &rest[(size_t)m], e - m);
-      m = e;
-    }
-    off += cnt;
-  }
-  const int32_t z = (int32_t)L.zero_brick;
-  for (int64_t w = 0; w < G / 2; ++w) {
-    Stream& A = st[(size_t)(2 * w)];
-    Stream& B = st[(size_t)(2 * w + 1)];
-    if (A.steps == 0 && B.steps == 0) continue;
-    for (Stream* s : {&A, &B}) {
-      const int64_t other = s == &A ? B.steps : A.steps;
-      while (s->steps < other) {
-        const int c = (int)std::min<int64_t>(8, other - s->steps);
-        push_item(*s, z, 0, 8 - c, 8);
-      }
-    }
-    const int64_t steps = A.steps, na = A.items, nbi = B.items;
-    if (na > 0xffff || nbi > 0xffff || steps > INT32_MAX) return LevelLayout::PairTable{0};
-    for (Stream* s : {&A, &B})
-      for (int i = 0; i < kW2Tail; ++i) push_item(*s, z, 0, 0, 8);
-    const int64_t oa = (int64_t)t.meta.size() / kW2Meta;
-    t.meta.insert(t.meta.end(), A.meta.begin(), A.meta.end());
-    const int64_t ob = (int64_t)t.meta.size() / kW2Meta;
-    t.meta.insert(t.meta.end(), B.meta.begin(), B.meta.end());
-    if (ob + B.items > INT32_MAX) return LevelLayout::PairTable{0};
-    t.warps.push_back((int32_t)oa);
-    t.warps.push_back((int32_t)ob);
-    t.warps.push_back((int32_t)steps);
-    t.warps.push_back((int32_t)(na | (nbi << 16)));
-  }
-  return t;
-}
-
 void build_pair_tables(LevelLayout& L, int64_t min_bricks, int kind) {
   L.pairs.clear();
   if (L.n_stored < min_bricks) return;
@@ -760,13 +700,13 @@ void build_pair_tables(LevelLayout& L, int64_t min_bricks, int kind) {
     if (dup) continue;
     LevelLayout::PairTable t;
     t.kind = 0;
-    if (kind == 3 || kind == 4) t = pencil_table(L, r[0], r[1], 0, kind);
-    if (t.kind == 0) t = kind == 2 ? warp_table(L, r[0], r[1]) : pair_table(L, r[0], r[1]);
+    if (kind == 3) t = pencil_table(L, r[0], r[1], 0, kind);
+    if (t.kind == 0) t = pair_table(L, r[0], r[1]);
     if (t.kind != 0) L.pairs.push_back(std::move(t));
   }
   // pencil passes over a level with a ghost shell: the units split by whether they read a ghost
   // brick, for the overlap of the exchange with the interior units (both parts or neither)
-  if ((kind == 3 || kind == 4) && L.n_ghost > 0)
+  if (kind == 3 && L.n_ghost > 0)
     for (const int64_t b1 : {L.n_owned, L.n_stored}) {
       bool have = false;
       for (const auto& c : L.pairs) have |= c.kind == kind && c.part == 0 && c.b0 == 0 && c.b1 == b1;

@@ -49,6 +49,7 @@ struct LevelLayout {
   std::vector<Run> sends, recvs;
   int64_t n_recv_slots = 0;     // receive runs before a non-periodic bc drops those across domain faces
   std::vector<int32_t> mirror;  // [n][3] ghost brick, source brick, reflected-axes mask (bc != periodic)
+  std::vector<int32_t> radj;    // [n_owned][8] owned adjacency with domain faces = -1 (one-rank bc != periodic)
   int64_t ext_index(int x, int y, int z) const;  // -1 if not stored
   std::vector<int32_t> ext2idx;  // dense map over the extended box
   // Column plans for the streaming sweep kernel: the bricks of a range [b0,b1)
@@ -67,21 +68,14 @@ struct LevelLayout {
   // cool-down brick (T neighbour of its last): item = (id, flags, W,E,S,N,
   // SW,NW,SE,NE, parent), flags bit0 = "previous item is a range brick", bit1 = warm-up,
   // bit2 = cool-down (the kernel computes only the x1 planes the run needs from those).
-  //
-  // kind 2 (sweep2w.cu): one stream per HALF-WARP, two streams per warp with
-  // equal step counts.  A step is one z-plane; item = (id, emit | kb<<8 | ke<<16,
-  // W,E,S,N, SW,NW,SE,NE, parent, 0) with [kb, ke) the planes the stream steps
-  // through: warm-up [5,8) (planes 5,6 prime the register windows), range bricks
-  // [0,8) (emit = 1), cool-down [0,1).  Streams end with kW2Tail dummy items.
   struct PairTable {
     int kind = 1;
     int64_t b0 = 0, b1 = 0;
     // kind 3 on a level with a ghost shell: 0 = every unit of the range; 1 = the units that read
     // no ghost brick (swept while the exchange fills the ghosts), 2 = the others (after it)
     int part = 0;
-    std::vector<int32_t> meta;   // [items][kPairMeta] (kind 1) / [items][kW2Meta] (kind 2)
-    std::vector<int32_t> ctas;   // kind 1: [nctas][2] offset (items), count
-    std::vector<int32_t> warps;  // kind 2: [nwarps][4] first item of half 0, of half 1, steps, items0 | items1<<16
+    std::vector<int32_t> meta;   // [items][kPairMeta] (kind 1) / [chunks][kPenRec] (kind 3)
+    std::vector<int32_t> ctas;   // [nctas][2] offset (items / chunks), count
   };
   std::vector<PairTable> pairs;
 };
@@ -110,14 +104,7 @@ constexpr int kPenMeta = 20;  // host-side tile-layer item: the 16 ids, parent, 
 constexpr int kPenRec = 20;   // chunk record (80 bytes: one 1D bulk copy)
 constexpr int kPenCtasPerSm = 6;                    // resident pencil CTAs per SM (shared-memory bound)
 constexpr int64_t kPenCtas = 148 * kPenCtasPerSm;
-// kind 4 (sweep2q.cu): the same chunk records for one-warp CTAs
-constexpr int kQuadCtasPerSm = 8;                   // resident one-warp pencil CTAs per SM (27.5 KB each)
-constexpr int64_t kQuadCtas = 148 * kQuadCtasPerSm;
-constexpr int kW2Meta = 12;
-constexpr int kW2WarpsPerSm = 7;                    // resident one-warp CTAs per SM (shared-memory bound)
-constexpr int64_t kW2Streams = 148 * kW2WarpsPerSm * 2;
-constexpr int kW2Tail = 9;                          // trailing dummy items per stream (lookahead + meta prefetch)
-// kind 1: CTA item streams (sweep2.cu), kind 2: half-warp plane streams (sweep2w.cu), kind 3: 2x2-brick
+// kind 1: CTA item streams (sweep2.cu), kind 3: 2x2-brick
 // pencil chunk streams (sweep2p.cu) for the owned range where the level tiles into aligned 2x2 pencils
 // (other ranges, and levels that do not tile, get kind 1)
 void build_pair_tables(LevelLayout& L, int64_t min_bricks, int kind);

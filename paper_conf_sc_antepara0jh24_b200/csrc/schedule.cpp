@@ -40,13 +40,13 @@ bool Builder::has_pair_table(int l, int64_t b0, int64_t b1) const {
 
 bool Builder::pencil_table(int l) const {
   for (const auto& pt : lay.lv[l].pairs)
-    if (pt.b0 == 0 && pt.b1 == lay.lv[l].n_owned && pt.part == 0) return pt.kind == 3 || pt.kind == 4;
+    if (pt.b0 == 0 && pt.b1 == lay.lv[l].n_owned && pt.part == 0) return pt.kind == 3;
   return false;
 }
 
 bool Builder::pair_zero_ok(int l) const {
   for (const auto& pt : lay.lv[l].pairs)
-    if (pt.b0 == 0 && pt.b1 == lay.lv[l].n_owned && pt.part == 0) return pt.kind == 3 || pt.kind == 4;
+    if (pt.b0 == 0 && pt.b1 == lay.lv[l].n_owned && pt.part == 0) return pt.kind == 3;
   return false;
 }
 
@@ -54,7 +54,7 @@ bool Builder::pencil_ghosts(int l) const {
   const LevelLayout& L = lay.lv[l];
   if (L.n_ghost == 0) return false;
   for (const auto& pt : L.pairs)
-    if (pt.b0 == 0 && pt.b1 == L.n_stored && pt.part == 0) return pt.kind == 3 || pt.kind == 4;
+    if (pt.b0 == 0 && pt.b1 == L.n_stored && pt.part == 0) return pt.kind == 3;
   return false;
 }
 
@@ -243,7 +243,9 @@ void Builder::bottom(int l, int n, bool zero) {
   }
   const LevelLayout& L = lay.lv[l];
   const int bm = lay.p.bottom_mode;
-  const bool can_res = !ghosts(l) && L.n_stored <= kResidentMaxBricks;
+  // (a one-rank non-periodic level: the owned bricks with the domain faces as images, L.radj)
+  const bool can_res = (!ghosts(l) && L.n_stored <= kResidentMaxBricks) ||
+                       (!L.radj.empty() && L.n_owned <= kResidentMaxBricks);
   const bool res = can_res && (bm == MG_BOTTOM_RESIDENT ||
                                 ((bm == MG_BOTTOM_AUTO || bm == MG_BOTTOM_CLUSTER || bm == MG_BOTTOM_GRID) && fusion(l) != MG_FUSION_PAPER));
   const bool fold_zero = zero && fusion(l) == MG_FUSION_FULL;

@@ -377,7 +377,7 @@ def test_full_size_512_sweep_sampled(oracle_mod):
 
 def test_full_size_512_pencil_pass_bitwise(oracle_mod):
     """512^3 (the bench workload, launch configuration of bench.py: the 2x2-brick pencil pass over
-    592 CTAs): one two-sweep pass with r, every point against the oracle's two sweeps."""
+    888 CTAs, 6 per SM): one two-sweep pass with r, every point against the oracle's two sweeps."""
     mg, _ = _mg()
     shape = (512, 512, 512)
     m = new(shape, 6)
@@ -488,12 +488,12 @@ def test_config5_1024_decomposition_invariant(pg):
 
 
 # ------------------------------------------------- streaming (column) kernel
-@pytest.mark.parametrize("tb", [0, 1, 2, 3, 4])
+@pytest.mark.parametrize("tb", [0, 1, 3])
 @pytest.mark.parametrize("fusion", [2, 3])
 @pytest.mark.parametrize("ghost_mode,period", [(0, 0), (1, 1), (1, 3), (1, 8)])
 def test_streaming_kernel_forced_bitwise(oracle_mod, fusion, ghost_mode, period, tb):
     """sweep_kernel = 2 forces the TMA-streamed column kernel (tb = 0) or a two-sweep
-    kernel (tb = 1: CTA streams, tb = 2: warp plane streams, tb = 3: 2x2-brick pencils) on every level (plain, +r and +restriction variants; owned,
+    kernel (tb = 1: CTA streams, tb = 3: 2x2-brick pencils) on every level (plain, +r and +restriction variants; owned,
     owned+ghost, interior and surface ranges)."""
     shape = (64, 32, 96)
     b = mg_inputs.random_rhs(shape, 13)
@@ -506,7 +506,7 @@ def test_streaming_kernel_forced_bitwise(oracle_mod, fusion, ghost_mode, period,
     m.close()
 
 
-@pytest.mark.parametrize("tb", [0, 1, 2, 3, 4])
+@pytest.mark.parametrize("tb", [0, 1, 3])
 @pytest.mark.parametrize("pg", [(2, 2, 2), (2, 1, 1)])
 def test_streaming_kernel_loopback_bitwise(oracle_mod, pg, tb):
     _, solver = _mg()
@@ -538,7 +538,7 @@ def test_vcycle_config2_256_bitwise(oracle_mod):
 
 
 # ------------------------------------------------- two sweeps per pass (temporal blocking)
-@pytest.mark.parametrize("tb", [1, 2, 3, 4])
+@pytest.mark.parametrize("tb", [1, 3])
 @pytest.mark.parametrize("n", [2, 3, 5])
 @pytest.mark.parametrize("shape,ghost_mode", [((64, 32, 96), 0), ((32, 48, 64), 1), ((40, 24, 56), 0)])
 def test_two_sweep_pass_per_op(oracle_mod, n, shape, ghost_mode, tb):
@@ -563,9 +563,9 @@ def test_two_sweep_pass_per_op(oracle_mod, n, shape, ghost_mode, tb):
 @pytest.mark.parametrize("n", [2, 3, 4])
 @pytest.mark.parametrize("shape,ghost_mode", [((16, 64, 64), 0), ((24, 64, 96), 0), ((96, 64, 128), 0),
                                               ((32, 64, 64), 0), ((64, 48, 32), 1), ((8, 16, 16), 0)])
-@pytest.mark.parametrize("tb", [3, 4])
+@pytest.mark.parametrize("tb", [3])
 def test_pencil_pass_work_splits(oracle_mod, n, shape, ghost_mode, tb):
-    """tb = 3 / 4 (2x2-brick pencil chunk streams, two-warp / one-warp CTAs): whole tile columns per CTA, several columns per CTA,
+    """tb = 3 (2x2-brick pencil chunk streams): whole tile columns per CTA, several columns per CTA,
     columns cut into pieces across CTAs, a ghost-shell level and a single-layer level all give the
     oracle's bits for x and r (n sweeps: n // 2 pencil passes plus a single sweep if n is odd)."""
     mg, _ = _mg()
@@ -605,7 +605,7 @@ def test_vcycle_512_grid_coarse_bitwise(oracle_mod):
     assert out[0][1] == out[1][1]
 
 
-@pytest.mark.parametrize("tb", [0, 1, 2, 3, 4])
+@pytest.mark.parametrize("tb", [0, 1, 3])
 def test_temporal_blocking_on_off_bitwise(oracle_mod, tb):
     """The V-cycle with and without temporal blocking gives the oracle's bits (256^3, L = 6,
     where levels 0 and 1 stream; 12/12/100)."""
@@ -717,12 +717,11 @@ def test_programmatic_dependent_launch_on_off_bitwise(oracle_mod, launch_pdl, us
 
 
 # ------------------------------------------------- Chebyshev smoother variant (N4, reading A19)
-@pytest.mark.parametrize("kw", [dict(), dict(temporal_blocking=0), dict(fusion=1), dict(temporal_blocking=2),
+@pytest.mark.parametrize("kw", [dict(), dict(temporal_blocking=0), dict(fusion=1), dict(temporal_blocking=1),
                                 dict(bottom_mode=1), dict(bottom_mode=3), dict(bottom_mode=4),
                                 dict(ghost_mode=1, ca_period=4),
                                 dict(sweep_kernel=2), dict(cheby_ratio=10), dict(temporal_blocking=3),
-                                dict(temporal_blocking=3, sweep_kernel=2), dict(temporal_blocking=4),
-                                dict(temporal_blocking=4, sweep_kernel=2)])
+                                dict(temporal_blocking=3, sweep_kernel=2), dict(temporal_blocking=1, sweep_kernel=2)])
 def test_chebyshev_smoother_vcycle_bitwise(oracle_mod, kw):
     """smoother = 1: per-sweep Chebyshev steps in every kernel that sweeps (single, two-sweep
     passes, paper kernel set, cluster coarse solve, ghost sweeps), bit for bit with the oracle's
@@ -768,10 +767,9 @@ def test_chebyshev_smoother_loopback_bitwise(oracle_mod):
 
 # ------------------------------------------------- red-black Gauss-Seidel variant (N4, reading A20)
 @pytest.mark.parametrize("kw", [dict(), dict(temporal_blocking=0), dict(fusion=1), dict(fusion=2),
-                                dict(temporal_blocking=2), dict(bottom_mode=1), dict(ghost_mode=1, ca_period=3),
+                                dict(temporal_blocking=1), dict(bottom_mode=1), dict(ghost_mode=1, ca_period=3),
                                 dict(ghost_mode=1, ca_period=8), dict(sweep_kernel=2), dict(temporal_blocking=3),
-                                dict(temporal_blocking=3, sweep_kernel=2), dict(temporal_blocking=4),
-                                dict(temporal_blocking=4, sweep_kernel=2)])
+                                dict(temporal_blocking=3, sweep_kernel=2), dict(temporal_blocking=1, sweep_kernel=2)])
 def test_gsrb_smoother_vcycle_bitwise(oracle_mod, kw):
     """smoother = 2: every pre / post sweep is a red then a black half-sweep (step h^2/6) in the
     single-sweep, two-sweep (red + black in one pass), paper-set and ghost-shell schedules; bit

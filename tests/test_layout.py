@@ -261,13 +261,12 @@ W_, E_, S_, N_, B_, T_ = range(6)
 @pytest.mark.parametrize("n_local,pg,L,gm", [((128, 128, 128), (1, 1, 1), 3, 0), ((256, 128, 64), (1, 1, 1), 2, 0),
                                             ((128, 128, 128), (1, 1, 1), 2, 1), ((128, 128, 128), (2, 1, 1), 2, 0),
                                             ((512, 512, 512), (1, 1, 1), 2, 0)])
-@pytest.mark.parametrize("tb", [3, 4])
+@pytest.mark.parametrize("tb", [3])
 def test_pencil_plan_covers_owned_bricks(n_local, pg, L, gm, tb):
     """Every owned brick is swept exactly once per half by the pencil chunk streams; each record's
     16 ids are the tile layer's bricks and neighbours by the adjacency table; tiles sit on even
     brick coordinates (one coarse brick's x-y octants 0-3); runs are [warm-up, layers linked by T,
-    cool-down] with the B / T neighbour layers; every CTA gets the same work to within a run.
-    tb = 3: two-warp CTAs (sweep2p.cu), tb = 4: the same records for one-warp CTAs (sweep2q.cu)."""
+    cool-down] with the B / T neighbour layers; every CTA gets the same work to within a run."""
     p, lays = layouts(n_local, pg, L, gm, temporal_blocking=tb)
     lay = lays[0]
     inf = lay.info(0)

@@ -30,8 +30,8 @@ B_PER_PT = [
     ("interp_kernel", "interpolation+increment", 17.0),
     ("sweep_kernel<1, 0>", "applyOp (paper kernel set)", 16.0),
     ("sweep_kernel<2, 0>", "maxNormRes", 16.0),
-    ("smooth_kernel<true>", "smooth+residual (paper kernel set)", 40.0),
-    ("smooth_kernel<false>", "smooth (paper kernel set)", 32.0),
+    ("smooth_kernel<1>", "smooth+residual (paper kernel set)", 40.0),
+    ("smooth_kernel<0>", "smooth (paper kernel set)", 32.0),
     ("restrict_kernel", "restriction", 9.0),
     ("zero_kernel", "initZero (per coarse point: 8 B)", 1.0),
 ]

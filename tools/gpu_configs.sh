@@ -6,6 +6,4 @@ mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1 || { tail -20 gpurun_out/build.log; exit 1; }
 timeout 1500 python tools/config_sweep.py --out gpurun_out/configs.json ${SWEEP_ARGS} > gpurun_out/configs.log 2>&1; echo "sweep rc=$?"
 tail -3 gpurun_out/configs.log
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:sweep2w -s 2 -c 1 \
-   -o gpurun_out/prof_sweep2w -f python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-e2e --tb 2 > gpurun_out/ncu_w.log 2>&1
 echo "ncu rc=$?"

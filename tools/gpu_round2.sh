@@ -1,7 +1,7 @@
 #!/bin/bash
 # One gpurun call (round 2 iteration): build, smoke, GPU tests, bench (default and A/B variants),
 # the launch list and one ncu --set full capture of the level-0 pass kernel.
-#   BENCH_AB="--tb 3;--tb 4 --bottom-mode 4"   extra bench variants (';'-separated), short runs
+#   BENCH_AB="--tb 3;--tb 1 --bottom-mode 4"   extra bench variants (';'-separated), short runs
 #   NCU_KERNEL=sweep2q_kernel                   regex of the kernel to capture (empty: skip)
 #   PYTEST_ARGS="-x -q"                         GPU test selection (PYTEST=0: skip)
 cd "${GRAFT_REPO_ROOT:-/root/repo}"
