@@ -274,6 +274,12 @@ static void build_parents(LevelLayout& F, const LevelLayout& C) {
   }
 }
 
+// smallest level with two-sweep passes under the auto kernel choice (MG_PAIR_MIN_BRICKS: A/B runs only)
+static int64_t pair_min_bricks() {
+  static const int64_t v = getenv("MG_PAIR_MIN_BRICKS") ? atoll(getenv("MG_PAIR_MIN_BRICKS")) : kPairMinBricks;
+  return v;
+}
+
 mg_status build_layout(const mg_params& p, int rank, int world, Layout& out, std::string& msg) {
   char buf[256];
   if (world < 1 || rank < 0 || rank >= world) {
@@ -352,7 +358,7 @@ mg_status build_layout(const mg_params& p, int rank, int world, Layout& out, std
   for (int l = 0; l + 1 < out.L; ++l) build_parents(out.lv[l], out.lv[l + 1]);
   if (p.temporal_blocking != 0)
     for (int l = 0; l < out.L; ++l)
-      build_pair_tables(out.lv[l], p.sweep_kernel == 0 ? kPairMinBricks : min_b,
+      build_pair_tables(out.lv[l], p.sweep_kernel == 0 ? pair_min_bricks() : min_b,
                         p.temporal_blocking == 3 ? 3 : 1);
   // replicated bottom: the global coarsest level as one rank would store it
   const LevelLayout& B = out.lv[(size_t)out.L - 1];

@@ -340,3 +340,31 @@ def test_brick4_solve_matches_oracle(oracle_mod):
     st, c_g, fin = m.solve(1e-10, 20)
     assert st == 0 and c_g == c_o and fin == norms[-1] and fin < 1e-10
     m.close()
+
+
+# ------------------------------------------------------------ the variants at the bench size
+@pytest.mark.parametrize("variant", ["dirichlet", "varcoef_neumann", "brick4"])
+def test_full_size_512_variant_vcycle_bitwise(oracle_mod, variant):
+    """512^3, L = 6, 12/12/100 (the bench workload, its launch configuration): one V-cycle of each
+    variant -- Dirichlet (pencil passes over the ghost-shell plan, mirror exchanges, the resident
+    bottom with domain faces), variable coefficients with Neumann faces (one-brick kernels), 4^3
+    bricks (generic kernels) -- bitwise equal to the oracle's, x and the norm (the column-kernel
+    norm for the 8^3 cases)."""
+    import gc
+    shape = (512, 512, 512)
+    bc = {"dirichlet": 1, "varcoef_neumann": 2, "brick4": 0}[variant]
+    vc = variant == "varcoef_neumann"
+    b = mg_inputs.dirichlet_sin_rhs(shape) if bc == 1 else mg_inputs.sin_rhs(shape)
+    c = mg_inputs.smooth_coef(shape) if vc else None
+    xs, ns = oracle_cycles(oracle_mod, b, 6, 1, bc=bc, coef=c)
+    gc.collect()
+    m = new(shape, 6, bc=bc, var_coef=int(vc), brick_edge=4 if variant == "brick4" else 0)
+    if vc:
+        m.set_coefficients(dev(c))
+    m.set_rhs(dev(b))
+    m.set_solution(None)
+    check_cycles(m, xs, ns)
+    m.close()
+    del m, xs
+    gc.collect()
+    torch.cuda.empty_cache()

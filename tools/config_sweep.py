@@ -23,8 +23,11 @@ from paper_conf_sc_antepara0jh24_b200.solver import Multigrid  # noqa: E402
 
 def run(tag, n, levels, cycles=5, solve=False, **kw):
     shape = (n, n, n)
-    b = torch.from_numpy(mg_inputs.sin_rhs(shape)).cuda()
+    bsrc = mg_inputs.dirichlet_sin_rhs(shape) if kw.get("bc") == 1 else mg_inputs.sin_rhs(shape)
+    b = torch.from_numpy(bsrc).cuda()
     m = Multigrid(shape, num_levels=levels, **kw)
+    if kw.get("var_coef"):
+        m.set_coefficients(torch.from_numpy(mg_inputs.smooth_coef(shape)).cuda())
     m.set_rhs(b)
     m.set_solution(None)
     rec = {"tag": tag, "n": n, "levels": levels, **{k: v for k, v in kw.items() if not isinstance(v, list)}}
@@ -81,10 +84,18 @@ def main():
         out.append(run("c1", 64, 4, solve=True, fusion=[fu] * 16))
     out.append(run("c1", 64, 4, solve=True, smoother=1))
     out.append(run("c1", 64, 4, solve=True, smoother=2))
+    # the N4 variants: Dirichlet / Neumann boundaries, variable coefficients, 4^3 bricks
+    out.append(run("c1", 64, 4, solve=True, bc=1))
+    out.append(run("c1", 64, 4, solve=True, bc=2))
+    out.append(run("c1", 64, 4, solve=True, var_coef=1, bc=1))
+    out.append(run("c1", 64, 4, solve=True, brick_edge=4))
     # config 2: 256^3, L = 6; paper kernel set / fused / fused + temporal blocking
     out.append(run("c2", 256, 6, fusion=[1] * 16, temporal_blocking=0))
     out.append(run("c2", 256, 6, fusion=[3] * 16, temporal_blocking=0))
     out.append(run("c2", 256, 6))
+    out.append(run("c2", 256, 6, bc=1))
+    out.append(run("c2", 256, 6, var_coef=1))
+    out.append(run("c2", 256, 6, brick_edge=4))
     # sizes for the fits: paper kernel set (every op separate) and the default, n = 32 .. 512
     for n in (32, 64, 128, 256, 512):
         lv = max(1, min(6, n.bit_length() - 4))

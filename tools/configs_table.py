@@ -13,6 +13,8 @@ def desc(r):
     fu = r.get("fusion", [0])[0]
     parts.append({0: "fusion auto(full)", 1: "paper kernel set", 2: "fused sweep", 3: "full fusion"}[fu])
     tb = r.get("temporal_blocking", 3) if fu != 1 else 0
+    if r.get("var_coef") or r.get("brick_edge") == 4:
+        tb = 0  # (the one-brick kernel family)
     parts.append({0: "1 sweep/pass", 1: "2 sweeps/pass (one-brick CTA streams)", 2: "2 sweeps/pass (warp streams)",
                   3: "2 sweeps/pass (2x2-brick pencils)"}[tb])
     if r.get("ghost_mode"):
@@ -23,6 +25,12 @@ def desc(r):
         parts.append({1: "Chebyshev smoother", 2: "red-black Gauss-Seidel smoother"}[r["smoother"]])
     if r.get("bottom_solver") == 1:
         parts.append("CG bottom")
+    if r.get("bc"):
+        parts.append({1: "Dirichlet", 2: "Neumann"}[r["bc"]])
+    if r.get("var_coef"):
+        parts.append("variable coefficients")
+    if r.get("brick_edge") == 4:
+        parts.append("4^3 bricks")
     return ", ".join(parts)
 
 

@@ -7,7 +7,8 @@ mkdir -p gpurun_out/sanitize
 python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
 CS=/usr/local/cuda/bin/compute-sanitizer
 for tool in memcheck racecheck synccheck; do
-  for cfg in "64 4 0 3 0" "128 5 0 3 0" "64 3 2 3 0" "128 4 2 3 0" "64 3 2 1 0" "64 3 2 0 0" "64 3 0 3 1"; do
+  IFS=';' read -ra LIST <<< "${CFGS:-64 4 0 3 0;128 5 0 3 0;64 3 2 3 0;128 4 2 3 0;64 3 2 1 0;64 3 2 0 0;64 3 0 3 1}"
+  for cfg in "${LIST[@]}"; do
     tag=$(echo $tool $cfg | tr ' ' '_')
     timeout 900 $CS --tool $tool --print-limit 20 python tools/sanitize_run.py $cfg \
        > gpurun_out/sanitize/$tag.log 2>&1
