@@ -78,6 +78,7 @@ struct PairArgs {
                         // kind 3: [chunks][20] chunk records (mg_internal.h kPenRec)
   const int2* ctas;     // (first item / chunk, count) per CTA
   int64_t nctas;
+  unsigned long long* trace = nullptr;  // sweep2p measurement (MG_PEN_TRACE): per CTA (start, end) globaltimer
 };
 struct PairMaps {
   CUtensorMap xwe;   // x boxes {2,8,8}: W (i=6,7) / E (i=0,1) face slabs

@@ -30,7 +30,11 @@
 // re-reads, no x1 round trip for own cells, a 25% instead of 50% redundant ring).
 #include <cudaTypedefs.h>
 
+#include <algorithm>
+#include <cstdio>
+#include <cstdlib>
 #include <type_traits>
+#include <vector>
 
 #include "kernels.h"
 #include "mg_internal.h"
@@ -92,12 +96,22 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
   int* const MR = reinterpret_cast<int*>(BAR + 2);  // [MRS][kPenRec] chunk records, 16-byte aligned slots
   const int col1 = COLOUR ? p.colour : -1, col2 = COLOUR ? p.colour2 : -1;
   const int t = threadIdx.x, w = t >> 5, l = t & 31;
+  if (pa.trace && threadIdx.x == 0) {  // (MG_PEN_TRACE measurement runs only)
+    unsigned long long t0;
+    unsigned sm;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t0));
+    asm volatile("mov.u32 %0, %smid;" : "=r"(sm));
+    pa.trace[2 * blockIdx.x] = t0;
+    pa.trace[2 * 65536 + blockIdx.x] = sm | ((unsigned long long)pa.ctas[blockIdx.x].y << 32);
+  }
   const int2 cr = pa.ctas[blockIdx.x];
   const int32_t* REC = pa.meta + (int64_t)cr.x * kPenRec;  // chunk records: code, 16 brick ids, parent
   const int cnt = cr.y;
   const double alpha = p.c.alpha, beta = p.c.beta, gamma = p.c.gamma, gamma2 = p.gamma2;
   // L2 policies (evict_normal for x0, b or x2 measured no different: DESIGN.md §7.1)
-  const uint64_t pol_keep = l2_evict_last(), pol_stream = l2_evict_first();
+  // (created at each use -- one ALU op -- rather than held: two 64-bit values fewer live in registers)
+#define pol_keep l2_evict_last()
+#define pol_stream l2_evict_first()
 
   // ---- own-cell role: cells (2p + a, 8w + 2jp + r) of the tile ----
   const int pc = l & 7, jp = l >> 3, bx = pc >> 2, ib = 2 * (pc & 3), jb = 2 * jp, q = bx + 2 * w;
@@ -385,7 +399,17 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
       step(c, I0{}, P1{}, false, true);
     }
   }
+  if (pa.trace) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      unsigned long long t1;
+      asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t1));
+      pa.trace[2 * blockIdx.x + 1] = t1;
+    }
+  }
   pdl_trigger();
+#undef pol_keep
+#undef pol_stream
 }
 
 bool pencil_supports(unsigned flags) {
@@ -409,9 +433,58 @@ cudaError_t encode_pencil_maps(const double* x, const double* b, int64_t n_alloc
   X(SW_ZERO_X) X(SW_ZERO_X | SW_WRITE_R) X(SW_ZERO_X | SW_RESTRICT) X(SW_ZERO_X | SW_COLOUR)             \
   X(SW_ZERO_X | SW_WRITE_R | SW_COLOUR) X(SW_ZERO_X | SW_RESTRICT | SW_COLOUR)
 
-cudaError_t launch_sweep2p(const SweepArgs& a, const PairArgs& pa, const PairMaps& pm, unsigned flags,
+// MG_PEN_TRACE=1 (measurement runs without graph capture only): every pencil pass records each CTA's
+// (start, end) globaltimer and prints the spread of the CTAs' end times -- the pass's tail
+static cudaError_t trace_report(const PairArgs& pa, cudaStream_t s) {
+  cudaError_t e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) return e;
+  std::vector<unsigned long long> h((size_t)pa.nctas * 2);
+  e = cudaMemcpy(h.data(), pa.trace, h.size() * 8, cudaMemcpyDeviceToHost);
+  if (e != cudaSuccess) return e;
+  unsigned long long s0 = ~0ull, s1 = 0, e0 = ~0ull, e1 = 0;
+  std::vector<double> ends;
+  for (int64_t g = 0; g < pa.nctas; ++g) {
+    s0 = std::min(s0, h[2 * g]), s1 = std::max(s1, h[2 * g]);
+    e0 = std::min(e0, h[2 * g + 1]), e1 = std::max(e1, h[2 * g + 1]);
+  }
+  for (int64_t g = 0; g < pa.nctas; ++g) ends.push_back((double)(h[2 * g + 1] - s0) / 1e3);
+  std::sort(ends.begin(), ends.end());
+  auto pct = [&](double q) { return ends[(size_t)std::min<double>(ends.size() - 1, q * ends.size())]; };
+  fprintf(stderr,
+          "MG_PEN_TRACE ctas=%lld start spread %.1f us; end: first %.1f, p10 %.1f, p50 %.1f, p90 %.1f, last %.1f us\n",
+          (long long)pa.nctas, (s1 - s0) / 1e3, (e0 - s0) / 1e3, pct(0.1), pct(0.5), pct(0.9), (e1 - s0) / 1e3);
+  // per CTA: end time vs chunk count and SM (is the tail static imbalance or run-time variation?)
+  static const bool dump = getenv("MG_PEN_TRACE_DUMP") != nullptr;
+  std::vector<unsigned long long> info((size_t)pa.nctas);
+  e = cudaMemcpy(info.data(), pa.trace + 2 * 65536, info.size() * 8, cudaMemcpyDeviceToHost);
+  if (e != cudaSuccess) return e;
+  std::vector<double> sm_end(256, 0.0);
+  std::vector<int> sm_n(256, 0);
+  double c_lo = 1e30, c_hi = 0;
+  for (int64_t g = 0; g < pa.nctas; ++g) {
+    const unsigned sm = (unsigned)(info[g] & 0xffffffffu), cnt = (unsigned)(info[g] >> 32);
+    const double end = (double)(h[2 * g + 1] - s0) / 1e3;
+    if (sm < 256) sm_end[sm] = std::max(sm_end[sm], end), sm_n[sm]++;
+    c_lo = std::min(c_lo, (double)cnt), c_hi = std::max(c_hi, (double)cnt);
+    if (dump) fprintf(stderr, "  cta %lld sm %u chunks %u end %.1f\n", (long long)g, sm, cnt, end);
+  }
+  double mn = 1e30, mx = 0;
+  for (int q = 0; q < 256; ++q)
+    if (sm_n[q]) mn = std::min(mn, sm_end[q]), mx = std::max(mx, sm_end[q]);
+  fprintf(stderr, "MG_PEN_TRACE   chunks per CTA %.0f..%.0f; per-SM last end %.1f..%.1f us\n", c_lo, c_hi, mn, mx);
+  return cudaSuccess;
+}
+
+cudaError_t launch_sweep2p(const SweepArgs& a, const PairArgs& pa_in, const PairMaps& pm, unsigned flags,
                            cudaStream_t s) {
-  if (pa.nctas <= 0) return cudaSuccess;
+  if (pa_in.nctas <= 0) return cudaSuccess;
+  static const bool trace = getenv("MG_PEN_TRACE") != nullptr;
+  static unsigned long long* tbuf = nullptr;
+  PairArgs pa = pa_in;
+  if (trace) {
+    if (!tbuf && cudaMalloc(&tbuf, 3 * 8 * 65536) != cudaSuccess) return cudaErrorMemoryAllocation;
+    pa.trace = tbuf;
+  }
   const unsigned g = (unsigned)pa.nctas;
   const size_t sm = SMEM_BYTES;
   const unsigned col = (a.colour >= 0 || a.colour2 >= 0) ? SW_COLOUR : 0u;
@@ -425,6 +498,7 @@ cudaError_t launch_sweep2p(const SweepArgs& a, const PairArgs& pa, const PairMap
     default:
       return cudaErrorInvalidValue;
   }
+  if (trace) return trace_report(pa, s);
   return cudaGetLastError();
 }
 

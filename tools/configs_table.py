@@ -59,10 +59,12 @@ def main():
         out.append("")
     # per level x op split of the config-2 / c3_fusion default runs (instrumented cycle)
     for tag in ("c2", "c3_fusion", "c5"):
-        rr = [r for r in runs if r["tag"] == tag and "fusion" not in r and not r.get("ghost_mode")]
+        variant = ("fusion", "ghost_mode", "smoother", "bottom_solver", "bc", "var_coef", "brick_edge",
+                   "temporal_blocking", "pre", "solve")
+        rr = [r for r in runs if r["tag"] == tag and not any(r.get(k) for k in variant)]
         if not rr:
             continue
-        r = rr[-1]
+        r = rr[0]
         out += [f"### Per level x op, `{tag}` {r['n']}^3 default (instrumented cycle, ms)", "",
                 "| level | n | " + " | ".join(OPS) + " | total | share |", "|---" * (len(OPS) + 4) + "|"]
         tot = sum(sum(v) for v in r["level_op_ms"])
