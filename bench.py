@@ -39,7 +39,8 @@ def parse():
     ap.add_argument("--steps", type=int, default=30)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--n", type=int, default=512, help="cells per GPU per axis")
+    ap.add_argument("--n", "--size", dest="n", type=int, default=512,
+                    help="cells per GPU per axis (--size under torchrun: '--n' is ambiguous to its parser)")
     ap.add_argument("--levels", type=int, default=6)
     ap.add_argument("--pre", type=int, default=12)
     ap.add_argument("--post", type=int, default=12)
@@ -323,10 +324,19 @@ def main():
 
     if world != a.gpus:
         a.gpus = world if world > 1 else a.gpus
+    # MG_BENCH_SHARED_GPU=1 (rehearsal of the multi-rank path on a one-GPU box, not a measurement):
+    # ranks share the visible GPUs round-robin, torch.distributed runs on gloo (the library exchanges
+    # ghosts over peer memory, which CUDA IPC allows between processes on one device)
+    shared = os.environ.get("MG_BENCH_SHARED_GPU") == "1"
+    if shared:
+        local = local % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if shared:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
     pg = PROC_GRIDS[world]
     n = a.n
     m = Multigrid((n, n, n), pg, a.levels, a.pre, a.post, a.bottom, ca_period=a.ca_period, fusion=a.fusion,
@@ -356,7 +366,7 @@ def main():
 
     def max_over_ranks(v):
         if world > 1:
-            t = torch.tensor([v], dtype=torch.float64, device=dev)
+            t = torch.tensor([v], dtype=torch.float64, device="cpu" if shared else dev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             return float(t.item())
         return v

@@ -842,7 +842,8 @@ def test_exchange_plan_and_timing_keep_the_bits(oracle_mod, transport):
     m.close()
 
 
-@pytest.mark.parametrize("args", ["32 32 32 2 1 1 3 2 0", "16 16 16 2 2 1 2 2 0", "32 32 32 2 1 1 3 1 1"])
+@pytest.mark.parametrize("args", ["32 32 32 2 1 1 3 2 0", "16 16 16 2 2 1 2 2 0", "32 32 32 2 1 1 3 1 1",
+                                  "16 16 16 2 2 2 2 2 0", "32 32 32 2 1 1 3 2 0 1", "16 16 32 2 2 2 2 2 1 2"])
 def test_peer_transport_multiprocess_bitwise(args):
     """The peer-memory transport between PROCESSES (CUDA IPC mappings, device-side ready/done flags, the
     norm's max and the replicated bottom's gather over peer memory): torchrun starts one process per
