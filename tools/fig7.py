@@ -34,6 +34,22 @@ B_PER_PT = [
     ("smooth_kernel<0>", "smooth (paper kernel set)", 32.0),
     ("restrict_kernel", "restriction", 9.0),
     ("zero_kernel", "initZero (per coarse point: 8 B)", 1.0),
+    # the N4 variants' level-0 kernels (one-brick family): variable coefficients read c too (32 B/pt);
+    # 4^3 bricks (generic.cu) move the paper's bytes
+    ("sweep_kernel<0, 64>", "fused sweep, variable coefficients (one-brick)", 32.0),
+    ("sweep_kernel<0, 65>", "fused sweep + r, variable coefficients (one-brick)", 40.0),
+    ("sweep_kernel<0, 66>", "fused sweep + restriction, variable coefficients (one-brick)", 33.0),
+    ("sweep_kernel<0, 68>", "interpolation + fused sweep, variable coefficients (one-brick)", 33.0),
+    ("sweep_kernel<2, 64>", "maxNormRes, variable coefficients", 24.0),
+    ("sweep_kernel<0, 0>", "fused sweep (one-brick)", 24.0),
+    ("sweep_kernel<0, 2>", "fused sweep + restriction (one-brick)", 25.0),
+    ("sweep_kernel<0, 4>", "interpolation + fused sweep (one-brick)", 25.0),
+    ("sweep_col_kernel<128>", "maxNormRes (TMA column kernel)", 16.0),
+    ("<unnamed>::gsweep_kernel<4, 0, 0>", "fused sweep, 4^3 bricks", 24.0),
+    ("<unnamed>::gsweep_kernel<4, 0, 2>", "fused sweep + restriction, 4^3 bricks", 25.0),
+    ("<unnamed>::gsweep_kernel<4, 0, 4>", "interpolation + fused sweep, 4^3 bricks", 25.0),
+    ("<unnamed>::gsweep_kernel<4, 2, 0>", "maxNormRes, 4^3 bricks", 16.0),
+    ("mirror_kernel", "mirror exchange (Dirichlet / Neumann faces)", 0.0),
 ]
 
 
@@ -76,6 +92,8 @@ def main():
         if op is None or "us" not in d or "dram" not in d:
             continue
         alg = b * pts
+        if alg == 0.0:
+            continue
         if op.startswith("initZero"):
             alg = 8.0 * pts / 8.0  # x of level 1 = one eighth of the fine points, 8 B each
         # level-0 launches only: their DRAM traffic is within a factor 2 of the algorithmic bytes
