@@ -57,9 +57,13 @@ __device__ __forceinline__ int coarse_off(int oct, int i, int j, int k) {
 // ---------------------------------------------------------------------------
 enum { MODE_SWEEP = 0, MODE_APPLY = 1, MODE_NORM = 2 };
 
-template <int MODE, unsigned FLAGS>
-__global__ void __launch_bounds__(256) sweep_kernel(SweepArgs p, unsigned long long* acc) {
+// NT threads per CTA (256: two cells per thread; 128: four, in two cell pairs t and t + 128 -- twice
+// the bricks in flight per SM for the same thread count, for the large ranges where the kernel's
+// dependent load chain (adjacency -> halos) is the limit)
+template <int MODE, unsigned FLAGS, int NT = 256>
+__global__ void __launch_bounds__(NT) sweep_kernel(SweepArgs p, unsigned long long* acc) {
   pdl_begin();
+  constexpr int HP = 256 / NT;  // cell pairs per thread
   constexpr bool WRITE_R = (FLAGS & SW_WRITE_R) != 0;
   constexpr bool RESTRICT = (FLAGS & SW_RESTRICT) != 0;
   constexpr bool INTERP = (FLAGS & SW_INTERP) != 0;
@@ -74,29 +78,35 @@ __global__ void __launch_bounds__(256) sweep_kernel(SweepArgs p, unsigned long l
 
   const int t = threadIdx.x;
   const int64_t brick = p.brick0 + blockIdx.x;
-  const int i0 = 2 * (t & 3), j = (t >> 2) & 7, k = t >> 5;
   const int32_t* adj = p.adj + brick * 8;
 
-  double2 bv = make_double2(0.0, 0.0);
-  if (MODE != MODE_APPLY) bv = ld_stream2(p.b + brick * 512 + 2 * t);
+  double2 bv[HP];
+#pragma unroll
+  for (int h = 0; h < HP; ++h)
+    bv[h] = MODE != MODE_APPLY ? ld_stream2(p.b + brick * 512 + 2 * (t + NT * h)) : make_double2(0.0, 0.0);
 
   if (!ZERO_X) {
-    double2 xv = ldg2(p.x + brick * 512 + 2 * t);
-    if (INTERP) {
-      const int pr = __ldg(p.parent + brick);
-      if (pr >= 0) {
-        const double* xc = p.xc + (int64_t)(pr >> 3) * 512;
-        const int co = coarse_off(pr & 7, i0, j, k);  // i0, i0+1 share a coarse cell
-        const double cv = __ldg(xc + co);
-        xv.x = DADD(xv.x, cv);
-        xv.y = DADD(xv.y, cv);
+#pragma unroll
+    for (int h = 0; h < HP; ++h) {
+      const int tt = t + NT * h, i0 = 2 * (tt & 3), j = (tt >> 2) & 7, k = tt >> 5;
+      double2 xv = ldg2(p.x + brick * 512 + 2 * tt);
+      if (INTERP) {
+        const int pr = __ldg(p.parent + brick);
+        if (pr >= 0) {
+          const double* xc = p.xc + (int64_t)(pr >> 3) * 512;
+          const int co = coarse_off(pr & 7, i0, j, k);  // i0, i0+1 share a coarse cell
+          const double cv = __ldg(xc + co);
+          xv.x = DADD(xv.x, cv);
+          xv.y = DADD(xv.y, cv);
+        }
       }
+      xs[2 * tt] = xv.x;
+      xs[2 * tt + 1] = xv.y;
     }
-    xs[2 * t] = xv.x;
-    xs[2 * t + 1] = xv.y;
-    // halos: faces W,E,S,N (t = 0..255), B,T (t = 0..127)
-    {
-      const int f = t >> 6, m = t & 63;
+    // halos: faces W,E,S,N (entries 0..255), B,T (entries 0..127)
+#pragma unroll
+    for (int h = 0; h < HP; ++h) {
+      const int tt = t + NT * h, f = tt >> 6, m = tt & 63;
       const int nb = __ldg(adj + f);
       int ci, cj, ck;
       if (f < 2) {
@@ -113,8 +123,8 @@ __global__ void __launch_bounds__(256) sweep_kernel(SweepArgs p, unsigned long l
         const int pr = __ldg(p.parent + nb);
         if (pr >= 0) v = DADD(v, __ldg(p.xc + (int64_t)(pr >> 3) * 512 + coarse_off(pr & 7, ci, cj, ck)));
       }
-      double* h = f == 0 ? hw : f == 1 ? he : f == 2 ? hs : hn;
-      h[m] = v;
+      double* hh = f == 0 ? hw : f == 1 ? he : f == 2 ? hs : hn;
+      hh[m] = v;
     }
     if (t < 128) {
       const int f = 4 + (t >> 6), m = t & 63;
@@ -130,11 +140,13 @@ __global__ void __launch_bounds__(256) sweep_kernel(SweepArgs p, unsigned long l
     __syncthreads();
   }
   if (VC) {
-    const double2 cv = ldg2(p.cf + brick * 512 + 2 * t);
-    cs[2 * t] = cv.x;
-    cs[2 * t + 1] = cv.y;
-    {
-      const int f = t >> 6, m = t & 63;
+#pragma unroll
+    for (int h = 0; h < HP; ++h) {
+      const int tt = t + NT * h;
+      const double2 cv = ldg2(p.cf + brick * 512 + 2 * tt);
+      cs[2 * tt] = cv.x;
+      cs[2 * tt + 1] = cv.y;
+      const int f = tt >> 6, m = tt & 63;
       const int nb = __ldg(adj + f);
       const int ci = f < 2 ? (f == 0 ? 7 : 0) : (m & 7), cj = f < 2 ? (m & 7) : (f == 2 ? 7 : 0), ck = m >> 3;
       ch[f][m] = __ldg(p.cf + (int64_t)nb * 512 + ci + 8 * cj + 64 * ck);
@@ -146,49 +158,53 @@ __global__ void __launch_bounds__(256) sweep_kernel(SweepArgs p, unsigned long l
     __syncthreads();
   }
 
-  double out[2], res[2];
+  double out[HP][2], res[HP][2];
   double mx = 0.0;
 #pragma unroll
-  for (int ii = 0; ii < 2; ++ii) {
-    const int i = i0 + ii;
-    const int o = i + 8 * j + 64 * k;
-    double c, w, e, s, n, bt, tp;
-    if (ZERO_X) {
-      c = w = e = s = n = bt = tp = 0.0;
-    } else {
-      c = xs[o];
-      w = i > 0 ? xs[o - 1] : hw[j + 8 * k];
-      e = i < 7 ? xs[o + 1] : he[j + 8 * k];
-      s = j > 0 ? xs[o - 8] : hs[i + 8 * k];
-      n = j < 7 ? xs[o + 8] : hn[i + 8 * k];
-      bt = k > 0 ? xs[o - 64] : hb[i + 8 * j];
-      tp = k < 7 ? xs[o + 64] : ht[i + 8 * j];
-    }
-    double a, gam = p.c.gamma;
-    if (VC) {
-      // (A x)_p = inv * sum_n ((c_p + c_n) * 0.5) * (x_n - x_p), gamma_p = (0.5 h h) / sum_n face coefficient
-      const double cp = cs[o];
-      const double cw = i > 0 ? cs[o - 1] : ch[0][j + 8 * k], ce = i < 7 ? cs[o + 1] : ch[1][j + 8 * k];
-      const double cS = j > 0 ? cs[o - 8] : ch[2][i + 8 * k], cN = j < 7 ? cs[o + 8] : ch[3][i + 8 * k];
-      const double cB = k > 0 ? cs[o - 64] : ch[4][i + 8 * j], cT = k < 7 ? cs[o + 64] : ch[5][i + 8 * j];
-      const double fw = DMUL(DADD(cp, cw), 0.5), fe = DMUL(DADD(cp, ce), 0.5), fs = DMUL(DADD(cp, cS), 0.5);
-      const double fn = DMUL(DADD(cp, cN), 0.5), fb = DMUL(DADD(cp, cB), 0.5), ft = DMUL(DADD(cp, cT), 0.5);
-      const double sum = DADD(DADD(DADD(DMUL(fw, DSUB(w, c)), DMUL(fe, DSUB(e, c))),
-                                   DADD(DMUL(fs, DSUB(s, c)), DMUL(fn, DSUB(n, c)))),
-                              DADD(DMUL(fb, DSUB(bt, c)), DMUL(ft, DSUB(tp, c))));
-      a = DMUL(p.c.beta, sum);
-      gam = __ddiv_rn(p.vc_g, DADD(DADD(DADD(fw, fe), DADD(fs, fn)), DADD(fb, ft)));
-    } else {
-      a = stencil_a(c, w, e, s, n, bt, tp, p.c.alpha, p.c.beta);
-    }
-    const double bb = ii ? bv.y : bv.x;
-    if (MODE == MODE_APPLY) {
-      out[ii] = a;
-    } else if (MODE == MODE_NORM) {
-      mx = nan_max(mx, fabs(DSUB(bb, a)));
-    } else {
-      res[ii] = DSUB(bb, a);
-      out[ii] = keep_cell(p.colour, i, j, k) ? c : DADD(c, DMUL(gam, DSUB(a, bb)));
+  for (int h = 0; h < HP; ++h) {
+    const int tt = t + NT * h, i0 = 2 * (tt & 3), j = (tt >> 2) & 7, k = tt >> 5;
+#pragma unroll
+    for (int ii = 0; ii < 2; ++ii) {
+      const int i = i0 + ii;
+      const int o = i + 8 * j + 64 * k;
+      double c, w, e, s, n, bt, tp;
+      if (ZERO_X) {
+        c = w = e = s = n = bt = tp = 0.0;
+      } else {
+        c = xs[o];
+        w = i > 0 ? xs[o - 1] : hw[j + 8 * k];
+        e = i < 7 ? xs[o + 1] : he[j + 8 * k];
+        s = j > 0 ? xs[o - 8] : hs[i + 8 * k];
+        n = j < 7 ? xs[o + 8] : hn[i + 8 * k];
+        bt = k > 0 ? xs[o - 64] : hb[i + 8 * j];
+        tp = k < 7 ? xs[o + 64] : ht[i + 8 * j];
+      }
+      double a, gam = p.c.gamma;
+      if (VC) {
+        // (A x)_p = inv * sum_n ((c_p + c_n) * 0.5) * (x_n - x_p), gamma_p = (0.5 h h) / sum_n face coefficient
+        const double cp = cs[o];
+        const double cw = i > 0 ? cs[o - 1] : ch[0][j + 8 * k], ce = i < 7 ? cs[o + 1] : ch[1][j + 8 * k];
+        const double cS = j > 0 ? cs[o - 8] : ch[2][i + 8 * k], cN = j < 7 ? cs[o + 8] : ch[3][i + 8 * k];
+        const double cB = k > 0 ? cs[o - 64] : ch[4][i + 8 * j], cT = k < 7 ? cs[o + 64] : ch[5][i + 8 * j];
+        const double fw = DMUL(DADD(cp, cw), 0.5), fe = DMUL(DADD(cp, ce), 0.5), fs = DMUL(DADD(cp, cS), 0.5);
+        const double fn = DMUL(DADD(cp, cN), 0.5), fb = DMUL(DADD(cp, cB), 0.5), ft = DMUL(DADD(cp, cT), 0.5);
+        const double sum = DADD(DADD(DADD(DMUL(fw, DSUB(w, c)), DMUL(fe, DSUB(e, c))),
+                                     DADD(DMUL(fs, DSUB(s, c)), DMUL(fn, DSUB(n, c)))),
+                                DADD(DMUL(fb, DSUB(bt, c)), DMUL(ft, DSUB(tp, c))));
+        a = DMUL(p.c.beta, sum);
+        gam = __ddiv_rn(p.vc_g, DADD(DADD(DADD(fw, fe), DADD(fs, fn)), DADD(fb, ft)));
+      } else {
+        a = stencil_a(c, w, e, s, n, bt, tp, p.c.alpha, p.c.beta);
+      }
+      const double bb = ii ? bv[h].y : bv[h].x;
+      if (MODE == MODE_APPLY) {
+        out[h][ii] = a;
+      } else if (MODE == MODE_NORM) {
+        mx = nan_max(mx, fabs(DSUB(bb, a)));
+      } else {
+        res[h][ii] = DSUB(bb, a);
+        out[h][ii] = keep_cell(p.colour, i, j, k) ? c : DADD(c, DMUL(gam, DSUB(a, bb)));
+      }
     }
   }
 
@@ -196,25 +212,29 @@ __global__ void __launch_bounds__(256) sweep_kernel(SweepArgs p, unsigned long l
     // exact max: compare as doubles, publish the bit pattern (monotone for >= 0)
 #pragma unroll
     for (int off = 16; off > 0; off >>= 1) mx = nan_max(mx, __shfl_xor_sync(0xffffffffu, mx, off));
-    __shared__ double wm[8];
+    __shared__ double wm[NT / 32];
     if ((t & 31) == 0) wm[t >> 5] = mx;
     __syncthreads();
     if (t == 0) {
       double m = wm[0];
-      for (int w = 1; w < 8; ++w) m = nan_max(m, wm[w]);
+      for (int w = 1; w < NT / 32; ++w) m = nan_max(m, wm[w]);
       atomicMax(acc, (unsigned long long)__double_as_longlong(m));
     }
     return;
   }
-  if (MODE == MODE_APPLY) {
-    st_stream2(p.xo + brick * 512 + 2 * t, make_double2(out[0], out[1]));
-    return;
+#pragma unroll
+  for (int h = 0; h < HP; ++h) {
+    const int tt = t + NT * h;
+    st_stream2(p.xo + brick * 512 + 2 * tt, make_double2(out[h][0], out[h][1]));
+    if (MODE == MODE_SWEEP && WRITE_R) st_stream2(p.r + brick * 512 + 2 * tt, make_double2(res[h][0], res[h][1]));
   }
-  st_stream2(p.xo + brick * 512 + 2 * t, make_double2(out[0], out[1]));
-  if (WRITE_R) st_stream2(p.r + brick * 512 + 2 * t, make_double2(res[0], res[1]));
-  if (RESTRICT) {
-    rs[2 * t] = res[0];
-    rs[2 * t + 1] = res[1];
+  if (MODE == MODE_SWEEP && RESTRICT) {
+#pragma unroll
+    for (int h = 0; h < HP; ++h) {
+      const int tt = t + NT * h;
+      rs[2 * tt] = res[h][0];
+      rs[2 * tt + 1] = res[h][1];
+    }
     __syncthreads();
     if (t < 64) {
       const int I = t & 3, J = (t >> 2) & 3, K = t >> 4;
@@ -231,10 +251,17 @@ __global__ void __launch_bounds__(256) sweep_kernel(SweepArgs p, unsigned long l
   }
 }
 
+// ranges of at least this many bricks run the 128-thread variant (more bricks in flight per SM)
+constexpr int64_t kSweep128Bricks = 4096;
+
 template <unsigned FLAGS>
 static cudaError_t launch_sweep_t(const SweepArgs& a, cudaStream_t s) {
   if (a.nbricks <= 0) return cudaSuccess;
-  launch_k(sweep_kernel<MODE_SWEEP, FLAGS>, (unsigned)a.nbricks, 256, 0, s, a, nullptr);
+  static const bool nt256 = getenv("MG_SWEEP_NT256") != nullptr;  // (A/B: the 256-thread variant everywhere)
+  if (a.nbricks >= kSweep128Bricks && !nt256)
+    launch_k(sweep_kernel<MODE_SWEEP, FLAGS, 128>, (unsigned)a.nbricks, 128, 0, s, a, nullptr);
+  else
+    launch_k(sweep_kernel<MODE_SWEEP, FLAGS>, (unsigned)a.nbricks, 256, 0, s, a, nullptr);
   return cudaGetLastError();
 }
 
@@ -526,7 +553,11 @@ cudaError_t launch_apply_op(const double* x, double* Ax, const int32_t* adj, int
   a.c = c;
   a.E = E;
   if (E != 8) return launch_gsweep(a, 0, 1, nullptr, s);
-  launch_k(sweep_kernel<MODE_APPLY, 0>, (unsigned)nbricks, 256, 0, s, a, nullptr);
+  static const bool nt256 = getenv("MG_SWEEP_NT256") != nullptr;
+  if (nbricks >= kSweep128Bricks && !nt256)
+    launch_k(sweep_kernel<MODE_APPLY, 0, 128>, (unsigned)nbricks, 128, 0, s, a, nullptr);
+  else
+    launch_k(sweep_kernel<MODE_APPLY, 0>, (unsigned)nbricks, 256, 0, s, a, nullptr);
   return cudaGetLastError();
 }
 
@@ -543,8 +574,14 @@ cudaError_t launch_norm(const double* x, const double* b, const int32_t* adj, in
   a.cf = cf;
   a.E = E;
   if (E != 8) return launch_gsweep(a, cf ? SW_VARCOEF : 0u, 2, acc, s);
-  if (cf)
+  static const bool nt256 = getenv("MG_SWEEP_NT256") != nullptr;
+  const bool big = nbricks >= kSweep128Bricks && !nt256;
+  if (cf && big)
+    launch_k(sweep_kernel<MODE_NORM, SW_VARCOEF, 128>, (unsigned)nbricks, 128, 0, s, a, acc);
+  else if (cf)
     launch_k(sweep_kernel<MODE_NORM, SW_VARCOEF>, (unsigned)nbricks, 256, 0, s, a, acc);
+  else if (big)
+    launch_k(sweep_kernel<MODE_NORM, 0, 128>, (unsigned)nbricks, 128, 0, s, a, acc);
   else
     launch_k(sweep_kernel<MODE_NORM, 0>, (unsigned)nbricks, 256, 0, s, a, acc);
   return cudaGetLastError();
