@@ -56,6 +56,7 @@ struct DevLevel {
   };
   std::vector<Col> cols;  // streaming-sweep plans (column segments) per brick range
   FaceMaps fmaps[2];      // TMA face-halo tensor maps over x[0], x[1] (levels with column plans)
+  FaceMaps cfmaps{};      // ... and over the coefficients (variable-coefficient variant)
   struct Pair {
     int64_t b0, b1;
     int part;  // LevelLayout::PairTable::part
@@ -293,10 +294,12 @@ mg_params normalized(const mg_params* p) {
     q.h0 = m > 0 ? 1.0 / (double)m : 1.0;
   }
   if (q.cheby_ratio <= 0) q.cheby_ratio = 6;
-  if (q.var_coef || q.brick_edge == 4) {  // A23 / 4^3 bricks: the one-brick kernels carry the variant
-    q.sweep_kernel = 1;
+  if (q.var_coef || q.brick_edge == 4) {  // A23 / 4^3 bricks: no pencil passes, per-sweep bottoms
     q.temporal_blocking = 0;
     q.bottom_mode = MG_BOTTOM_SWEEPS;
+    // 4^3 bricks: the one-brick kernels of generic.cu only; variable coefficients: the TMA column
+    // kernel's coefficient variant on the large levels, the one-brick kernel elsewhere
+    if (q.brick_edge == 4) q.sweep_kernel = 1;
   }
   return q;
 }
@@ -506,10 +509,16 @@ mg_status sweep_range(mg_ctx* c, const Op& o, int64_t b0, int64_t b1, cudaStream
   a.colour2 = o.c2;
   a.E = c->lay.E;
   unsigned fl = o.flags;
-  if (d.cf) {  // variable coefficients (reading A23): the one-brick kernel only (normalized() forces it)
+  if (d.cf) {  // variable coefficients (reading A23): the column kernel's variant where a plan exists
     a.cf = d.cf;
     a.vc_g = 0.5 * (d.h * d.h);
     fl |= SW_VARCOEF;
+    if (c->use_col && col_supports(o.flags) && c->lay.E == 8)
+      for (const auto& col : d.cols)
+        if (col.b0 == b0 && col.b1 == b1) {
+          CKC(c, launch_sweep_col(a, col.args, d.fmaps[o.src], fl, s, &d.cfmaps));
+          return MG_OK;
+        }
     CKC(c, launch_sweep(a, fl, s));
     return MG_OK;
   }
@@ -867,8 +876,10 @@ mg_status init_ctx(mg_ctx* c, const mg_params& p, int rank, int world, int devic
       CKC(c, cudaMemcpyAsync((void*)ca.side, ct.side.data(), ct.side.size() * 4, cudaMemcpyHostToDevice, stream));
       CKC(c, cudaMemcpyAsync((void*)ca.segs, ct.segs.data(), ct.segs.size() * 4, cudaMemcpyHostToDevice, stream));
     }
-    if (!L.cols.empty())
+    if (!L.cols.empty()) {
       for (int xb = 0; xb < 2; ++xb) CKC(c, encode_face_maps(d.x[xb], L.n_alloc, &d.fmaps[xb]));
+      if (d.cf) CKC(c, encode_face_maps(d.cf, L.n_alloc, &d.cfmaps));
+    }
     for (size_t k = 0; k < L.pairs.size(); ++k) {
       const auto& pt = L.pairs[k];
       const PairArgs& pa = d.pairs[k].args;
@@ -1171,7 +1182,7 @@ static mg_status norm_launch(mg_ctx* c, unsigned long long* acc, cudaStream_t s)
   const LevelLayout& L = c->lay.lv[0];
   DevLevel& d = c->dl[0];
   const int cur = c->st[0].cur;
-  if (c->use_col && !d.cf && c->lay.E == 8) {
+  if (c->use_col && c->lay.E == 8) {
     for (const auto& col : d.cols) {
       if (col.b0 == 0 && col.b1 == L.n_owned) {
         SweepArgs a{};
@@ -1182,7 +1193,9 @@ static mg_status norm_launch(mg_ctx* c, unsigned long long* acc, cudaStream_t s)
         a.nbricks = L.n_owned;
         a.c = d.c;
         a.acc = acc;
-        CKC(c, launch_sweep_col(a, col.args, d.fmaps[cur], SW_NORM, s));
+        a.cf = d.cf;  // (variable coefficients: the column kernel's coefficient variant)
+        a.vc_g = 0.5 * (d.h * d.h);
+        CKC(c, launch_sweep_col(a, col.args, d.fmaps[cur], SW_NORM | (d.cf ? SW_VARCOEF : 0u), s, &d.cfmaps));
         return MG_OK;
       }
     }

@@ -18,6 +18,7 @@
 
 #include <algorithm>
 #include <cstdlib>
+#include <cstddef>
 #include <cstdint>
 
 #include <cudaTypedefs.h>
@@ -313,19 +314,30 @@ cudaError_t launch_sweep(const SweepArgs& a, unsigned flags, cudaStream_t s) {
 constexpr int COL_NST = 3;  // ring stages: current, next (plane 0 = k-halo), one in flight
 constexpr int COL_MAXSEG = 16;
 
-struct ColStage {
+template <bool VC>
+struct alignas(128) ColStage {  // (every stage and its TMA destinations 128-byte aligned)
   double x[512];
   double b[512];
   double fwe[2][64][2];  // W box (i=6,7 of the W brick) and E box (i=0,1 of the E brick), [k][j][2]
   double fsn[2][64];     // S row (j=7 of the S brick) and N row (j=0 of the N brick), [k][i]
+  // variable coefficients (reading A23): the c brick and its face halos, boxes as for x
+  double c[VC ? 512 : 1];
+  double cwe[VC ? 2 : 1][VC ? 64 : 1][2];
+  double csn[VC ? 2 : 1][VC ? 64 : 1];
 };
 constexpr uint32_t kStageBytes = 8192 + 2 * 1024 + 2 * 512;  // TMA bytes landing in one full stage
+constexpr uint32_t kStageBytesC = 4096 + 2 * 1024 + 2 * 512;  // ... and the c brick + halos (VC)
+static_assert(offsetof(ColStage<false>, fsn) % 128 == 0 && offsetof(ColStage<true>, c) % 128 == 0 &&
+                  offsetof(ColStage<true>, cwe) % 128 == 0 && offsetof(ColStage<true>, csn) % 128 == 0 &&
+                  sizeof(ColStage<false>) % 128 == 0 && sizeof(ColStage<true>) % 128 == 0,
+              "TMA destinations 128-byte aligned");
 
-template <bool RESTRICT>
+template <bool RESTRICT, bool VC>
 struct ColSmem {
-  ColStage st[COL_NST];  // stage of "brick" cnt holds only plane 0 of the brick above the segment
+  ColStage<VC> st[COL_NST];  // stage of "brick" cnt holds only plane 0 of the brick above the segment
   double carry[2][64];   // plane 7 of the previous brick (k-halo of plane 0), double-buffered;
                          // carry[1] first holds plane 7 of the brick below the segment
+  double ccarry[VC ? 2 : 1][64];  // the same for c (VC)
   double rs[RESTRICT ? 2 : 1][RESTRICT ? 512 : 2];  // residual of the current brick (fused restriction)
   uint64_t bar[COL_NST + 1];
   int sid[COL_MAXSEG];
@@ -335,15 +347,31 @@ struct ColSmem {
 
 constexpr int COL_WARPS = 4;  // warp w streams planes 2w, 2w+1 of every brick
 
+// variable-coefficient cell (reading A23, the expression of sweep_kernel<..., SW_VARCOEF>): returns a = A x
+// and sets gam = (0.5 h h) / (sum of the face coefficients)
+__device__ __forceinline__ double vc_cell(double c, double w, double e, double s, double n, double bt, double tp,
+                                          double cp, double cw, double ce, double cS, double cN, double cB,
+                                          double cT, double beta, double vc_g, double& gam) {
+  const double fw = DMUL(DADD(cp, cw), 0.5), fe = DMUL(DADD(cp, ce), 0.5), fs = DMUL(DADD(cp, cS), 0.5);
+  const double fn = DMUL(DADD(cp, cN), 0.5), fb = DMUL(DADD(cp, cB), 0.5), ft = DMUL(DADD(cp, cT), 0.5);
+  const double sum = DADD(DADD(DADD(DMUL(fw, DSUB(w, c)), DMUL(fe, DSUB(e, c))),
+                               DADD(DMUL(fs, DSUB(s, c)), DMUL(fn, DSUB(n, c)))),
+                          DADD(DMUL(fb, DSUB(bt, c)), DMUL(ft, DSUB(tp, c))));
+  gam = __ddiv_rn(vc_g, DADD(DADD(DADD(fw, fe), DADD(fs, fn)), DADD(fb, ft)));
+  return DMUL(beta, sum);
+}
+
 template <unsigned FLAGS>
-__global__ void __launch_bounds__(COL_WARPS * 32, 6)
-    sweep_col_kernel(SweepArgs p, ColArgs ca, const __grid_constant__ FaceMaps fm) {
+__global__ void __launch_bounds__(COL_WARPS * 32, (FLAGS & SW_VARCOEF) ? 4 : 6)
+    sweep_col_kernel(SweepArgs p, ColArgs ca, const __grid_constant__ FaceMaps fm,
+                     const __grid_constant__ FaceMaps fmc) {
   pdl_wait();
   constexpr bool WRITE_R = (FLAGS & SW_WRITE_R) != 0;
   constexpr bool RESTRICT = (FLAGS & SW_RESTRICT) != 0;
   constexpr bool NORM = (FLAGS & SW_NORM) != 0;  // maxNormRes: only max |b - Ax| leaves the kernel
+  constexpr bool VC = (FLAGS & SW_VARCOEF) != 0;  // variable coefficients: the c field streams too
   extern __shared__ __align__(128) unsigned char smem_raw[];
-  ColSmem<RESTRICT>& S = *reinterpret_cast<ColSmem<RESTRICT>*>(smem_raw);
+  ColSmem<RESTRICT, VC>& S = *reinterpret_cast<ColSmem<RESTRICT, VC>*>(smem_raw);
   double mx = 0.0;
   const int t = threadIdx.x, w = t >> 5, l = t & 31;
   const int i0 = 2 * (l & 3), j = l >> 2;
@@ -362,30 +390,39 @@ __global__ void __launch_bounds__(COL_WARPS * 32, 6)
   }
   __syncthreads();
   // stage brick n (thread 0): x and b bricks by 1D bulk copies, the four face halos
-  // by 3D tensor copies.  n == cnt stages only plane 0 of the brick above the segment.
+  // by 3D tensor copies (+ the same for c).  n == cnt stages only plane 0 of the brick above the segment.
   auto issue = [&](int n) {
     if (t != 0) return;
     const int s = n % COL_NST;
     if (n == cnt) {
       const int64_t above = __ldg(p.adj + (int64_t)S.sid[cnt - 1] * 8 + 5);
-      mbar_expect_tx(&S.bar[s], 512);
+      mbar_expect_tx(&S.bar[s], VC ? 1024 : 512);
       tma_load_1d(S.st[s].x, p.x + above * 512, 512, &S.bar[s]);
+      if (VC) tma_load_1d(S.st[s].c, p.cf + above * 512, 512, &S.bar[s]);
       return;
     }
     const int64_t id = S.sid[n];
     const int4 sd = S.sside[n];
-    mbar_expect_tx(&S.bar[s], kStageBytes);
+    mbar_expect_tx(&S.bar[s], kStageBytes + (VC ? kStageBytesC : 0));
     tma_load_1d(S.st[s].x, p.x + id * 512, 4096, &S.bar[s]);
     tma_load_1d(S.st[s].b, p.b + id * 512, 4096, &S.bar[s]);
     tma_load_3d(S.st[s].fwe[0], &fm.we, 6, 0, sd.x * 8, &S.bar[s]);  // W brick, i = 6..7
     tma_load_3d(S.st[s].fwe[1], &fm.we, 0, 0, sd.y * 8, &S.bar[s]);  // E brick, i = 0..1
     tma_load_3d(S.st[s].fsn[0], &fm.sn, 0, 7, sd.z * 8, &S.bar[s]);  // S brick, j = 7
     tma_load_3d(S.st[s].fsn[1], &fm.sn, 0, 0, sd.w * 8, &S.bar[s]);  // N brick, j = 0
+    if (VC) {
+      tma_load_1d(S.st[s].c, p.cf + id * 512, 4096, &S.bar[s]);
+      tma_load_3d(S.st[s].cwe[0], &fmc.we, 6, 0, sd.x * 8, &S.bar[s]);
+      tma_load_3d(S.st[s].cwe[1], &fmc.we, 0, 0, sd.y * 8, &S.bar[s]);
+      tma_load_3d(S.st[s].csn[0], &fmc.sn, 0, 7, sd.z * 8, &S.bar[s]);
+      tma_load_3d(S.st[s].csn[1], &fmc.sn, 0, 0, sd.w * 8, &S.bar[s]);
+    }
   };
   if (t == 0) {
     const int64_t below = __ldg(p.adj + (int64_t)S.sid[0] * 8 + 4);
-    mbar_expect_tx(&S.bar[COL_NST], 512);
+    mbar_expect_tx(&S.bar[COL_NST], VC ? 1024 : 512);
     tma_load_1d(S.carry[1], p.x + below * 512 + 448, 512, &S.bar[COL_NST]);
+    if (VC) tma_load_1d(S.ccarry[VC ? 1 : 0], p.cf + below * 512 + 448, 512, &S.bar[COL_NST]);
   }
   issue(0);
   issue(1);  // brick 1, or the plane above when cnt == 1
@@ -398,25 +435,31 @@ __global__ void __launch_bounds__(COL_WARPS * 32, 6)
     }
     const int s = n % COL_NST;
     mbar_wait(&S.bar[s], (uint32_t)((n / COL_NST) & 1));
-    const ColStage& G = S.st[s];
+    const ColStage<VC>& G = S.st[s];
     const double* X = G.x;
     const int k0 = 2 * w;
-    double2 xm, xc, xp;
-    if (w > 0)
+    double2 xm, xc, xp, cm = make_double2(0.0, 0.0), cc = cm, cpn = cm;
+    if (w > 0) {
       xm = *reinterpret_cast<const double2*>(X + 64 * (k0 - 1) + q);
-    else
+      if (VC) cm = *reinterpret_cast<const double2*>(G.c + 64 * (k0 - 1) + q);
+    } else {
       xm = *reinterpret_cast<const double2*>(S.carry[(n + 1) & 1] + q);  // = carry[(n-1)&1]
+      if (VC) cm = *reinterpret_cast<const double2*>(S.ccarry[VC ? (n + 1) & 1 : 0] + q);
+    }
     xc = *reinterpret_cast<const double2*>(X + 64 * k0 + q);
+    if (VC) cc = *reinterpret_cast<const double2*>(G.c + 64 * k0 + q);
     const int64_t gbase = (int64_t)S.sid[n] * 512 + q;
 #pragma unroll
     for (int kk = 0; kk < 2; ++kk) {
       const int k = k0 + kk;
       if (k < 7) {
         xp = *reinterpret_cast<const double2*>(X + 64 * (k + 1) + q);
+        if (VC) cpn = *reinterpret_cast<const double2*>(G.c + 64 * (k + 1) + q);
       } else {  // plane 0 of the next brick (or of the brick above the segment)
         const int s1 = (n + 1) % COL_NST;
         mbar_wait(&S.bar[s1], (uint32_t)(((n + 1) / COL_NST) & 1));
         xp = *reinterpret_cast<const double2*>(S.st[s1].x + q);
+        if (VC) cpn = *reinterpret_cast<const double2*>(S.st[s1].c + q);
       }
       const double2 bb = *reinterpret_cast<const double2*>(G.b + 64 * k + q);
       const double2 rs_ = *reinterpret_cast<const double2*>(X + 64 * k + (j > 0 ? q - 8 : q));
@@ -431,11 +474,28 @@ __global__ void __launch_bounds__(COL_WARPS * 32, 6)
       const double ev = i0 < 6 ? er : fe;
       const double2 sv = j > 0 ? rs_ : fs;
       const double2 nv = j < 7 ? rn_ : fn;
-      const double a0 = stencil_a(xc.x, wv, xc.y, sv.x, nv.x, xm.x, xp.x, p.c.alpha, p.c.beta);
-      const double a1 = stencil_a(xc.y, xc.x, ev, sv.y, nv.y, xm.y, xp.y, p.c.alpha, p.c.beta);
+      double a0, a1, g0 = p.c.gamma, g1 = p.c.gamma;
+      if (VC) {
+        const double2 crs = *reinterpret_cast<const double2*>(G.c + 64 * k + (j > 0 ? q - 8 : q));
+        const double2 crn = *reinterpret_cast<const double2*>(G.c + 64 * k + (j < 7 ? q + 8 : q));
+        const double cfw = G.cwe[0][j + 8 * k][1], cfe = G.cwe[VC ? 1 : 0][j + 8 * k][0];
+        const double2 cfs = *reinterpret_cast<const double2*>(&G.csn[0][i0 + 8 * k]);
+        const double2 cfn = *reinterpret_cast<const double2*>(&G.csn[VC ? 1 : 0][i0 + 8 * k]);
+        const double cwl = __shfl_up_sync(0xffffffffu, cc.y, 1);
+        const double cer = __shfl_down_sync(0xffffffffu, cc.x, 1);
+        const double cwv = i0 > 0 ? cwl : cfw, cev = i0 < 6 ? cer : cfe;
+        const double2 csv = j > 0 ? crs : cfs, cnv = j < 7 ? crn : cfn;
+        a0 = vc_cell(xc.x, wv, xc.y, sv.x, nv.x, xm.x, xp.x, cc.x, cwv, cc.y, csv.x, cnv.x, cm.x, cpn.x,
+                     p.c.beta, p.vc_g, g0);
+        a1 = vc_cell(xc.y, xc.x, ev, sv.y, nv.y, xm.y, xp.y, cc.y, cc.x, cev, csv.y, cnv.y, cm.y, cpn.y,
+                     p.c.beta, p.vc_g, g1);
+      } else {
+        a0 = stencil_a(xc.x, wv, xc.y, sv.x, nv.x, xm.x, xp.x, p.c.alpha, p.c.beta);
+        a1 = stencil_a(xc.y, xc.x, ev, sv.y, nv.y, xm.y, xp.y, p.c.alpha, p.c.beta);
+      }
       double2 xn, rv;
-      xn.x = keep_cell(p.colour, i0, j, k) ? xc.x : DADD(xc.x, DMUL(p.c.gamma, DSUB(a0, bb.x)));
-      xn.y = keep_cell(p.colour, i0 + 1, j, k) ? xc.y : DADD(xc.y, DMUL(p.c.gamma, DSUB(a1, bb.y)));
+      xn.x = keep_cell(p.colour, i0, j, k) ? xc.x : DADD(xc.x, DMUL(g0, DSUB(a0, bb.x)));
+      xn.y = keep_cell(p.colour, i0 + 1, j, k) ? xc.y : DADD(xc.y, DMUL(g1, DSUB(a1, bb.y)));
       rv.x = DSUB(bb.x, a0);
       rv.y = DSUB(bb.y, a1);
       if (NORM) {
@@ -446,9 +506,14 @@ __global__ void __launch_bounds__(COL_WARPS * 32, 6)
       }
       if (WRITE_R) st_stream2(p.r + gbase + 64 * k, rv);
       if (RESTRICT) *reinterpret_cast<double2*>(S.rs[n & 1] + 64 * k + q) = rv;
-      if (k == 7) *reinterpret_cast<double2*>(S.carry[n & 1] + q) = xc;  // k-halo of the next brick
+      if (k == 7) {
+        *reinterpret_cast<double2*>(S.carry[n & 1] + q) = xc;  // k-halo of the next brick
+        if (VC) *reinterpret_cast<double2*>(S.ccarry[VC ? n & 1 : 0] + q) = cc;
+      }
       xm = xc;
       xc = xp;
+      cm = cc;
+      cc = cpn;
     }
     __syncthreads();  // stage n-1 free for refill; carry / rs of brick n complete
     if (RESTRICT && t < 64) {
@@ -483,19 +548,29 @@ bool col_supports(unsigned flags) {
   return f == 0 || f == SW_WRITE_R || f == SW_RESTRICT;
 }
 
+#define COL_FLAG_LIST(X) \
+  X(0) X(SW_WRITE_R) X(SW_RESTRICT) X(SW_NORM) X(SW_VARCOEF) X(SW_VARCOEF | SW_WRITE_R) X(SW_VARCOEF | SW_RESTRICT) \
+  X(SW_VARCOEF | SW_NORM)
+
+template <unsigned F>
+constexpr size_t col_smem() {
+  return sizeof(ColSmem<(F & SW_RESTRICT) != 0, (F & SW_VARCOEF) != 0>);
+}
+
 cudaError_t launch_sweep_col(const SweepArgs& a, const ColArgs& c, const FaceMaps& fm, unsigned flags,
-                             cudaStream_t s) {
+                             cudaStream_t s, const FaceMaps* fmc) {
   if (c.nseg <= 0) return cudaSuccess;
-  const size_t sm = sizeof(ColSmem<false>), smr = sizeof(ColSmem<true>);
   const unsigned g = (unsigned)c.nseg, b = COL_WARPS * 32;
-  if (flags == SW_NORM) {
-    launch_plain(sweep_col_kernel<SW_NORM>, g, b, sm, s, a, c, fm);
-    return cudaGetLastError();
-  }
-  switch (flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP | SW_ZERO_X | SW_NORM)) {
-    case 0: launch_plain(sweep_col_kernel<0>, g, b, sm, s, a, c, fm); break;
-    case SW_WRITE_R: launch_plain(sweep_col_kernel<SW_WRITE_R>, g, b, sm, s, a, c, fm); break;
-    case SW_RESTRICT: launch_plain(sweep_col_kernel<SW_RESTRICT>, g, b, smr, s, a, c, fm); break;
+  const unsigned f = flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP | SW_ZERO_X | SW_NORM | SW_VARCOEF);
+  if ((f & SW_VARCOEF) && (!fmc || !a.cf)) return cudaErrorInvalidValue;
+  const FaceMaps& mc = fmc ? *fmc : fm;
+  switch (f) {
+#define COL_CASE(F)                                                        \
+  case (F):                                                                \
+    launch_plain(sweep_col_kernel<(F)>, g, b, col_smem<(F)>(), s, a, c, fm, mc); \
+    break;
+    COL_FLAG_LIST(COL_CASE)
+#undef COL_CASE
     default:
       return cudaErrorInvalidValue;
   }
@@ -851,16 +926,13 @@ cudaError_t kernels_init() {
   if (e != cudaSuccess) return e;
   e = cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev);
   if (e != cudaSuccess) return e;
-  const int colsm = (int)sizeof(ColSmem<false>), colsmr = (int)sizeof(ColSmem<true>);
-  const void* colk[4] = {(const void*)sweep_col_kernel<0>, (const void*)sweep_col_kernel<SW_WRITE_R>,
-                         (const void*)sweep_col_kernel<SW_RESTRICT>, (const void*)sweep_col_kernel<SW_NORM>};
-  for (int k = 0; k < 4; ++k) {
-    e = cudaFuncSetAttribute(colk[k], cudaFuncAttributeMaxDynamicSharedMemorySize, k == 2 ? colsmr : colsm);
-    if (e != cudaSuccess) return e;
-    // the streaming kernel is shared-memory-resident: ask for the full 228 KB carveout
-    e = cudaFuncSetAttribute(colk[k], cudaFuncAttributePreferredSharedMemoryCarveout, 100);
-    if (e != cudaSuccess) return e;
-  }
+#define COL_ATTR(F)                                                                                        \
+  e = cudaFuncSetAttribute(sweep_col_kernel<(F)>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)col_smem<(F)>()); \
+  if (e != cudaSuccess) return e;                                                                           \
+  e = cudaFuncSetAttribute(sweep_col_kernel<(F)>, cudaFuncAttributePreferredSharedMemoryCarveout, 100);       \
+  if (e != cudaSuccess) return e;
+  COL_FLAG_LIST(COL_ATTR)
+#undef COL_ATTR
   e = cudaFuncSetAttribute(bottom_resident_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                            kResidentMaxBricks * 512 * 2 * (int)sizeof(double));
   if (e != cudaSuccess) return e;

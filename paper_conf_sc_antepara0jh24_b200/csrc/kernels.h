@@ -103,8 +103,9 @@ cudaError_t pencil_kernels_init();
 
 // true if the streaming kernel implements `flags` (plain, +r, +restriction)
 bool col_supports(unsigned flags);
+// flags: plain / +r / +restriction, or SW_NORM; | SW_VARCOEF with fmc = the face maps over SweepArgs::cf
 cudaError_t launch_sweep_col(const SweepArgs& a, const ColArgs& c, const FaceMaps& fm, unsigned flags,
-                             cudaStream_t s);
+                             cudaStream_t s, const FaceMaps* fmc = nullptr);
 // applyOp (paper kernel set): Ax = alpha x + beta sum6
 cudaError_t launch_apply_op(const double* x, double* Ax, const int32_t* adj, int64_t brick0, int64_t nbricks,
                             Coeffs c, cudaStream_t s, int E = 8);

@@ -197,6 +197,25 @@ def test_var_coef_ca_periods_and_ghost_shells_bitwise(oracle_mod, period, ghost_
     m.close()
 
 
+@pytest.mark.parametrize("bc", [0, 1, 2])
+@pytest.mark.parametrize("ghost_mode,period", [(0, 0), (1, 3), (1, 8)])
+def test_var_coef_column_kernel_bitwise(oracle_mod, bc, ghost_mode, period):
+    """The TMA column kernel's coefficient variant (c brick + face halos staged with x and b, c k-halos
+    carried like x), forced on every level (sweep_kernel = 2: plain, +r, +restriction sweeps over owned,
+    ghost-shell, interior and surface ranges, and the norm) gives the oracle's bits."""
+    shape = (64, 32, 96)
+    b = mg_inputs.random_field(shape, 35) if bc == 1 else mg_inputs.random_rhs(shape, 35)
+    c = mg_inputs.random_coef(shape, 35)
+    xs, ns = oracle_cycles(oracle_mod, b, 3, 2, 5, 4, 20, bc=bc, coef=c)
+    m = new(shape, 3, pre=5, post=4, bottom=20, bc=bc, var_coef=1, sweep_kernel=2, ghost_mode=ghost_mode,
+            ca_period=period)
+    m.set_coefficients(dev(c))
+    m.set_rhs(dev(b))
+    m.set_solution(None)
+    check_cycles(m, xs, ns)
+    m.close()
+
+
 @pytest.mark.parametrize("bc", [0, 1])
 @pytest.mark.parametrize("pg,n_local,L", [((2, 1, 1), (32, 32, 32), 3), ((2, 2, 2), (16, 16, 16), 2),
                                           ((1, 2, 3), (16, 32, 16), 2)])

@@ -45,6 +45,10 @@ B_PER_PT = [
     ("sweep_kernel<0, 2>", "fused sweep + restriction (one-brick)", 25.0),
     ("sweep_kernel<0, 4>", "interpolation + fused sweep (one-brick)", 25.0),
     ("sweep_col_kernel<128>", "maxNormRes (TMA column kernel)", 16.0),
+    ("sweep_col_kernel<64>", "fused sweep, variable coefficients (column)", 32.0),
+    ("sweep_col_kernel<65>", "fused sweep + r, variable coefficients (column)", 40.0),
+    ("sweep_col_kernel<66>", "fused sweep + restriction, variable coefficients (column)", 33.0),
+    ("sweep_col_kernel<192>", "maxNormRes, variable coefficients (column)", 24.0),
     ("unnamed>::gsweep_kernel<4, 0, 0>", "fused sweep, 4^3 bricks", 24.0),
     ("unnamed>::gsweep_kernel<4, 0, 2>", "fused sweep + restriction, 4^3 bricks", 25.0),
     ("unnamed>::gsweep_kernel<4, 0, 4>", "interpolation + fused sweep, 4^3 bricks", 25.0),
