@@ -110,7 +110,10 @@ typedef struct {
   int32_t pre_smooths;           /* paper: 12 */
   int32_t post_smooths;          /* paper: 12 */
   int32_t bottom_smooths;        /* paper: 100 */
-  int32_t ca_period[MG_MAX_LEVELS]; /* sweeps per x-exchange per level, 1..8; 0 = auto (8) */
+  int32_t ca_period[MG_MAX_LEVELS]; /* sweeps per x-exchange per level, 1..8; 0 = auto: 2 at level 0
+                                       and 8 below on the copy transports (local, peer: an exchange
+                                       copies only the ghost cells within the period of the owned
+                                       box), 8 everywhere over NCCL (whole bricks) */
   int32_t fusion[MG_MAX_LEVELS];    /* MG_FUSION_*; 0 = auto */
   int32_t ghost_mode;            /* MG_GHOST_* */
   int32_t transport;             /* MG_TRANSPORT_*.  Between processes (world_size > 1): auto / PEER = every
@@ -258,7 +261,8 @@ mg_status mg_exchange_stats(mg_ctx* c, int64_t* bytes_per_cycle, int64_t* messag
 
 /* Per level l < cap of the V-cycle mg_vcycle would run next: exchanges[l] = ghost exchanges (x before
  * a sweep, b after the restriction), bytes[l] = bytes this rank sends in one exchange of the level
- * (0 without a ghost shell).  Host-only, no device work. */
+ * (0 without a ghost shell; on the copy transports only the ghost cells within the level's CA period
+ * of the owned box, whole bricks over NCCL).  Host-only, no device work. */
 mg_status mg_exchange_plan(mg_ctx* c, int32_t cap, int64_t* exchanges, int64_t* bytes);
 /* Device time of one ghost exchange of x at `level` (the V-cycle's transport: NCCL grouped
  * send/recv of the brick runs, or the local copy kernel), averaged over `reps` back-to-back

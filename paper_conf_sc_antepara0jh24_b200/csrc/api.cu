@@ -25,6 +25,7 @@
 #include <vector>
 
 #include "kernels.h"
+#include "copyrun.cuh"
 #include "mg_internal.h"
 #include "schedule.h"
 
@@ -377,6 +378,27 @@ double* field_ptr(mg_ctx* c, int l, int field, int xbuf) {
   return field == 0 ? c->dl[l].x[xbuf] : field == 1 ? c->dl[l].b : c->dl[l].cf;
 }
 
+// ghost cells (from the owned region) an exchange of x or b at level l makes valid (schedule.cpp)
+int exch_depth(const mg_ctx* c, int l) { return Builder(c->lay).xdepth(l); }
+
+// the cells per brick an exchange of x or b copies for a run of ghost direction r.dir: a sub-box
+// [lo, hi) per axis, the whole brick when the exchange depth is the brick edge; returns the count
+int64_t exch_box(const mg_ctx* c, int l, const Run& r, int32_t* box) {
+  const int E = c->lay.E, dep = exch_depth(c, l);
+  *box = 0;
+  if (dep >= E) return c->lay.BV;
+  int dd[3], lo[3], hi[3];
+  dir_from_index(r.dir, dd[0], dd[1], dd[2]);
+  int64_t cells = 1;
+  for (int a = 0; a < 3; ++a) {  // ghost below the owned box: its top cells; above: its bottom ones
+    lo[a] = dd[a] < 0 ? E - dep : 0;
+    hi[a] = dd[a] > 0 ? dep : E;
+    cells *= hi[a] - lo[a];
+  }
+  *box = copy_box(lo[0], hi[0], lo[1], hi[1], lo[2], hi[2], E);
+  return cells;
+}
+
 mg_status do_exchange(mg_ctx* c, int l, int field, int xbuf, cudaStream_t s) {
   const LevelLayout& L = c->lay.lv[l];
   double* f = field_ptr(c, l, field, xbuf);
@@ -453,6 +475,9 @@ mg_status fill_copy_tables(mg_ctx* c) {
     if (d.ncruns == 0) continue;
     std::vector<CopyRun> h((size_t)d.ncruns * 4, CopyRun{nullptr, nullptr, 0});
     d.cmax = 0;
+    // x and b: only the ghost cells within the exchange depth of the owned region (the cells the
+    // sweeps up to the next exchange read: a sub-box per ghost region, from its direction); the
+    // coefficients (exchanged once) whole
     for (int fv = 0; fv < 4; ++fv) {  // x[0], x[1], b, coefficients
       const int field = fv < 2 ? 0 : fv - 1, xbuf = fv < 2 ? fv : 0;
       double* f = field_ptr(c, l, field, xbuf);
@@ -463,8 +488,10 @@ mg_status fill_copy_tables(mg_ctx* c) {
         const double* sf = field_ptr(src, l, field, xbuf);
         if (c->use_peer)  // the sender's field at the same workspace offset, through its IPC mapping
           sf = (const double*)(c->peer_ws[(size_t)r.peer] + ((const char*)f - (const char*)c->peer_ws[(size_t)c->lay.rank]));
-        h[(size_t)fv * d.ncruns + i] = {sf + r.remote * bb, f + r.local * bb, (int64_t)r.count * (int64_t)bb};
-        d.cmax = std::max<int64_t>(d.cmax, (int64_t)r.count * (int64_t)bb);
+        CopyRun cr{sf + r.remote * bb, f + r.local * bb, (int64_t)r.count * (int64_t)bb};
+        const int64_t cells = fv < 3 ? exch_box(c, l, r, &cr.box) : (int64_t)bb;
+        h[(size_t)fv * d.ncruns + i] = cr;
+        d.cmax = std::max<int64_t>(d.cmax, (int64_t)r.count * cells);
       }
     }
     CKC(c, cudaMemcpy(d.cruns, h.data(), h.size() * sizeof(CopyRun), cudaMemcpyHostToDevice));
@@ -956,7 +983,7 @@ mg_status set_level_field(mg_ctx* c, int l, int field, const double* src, bool e
     c->st[l].db = 0;
     if (exchange_b && L.n_ghost > 0) {
       CKS(do_exchange(c, l, 1, 0, c->stream));
-      c->st[l].db = c->lay.E;
+      c->st[l].db = exch_depth(c, l);
     }
   }
   return MG_OK;
@@ -1214,7 +1241,7 @@ mg_status mg_residual_norm_async(mg_ctx* c) {
   DevLevel& d = c->dl[0];
   if (L.n_ghost > 0) {
     CKS(do_exchange(c, 0, 0, c->st[0].cur, c->stream));
-    c->st[0].dx = c->lay.E;
+    c->st[0].dx = exch_depth(c, 0);
     c->st[0].since = 0;
   }
   CKC(c, cudaMemsetAsync(c->acc, 0, sizeof(unsigned long long), c->stream));
@@ -1316,7 +1343,8 @@ mg_status mg_exchange_stats(mg_ctx* c, int64_t* bytes_per_cycle, int64_t* messag
     const bool ex = o.kind == OP_EXCH || ((o.kind == OP_SWEEP || o.kind == OP_SWEEP2) && o.exch_before);
     if (!ex) continue;
     for (const Run& r : c->lay.lv[o.level].sends) {
-      bytes += r.count * c->lay.BV * (int64_t)sizeof(double);
+      int32_t box;
+      bytes += r.count * exch_box(c, o.level, r, &box) * (int64_t)sizeof(double);
       ++msgs;
     }
   }
@@ -1334,7 +1362,8 @@ mg_status mg_exchange_plan(mg_ctx* c, int32_t cap, int64_t* exchanges, int64_t* 
   for (int l = 0; l < c->lay.L; ++l) {
     exchanges[l] = 0;
     bytes[l] = 0;
-    for (const Run& r : c->lay.lv[l].sends) bytes[l] += r.count * c->lay.BV * (int64_t)sizeof(double);
+    int32_t box;
+    for (const Run& r : c->lay.lv[l].sends) bytes[l] += r.count * exch_box(c, l, r, &box) * (int64_t)sizeof(double);
   }
   for (const Op& o : b.ops)
     if (o.kind == OP_EXCH || ((o.kind == OP_SWEEP || o.kind == OP_SWEEP2) && o.exch_before)) ++exchanges[o.level];
@@ -1643,7 +1672,7 @@ mg_status mg_group_commit_rhs(mg_group* g) {
   for (mg_ctx* c : g->r) {
     CKS(check_ctx(c));
     if (c->lay.lv[0].n_ghost > 0) CKS(do_exchange(c, 0, 1, 0, g->stream));
-    c->st[0].db = c->lay.E;
+    c->st[0].db = exch_depth(c, 0);
   }
   return MG_OK;
 }
@@ -1666,7 +1695,7 @@ mg_status mg_group_residual_norm(mg_group* g, double* out) {
     }
   }
   for (mg_ctx* c : g->r) {
-    c->st[0].dx = c->lay.E;
+    c->st[0].dx = exch_depth(c, 0);
     c->st[0].since = 0;
   }
   CKC(c0, cudaMemsetAsync(c0->acc, 0, sizeof(unsigned long long), g->stream));

@@ -24,6 +24,7 @@
 #include <cudaTypedefs.h>
 
 #include "kernels.h"
+#include "copyrun.cuh"
 #include "ptx.cuh"
 #include "resident.cuh"
 
@@ -903,11 +904,7 @@ cudaError_t launch_mirror(double* f, const int32_t* table, int n, double sign, c
 __global__ void __launch_bounds__(256) copy_runs_kernel(const CopyRun* __restrict__ runs) {
   pdl_begin();
   const CopyRun r = runs[blockIdx.y];
-  const double2* src = reinterpret_cast<const double2*>(r.src);
-  double2* dst = reinterpret_cast<double2*>(r.dst);
-  const int64_t n2 = r.n / 2;
-  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n2; i += (int64_t)gridDim.x * blockDim.x)
-    dst[i] = ldg2(reinterpret_cast<const double*>(src + i));
+  copy_run_body<false>(r, (int64_t)blockIdx.x * blockDim.x + threadIdx.x, (int64_t)gridDim.x * blockDim.x);
 }
 
 cudaError_t launch_copy_runs(const CopyRun* runs, int nruns, int64_t max_n, cudaStream_t s) {

@@ -134,11 +134,14 @@ cudaError_t launch_lex_to_brick(const double* lex, double* bricks, const int32_t
 cudaError_t launch_brick_to_lex(const double* bricks, double* lex, const int32_t* coord, int64_t nowned, int nx,
                                 int ny, cudaStream_t s, int E = 8);
 // Local (self / loopback) ghost exchange: every run of one exchange in ONE launch instead of one
-// cudaMemcpyAsync per run (n doubles from src to dst, both 16-byte aligned, n even).
+// cudaMemcpyAsync per run (n doubles from src to dst, both 16-byte aligned, n even).  box != 0: the
+// run is n / E^3 bricks of which only the cells of a sub-box are copied (copyrun.cuh copy_box).
 struct CopyRun {
   const double* src;
   double* dst;
   int64_t n;
+  int32_t box = 0;
+  int32_t pad_ = 0;
 };
 cudaError_t launch_copy_runs(const CopyRun* runs, int nruns, int64_t max_n, cudaStream_t s);
 // Mirror exchange (non-periodic bc, reading A22): for each entry (dst, src, mask) of the

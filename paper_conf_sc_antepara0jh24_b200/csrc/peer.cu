@@ -24,6 +24,7 @@
 #include <algorithm>
 
 #include "kernels.h"
+#include "copyrun.cuh"
 #include "ptx.cuh"
 
 namespace mgb {
@@ -87,11 +88,8 @@ __global__ void __launch_bounds__(256) peer_copy_kernel(const CopyRun* __restric
   }
   __syncthreads();
   const CopyRun r = runs[blockIdx.y];
-  const double2* src = reinterpret_cast<const double2*>(r.src);
-  double2* dst = reinterpret_cast<double2*>(r.dst);
-  const int64_t n2 = r.n / 2;
-  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n2; i += (int64_t)gridDim.x * blockDim.x)
-    dst[i] = src[i];  // remote (peer-mapped) loads: no read-only cache, the data changes between epochs
+  // remote (peer-mapped) loads: no read-only cache, the data changes between epochs
+  copy_run_body<true>(r, (int64_t)blockIdx.x * blockDim.x + threadIdx.x, (int64_t)gridDim.x * blockDim.x);
   peer_finish(s, e);
   pdl_trigger();
 }

@@ -23,13 +23,20 @@ int Builder::period(int l) const {
   const int k = lay.p.ca_period[l];
   if (k) return k;
   // auto (measured, one B200, self-exchanged ghost shell on every axis, profiles/r02_exchange.md):
-  // with exchanges as device copies on the same GPU (one rank, or a loopback group) an exchange of the
-  // finest level costs less than the redundant ghost-shell sweeping a longer period needs (period 2 at
-  // level 0: 8.42 vs 8.62 ms per cycle), the coarser levels are better at 8 (fewer launches); between
-  // processes an exchange crosses NVLink (~6x the bytes-time of a local copy, plus flag latency) and
-  // the brick-deep ghost zone's period 8 stays the default
-  const bool local = lay.world == 1 ? lay.p.transport != MG_TRANSPORT_NCCL : lay.p.transport == MG_TRANSPORT_LOCAL;
-  return (l == 0 && local) ? std::min(2, lay.E) : lay.E;
+  // where an exchange is a device copy kernel (local copies on one GPU, peer memory between
+  // processes) it copies only the ghost cells within the period of the owned region, so at level 0
+  // a period of 2 -- an exchange of the two nearest cell layers before every two-sweep pass over the
+  // owned bricks -- costs less than the redundant ghost-shell sweeping a longer period needs; the
+  // coarser levels are better at 8 (fewer launches).  NCCL moves whole bricks: period 8.
+  const bool box = lay.p.transport != MG_TRANSPORT_NCCL;
+  static const int nl2 = getenv("MG_CA2_LEVELS") ? atoi(getenv("MG_CA2_LEVELS")) : 1;  // (experiments)
+  return (l < nl2 && box) ? std::min(2, lay.E) : lay.E;
+}
+
+int Builder::xdepth(int l) const {
+  static const bool whole = getenv("MG_EXCH_WHOLE") && atoi(getenv("MG_EXCH_WHOLE"));  // (A/B runs)
+  if (whole || lay.p.transport == MG_TRANSPORT_NCCL) return lay.E;
+  return std::max(1, std::min(period(l), lay.E));
 }
 
 bool Builder::has_pair_table(int l, int64_t b0, int64_t b1) const {
@@ -113,7 +120,7 @@ void Builder::phase(int l, int n, bool zero_first, int last, bool interp_first, 
       o.zero = zero_first && s == 0;  // the first sweep reads x0 == 0 (SW_ZERO_X)
       const bool ex = g && !o.zero && (S.dx < 2 || S.since + 2 > k);
       if (ex) {
-        S.dx = lay.E;
+        S.dx = xdepth(l);
         S.since = 0;
       }
       o.exch_before = ex;
@@ -146,7 +153,7 @@ void Builder::phase(int l, int n, bool zero_first, int last, bool interp_first, 
     const bool zero = zero_first && s == 0;
     const bool ex = g && !zero && (S.dx < 1 || S.since >= k);
     if (ex) {
-      S.dx = lay.E;
+      S.dx = xdepth(l);
       S.since = 0;
     }
     o.exch_before = ex;
@@ -178,7 +185,7 @@ void Builder::exchange_b(int l) {
   o.field = 1;
   o.timer = MG_OP_EXCHANGE;
   ops.push_back(o);
-  st[l].db = lay.E;
+  st[l].db = xdepth(l);
 }
 
 void Builder::restrict_op(int l) {

@@ -61,6 +61,9 @@ struct Builder {
   bool ghosts(int l) const { return lay.lv[l].n_ghost > 0; }
   int fusion(int l) const;
   int period(int l) const;
+  // cells of a ghost brick an exchange of level l refreshes, counted from the owned region: the
+  // period (depth-limited copies, local and peer transports) or the whole brick (NCCL)
+  int xdepth(int l) const;
   bool pair_ok(int l) const;  // two-sweep passes possible at level l
   bool pencil_table(int l) const;  // the owned range of level l has a 2x2-brick pencil plan (kind 3)
   bool pencil_ghosts(int l) const;  // ... and so has its whole stored range (owned + ghost shell)

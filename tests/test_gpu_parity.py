@@ -827,9 +827,15 @@ def test_exchange_plan_and_timing_keep_the_bits(oracle_mod, transport):
     counts, nbytes = m.exchange_plan()
     # (the coarsest level runs the replicated bottom: its b is all-gathered, no ghost exchange)
     assert all(c > 0 for c in counts[:-1]) and counts[-1] == 0 and all(v > 0 for v in nbytes)
-    # one exchange of level 0 fills the whole one-brick ghost shell: 10^3 - 8^3 bricks of 4 KiB (a
-    # surface brick goes to every face / edge / corner direction it borders)
-    assert nbytes[0] == (10**3 - 8**3) * 4096
+    # NCCL: one exchange of level 0 fills the whole one-brick ghost shell, 10^3 - 8^3 bricks of 4 KiB
+    # (a surface brick goes to every face / edge / corner direction it borders); the copy transports
+    # (local, peer) at level 0's period 2 copy only the ghost cells within 2 of the owned box
+    if transport == 1:
+        assert nbytes[0] == (10**3 - 8**3) * 4096
+    else:
+        assert nbytes[0] == (68**3 - 64**3) * 8
+    # level 1 (period 8 = the brick edge): whole bricks on every transport
+    assert nbytes[1] == (6**3 - 4**3) * 4096
     m.vcycle()
     for l in range(3):
         assert m.exchange_time(l, 3) > 0
