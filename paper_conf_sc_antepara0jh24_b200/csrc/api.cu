@@ -863,6 +863,27 @@ mg_status vcycle_impl(mg_ctx* c, mg_group* g) {
   return MG_OK;
 }
 
+// MG_POISON_GHOSTS=1 (tests): every ghost cell of every field starts as NaN (and x's ghosts again after
+// mg_set_solution(NULL)), so a kernel reading a ghost cell the exchange did not refresh -- a cell
+// beyond the exchange depth, or one stale since the last exchange -- poisons the owned results
+bool poison_ghosts_on() {
+  const char* e = getenv("MG_POISON_GHOSTS");
+  return e && atoi(e) != 0;
+}
+cudaError_t poison_ghosts(mg_ctx* c, int l, bool x_only, cudaStream_t s) {
+  const LevelLayout& L = c->lay.lv[(size_t)l];
+  const DevLevel& d = c->dl[(size_t)l];
+  if (L.n_ghost == 0) return cudaSuccess;
+  const size_t off = (size_t)L.n_owned * c->lay.BV, bytes = (size_t)L.n_ghost * c->lay.BV * sizeof(double);
+  double* f[6] = {d.x[0], d.x[1], d.b, d.r, d.Ax, d.cf};
+  for (int k = 0; k < (x_only ? 2 : 6); ++k) {
+    if (!f[k]) continue;
+    cudaError_t e = cudaMemsetAsync(f[k] + off, 0xff, bytes, s);  // all-ones: a NaN
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
+}
+
 mg_status init_ctx(mg_ctx* c, const mg_params& p, int rank, int world, int device, cudaStream_t stream,
                    void* workspace, size_t ws_bytes, bool tables_only_upload) {
   std::string msg;
@@ -882,6 +903,8 @@ mg_status init_ctx(mg_ctx* c, const mg_params& p, int rank, int world, int devic
   c->peer_ws[(size_t)rank] = (char*)workspace;
   (void)tables_only_upload;
   CKC(c, cudaMemsetAsync(workspace, 0, need, stream));
+  if (poison_ghosts_on())
+    for (int l = 0; l < c->lay.L; ++l) CKC(c, poison_ghosts(c, l, false, stream));
   for (int l = 0; l < c->lay.L; ++l) {
     const LevelLayout& L = c->lay.lv[l];
     DevLevel& d = c->dl[l];
@@ -1170,6 +1193,7 @@ mg_status mg_set_solution(mg_ctx* c, const double* x_dev) {
   if (!x_dev) {
     const LevelLayout& L = c->lay.lv[0];
     CKC(c, cudaMemsetAsync(c->dl[0].x[c->st[0].cur], 0, (size_t)L.n_stored * c->lay.BV * sizeof(double), c->stream));
+    if (poison_ghosts_on()) CKC(c, poison_ghosts(c, 0, true, c->stream));
     c->st[0].dx = 0;
     return MG_OK;
   }
