@@ -29,8 +29,20 @@ int Builder::period(int l) const {
   // owned bricks -- costs less than the redundant ghost-shell sweeping a longer period needs; the
   // coarser levels are better at 8 (fewer launches).  NCCL moves whole bricks: period 8.
   const bool box = lay.p.transport != MG_TRANSPORT_NCCL;
-  static const int nl2 = getenv("MG_CA2_LEVELS") ? atoi(getenv("MG_CA2_LEVELS")) : 1;  // (experiments)
-  return (l < nl2 && box) ? std::min(2, lay.E) : lay.E;
+  if (box)
+    if (const char* e = getenv("MG_CA_AUTO")) {  // (experiments) per-level auto periods "k0,k1,..."
+      int k = 0, i = 0;
+      for (const char* q = e; *q; ++q) {
+        if (*q == ',') {
+          if (i++ == l) break;
+          k = 0;
+        } else {
+          k = 10 * k + (*q - '0');
+        }
+      }
+      if (i == l && k > 0) return std::min(k, lay.E);
+    }
+  return (l == 0 && box) ? std::min(2, lay.E) : lay.E;
 }
 
 int Builder::xdepth(int l) const {
