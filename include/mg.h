@@ -358,6 +358,10 @@ mg_status mg_layout_repl(const mg_layout* lay, int64_t info[2], int32_t* gb_src,
  * mg_vcycle_launches gives on a GPU (exchanges: one copy kernel each if local_exchange, none of
  * ours over NCCL). */
 mg_status mg_layout_vcycle_launches(const mg_layout* lay, int32_t local_exchange, int64_t* out);
+/* mg_exchange_plan for the first V-cycle of a fresh context with this layout (host-only): per level
+ * l < cap, the exchanges of the cycle and the bytes one exchange of x sends (the copy transports move
+ * only the ghost cells within the level's CA period of the owned box; NCCL whole bricks). */
+mg_status mg_layout_exchange_plan(const mg_layout* lay, int32_t cap, int64_t* exchanges, int64_t* bytes);
 mg_status mg_layout_destroy(mg_layout* lay);
 
 #ifdef __cplusplus

@@ -383,10 +383,10 @@ int exch_depth(const mg_ctx* c, int l) { return Builder(c->lay).xdepth(l); }
 
 // the cells per brick an exchange of x or b copies for a run of ghost direction r.dir: a sub-box
 // [lo, hi) per axis, the whole brick when the exchange depth is the brick edge; returns the count
-int64_t exch_box(const mg_ctx* c, int l, const Run& r, int32_t* box) {
-  const int E = c->lay.E, dep = exch_depth(c, l);
+int64_t exch_box(const Layout& lay, int l, const Run& r, int32_t* box) {
+  const int E = lay.E, dep = Builder(lay).xdepth(l);
   *box = 0;
-  if (dep >= E) return c->lay.BV;
+  if (dep >= E) return lay.BV;
   int dd[3], lo[3], hi[3];
   dir_from_index(r.dir, dd[0], dd[1], dd[2]);
   int64_t cells = 1;
@@ -489,7 +489,7 @@ mg_status fill_copy_tables(mg_ctx* c) {
         if (c->use_peer)  // the sender's field at the same workspace offset, through its IPC mapping
           sf = (const double*)(c->peer_ws[(size_t)r.peer] + ((const char*)f - (const char*)c->peer_ws[(size_t)c->lay.rank]));
         CopyRun cr{sf + r.remote * bb, f + r.local * bb, (int64_t)r.count * (int64_t)bb};
-        const int64_t cells = fv < 3 ? exch_box(c, l, r, &cr.box) : (int64_t)bb;
+        const int64_t cells = fv < 3 ? exch_box(c->lay, l, r, &cr.box) : (int64_t)bb;
         h[(size_t)fv * d.ncruns + i] = cr;
         d.cmax = std::max<int64_t>(d.cmax, (int64_t)r.count * cells);
       }
@@ -1368,7 +1368,7 @@ mg_status mg_exchange_stats(mg_ctx* c, int64_t* bytes_per_cycle, int64_t* messag
     if (!ex) continue;
     for (const Run& r : c->lay.lv[o.level].sends) {
       int32_t box;
-      bytes += r.count * exch_box(c, o.level, r, &box) * (int64_t)sizeof(double);
+      bytes += r.count * exch_box(c->lay, o.level, r, &box) * (int64_t)sizeof(double);
       ++msgs;
     }
   }
@@ -1377,20 +1377,27 @@ mg_status mg_exchange_stats(mg_ctx* c, int64_t* bytes_per_cycle, int64_t* messag
   return MG_OK;
 }
 
-mg_status mg_exchange_plan(mg_ctx* c, int32_t cap, int64_t* exchanges, int64_t* bytes) {
-  CKS(check_ctx(c));
-  if (cap < c->lay.L || !exchanges || !bytes) return set_err(MG_ERR_INVALID_ARG, "need cap >= num_levels and outputs");
-  Builder b(c->lay);
-  for (int l = 0; l < MG_MAX_LEVELS; ++l) b.st[l] = c->st[l];
+// per level: exchanges in the cycle the builder compiles from state st (NULL: a fresh context's), and
+// the bytes one exchange of x sends
+static void exchange_plan_of(const Layout& lay, const LevelState* st, int64_t* exchanges, int64_t* bytes) {
+  Builder b(lay);
+  if (st)
+    for (int l = 0; l < MG_MAX_LEVELS; ++l) b.st[l] = st[l];
   b.vcycle();
-  for (int l = 0; l < c->lay.L; ++l) {
+  for (int l = 0; l < lay.L; ++l) {
     exchanges[l] = 0;
     bytes[l] = 0;
     int32_t box;
-    for (const Run& r : c->lay.lv[l].sends) bytes[l] += r.count * exch_box(c, l, r, &box) * (int64_t)sizeof(double);
+    for (const Run& r : lay.lv[l].sends) bytes[l] += r.count * exch_box(lay, l, r, &box) * (int64_t)sizeof(double);
   }
   for (const Op& o : b.ops)
     if (o.kind == OP_EXCH || ((o.kind == OP_SWEEP || o.kind == OP_SWEEP2) && o.exch_before)) ++exchanges[o.level];
+}
+
+mg_status mg_exchange_plan(mg_ctx* c, int32_t cap, int64_t* exchanges, int64_t* bytes) {
+  CKS(check_ctx(c));
+  if (cap < c->lay.L || !exchanges || !bytes) return set_err(MG_ERR_INVALID_ARG, "need cap >= num_levels and outputs");
+  exchange_plan_of(c->lay, c->st, exchanges, bytes);
   return MG_OK;
 }
 
@@ -1870,6 +1877,13 @@ mg_status mg_layout_vcycle_launches(const mg_layout* m, int32_t local_exchange, 
   int64_t n = 0;
   for (const Op& o : b.ops) n += op_launches(o, m->lay, m->lay.p.overlap != 0, pencil_overlap, local_exchange != 0);
   *out = n;
+  return MG_OK;
+}
+
+mg_status mg_layout_exchange_plan(const mg_layout* m, int32_t cap, int64_t* exchanges, int64_t* bytes) {
+  if (!m || !exchanges || !bytes) return set_err(MG_ERR_INVALID_ARG, "null argument");
+  if (cap < m->lay.L) return set_err(MG_ERR_INVALID_ARG, "need cap >= num_levels");
+  exchange_plan_of(m->lay, nullptr, exchanges, bytes);
   return MG_OK;
 }
 

@@ -132,6 +132,8 @@ _SIGS = {
     "mg_layout_repl": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
                                       ctypes.c_void_p]),
     "mg_layout_vcycle_launches": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.POINTER(ctypes.c_int64)]),
+    "mg_layout_exchange_plan": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.POINTER(ctypes.c_int64),
+                                               ctypes.POINTER(ctypes.c_int64)]),
     "mg_layout_destroy": (ctypes.c_int, [ctypes.c_void_p]),
 }
 
@@ -477,6 +479,13 @@ class Layout:
                   "mg_layout_pass_plan")
             out.append((info[0], info[1], info[2], meta[:info[3]], ctas[:info[4]].reshape(-1, 2), info[5]))
         return out
+
+    def exchange_plan(self):
+        """(exchanges per level, bytes per x-exchange per level) of a fresh context's first V-cycle."""
+        n = self.p.num_levels
+        ex, by = (ctypes.c_int64 * n)(), (ctypes.c_int64 * n)()
+        check(lib().mg_layout_exchange_plan(self.h, n, ex, by), "mg_layout_exchange_plan")
+        return list(ex), list(by)
 
     def vcycle_launches(self, local_exchange=True) -> int:
         """Own kernel launches of one V-cycle (mg_layout_vcycle_launches)."""

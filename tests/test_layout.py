@@ -440,3 +440,31 @@ def test_brick4_params():
               mg.params((16, 16, 16), num_levels=2, brick_edge=4, bottom_solver=1)):
         with pytest.raises(mg.MGError):
             mg.mg_workspace_bytes(p, 0, 1)
+
+
+@pytest.mark.parametrize("n,L", [(64, 3), (128, 4)])
+@pytest.mark.parametrize("transport", [mg.MG_TRANSPORT_LOCAL, mg.MG_TRANSPORT_PEER, mg.MG_TRANSPORT_NCCL])
+@pytest.mark.parametrize("period", [0, 1, 3, 8])
+def test_depth_limited_exchange_bytes(n, L, transport, period):
+    """Bytes one x-exchange sends (the schedule's own plan, host-only): with a ghost shell on every axis a
+    copy transport (local, peer) moves exactly the ghost cells within the CA period d of the owned box,
+    ((n + 2 d)^3 - n^3) * 8 B (faces d planes, edges d x d columns, corners d^3), NCCL the whole one-brick
+    shell ((n + 16)^3 - n^3) * 8 B; the auto period is 2 at level 0 and 8 below."""
+    p = mg.params((n, n, n), num_levels=L, ghost_mode=1, transport=transport,
+                  ca_period=period if period else None)
+    lay = mg.Layout(p, 0, 1)
+    exchanges, nbytes = lay.exchange_plan()
+    for l in range(L):
+        nl = n >> l
+        if l == L - 1:  # the replicated bottom gathers the coarsest level: no ghost exchange of x
+            assert exchanges[l] == 0
+            continue
+        d = period if period else (2 if l == 0 else 8)
+        if transport == mg.MG_TRANSPORT_NCCL:
+            d = 8
+        assert nbytes[l] == ((nl + 2 * d) ** 3 - nl ** 3) * 8, (l, d)
+        assert exchanges[l] > 0
+    # two-sweep pencil passes at level 0 (128^3): one exchange of two cell layers before each of the 12
+    # passes at the auto period 2
+    if n == 128 and transport != mg.MG_TRANSPORT_NCCL and period == 0:
+        assert exchanges[0] == 12

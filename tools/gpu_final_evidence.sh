@@ -19,3 +19,6 @@ for v in "varcoef --var-coef" "brick4 --brick-edge 4" "dirichlet --bc 1" "paper 
 done
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:sweep2p_kernel -s 2 -c 1 \
    -o gpurun_out/fin/prof_pass -f python bench.py $A > gpurun_out/fin/ncu_full.log 2>&1; echo "full rc=$?"
+if [ "${CONFIGS:-0}" = "1" ]; then
+  timeout 1800 python tools/config_sweep.py --out gpurun_out/fin/configs.json > gpurun_out/fin/configs.log 2>&1; echo "configs rc=$?"
+fi
