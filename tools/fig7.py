@@ -14,6 +14,7 @@ import csv
 import io
 import json
 import os
+import re
 import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
@@ -65,6 +66,8 @@ def read_csv(path):
 
 def classify(name):
     name = name[5:] if name.startswith("void ") else name
+    # (the one-brick sweep kernel's thread-count template argument does not change the operation)
+    name = re.sub(r"^sweep_kernel<(\d+), (\d+), \d+>", r"sweep_kernel<\1, \2>", name)
     for pre, op, b in B_PER_PT:
         if name.startswith(pre):
             return op, b
