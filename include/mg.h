@@ -129,7 +129,9 @@ typedef struct {
                                     cluster = the coarse levels run in one cluster launch, grid = the
                                     ghost-free levels of <= 512 bricks run in one launch of one CTA per
                                     SM with grid barriers between dependent steps) */
-  int32_t overlap;               /* 1 = sweep interior bricks while the exchange is in flight */
+  int32_t overlap;               /* 1 = sweep interior bricks while the exchange is in flight
+                                    (single-sweep levels; the two-sweep pencil passes only with
+                                    MG_PENCIL_OVERLAP=1, measured slower by default: DESIGN.md §9) */
   int32_t sweep_kernel;          /* 0 = auto (streaming column kernel on levels >= 16384 bricks),
                                     1 = one-brick-per-CTA kernel only, 2 = streaming kernel on every level */
   int32_t temporal_blocking;     /* two Jacobi sweeps per HBM pass (bit-identical): 3 = over 2x2-brick pencils

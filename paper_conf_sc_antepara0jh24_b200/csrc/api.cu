@@ -863,6 +863,16 @@ mg_status vcycle_impl(mg_ctx* c, mg_group* g) {
   return MG_OK;
 }
 
+// Pencil passes with the exchange overlapped (the units that read no ghost brick swept while the exchange
+// runs, the rest after it): off by default -- measured on one B200 with the 2x2x2 halo pattern (peer
+// kernel or local copies), the split costs 1.0-1.2 ms per 512^3 cycle (two launches per pass, part 1 on
+// fewer CTAs, part 2's tail), more than the 12 depth-limited level-0 exchanges it could hide (~0.5 ms
+// over NVLink).  MG_PENCIL_OVERLAP=1 turns it on.
+bool pencil_overlap_on() {
+  const char* e = getenv("MG_PENCIL_OVERLAP");
+  return e && atoi(e) != 0;
+}
+
 // MG_POISON_GHOSTS=1 (tests): every ghost cell of every field starts as NaN (and x's ghosts again after
 // mg_set_solution(NULL)), so a kernel reading a ghost cell the exchange did not refresh -- a cell
 // beyond the exchange depth, or one stale since the last exchange -- poisons the owned results
@@ -892,8 +902,7 @@ mg_status init_ctx(mg_ctx* c, const mg_params& p, int rank, int world, int devic
   c->device = device;
   c->stream = stream;
   c->use_col = p.sweep_kernel != 1;
-  c->pencil_overlap = world > 1 && p.transport != MG_TRANSPORT_LOCAL;
-  if (const char* e = getenv("MG_PENCIL_OVERLAP")) c->pencil_overlap = atoi(e) != 0;
+  c->pencil_overlap = pencil_overlap_on();
   const size_t need = carve(c->lay, nullptr, nullptr, nullptr, nullptr);
   if (!workspace || ws_bytes < need)
     return set_err(MG_ERR_OOM, "workspace too small: need " + std::to_string(need) + " bytes");
@@ -1873,7 +1882,7 @@ mg_status mg_layout_vcycle_launches(const mg_layout* m, int32_t local_exchange, 
   if (!m || !out) return set_err(MG_ERR_INVALID_ARG, "null argument");
   Builder b(m->lay);
   b.vcycle();  // from the state of a fresh context (every level's ghosts stale)
-  const bool pencil_overlap = m->lay.world > 1 && m->lay.p.transport != MG_TRANSPORT_LOCAL;
+  const bool pencil_overlap = pencil_overlap_on();
   int64_t n = 0;
   for (const Op& o : b.ops) n += op_launches(o, m->lay, m->lay.p.overlap != 0, pencil_overlap, local_exchange != 0);
   *out = n;
