@@ -849,7 +849,8 @@ def test_exchange_plan_and_timing_keep_the_bits(oracle_mod, transport):
 
 
 @pytest.mark.parametrize("args", ["32 32 32 2 1 1 3 2 0", "16 16 16 2 2 1 2 2 0", "32 32 32 2 1 1 3 1 1",
-                                  "16 16 16 2 2 2 2 2 0", "32 32 32 2 1 1 3 2 0 1", "16 16 32 2 2 2 2 2 1 2"])
+                                  "16 16 16 2 2 2 2 2 0", "32 32 32 2 1 1 3 2 0 1", "16 16 32 2 2 2 2 2 1 2",
+                                  "128 128 128 2 1 1 3 2 0 0 pencil-overlap", "128 128 128 2 2 1 3 2 0 0 pencil-overlap"])
 def test_peer_transport_multiprocess_bitwise(args):
     """The peer-memory transport between PROCESSES (CUDA IPC mappings, device-side ready/done flags, the
     norm's max and the replicated bottom's gather over peer memory): torchrun starts one process per
@@ -862,11 +863,15 @@ def test_peer_transport_multiprocess_bitwise(args):
 
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
     a = args.split()
+    env = dict(os.environ)
+    if a[-1] == "pencil-overlap":  # the pencil passes' exchange overlap (units without ghosts first)
+        a = a[:-1]
+        env["MG_PENCIL_OVERLAP"] = "1"
     nproc = int(a[3]) * int(a[4]) * int(a[5])
     with socket.socket() as sk:
         sk.bind(("127.0.0.1", 0))
         port = sk.getsockname()[1]
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={nproc}",
            "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.join(root, "tools", "peer_check.py"), *a]
-    r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, cwd=root)
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, cwd=root, env=env)
     assert r.returncode == 0 and "peer_check ok" in r.stdout, (r.stdout[-2000:], r.stderr[-3000:])
