@@ -1,6 +1,6 @@
 """One small V-cycle through the C ABI for compute-sanitizer (tools/gpu_sanitize.sh).
 
-python tools/sanitize_run.py N L SWEEP_KERNEL TB [GHOST_MODE] [bc=B] [vc=1] [E=4]
+python tools/sanitize_run.py N L SWEEP_KERNEL TB [GHOST_MODE] [bc=B] [vc=1] [E=4] [tr=T] [ca=K]
 Runs one V-cycle (no graph: each kernel is launched and checked on its own) and the residual norm
 on an N^3 grid with L levels, sweep_kernel / temporal_blocking as given (sweep_kernel 2 forces the
 streaming / two-sweep kernels on every level), and checks x against the CPU oracle bit for bit.
@@ -24,11 +24,12 @@ def main():
     kv = dict(a.split("=") for a in sys.argv[5:] if "=" in a)
     gm = int(pos[0]) if pos else 0
     bc, vc, E = int(kv.get("bc", 0)), int(kv.get("vc", 0)), int(kv.get("E", 0))
+    tr, ca = int(kv.get("tr", 0)), int(kv.get("ca", 0))  # transport (3: peer kernel), CA period
     shape = (n, n, n)
     b = mg_inputs.random_rhs(shape, 0)
     c = mg_inputs.random_coef(shape, 0) if vc else None
     m = Multigrid(shape, num_levels=L, use_graph=False, sweep_kernel=sk, temporal_blocking=tb, ghost_mode=gm,
-                  bc=bc, var_coef=vc, brick_edge=E)
+                  bc=bc, var_coef=vc, brick_edge=E, transport=tr, ca_period=ca or None)
     if vc:
         m.set_coefficients(torch.from_numpy(c).cuda())
     m.set_rhs(torch.from_numpy(b).cuda())
