@@ -468,3 +468,21 @@ def test_depth_limited_exchange_bytes(n, L, transport, period):
     # passes at the auto period 2
     if n == 128 and transport != mg.MG_TRANSPORT_NCCL and period == 0:
         assert exchanges[0] == 12
+
+
+@pytest.mark.parametrize("pg", [(2, 1, 1), (2, 2, 1), (2, 2, 2), (1, 2, 3)])
+def test_depth_limited_exchange_bytes_decomposed(pg):
+    """Every rank of a decomposition sends, per x-exchange, exactly the cells the peers' ghost regions
+    within the CA period d need: the ghost shell of the decomposed axes only, ((n + 2 d_a) product) - n^3
+    with d_a = d on decomposed axes and 0 on the wrapped ones (level 0 at the auto period 2 on the
+    peer transport; level 1 whole bricks, d = 8)."""
+    n = 64
+    p = mg.params((n, n, n), pg, num_levels=3, transport=mg.MG_TRANSPORT_PEER)
+    world = pg[0] * pg[1] * pg[2]
+    for r in range(world):
+        lay = mg.Layout(p, r, world)
+        _, nbytes = lay.exchange_plan()
+        for l, d in ((0, 2), (1, 8)):
+            nl = n >> l
+            ext = np.prod([nl + (2 * d if g > 1 else 0) for g in pg])
+            assert nbytes[l] == (ext - nl ** 3) * 8, (r, l)
