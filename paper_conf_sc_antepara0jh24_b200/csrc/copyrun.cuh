@@ -29,26 +29,24 @@ __device__ __forceinline__ void copy_run_body(const CopyRun& r, int64_t i0, int6
   const int ly = (r.box >> 8) & 15, ny = ((r.box >> 12) & 15) - ly;
   const int lz = (r.box >> 16) & 15, nz = ((r.box >> 20) & 15) - lz;
   const int E = (r.box >> 24) & 15, BV = E * E * E;
-  const int64_t nb = r.n / BV;
+  // 32-bit index arithmetic (a run holds at most a few thousand bricks of <= 512 cells: < 2^31 items);
+  // 64-bit division costs an order of magnitude more instructions than the copy itself
+  const unsigned nb = (unsigned)(r.n / BV), st = (unsigned)step;
   if (((lx | nx) & 1) == 0) {  // 16-byte words
-    const int w = nx >> 1, per = w * ny * nz;
-    const int64_t total = nb * per;
-    for (int64_t i = i0; i < total; i += step) {
-      const int64_t b = i / per;
-      const int q = (int)(i - b * per);
-      const int ix = q % w, t = q / w, iy = t % ny, iz = t / ny;
-      const int64_t off = b * BV + ((int64_t)(lz + iz) * E + (ly + iy)) * E + lx + 2 * ix;
+    const unsigned w = (unsigned)nx >> 1, per = w * (unsigned)(ny * nz), total = nb * per;
+    for (unsigned i = (unsigned)i0; i < total; i += st) {
+      const unsigned b = i / per, q = i - b * per;
+      const unsigned ix = q % w, t = q / w, iy = t % (unsigned)ny, iz = t / (unsigned)ny;
+      const int64_t off = (int64_t)b * BV + (int)(((lz + iz) * E + (ly + iy)) * E + lx + 2 * ix);
       const double2* s = reinterpret_cast<const double2*>(r.src + off);
       *reinterpret_cast<double2*>(r.dst + off) = REMOTE ? *s : __ldg(s);
     }
   } else {
-    const int per = nx * ny * nz;
-    const int64_t total = nb * per;
-    for (int64_t i = i0; i < total; i += step) {
-      const int64_t b = i / per;
-      const int q = (int)(i - b * per);
-      const int ix = q % nx, t = q / nx, iy = t % ny, iz = t / ny;
-      const int64_t off = b * BV + ((int64_t)(lz + iz) * E + (ly + iy)) * E + lx + ix;
+    const unsigned per = (unsigned)(nx * ny * nz), total = nb * per;
+    for (unsigned i = (unsigned)i0; i < total; i += st) {
+      const unsigned b = i / per, q = i - b * per;
+      const unsigned ix = q % (unsigned)nx, t = q / (unsigned)nx, iy = t % (unsigned)ny, iz = t / (unsigned)ny;
+      const int64_t off = (int64_t)b * BV + (int)(((lz + iz) * E + (ly + iy)) * E + lx + ix);
       r.dst[off] = REMOTE ? r.src[off] : __ldg(r.src + off);
     }
   }

@@ -33,8 +33,11 @@ def samples(runs):
             nl = n >> lvl
             name = OPS[op]
             if name == "exchange":
-                nb = nl // 8
-                x = ((nb + 2) ** 3 - nb ** 3) * 4096.0 if gm == 1 else None
+                # bytes of one x-exchange: the ghost cells within the exchange depth d of the owned box
+                # (the copy transports move only those; NCCL whole bricks, d = 8)
+                k = (r.get("ca_period") or [0] * 16)[lvl]
+                d = 8 if r.get("transport") == 1 else min(k if k else (2 if lvl == 0 else 8), 8)
+                x = ((nl + 2 * d) ** 3 - nl ** 3) * 8.0 if gm == 1 else None
             elif name == "bottom":
                 if nbot > 1:  # one record per bottom sweep (launched sweeps)
                     name, x = "bottom_sweep", float(nl ** 3)
