@@ -652,7 +652,48 @@ static LevelLayout::PairTable pencil_table(const LevelLayout& L, int64_t b0, int
     const int64_t cost = *std::max_element(cta.begin(), cta.end());
     if (cost < best_cost) best_cost = cost, best = nzr;
   }
+  // Second candidate (whole range only): runs of Lmax layers plus each column's remainder run, dealt
+  // band by band (z-run-major, column-minor, as above) to the least-loaded CTA (ties: the lowest
+  // index, so a band's long runs still land on consecutive CTAs).  When the columns' layers do not
+  // split evenly over the CTAs (level 1 at 512^3: 256 columns of 32 layers on 888 CTAs), one long
+  // run per CTA and the short remainders on the CTAs left over beat equal runs dealt round-robin
+  // (busiest CTA 41 instead of 43 quarter layers).
+  struct HRun {
+    int64_t col;
+    int z0, len;
+  };
+  std::vector<std::vector<HRun>> hybrid;
+  // (only when it trims the busiest CTA by >= 2%: level 0's equal runs keep their exact banding)
+  const int64_t equal_cost = best_cost;
   if (part == 0) {
+    for (int lmax = 1; lmax < nz; ++lmax) {
+      std::vector<HRun> runs;
+      for (int z0 = 0; z0 < nz; z0 += lmax)
+        for (int64_t col = 0; col < ncol; ++col) runs.push_back({col, z0, std::min(lmax, nz - z0)});
+      std::vector<int64_t> load((size_t)G, 0);
+      std::vector<std::vector<HRun>> deal((size_t)G);
+      // least-loaded CTA, lowest index first (loads only grow: a simple scan stays O(runs x G) on
+      // the host at setup; G <= 888)
+      int64_t worst = 0;
+      for (const HRun& r : runs) {
+        size_t g = 0;
+        for (size_t q = 1; q < (size_t)G; ++q)
+          if (load[q] < load[g]) g = q;
+        load[g] += 4 * r.len + 1;
+        worst = std::max(worst, load[g]);
+        deal[g].push_back(r);
+        if (worst >= best_cost) break;
+      }
+      if (worst < best_cost && 50 * worst <= 49 * equal_cost) {
+        best_cost = worst;
+        hybrid = std::move(deal);
+      }
+    }
+  }
+  if (part == 0 && !hybrid.empty()) {
+    for (int64_t g = 0; g < G; ++g)
+      for (const HRun& r : hybrid[(size_t)g]) push_run(stream[(size_t)g], r.col, r.z0, r.len);
+  } else if (part == 0) {
     for (int64_t u = 0; u < ncol * best; ++u) {
       const int r = (int)(u / ncol);
       const int64_t col = u % ncol;
