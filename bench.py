@@ -278,6 +278,7 @@ def exchange_block(m, a, world, max_over_ranks, tm, ninst):
     t = alpha + bytes / beta over the levels (P:L216-236, N3) and the Table-II-style share of the
     exchanges in the level time (P:L198-206)."""
     counts, nbytes = m.exchange_plan()
+    fused = m.exchange_fused()  # of which: fused into the pencil pass after them (no exchange kernel)
     if not any(nbytes):
         return {"levels": [], "note": "no ghost shell (one rank, periodic wrap): no exchanges"}
     transport = {mg.MG_TRANSPORT_NCCL: "nccl", mg.MG_TRANSPORT_PEER: "peer memory (CUDA IPC, device flags)"}.get(
@@ -289,10 +290,11 @@ def exchange_block(m, a, world, max_over_ranks, tm, ninst):
         t = max_over_ranks(m.exchange_time(l, 20))
         gbs = b / (t / 1e3) / 1e9 if t > 0 else None
         lvl_ms = sum(tm[l]) / ninst if l < len(tm) else None
-        out.append({"level": l, "exchanges_per_cycle": c, "bytes_per_exchange": b, "ms_per_exchange": t,
+        out.append({"level": l, "exchanges_per_cycle": c, "fused_into_pencil_pass": fused[l],
+                    "bytes_per_exchange": b, "ms_per_exchange": t,
                     "gbs": gbs, "frac_of_nvlink_900": (gbs / NVLINK_GBS) if (gbs and world > 1) else None,
-                    "ms_per_cycle_if_serial": c * t,
-                    "share_of_level_time": (c * t / lvl_ms) if lvl_ms else None})
+                    "ms_per_cycle_if_serial": (c - fused[l]) * t,
+                    "share_of_level_time": ((c - fused[l]) * t / lvl_ms) if lvl_ms else None})
     fit = None
     pts = [(d["bytes_per_exchange"], d["ms_per_exchange"]) for d in out if d["ms_per_exchange"] > 0]
     if len(pts) >= 2:

@@ -266,6 +266,14 @@ mg_status mg_exchange_stats(mg_ctx* c, int64_t* bytes_per_cycle, int64_t* messag
  * (0 without a ghost shell; on the copy transports only the ghost cells within the level's CA period
  * of the owned box, whole bricks over NCCL).  Host-only, no device work. */
 mg_status mg_exchange_plan(mg_ctx* c, int32_t cap, int64_t* exchanges, int64_t* bytes);
+/* Per level l < cap: how many of mg_exchange_plan's exchanges[l] are fused into the pencil pass that
+ * follows them (DESIGN.md §9 "fused exchange"): the pass stages its ghost bricks' x straight from the
+ * owners' fields (peer memory between processes, the other contexts of a loopback group, or the own
+ * field for a one-rank self-exchange) instead of a separate exchange kernel; between processes a
+ * flag handshake kernel (no data) precedes the pass.  Only levels with a pencil plan over the owned
+ * range, a periodic box and constant coefficients, on the copy transports (not NCCL); off with
+ * MG_NO_FUSED_EXCH=1.  Host-only, no device work. */
+mg_status mg_exchange_fused(mg_ctx* c, int32_t cap, int64_t* fused);
 /* Device time of one ghost exchange of x at `level` (the V-cycle's transport: NCCL grouped
  * send/recv of the brick runs, or the local copy kernel), averaged over `reps` back-to-back
  * exchanges on the context's stream after one warm-up exchange (CUDA events; synchronises).

@@ -74,6 +74,13 @@ struct DevLevel {
   int32_t* mirror = nullptr;
   int nmirror = 0;
   double mirror_sign = 1.0;
+  // the exchange fused into the level's pencil passes (SW_PEER): ghost brick -> (owner
+  // rank, its brick id), [2 buffers][world] x base pointers and x tensor maps (xwe, xsn, xcor) of the owners
+  bool fused = false;
+  int32_t* pid = nullptr;  // [chunks of the owned pencil plan][16] (PairArgs::pid)
+  CUtensorMap* rmaps = nullptr;
+  std::vector<const double*> rbase;  // [2][rworld] (PairMaps::rbase)
+  int rworld = 0;
 };
 
 struct Plan {
@@ -467,6 +474,81 @@ mg_status fill_repl_tables(mg_ctx* c) {
 
 // Copy descriptors of the local transport: receiver ghost run <- sender surface run, for the
 // three exchanged fields (x[0], x[1], b).  Needs every rank's workspace carved (loopback groups).
+// The exchange fused into the pencil passes (SW_PEER): on a level whose owned range has a pencil plan,
+// a periodic box (no mirrored faces) and constant coefficients, a pass that would follow an x exchange
+// instead stages the side slabs, corner columns and warm-up / cool-down bricks of its ghost bricks
+// straight from the owners' fields (the receive runs say which brick of which rank a ghost mirrors).
+// MG_NO_FUSED_EXCH=1 keeps the separate exchange (A/B).
+static bool fused_exchange_on() {
+  static const bool off = getenv("MG_NO_FUSED_EXCH") != nullptr;
+  return !off;
+}
+
+static mg_status fill_fused_tables(mg_ctx* c) {
+  if (!fused_exchange_on() || c->use_nccl) return MG_OK;
+  const int W = c->group ? (int)c->group->r.size() : c->lay.world;
+  if (W > 8) return MG_OK;  // (PairMaps::rbase)
+  for (int l = 0; l < c->lay.L; ++l) {
+    const LevelLayout& L = c->lay.lv[l];
+    DevLevel& d = c->dl[l];
+    d.fused = false;
+    if (d.ncruns == 0 || L.n_ghost == 0 || d.nmirror > 0 || d.cf) continue;
+    const LevelLayout::PairTable* pt = nullptr;
+    for (const auto& t : L.pairs)
+      if (t.b0 == 0 && t.b1 == L.n_owned && t.part == 0 && t.kind == 3) pt = &t;
+    if (!pt) continue;
+    // ghost brick -> (owner rank, the owner's brick it mirrors), from the receive runs
+    std::vector<int2> g((size_t)L.n_ghost, make_int2(-1, -1));
+    for (const Run& r : L.recvs)
+      for (int64_t k = 0; k < r.count; ++k)
+        if (r.local + k >= L.n_owned && r.local + k < L.n_stored)
+          g[(size_t)(r.local + k - L.n_owned)] = make_int2(r.peer, (int)(r.remote + k));
+    const size_t nch = pt->meta.size() / kPenRec;
+    std::vector<int32_t> pid(nch * 16, -1);
+    bool ok = true;
+    for (size_t ch = 0; ch < nch && ok; ++ch)
+      for (int e = 0; e < 16; ++e) {
+        const int32_t id = pt->meta[ch * kPenRec + 1 + (size_t)e];
+        if (id < L.n_owned) continue;
+        if (id >= L.n_stored) { ok = false; break; }
+        const int2 src = g[(size_t)(id - L.n_owned)];
+        if (src.x < 0 || src.x >= W || src.y >= (1 << 24)) { ok = false; break; }
+        pid[ch * 16 + (size_t)e] = (src.x << 24) | src.y;
+      }
+    if (!ok) continue;
+    std::vector<CUtensorMap> maps((size_t)2 * W * 3);
+    d.rbase.assign((size_t)2 * W, nullptr);
+    for (int xb = 0; xb < 2; ++xb)
+      for (int r = 0; r < W; ++r) {
+        const double* f = d.x[xb];
+        if (c->group) f = c->group->r[(size_t)r]->dl[l].x[xb];
+        else if (c->use_peer)
+          f = (const double*)(c->peer_ws[(size_t)r] + ((const char*)d.x[xb] - (const char*)c->peer_ws[(size_t)c->lay.rank]));
+        else if (r != c->lay.rank) return set_err(MG_ERR_STATE, "fused exchange: no mapping of another rank");
+        PairMaps pm{};
+        CKC(c, encode_pencil_maps(f, f, L.n_alloc, &pm));
+        CUtensorMap* m = &maps[((size_t)xb * W + r) * 3];
+        m[0] = pm.xwe;
+        m[1] = pm.xsn;
+        m[2] = pm.xcor;
+        d.rbase[(size_t)xb * W + r] = f;
+      }
+    auto upload = [&](void** dst, const void* h, size_t bytes) -> mg_status {
+      if (!*dst) {
+        CKC(c, cudaMalloc(dst, bytes));
+        c->allocs.push_back(*dst);
+      }
+      CKC(c, cudaMemcpy(*dst, h, bytes, cudaMemcpyHostToDevice));
+      return MG_OK;
+    };
+    CKS(upload((void**)&d.pid, pid.data(), pid.size() * sizeof(int32_t)));
+    CKS(upload((void**)&d.rmaps, maps.data(), maps.size() * sizeof(CUtensorMap)));
+    d.rworld = W;
+    d.fused = true;
+  }
+  return MG_OK;
+}
+
 mg_status fill_copy_tables(mg_ctx* c) {
   const size_t bb = (size_t)c->lay.BV;
   for (int l = 0; l < c->lay.L; ++l) {
@@ -496,7 +578,7 @@ mg_status fill_copy_tables(mg_ctx* c) {
     }
     CKC(c, cudaMemcpy(d.cruns, h.data(), h.size() * sizeof(CopyRun), cudaMemcpyHostToDevice));
   }
-  return MG_OK;
+  return fill_fused_tables(c);
 }
 
 // ------------------------------------------------------------- executor
@@ -504,7 +586,7 @@ mg_status fill_copy_tables(mg_ctx* c) {
 // paper_stage (the paper's kernel set, in-place smooth): 0 = applyOp then smooth, 1 = applyOp only,
 // 2 = smooth only -- a split sweep must finish every applyOp before the first in-place smooth
 mg_status sweep_range(mg_ctx* c, const Op& o, int64_t b0, int64_t b1, cudaStream_t s, int part = 0,
-                      int paper_stage = 0) {
+                      int paper_stage = 0, bool peer = false) {
   if (b1 <= b0) return MG_OK;
   DevLevel& d = c->dl[o.level];
   const int l = o.level;
@@ -552,7 +634,14 @@ mg_status sweep_range(mg_ctx* c, const Op& o, int64_t b0, int64_t b1, cudaStream
   if (o.kind == OP_SWEEP2) {  // two sweeps in one pass: the builder only emits it where a plan exists
     for (const auto& pr : d.pairs) {
       if (pr.b0 == b0 && pr.b1 == b1 && pr.part == part) {
-        if (pr.args.kind == 3)
+        if (pr.args.kind == 3 && peer) {  // the exchange fused into the pass: ghost x from the owners
+          PairArgs pa = pr.args;
+          pa.pid = d.pid;
+          pa.rmaps = d.rmaps + (size_t)o.src * d.rworld * 3;
+          PairMaps pm = d.nmaps[o.src];
+          for (int r = 0; r < d.rworld; ++r) pm.rbase[r] = d.rbase[(size_t)o.src * d.rworld + r];
+          CKC(c, launch_sweep2p(a, pa, pm, o.flags | SW_PEER, s));
+        } else if (pr.args.kind == 3)
           CKC(c, launch_sweep2p(a, pr.args, d.nmaps[o.src], o.flags | (o.zero ? SW_ZERO_X : 0u), s));
         else
           CKC(c, launch_sweep2(a, pr.args, d.pmaps[o.src], o.flags, s));
@@ -595,6 +684,13 @@ mg_status exec_op(mg_ctx* c, const Op& o, cudaStream_t s) {
     case OP_SWEEP:
     case OP_SWEEP2: {
       const int64_t end = o.ghosts ? L.n_stored : L.n_owned;
+      if (o.fused) {  // the exchange fused into the pencil pass (fill_fused_tables)
+        CKS(timer_begin(c, s, &t0));
+        if (o.fused == 2) CKC(c, launch_peer_handshake(c->ps_nb, s));
+        CKS(sweep_range(c, o, 0, end, s, 0, 0, true));
+        CKS(timer_end(c, s, t0, o.level, o.timer));
+        return MG_OK;
+      }
       if (o.exch_before) {
         // pencil passes: the units that read no ghost brick overlap the exchange, the rest follow
         bool pen_split = false;
@@ -715,8 +811,10 @@ mg_status exec_op(mg_ctx* c, const Op& o, cudaStream_t s) {
       if (lay.p.bottom_solver == 1) {
         CKC(c, launch_bottom_cg(c->rp.x[1], c->rp.b, c->rp.adj, c->rp.coord, (int)ng, lay.gb.n[0], lay.gb.n[1], o.n,
                                 d.c, s));
-      } else if (ng <= kResidentMaxBricks) {
+      } else if (ng <= kResidentMaxBricks && !cluster_bottom_small()) {
         CKC(c, launch_bottom_resident(c->rp.x[0], c->rp.x[1], c->rp.b, c->rp.adj, (int)ng, o.n, true, d.c, s));
+      } else if (ng <= kClusterBottomMaxBricks && cluster_bottom_enabled()) {
+        CKC(c, launch_bottom_cluster(c->rp.x[0], c->rp.x[1], c->rp.b, c->rp.adj, (int)ng, o.n, true, d.c, s));
       } else {
         CoarseArgs a{};
         a.nlev = 1;
@@ -738,20 +836,34 @@ mg_status exec_op(mg_ctx* c, const Op& o, cudaStream_t s) {
       return MG_OK;
     case OP_BOTTOM_RES:
       CKS(timer_begin(c, s, &t0));
-      if (!L.radj.empty())  // non-periodic bc, one rank: owned bricks, domain faces as images
-        CKC(c, launch_bottom_resident(d.x[o.src], d.x[o.dst], d.b, d.radj, (int)L.n_owned, o.n, o.zero, d.c, s,
-                                      d.mirror_sign));
-      else
-        CKC(c, launch_bottom_resident(d.x[o.src], d.x[o.dst], d.b, d.adj, (int)L.n_stored, o.n, o.zero, d.c, s));
+      if (!L.radj.empty()) {  // non-periodic bc, one rank: owned bricks, domain faces as images
+        auto f = L.n_owned <= kResidentMaxBricks && !cluster_bottom_small() ? launch_bottom_resident : launch_bottom_cluster;
+        CKC(c, f(d.x[o.src], d.x[o.dst], d.b, d.radj, (int)L.n_owned, o.n, o.zero, d.c, s, d.mirror_sign));
+      } else {
+        auto f = L.n_stored <= kResidentMaxBricks && !cluster_bottom_small() ? launch_bottom_resident : launch_bottom_cluster;
+        CKC(c, f(d.x[o.src], d.x[o.dst], d.b, d.adj, (int)L.n_stored, o.n, o.zero, d.c, s, 0.0));
+      }
       CKS(timer_end(c, s, t0, o.level, o.timer));
       return MG_OK;
   }
   return set_err(MG_ERR_STATE, "unknown op");
 }
 
-Plan make_plan(const Builder& b, const Layout& lay, bool pencil_overlap, bool local_exchange) {
+Plan make_plan(const Builder& b, const Layout& lay, bool pencil_overlap, bool local_exchange,
+               const mg_ctx* c = nullptr) {
   Plan p;
   p.ops = b.ops;
+  if (c)  // pencil passes after an x exchange over the owned range of a fused-exchange level
+    for (Op& o : p.ops) {
+      const DevLevel& d = c->dl[o.level];
+      if (o.kind == OP_SWEEP2 && o.exch_before && !o.ghosts && !o.zero && o.c1 < 0 && o.c2 < 0 && d.fused &&
+          pencil_supports(o.flags) && !(lay.p.overlap && c->pencil_overlap)) {
+        bool plan = false;
+        for (const auto& pr : d.pairs)
+          plan |= pr.b0 == 0 && pr.b1 == lay.lv[o.level].n_owned && pr.part == 0 && pr.args.kind == 3;
+        if (plan) o.fused = (c->use_peer && lay.world > 1) ? 2 : 1;
+      }
+    }
   for (int l = 0; l < MG_MAX_LEVELS; ++l) p.final_st[l] = b.st[l];
   for (const Op& o : p.ops) p.launches += op_launches(o, lay, lay.p.overlap != 0, pencil_overlap, local_exchange);
   return p;
@@ -792,7 +904,7 @@ mg_status check_ctx(mg_ctx* c) {
 }
 
 mg_status build_and_run(mg_ctx* c, mg_group* g, bool vcycle_graph, Builder& b) {
-  const Plan p = make_plan(b, c->lay, c->pencil_overlap, !c->use_nccl);  // (peer: one copy kernel too)
+  const Plan p = make_plan(b, c->lay, c->pencil_overlap, !c->use_nccl, c);  // (peer: one copy kernel too)
   CKS(prepare_plan(c, g, p.ops));
   CKS(run_plan(c, g, p, g ? g->stream : c->stream));
   if (g) {
@@ -821,7 +933,7 @@ mg_status vcycle_impl(mg_ctx* c, mg_group* g) {
     Builder b(c0->lay);
     for (int l = 0; l < MG_MAX_LEVELS; ++l) b.st[l] = c0->st[l];
     b.vcycle();
-    Plan p = make_plan(b, c0->lay, c0->pencil_overlap, !c0->use_nccl);
+    Plan p = make_plan(b, c0->lay, c0->pencil_overlap, !c0->use_nccl, c0);
     CKS(prepare_plan(c0, g, p.ops));
     if (graph) {
       // capture on a private non-blocking stream; the graph is then launched on the caller's stream
@@ -1362,7 +1474,7 @@ mg_status mg_vcycle_launches(mg_ctx* c, int64_t* out) {
   Builder b(c->lay);
   for (int l = 0; l < MG_MAX_LEVELS; ++l) b.st[l] = c->st[l];
   b.vcycle();
-  *out = make_plan(b, c->lay, c->pencil_overlap, !c->use_nccl).launches;
+  *out = make_plan(b, c->lay, c->pencil_overlap, !c->use_nccl, c).launches;
   return MG_OK;
 }
 
@@ -1407,6 +1519,19 @@ mg_status mg_exchange_plan(mg_ctx* c, int32_t cap, int64_t* exchanges, int64_t* 
   CKS(check_ctx(c));
   if (cap < c->lay.L || !exchanges || !bytes) return set_err(MG_ERR_INVALID_ARG, "need cap >= num_levels and outputs");
   exchange_plan_of(c->lay, c->st, exchanges, bytes);
+  return MG_OK;
+}
+
+mg_status mg_exchange_fused(mg_ctx* c, int32_t cap, int64_t* fused) {
+  CKS(check_ctx(c));
+  if (cap < c->lay.L || !fused) return set_err(MG_ERR_INVALID_ARG, "need cap >= num_levels and an output");
+  Builder b(c->lay);
+  for (int l = 0; l < MG_MAX_LEVELS; ++l) b.st[l] = c->st[l];
+  b.vcycle();
+  const Plan p = make_plan(b, c->lay, c->pencil_overlap, !c->use_nccl, c);
+  for (int l = 0; l < c->lay.L; ++l) fused[l] = 0;
+  for (const Op& o : p.ops)
+    if (o.fused) ++fused[o.level];
   return MG_OK;
 }
 

@@ -939,6 +939,8 @@ cudaError_t kernels_init() {
   if (e != cudaSuccess) return e;
   e = coarse_kernels_init();
   if (e != cudaSuccess) return e;
+  e = bottom_cluster_init();
+  if (e != cudaSuccess) return e;
   e = cg_kernels_init();
   if (e != cudaSuccess) return e;
   return coarse_grid_init();

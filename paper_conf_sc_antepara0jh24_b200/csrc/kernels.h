@@ -24,6 +24,7 @@ enum SweepFlags : unsigned {
   SW_COLOUR = 32u,     // two-sweep kernel: red-black half-sweeps (colour masks compiled in only here)
   SW_VARCOEF = 64u,    // one-brick kernel: variable coefficients div(c grad x) (reading A23), SweepArgs::cf
   SW_NORM = 128u,      // column kernel: no stores, max |b - Ax| into SweepArgs::acc (maxNormRes)
+  SW_PEER = 256u,      // pencil kernel: x of ghost bricks read from their owners' fields (fused exchange)
 };
 
 struct SweepArgs {
@@ -79,6 +80,13 @@ struct PairArgs {
   const int2* ctas;     // (first item / chunk, count) per CTA
   int64_t nctas;
   unsigned long long* trace = nullptr;  // sweep2p measurement (MG_PEN_TRACE): per CTA (start, end) globaltimer
+  // SW_PEER (the exchange fused into the pencil pass): pid[chunk][e] for the x copies of
+  // record entries e = 0..15 (ids 1..16): -1 = the local brick, else (rank << 24) | the brick of rank's
+  // field that the ghost brick mirrors, staged through rank's x tensor maps rmaps[3 rank + 0..2] (xwe,
+  // xsn, xcor) or, for a whole half brick, from PairMaps::rbase[rank]; b stays local (its ghosts are
+  // exchanged once per level)
+  const int32_t* pid = nullptr;
+  const CUtensorMap* rmaps = nullptr;
 };
 struct PairMaps {
   CUtensorMap xwe;   // x boxes {2,8,8}: W (i=6,7) / E (i=0,1) face slabs
@@ -86,6 +94,7 @@ struct PairMaps {
   CUtensorMap xcor;  // x boxes {2,1,8}: the four diagonal-corner columns
   CUtensorMap bwe;   // b boxes {2,8,8}
   CUtensorMap bsn;   // b boxes {8,1,8}
+  const double* rbase[8] = {};  // SW_PEER (pencil kernel): x base pointer of the src buffer of rank r
 };
 cudaError_t encode_pair_maps(const double* x, const double* b, int64_t n_alloc, PairMaps* out);
 // flags apply to the SECOND sweep of the pair: plain, +r, +restriction
@@ -128,6 +137,15 @@ constexpr int kResidentMaxBricks = 8;
 cudaError_t launch_bottom_resident(const double* x, double* xo, const double* b, const int32_t* adj, int nbricks,
                                    int sweeps, bool zero_x, Coeffs c, cudaStream_t s,
                                    double msign = 0.0);
+// cluster-resident bottom solve (bottom_cluster.cu): 9 .. kClusterBottomMaxBricks bricks (no ghosts)
+// over ceil(nbricks / 8) CTAs of one cluster, the resident kernel's arithmetic and arguments
+constexpr int kClusterBottomMaxBricks = 64;
+cudaError_t launch_bottom_cluster(const double* x, double* xo, const double* b, const int32_t* adj, int nbricks,
+                                  int sweeps, bool zero_x, Coeffs c, cudaStream_t s, double msign = 0.0);
+cudaError_t bottom_cluster_init();
+// the bottom kernel for a level of nbricks: resident (<= 8), cluster (<= 64; MG_NO_CLUSTER_BOTTOM=1 for A/B)
+bool cluster_bottom_enabled();
+bool cluster_bottom_small();
 // layout conversion (not part of the V-cycle): lexicographic local <-> bricks [0, nowned)
 cudaError_t launch_lex_to_brick(const double* lex, double* bricks, const int32_t* coord, int64_t nowned, int nx,
                                 int ny, cudaStream_t s, int E = 8);
@@ -171,6 +189,8 @@ struct PeerSync {
   const CopyRun* dummy_run;           // a zero-length run (a rank without runs still takes part)
 };
 cudaError_t launch_peer_copy(const CopyRun* runs, int nruns, int64_t max_n, const PeerSync& s, cudaStream_t st);
+// ready(e) to / from every participant, no copy (the pencil passes with SW_PEER read the neighbours' x)
+cudaError_t launch_peer_handshake(const PeerSync& s, cudaStream_t st);
 // global max of the uint64 bits at *acc over the participants (+ this rank): vals = this rank's
 // [world] value slots, remote_vals[n] = rank n's value slots
 cudaError_t launch_peer_allmax(unsigned long long* acc, const PeerSync& s, unsigned long long* const* remote_vals,

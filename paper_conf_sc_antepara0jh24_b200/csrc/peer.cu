@@ -114,7 +114,29 @@ __global__ void peer_allmax_kernel(unsigned long long* acc, PeerSync s, unsigned
   pdl_trigger();
 }
 
+// Before a pencil pass that reads its ghost bricks straight from the neighbours' fields (SW_PEER, the
+// exchange fused into the pass): publish ready(e) -- this rank's x of the pass is complete, and its
+// previous pass has finished reading the neighbours' fields -- and wait for every neighbour's ready(e).
+// Then no rank reads a field its owner has not finished (RAW) and no rank overwrites, in its next
+// pass, a buffer a neighbour is still reading (WAR: the neighbour's ready(e+1) comes after its pass e).
+__global__ void peer_handshake_kernel(PeerSync s) {
+  pdl_wait();
+  if (threadIdx.x == 0) {
+    const unsigned long long e = *(volatile unsigned long long*)s.epoch + 1;
+    peer_signal(s, 0, e);
+    peer_wait(s, 0, e);
+    *s.epoch = e;
+    __threadfence();
+  }
+  pdl_trigger();
+}
+
 }  // namespace
+
+cudaError_t launch_peer_handshake(const PeerSync& s, cudaStream_t st) {
+  launch_k(peer_handshake_kernel, 1, 32, 0, st, s);
+  return cudaGetLastError();
+}
 
 cudaError_t launch_peer_copy(const CopyRun* runs, int nruns, int64_t max_n, const PeerSync& s, cudaStream_t st) {
   // every rank launches the kernel even without runs of its own (the flags keep the epochs in step)

@@ -263,8 +263,9 @@ void Builder::bottom(int l, int n, bool zero) {
   const LevelLayout& L = lay.lv[l];
   const int bm = lay.p.bottom_mode;
   // (a one-rank non-periodic level: the owned bricks with the domain faces as images, L.radj)
-  const bool can_res = (!ghosts(l) && L.n_stored <= kResidentMaxBricks) ||
-                       (!L.radj.empty() && L.n_owned <= kResidentMaxBricks);
+  // (<= 8 bricks: one CTA, resident.cuh; <= 64: one cluster, bottom_cluster.cu)
+  const int64_t max_res = cluster_bottom_enabled() ? kClusterBottomMaxBricks : kResidentMaxBricks;
+  const bool can_res = (!ghosts(l) && L.n_stored <= max_res) || (!L.radj.empty() && L.n_owned <= max_res);
   const bool res = can_res && (bm == MG_BOTTOM_RESIDENT ||
                                 ((bm == MG_BOTTOM_AUTO || bm == MG_BOTTOM_CLUSTER || bm == MG_BOTTOM_GRID) && fusion(l) != MG_FUSION_PAPER));
   const bool fold_zero = zero && fusion(l) == MG_FUSION_FULL;
@@ -395,7 +396,7 @@ int64_t op_launches(const Op& o, const Layout& lay, bool overlap, bool pencil_ov
     case OP_SWEEP2: {
       const int per = o.paper ? 2 : 1;  // applyOp + smooth(+residual)
       const int64_t end = o.ghosts ? L.n_stored : L.n_owned;
-      const int64_t x = o.exch_before ? ex : 0;
+      const int64_t x = o.fused ? o.fused - 1 : o.exch_before ? ex : 0;
       bool pen_split = false;
       if (o.kind == OP_SWEEP2 && o.exch_before && overlap && pencil_overlap)
         for (const auto& pt : L.pairs) pen_split |= pt.b0 == 0 && pt.b1 == end && pt.part == 1;

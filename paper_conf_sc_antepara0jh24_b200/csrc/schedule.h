@@ -42,6 +42,9 @@ struct Op {
   double g1 = 0, g2 = 0;    // smoothing steps of the (first, second) sweep; 0 = the level's Jacobi h^2/12
   int c1 = -1, c2 = -1;     // red-black colour of the (first, second) half-sweep (GSRB); -1 = every cell
   bool nosplit = false;     // exchange before the whole sweep (pencil passes: no interior / surface split)
+  int fused = 0;            // OP_SWEEP2 with exch_before over the owned range: the exchange fused into the
+                            // pencil pass (SW_PEER; set by the executor's plan): 1 no sync needed (one
+                            // rank / a lockstep group), 2 after a peer handshake kernel (processes)
 };
 
 struct LevelState {

@@ -82,6 +82,7 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
   constexpr bool RESTRICT = (FLAGS & SW_RESTRICT) != 0;
   constexpr bool COLOUR = (FLAGS & SW_COLOUR) != 0;  // red-black half-sweeps (GSRB variant)
   constexpr bool ZX = (FLAGS & SW_ZERO_X) != 0;      // x0 == 0: initZero folded into the first sweep
+  constexpr bool PEER = (FLAGS & SW_PEER) != 0;      // x of ghost bricks from their owners' fields
   constexpr unsigned FULL = 0xffffffffu;
   constexpr int RANGE = 0, WARM = 1, COOL = 2;
   // x0 read from the stage, or 0 (ZX: nothing of x0 is staged; every sweep-1 operand is +0, so the
@@ -181,6 +182,13 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
   // bricks' half (1D bulk) and the 8 x0 side slabs; warp 1: the 8 b faces, the 4 corner columns
   // and (lane 12) the record of the chunk after ----
   int issued = 0;
+  // PEER: this lane's entry of the chunk's peer ids (warp 0 lanes 0-11: own bricks, side slabs; warp 1
+  // lanes 8-11: corner columns), the one of the chunk to issue next held in a register
+  const bool xlane = (w == 0 && l < 12) || (w == 1 && l >= 8 && l < 12);
+  auto pid_load = [&](int n) -> int {
+    return (PEER && xlane && n < cnt) ? __ldg(pa.pid + ((int64_t)(cr.x + n) * 16 + (w == 0 ? l : l + 4))) : -1;
+  };
+  int pid_cur = pid_load(0);
   auto issue = [&]() {  // both warps (uniform): stage chunk `issued`
     const int n = issued, s = n % PN_ST, code = mr(n, 0), half = code & 1;
     const bool rec = n + 1 >= 2 && n + 1 < cnt;
@@ -192,16 +200,35 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
                                      : 4 * 512 + 4 * 256 + (ZX ? 0 : 4 * 64) + (rec ? kPenRec * 4 : 0));
     __syncwarp();
     const int kz = id * 8 + 4 * half;
+    // x source of this lane's copy: the local field, or (PEER, a ghost brick) its owner's field; the
+    // entry's peer id was loaded one chunk ahead (no dependent load in the issue)
+    int xid = id;
+    const CUtensorMap* xmaps = &mp.xwe;  // xwe, xsn, xcor (consecutive in PairMaps and in rmaps)
+    bool remote = false;
+    int pid_rank = 0;
+    if (PEER) {
+      const int pv = pid_cur;
+      pid_cur = pid_load(n + 1);
+      if (pv >= 0) {
+        remote = true;
+        pid_rank = pv >> 24;
+        xid = pv & 0xffffff;
+        xmaps = pa.rmaps + 3 * (pv >> 24);
+      }
+    }
+    const int xkz = xid * 8 + 4 * half;
     if (w == 0) {
       if (ZX) {
         // nothing of x0 is staged
+      } else if (PEER && remote && l < 4) {  // the owner's half brick
+        tma_load_1d(D + OWN_STRIDE * l, mp.rbase[pid_rank] + (int64_t)xid * 512 + 256 * half, 2048, &BAR[s]);
       } else if (l < 4) {
         // evict_last: the neighbour tiles' slab copies read these bricks' faces shortly after
         tma_load_1d_hint(D + OWN_STRIDE * l, p.x + (int64_t)id * 512 + 256 * half, 2048, &BAR[s], pol_keep);
       } else if (l < 12) {
         const bool xf = l < 8, lowside = ((l - 4) & 2) == 0;  // W / S boxes sit at the high face
-        tma_load_3d(D + XW + 64 * (l - 4), xf ? &mp.xwe : &mp.xsn, xf && lowside ? 6 : 0,
-                    !xf && lowside ? 6 : 0, kz, &BAR[s]);
+        tma_load_3d(D + XW + 64 * (l - 4), xf ? xmaps : xmaps + 1, xf && lowside ? 6 : 0,
+                    !xf && lowside ? 6 : 0, xkz, &BAR[s]);
       }
     } else {
       if (l < 4) {
@@ -210,7 +237,7 @@ __global__ void __launch_bounds__(PN_THREADS, PN_MINB)
         tma_load_3d(D + BS + 32 * (l - 4), &mp.bsn, 0, l < 6 ? 7 : 0, kz, &BAR[s]);
       } else if (l < 12) {  // SW (6,7), NW (6,0), SE (0,7), NE (0,0)
         const int cc = l - 8;
-        if (!ZX) tma_load_3d(D + COR + 16 * cc, &mp.xcor, cc < 2 ? 6 : 0, (cc & 1) ? 0 : 7, kz, &BAR[s]);
+        if (!ZX) tma_load_3d(D + COR + 16 * cc, xmaps + 2, cc < 2 ? 6 : 0, (cc & 1) ? 0 : 7, xkz, &BAR[s]);
       } else if (l == 12 && rec) {  // slot (n+1) % 4 held record n-3, consumed long ago
         tma_load_1d(MR + ((n + 1) % MRS) * kPenRec, REC + (int64_t)(n + 1) * kPenRec, kPenRec * 4, &BAR[s]);
       }
@@ -431,7 +458,8 @@ cudaError_t encode_pencil_maps(const double* x, const double* b, int64_t n_alloc
 #define PENCIL_FLAG_LIST(X)                                                                              \
   X(0) X(SW_WRITE_R) X(SW_RESTRICT) X(SW_COLOUR) X(SW_WRITE_R | SW_COLOUR) X(SW_RESTRICT | SW_COLOUR)   \
   X(SW_ZERO_X) X(SW_ZERO_X | SW_WRITE_R) X(SW_ZERO_X | SW_RESTRICT) X(SW_ZERO_X | SW_COLOUR)             \
-  X(SW_ZERO_X | SW_WRITE_R | SW_COLOUR) X(SW_ZERO_X | SW_RESTRICT | SW_COLOUR)
+  X(SW_ZERO_X | SW_WRITE_R | SW_COLOUR) X(SW_ZERO_X | SW_RESTRICT | SW_COLOUR)                          \
+  X(SW_PEER) X(SW_PEER | SW_WRITE_R) X(SW_PEER | SW_RESTRICT)
 
 // MG_PEN_TRACE=1 (measurement runs without graph capture only): every pencil pass records each CTA's
 // (start, end) globaltimer and prints the spread of the CTAs' end times -- the pass's tail
@@ -488,7 +516,7 @@ cudaError_t launch_sweep2p(const SweepArgs& a, const PairArgs& pa_in, const Pair
   const unsigned g = (unsigned)pa.nctas;
   const size_t sm = SMEM_BYTES;
   const unsigned col = (a.colour >= 0 || a.colour2 >= 0) ? SW_COLOUR : 0u;
-  switch ((flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP | SW_ZERO_X)) | col) {
+  switch ((flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP | SW_ZERO_X | SW_PEER)) | col) {
 #define PENCIL_CASE(F)                                                      \
   case (F):                                                                 \
     launch_plain(sweep2p_kernel<(F)>, g, PN_THREADS, sm, s, a, pa, pm); \

@@ -94,6 +94,7 @@ _SIGS = {
                                          ctypes.POINTER(ctypes.c_int64)]),
     "mg_peer_blob": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_char_p]),
     "mg_peer_connect": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_char_p]),
+    "mg_exchange_fused": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.POINTER(ctypes.c_int64)]),
     "mg_exchange_plan": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.POINTER(ctypes.c_int64),
                                         ctypes.POINTER(ctypes.c_int64)]),
     "mg_exchange_time": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32,
@@ -313,6 +314,12 @@ def mg_exchange_plan(ctx, num_levels):
     by = (ctypes.c_int64 * num_levels)()
     check(lib().mg_exchange_plan(ctx, num_levels, ex, by), "mg_exchange_plan")
     return list(ex), list(by)
+
+
+def mg_exchange_fused(ctx, num_levels):
+    fu = (ctypes.c_int64 * num_levels)()
+    check(lib().mg_exchange_fused(ctx, num_levels, fu), "mg_exchange_fused")
+    return list(fu)
 
 
 def mg_exchange_time(ctx, level, reps=20):

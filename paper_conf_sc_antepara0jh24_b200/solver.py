@@ -181,6 +181,10 @@ class Multigrid:
         """([exchanges per V-cycle per level], [bytes this rank sends per exchange per level])."""
         return mg.mg_exchange_plan(self.ctx, self.num_levels)
 
+    def exchange_fused(self):
+        """[exchanges per V-cycle per level fused into the pencil pass after them] (mg_exchange_fused)."""
+        return mg.mg_exchange_fused(self.ctx, self.num_levels)
+
     def exchange_time(self, level, reps=20) -> float:
         """Device ms of one ghost exchange of x at `level` (collective over NCCL)."""
         return mg.mg_exchange_time(self.ctx, level, reps)

@@ -5,6 +5,8 @@ relative on the residual norm after each V-cycle.  The design target is
 BITWISE equality (same expression DAG, no FMA), so most
 assertions are exact; the stated tolerances are asserted too.
 """
+import os
+
 import numpy as np
 import pytest
 
@@ -96,9 +98,12 @@ def test_restriction_and_interpolation_per_op(oracle_mod):
 
 
 @pytest.mark.parametrize("bottom_mode", [1, 2])
-@pytest.mark.parametrize("shape", [(8, 8, 8), (16, 16, 16), (8, 16, 32)])
+@pytest.mark.parametrize("shape", [(8, 8, 8), (16, 16, 16), (8, 16, 32), (8, 24, 40), (16, 32, 32), (32, 32, 32),
+                                   (24, 24, 24)])
 def test_bottom_solver(oracle_mod, bottom_mode, shape):
-    """100 point-Jacobi sweeps: resident one-CTA kernel and per-sweep launches."""
+    """100 point-Jacobi sweeps: the resident kernels (one CTA for <= 8 bricks, one
+    cluster of ceil(n / 8) CTAs for 9-64: 15 bricks = a part-filled second CTA, 27 and 64 = the
+    replicated bottoms' sizes) and per-sweep launches."""
     mg, _ = _mg()
     m = new(shape, 1, bottom_mode=bottom_mode)
     h = mg_inputs.default_h0(shape)
@@ -192,6 +197,50 @@ def test_self_exchange_ca_periods_bitwise(oracle_mod, transport, period):
     m.set_solution(None)
     check_cycles(m, xs, ns)
     m.close()
+
+
+@pytest.mark.parametrize("transport", [3, 2])
+@pytest.mark.parametrize("shape,L", [((128, 128, 128), 4), ((64, 96, 128), 3)])
+def test_fused_exchange_pencil_pass_bitwise(oracle_mod, transport, shape, L):
+    """The exchange fused into the pencil pass: with a self-exchanged ghost shell on every
+    axis, level 0's passes after an x exchange stage their ghost bricks' slabs, corners and warm-up /
+    cool-down half bricks straight from the owner's field (here: this rank's own owned bricks across the
+    periodic wrap) instead of running the exchange kernel -- the plan says so (exchange_fused), and x and
+    the norm stay bitwise equal to the oracle's after each cycle."""
+    b = mg_inputs.random_rhs(shape, 14)
+    xs, ns = oracle_cycles(oracle_mod, b, L, 2, 12, 12, 100)
+    m = new(shape, L, ghost_mode=1, transport=transport)
+    fused = m.exchange_fused()
+    counts, _ = m.exchange_plan()
+    if os.environ.get("MG_NO_FUSED_EXCH"):
+        assert not any(fused)
+    else:
+        assert fused[0] >= 5 and fused[0] <= counts[0], (fused, counts)
+    m.set_rhs(dev(b))
+    m.set_solution(None)
+    check_cycles(m, xs, ns)
+    m.close()
+
+
+def test_fused_exchange_loopback_group_bitwise(oracle_mod):
+    """2x2x1 loopback group of 64^3 ranks: every rank's fused level-0 passes read the neighbour ranks'
+    fields directly (the group runs the ranks in lockstep); x of every rank bitwise after 2 cycles."""
+    _, solver = _mg()
+    pg, n_local, L = (2, 2, 1), (64, 64, 64), 4
+    gshape = (n_local[2] * pg[2], n_local[1] * pg[1], n_local[0] * pg[0])
+    b = mg_inputs.random_rhs(gshape, 15)
+    xs, ns = oracle_cycles(oracle_mod, b, L, 2)
+    g = solver.LoopbackGroup(n_local, pg, num_levels=L)
+    P = pg[0] * pg[1] * pg[2]
+    g.set_rhs([dev(mg_inputs.local_block(b, r, pg)) for r in range(P)])
+    g.set_solution(None)
+    for c in range(2):
+        g.vcycle()
+        nr = g.residual_norm()
+        assert nr == ns[c], (c, nr, ns[c])
+        for r in range(P):
+            assert_bitwise(host(g.get_solution(r)), mg_inputs.local_block(xs[c], r, pg), what=f"rank {r} cycle {c}")
+    g.close()
 
 
 @pytest.mark.parametrize("pg,n_local,L", [((2, 1, 1), (32, 32, 32), 3), ((2, 2, 2), (32, 32, 32), 3),
@@ -850,7 +899,8 @@ def test_exchange_plan_and_timing_keep_the_bits(oracle_mod, transport):
 
 @pytest.mark.parametrize("args", ["32 32 32 2 1 1 3 2 0", "16 16 16 2 2 1 2 2 0", "32 32 32 2 1 1 3 1 1",
                                   "16 16 16 2 2 2 2 2 0", "32 32 32 2 1 1 3 2 0 1", "16 16 32 2 2 2 2 2 1 2",
-                                  "128 128 128 2 1 1 3 2 0 0 pencil-overlap", "128 128 128 2 2 1 3 2 0 0 pencil-overlap"])
+                                  "128 128 128 2 1 1 3 2 0 0 pencil-overlap", "128 128 128 2 2 1 3 2 0 0 pencil-overlap",
+                                  "128 128 128 2 2 1 3 2 0", "64 64 64 2 2 2 3 2 0"])
 def test_peer_transport_multiprocess_bitwise(args):
     """The peer-memory transport between PROCESSES (CUDA IPC mappings, device-side ready/done flags, the
     norm's max and the replicated bottom's gather over peer memory): torchrun starts one process per
@@ -875,3 +925,6 @@ def test_peer_transport_multiprocess_bitwise(args):
            "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.join(root, "tools", "peer_check.py"), *a]
     r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, cwd=root, env=env)
     assert r.returncode == 0 and "peer_check ok" in r.stdout, (r.stdout[-2000:], r.stderr[-3000:])
+    if "MG_PENCIL_OVERLAP" not in env and not env.get("MG_NO_FUSED_EXCH") and int(a[0]) >= 64:
+        # level 0's passes take the fused exchange: a handshake kernel, then slabs from the peers' fields
+        assert "fused exchanges per level [0, " not in r.stdout and "fused exchanges per level [" in r.stdout, r.stdout

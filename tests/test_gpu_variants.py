@@ -70,10 +70,12 @@ def check_cycles(m, xs, ns):
 
 # ------------------------------------------------------------ boundary conditions (A22)
 @pytest.mark.parametrize("bc", [1, 2])
-@pytest.mark.parametrize("shape,L", [((64, 64, 64), 4), ((32, 16, 48), 2), ((128, 128, 128), 5)])
+@pytest.mark.parametrize("shape,L", [((64, 64, 64), 4), ((32, 16, 48), 2), ((128, 128, 128), 5), ((64, 64, 64), 2),
+                                     ((48, 32, 64), 2)])
 def test_bc_vcycle_bitwise(oracle_mod, bc, shape, L):
     """Dirichlet / Neumann V-cycles (12/12/100) bitwise equal to the oracle's after each of 2 cycles,
-    x and the norm; 128^3 runs the pencil passes over the ghost-shell plan on level 0."""
+    x and the norm; 128^3 runs the pencil passes over the ghost-shell plan on level 0; L = 2 at 64^3
+    / 48x32x64 ends on 64 / 24 bricks: the cluster-resident bottom with the mirror images."""
     b = mg_inputs.random_field(shape, 21)
     xs, ns = oracle_cycles(oracle_mod, b, L, 2, bc=bc)
     m = new(shape, L, bc=bc)

@@ -55,10 +55,12 @@ def main():
             raise SystemExit(f"peer_check FAILED cycle {c + 1} (rank, ok, max|dx|, norm): "
                              f"{[(r,) + f for r, f in enumerate(flags)]} oracle norm {o.norm()}")
     launches = m.launches_per_vcycle()
+    fused = m.exchange_fused()  # exchanges fused into level pencil passes (SW_PEER + handshake kernel)
     m.close()
     if rank == 0:
         print(f"peer_check ok: {world} processes, proc grid {pg}, {nl} per rank, L={L}, ghost_mode={ghost}, bc={bc}, "
-              f"{ncyc} V-cycles bitwise equal to the oracle (last norm {nr:.6e}, {launches} launches per cycle)")
+              f"{ncyc} V-cycles bitwise equal to the oracle (last norm {nr:.6e}, {launches} launches per cycle, "
+              f"fused exchanges per level {fused})")
     dist.destroy_process_group()
 
 
