@@ -479,13 +479,9 @@ mg_status fill_repl_tables(mg_ctx* c) {
 // instead stages the side slabs, corner columns and warm-up / cool-down bricks of its ghost bricks
 // straight from the owners' fields (the receive runs say which brick of which rank a ghost mirrors).
 // MG_NO_FUSED_EXCH=1 keeps the separate exchange (A/B).
-static bool fused_exchange_on() {
-  static const bool off = getenv("MG_NO_FUSED_EXCH") != nullptr;
-  return !off;
-}
 
 static mg_status fill_fused_tables(mg_ctx* c) {
-  if (!fused_exchange_on() || c->use_nccl) return MG_OK;
+  if (!fused_exchange_enabled() || c->use_nccl) return MG_OK;
   const int W = c->group ? (int)c->group->r.size() : c->lay.world;
   if (W > 8) return MG_OK;  // (PairMaps::rbase)
   for (int l = 0; l < c->lay.L; ++l) {

@@ -42,7 +42,27 @@ int Builder::period(int l) const {
       }
       if (i == l && k > 0) return std::min(k, lay.E);
     }
+  // a level whose exchanges fuse into its pencil passes (api.cu fill_fused_tables: no exchange kernel,
+  // no redundant ghost sweeping) takes period 2 like level 0 (MG_FUSED_P8=1: period 8, A/B runs)
+  static const bool p8 = getenv("MG_FUSED_P8") != nullptr;
+  if (box && l > 0 && !p8 && fused_level(l)) return std::min(2, lay.E);
   return (l == 0 && box) ? std::min(2, lay.E) : lay.E;
+}
+
+bool fused_exchange_enabled() {
+  static const bool off = getenv("MG_NO_FUSED_EXCH") != nullptr;
+  return !off;
+}
+
+// the conditions under which the executor fuses this level's x exchanges into its pencil passes
+// (api.cu make_plan / fill_fused_tables): copy transport, periodic box, constant coefficients, Jacobi
+// or Chebyshev pre / post sweeps, a pencil plan over the owned range, <= 8 ranks, no pencil overlap
+bool Builder::fused_level(int l) const {
+  const LevelLayout& L = lay.lv[l];
+  static const bool pen_ov = getenv("MG_PENCIL_OVERLAP") && atoi(getenv("MG_PENCIL_OVERLAP")) != 0;
+  return fused_exchange_enabled() && lay.p.transport != MG_TRANSPORT_NCCL && lay.p.bc == 0 && !lay.p.var_coef &&
+         lay.p.smoother != 2 && L.n_ghost > 0 && lay.world <= 8 && !(pen_ov && lay.p.overlap) &&
+         fusion(l) != MG_FUSION_PAPER && lay.p.temporal_blocking && pencil_table(l);
 }
 
 int Builder::xdepth(int l) const {

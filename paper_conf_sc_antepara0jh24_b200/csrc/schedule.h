@@ -68,7 +68,8 @@ struct Builder {
   // period (depth-limited copies, local and peer transports) or the whole brick (NCCL)
   int xdepth(int l) const;
   bool pair_ok(int l) const;  // two-sweep passes possible at level l
-  bool pencil_table(int l) const;  // the owned range of level l has a 2x2-brick pencil plan (kind 3)
+  bool pencil_table(int l) const;
+  bool fused_level(int l) const;    // level l's x exchanges fuse into its pencil passes (period 2)  // the owned range of level l has a 2x2-brick pencil plan (kind 3)
   bool pencil_ghosts(int l) const;  // ... and so has its whole stored range (owned + ghost shell)
   bool pair_zero_ok(int l) const;   // the owned range's pencil kernel folds x0 == 0 into a pair (SW_ZERO_X)
   bool pair_ghosts_ok(int l) const;  // two-sweep passes may include the ghost shell at level l
@@ -85,6 +86,7 @@ struct Builder {
 };
 
 // own kernel launches of one op (local_exchange: exchanges run as one copy kernel, else NCCL)
+bool fused_exchange_enabled();  // MG_NO_FUSED_EXCH=1: the separate exchange kernel everywhere (A/B)
 int64_t op_launches(const Op& o, const Layout& lay, bool overlap, bool pencil_overlap, bool local_exchange);
 
 }  // namespace mgb

@@ -200,7 +200,7 @@ def test_self_exchange_ca_periods_bitwise(oracle_mod, transport, period):
 
 
 @pytest.mark.parametrize("transport", [3, 2])
-@pytest.mark.parametrize("shape,L", [((128, 128, 128), 4), ((64, 96, 128), 3)])
+@pytest.mark.parametrize("shape,L", [((128, 128, 128), 4), ((128, 128, 256), 3)])
 def test_fused_exchange_pencil_pass_bitwise(oracle_mod, transport, shape, L):
     """The exchange fused into the pencil pass: with a self-exchanged ghost shell on every
     axis, level 0's passes after an x exchange stage their ghost bricks' slabs, corners and warm-up /
@@ -223,10 +223,11 @@ def test_fused_exchange_pencil_pass_bitwise(oracle_mod, transport, shape, L):
 
 
 def test_fused_exchange_loopback_group_bitwise(oracle_mod):
-    """2x2x1 loopback group of 64^3 ranks: every rank's fused level-0 passes read the neighbour ranks'
-    fields directly (the group runs the ranks in lockstep); x of every rank bitwise after 2 cycles."""
+    """2x2x1 loopback group of 128^3 ranks (level 0: 4096 bricks, pencil passes): every rank's fused
+    level-0 passes read the neighbour ranks' fields directly (the group runs the ranks in lockstep); x of
+    every rank bitwise after 2 cycles."""
     _, solver = _mg()
-    pg, n_local, L = (2, 2, 1), (64, 64, 64), 4
+    pg, n_local, L = (2, 2, 1), (128, 128, 128), 4
     gshape = (n_local[2] * pg[2], n_local[1] * pg[1], n_local[0] * pg[0])
     b = mg_inputs.random_rhs(gshape, 15)
     xs, ns = oracle_cycles(oracle_mod, b, L, 2)
@@ -900,7 +901,7 @@ def test_exchange_plan_and_timing_keep_the_bits(oracle_mod, transport):
 @pytest.mark.parametrize("args", ["32 32 32 2 1 1 3 2 0", "16 16 16 2 2 1 2 2 0", "32 32 32 2 1 1 3 1 1",
                                   "16 16 16 2 2 2 2 2 0", "32 32 32 2 1 1 3 2 0 1", "16 16 32 2 2 2 2 2 1 2",
                                   "128 128 128 2 1 1 3 2 0 0 pencil-overlap", "128 128 128 2 2 1 3 2 0 0 pencil-overlap",
-                                  "128 128 128 2 2 1 3 2 0", "64 64 64 2 2 2 3 2 0"])
+                                  "128 128 128 2 2 1 3 2 0", "128 128 128 2 2 2 3 2 0"])
 def test_peer_transport_multiprocess_bitwise(args):
     """The peer-memory transport between PROCESSES (CUDA IPC mappings, device-side ready/done flags, the
     norm's max and the replicated bottom's gather over peer memory): torchrun starts one process per
@@ -925,6 +926,6 @@ def test_peer_transport_multiprocess_bitwise(args):
            "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.join(root, "tools", "peer_check.py"), *a]
     r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, cwd=root, env=env)
     assert r.returncode == 0 and "peer_check ok" in r.stdout, (r.stdout[-2000:], r.stderr[-3000:])
-    if "MG_PENCIL_OVERLAP" not in env and not env.get("MG_NO_FUSED_EXCH") and int(a[0]) >= 64:
+    if "MG_PENCIL_OVERLAP" not in env and not env.get("MG_NO_FUSED_EXCH") and int(a[0]) >= 128:
         # level 0's passes take the fused exchange: a handshake kernel, then slabs from the peers' fields
         assert "fused exchanges per level [0, " not in r.stdout and "fused exchanges per level [" in r.stdout, r.stdout
