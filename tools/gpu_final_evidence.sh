@@ -12,7 +12,7 @@ timeout 900 python bench.py --steps 20 --warmup 5 > gpurun_out/fin/bench.json 2>
 A="--steps 2 --warmup 1 --no-cpu-baseline --no-e2e"
 M="--metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none --csv"
 timeout 900 ncu $M -c 400 --log-file gpurun_out/fin/launches.csv python bench.py $A > /dev/null 2>&1; echo "launches rc=$?"
-for v in "varcoef --var-coef" "brick4 --brick-edge 4" "dirichlet --bc 1" "paper --fusion 1 --tb 0"; do
+for v in "varcoef --var-coef" "brick4 --brick-edge 4" "dirichlet --bc 1" "paper --fusion 1 --tb 0" "ghostall_peer --ghost-all --transport peer"; do
   set -- $v
   tag=$1; shift
   timeout 900 ncu $M -c 800 --log-file gpurun_out/fin/launches_$tag.csv python bench.py $A "$@" > /dev/null 2>&1; echo "launches $tag rc=$?"
