@@ -24,6 +24,9 @@ B_PER_PT = [
     ("sweep2p_kernel<2>", "two-sweep pass + restriction (pencil)", 25.0),
     ("sweep2p_kernel<0>", "two-sweep pass (pencil)", 24.0),
     ("sweep2p_kernel<1>", "two-sweep pass + r (pencil)", 32.0),
+    # SW_PEER (256): the exchange fused into the pass -- ghost slabs from the owners' fields
+    ("sweep2p_kernel<258>", "two-sweep pass + restriction, exchange fused (pencil, SW_PEER)", 25.0),
+    ("sweep2p_kernel<256>", "two-sweep pass, exchange fused (pencil, SW_PEER)", 24.0),
     ("sweep_col_kernel<0>", "fused sweep (column)", 24.0),
     ("sweep_col_kernel<1>", "fused sweep + r (column)", 32.0),
     ("sweep_col_kernel<2>", "fused sweep + restriction (column)", 25.0),
