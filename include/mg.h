@@ -96,7 +96,9 @@ enum { MG_TRANSPORT_AUTO = 0, MG_TRANSPORT_NCCL = 1, MG_TRANSPORT_LOCAL = 2, MG_
 #define MG_PEER_BLOB_BYTES 128
 
 /* bottom_mode.  AUTO: a bottom level of <= 8 bricks without ghosts runs all its sweeps in one
- * CTA (resident), otherwise per-sweep launches.  CLUSTER (opt-in): the deepest
+ * CTA (resident), one of 9-64 bricks in one thread-block cluster of up to 16 CTAs (bottom_cluster.cu,
+ * neighbours through distributed shared memory; also the replicated global bottom of a
+ * decomposition), otherwise per-sweep launches.  CLUSTER (opt-in): the deepest
  * levels without ghosts that fit (<= 64 bricks per level, <= 200 KB of fields) run as ONE
  * 8-CTA cluster launch (coarse.cu: pre-sweeps, restriction, initZero, bottom, interpolation,
  * post-sweeps of those levels); measured no faster than graph-replayed launches (DESIGN.md
@@ -123,7 +125,13 @@ typedef struct {
                                     NCCL; the norm's max and the replicated bottom's gather likewise);
                                     NCCL = grouped ncclSend/ncclRecv + ncclAllReduce (needs nccl_id).  One
                                     rank: local device copies, or NCCL self send/recv with
-                                    MG_TRANSPORT_NCCL (nccl_id may then be NULL) */
+                                    MG_TRANSPORT_NCCL (nccl_id may then be NULL).  On the copy
+                                    transports (PEER, LOCAL) a level with a pencil plan over its owned
+                                    bricks (periodic box, constant coefficients, <= 8 ranks) runs NO
+                                    x exchange kernel: its two-sweep passes stage the ghost bricks' x
+                                    straight from the owners' fields (the exchange fused into the pass,
+                                    after a flag handshake between processes; mg_exchange_fused) and
+                                    take CA period 2 by default */
   int32_t use_graph;             /* 1 = replay the V-cycle as one CUDA graph (default 1) */
   int32_t bottom_mode;           /* MG_BOTTOM_* (resident = one CTA runs all bottom sweeps in smem,
                                     cluster = the coarse levels run in one cluster launch, grid = the
