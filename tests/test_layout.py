@@ -1,6 +1,7 @@
 """CPU tests of the brick layout, adjacency, region ordering and exchange plans
 (host-only C-ABI queries; no GPU), plus a bitwise V-cycle of the host brick
 interpreter on those tables against the lexicographic oracle."""
+import os
 import itertools
 
 import numpy as np
@@ -486,3 +487,23 @@ def test_depth_limited_exchange_bytes_decomposed(pg):
             nl = n >> l
             ext = np.prod([nl + (2 * d if g > 1 else 0) for g in pg])
             assert nbytes[l] == (ext - nl ** 3) * 8, (r, l)
+
+
+@pytest.mark.parametrize("transport", [mg.MG_TRANSPORT_PEER, mg.MG_TRANSPORT_LOCAL, mg.MG_TRANSPORT_NCCL])
+def test_fused_levels_take_period_two(transport):
+    """Levels whose x exchanges fuse into their pencil passes (a pencil plan over the
+    owned range -- >= 4096 bricks --, a periodic box, constant coefficients, a copy transport) take the CA
+    period 2 like level 0: at 256^3 with a ghost shell on every axis level 1 (128^3, 4096 bricks) exchanges
+    two cell layers before each of its 11 x-passes (+ b's after the restriction), level 2 (64^3, 512
+    bricks, one-brick kernels) keeps whole bricks at period 8; NCCL keeps whole bricks everywhere."""
+    n, L = 256, 4
+    p = mg.params((n, n, n), num_levels=L, ghost_mode=1, transport=transport)
+    exchanges, nbytes = mg.Layout(p, 0, 1).exchange_plan()
+    fused = os.environ.get("MG_NO_FUSED_EXCH") is None and transport != mg.MG_TRANSPORT_NCCL
+    for l, d in ((0, 2), (1, 2 if fused else 8), (2, 8)):
+        if transport == mg.MG_TRANSPORT_NCCL:
+            d = 8
+        nl = n >> l
+        assert nbytes[l] == ((nl + 2 * d) ** 3 - nl ** 3) * 8, (l, d, nbytes)
+    if fused:
+        assert exchanges[1] == 12, exchanges
