@@ -636,7 +636,7 @@ mg_status sweep_range(mg_ctx* c, const Op& o, int64_t b0, int64_t b1, cudaStream
           pa.rmaps = d.rmaps + (size_t)o.src * d.rworld * 3;
           PairMaps pm = d.nmaps[o.src];
           for (int r = 0; r < d.rworld; ++r) pm.rbase[r] = d.rbase[(size_t)o.src * d.rworld + r];
-          CKC(c, launch_sweep2p(a, pa, pm, o.flags | SW_PEER, s));
+          CKC(c, launch_sweep2p(a, pa, pm, o.flags | SW_PEER, s, o.fused == 2));
         } else if (pr.args.kind == 3)
           CKC(c, launch_sweep2p(a, pr.args, d.nmaps[o.src], o.flags | (o.zero ? SW_ZERO_X : 0u), s));
         else

@@ -106,8 +106,10 @@ cudaError_t pair_kernels_init();
 // {2,1,4}; b {2,8,4}, {8,1,4}) in the PairMaps fields
 cudaError_t encode_pencil_maps(const double* x, const double* b, int64_t n_alloc, PairMaps* out);
 bool pencil_supports(unsigned flags);
+// early: launch with PDL (only after a one-CTA peer handshake, which triggers once the previous
+// kernel is complete: the pass's CTAs land on a drained GPU and wait for the handshake in pdl_wait)
 cudaError_t launch_sweep2p(const SweepArgs& a, const PairArgs& pa, const PairMaps& pm, unsigned flags,
-                           cudaStream_t s);
+                           cudaStream_t s, bool early = false);
 cudaError_t pencil_kernels_init();
 
 // true if the streaming kernel implements `flags` (plain, +r, +restriction)

@@ -120,7 +120,8 @@ __global__ void peer_allmax_kernel(unsigned long long* acc, PeerSync s, unsigned
 // Then no rank reads a field its owner has not finished (RAW) and no rank overwrites, in its next
 // pass, a buffer a neighbour is still reading (WAR: the neighbour's ready(e+1) comes after its pass e).
 __global__ void peer_handshake_kernel(PeerSync s) {
-  pdl_wait();
+  pdl_wait();     // the kernel that wrote this pass's x is complete ...
+  pdl_trigger();  // ... so the pass (launched early) may place its CTAs now; they wait for this kernel
   if (threadIdx.x == 0) {
     const unsigned long long e = *(volatile unsigned long long*)s.epoch + 1;
     peer_signal(s, 0, e);
@@ -128,7 +129,6 @@ __global__ void peer_handshake_kernel(PeerSync s) {
     *s.epoch = e;
     __threadfence();
   }
-  pdl_trigger();
 }
 
 }  // namespace

@@ -504,7 +504,7 @@ static cudaError_t trace_report(const PairArgs& pa, cudaStream_t s) {
 }
 
 cudaError_t launch_sweep2p(const SweepArgs& a, const PairArgs& pa_in, const PairMaps& pm, unsigned flags,
-                           cudaStream_t s) {
+                           cudaStream_t s, bool early) {
   if (pa_in.nctas <= 0) return cudaSuccess;
   static const bool trace = getenv("MG_PEN_TRACE") != nullptr;
   static unsigned long long* tbuf = nullptr;
@@ -519,7 +519,7 @@ cudaError_t launch_sweep2p(const SweepArgs& a, const PairArgs& pa_in, const Pair
   switch ((flags & (SW_WRITE_R | SW_RESTRICT | SW_INTERP | SW_ZERO_X | SW_PEER)) | col) {
 #define PENCIL_CASE(F)                                                      \
   case (F):                                                                 \
-    launch_plain(sweep2p_kernel<(F)>, g, PN_THREADS, sm, s, a, pa, pm); \
+    launch_ex(early && g_launch_pdl, sweep2p_kernel<(F)>, g, PN_THREADS, sm, s, a, pa, pm); \
     break;
     PENCIL_FLAG_LIST(PENCIL_CASE)
 #undef PENCIL_CASE
