@@ -637,8 +637,11 @@ mg_status sweep_range(mg_ctx* c, const Op& o, int64_t b0, int64_t b1, cudaStream
           PairMaps pm = d.nmaps[o.src];
           for (int r = 0; r < d.rworld; ++r) pm.rbase[r] = d.rbase[(size_t)o.src * d.rworld + r];
           CKC(c, launch_sweep2p(a, pa, pm, o.flags | SW_PEER, s, o.fused == 2));
-        } else if (pr.args.kind == 3)
-          CKC(c, launch_sweep2p(a, pr.args, d.nmaps[o.src], o.flags | (o.zero ? SW_ZERO_X : 0u), s));
+        } else if (pr.args.kind == 3) {
+          // MG_PEN_PDL=<l0> (A/B runs): pencil passes of levels >= l0 launched with PDL
+          static const int pen_pdl = getenv("MG_PEN_PDL") ? atoi(getenv("MG_PEN_PDL")) : 1 << 30;
+          CKC(c, launch_sweep2p(a, pr.args, d.nmaps[o.src], o.flags | (o.zero ? SW_ZERO_X : 0u), s, l >= pen_pdl));
+        }
         else
           CKC(c, launch_sweep2(a, pr.args, d.pmaps[o.src], o.flags, s));
         return MG_OK;
