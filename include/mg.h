@@ -363,6 +363,11 @@ mg_status mg_layout_plan(const mg_layout* lay, int32_t level, int32_t which /*0 
  * query the count).  The ghost brick's cell (i,j,k) is the source's cell with i -> 7-i etc. on the
  * reflected axes, negated once per reflection for Dirichlet. */
 mg_status mg_layout_mirror(const mg_layout* lay, int32_t level, int64_t* count, int32_t* out);
+/* The exchange fused into the level's pencil passes: per chunk record of the owned pencil
+ * plan and entry e = 0..15 (the record's brick ids 1..16), -1 for a local brick or (rank << 24) | the
+ * brick of rank's field that the ghost brick mirrors -- the table the pass stages its ghost x from.
+ * *count = chunks * 16, 0 if the level does not fuse its exchanges; out (count int32) may be NULL. */
+mg_status mg_layout_fused_pid(const mg_layout* lay, int32_t level, int64_t* count, int32_t* out);
 mg_status mg_layout_pass_plan(const mg_layout* lay, int32_t level, int32_t idx, int64_t info[6], int32_t* meta,
                               int32_t* ctas);
 /* Replicated bottom (the coarsest level has a ghost shell and the global coarsest grid <= 64

@@ -480,6 +480,35 @@ mg_status fill_repl_tables(mg_ctx* c) {
 // straight from the owners' fields (the receive runs say which brick of which rank a ghost mirrors).
 // MG_NO_FUSED_EXCH=1 keeps the separate exchange (A/B).
 
+// The fused exchange's per-chunk source table of level L (PairArgs::pid) from its owned pencil plan and
+// receive runs: [chunks][16] -1 (a local brick) or (rank << 24) | the brick of that rank's layout the
+// ghost mirrors.  False if the level has no owned pencil plan or a ghost brick without a source.
+static bool fused_pid_table(const LevelLayout& L, int W, std::vector<int32_t>& pid) {
+  pid.clear();
+  if (L.n_ghost == 0) return false;
+  const LevelLayout::PairTable* pt = nullptr;
+  for (const auto& t : L.pairs)
+    if (t.b0 == 0 && t.b1 == L.n_owned && t.part == 0 && t.kind == 3) pt = &t;
+  if (!pt) return false;
+  std::vector<int2> g((size_t)L.n_ghost, make_int2(-1, -1));  // ghost brick -> (owner rank, its brick)
+  for (const Run& r : L.recvs)
+    for (int64_t k = 0; k < r.count; ++k)
+      if (r.local + k >= L.n_owned && r.local + k < L.n_stored)
+        g[(size_t)(r.local + k - L.n_owned)] = make_int2(r.peer, (int)(r.remote + k));
+  const size_t nch = pt->meta.size() / kPenRec;
+  pid.assign(nch * 16, -1);
+  for (size_t ch = 0; ch < nch; ++ch)
+    for (int e = 0; e < 16; ++e) {
+      const int32_t id = pt->meta[ch * kPenRec + 1 + (size_t)e];
+      if (id < L.n_owned) continue;
+      if (id >= L.n_stored) return false;
+      const int2 src = g[(size_t)(id - L.n_owned)];
+      if (src.x < 0 || src.x >= W || src.y >= (1 << 24)) return false;
+      pid[ch * 16 + (size_t)e] = (src.x << 24) | src.y;
+    }
+  return true;
+}
+
 static mg_status fill_fused_tables(mg_ctx* c) {
   if (!fused_exchange_enabled() || c->use_nccl) return MG_OK;
   const int W = c->group ? (int)c->group->r.size() : c->lay.world;
@@ -489,29 +518,8 @@ static mg_status fill_fused_tables(mg_ctx* c) {
     DevLevel& d = c->dl[l];
     d.fused = false;
     if (d.ncruns == 0 || L.n_ghost == 0 || d.nmirror > 0 || d.cf) continue;
-    const LevelLayout::PairTable* pt = nullptr;
-    for (const auto& t : L.pairs)
-      if (t.b0 == 0 && t.b1 == L.n_owned && t.part == 0 && t.kind == 3) pt = &t;
-    if (!pt) continue;
-    // ghost brick -> (owner rank, the owner's brick it mirrors), from the receive runs
-    std::vector<int2> g((size_t)L.n_ghost, make_int2(-1, -1));
-    for (const Run& r : L.recvs)
-      for (int64_t k = 0; k < r.count; ++k)
-        if (r.local + k >= L.n_owned && r.local + k < L.n_stored)
-          g[(size_t)(r.local + k - L.n_owned)] = make_int2(r.peer, (int)(r.remote + k));
-    const size_t nch = pt->meta.size() / kPenRec;
-    std::vector<int32_t> pid(nch * 16, -1);
-    bool ok = true;
-    for (size_t ch = 0; ch < nch && ok; ++ch)
-      for (int e = 0; e < 16; ++e) {
-        const int32_t id = pt->meta[ch * kPenRec + 1 + (size_t)e];
-        if (id < L.n_owned) continue;
-        if (id >= L.n_stored) { ok = false; break; }
-        const int2 src = g[(size_t)(id - L.n_owned)];
-        if (src.x < 0 || src.x >= W || src.y >= (1 << 24)) { ok = false; break; }
-        pid[ch * 16 + (size_t)e] = (src.x << 24) | src.y;
-      }
-    if (!ok) continue;
+    std::vector<int32_t> pid;
+    if (!fused_pid_table(L, W, pid)) continue;
     std::vector<CUtensorMap> maps((size_t)2 * W * 3);
     d.rbase.assign((size_t)2 * W, nullptr);
     for (int xb = 0; xb < 2; ++xb)
@@ -1943,6 +1951,19 @@ mg_status mg_layout_adjacency(const mg_layout* m, int32_t level, int32_t* out) {
   const LevelLayout* L = nullptr;
   CKS(lay_level(m, level, &L));
   std::memcpy(out, L->adj.data(), L->adj.size() * sizeof(int32_t));
+  return MG_OK;
+}
+
+mg_status mg_layout_fused_pid(const mg_layout* m, int32_t level, int64_t* count, int32_t* out) {
+  const LevelLayout* L = nullptr;
+  CKS(lay_level(m, level, &L));
+  if (!count) return set_err(MG_ERR_INVALID_ARG, "null count");
+  Builder b(m->lay);
+  std::vector<int32_t> pid;
+  *count = 0;
+  if (!b.fused_level(level) || !fused_pid_table(*L, m->lay.world, pid)) return MG_OK;
+  *count = (int64_t)pid.size();
+  if (out) std::memcpy(out, pid.data(), pid.size() * sizeof(int32_t));
   return MG_OK;
 }
 

@@ -94,6 +94,8 @@ _SIGS = {
                                          ctypes.POINTER(ctypes.c_int64)]),
     "mg_peer_blob": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_char_p]),
     "mg_peer_connect": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_char_p]),
+    "mg_layout_fused_pid": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.POINTER(ctypes.c_int64),
+                                           ctypes.c_void_p]),
     "mg_exchange_fused": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.POINTER(ctypes.c_int64)]),
     "mg_exchange_plan": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.POINTER(ctypes.c_int64),
                                         ctypes.POINTER(ctypes.c_int64)]),
@@ -471,6 +473,16 @@ class Layout:
         a = self._np.zeros(inf["owned"] + inf["nghost"], dtype=self._np.int32)
         check(lib().mg_layout_parent(self.h, level, a.ctypes.data), "mg_layout_parent")
         return a
+
+    def fused_pid(self, level):
+        """The fused exchange's source table of a level (mg_layout_fused_pid): int32 [chunks][16], or None."""
+        n = ctypes.c_int64()
+        check(lib().mg_layout_fused_pid(self.h, level, ctypes.byref(n), None), "mg_layout_fused_pid")
+        if n.value == 0:
+            return None
+        a = self._np.zeros(n.value, dtype=self._np.int32)
+        check(lib().mg_layout_fused_pid(self.h, level, ctypes.byref(n), a.ctypes.data), "mg_layout_fused_pid")
+        return a.reshape(-1, 16)
 
     def pass_plans(self, level):
         """Two-sweep pass plans of a level: [(kind, b0, b1, meta int32 array, ctas int32 [n][2], part)]."""

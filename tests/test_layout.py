@@ -507,3 +507,47 @@ def test_fused_levels_take_period_two(transport):
         assert nbytes[l] == ((nl + 2 * d) ** 3 - nl ** 3) * 8, (l, d, nbytes)
     if fused:
         assert exchanges[1] == 12, exchanges
+
+
+@pytest.mark.parametrize("pg", [(2, 1, 1), (2, 2, 1), (2, 2, 2)])
+def test_fused_exchange_source_table(pg):
+    """The fused exchange's source table (mg_layout_fused_pid: what a level-0 pencil pass stages its ghost
+    bricks' x from) checked against the geometry alone: every record entry naming an owned brick stays
+    local (-1); every ghost brick at extended coords X is read from the rank that owns the periodic image
+    of X in the process grid, at the brick of that rank's own layout with coords X mod nb -- never from the
+    receive runs the table was built from.  128^3 per rank (level 0: 4096 bricks, pencil plan)."""
+    n = 128
+    world = pg[0] * pg[1] * pg[2]
+    p = mg.params((n, n, n), pg, num_levels=3, transport=mg.MG_TRANSPORT_PEER)
+    lays = [mg.Layout(p, r, world) for r in range(world)]
+    owned_ids = []
+    for lay in lays:
+        inf = lay.info(0)
+        c = lay.coords(0)[: inf["owned"]]
+        owned_ids.append({tuple(v): i for i, v in enumerate(c.tolist())})
+    nb = np.array(lays[0].info(0)["nb"])
+    for r, lay in enumerate(lays):
+        inf = lay.info(0)
+        pid = lay.fused_pid(0)
+        assert pid is not None
+        plan = [t for t in lay.pass_plans(0) if t[0] == 3 and t[1] == 0 and t[2] == inf["owned"] and t[5] == 0]
+        assert len(plan) == 1
+        meta = plan[0][3].reshape(-1, 20)
+        assert meta.shape[0] == pid.shape[0]
+        coords = lay.coords(0)
+        rc = np.array([r % pg[0], (r // pg[0]) % pg[1], r // (pg[0] * pg[1])])
+        remote = 0
+        for ch in range(meta.shape[0]):
+            for e in range(16):
+                bid = meta[ch, 1 + e]
+                if bid < inf["owned"]:
+                    assert pid[ch, e] == -1, (r, ch, e)
+                    continue
+                X = coords[bid]
+                off = np.floor_divide(X, nb)
+                oc = (rc + off) % np.array(pg)
+                owner = int(oc[0] + pg[0] * (oc[1] + pg[1] * oc[2]))
+                rid = owned_ids[owner][tuple(int(v) for v in np.mod(X, nb))]
+                assert pid[ch, e] == (owner << 24) | rid, (r, ch, e, X.tolist(), owner, rid, pid[ch, e])
+                remote += 1
+        assert remote > 0
