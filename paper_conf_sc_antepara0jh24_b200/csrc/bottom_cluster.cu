@@ -4,8 +4,10 @@
 // and a one-rank coarsest level of up to 64 bricks.
 //
 // The one-CTA resident bottom (resident.cuh) holds <= 8 bricks; this is the same thread mapping
-// spread over a cluster of ceil(nbricks / 8) CTAs of 1024 threads: brick q lives in CTA q / 8,
-// slot q % 8 (contiguous ids: the x rows of a brick layer stay in one CTA).  A thread owns a
+// spread over a cluster of ceil(nbricks / BPC) CTAs of 128 BPC threads, BPC bricks per CTA -- the
+// fewest that keep the cluster within 16 CTAs (a sweep is bound by each SM's shared-memory traffic,
+// so more SMs per level pay: 64 bricks 0.10 ms on 16 CTAs vs 0.14 ms on 8): brick q
+// lives in CTA q / BPC, slot q % BPC (contiguous ids: the x rows of a brick layer stay together).  A thread owns a
 // k-column of 4 cells of one brick (x in registers, b in registers), and every neighbour cell --
 // in its own brick, in another brick of its CTA or in another CTA's shared memory -- is addressed
 // through the cluster's shared window (mapa), resolved ONCE before the sweeps.  Per sweep: the 18
