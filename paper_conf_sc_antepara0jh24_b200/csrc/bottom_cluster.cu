@@ -10,8 +10,9 @@
 // lives in CTA q / BPC, slot q % BPC (contiguous ids: the x rows of a brick layer stay together).  A thread owns a
 // k-column of 4 cells of one brick (x in registers, b in registers), and every neighbour cell --
 // in its own brick, in another brick of its CTA or in another CTA's shared memory -- is addressed
-// through the cluster's shared window (mapa), resolved ONCE before the sweeps.  Per sweep: the 18
-// neighbour loads of a thread issued back to back (local ~40 cycles, remote ~215, overlapped), the
+// by a generic address -- plain shared memory in the own CTA, the cluster window (mapa) for another
+// CTA's -- resolved ONCE before the sweeps.  Per sweep: the 18 neighbour loads of a thread issued
+// back to back (local ~30 cycles, remote ~215, overlapped), the
 // canonical sweep expression, the new x to the local ping-pong buffer, one cluster barrier
 // (arrive.release / wait.acquire) -- instead of a grid-wide step per sweep.
 //
@@ -35,15 +36,11 @@ __device__ __forceinline__ uint32_t cl_rank() {
   asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
   return r;
 }
-__device__ __forceinline__ uint32_t cl_map(uint32_t saddr, uint32_t rank) {
-  uint32_t r;
-  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(saddr), "r"(rank));
-  return r;
-}
-__device__ __forceinline__ double ld_cl(uint32_t a) {
-  double v;
-  asm volatile("ld.shared::cluster.f64 %0, [%1];" : "=d"(v) : "r"(a));
-  return v;
+// the generic address of the same shared-memory location in CTA `rank` of the cluster
+__device__ __forceinline__ const double* cl_map_generic(const double* p, uint32_t rank) {
+  uint64_t r;
+  asm volatile("mapa.u64 %0, %1, %2;" : "=l"(r) : "l"(p), "r"(rank));
+  return reinterpret_cast<const double*>(r);
 }
 // every CTA's writes of this sweep visible to every CTA's reads of the next (and no CTA leaves
 // while another may still read its buffers)
@@ -70,24 +67,26 @@ __global__ void __launch_bounds__(128 * BPC, 1)
   const int br = (int)me * kBcPerCta + bl;  // global brick id
   const bool act = br < nbricks;
   const int o = bl * 512 + i + 8 * j + 64 * k0;  // my cell k0 in this CTA's buffer
-  const uint32_t base = (uint32_t)__cvta_generic_to_shared(sm);
-  // cluster-window address (buffer 0) of cell `cell` of brick nq
-  auto at = [&](int nq, int cell) {
-    return cl_map(base + 8u * (uint32_t)((nq % kBcPerCta) * 512 + cell), (uint32_t)(nq / kBcPerCta));
+  // generic address (buffer 0) of cell `cell` of brick nq: this CTA's shared memory directly (plain
+  // shared loads), another CTA's through its window in the cluster (mapa: distributed shared memory)
+  auto at = [&](int nq, int cell) -> const double* {
+    const double* p = sm + (nq % kBcPerCta) * 512 + cell;
+    const uint32_t r = (uint32_t)(nq / kBcPerCta);
+    return r == me ? p : cl_map_generic(p, r);
   };
-  uint32_t aW = 0, aE = 0, aS = 0, aN = 0, aB = 0, aT = 0;
+  const double *aW = sm, *aE = sm, *aS = sm, *aN = sm, *aB = sm, *aT = sm;
   unsigned img = 0;  // bit d: neighbour d is this cell's image across a domain face (MS)
   double xv[4] = {0.0, 0.0, 0.0, 0.0}, bv[4] = {0.0, 0.0, 0.0, 0.0};
   if (act) {
     const int32_t* a = adj + br * 8;
     const int cl = i + 8 * j + 64 * k0;  // my cell k0 in its brick
-    const uint32_t own = at(br, cl);
-    aW = i > 0 ? own - 8 : (a[0] < 0 ? own : at(a[0], 7 + 8 * j + 64 * k0));
-    aE = i < 7 ? own + 8 : (a[1] < 0 ? own : at(a[1], 0 + 8 * j + 64 * k0));
-    aS = j > 0 ? own - 64 : (a[2] < 0 ? own : at(a[2], i + 56 + 64 * k0));
-    aN = j < 7 ? own + 64 : (a[3] < 0 ? own : at(a[3], i + 0 + 64 * k0));
-    aB = k0 > 0 ? own - 512 : (a[4] < 0 ? own : at(a[4], i + 8 * j + 448));
-    aT = k0 < 4 ? own + 2048 : (a[5] < 0 ? own + 1536 : at(a[5], i + 8 * j));  // (image: cell k = 7)
+    const double* own = sm + o;
+    aW = i > 0 ? own - 1 : (a[0] < 0 ? own : at(a[0], 7 + 8 * j + 64 * k0));
+    aE = i < 7 ? own + 1 : (a[1] < 0 ? own : at(a[1], 0 + 8 * j + 64 * k0));
+    aS = j > 0 ? own - 8 : (a[2] < 0 ? own : at(a[2], i + 56 + 64 * k0));
+    aN = j < 7 ? own + 8 : (a[3] < 0 ? own : at(a[3], i + 0 + 64 * k0));
+    aB = k0 > 0 ? own - 64 : (a[4] < 0 ? own : at(a[4], i + 8 * j + 448));
+    aT = k0 < 4 ? own + 256 : (a[5] < 0 ? own + 192 : at(a[5], i + 8 * j));  // (image: cell k = 7)
     if (MS)
       img = (i == 0 && a[0] < 0 ? 1u : 0u) | (i == 7 && a[1] < 0 ? 2u : 0u) | (j == 0 && a[2] < 0 ? 4u : 0u) |
             (j == 7 && a[3] < 0 ? 8u : 0u) | (k0 == 0 && a[4] < 0 ? 16u : 0u) | (k0 == 4 && a[5] < 0 ? 32u : 0u);
@@ -102,18 +101,18 @@ __global__ void __launch_bounds__(128 * BPC, 1)
   auto im = [&](unsigned bit, double v) { return (MS && (img & bit)) ? DMUL(msign, v) : v; };
   cl_barrier();
   for (int s = 0; s < sweeps; ++s) {
-    const uint32_t rd = (s & 1) ? 8u * kBcField : 0u;  // buffer holding x of this sweep
+    const int rd = (s & 1) ? kBcField : 0;  // buffer holding x of this sweep
     double* wr = sm + ((s & 1) ? 0 : kBcField);          // buffer of the next
     if (act) {
       double w[4], e[4], sv[4], nv[4];
 #pragma unroll
       for (int kk = 0; kk < 4; ++kk) {
-        w[kk] = ld_cl(aW + rd + 512 * kk);
-        e[kk] = ld_cl(aE + rd + 512 * kk);
-        sv[kk] = ld_cl(aS + rd + 512 * kk);
-        nv[kk] = ld_cl(aN + rd + 512 * kk);
+        w[kk] = aW[rd + 64 * kk];
+        e[kk] = aE[rd + 64 * kk];
+        sv[kk] = aS[rd + 64 * kk];
+        nv[kk] = aN[rd + 64 * kk];
       }
-      const double bo = ld_cl(aB + rd), to = ld_cl(aT + rd);
+      const double bo = aB[rd], to = aT[rd];
 #pragma unroll
       for (int kk = 0; kk < 4; ++kk) {
         // (multiplying by +-1 is exact: reading A22's -x_p / +x_p)
