@@ -863,7 +863,7 @@ Plan make_plan(const Builder& b, const Layout& lay, bool pencil_overlap, bool lo
   if (c)  // pencil passes after an x exchange over the owned range of a fused-exchange level
     for (Op& o : p.ops) {
       const DevLevel& d = c->dl[o.level];
-      if (o.kind == OP_SWEEP2 && o.exch_before && !o.ghosts && !o.zero && o.c1 < 0 && o.c2 < 0 && d.fused &&
+      if (o.kind == OP_SWEEP2 && o.exch_before && !o.ghosts && !o.zero && d.fused &&
           pencil_supports(o.flags) && !(lay.p.overlap && c->pencil_overlap)) {
         bool plan = false;
         for (const auto& pr : d.pairs)

@@ -55,13 +55,14 @@ bool fused_exchange_enabled() {
 }
 
 // the conditions under which the executor fuses this level's x exchanges into its pencil passes
-// (api.cu make_plan / fill_fused_tables): copy transport, periodic box, constant coefficients, Jacobi
-// or Chebyshev pre / post sweeps, a pencil plan over the owned range, <= 8 ranks, no pencil overlap
+// (api.cu make_plan / fill_fused_tables): copy transport, periodic box, constant coefficients, a
+// pencil plan over the owned range, <= 8 ranks, no pencil overlap (any smoother: Jacobi, Chebyshev,
+// red-black Gauss-Seidel half-sweep pairs)
 bool Builder::fused_level(int l) const {
   const LevelLayout& L = lay.lv[l];
   static const bool pen_ov = getenv("MG_PENCIL_OVERLAP") && atoi(getenv("MG_PENCIL_OVERLAP")) != 0;
   return fused_exchange_enabled() && lay.p.transport != MG_TRANSPORT_NCCL && lay.p.bc == 0 && !lay.p.var_coef &&
-         lay.p.smoother != 2 && L.n_ghost > 0 && lay.world <= 8 && !(pen_ov && lay.p.overlap) &&
+         L.n_ghost > 0 && lay.world <= 8 && !(pen_ov && lay.p.overlap) &&
          fusion(l) != MG_FUSION_PAPER && lay.p.temporal_blocking && pencil_table(l);
 }
 

@@ -459,7 +459,8 @@ cudaError_t encode_pencil_maps(const double* x, const double* b, int64_t n_alloc
   X(0) X(SW_WRITE_R) X(SW_RESTRICT) X(SW_COLOUR) X(SW_WRITE_R | SW_COLOUR) X(SW_RESTRICT | SW_COLOUR)   \
   X(SW_ZERO_X) X(SW_ZERO_X | SW_WRITE_R) X(SW_ZERO_X | SW_RESTRICT) X(SW_ZERO_X | SW_COLOUR)             \
   X(SW_ZERO_X | SW_WRITE_R | SW_COLOUR) X(SW_ZERO_X | SW_RESTRICT | SW_COLOUR)                          \
-  X(SW_PEER) X(SW_PEER | SW_WRITE_R) X(SW_PEER | SW_RESTRICT)
+  X(SW_PEER) X(SW_PEER | SW_WRITE_R) X(SW_PEER | SW_RESTRICT)                                             \
+  X(SW_PEER | SW_COLOUR) X(SW_PEER | SW_WRITE_R | SW_COLOUR) X(SW_PEER | SW_RESTRICT | SW_COLOUR)
 
 // MG_PEN_TRACE=1 (measurement runs without graph capture only): every pencil pass records each CTA's
 // (start, end) globaltimer and prints the spread of the CTAs' end times -- the pass's tail

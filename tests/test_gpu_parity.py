@@ -842,6 +842,30 @@ def test_gsrb_smoother_vcycle_bitwise(oracle_mod, kw):
     orc.close()
 
 
+def test_gsrb_fused_exchange_bitwise(oracle_mod):
+    """Red-black Gauss-Seidel with a self-exchanged ghost shell at 128^3 (level 0: pencil passes of a red
+    and a black half-sweep): the passes after an x exchange stage their ghost bricks from the owner's
+    field (the fused exchange, colour-masked variant); bit for bit with the oracle's GSRB V-cycle."""
+    shape = (128, 128, 128)
+    b = mg_inputs.random_rhs(shape, 45)
+    orc = oracle_mod.OracleMG(shape, 4, 12, 12, 100, smoother=2)
+    orc.set_b(b)
+    orc.set_x(None)
+    xs, ns = [], []
+    for _ in range(2):
+        orc.vcycle()
+        xs.append(orc.get_x())
+        ns.append(orc.norm())
+    m = new(shape, 4, smoother=2, ghost_mode=1, transport=3)
+    if not os.environ.get("MG_NO_FUSED_EXCH"):
+        assert m.exchange_fused()[0] >= 5, m.exchange_fused()
+    m.set_rhs(dev(b))
+    m.set_solution(None)
+    check_cycles(m, xs, ns)
+    m.close()
+    orc.close()
+
+
 def test_gsrb_smoother_loopback_bitwise(oracle_mod):
     _, solver = _mg()
     pg, n_local = (2, 1, 2), (32, 32, 32)
